@@ -1,0 +1,413 @@
+"""Pins for the CPU oracle (-m "not gpu").
+
+The oracle (oracle/oracle.c) is checked against things the paper and
+mathematics fix, never against itself:
+  * div7: big-integer value mod 7, and an independent closed form
+    for prefix residues (powers of two mod 7 have period 3);
+  * Fig. 4: the worked transformation example (golden file);
+  * Aho–Corasick DFAs: brute-force multi-pattern search from first principles;
+  * AC x Z16 counter: closed form per component;
+  * enumeration / composition: brute force over all starts and chunkings;
+  * lookback containment and the div7 closed form of its image.
+"""
+import os
+import random
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+# ---------------------------------------------------------------- div7 ------
+def div7_prefix_residues(bits: np.ndarray) -> np.ndarray:
+    """value(prefix of length m) mod 7 for m = 1..len, WITHOUT the DFA recurrence:
+    value = sum_i b_i 2^(m-1-i);  2^j mod 7 = (1,2,4)[j mod 3]."""
+    b = bits.astype(np.int64)
+    L = b.size
+    i = np.arange(L)
+    S = np.zeros((3, L), np.int64)  # S[r][m-1] = sum_{i<m, i%3==r} b_i
+    for r in range(3):
+        S[r] = np.cumsum(np.where(i % 3 == r, b, 0))
+    m = np.arange(1, L + 1)
+    pw = np.array([1, 2, 4])
+    val = np.zeros(L, np.int64)
+    for r in range(3):
+        val += S[r] * pw[(m - 1 - r) % 3]
+    return val % 7
+
+
+@pytest.mark.parametrize("seed,length,B", [(1, 1, 16), (2, 1000, 16), (3, 4096, 64), (4, 20000, 4096),
+                                          (5, 33333, 48), (0x5EED0001, 1 << 16, 4096)])
+def test_div7_closed_form(seed, length, B):
+    w = gen.workload("c1", length=length, seed=seed)
+    bits = w.host()
+    r = oracle.run(w.table, w.start, w.accept, bits, B)
+    assert r["status"] == 0
+    big = int("".join("01"[x] for x in bits), 2)  # the paper's "binary number"
+    assert r["final"] == big % 7
+    assert r["accept"] == (big % 7 == 0)
+    res = div7_prefix_residues(bits)
+    assert r["count"] == int((res == 0).sum())
+    nb = oracle.nchunks(length, B)
+    ends = [min(length, (c + 1) * B) for c in range(nb)]
+    assert list(r["chunk_end"]) == [int(res[e - 1]) for e in ends]
+    # spot-check chunk ends with Python big ints as well
+    for c in sorted(set([0, nb // 2, nb - 1])):
+        assert r["chunk_end"][c] == int("".join("01"[x] for x in bits[:ends[c]]), 2) % 7
+
+
+def test_div7_empty_and_invalid():
+    t, s, a = gen.dfa_div7()
+    r = oracle.run(t, s, a, np.zeros(0, np.uint8))
+    assert r["status"] == 0 and r["final"] == 0 and r["accept"] == 1 and r["count"] == 0
+    assert len(r["chunk_end"]) == 0
+    r = oracle.run(t, s, a, np.array([1, 0, 2, 1], np.uint8))
+    assert r["status"] == oracle.OR_ESYMBOL
+
+
+# ---------------------------------------------------------------- Fig. 4 ----
+def _fig4():
+    orig, trans, mapping, hot = {}, [], {}, None
+    for line in open(os.path.join(GOLD, "fig4_transform.txt")):
+        if line.startswith("#") or not line.strip():
+            continue
+        f = line.split()
+        if f[0] == "original":
+            orig[int(f[1][1:])] = [int(x[1:]) for x in f[2:5]]
+        elif f[0] == "transformed":
+            trans.append(([int(x[1:-1]) for x in f[2:5]], int(f[5])))
+        elif f[0] == "mapping":
+            mapping[int(f[1][1:])] = int(f[2][1:-1])
+        elif f[0] == "hot":
+            hot = int(f[1])
+    table = np.array([orig[i] for i in range(4)], np.uint32)
+    return table, trans, mapping, hot
+
+
+def test_fig4_transformation_golden():
+    table, trans, mapping, hot = _fig4()
+    perm, inv, freq, tt, acc = oracle.transform(table, np.zeros(4, np.uint8))
+    assert [int(perm[q]) for q in range(4)] == [mapping[q] for q in range(4)]
+    for r, (row, fr) in enumerate(trans):
+        assert list(tt[r]) == row
+        assert freq[inv[r]] == fr
+    # hot test "state ID < 2" selects exactly the two highest-frequency states
+    assert sorted(freq, reverse=True)[:hot] == [freq[inv[r]] for r in range(hot)]
+    # poison row appended last, absorbing
+    assert perm[4] == 4 and inv[4] == 4 and list(tt[4]) == [4, 4, 4]
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_transform_is_renaming(seed):
+    rng = np.random.default_rng(seed)
+    n, ns = int(rng.integers(1, 40)), int(rng.integers(1, 20))
+    t, s, a = gen.dfa_random(seed, n, ns)
+    perm, inv, freq, tt, acc = oracle.transform(t, a)
+    assert sorted(perm[:n]) == list(range(n))
+    assert all(inv[perm[q]] == q for q in range(n))
+    # ranks are non-increasing in frequency; ties ordered by original id
+    for r in range(n - 1):
+        q1, q2 = inv[r], inv[r + 1]
+        assert freq[q1] > freq[q2] or (freq[q1] == freq[q2] and q1 < q2)
+    # independent in-degree count
+    indeg = np.bincount(t.ravel(), minlength=n)
+    assert (freq == indeg).all()
+    for q in range(n):
+        assert acc[perm[q]] == a[q]
+        for c in range(ns):
+            assert tt[perm[q], c] == perm[t[q, c]]
+    # running the transformed DFA gives the renamed result ("preserve the semantics")
+    data = gen.workload(f"rand:{n}:{ns}:{seed}", length=3000, seed=seed).host()
+    r1 = oracle.run(t, s, a, data, 64)
+    r2 = oracle.run(tt[:n], int(perm[s]), acc[:n], data, 64)
+    assert r2["count"] == r1["count"] and inv[r2["final"]] == r1["final"]
+    assert (inv[r2["chunk_end"]] == r1["chunk_end"]).all()
+
+
+def test_transform_profile_policy():
+    t, s, a = gen.dfa_random(11, 20, 4)
+    data = gen.workload("rand:20:4:11", length=5000).host()
+    perm, inv, freq, tt, acc = oracle.transform(t, a, policy=1, profile=data, start=s)
+    # visit counts: independent count of states visited by the walk (incl. the start)
+    visits = np.zeros(20, np.int64)
+    st = s
+    visits[st] += 1
+    for x in data:
+        st = t[st, x]
+        visits[st] += 1
+    assert (freq == visits).all()
+    assert sorted(perm[:20]) == list(range(20))
+
+
+# ---------------------------------------------------------------- AC --------
+def ac_bruteforce(lits, text: bytes):
+    """Accept positions = positions where some literal ends (naive search)."""
+    ends = set()
+    for L in lits:
+        if not L:
+            continue
+        i = text.find(L)
+        while i >= 0:
+            ends.add(i + len(L))
+            i = text.find(L, i + 1)
+    return ends
+
+
+def ac_state_after(table, lits, text: bytes, m: int, maxlen: int):
+    """Trie node of the longest suffix of text[:m] that is a prefix of a literal."""
+    prefixes = set()
+    for L in lits:
+        for k in range(len(L) + 1):
+            prefixes.add(L[:k])
+    for k in range(min(m, maxlen), -1, -1):
+        suf = text[m - k:m]
+        if suf in prefixes:
+            node = 0
+            for ch in suf:  # goto edges of the trie (every step stays on the trie)
+                node = int(table[node, ch])
+            return node
+    return 0
+
+
+@pytest.mark.parametrize("seed,length,B", [(7, 3000, 64), (8, 9000, 512), (0x5EED0002, 1 << 14, 4096)])
+def test_ac_bruteforce(seed, length, B):
+    w = gen.workload("c2", length=length, seed=seed)
+    text = w.host()
+    tb = bytes(text)
+    r = oracle.run(w.table, w.start, w.accept, text, B)
+    ends = ac_bruteforce(w.literals, tb)
+    assert r["count"] == len(ends)
+    maxlen = max(len(L) for L in w.literals)
+    nb = oracle.nchunks(length, B)
+    for c in range(nb):
+        m = min(length, (c + 1) * B)
+        assert r["chunk_end"][c] == ac_state_after(w.table, w.literals, tb, m, maxlen)
+    assert r["final"] == ac_state_after(w.table, w.literals, tb, length, maxlen)
+
+
+def test_ac_counter_closed_form():
+    w = gen.workload("c3", length=40000, seed=99)
+    text = w.host()
+    tb = bytes(text)
+    r = oracle.run(w.table, w.start, w.accept, text, 256)
+    lb, lo = w.keep
+    tac, _, aac = gen.dfa_ac(lb, lo)
+    maxlen = max(len(L) for L in w.literals)
+    vowels = set(b"aeiou")
+    k = 0
+    ks = []
+    for ch in tb:  # counter: vowels since the last reset, mod 16
+        k = 0 if ch == gen.RESET_BYTE else ((k + 1) % 16 if ch in vowels else k)
+        ks.append(k)
+    ends = ac_bruteforce(w.literals, tb)
+    expect_cnt = sum(1 for m in ends if ks[m - 1] == 0)
+    assert r["count"] == expect_cnt
+    for c in range(0, oracle.nchunks(len(tb), 256), 7):
+        m = min(len(tb), (c + 1) * 256)
+        a = ac_state_after(tac, w.literals, tb, m, maxlen)
+        assert r["chunk_end"][c] == a * 16 + ks[m - 1]
+
+
+# -------------------------------------------------------- enumeration -------
+@pytest.mark.parametrize("seed", range(8))
+def test_enum_bruteforce_all_chunkings(seed):
+    rng = random.Random(seed)
+    n, ns = rng.randint(1, 16), rng.randint(1, 6)
+    t, s, a = gen.dfa_random(seed + 100, n, ns)
+    data = gen.workload(f"rand:{n}:{ns}:{seed}", length=rng.randint(0, 200), seed=seed).host()
+    seq = oracle.run(t, s, a, data, 16)
+    # every start, every split point: enum(prefix) then enum(suffix) composes to the run
+    for cut in range(0, len(data) + 1, max(1, len(data) // 13)):
+        M1, C1 = oracle.enum(t, a, data[:cut])
+        M2, C2 = oracle.enum(t, a, data[cut:])
+        M, C = oracle.compose(M1, C1, M2, C2)
+        for q in range(n):
+            rq = oracle.run(t, q, a, data, 16)
+            assert M[q] == rq["final"] and C[q] == rq["count"]
+        assert M[s] == seq["final"] and C[s] == seq["count"]
+
+
+def test_enum_composition_invariant_chunks():
+    w = gen.workload("c1", length=5000, seed=5)
+    data = w.host()
+    B = 256
+    seq = oracle.run(w.table, w.start, w.accept, data, B)
+    M = np.arange(7, dtype=np.uint32)
+    C = np.zeros(7, np.uint64)
+    starts = []
+    for c in range(oracle.nchunks(len(data), B)):
+        starts.append(int(M[w.start]))
+        Mc, Cc = oracle.enum(w.table, w.accept, data[c * B:(c + 1) * B])
+        M, C = oracle.compose(M, C, Mc, Cc)
+        assert M[w.start] == seq["chunk_end"][c]
+    assert M[w.start] == seq["final"] and C[w.start] == seq["count"]
+
+
+# ------------------------------------------------------------ lookback ------
+def test_lookback_div7_closed_form():
+    t, s, a = gen.dfa_div7()
+    # delta*(q, ab) = 4q + 2a + b mod 7 is a bijection in q: image = all 7, mult 1 each
+    for w in ([0, 0], [0, 1], [1, 0], [1, 1]):
+        qs, img = oracle.lookback(t, 7, np.array(w, np.uint8), K=16)
+        assert img == 7 and list(qs) == list(range(7))
+    qs, img = oracle.lookback(t, 7, np.array([1, 5], np.uint8))
+    assert img == 1 and list(qs) == [7]  # invalid symbol -> poison only
+
+
+@pytest.mark.parametrize("seed", range(5))
+def test_lookback_containment(seed):
+    """the real start state must be in the produced end state set."""
+    rng = random.Random(seed)
+    n, ns = rng.randint(2, 30), rng.randint(1, 8)
+    t, s, a = gen.dfa_random(seed + 7, n, ns)
+    data = gen.workload(f"rand:{n}:{ns}:{seed}", length=2000, seed=seed).host()
+    B = 64
+    r = oracle.run(t, s, a, data, B)
+    for L in (1, 2, 3):
+        for c in range(1, oracle.nchunks(len(data), B)):
+            qs, img = oracle.lookback(t, n, data[c * B - L:c * B], K=n)
+            assert img == len(qs)
+            assert r["chunk_end"][c - 1] in set(qs.tolist())
+    # ranking by multiplicity: brute-force count
+    w = data[62:64]
+    qs, img = oracle.lookback(t, n, w, K=n)
+    mult = {}
+    for q in range(n):
+        e = t[t[q, w[0]], w[1]]
+        mult[int(e)] = mult.get(int(e), 0) + 1
+    expect = sorted(mult, key=lambda e: (-mult[e], e))
+    assert list(qs) == expect
+
+
+# ----------------------------------------------------------- simulate -------
+@pytest.mark.parametrize("scheme", ["seq", "pm", "sre", "rr", "nf"])
+@pytest.mark.parametrize("seed", range(6))
+def test_simulate_equals_sequential(scheme, seed):
+    rng = random.Random(seed * 31 + len(scheme))
+    n, ns = rng.randint(1, 24), rng.randint(1, 5)
+    t, s, a = gen.dfa_random(seed + 3, n, ns)
+    length = rng.randint(0, 3000)
+    data = gen.workload(f"rand:{n}:{ns}:{seed}", length=length, seed=seed).host()
+    for B in (16, 48, 256):
+        r = oracle.run(t, s, a, data, B)
+        o = oracle.simulate(t, s, a, data, B, scheme=scheme, spec_k=rng.randint(1, 4), qs_cap=rng.randint(1, 16),
+                            vr_end=rng.randint(1, 16), vr_oth=rng.randint(1, 16))
+        assert o["status"] == 0
+        assert o["final_state"] == r["final"] and o["accept_count"] == r["count"]
+        assert (o["chunk_end"] == r["chunk_end"]).all()
+        assert o["accept"] == a[r["final"]]
+
+
+def test_simulate_seq_is_alg2():
+    """SEQ = Alg. 2: one must-do recovery per mismatch of the sequential chain."""
+    w = gen.workload("c3", length=60000, seed=4)
+    data = w.host()
+    B = 1024
+    o = oracle.simulate(w.table, w.start, w.accept, data, B, scheme="seq", max_tasks=10000)
+    perm, inv, _, tt, acc = oracle.transform(w.table, w.accept)
+    r = oracle.run(w.table, w.start, w.accept, data, B)
+    # Alg. 2 L9-14 literally: compare end_p with VR_i[0].start
+    mism = 0
+    endp = int(perm[r["chunk_end"][0]])
+    for c in range(1, oracle.nchunks(len(data), B)):
+        qs, _ = oracle.lookback(tt, w.nstates, data[c * B - 2:c * B], K=16)
+        if endp != qs[0]:
+            mism += 1
+        endp = int(perm[r["chunk_end"][c]])
+    assert o["rounds"] == mism == o["tasks_mustdo"] == o["tasks_total"]
+    assert all(k == 0 for (_, _, _, k) in o["tasks"])
+
+
+def test_simulate_rr_bound_and_nf_order():
+    w = gen.workload("c3", length=1 << 16, seed=8)
+    data = w.host()
+    B = 512
+    N = oracle.nchunks(len(data), B)
+    for scheme in ("rr", "nf"):
+        o = oracle.simulate(w.table, w.start, w.accept, data, B, scheme=scheme, max_tasks=1 << 20)
+        assert o["ntasks"] == o["tasks_total"] == o["tasks_mustdo"] + o["tasks_sre"] + o["tasks_helper"]
+        rounds = {}
+        for (rd, c, st, k) in o["tasks"]:
+            rounds.setdefault(rd, []).append((c, st, k))
+        for rd, tasks in rounds.items():
+            f = [c for (c, _, k) in tasks if k == 0]
+            assert len(f) == 1
+            f = f[0]
+            helpers = [(c, st) for (c, st, k) in tasks if k == 2]
+            assert all(c > f for c, _ in helpers)  # no helper on verified chunks
+            per = {}
+            for c, st in helpers:
+                per.setdefault(c, []).append(st)
+            for c, sts in per.items():
+                assert len(sts) == len(set(sts))  # distinct speculative states
+            if scheme == "rr" and helpers:
+                # at most 1 + ceil((i-1)/(T-i)) threads per chunk, i = f+1, T = N
+                i = f + 1
+                bound = 1 + -(-(i - 1) // (N - i)) if N > i else 1
+                idle = N - sum(1 for (_, _, k) in tasks if k in (0, 1))
+                bound = 1 + -(-idle // (N - f - 1))
+                for c, sts in per.items():
+                    assert len(sts) + 1 <= bound
+            if scheme == "nf" and helpers:
+                # nearest first: helper chunks are a contiguous run starting at f+1
+                cs = sorted(per)
+                assert cs[0] == f + 1 and cs == list(range(cs[0], cs[-1] + 1))
+                assert [c for c, _ in helpers] == sorted(c for c, _ in helpers)
+
+
+def test_simulate_invalid_symbol():
+    t, s, a = gen.dfa_div7()
+    data = np.array([1, 0, 1] * 100 + [3] + [1] * 50, np.uint8)
+    for scheme in ("seq", "sre", "rr", "nf", "pm"):
+        o = oracle.simulate(t, s, a, data, 16, scheme=scheme)
+        assert o["status"] == oracle.OR_ESYMBOL
+
+
+# ----------------------------------------------------------- features -------
+def test_features_closed_forms():
+    w = gen.workload("c1", length=1 << 16)
+    f = oracle.features(w.table, w.start, w.accept, w.host(), B=4096)
+    assert f["uniq10"] == 7.0  # delta*(., 10 bits) is a bijection for div7
+    assert 0.0 <= f["acc1"] <= f["acck"] <= 1.0
+    assert oracle.select(f, 7) == oracle.ENUM
+    w = gen.workload("c2", length=1 << 18)
+    f = oracle.features(w.table, w.start, w.accept, w.host(), B=4096)
+    assert f["uniq10"] <= 4.0 and oracle.select(f, w.nstates) == oracle.SRE
+    w = gen.workload("c3", length=1 << 18)
+    data = w.host()
+    f = oracle.features(w.table, w.start, w.accept, data, B=4096)
+    # product structure: |image| = |AC image| x |counter image|; the Z16 counter
+    # keeps all 16 values unless a reset byte falls in the 10-symbol window
+    tac, _, _ = gen.dfa_ac(*w.keep)
+    L = len(data)
+    tot = 0
+    for j in range(64):
+        p = j * (L - 10) // 64
+        win = data[p:p + 10]
+        img = set(range(tac.shape[0]))
+        for ch in win:
+            img = {int(tac[q, ch]) for q in img}
+        tot += len(img) * (1 if gen.RESET_BYTE in win else 16)
+    assert f["uniq10"] == tot / 64 and f["uniq10"] > 8
+    assert oracle.select(f, w.nstates) in (oracle.RR, oracle.NF)
+
+
+def test_features_accuracy_bruteforce():
+    t, s, a = gen.dfa_random(5, 12, 3)
+    data = gen.workload("rand:12:3:5", length=4000).host()
+    B = 64
+    perm, inv, _, tt, acc = oracle.transform(t, a)
+    r = oracle.run(t, s, a, data, B)
+    hit1 = hitk = 0
+    N = oracle.nchunks(len(data), B)
+    for c in range(1, N):
+        qs, _ = oracle.lookback(tt, 12, data[c * B - 2:c * B], K=16)
+        truth = int(perm[r["chunk_end"][c - 1]])
+        hit1 += int(qs[0] == truth)
+        hitk += int(truth in list(qs[:4]))
+    f = oracle.features(t, s, a, data, B=B)
+    assert f["acc1"] == pytest.approx(hit1 / (N - 1)) and f["acck"] == pytest.approx(hitk / (N - 1))
