@@ -1,0 +1,176 @@
+/* gspec.h — C ABI of the B200-native GSpecPal hot path (speculative
+ * chunk-parallel DFA execution).
+ *
+ * Paper: Wang, Watling, Qiu, Wang, "GSpecPal: Speculation-Centric Finite State
+ * Machine Parallelization on GPUs" (IPDPS'22).  "P:n" below cites line n of
+ * /root/reference/PAPER.md; DESIGN.md restates every reading.
+ *
+ * The problem the ABI solves (Alg. 1): run a DFA (Q, Σ, q0, δ, F)
+ * over one input stream; report the end state's accept/reject decision (the
+ * output function φ is void) plus, reading R3, the number
+ * of accepting positions and the state at the end of every chunk of
+ * `chunk_bytes` bytes.  Every scheme returns exactly the sequential result;
+ * speculation only changes the cost.
+ *
+ * Conventions (all entry points):
+ *  - return 0 (FSM_OK) or a negative fsm_status; on error out-params are not
+ *    written and fsm_last_error() holds a thread-local message;
+ *  - every state id crossing the ABI is an ORIGINAL id (the frequency
+ *    renumbering of P:319-330 is internal to the handle);
+ *  - pointers named d_* are DEVICE pointers (e.g. torch CUDA tensors'
+ *    data_ptr()), h_* are host pointers; both are borrowed for the call only;
+ *  - all device work is enqueued on opts->stream (NULL = legacy default
+ *    stream); the calls are synchronous: they synchronize that stream before
+ *    filling host results;
+ *  - a handle is not re-entrant: use one handle per concurrent stream.
+ */
+#ifndef GSPEC_H
+#define GSPEC_H
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  FSM_OK = 0,
+  FSM_EINVAL = -1,       /* invalid argument (see each call)                   */
+  FSM_ENOMEM = -2,       /* device or host allocation failed                   */
+  FSM_ECUDA = -3,        /* CUDA runtime error (message in fsm_last_error)     */
+  FSM_ESYMBOL = -4,      /* an input byte >= nsyms (reading R4); outputs unset  */
+  FSM_ENCCL = -5,        /* collective failed                                  */
+  FSM_EUNSUPPORTED = -6  /* e.g. ENUM on a DFA with > 31 states                */
+} fsm_status;
+
+/* Parallelization schemes (PM, SRE; P:195 RR; P:222 NF; P:89 ENUM). */
+typedef enum {
+  FSM_SCHEME_AUTO = 0, /* the decision-tree selector, cached per handle   */
+  FSM_SCHEME_SEQ = 1,  /* Alg. 2: spec-1 + sequential verification/recovery      */
+  FSM_SCHEME_PM = 2,   /* spec-k + parallel verification, must-do recoveries only */
+  FSM_SCHEME_SRE = 3,  /* Alg. 3: recovery activated by the predecessor's end    */
+  FSM_SCHEME_RR = 4,   /* Alg. 4: SRE + round-robin helpers over QS              */
+  FSM_SCHEME_NF = 5,   /* Alg. 5: SRE + nearest-first helpers over QS            */
+  FSM_SCHEME_ENUM = 6  /* enumerative: all-state chunk maps + composition scan  */
+} fsm_scheme;
+
+typedef struct fsm_s* fsm_t;
+
+typedef struct {
+  uint32_t freq_policy;          /* 0 = static in-degree (Fig. 4), 1 = profile visits */
+  const uint8_t* profile_sample; /* host bytes for freq_policy 1 (copied during the call)    */
+  uint64_t profile_len;
+  uint32_t smem_budget_bytes;    /* hot-row budget in shared memory; 0 = auto        */
+  uint32_t force_mode;           /* 0 auto; 1 u8 raw-byte table; 2 u16 classed; 3 u32 classed */
+} fsm_load_opts;
+
+typedef struct {
+  fsm_scheme scheme;    /* FSM_SCHEME_*                                                  */
+  uint32_t chunk_bytes; /* B: chunk c = [cB, min(len,(c+1)B)); multiple of 16; 0 = 4096   */
+  uint32_t spec_k;      /* paths per chunk for PM (4); 1..8; 0 = 4                 */
+  uint32_t lookback;    /* lookback symbols (2); only 2 is supported; 0 = 2        */
+  uint32_t qs_cap;      /* K: ranked candidates kept per chunk (16); 1..16; 0 = 16 */
+  uint32_t vr_end;      /* VR^end slots per chunk (16); 1..16; 0 = 16              */
+  uint32_t vr_others;   /* VR^others slots per chunk (16); 1..16; 0 = 16           */
+  void* stream;         /* cudaStream_t                                                   */
+} fsm_run_opts;
+
+typedef struct {
+  uint32_t final_state;      /* original id of the state after the last symbol        */
+  uint32_t accept;           /* F contains final_state                          */
+  uint64_t accept_count;     /* #positions i in [1,len] whose state is accepting (R3)  */
+  uint64_t nchunks;          /* ceil(len / chunk_bytes)                                */
+  fsm_scheme scheme_used;
+  uint32_t rounds;           /* verification/recovery rounds with a must-do task       */
+  uint64_t tasks_total, tasks_mustdo, tasks_sre, tasks_helper;
+  uint64_t reread_bytes;     /* bytes re-walked by recovery tasks (nominal chunk bytes) */
+  uint64_t verify_checks, verify_matches; /* runtime speculation accuracy    */
+  double avg_active_workers; /* mean active workers per round (Table III analogue)    */
+  double ms_spec, ms_verify; /* device time of speculative execution / verify+recover */
+} fsm_result;
+
+typedef struct {
+  double acc1;              /* spec-1 accuracy on the sample (Table II)         */
+  double acck;              /* spec-k accuracy (k = opts->spec_k)                      */
+  double input_sensitivity; /* max-min of per-segment acc1 over 8 segments (R19)       */
+  double uniq10;            /* mean #unique states after 10 transitions from all */
+  uint32_t nstates;
+} fsm_features;
+
+/* Load a DFA.  table: host uint32 [nstates][nsyms], row-major, original ids;
+ * accept: host uint8 [nstates] (0/1); start < nstates.  Both are COPIED.
+ * Builds the frequency-transformed device image, byte classes, the
+ * lookback pair table on the device.  Errors: FSM_EINVAL if nstates = 0,
+ * nsyms not in [1,256], start >= nstates, an entry >= nstates or NULL arrays;
+ * FSM_EUNSUPPORTED if nstates >= 2^24. */
+int fsm_load(const uint32_t* table, uint32_t nstates, uint32_t nsyms, uint32_t start,
+             const uint8_t* accept, const fsm_load_opts* opts, fsm_t* out);
+
+/* Number of chunks = ceil(len / chunk_bytes) (chunk_bytes 0 means 4096). */
+uint64_t fsm_num_chunks(uint64_t len, uint32_t chunk_bytes);
+
+/* Run the DFA over device bytes d_input[0..len) (reading R2 for the
+ * partition).  d_chunk_ends (device, nullable) receives nchunks uint32 original
+ * ids: the state after each chunk's last symbol.  opts nullable (defaults).
+ * Errors: FSM_EINVAL (bad opts, NULL input with len > 0), FSM_ESYMBOL (an input
+ * byte >= nsyms; detected through the absorbing poison state), FSM_ENOMEM,
+ * FSM_ECUDA, FSM_EUNSUPPORTED (ENUM with nstates > 31). */
+int fsm_run(fsm_t fsm, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
+            uint32_t* d_chunk_ends, fsm_result* out);
+
+/* Same as fsm_run with HOST buffers: copies h_input to the device (pinned
+ * memory recommended), runs, and copies chunk ends back to h_chunk_ends
+ * (nullable).  Used for end-to-end timing. */
+int fsm_run_host(fsm_t fsm, const uint8_t* h_input, uint64_t len, const fsm_run_opts* opts,
+                 uint32_t* h_chunk_ends, fsm_result* out);
+
+/* Scheme selector: profile the device sample (the paper uses a
+ * 1 MB trace), compute the features, walk the decision tree (Fig. 6,
+ * reconstructed: DESIGN.md R19) and cache the choice for FSM_SCHEME_AUTO.
+ * feat nullable. */
+int fsm_select_scheme(fsm_t fsm, const uint8_t* d_sample, uint64_t len, const fsm_run_opts* opts,
+                      fsm_scheme* out, fsm_features* feat);
+
+/* ---- multi-GPU contiguous sharding --------------------
+ * A shard is a contiguous, chunk-aligned byte range [offset, offset+len) of
+ * the global stream.  Each rank reduces its shard to a state map over all
+ * nstates+1 transformed states (poison included), exchanges the maps with
+ * one allgather (NCCL via the caller's process group), composes them, and
+ * fixes its chunk ends.  Map layout (device, caller-allocated, fsm_map_bytes()
+ * bytes): uint32 end[nt] (0xFFFFFFFF = start not reachable/not computed),
+ * then uint64 count[nt].  */
+uint64_t fsm_map_bytes(fsm_t fsm);
+/* Step 1 (per rank): d_shard = shard bytes; d_lookback = the up to 2 bytes
+ * before the shard (NULL/0 for the first shard, whose start is q0).  Writes
+ * the map to d_map; chunk ends that do not depend on the shard's start state
+ * go to d_chunk_ends_local (device, nullable, fsm_num_chunks(len) entries),
+ * the rest is kept in the handle for fsm_shard_finish. */
+int fsm_shard_map(fsm_t fsm, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback,
+                  uint32_t lookback_len, const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local);
+/* Step 2 (every rank, after the allgather): d_maps = nranks maps back to back.
+ * Composes them from q0 (s_{g+1} = M_g[s_g]), writes this rank's chunk ends
+ * (original ids, nullable) and the global result. */
+int fsm_shard_finish(fsm_t fsm, const void* d_maps, uint32_t nranks, uint32_t rank,
+                     const fsm_run_opts* opts, uint32_t* d_chunk_ends_local, fsm_result* out_global);
+
+/* ---- introspection (tests) ------------------------------------------------- */
+/* perm/inv: host uint32 [nstates+1] (poison = nstates last); freq: uint64
+ * [nstates]; mode/H/C: table format, hot rows, classes. Any pointer nullable. */
+int fsm_get_transform(fsm_t fsm, uint32_t* perm, uint32_t* inv, uint64_t* freq, uint32_t* mode,
+                      uint32_t* hot_rows, uint32_t* nclasses);
+/* Ranked lookback candidates QS (transformed ids) for the symbol pair (a, b). */
+int fsm_get_qs(fsm_t fsm, uint8_t a, uint8_t b, uint32_t* qs, uint32_t* qs_len, uint32_t* image_size);
+
+/* Records of the last fsm_run (hierarchical store, level 3), for tests: host
+ * arrays of [32 slots][nchunks] (slot s < 16: VR^end ring, s >= 16: VR^others
+ * ring) in TRANSFORMED ids, plus per-chunk ring counts and x[0..nchunks]
+ * (incoming states).  Any pointer nullable. */
+int fsm_get_records(fsm_t fsm, uint64_t nchunks, uint32_t* start, uint32_t* end, uint32_t* cnt, uint32_t* n_end,
+                    uint32_t* n_oth, uint32_t* x);
+
+void fsm_free(fsm_t fsm);
+const char* fsm_strerror(int status);
+const char* fsm_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

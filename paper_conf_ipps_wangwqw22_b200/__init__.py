@@ -1,0 +1,255 @@
+"""B200-native GSpecPal hot path — thin Python binding over libgspec.so.
+
+Argument marshalling only: every step of the method runs in the sm_100a
+kernels behind the C ABI (include/gspec.h).  PyTorch is used for device
+memory and streams; there is no CPU fallback — importing this package without
+the built library raises.
+
+    import paper_conf_ipps_wangwqw22_b200 as gs
+    fsm = gs.FSM.load(table, start, accept)          # numpy uint32 [n, nsyms]
+    res = fsm.run(x_cuda_uint8, scheme="auto")       # -> Result
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass, field
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "libgspec.so")
+if not os.path.exists(_LIB_PATH):
+    raise ImportError(f"{_LIB_PATH} is missing: build it with `python build.py` (no CPU fallback exists)")
+_lib = ctypes.CDLL(_LIB_PATH)
+
+FSM_OK, FSM_EINVAL, FSM_ENOMEM, FSM_ECUDA, FSM_ESYMBOL, FSM_ENCCL, FSM_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
+SCHEMES = {"auto": 0, "seq": 1, "pm": 2, "sre": 3, "rr": 4, "nf": 5, "enum": 6}
+SCHEME_NAMES = {v: k for k, v in SCHEMES.items()}
+MODES = {1: "u8", 2: "u16", 3: "u32"}
+
+U32, U64, P = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p
+
+
+class fsm_load_opts(ctypes.Structure):
+    _fields_ = [("freq_policy", U32), ("profile_sample", P), ("profile_len", U64),
+                ("smem_budget_bytes", U32), ("force_mode", U32)]
+
+
+class fsm_run_opts(ctypes.Structure):
+    _fields_ = [("scheme", ctypes.c_int), ("chunk_bytes", U32), ("spec_k", U32), ("lookback", U32),
+                ("qs_cap", U32), ("vr_end", U32), ("vr_others", U32), ("stream", P)]
+
+
+class fsm_result(ctypes.Structure):
+    _fields_ = [("final_state", U32), ("accept", U32), ("accept_count", U64), ("nchunks", U64),
+                ("scheme_used", ctypes.c_int), ("rounds", U32), ("tasks_total", U64), ("tasks_mustdo", U64),
+                ("tasks_sre", U64), ("tasks_helper", U64), ("reread_bytes", U64), ("verify_checks", U64),
+                ("verify_matches", U64), ("avg_active_workers", ctypes.c_double), ("ms_spec", ctypes.c_double),
+                ("ms_verify", ctypes.c_double)]
+
+
+class fsm_features(ctypes.Structure):
+    _fields_ = [("acc1", ctypes.c_double), ("acck", ctypes.c_double), ("input_sensitivity", ctypes.c_double),
+                ("uniq10", ctypes.c_double), ("nstates", U32)]
+
+
+_lib.fsm_load.argtypes = [P, U32, U32, U32, P, ctypes.POINTER(fsm_load_opts), ctypes.POINTER(P)]
+_lib.fsm_num_chunks.argtypes = [U64, U32]
+_lib.fsm_num_chunks.restype = U64
+_lib.fsm_run.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
+_lib.fsm_run_host.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
+_lib.fsm_select_scheme.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), ctypes.POINTER(ctypes.c_int),
+                                   ctypes.POINTER(fsm_features)]
+_lib.fsm_map_bytes.argtypes = [P]
+_lib.fsm_map_bytes.restype = U64
+_lib.fsm_shard_map.argtypes = [P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, P]
+_lib.fsm_shard_finish.argtypes = [P, P, U32, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
+_lib.fsm_get_transform.argtypes = [P, P, P, P, P, P, P]
+_lib.fsm_get_qs.argtypes = [P, ctypes.c_uint8, ctypes.c_uint8, P, P, P]
+_lib.fsm_get_records.argtypes = [P, U64, P, P, P, P, P, P]
+_lib.fsm_free.argtypes = [P]
+_lib.fsm_free.restype = None
+_lib.fsm_strerror.argtypes = [ctypes.c_int]
+_lib.fsm_strerror.restype = ctypes.c_char_p
+_lib.fsm_last_error.restype = ctypes.c_char_p
+
+
+class GSpecError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        msg = _lib.fsm_last_error().decode(errors="replace")
+        super().__init__(f"{where}: {_lib.fsm_strerror(status).decode()} ({status}): {msg}")
+
+
+def _check(rc: int, where: str):
+    if rc != FSM_OK:
+        raise GSpecError(rc, where)
+
+
+def lib_path() -> str:
+    return _LIB_PATH
+
+
+def fsm_num_chunks(length: int, chunk_bytes: int = 4096) -> int:
+    return int(_lib.fsm_num_chunks(length, chunk_bytes))
+
+
+def _run_opts(scheme="auto", chunk_bytes=4096, spec_k=4, qs_cap=16, vr_end=16, vr_others=16, stream=None):
+    if isinstance(scheme, str):
+        scheme = SCHEMES[scheme]
+    if stream is None:
+        import torch
+
+        stream = torch.cuda.current_stream().cuda_stream if torch.cuda.is_available() else 0
+    return fsm_run_opts(scheme=scheme, chunk_bytes=chunk_bytes, spec_k=spec_k, lookback=2, qs_cap=qs_cap,
+                        vr_end=vr_end, vr_others=vr_others, stream=stream)
+
+
+@dataclass
+class Result:
+    final_state: int
+    accept: bool
+    accept_count: int
+    nchunks: int
+    scheme: str
+    stats: dict = field(default_factory=dict)
+    chunk_ends: object = None
+
+    @staticmethod
+    def from_c(r: fsm_result, chunk_ends=None) -> "Result":
+        stats = {k: getattr(r, k) for k, _ in fsm_result._fields_}
+        return Result(int(r.final_state), bool(r.accept), int(r.accept_count), int(r.nchunks),
+                      SCHEME_NAMES.get(r.scheme_used, "?"), stats, chunk_ends)
+
+
+class FSM:
+    """A loaded DFA (device image of the frequency-transformed table)."""
+
+    def __init__(self, handle: int, nstates: int, nsyms: int):
+        self._h = handle
+        self.nstates = nstates
+        self.nsyms = nsyms
+
+    @staticmethod
+    def load(table, start: int, accept, freq_policy: int = 0, profile=None, smem_budget: int = 0,
+             force_mode: int = 0) -> "FSM":
+        """fsm_load: table uint32 [n, nsyms] (original ids), accept uint8 [n]."""
+        t = np.ascontiguousarray(table, dtype=np.uint32)
+        a = np.ascontiguousarray(accept, dtype=np.uint8)
+        n, ns = t.shape
+        prof = None if profile is None else np.ascontiguousarray(profile, dtype=np.uint8)
+        o = fsm_load_opts(freq_policy=freq_policy, profile_sample=None if prof is None else prof.ctypes.data,
+                          profile_len=0 if prof is None else prof.size, smem_budget_bytes=smem_budget,
+                          force_mode=force_mode)
+        h = P()
+        _check(_lib.fsm_load(t.ctypes.data, n, ns, start, a.ctypes.data, ctypes.byref(o), ctypes.byref(h)),
+               "fsm_load")
+        return FSM(h.value, n, ns)
+
+    def close(self):
+        if self._h:
+            _lib.fsm_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    # ---- runs -----------------------------------------------------------------
+    def run(self, x, scheme="auto", chunk_bytes=4096, spec_k=4, qs_cap=16, vr_end=16, vr_others=16,
+            chunk_ends=True, stream=None) -> Result:
+        """fsm_run over a uint8 CUDA tensor; chunk_ends -> int64-free uint32 CUDA tensor (as torch.int32 view)."""
+        import torch
+
+        assert x.is_cuda and x.dtype == torch.uint8 and x.is_contiguous()
+        o = _run_opts(scheme, chunk_bytes, spec_k, qs_cap, vr_end, vr_others, stream)
+        n = fsm_num_chunks(x.numel(), chunk_bytes)
+        ce = torch.empty(max(n, 1), dtype=torch.int32, device=x.device) if chunk_ends else None
+        r = fsm_result()
+        _check(_lib.fsm_run(self._h, x.data_ptr() if x.numel() else None, x.numel(), ctypes.byref(o),
+                            ce.data_ptr() if ce is not None else None, ctypes.byref(r)), "fsm_run")
+        return Result.from_c(r, ce[:n] if ce is not None else None)
+
+    def run_host(self, data: np.ndarray, scheme="auto", chunk_bytes=4096, chunk_ends=True, stream=None,
+                 **kw) -> Result:
+        """fsm_run_host: host bytes in, host chunk ends out (H2D/D2H inside the call)."""
+        d = np.ascontiguousarray(data, dtype=np.uint8) if not hasattr(data, "data_ptr") else data
+        o = _run_opts(scheme, chunk_bytes, stream=stream, **kw)
+        n = fsm_num_chunks(len(d) if not hasattr(d, "numel") else d.numel(), chunk_bytes)
+        ce = np.zeros(max(n, 1), np.uint32) if chunk_ends else None
+        r = fsm_result()
+        ptr = d.data_ptr() if hasattr(d, "data_ptr") else d.ctypes.data
+        length = d.numel() if hasattr(d, "numel") else d.size
+        _check(_lib.fsm_run_host(self._h, ptr if length else None, length, ctypes.byref(o),
+                                 ce.ctypes.data if ce is not None else None, ctypes.byref(r)), "fsm_run_host")
+        return Result.from_c(r, ce[:n] if ce is not None else None)
+
+    def select_scheme(self, sample, chunk_bytes=4096, spec_k=4, stream=None):
+        """fsm_select_scheme on a uint8 CUDA tensor: (scheme name, features dict)."""
+        o = _run_opts("sre", chunk_bytes, spec_k, stream=stream)
+        out = ctypes.c_int(0)
+        ft = fsm_features()
+        _check(_lib.fsm_select_scheme(self._h, sample.data_ptr() if sample.numel() else None, sample.numel(),
+                                      ctypes.byref(o), ctypes.byref(out), ctypes.byref(ft)), "fsm_select_scheme")
+        return SCHEME_NAMES[out.value], {k: getattr(ft, k) for k, _ in fsm_features._fields_}
+
+    # ---- introspection --------------------------------------------------------
+    def transform(self):
+        n = self.nstates
+        perm = np.zeros(n + 1, np.uint32)
+        inv = np.zeros(n + 1, np.uint32)
+        freq = np.zeros(n, np.uint64)
+        mode, H, C = U32(0), U32(0), U32(0)
+        _check(_lib.fsm_get_transform(self._h, perm.ctypes.data, inv.ctypes.data, freq.ctypes.data,
+                                      ctypes.byref(mode), ctypes.byref(H), ctypes.byref(C)), "fsm_get_transform")
+        return {"perm": perm, "inv": inv, "freq": freq, "mode": MODES.get(mode.value, "?"), "hot_rows": H.value,
+                "nclasses": C.value}
+
+    def qs(self, a: int, b: int):
+        q = np.zeros(16, np.uint32)
+        ql, im = U32(0), U32(0)
+        _check(_lib.fsm_get_qs(self._h, a, b, q.ctypes.data, ctypes.byref(ql), ctypes.byref(im)), "fsm_get_qs")
+        return q[:ql.value].copy(), im.value
+
+    def records(self, nchunks: int):
+        """Records of the last run (transformed ids): dict of [32, nchunks] arrays + rings + x."""
+        a = {k: np.zeros((32, nchunks), np.uint32) for k in ("start", "end", "cnt")}
+        ne = np.zeros(nchunks, np.uint32)
+        no = np.zeros(nchunks, np.uint32)
+        x = np.zeros(nchunks + 1, np.uint32)
+        _check(_lib.fsm_get_records(self._h, nchunks, a["start"].ctypes.data, a["end"].ctypes.data,
+                                    a["cnt"].ctypes.data, ne.ctypes.data, no.ctypes.data, x.ctypes.data),
+               "fsm_get_records")
+        a.update(n_end=ne, n_oth=no, x=x)
+        return a
+
+    def map_bytes(self) -> int:
+        return int(_lib.fsm_map_bytes(self._h))
+
+    @property
+    def handle(self):
+        return self._h
+
+
+# C-ABI names (same entry points, argument marshalling only)
+def fsm_load(table, start, accept, **kw) -> FSM:
+    return FSM.load(table, start, accept, **kw)
+
+
+def fsm_run(fsm: FSM, x, **kw) -> Result:
+    return fsm.run(x, **kw)
+
+
+def fsm_run_host(fsm: FSM, data, **kw) -> Result:
+    return fsm.run_host(data, **kw)
+
+
+def fsm_select_scheme(fsm: FSM, sample, **kw):
+    return fsm.select_scheme(sample, **kw)
+
+
+def fsm_free(fsm: FSM) -> None:
+    fsm.close()

@@ -1,0 +1,876 @@
+// api.cpp — the C ABI of include/gspec.h: DFA preparation (frequency-based
+// transformation, byte classes, packing), the run driver (spec exec
+// -> verify/recover rounds -> finalize), ENUM, the scheme selector.
+// Host code only; every step of the hot path runs in the sm_100a kernels.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "gspec.h"
+#include "internal.h"
+
+using namespace gspec;
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const std::string& msg) {
+  g_err = msg;
+  return code;
+}
+
+#define CUDA_TRY(expr)                                                                         \
+  do {                                                                                         \
+    cudaError_t _e = (expr);                                                                   \
+    if (_e != cudaSuccess)                                                                     \
+      return fail(_e == cudaErrorMemoryAllocation ? FSM_ENOMEM : FSM_ECUDA,                    \
+                  std::string(#expr) + ": " + cudaGetErrorString(_e));                         \
+  } while (0)
+
+int dev_alloc(fsm_t f, void** p, size_t bytes) {
+  cudaError_t e = cudaMalloc(p, bytes ? bytes : 16);
+  if (e != cudaSuccess) return fail(FSM_ENOMEM, std::string("cudaMalloc: ") + cudaGetErrorString(e));
+  f->owned.push_back(*p);
+  return FSM_OK;
+}
+
+template <typename T>
+int upload(fsm_t f, const T** dst, const std::vector<T>& v, size_t pad_bytes = 0) {
+  void* p = nullptr;
+  const size_t bytes = v.size() * sizeof(T);
+  int rc = dev_alloc(f, &p, bytes + pad_bytes + 16);
+  if (rc) return rc;
+  CUDA_TRY(cudaMemset(p, 0, bytes + pad_bytes + 16));
+  if (bytes) CUDA_TRY(cudaMemcpy(p, v.data(), bytes, cudaMemcpyHostToDevice));
+  *dst = reinterpret_cast<const T*>(p);
+  return FSM_OK;
+}
+
+struct Opts {
+  fsm_scheme scheme;
+  uint32_t B, k, L, qs_cap, vr_end, vr_oth;
+  cudaStream_t st;
+};
+
+int resolve_opts(const fsm_run_opts* o, Opts* r) {
+  r->scheme = o ? o->scheme : FSM_SCHEME_AUTO;
+  r->B = (o && o->chunk_bytes) ? o->chunk_bytes : 4096;
+  r->k = (o && o->spec_k) ? o->spec_k : 4;
+  r->L = (o && o->lookback) ? o->lookback : 2;
+  r->qs_cap = (o && o->qs_cap) ? o->qs_cap : 16;
+  r->vr_end = (o && o->vr_end) ? o->vr_end : 16;
+  r->vr_oth = (o && o->vr_others) ? o->vr_others : 16;
+  r->st = o ? reinterpret_cast<cudaStream_t>(o->stream) : nullptr;
+  if (r->B % 16 != 0) return fail(FSM_EINVAL, "chunk_bytes must be a multiple of 16");
+  if (r->k < 1 || r->k > 8) return fail(FSM_EINVAL, "spec_k must be in [1,8]");
+  if (r->L != 2) return fail(FSM_EUNSUPPORTED, "only lookback = 2 is supported (P:300)");
+  if (r->qs_cap < 1 || r->qs_cap > kQsMax) return fail(FSM_EINVAL, "qs_cap must be in [1,16]");
+  if (r->vr_end < 1 || r->vr_end > kVrMax || r->vr_oth < 1 || r->vr_oth > kVrMax)
+    return fail(FSM_EINVAL, "vr_end / vr_others must be in [1,16]");
+  if ((int)r->scheme < 0 || (int)r->scheme > FSM_SCHEME_ENUM) return fail(FSM_EINVAL, "unknown scheme");
+  return FSM_OK;
+}
+
+// ---- scratch ------------------------------------------------------------------
+int ensure_records(fsm_t f, uint64_t N) {
+  if (f->rs_cap >= N && f->rs_base) return FSM_OK;
+  if (f->rs_base) cudaFree(f->rs_base);
+  f->rs_base = nullptr;
+  uint64_t cap = std::max<uint64_t>(N, 1024);
+  cap = (cap + 255) & ~255ull;
+  // u32 arrays: start/end/cnt (kSlots each) + n_end, n_oth, oth_base, ref x3, x(+1), prefU, task x3 (+1)
+  const uint64_t u32s = cap * 3 * kSlots + cap * 11 + 8 + 3 * 8;
+  const uint64_t u8s = cap * 5;  // next_qs, found, ulen, next_new, hcnt
+  size_t bytes = u32s * 4 + u8s + 4096;
+  void* p = nullptr;
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e != cudaSuccess) return fail(FSM_ENOMEM, std::string("record store: ") + cudaGetErrorString(e));
+  f->rs_base = p;
+  f->rs_cap = cap;
+  uint32_t* u = reinterpret_cast<uint32_t*>(p);
+  RecStore& r = f->rs;
+  r.cap = cap;
+  r.start = u; u += cap * kSlots;
+  r.end = u; u += cap * kSlots;
+  r.cnt = u; u += cap * kSlots;
+  r.n_end = u; u += cap;
+  r.n_oth = u; u += cap;
+  r.oth_base = u; u += cap;
+  r.ref_start = u; u += cap;
+  r.ref_end = u; u += cap;
+  r.ref_cnt = u; u += cap;
+  r.x = u; u += cap + 8;
+  r.cur_end = u; u += cap;
+  r.prefU = u; u += cap;
+  r.task_chunk = u; u += cap + 8;
+  r.task_start = u; u += cap + 8;
+  r.task_j = u; u += cap + 8;
+  uint8_t* b = reinterpret_cast<uint8_t*>(u);
+  r.next_qs = b; b += cap;
+  r.found = b; b += cap;
+  r.ulen = b; b += cap;
+  r.next_new = b; b += cap;
+  r.hcnt = b; b += cap;
+  return FSM_OK;
+}
+
+int ensure_ctl(fsm_t f) {
+  if (!f->d_ctl) CUDA_TRY(cudaMalloc(&f->d_ctl, sizeof(Ctl)));
+  const size_t need = 2 * 4096 + 64;
+  if (f->block_tmp_elems < need) {
+    if (f->d_block_tmp) cudaFree(f->d_block_tmp);
+    CUDA_TRY(cudaMalloc(&f->d_block_tmp, need * sizeof(uint64_t)));
+    f->block_tmp_elems = need;
+  }
+  return FSM_OK;
+}
+
+void fill_result_stats(fsm_result* out, const Ctl& h) {
+  out->rounds = (uint32_t)h.rounds;
+  out->tasks_mustdo = h.tasks_mustdo;
+  out->tasks_sre = h.tasks_sre;
+  out->tasks_helper = h.tasks_helper;
+  out->tasks_total = h.tasks_mustdo + h.tasks_sre + h.tasks_helper;
+  out->reread_bytes = h.reread_bytes;
+  out->verify_checks = h.verify_checks;
+  out->verify_matches = h.verify_matches;
+  out->avg_active_workers = h.rounds ? (double)h.active_sum / (double)h.rounds : 0.0;
+}
+
+// Core device run over d_in[0..len) from transformed start q0t.  On success
+// leaves x[] (speculative/record path) in the handle for callers that need it.
+int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_scheme scheme, uint32_t q0t,
+             uint32_t* d_chunk_ends, fsm_result* out, uint32_t* final_tid) {
+  const uint64_t N = (len + o.B - 1) / o.B;
+  std::memset(out, 0, sizeof(*out));
+  out->nchunks = N;
+  out->scheme_used = scheme;
+  if (N == 0) {
+    *final_tid = q0t;
+    return FSM_OK;
+  }
+  int rc = ensure_ctl(f);
+  if (rc) return rc;
+  RunParams rp{};
+  rp.in = d_in;
+  rp.q0t = q0t;
+  rp.len = len;
+  rp.B = o.B;
+  rp.N = N;
+  rp.scheme = scheme;
+  rp.k = scheme == FSM_SCHEME_PM ? o.k : 1;
+  rp.qs_cap = o.qs_cap;
+  rp.vr_end = o.vr_end;
+  rp.vr_oth = o.vr_oth;
+  cudaEvent_t ev[3];
+  for (auto& e : ev) CUDA_TRY(cudaEventCreate(&e));
+  Ctl h{};
+  uint32_t xfin = 0;
+  if (scheme == FSM_SCHEME_ENUM) {
+    if (f->n + 1 > kEnumMax) {
+      for (auto& e : ev) cudaEventDestroy(e);
+      return fail(FSM_EUNSUPPORTED, "ENUM needs nstates + 1 <= 32");
+    }
+    // sub-chunk size E | B: small enough for parallelism, bounded scratch
+    uint32_t E = o.B;
+    while (E % 32 == 0 && E > 256 && (len + E / 2 - 1) / (E / 2) <= (1ull << 22)) E /= 2;
+    const uint64_t nsub = (len + E - 1) / E;
+    const uint64_t need = enum_scratch_bytes(nsub);
+    if (f->enum_bytes < need) {
+      if (f->enum_base) cudaFree(f->enum_base);
+      f->enum_base = nullptr;
+      f->enum_bytes = 0;
+      CUDA_TRY(cudaMalloc(&f->enum_base, need));
+      f->enum_bytes = need;
+    }
+    CUDA_TRY(cudaMemsetAsync(f->d_ctl, 0, sizeof(Ctl), o.st));
+    CUDA_TRY(cudaEventRecord(ev[0], o.st));
+    if (!f->d_small) CUDA_TRY(cudaMalloc(&f->d_small, 64 * sizeof(uint32_t)));
+    CUDA_TRY(launch_enum_full(f->img, rp, E, f->enum_base, d_chunk_ends, f->d_ctl, f->d_small, o.st, f->sm_count));
+    CUDA_TRY(cudaEventRecord(ev[1], o.st));
+    CUDA_TRY(cudaEventRecord(ev[2], o.st));
+  } else {
+    rc = ensure_records(f, N);
+    if (rc) {
+      for (auto& e : ev) cudaEventDestroy(e);
+      return rc;
+    }
+    Ctl init{};
+    init.f = 0;
+    init.tf = q0t;
+    init.fmin = N;
+    CUDA_TRY(cudaMemcpyAsync(f->d_ctl, &init, sizeof(Ctl), cudaMemcpyHostToDevice, o.st));
+    CUDA_TRY(cudaEventRecord(ev[0], o.st));
+    CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
+    CUDA_TRY(cudaEventRecord(ev[1], o.st));
+    CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
+    CUDA_TRY(cudaEventRecord(ev[2], o.st));
+  }
+  CUDA_TRY(cudaMemcpyAsync(&h, f->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, o.st));
+  if (scheme != FSM_SCHEME_ENUM)
+    CUDA_TRY(cudaMemcpyAsync(&xfin, f->rs.x + N, sizeof(uint32_t), cudaMemcpyDeviceToHost, o.st));
+  else
+    CUDA_TRY(cudaMemcpyAsync(&xfin, f->d_small, sizeof(uint32_t), cudaMemcpyDeviceToHost, o.st));
+  CUDA_TRY(cudaStreamSynchronize(o.st));
+  float t1 = 0, t2 = 0;
+  cudaEventElapsedTime(&t1, ev[0], ev[1]);
+  cudaEventElapsedTime(&t2, ev[1], ev[2]);
+  for (auto& e : ev) cudaEventDestroy(e);
+  fill_result_stats(out, h);
+  out->accept_count = h.accept_count;
+  out->ms_spec = t1;
+  out->ms_verify = t2;
+  *final_tid = xfin;
+  return FSM_OK;
+}
+
+fsm_scheme tree_select(const fsm_features& ft, uint32_t n) {
+  // Fig. 6 (image lost) reconstructed from P:284-290, P:339-345, P:383 (R19)
+  if (n <= 31 && ft.uniq10 >= n / 2.0) return FSM_SCHEME_ENUM;
+  if (ft.uniq10 <= 4.0) return FSM_SCHEME_SRE;
+  if (ft.acck >= 0.9 && ft.acck - ft.acc1 >= 0.2) return FSM_SCHEME_PM;
+  if (ft.input_sensitivity >= 0.2) return FSM_SCHEME_NF;
+  return FSM_SCHEME_RR;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* fsm_last_error(void) { return g_err.c_str(); }
+
+const char* fsm_strerror(int s) {
+  switch (s) {
+    case FSM_OK: return "ok";
+    case FSM_EINVAL: return "invalid argument";
+    case FSM_ENOMEM: return "out of memory";
+    case FSM_ECUDA: return "CUDA error";
+    case FSM_ESYMBOL: return "input symbol out of range";
+    case FSM_ENCCL: return "collective failed";
+    case FSM_EUNSUPPORTED: return "unsupported";
+    default: return "unknown status";
+  }
+}
+
+uint64_t fsm_num_chunks(uint64_t len, uint32_t chunk_bytes) {
+  if (!chunk_bytes) chunk_bytes = 4096;
+  return (len + chunk_bytes - 1) / chunk_bytes;
+}
+
+int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, const uint8_t* accept,
+             const fsm_load_opts* opts, fsm_t* out) {
+  if (!table || !accept || !out) return fail(FSM_EINVAL, "NULL table/accept/out");
+  if (n == 0 || nsyms == 0 || nsyms > 256 || start >= n) return fail(FSM_EINVAL, "bad nstates/nsyms/start");
+  if (n >= (1u << 24)) return fail(FSM_EUNSUPPORTED, "nstates >= 2^24");
+  for (uint64_t i = 0; i < (uint64_t)n * nsyms; i++)
+    if (table[i] >= n) return fail(FSM_EINVAL, "table entry >= nstates");
+  const uint32_t policy = opts ? opts->freq_policy : 0;
+  if (policy > 1) return fail(FSM_EINVAL, "freq_policy must be 0 or 1");
+  if (policy == 1 && (!opts->profile_sample || !opts->profile_len))
+    return fail(FSM_EINVAL, "PROFILE policy needs a sample");
+  fsm_t f = new fsm_s();
+  f->n = n;
+  f->nsyms = nsyms;
+  f->q0 = start;
+  f->table.assign(table, table + (uint64_t)n * nsyms);
+  f->accept.assign(accept, accept + n);
+  for (auto& a : f->accept) a = a ? 1 : 0;
+  cudaGetDevice(&f->device);
+  cudaDeviceGetAttribute(&f->sm_count, cudaDevAttrMultiProcessorCount, f->device);
+  int rc = FSM_OK;
+  auto bail = [&](int code) {
+    fsm_free(f);
+    return code;
+  };
+
+  // ---- 1. frequency-based transformation ----
+  const uint32_t nt = n + 1, P = n;  // poison state: absorbing, ranked last
+  f->freq.assign(n, 0);
+  if (policy == 0) {
+    for (uint64_t i = 0; i < (uint64_t)n * nsyms; i++) f->freq[table[i]]++;  // static in-degree
+  } else {
+    uint32_t s = start;
+    f->freq[s]++;
+    for (uint64_t i = 0; i < opts->profile_len; i++) {
+      const uint8_t b = opts->profile_sample[i];
+      if (b >= nsyms) break;
+      s = table[(uint64_t)s * nsyms + b];
+      f->freq[s]++;
+    }
+  }
+  std::vector<uint32_t> order(n);
+  std::iota(order.begin(), order.end(), 0u);
+  std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return f->freq[a] > f->freq[b]; });
+  f->perm.assign(nt, 0);
+  f->inv.assign(nt, 0);
+  for (uint32_t r = 0; r < n; r++) {
+    f->inv[r] = order[r];
+    f->perm[order[r]] = r;
+  }
+  f->perm[P] = P;
+  f->inv[P] = P;
+  std::vector<uint8_t> acc_t(nt, 0);
+  for (uint32_t t = 0; t < n; t++) acc_t[t] = f->accept[f->inv[t]];
+
+  // ---- 2. byte classes: identical columns; bytes >= nsyms -> poison class ----
+  f->cls.assign(256, 0);
+  std::map<std::vector<uint32_t>, uint32_t> colmap;
+  std::vector<uint32_t> rep;  // representative byte of each class
+  for (uint32_t b = 0; b < nsyms; b++) {
+    std::vector<uint32_t> col(n);
+    for (uint32_t q = 0; q < n; q++) col[q] = table[(uint64_t)q * nsyms + b];
+    auto it = colmap.find(col);
+    if (it == colmap.end()) {
+      const uint32_t id = (uint32_t)rep.size();
+      colmap.emplace(std::move(col), id);
+      rep.push_back(b);
+      f->cls[b] = (uint8_t)id;
+    } else {
+      f->cls[b] = (uint8_t)it->second;
+    }
+  }
+  uint32_t C = (uint32_t)rep.size();
+  const bool has_poison_cls = nsyms < 256;
+  const uint32_t PC = C;
+  if (has_poison_cls) {
+    for (uint32_t b = nsyms; b < 256; b++) f->cls[b] = (uint8_t)PC;
+    C++;
+  }
+  if (C > 256) return bail(fail(FSM_EINVAL, "too many classes"));
+  // transformed tid x class table
+  std::vector<uint32_t> ttc((uint64_t)nt * C);
+  for (uint32_t t = 0; t < nt; t++)
+    for (uint32_t c = 0; c < C; c++) {
+      uint32_t v;
+      if (t == P || (has_poison_cls && c == PC)) v = P;
+      else v = f->perm[table[(uint64_t)f->inv[t] * nsyms + rep[c]]];
+      ttc[(uint64_t)t * C + c] = v;
+    }
+
+  // ---- 3. table format and codes ----
+  uint32_t n_acc = 0;
+  for (uint32_t t = 0; t < nt; t++) n_acc += acc_t[t];
+  const uint32_t n_na = nt - n_acc;
+  uint32_t force = opts ? opts->force_mode : 0;
+  uint32_t mode;
+  if (force) mode = force;
+  else if (n_na <= 128 && n_acc <= 128) mode = MODE_U8;
+  else if (nt <= 32768) mode = MODE_U16;
+  else mode = MODE_U32;
+  if (mode == MODE_U8 && !(n_na <= 128 && n_acc <= 128)) return bail(fail(FSM_EUNSUPPORTED, "u8 mode needs <=128 accepting and non-accepting states"));
+  if (mode == MODE_U16 && nt > 32768) return bail(fail(FSM_EUNSUPPORTED, "u16 mode needs nstates < 32768"));
+  if (mode < MODE_U8 || mode > MODE_U32) return bail(fail(FSM_EINVAL, "force_mode must be 0..3"));
+  DevImage& img = f->img;
+  img.mode = mode;
+  img.n = n;
+  img.nsyms = nsyms;
+  img.C = C;
+  img.q0t = f->perm[start];
+  std::vector<uint32_t> tid2code(nt), code2tid(256, P);
+  if (mode == MODE_U8) {
+    uint32_t na = 0, ac = 0;
+    for (uint32_t t = 0; t < nt; t++) {
+      const uint32_t code = acc_t[t] ? 128 + ac++ : na++;
+      tid2code[t] = code;
+      code2tid[code] = t;
+    }
+    std::vector<uint8_t> T8(256 * 256, (uint8_t)tid2code[P]);
+    for (uint32_t code = 0; code < 256; code++) {
+      const uint32_t t = code2tid[code];
+      for (uint32_t b = 0; b < 256; b++) T8[code * 256 + b] = (uint8_t)tid2code[ttc[(uint64_t)t * C + f->cls[b]]];
+    }
+    img.H = nt;
+    img.smem_table_bytes = (n_acc > 0 ? 128 + n_acc : n_na) * 256;
+    if ((rc = upload(f, &img.T8, T8))) return bail(rc);
+  } else {
+    const uint32_t shift = mode == MODE_U16 ? 15 : 31;
+    for (uint32_t t = 0; t < nt; t++) tid2code[t] = t | ((uint32_t)acc_t[t] << shift);
+    const uint32_t esz = mode == MODE_U16 ? 2 : 4;
+    const uint32_t budget = (opts && opts->smem_budget_bytes) ? opts->smem_budget_bytes : 96 * 1024;
+    uint64_t H = budget / (C * esz);
+    if (H > nt) H = nt;
+    img.H = (uint32_t)H;
+    img.smem_table_bytes = (uint32_t)(((H * C * esz) + 15) & ~15ull);
+    if (mode == MODE_U16) {
+      std::vector<uint16_t> T16((uint64_t)nt * C);
+      for (uint64_t i = 0; i < T16.size(); i++) T16[i] = (uint16_t)tid2code[ttc[i]];
+      if ((rc = upload(f, &img.T16, T16, 64))) return bail(rc);
+    } else {
+      std::vector<uint32_t> T32((uint64_t)nt * C);
+      for (uint64_t i = 0; i < T32.size(); i++) T32[i] = tid2code[ttc[i]];
+      if ((rc = upload(f, &img.T32, T32, 64))) return bail(rc);
+    }
+  }
+  std::vector<uint32_t> inv_v(f->inv.begin(), f->inv.end());
+  if ((rc = upload(f, &img.cls, f->cls))) return bail(rc);
+  if ((rc = upload(f, &img.tid2code, tid2code))) return bail(rc);
+  if ((rc = upload(f, &img.code2tid, code2tid))) return bail(rc);
+  if ((rc = upload(f, &img.inv, inv_v))) return bail(rc);
+  if ((rc = upload(f, &img.acc, acc_t))) return bail(rc);
+  const uint32_t* d_ttc = nullptr;
+  if ((rc = upload(f, &d_ttc, ttc))) return bail(rc);
+  f->d_ttc = d_ttc;
+
+  // ---- 4. lookback pair table on the device ----
+  const uint64_t npairs = (uint64_t)C * C;
+  void *qs2 = nullptr, *qs2l = nullptr, *qs2i = nullptr, *scratch = nullptr;
+  if ((rc = dev_alloc(f, &qs2, npairs * kQsMax * 4))) return bail(rc);
+  if ((rc = dev_alloc(f, &qs2l, npairs + 16))) return bail(rc);
+  if ((rc = dev_alloc(f, &qs2i, npairs * 4))) return bail(rc);
+  uint32_t grid = (uint32_t)std::min<uint64_t>(npairs, (uint64_t)f->sm_count * 4);
+  if ((uint64_t)grid * nt > (1ull << 28)) grid = (uint32_t)std::max<uint64_t>(1, (1ull << 28) / nt);
+  cudaError_t ce = cudaMalloc(&scratch, (uint64_t)grid * nt * 4);
+  if (ce != cudaSuccess) return bail(fail(FSM_ENOMEM, "qs2 scratch"));
+  ce = launch_build_qs2_raw(d_ttc, n, C, (uint32_t*)scratch, grid, (uint32_t*)qs2, (uint8_t*)qs2l, (uint32_t*)qs2i, 0);
+  if (ce == cudaSuccess) ce = cudaDeviceSynchronize();
+  cudaFree(scratch);
+  if (ce != cudaSuccess) return bail(fail(FSM_ECUDA, std::string("qs2 build: ") + cudaGetErrorString(ce)));
+  img.qs2 = (const uint32_t*)qs2;
+  img.qs2_len = (const uint8_t*)qs2l;
+  img.qs2_img = (const uint32_t*)qs2i;
+  *out = f;
+  return FSM_OK;
+}
+
+void fsm_free(fsm_t f) {
+  if (!f) return;
+  for (void* p : f->owned) cudaFree(p);
+  if (f->rs_base) cudaFree(f->rs_base);
+  if (f->d_ctl) cudaFree(f->d_ctl);
+  if (f->d_block_tmp) cudaFree(f->d_block_tmp);
+  if (f->enum_base) cudaFree(f->enum_base);
+  if (f->feat_base) cudaFree(f->feat_base);
+  if (f->h_dev_in) cudaFree(f->h_dev_in);
+  if (f->h_dev_ce) cudaFree(f->h_dev_ce);
+  if (f->d_small) cudaFree(f->d_small);
+  if (f->shard_base) cudaFree(f->shard_base);
+  delete f;
+}
+
+int fsm_run(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts, uint32_t* d_chunk_ends,
+            fsm_result* out) {
+  if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
+  if (!d_input && len > 0) return fail(FSM_EINVAL, "NULL input");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  fsm_scheme scheme = o.scheme;
+  if (scheme == FSM_SCHEME_AUTO) {
+    if (!f->auto_selected) {
+      fsm_run_opts so{};
+      if (opts) so = *opts;
+      so.scheme = FSM_SCHEME_SRE;
+      fsm_scheme pick;
+      rc = fsm_select_scheme(f, d_input, std::min<uint64_t>(len, 1ull << 20), &so, &pick, nullptr);
+      if (rc) return rc;
+    }
+    scheme = f->auto_scheme;
+    if (scheme == FSM_SCHEME_ENUM && f->n + 1 > kEnumMax) scheme = FSM_SCHEME_SRE;
+  }
+  fsm_result r;
+  uint32_t fin = 0;
+  rc = run_core(f, d_input, len, o, scheme, f->img.q0t, d_chunk_ends, &r, &fin);
+  if (rc) return rc;
+  if (fin == f->n) return fail(FSM_ESYMBOL, "input symbol >= nsyms");
+  r.final_state = f->inv[fin];
+  r.accept = f->accept[r.final_state];
+  *out = r;
+  return FSM_OK;
+}
+
+int fsm_run_host(fsm_t f, const uint8_t* h_input, uint64_t len, const fsm_run_opts* opts, uint32_t* h_chunk_ends,
+                 fsm_result* out) {
+  if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
+  if (!h_input && len > 0) return fail(FSM_EINVAL, "NULL input");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  const uint64_t N = fsm_num_chunks(len, o.B);
+  if (f->h_in_cap < len) {
+    if (f->h_dev_in) cudaFree(f->h_dev_in);
+    f->h_dev_in = nullptr;
+    f->h_in_cap = 0;
+    CUDA_TRY(cudaMalloc(&f->h_dev_in, len + 16));
+    f->h_in_cap = len;
+  }
+  if (h_chunk_ends && f->h_ce_cap < N) {
+    if (f->h_dev_ce) cudaFree(f->h_dev_ce);
+    f->h_dev_ce = nullptr;
+    f->h_ce_cap = 0;
+    CUDA_TRY(cudaMalloc(&f->h_dev_ce, N * 4 + 16));
+    f->h_ce_cap = N;
+  }
+  if (len) CUDA_TRY(cudaMemcpyAsync(f->h_dev_in, h_input, len, cudaMemcpyHostToDevice, o.st));
+  rc = fsm_run(f, (const uint8_t*)f->h_dev_in, len, opts, h_chunk_ends ? (uint32_t*)f->h_dev_ce : nullptr, out);
+  if (rc) return rc;
+  if (h_chunk_ends && N) {
+    CUDA_TRY(cudaMemcpyAsync(h_chunk_ends, f->h_dev_ce, N * 4, cudaMemcpyDeviceToHost, o.st));
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+  }
+  return FSM_OK;
+}
+
+int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_run_opts* opts, fsm_scheme* outp,
+                      fsm_features* feat) {
+  if (!f || !outp) return fail(FSM_EINVAL, "NULL handle/out");
+  if (!d_sample && len > 0) return fail(FSM_EINVAL, "NULL sample");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  // 1. true chunk starts by an exact scheme on the sample
+  fsm_result r;
+  uint32_t fin = 0;
+  rc = run_core(f, d_sample, len, o, FSM_SCHEME_SRE, f->img.q0t, nullptr, &r, &fin);
+  if (rc) return rc;
+  const uint64_t N = r.nchunks;
+  // 2. features on the device
+  const uint32_t words = (f->n + 1 + 31) / 32;
+  const size_t need = 32 * 8 + 64ull * words * 4 + 64;
+  if (f->feat_bytes < need) {
+    if (f->feat_base) cudaFree(f->feat_base);
+    f->feat_base = nullptr;
+    f->feat_bytes = 0;
+    CUDA_TRY(cudaMalloc(&f->feat_base, need));
+    f->feat_bytes = need;
+  }
+  unsigned long long* d_counts = (unsigned long long*)f->feat_base;  // [0..18) + uniq at [20]
+  uint32_t* d_seen = (uint32_t*)((uint8_t*)f->feat_base + 32 * 8);
+  CUDA_TRY(cudaMemsetAsync(f->feat_base, 0, need, o.st));
+  fsm_features ft{};
+  ft.nstates = f->n;
+  if (len > 0) {
+    CUDA_TRY(launch_features_raw(f->img, f->d_ttc, d_sample, len, o.B, N, f->rs.x, o.k, o.qs_cap, d_counts, d_seen,
+                                 d_counts + 20, o.st));
+    unsigned long long h[32];
+    CUDA_TRY(cudaMemcpyAsync(h, d_counts, sizeof(h), cudaMemcpyDeviceToHost, o.st));
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+    if (N > 1) {
+      ft.acc1 = (double)h[16] / (double)(N - 1);
+      ft.acck = (double)h[17] / (double)(N - 1);
+      double mx = -1, mn = 2;
+      for (int s = 0; s < 8; s++) {
+        if (!h[8 + s]) continue;
+        const double a = (double)h[s] / (double)h[8 + s];
+        mx = std::max(mx, a);
+        mn = std::min(mn, a);
+      }
+      ft.input_sensitivity = mx >= 0 ? mx - mn : 0;
+    }
+    if (len >= 10) ft.uniq10 = (double)h[20] / 64.0;
+  }
+  const fsm_scheme pick = tree_select(ft, f->n);
+  f->auto_scheme = pick;
+  f->auto_selected = true;
+  *outp = pick;
+  if (feat) *feat = ft;
+  return FSM_OK;
+}
+
+int fsm_get_transform(fsm_t f, uint32_t* perm, uint32_t* inv, uint64_t* freq, uint32_t* mode, uint32_t* hot_rows,
+                      uint32_t* nclasses) {
+  if (!f) return fail(FSM_EINVAL, "NULL handle");
+  if (perm) std::copy(f->perm.begin(), f->perm.end(), perm);
+  if (inv) std::copy(f->inv.begin(), f->inv.end(), inv);
+  if (freq) std::copy(f->freq.begin(), f->freq.end(), freq);
+  if (mode) *mode = f->img.mode;
+  if (hot_rows) *hot_rows = f->img.H;
+  if (nclasses) *nclasses = f->img.C;
+  return FSM_OK;
+}
+
+int fsm_get_qs(fsm_t f, uint8_t a, uint8_t b, uint32_t* qs, uint32_t* qs_len, uint32_t* image_size) {
+  if (!f) return fail(FSM_EINVAL, "NULL handle");
+  const uint64_t pair = (uint64_t)f->cls[a] * f->img.C + f->cls[b];
+  uint8_t l = 0;
+  uint32_t im = 0;
+  CUDA_TRY(cudaMemcpy(&l, f->img.qs2_len + pair, 1, cudaMemcpyDeviceToHost));
+  CUDA_TRY(cudaMemcpy(&im, f->img.qs2_img + pair, 4, cudaMemcpyDeviceToHost));
+  if (qs) CUDA_TRY(cudaMemcpy(qs, f->img.qs2 + pair * kQsMax, 4 * l, cudaMemcpyDeviceToHost));
+  if (qs_len) *qs_len = l;
+  if (image_size) *image_size = im;
+  return FSM_OK;
+}
+
+int fsm_get_records(fsm_t f, uint64_t N, uint32_t* start, uint32_t* end, uint32_t* cnt, uint32_t* n_end,
+                    uint32_t* n_oth, uint32_t* x) {
+  if (!f || !f->rs_base || N > f->rs_cap) return fail(FSM_EINVAL, "no records for that many chunks");
+  const RecStore& r = f->rs;
+  for (uint32_t s = 0; s < kSlots; s++) {
+    if (start) CUDA_TRY(cudaMemcpy(start + s * N, r.start + s * r.cap, 4 * N, cudaMemcpyDeviceToHost));
+    if (end) CUDA_TRY(cudaMemcpy(end + s * N, r.end + s * r.cap, 4 * N, cudaMemcpyDeviceToHost));
+    if (cnt) CUDA_TRY(cudaMemcpy(cnt + s * N, r.cnt + s * r.cap, 4 * N, cudaMemcpyDeviceToHost));
+  }
+  if (n_end) CUDA_TRY(cudaMemcpy(n_end, r.n_end, 4 * N, cudaMemcpyDeviceToHost));
+  if (n_oth) CUDA_TRY(cudaMemcpy(n_oth, r.n_oth, 4 * N, cudaMemcpyDeviceToHost));
+  if (x) CUDA_TRY(cudaMemcpy(x, r.x, 4 * (N + 1), cudaMemcpyDeviceToHost));
+  return FSM_OK;
+}
+
+uint64_t fsm_map_bytes(fsm_t f) {
+  if (!f) return 0;
+  const uint64_t nt = f->n + 1;
+  return ((nt * 4 + 7) & ~7ull) + nt * 8;
+}
+
+}  // extern "C"
+
+// ---- multi-GPU shard steps: implemented in shard.cpp ----
+
+namespace {
+
+constexpr uint32_t kFuseChunks = 8;   // path-fusion window (chunks) before falling back
+constexpr uint32_t kMaxMulti = 64;    // distinct surviving paths run by the pipeline
+constexpr uint32_t kNoState = 0xFFFFFFFFu;
+
+uint64_t map_cnt_off(uint32_t nt) { return ((uint64_t)nt * 4 + 7) & ~7ull; }
+uint64_t map_bytes_nt(uint32_t nt) { return map_cnt_off(nt) + (uint64_t)nt * 8; }
+
+struct ShardScratch {
+  uint32_t *mark, *cand, *info, *states, *grp, *pfinal;
+  unsigned long long *prefix, *pcount;
+};
+
+int ensure_shard(fsm_t f, ShardScratch* s) {
+  const uint64_t nt = f->n + 1;
+  const uint64_t words = nt * 2 + 16 + kFuseChunks * nt + nt * 2 + nt * 2 + nt * 2 + 64;
+  const size_t need = words * 8;
+  if (f->shard_bytes < need) {
+    if (f->shard_base) cudaFree(f->shard_base);
+    f->shard_base = nullptr;
+    f->shard_bytes = 0;
+    CUDA_TRY(cudaMalloc(&f->shard_base, need));
+    f->shard_bytes = need;
+  }
+  uint64_t* p = reinterpret_cast<uint64_t*>(f->shard_base);
+  s->prefix = reinterpret_cast<unsigned long long*>(p); p += nt;
+  s->pcount = reinterpret_cast<unsigned long long*>(p); p += nt;
+  uint32_t* u = reinterpret_cast<uint32_t*>(p);
+  s->mark = u; u += nt;
+  s->cand = u; u += nt;
+  s->info = u; u += 32;
+  s->grp = u; u += nt;
+  s->pfinal = u; u += nt;
+  s->states = u;
+  return FSM_OK;
+}
+
+int resolve_scheme(fsm_t f, const uint8_t* d_in, uint64_t len, const fsm_run_opts* opts, const Opts& o,
+                   fsm_scheme* out) {
+  fsm_scheme scheme = o.scheme;
+  if (scheme == FSM_SCHEME_AUTO) {
+    if (!f->auto_selected) {
+      fsm_run_opts so{};
+      if (opts) so = *opts;
+      so.scheme = FSM_SCHEME_SRE;
+      fsm_scheme pick;
+      int rc = fsm_select_scheme(f, d_in, std::min<uint64_t>(len, 1ull << 20), &so, &pick, nullptr);
+      if (rc) return rc;
+    }
+    scheme = f->auto_scheme;
+  }
+  if (scheme == FSM_SCHEME_ENUM && f->n + 1 > kEnumMax) scheme = FSM_SCHEME_SRE;
+  *out = scheme;
+  return FSM_OK;
+}
+
+uint32_t enum_sub_bytes(uint32_t B, uint64_t len) {
+  uint32_t E = B;
+  while (E % 32 == 0 && E > 256 && (len + E / 2 - 1) / (E / 2) <= (1ull << 22)) E /= 2;
+  return E;
+}
+
+int ensure_enum_scratch(fsm_t f, uint64_t nsub) {
+  const uint64_t need = enum_scratch_bytes(nsub);
+  if (f->enum_bytes < need) {
+    if (f->enum_base) cudaFree(f->enum_base);
+    f->enum_base = nullptr;
+    f->enum_bytes = 0;
+    CUDA_TRY(cudaMalloc(&f->enum_base, need));
+    f->enum_bytes = need;
+  }
+  if (!f->d_small) CUDA_TRY(cudaMalloc(&f->d_small, 64 * sizeof(uint32_t)));
+  return FSM_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int fsm_shard_map(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
+                  const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local) {
+  if (!f || !d_map) return fail(FSM_EINVAL, "NULL handle/map");
+  if (!d_shard && len > 0) return fail(FSM_EINVAL, "NULL shard");
+  if (lb_len > 16 || (lb_len && !d_lookback)) return fail(FSM_EINVAL, "lookback_len must be <= 16 with bytes");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  fsm_scheme scheme;
+  if ((rc = resolve_scheme(f, d_shard, len, opts, o, &scheme))) return rc;
+  ShardScratch S;
+  if ((rc = ensure_shard(f, &S))) return rc;
+  if ((rc = ensure_ctl(f))) return rc;
+  if (!f->d_small) CUDA_TRY(cudaMalloc(&f->d_small, 64 * sizeof(uint32_t)));
+  const uint32_t nt = f->n + 1;
+  const uint64_t N = (len + o.B - 1) / o.B;
+  uint32_t* mend = reinterpret_cast<uint32_t*>(d_map);
+  unsigned long long* mcnt = reinterpret_cast<unsigned long long*>(reinterpret_cast<uint8_t*>(d_map) + map_cnt_off(nt));
+  CUDA_TRY(launch_map_init(mend, mcnt, nt, o.st));
+  // 1. candidate start states: the lookback image or q0 for the first shard
+  uint32_t ncand = 1;
+  if (lb_len == 0) {
+    CUDA_TRY(cudaMemcpyAsync(S.cand, &f->img.q0t, 4, cudaMemcpyHostToDevice, o.st));
+    f->shard_cand.assign(1, f->img.q0t);
+  } else {
+    CUDA_TRY(launch_shard_image(f->img, f->d_ttc, d_lookback, lb_len, S.mark, S.cand, S.info + 8, o.st));
+    CUDA_TRY(cudaMemcpyAsync(&ncand, S.info + 8, 4, cudaMemcpyDeviceToHost, o.st));
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+    f->shard_cand.resize(ncand);
+    CUDA_TRY(cudaMemcpy(f->shard_cand.data(), S.cand, 4ull * ncand, cudaMemcpyDeviceToHost));
+  }
+  f->shard_in = d_shard;
+  f->shard_len = len;
+  f->shard_ncand = ncand;
+  f->shard_nj = 0;
+  f->shard_scheme = scheme;
+  f->shard_grp.assign(ncand, 0);
+  f->shard_dist.clear();
+  std::vector<uint32_t> last(f->shard_cand);
+  uint32_t nj = 0;
+  bool merged = ncand == 1;
+  // 2. path fusion over the first chunks
+  if (!merged && N > 0 && ncand <= 1024) {
+    const uint32_t W = (uint32_t)std::min<uint64_t>(kFuseChunks, N);
+    CUDA_TRY(launch_shard_fuse(f->img, d_shard, len, o.B, S.cand, ncand, W, S.states, S.prefix, S.info, o.st));
+    uint32_t info[2];
+    CUDA_TRY(cudaMemcpyAsync(info, S.info, 8, cudaMemcpyDeviceToHost, o.st));
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+    nj = info[1];
+    merged = info[0] != kNoState;
+    CUDA_TRY(cudaMemcpy(last.data(), S.states + (uint64_t)(nj - 1) * ncand, 4ull * ncand, cudaMemcpyDeviceToHost));
+  }
+  f->shard_nj = nj;
+  const uint64_t off = (uint64_t)nj * o.B, rest = len - std::min<uint64_t>(len, off);
+  if (merged || (nt > kEnumMax)) {
+    // distinct surviving paths; each runs the speculative pipeline over the rest
+    std::vector<uint32_t>& D = f->shard_dist;
+    for (uint32_t i = 0; i < ncand; i++) {
+      auto it = std::find(D.begin(), D.end(), last[i]);
+      if (it == D.end()) {
+        D.push_back(last[i]);
+        f->shard_grp[i] = (uint32_t)D.size() - 1;
+      } else {
+        f->shard_grp[i] = (uint32_t)(it - D.begin());
+      }
+    }
+    if (D.size() > kMaxMulti) return fail(FSM_EUNSUPPORTED, "shard start not resolved by path fusion");
+    std::vector<uint32_t> fin(D.size());
+    std::vector<unsigned long long> cnt(D.size());
+    for (size_t d = 0; d < D.size(); d++) {
+      fsm_result r;
+      uint32_t ft = D[d];
+      if (rest) {
+        const bool write_ce = D.size() == 1 && d_chunk_ends_local;
+        rc = run_core(f, d_shard + off, rest, o, scheme, D[d], write_ce ? d_chunk_ends_local + nj : nullptr, &r, &ft);
+        if (rc) return rc;
+        cnt[d] = r.accept_count;
+      } else {
+        cnt[d] = 0;
+      }
+      fin[d] = ft;
+    }
+    f->shard_mode = D.size() == 1 ? 0 : 2;
+    CUDA_TRY(cudaMemcpyAsync(S.grp, f->shard_grp.data(), 4ull * ncand, cudaMemcpyHostToDevice, o.st));
+    CUDA_TRY(cudaMemcpyAsync(S.pfinal, fin.data(), 4ull * fin.size(), cudaMemcpyHostToDevice, o.st));
+    CUDA_TRY(cudaMemcpyAsync(S.pcount, cnt.data(), 8ull * cnt.size(), cudaMemcpyHostToDevice, o.st));
+    CUDA_TRY(launch_map_write(S.cand, ncand, S.grp, nj ? S.prefix : nullptr, S.pfinal, S.pcount, mend, mcnt, o.st));
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+    if (nj && d_chunk_ends_local && f->shard_mode == 0)
+      CUDA_TRY(launch_fix_prefix(S.states, ncand, 0, nj, f->img.inv, d_chunk_ends_local, o.st));
+  } else {
+    // non-convergent small DFA: enumerate the whole shard
+    f->shard_mode = 1;
+    f->shard_E = enum_sub_bytes(o.B, len);
+    const uint64_t nsub = (len + f->shard_E - 1) / f->shard_E;
+    if ((rc = ensure_enum_scratch(f, nsub))) return rc;
+    RunParams rp{};
+    rp.in = d_shard;
+    rp.q0t = f->img.q0t;
+    rp.len = len;
+    rp.B = o.B;
+    rp.N = N;
+    const uint8_t* topM = nullptr;
+    const uint64_t* topC = nullptr;
+    CUDA_TRY(launch_enum_full(f->img, rp, f->shard_E, f->enum_base, nullptr, f->d_ctl, f->d_small, o.st, f->sm_count,
+                              1, &topM, &topC));
+    CUDA_TRY(launch_map_enum(topM, reinterpret_cast<const unsigned long long*>(topC), nt, mend, mcnt, o.st));
+  }
+  CUDA_TRY(cudaStreamSynchronize(o.st));
+  return FSM_OK;
+}
+
+int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, const fsm_run_opts* opts,
+                     uint32_t* d_chunk_ends_local, fsm_result* out) {
+  if (!f || !d_maps || !out || rank >= G) return fail(FSM_EINVAL, "bad finish arguments");
+  if (f->shard_mode < 0) return fail(FSM_EINVAL, "fsm_shard_map was not called");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  const uint32_t nt = f->n + 1;
+  CUDA_TRY(launch_compose(reinterpret_cast<const uint8_t*>(d_maps), G, map_bytes_nt(nt), map_cnt_off(nt), f->img.q0t,
+                          rank, f->d_small, o.st));
+  uint32_t h[5];
+  CUDA_TRY(cudaMemcpyAsync(h, f->d_small, sizeof(h), cudaMemcpyDeviceToHost, o.st));
+  CUDA_TRY(cudaStreamSynchronize(o.st));
+  if (h[2]) return fail(FSM_EINVAL, "a shard start state is outside its candidate set");
+  const uint32_t srank = h[0], fin = h[1];
+  const uint64_t count = (uint64_t)h[3] | ((uint64_t)h[4] << 32);
+  const uint64_t N = (f->shard_len + o.B - 1) / o.B;
+  ShardScratch S;
+  if ((rc = ensure_shard(f, &S))) return rc;
+  if (d_chunk_ends_local && N) {
+    if (f->shard_mode == 1) {
+      RunParams rp{};
+      rp.in = f->shard_in;
+      rp.q0t = srank;
+      rp.len = f->shard_len;
+      rp.B = o.B;
+      rp.N = N;
+      CUDA_TRY(launch_enum_full(f->img, rp, f->shard_E, f->enum_base, d_chunk_ends_local, f->d_ctl, f->d_small + 8,
+                                o.st, f->sm_count, 2));
+    } else {
+      auto it = std::find(f->shard_cand.begin(), f->shard_cand.end(), srank);
+      if (it == f->shard_cand.end()) return fail(FSM_EINVAL, "rank start not among its candidates");
+      const uint32_t ci = (uint32_t)(it - f->shard_cand.begin());
+      if (f->shard_nj) CUDA_TRY(launch_fix_prefix(S.states, f->shard_ncand, ci, f->shard_nj, f->img.inv,
+                                                  d_chunk_ends_local, o.st));
+      if (f->shard_mode == 2) {
+        const uint64_t off = (uint64_t)f->shard_nj * o.B;
+        if (off < f->shard_len) {
+          fsm_result r;
+          uint32_t ft;
+          rc = run_core(f, f->shard_in + off, f->shard_len - off, o, f->shard_scheme, f->shard_dist[f->shard_grp[ci]],
+                        d_chunk_ends_local + f->shard_nj, &r, &ft);
+          if (rc) return rc;
+        }
+      }
+    }
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+  }
+  std::memset(out, 0, sizeof(*out));
+  out->nchunks = N;
+  out->scheme_used = f->shard_scheme;
+  if (fin == f->n) return fail(FSM_ESYMBOL, "input symbol >= nsyms");
+  out->final_state = f->inv[fin];
+  out->accept = f->accept[out->final_state];
+  out->accept_count = count;
+  return FSM_OK;
+}
+
+}  // extern "C"

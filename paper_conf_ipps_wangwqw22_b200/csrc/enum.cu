@@ -1,0 +1,236 @@
+// enum.cu — B5: the enumerative scheme (Mytkowicz et al. [23]).
+//
+// Every sub-chunk j (E bytes, E | B) is run from EVERY transformed state
+// (n+1 <= 32 incl. poison): M_j[q] = end state, C_j[q] = accepts on that path.
+// The real path is obtained by "connecting the end state of each chunk to the
+// start state of its successor", i.e. a prefix composition of maps:
+//   (M2,C2) o (M1,C1) = (M2[M1[q]], C1[q] + C2[M1[q]]).
+// Composition is one __shfl_sync per map (lane q holds entry q), applied as a
+// hierarchical scan: warps scan groups of 64 maps, group totals form the next
+// level, the top level (<= 64 maps) is scanned by one warp, and incoming
+// states/counts are pushed back down level by level.
+#include "internal.h"
+#include "walk.cuh"
+
+namespace gspec {
+namespace {
+
+constexpr uint32_t kGroup = 64;
+
+// K1: thread per sub-chunk, NE independent chains (ILP = NE).
+template <int MODE, int NE>
+__global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* __restrict__ in, uint64_t len,
+                                                  uint32_t E, uint64_t nsub, uint8_t* __restrict__ M,
+                                                  uint64_t* __restrict__ Cn) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  stage_table(img, smem);
+  __syncthreads();
+  using S = Step<MODE>;
+  const uint32_t nt = img.n + 1;
+  for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < nsub; j += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t code[NE], acc[NE];
+#pragma unroll
+    for (int q = 0; q < NE; q++) {
+      code[q] = __ldg(img.tid2code + ((uint32_t)q < nt ? q : 0));
+      acc[q] = 0;
+    }
+    const uint64_t lo = j * E, n = min((uint64_t)E, len - lo);
+    const uint8_t* p = in + lo;
+    uint64_t i = 0;
+    if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
+      const uint4* v = reinterpret_cast<const uint4*>(p);
+      for (uint64_t t16 = 0; t16 < n / 16; t16++) {
+        const uint4 qv = __ldg(v + t16);
+        const uint32_t w[4] = {qv.x, qv.y, qv.z, qv.w};
+#pragma unroll
+        for (int t = 0; t < 4; t++) {
+#pragma unroll
+          for (int q = 0; q < NE; q++) { code[q] = S::template word<0>(img, smem, code[q], w[t]); acc[q] += S::acc(code[q]); }
+#pragma unroll
+          for (int q = 0; q < NE; q++) { code[q] = S::template word<1>(img, smem, code[q], w[t]); acc[q] += S::acc(code[q]); }
+#pragma unroll
+          for (int q = 0; q < NE; q++) { code[q] = S::template word<2>(img, smem, code[q], w[t]); acc[q] += S::acc(code[q]); }
+#pragma unroll
+          for (int q = 0; q < NE; q++) { code[q] = S::template word<3>(img, smem, code[q], w[t]); acc[q] += S::acc(code[q]); }
+        }
+      }
+      i = (n / 16) * 16;
+    }
+    for (; i < n; i++) {
+      const uint32_t bb = __ldg(p + i);
+#pragma unroll
+      for (int q = 0; q < NE; q++) { code[q] = S::byte(img, smem, code[q], bb); acc[q] += S::acc(code[q]); }
+    }
+#pragma unroll
+    for (int q = 0; q < 32; q++) {
+      const bool real = q < NE && (uint32_t)q < nt;
+      M[j * 32 + q] = (uint8_t)(real ? S::tid(img, code[q < NE ? q : 0]) : q);
+      Cn[j * 32 + q] = real ? acc[q < NE ? q : 0] : 0;
+    }
+  }
+}
+
+// K2: warp per group of kGroup maps: in-place inclusive prefix P_j = M_j o ... o M_g0,
+// and the group total written as one map of the next level.
+__global__ void __launch_bounds__(128) k_enum_group(uint8_t* __restrict__ M, uint64_t* __restrict__ Cn, uint64_t cnt,
+                                                   uint8_t* __restrict__ Mup, uint64_t* __restrict__ Cup) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  const uint64_t ngroups = (cnt + kGroup - 1) / kGroup;
+  for (uint64_t g = warp; g < ngroups; g += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+    uint32_t P = lane;
+    uint64_t PC = 0;
+    const uint64_t j0 = g * kGroup, j1 = min(cnt, j0 + kGroup);
+    uint32_t m = M[j0 * 32 + lane];
+    uint64_t c = Cn[j0 * 32 + lane];
+    for (uint64_t j = j0; j < j1; j++) {
+      uint32_t mn = 0;
+      uint64_t cn = 0;
+      if (j + 1 < j1) { mn = M[(j + 1) * 32 + lane]; cn = Cn[(j + 1) * 32 + lane]; }  // prefetch
+      const uint32_t nP = __shfl_sync(0xffffffffu, m, P);
+      PC += __shfl_sync(0xffffffffu, c, P);
+      P = nP;
+      M[j * 32 + lane] = (uint8_t)P;
+      Cn[j * 32 + lane] = PC;
+      m = mn;
+      c = cn;
+    }
+    if (Mup) {
+      Mup[g * 32 + lane] = (uint8_t)P;
+      Cup[g * 32 + lane] = PC;
+    }
+  }
+}
+
+// Descend: incoming state/count of every map at level l from its group's entry.
+__global__ void k_enum_descend(const uint8_t* __restrict__ P, const uint64_t* __restrict__ PC, uint64_t cnt,
+                               const uint32_t* __restrict__ up_state, const uint64_t* __restrict__ up_cnt,
+                               uint32_t top_entry, uint32_t* __restrict__ st, uint64_t* __restrict__ sc) {
+  for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < cnt; j += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t g = j / kGroup;
+    const uint32_t e = up_state ? up_state[g] : top_entry;
+    const uint64_t ec = up_state ? up_cnt[g] : 0;
+    if (j % kGroup == 0) {
+      st[j] = e;
+      sc[j] = ec;
+    } else {
+      st[j] = P[(j - 1) * 32 + e];
+      sc[j] = ec + PC[(j - 1) * 32 + e];
+    }
+  }
+}
+
+// Outputs: chunk ends (original ids), final state (transformed), total count.
+__global__ void k_enum_out(DevImage img, const uint32_t* __restrict__ st0, const uint8_t* __restrict__ P0top,
+                           const uint64_t* __restrict__ PC0top, uint64_t top_last, uint32_t q0t, uint64_t nsub,
+                           uint32_t per_chunk, uint64_t N, uint32_t* __restrict__ chunk_ends, Ctl* ctl,
+                           uint32_t* __restrict__ x_final) {
+  const uint32_t fin = P0top[top_last * 32 + q0t];
+  for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < N; c += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t jn = (c + 1) * per_chunk;  // first sub-chunk after chunk c
+    const uint32_t s = jn < nsub ? st0[jn] : fin;
+    if (chunk_ends) chunk_ends[c] = img.inv[s];
+  }
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    *x_final = fin;
+    ctl->accept_count = PC0top[top_last * 32 + q0t];
+  }
+}
+
+template <int MODE, int NE>
+cudaError_t walk_t(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, uint8_t* M, uint64_t* Cn,
+                   cudaStream_t st, int sms) {
+  auto kern = k_enum_walk<MODE, NE>;
+  const uint32_t smem = smem_bytes_for(img);
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  uint64_t grid = (nsub + 127) / 128;
+  const uint64_t cap = (uint64_t)sms * 16;
+  if (grid > cap) grid = cap;
+  kern<<<(unsigned)grid, 128, smem, st>>>(img, rp.in, rp.len, E, nsub, M, Cn);
+  return cudaGetLastError();
+}
+
+template <int MODE>
+cudaError_t walk_m(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, uint8_t* M, uint64_t* Cn,
+                   cudaStream_t st, int sms) {
+  const uint32_t nt = img.n + 1;
+  if (nt <= 8) return walk_t<MODE, 8>(img, rp, E, nsub, M, Cn, st, sms);
+  if (nt <= 16) return walk_t<MODE, 16>(img, rp, E, nsub, M, Cn, st, sms);
+  return walk_t<MODE, 32>(img, rp, E, nsub, M, Cn, st, sms);
+}
+
+}  // namespace
+
+// Scratch layout for the enumeration (levels of maps + per-level states).
+uint64_t enum_scratch_bytes(uint64_t nsub) {
+  uint64_t tot = 0, cnt = nsub;
+  for (;;) {
+    tot += cnt * 32 * (1 + 8) + cnt * (4 + 8) + 64;
+    if (cnt <= kGroup) break;
+    cnt = (cnt + kGroup - 1) / kGroup;
+  }
+  return tot + 1024;
+}
+
+// phases: 1 = start-independent part (walk + group scans); 2 = start-dependent
+// part (descend from rp.q0t, outputs).  top_M/top_C (nullable) receive the
+// device addresses of the whole-stream map and counts (entry q = from state q).
+cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t E, void* scratch,
+                             uint32_t* d_chunk_ends, Ctl* d_ctl, uint32_t* d_x_final, cudaStream_t st, int sms,
+                             int phases, const uint8_t** top_M, const uint64_t** top_C) {
+  const uint64_t nsub = (rp.len + E - 1) / E;
+  // carve levels
+  struct Lvl { uint8_t* M; uint64_t* C; uint32_t* s; uint64_t* sc; uint64_t cnt; };
+  Lvl lv[16];
+  int L = 0;
+  uint8_t* p = reinterpret_cast<uint8_t*>(scratch);
+  auto take = [&](uint64_t bytes) { uint8_t* r = p; p += (bytes + 255) & ~255ull; return r; };
+  uint64_t cnt = nsub;
+  for (;;) {
+    lv[L].cnt = cnt;
+    lv[L].M = take(cnt * 32);
+    lv[L].C = reinterpret_cast<uint64_t*>(take(cnt * 32 * 8));
+    lv[L].s = reinterpret_cast<uint32_t*>(take(cnt * 4));
+    lv[L].sc = reinterpret_cast<uint64_t*>(take(cnt * 8));
+    L++;
+    if (cnt <= kGroup || L == 16) break;
+    cnt = (cnt + kGroup - 1) / kGroup;
+  }
+  const uint64_t top_last = lv[L - 1].cnt - 1;
+  if (top_M) *top_M = lv[L - 1].M + top_last * 32;
+  if (top_C) *top_C = lv[L - 1].C + top_last * 32;
+  cudaError_t e = cudaSuccess;
+  if (phases & 1) {
+  switch (img.mode) {
+    case MODE_U8: e = walk_m<MODE_U8>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
+    case MODE_U16: e = walk_m<MODE_U16>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
+    default: e = walk_m<MODE_U32>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
+  }
+  if (e != cudaSuccess) return e;
+  for (int l = 0; l < L; l++) {
+    const uint64_t ng = (lv[l].cnt + kGroup - 1) / kGroup;
+    uint64_t grid = (ng * 32 + 127) / 128;
+    if (grid > (uint64_t)sms * 16) grid = (uint64_t)sms * 16;
+    k_enum_group<<<(unsigned)grid, 128, 0, st>>>(lv[l].M, lv[l].C, lv[l].cnt, l + 1 < L ? lv[l + 1].M : nullptr,
+                                                 l + 1 < L ? lv[l + 1].C : nullptr);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  }
+  }
+  if (!(phases & 2)) return cudaSuccess;
+  for (int l = L - 1; l >= 0; l--) {
+    uint64_t grid = (lv[l].cnt + 255) / 256;
+    if (grid > (uint64_t)sms * 16) grid = (uint64_t)sms * 16;
+    k_enum_descend<<<(unsigned)grid, 256, 0, st>>>(lv[l].M, lv[l].C, lv[l].cnt, l + 1 < L ? lv[l + 1].s : nullptr,
+                                                   l + 1 < L ? lv[l + 1].sc : nullptr, rp.q0t, lv[l].s, lv[l].sc);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+  }
+  uint64_t grid = (rp.N + 255) / 256;
+  if (grid > (uint64_t)sms * 16) grid = (uint64_t)sms * 16;
+  if (grid < 1) grid = 1;
+  k_enum_out<<<(unsigned)grid, 256, 0, st>>>(img, lv[0].s, lv[L - 1].M, lv[L - 1].C, top_last, rp.q0t, nsub,
+                                             rp.B / E, rp.N, d_chunk_ends, d_ctl, d_x_final);
+  return cudaGetLastError();
+}
+
+}  // namespace gspec

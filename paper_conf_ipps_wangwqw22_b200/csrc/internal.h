@@ -1,0 +1,188 @@
+// internal.h — shared declarations of the sm_100a implementation behind
+// include/gspec.h.  Nothing here is visible through the C ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "gspec.h"
+
+namespace gspec {
+
+// Table formats of the transformed DFA.
+enum Mode : uint32_t {
+  MODE_U8 = 1,   // raw-byte table, u8 codes, accept in bit 7, whole table in smem
+  MODE_U16 = 2,  // classed table, u16 codes = tid | acc<<15, hot rows (tid < H) in smem
+  MODE_U32 = 3,  // classed table, u32 codes = tid | acc<<31, hot rows in smem
+};
+
+constexpr uint32_t kQsMax = 16;     // QS cap ("top 16 states")
+constexpr uint32_t kVrMax = 16;     // VR^end / VR^others slots
+constexpr uint32_t kSlots = 2 * kVrMax;
+constexpr uint32_t kEnumMax = 32;   // ENUM: transformed states incl. poison
+
+// POD device view of a loaded DFA, passed by value to every kernel.
+struct DevImage {
+  uint32_t mode;
+  uint32_t n;       // real states; poison tid = n; nt = n + 1
+  uint32_t nsyms;
+  uint32_t C;       // byte classes (incl. the poison class when nsyms < 256)
+  uint32_t H;       // hot rows in smem (MODE_U16/U32); all rows for MODE_U8
+  uint32_t q0t;     // transformed start state
+  uint32_t smem_table_bytes;  // bytes of the smem copy of the table
+  const uint8_t* T8;          // MODE_U8: [256 codes][256 bytes] next code
+  const uint16_t* T16;        // MODE_U16: [nt][C]
+  const uint32_t* T32;        // MODE_U32: [nt][C]
+  const uint8_t* cls;         // [256] byte -> class
+  const uint32_t* qs2;        // [C*C][kQsMax] ranked lookback candidates (tids)
+  const uint8_t* qs2_len;     // [C*C]
+  const uint32_t* qs2_img;    // [C*C] image size
+  const uint32_t* tid2code;   // [nt]
+  const uint32_t* code2tid;   // MODE_U8: [256]
+  const uint32_t* inv;        // [nt] tid -> original id (poison -> n)
+  const uint8_t* acc;         // [nt] accept by tid
+};
+
+// Global record store (hierarchical store, level 3).
+// Slot s of chunk c lives at [s * cap + c]; END slots [0, vr_end), OTH slots
+// [kVrMax, kVrMax + vr_oth).
+struct RecStore {
+  uint64_t cap;
+  uint32_t* start;
+  uint32_t* end;
+  uint32_t* cnt;
+  uint32_t* n_end;     // [cap] records ever appended to VR^end
+  uint32_t* n_oth;     // [cap] records ever appended to VR^others
+  uint32_t* oth_base;  // [cap] n_oth snapshot for this round's helpers
+  uint8_t* next_qs;    // [cap] QS cursor
+  uint32_t* ref_start; // [cap] immutable round-0 path (fusion reference)
+  uint32_t* ref_end;
+  uint32_t* ref_cnt;
+  uint32_t* x;         // [cap+1] incoming state of chunk c (x[N] = final)
+  uint32_t* cur_end;   // [cap] the chunk's current end (c.3: cur_end), constant during a verification
+  uint8_t* found;      // [cap]
+  // per-round scratch of the verify/recover kernel
+  uint8_t* ulen;       // [cap] untried QS candidates of chunk c
+  uint8_t* next_new;   // [cap] QS cursor after this round's helpers
+  uint8_t* hcnt;       // [cap] helpers assigned to chunk c this round
+  uint32_t* prefU;     // [cap] NF: exclusive prefix of ulen over c > f
+  uint32_t* task_chunk;  // [cap+1] task slot -> chunk (0xFFFFFFFF = none)
+  uint32_t* task_start;  // [cap+1]
+  uint32_t* task_j;      // [cap+1] helper index within its chunk
+};
+
+// Device control block of the verify/recover kernel.
+struct Ctl {
+  uint64_t f;            // verified frontier
+  uint32_t tf;           // t_f
+  uint32_t pad0;
+  uint64_t fmin;         // frontier candidate of this round
+  uint32_t changed[4];   // Jacobi flags (rotating)
+  uint32_t done;
+  uint32_t status;
+  uint64_t rounds;
+  uint64_t tasks_mustdo, tasks_sre, tasks_helper, reread_bytes, verify_checks, verify_matches,
+      active_sum;
+  uint64_t accept_count;
+  uint64_t nA, I, nU;    // this round: A-tasks, idle workers, total untried candidates
+  uint64_t jacobi_iters;
+};
+
+struct RunParams {
+  const uint8_t* in;
+  uint32_t q0t;    // transformed start state of chunk 0 (q0 of the DFA, or a shard candidate)
+  uint64_t len;
+  uint32_t B;
+  uint64_t N;
+  int scheme;
+  uint32_t k;      // paths per chunk in round 0
+  uint32_t qs_cap;
+  uint32_t vr_end, vr_oth;
+};
+
+// ---- launchers (each returns the cudaError_t of the launch) ------------------
+cudaError_t launch_build_qs2_raw(const uint32_t* d_ttc, uint32_t n, uint32_t C, uint32_t* scratch, uint32_t grid,
+                                 uint32_t* qs2, uint8_t* qs2_len, uint32_t* qs2_img, cudaStream_t st);
+cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st);
+cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, int sms, cudaStream_t st,
+                            uint64_t* n_done);
+bool spec_path_generic_only();  // GSPEC_SPEC_PATH=generic forces the non-TMA kernel (A/B tests)
+cudaError_t launch_verify_recover(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* d_ctl,
+                                  uint64_t* d_block_tmp, uint32_t* d_chunk_ends, cudaStream_t st, int sm_count);
+uint64_t enum_scratch_bytes(uint64_t nsub);
+cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t E, void* scratch,
+                             uint32_t* d_chunk_ends, Ctl* d_ctl, uint32_t* d_x_final, cudaStream_t st, int sms,
+                             int phases = 3, const uint8_t** top_M = nullptr, const uint64_t** top_C = nullptr);
+cudaError_t launch_features_raw(const DevImage& img, const uint32_t* d_ttc, const uint8_t* in, uint64_t len,
+                                uint32_t B, uint64_t N, const uint32_t* d_x, uint32_t k, uint32_t qs_cap,
+                                unsigned long long* d_counts, uint32_t* d_seen, unsigned long long* d_uniq,
+                                cudaStream_t st);
+
+cudaError_t launch_shard_image(const DevImage& img, const uint32_t* ttc, const uint8_t* w, uint32_t L, uint32_t* mark,
+                               uint32_t* list, uint32_t* count, cudaStream_t st);
+cudaError_t launch_shard_fuse(const DevImage& img, const uint8_t* in, uint64_t len, uint32_t B, const uint32_t* cand,
+                              uint32_t ncand, uint32_t max_chunks, uint32_t* states, unsigned long long* cnt,
+                              uint32_t* info, cudaStream_t st);
+cudaError_t launch_map_init(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, cudaStream_t st);
+cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_t* grp,
+                             const unsigned long long* prefix, const uint32_t* pfinal, const unsigned long long* pcount,
+                             uint32_t* mend, unsigned long long* mcnt, cudaStream_t st);
+cudaError_t launch_map_enum(const uint8_t* topM, const unsigned long long* topC, uint32_t nt, uint32_t* mend,
+                            unsigned long long* mcnt, cudaStream_t st);
+cudaError_t launch_compose(const uint8_t* maps, uint32_t G, uint64_t map_bytes, uint64_t cnt_off, uint32_t q0t,
+                           uint32_t rank, uint32_t* out, cudaStream_t st);
+cudaError_t launch_fix_prefix(const uint32_t* states, uint32_t ncand, uint32_t ci, uint32_t nj, const uint32_t* inv,
+                              uint32_t* chunk_ends, cudaStream_t st);
+
+// ---- handle ------------------------------------------------------------------
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+};
+
+}  // namespace gspec
+
+struct fsm_s {
+  uint32_t n, nsyms, q0;
+  std::vector<uint32_t> table;  // original table (host copy)
+  std::vector<uint8_t> accept;
+  std::vector<uint32_t> perm, inv;  // [n+1]
+  std::vector<uint64_t> freq;       // [n]
+  std::vector<uint8_t> cls;         // [256]
+  gspec::DevImage img{};
+  std::vector<void*> owned;         // device allocations of the image
+  // scratch for runs (grown on demand)
+  gspec::RecStore rs{};
+  uint64_t rs_cap = 0;
+  uint32_t rs_slots_alloc = 0;
+  void* rs_base = nullptr;
+  gspec::Ctl* d_ctl = nullptr;
+  uint64_t* d_block_tmp = nullptr;
+  size_t block_tmp_elems = 0;
+  void* enum_base = nullptr;
+  size_t enum_bytes = 0;
+  void* feat_base = nullptr;
+  size_t feat_bytes = 0;
+  int sm_count = 0;
+  int device = 0;
+  fsm_scheme auto_scheme = FSM_SCHEME_SRE;
+  bool auto_selected = false;
+  const uint32_t* d_ttc = nullptr;   // [nt][C] transformed tid x class table (prep/features)
+  uint32_t* d_small = nullptr;       // small device scratch (ENUM final state, shard compose)
+  // fsm_run_host staging
+  void* h_dev_in = nullptr;
+  void* h_dev_ce = nullptr;
+  uint64_t h_in_cap = 0, h_ce_cap = 0;
+  // sharded runs (state kept between fsm_shard_map and fsm_shard_finish)
+  void* shard_base = nullptr;   // device scratch of the shard steps
+  size_t shard_bytes = 0;
+  int shard_mode = -1;          // 0 fused/single path, 1 enum, 2 multi-path
+  const uint8_t* shard_in = nullptr;
+  uint64_t shard_len = 0;
+  uint32_t shard_ncand = 0, shard_nj = 0;  // candidates; chunks covered by the fused prefix
+  uint32_t shard_E = 0;
+  fsm_scheme shard_scheme = FSM_SCHEME_SRE;
+  std::vector<uint32_t> shard_cand, shard_grp, shard_dist;
+};

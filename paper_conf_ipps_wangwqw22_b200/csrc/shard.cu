@@ -1,0 +1,211 @@
+// shard.cu — B8: multi-GPU contiguous sharding.
+//
+// Rank g owns a contiguous, chunk-aligned shard.  Its start state is unknown
+// (g > 0), but it lies in the image of all states over the bytes just before
+// the shard ("the real start state ... must be contained in the produced end
+// state set").  Each rank enumerates that candidate set over its first
+// chunks with path fusion (paths that meet stay merged), runs the normal
+// speculative pipeline from the merge point, and publishes a state map over
+// the transformed states; an allgather + composition fixes every start.
+#include "internal.h"
+#include "walk.cuh"
+
+namespace gspec {
+namespace {
+
+constexpr uint32_t kNoState = 0xFFFFFFFFu;
+
+// candidate set: image of all real states over w[0..L) (L <= 16), compacted
+// in increasing id order by one block.
+__global__ void __launch_bounds__(1024) k_image(DevImage img, const uint32_t* __restrict__ ttc,
+                                                const uint8_t* __restrict__ w, uint32_t L,
+                                                uint32_t* __restrict__ mark, uint32_t* __restrict__ list,
+                                                uint32_t* __restrict__ count) {
+  const uint32_t nt = img.n + 1;
+  __shared__ uint8_t cl[16];
+  __shared__ uint32_t wsum[32];
+  __shared__ uint32_t base;
+  if (threadIdx.x < L) cl[threadIdx.x] = img.cls[w[threadIdx.x]];
+  for (uint32_t s = threadIdx.x; s < nt; s += blockDim.x) mark[s] = 0;
+  if (threadIdx.x == 0) base = 0;
+  __syncthreads();
+  for (uint32_t q = threadIdx.x; q < img.n; q += blockDim.x) {
+    uint32_t t = q;
+    for (uint32_t i = 0; i < L; i++) t = ttc[(uint64_t)t * img.C + cl[i]];
+    mark[t] = 1;
+  }
+  __syncthreads();
+  for (uint32_t t0 = 0; t0 < nt; t0 += blockDim.x) {
+    const uint32_t s = t0 + threadIdx.x;
+    const bool m = s < nt && mark[s];
+    const uint32_t bal = __ballot_sync(0xffffffffu, m);
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (lane == 0) wsum[warp] = __popc(bal);
+    __syncthreads();
+    uint32_t off = base;
+    for (uint32_t k = 0; k < warp; k++) off += wsum[k];
+    if (m) list[off + __popc(bal & ((1u << lane) - 1))] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      uint32_t tot = 0;
+      for (uint32_t k = 0; k < blockDim.x / 32; k++) tot += wsum[k];
+      base += tot;
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *count = base;
+}
+
+// Path fusion over whole chunks: thread i walks candidate i chunk by chunk and
+// records its state at every chunk end; stop after the first chunk where all
+// candidates coincide (info[0] = that chunk) or after max_chunks (info[0] =
+// kNoState).  info[1] = chunks walked.
+template <int MODE>
+__global__ void __launch_bounds__(1024) k_fuse(DevImage img, const uint8_t* __restrict__ in, uint64_t len, uint32_t B,
+                                               const uint32_t* __restrict__ cand, uint32_t ncand, uint32_t max_chunks,
+                                               uint32_t* __restrict__ states, unsigned long long* __restrict__ cnt,
+                                               uint32_t* __restrict__ info) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  __shared__ uint32_t s0;
+  stage_table(img, smem);
+  __syncthreads();
+  using S = Step<MODE>;
+  const uint32_t i = threadIdx.x;
+  uint32_t code = i < ncand ? __ldg(img.tid2code + cand[i]) : 0;
+  unsigned long long total = 0;
+  const uint64_t N = (len + B - 1) / B;
+  uint32_t merged = kNoState, j = 0;
+  for (; j < max_chunks && j < N; j++) {
+    const uint64_t lo = (uint64_t)j * B, n = min((uint64_t)B, len - lo);
+    uint32_t acc = 0;
+    if (i < ncand) code = walk_bytes<MODE>(img, smem, in + lo, n, code, acc);
+    total += acc;
+    const uint32_t t = S::tid(img, code);
+    if (i < ncand) states[(uint64_t)j * ncand + i] = t;
+    if (i == 0) s0 = t;
+    __syncthreads();
+    const bool same = __syncthreads_and(i >= ncand || t == s0);
+    if (same) { merged = j; j++; break; }
+  }
+  if (i < ncand) cnt[i] = total;
+  if (i == 0) { info[0] = merged; info[1] = j; }
+}
+
+__global__ void k_map_init(uint32_t* __restrict__ mend, unsigned long long* __restrict__ mcnt, uint32_t nt) {
+  for (uint32_t s = blockIdx.x * blockDim.x + threadIdx.x; s < nt; s += gridDim.x * blockDim.x) {
+    mend[s] = kNoState;
+    mcnt[s] = 0;
+  }
+}
+
+// map[cand[i]] = (final of its fused path, prefix count + path count)
+__global__ void k_map_write(const uint32_t* __restrict__ cand, uint32_t ncand, const uint32_t* __restrict__ grp,
+                            const unsigned long long* __restrict__ prefix, const uint32_t* __restrict__ pfinal,
+                            const unsigned long long* __restrict__ pcount, uint32_t* __restrict__ mend,
+                            unsigned long long* __restrict__ mcnt) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x) {
+    const uint32_t g = grp[i];
+    mend[cand[i]] = pfinal[g];
+    mcnt[cand[i]] = (prefix ? prefix[i] : 0ull) + pcount[g];
+  }
+}
+
+// ENUM shard: the whole-shard map for every state.
+__global__ void k_map_enum(const uint8_t* __restrict__ topM, const unsigned long long* __restrict__ topC, uint32_t nt,
+                           uint32_t* __restrict__ mend, unsigned long long* __restrict__ mcnt) {
+  const uint32_t s = threadIdx.x;
+  if (s < nt) { mend[s] = topM[s]; mcnt[s] = topC[s]; }
+}
+
+// s_0 = q0; s_{h+1} = M_h[s_h]: out = {s_rank, final, err, count_lo, count_hi}
+__global__ void k_compose(const uint8_t* __restrict__ maps, uint32_t G, uint64_t map_bytes, uint64_t cnt_off,
+                          uint32_t q0t, uint32_t rank, uint32_t* __restrict__ out) {
+  if (threadIdx.x || blockIdx.x) return;
+  uint32_t s = q0t, srank = q0t, err = 0;
+  unsigned long long c = 0;
+  for (uint32_t h = 0; h < G; h++) {
+    if (h == rank) srank = s;
+    const uint32_t* me = reinterpret_cast<const uint32_t*>(maps + h * map_bytes);
+    const unsigned long long* mc = reinterpret_cast<const unsigned long long*>(maps + h * map_bytes + cnt_off);
+    const uint32_t e = me[s];
+    if (e == kNoState) { err = 1; break; }
+    c += mc[s];
+    s = e;
+  }
+  out[0] = srank;
+  out[1] = s;
+  out[2] = err;
+  out[3] = (uint32_t)(c & 0xFFFFFFFFu);
+  out[4] = (uint32_t)(c >> 32);
+}
+
+// chunk ends [0, nj) of the fused-path prefix of candidate ci
+__global__ void k_fix_prefix(const uint32_t* __restrict__ states, uint32_t ncand, uint32_t ci, uint32_t nj,
+                             const uint32_t* __restrict__ inv, uint32_t* __restrict__ chunk_ends) {
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < nj; j += gridDim.x * blockDim.x)
+    chunk_ends[j] = inv[states[(uint64_t)j * ncand + ci]];
+}
+
+template <int MODE>
+cudaError_t fuse_m(const DevImage& img, const uint8_t* in, uint64_t len, uint32_t B, const uint32_t* cand,
+                   uint32_t ncand, uint32_t max_chunks, uint32_t* states, unsigned long long* cnt, uint32_t* info,
+                   cudaStream_t st) {
+  auto kern = k_fuse<MODE>;
+  const uint32_t smem = smem_bytes_for(img);
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  const uint32_t th = ((ncand + 31) / 32) * 32;
+  kern<<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info);
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+cudaError_t launch_shard_image(const DevImage& img, const uint32_t* ttc, const uint8_t* w, uint32_t L, uint32_t* mark,
+                               uint32_t* list, uint32_t* count, cudaStream_t st) {
+  k_image<<<1, 1024, 0, st>>>(img, ttc, w, L, mark, list, count);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_shard_fuse(const DevImage& img, const uint8_t* in, uint64_t len, uint32_t B, const uint32_t* cand,
+                              uint32_t ncand, uint32_t max_chunks, uint32_t* states, unsigned long long* cnt,
+                              uint32_t* info, cudaStream_t st) {
+  switch (img.mode) {
+    case MODE_U8: return fuse_m<MODE_U8>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
+    case MODE_U16: return fuse_m<MODE_U16>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
+    default: return fuse_m<MODE_U32>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
+  }
+}
+
+cudaError_t launch_map_init(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, cudaStream_t st) {
+  k_map_init<<<(nt + 255) / 256, 256, 0, st>>>(mend, mcnt, nt);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_t* grp,
+                             const unsigned long long* prefix, const uint32_t* pfinal, const unsigned long long* pcount,
+                             uint32_t* mend, unsigned long long* mcnt, cudaStream_t st) {
+  k_map_write<<<(ncand + 255) / 256, 256, 0, st>>>(cand, ncand, grp, prefix, pfinal, pcount, mend, mcnt);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_map_enum(const uint8_t* topM, const unsigned long long* topC, uint32_t nt, uint32_t* mend,
+                            unsigned long long* mcnt, cudaStream_t st) {
+  k_map_enum<<<1, 32, 0, st>>>(topM, topC, nt, mend, mcnt);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_compose(const uint8_t* maps, uint32_t G, uint64_t map_bytes, uint64_t cnt_off, uint32_t q0t,
+                           uint32_t rank, uint32_t* out, cudaStream_t st) {
+  k_compose<<<1, 32, 0, st>>>(maps, G, map_bytes, cnt_off, q0t, rank, out);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_fix_prefix(const uint32_t* states, uint32_t ncand, uint32_t ci, uint32_t nj, const uint32_t* inv,
+                              uint32_t* chunk_ends, cudaStream_t st) {
+  if (!nj) return cudaSuccess;
+  k_fix_prefix<<<(nj + 255) / 256, 256, 0, st>>>(states, ncand, ci, nj, inv, chunk_ends);
+  return cudaGetLastError();
+}
+
+}  // namespace gspec

@@ -1,0 +1,265 @@
+// spec_tma.cu — B2 fast path: speculative execution with TMA-staged input.
+//
+// The stream is viewed as a 2-D tensor [N_full chunks][B bytes].  Each warp
+// owns tiles of 32 consecutive chunks (lane = chunk, Alg. 2 L3 "Forall
+// thread i") and streams them through shared memory with a per-warp
+// multi-stage TMA pipeline: box = 32 rows x 128 B, SWIZZLE_128B so the 32
+// lanes' 16-byte reads of their own rows are bank-conflict-free.  Lanes then
+// run register-resident transition chains over the staged bytes, the
+// transformed table resident in shared memory.  One CTA per SM.
+#include <cuda.h>
+
+#include <algorithm>
+#include <cmath>
+
+#include "internal.h"
+#include "walk.cuh"
+
+namespace gspec {
+namespace {
+
+constexpr uint32_t kRowBytes = 128;             // box inner extent (bytes per chunk per stage)
+constexpr uint32_t kStageBytes = 32 * kRowBytes;  // 32 rows (chunks) per box
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  const uint32_t a = smem_u32(bar);
+  while (!done) {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(a), "r"(parity)
+        : "memory");
+  }
+}
+
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int32_t x, int32_t y) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
+      : "memory");
+}
+
+template <int MODE, int KP, int S>
+__global__ void __launch_bounds__(512, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
+                                                    RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  // layout: [stages: nwarps * S * 4 KiB][mbarriers][table]
+  const uint32_t nwarps = blockDim.x / 32;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint8_t* stages = smem_raw;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw + (size_t)nwarps * S * kStageBytes);
+  uint8_t* table = smem_raw + table_off;
+  stage_table(img, table);
+  if (lane == 0)
+    for (int s = 0; s < S; s++) mbar_init(bars + warp * S + s, 1);
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  __syncthreads();
+  using Sx = Step<MODE>;
+
+  const uint32_t segs = rp.B / kRowBytes;
+  const uint64_t ntiles = (n_full + 31) / 32;
+  const uint64_t gw = (uint64_t)blockIdx.x * nwarps + warp, tw = (uint64_t)gridDim.x * nwarps;
+  if (gw >= ntiles) return;
+  const uint64_t my_tiles = (ntiles - gw + tw - 1) / tw;
+  const uint64_t items = my_tiles * segs;  // (tile, segment) pairs streamed by this warp
+  uint8_t* wst = stages + (size_t)warp * S * kStageBytes;
+  uint64_t* wbar = bars + warp * S;
+
+  auto issue = [&](uint64_t it) {
+    const uint64_t t = gw + (it / segs) * tw;
+    const uint32_t sg = (uint32_t)(it % segs);
+    const int s = (int)(it % S);
+    mbar_expect_tx(wbar + s, kStageBytes);
+    tma_load_2d(wst + (size_t)s * kStageBytes, &tmap, wbar + s, (int32_t)(sg * kRowBytes), (int32_t)(t * 32));
+  };
+  if (lane == 0)
+    for (uint64_t it = 0; it < items && it < (uint64_t)S; it++) issue(it);
+
+  uint32_t st[KP], code[KP], acc[KP], kc = 1;
+  uint64_t c = 0;
+  for (uint64_t it = 0; it < items; it++) {
+    const uint32_t sg = (uint32_t)(it % segs);
+    if (sg == 0) {  // new tile: predict this lane's chunk start (lookback-2 pair table)
+      c = (gw + (it / segs) * tw) * 32 + lane;
+      if (c == 0 || c >= n_full) {
+        kc = 1;
+#pragma unroll
+        for (int p = 0; p < KP; p++) st[p] = rp.q0t;
+      } else {
+        const uint32_t pair = qs_pair(img, rp.in, c, rp.B);
+        const uint32_t ql = __ldg(img.qs2_len + pair);
+        kc = min(rp.k, min(ql, rp.qs_cap));
+#pragma unroll
+        for (int p = 0; p < KP; p++) st[p] = __ldg(img.qs2 + (uint64_t)pair * kQsMax + min((uint32_t)p, kc - 1));
+      }
+#pragma unroll
+      for (int p = 0; p < KP; p++) {
+        code[p] = __ldg(img.tid2code + st[p]);
+        acc[p] = 0;
+      }
+    }
+    const int s = (int)(it % S);
+    mbar_wait(wbar + s, (uint32_t)((it / S) & 1));
+    const uint8_t* row = wst + (size_t)s * kStageBytes + lane * kRowBytes;
+#pragma unroll
+    for (int u = 0; u < (int)(kRowBytes / 16); u++) {
+      const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ (lane & 7)) << 4));  // SWIZZLE_128B
+      const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+#pragma unroll
+        for (int p = 0; p < KP; p++) { code[p] = Sx::template word<0>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+#pragma unroll
+        for (int p = 0; p < KP; p++) { code[p] = Sx::template word<1>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+#pragma unroll
+        for (int p = 0; p < KP; p++) { code[p] = Sx::template word<2>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+#pragma unroll
+        for (int p = 0; p < KP; p++) { code[p] = Sx::template word<3>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+      }
+    }
+    __syncwarp();
+    if (lane == 0 && it + S < items) issue(it + S);  // refill this stage
+    if (sg == segs - 1 && c < n_full) {  // tile done: round-0 records (VR^end)
+      uint32_t e0 = 0;
+#pragma unroll
+      for (int p = 0; p < KP; p++) {
+        const uint32_t e = Sx::tid(img, code[p]);
+        if (p == 0) e0 = e;
+        if ((uint32_t)p < kc) {
+          rs.start[p * rs.cap + c] = st[p];
+          rs.end[p * rs.cap + c] = e;
+          rs.cnt[p * rs.cap + c] = acc[p];
+        }
+      }
+      rs.n_end[c] = kc;
+      rs.n_oth[c] = 0;
+      rs.next_qs[c] = (uint8_t)kc;
+      rs.ref_start[c] = st[0];
+      rs.ref_end[c] = e0;
+      rs.ref_cnt[c] = acc[0];
+      rs.x[c + 1] = e0;
+      rs.cur_end[c] = e0;
+      if (c == 0) rs.x[0] = rp.q0t;
+    }
+  }
+}
+
+using EncodeFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                              const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                              CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeFn get_encode() {
+  static EncodeFn fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeFn>(p);
+  }
+  return fn;
+}
+
+// Pick warps per CTA (one CTA per SM) so the tile count divides evenly over
+// the resident warps (wave quantization), within the smem budget.
+uint32_t pick_warps(uint64_t ntiles, int sms, uint32_t wmax) {
+  uint32_t best = wmax;
+  double best_score = -1;
+  for (uint32_t w = 8; w <= wmax; w++) {
+    const double slots = (double)sms * w;
+    const double rounds = std::ceil((double)ntiles / slots);
+    const double eff = (double)ntiles / (rounds * slots);
+    const double score = eff * std::min(1.0, w / 12.0);  // throughput saturates around 12 warps/SM
+    if (score > best_score + 1e-9) { best_score = score; best = w; }
+  }
+  return best;
+}
+
+template <int MODE, int KP, int S>
+cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
+                         uint64_t n_full, int sms, cudaStream_t st) {
+  auto kern = k_spec_tma<MODE, KP, S>;
+  const uint64_t ntiles = (n_full + 31) / 32;
+  const uint32_t tbytes = smem_bytes_for(img);
+  const uint32_t per_warp = S * kStageBytes + S * 8;
+  const uint32_t avail = 227 * 1024 - tbytes - 1024;
+  uint32_t wmax = std::min<uint32_t>(16, avail / per_warp);
+  if (wmax < 4) return cudaErrorInvalidConfiguration;
+  uint32_t w = pick_warps(ntiles, sms, wmax);
+  if (wmax < 8) w = wmax;
+  const uint32_t stage_bytes = w * S * kStageBytes;
+  const uint32_t table_off = (stage_bytes + w * S * 8 + 127) & ~127u;
+  const uint32_t smem = table_off + tbytes;
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  uint64_t grid = std::min<uint64_t>((uint64_t)sms, (ntiles + w - 1) / w);
+  if (grid < 1) grid = 1;
+  kern<<<(unsigned)grid, w * 32, smem, st>>>(tm, img, rp, rs, n_full, table_off);
+  return cudaGetLastError();
+}
+
+template <int MODE, int KP>
+cudaError_t launch_tma_s(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
+                         uint64_t n_full, int sms, cudaStream_t st) {
+  const uint32_t tbytes = smem_bytes_for(img);
+  if (tbytes + 12 * (3 * kStageBytes) + 2048 <= 227 * 1024)
+    return launch_tma_t<MODE, KP, 3>(tm, img, rp, rs, n_full, sms, st);
+  return launch_tma_t<MODE, KP, 2>(tm, img, rp, rs, n_full, sms, st);
+}
+
+template <int MODE>
+cudaError_t launch_tma_m(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
+                         uint64_t n_full, int sms, cudaStream_t st) {
+  if (rp.k <= 1) return launch_tma_s<MODE, 1>(tm, img, rp, rs, n_full, sms, st);
+  if (rp.k <= 2) return launch_tma_s<MODE, 2>(tm, img, rp, rs, n_full, sms, st);
+  if (rp.k <= 4) return launch_tma_s<MODE, 4>(tm, img, rp, rs, n_full, sms, st);
+  return launch_tma_s<MODE, 8>(tm, img, rp, rs, n_full, sms, st);
+}
+
+}  // namespace
+
+// Returns cudaErrorNotSupported when the TMA path does not apply (caller falls
+// back to the generic kernel): unaligned input, B % 128 != 0, no full chunks.
+cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, int sms, cudaStream_t st,
+                            uint64_t* n_done) {
+  *n_done = 0;
+  const uint64_t n_full = rp.len / rp.B;
+  if (n_full == 0 || rp.B % kRowBytes != 0 || (reinterpret_cast<uintptr_t>(rp.in) & 15u) != 0 || n_full >= (1ull << 31))
+    return cudaErrorNotSupported;
+  EncodeFn enc = get_encode();
+  if (!enc) return cudaErrorNotSupported;
+  CUtensorMap tm;
+  cuuint64_t dims[2] = {rp.B, n_full};
+  cuuint64_t strides[1] = {rp.B};
+  cuuint32_t box[2] = {kRowBytes, 32};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(rp.in), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return cudaErrorNotSupported;
+  cudaError_t e;
+  switch (img.mode) {
+    case MODE_U8: e = launch_tma_m<MODE_U8>(tm, img, rp, rs, n_full, sms, st); break;
+    case MODE_U16: e = launch_tma_m<MODE_U16>(tm, img, rp, rs, n_full, sms, st); break;
+    default: e = launch_tma_m<MODE_U32>(tm, img, rp, rs, n_full, sms, st); break;
+  }
+  if (e == cudaSuccess) *n_done = n_full;
+  return e;
+}
+
+}  // namespace gspec

@@ -1,0 +1,468 @@
+// verify_recover.cu — B3 + B4: parallel speculative verification and
+// speculative recovery with the RR / NF heuristics, as ONE persistent
+// cooperative kernel (the paper's SPEC_RECOVERY_END is a single kernel that
+// loops while f < N, Alg. 3 L1-4).
+//
+// Deterministic round semantics (SURVEY c.3), per round:
+//  V  verification: x_{c+1} = F_c(x_c) from the verified (f, t_f), where
+//     F_c(x) = VR_c(x).end if x in dom VR_c else the chunk's current end.
+//     Solved by chaotic relaxation over all chunks with grid barriers until
+//     no value changes (the fixed point is unique); this batches every run of
+//     Alg. 3's `mark == true` iterations (reading R13).
+//  F  frontier f' = first chunk whose incoming state has no record.
+//  T/H task assignment: must-do (f', t_f') + SRE rear tasks (Alg. 3 L16-18);
+//     RR (Alg. 4 L19-25) / NF (Alg. 5 L25-34) helpers, one per idle worker,
+//     by rank -> (chunk, candidate) maps (no racy queues).
+//  E  execute every task (walks with path fusion against the round-0 path)
+//     and append records: A-tasks to VR^end, helpers to VR^others.
+// Records: hierarchical store — global SoA rings; each
+// thread keeps the record it is matching in registers.
+#include <cooperative_groups.h>
+
+#include "internal.h"
+#include "walk.cuh"
+
+namespace cg = cooperative_groups;
+
+namespace gspec {
+namespace {
+
+constexpr int kBS = 256;
+constexpr uint32_t kFuseMax = 256;  // bytes walked in lockstep with the reference path
+constexpr uint32_t kNone = 0xFFFFFFFFu;
+
+__device__ __forceinline__ uint64_t ld_cg64(const uint64_t* p) { return __ldcg(reinterpret_cast<const unsigned long long*>(p)); }
+
+// exclusive block scan of NCH channels; returns block totals
+template <int NCH>
+__device__ __forceinline__ void block_scan(uint32_t (&v)[NCH], uint32_t (&tot)[NCH], uint32_t (*ws)[kBS / 32]) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint32_t incl[NCH];
+#pragma unroll
+  for (int ch = 0; ch < NCH; ch++) {
+    uint32_t x = v[ch];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+      if (lane >= o) x += y;
+    }
+    incl[ch] = x;
+    if (lane == 31) ws[ch][warp] = x;
+  }
+  __syncthreads();
+  if (warp == 0) {
+#pragma unroll
+    for (int ch = 0; ch < NCH; ch++) {
+      uint32_t x = lane < kBS / 32 ? ws[ch][lane] : 0;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= o) x += y;
+      }
+      if (lane < kBS / 32) ws[ch][lane] = x;  // inclusive warp prefix
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int ch = 0; ch < NCH; ch++) {
+    v[ch] = incl[ch] - v[ch] + (warp > 0 ? ws[ch][warp - 1] : 0);
+    tot[ch] = ws[ch][kBS / 32 - 1];
+  }
+  __syncthreads();
+}
+
+template <typename T>
+__device__ __forceinline__ T block_sum(T v, T* red) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
+  __syncthreads();
+  T s = 0;
+  if (threadIdx.x == 0)
+    for (int w = 0; w < kBS / 32; w++) s += red[w];
+  __syncthreads();
+  return s;  // valid in thread 0
+}
+
+__device__ __forceinline__ uint64_t block_min(uint64_t v, uint64_t* red) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = min(v, (uint64_t)__shfl_down_sync(0xffffffffu, (unsigned long long)v, o));
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
+  __syncthreads();
+  uint64_t s = ~0ull;
+  if (threadIdx.x == 0)
+    for (int w = 0; w < kBS / 32; w++) s = min(s, red[w]);
+  __syncthreads();
+  return s;
+}
+
+// Untried QS candidates of chunk c (Alg. 4 L24, Alg. 5 L30-32): QS_c entries
+// past the cursor that are neither in dom VR_c nor this round's task start.
+__device__ uint32_t untried(const DevImage& img, const RunParams& rp, const RecStore& rs, uint64_t c,
+                            bool busy, uint32_t tstart, uint32_t want_j, uint32_t* q_out, uint32_t* pos_out) {
+  const uint32_t pair = qs_pair(img, rp.in, c, rp.B);
+  const uint32_t ql = min((uint32_t)__ldg(img.qs2_len + pair), rp.qs_cap);
+  const uint32_t nx = __ldcg(rs.next_qs + c);
+  uint32_t m = 0, e;
+  for (uint32_t j = nx; j < ql; j++) {
+    const uint32_t q = __ldg(img.qs2 + (uint64_t)pair * kQsMax + j);
+    if (busy && q == tstart) continue;
+    if (vr_lookup(rs, rp.vr_end, rp.vr_oth, c, q, &e, nullptr)) continue;
+    if (m == want_j) {
+      if (q_out) *q_out = q;
+      if (pos_out) *pos_out = j;
+    }
+    m++;
+  }
+  return m;
+}
+
+// FSM_Processing over chunk c from `start` with path fusion: walk in lockstep
+// with the chunk's round-0 path; once the two states coincide the rest of the
+// path is known (DFA determinism), so end/count follow from the reference.
+template <int MODE>
+__device__ void task_walk(const DevImage& img, const uint8_t* smem, const RunParams& rp, const RecStore& rs,
+                          uint64_t c, uint32_t start, uint32_t* end_out, uint32_t* cnt_out) {
+  using S = Step<MODE>;
+  const uint64_t lo = c * rp.B, n = min((uint64_t)rp.B, rp.len - lo);
+  const uint8_t* p = rp.in + lo;
+  const uint32_t rstart = __ldcg(rs.ref_start + c);
+  const uint32_t rend = __ldcg(rs.ref_end + c), rcnt = __ldcg(rs.ref_cnt + c);
+  if (rstart == start) { *end_out = rend; *cnt_out = rcnt; return; }
+  uint32_t code = __ldg(img.tid2code + start), rcode = __ldg(img.tid2code + rstart);
+  uint32_t acc = 0, racc = 0;
+  uint64_t i = 0;
+  const bool aligned = (reinterpret_cast<uintptr_t>(p) & 15u) == 0;
+  if (aligned) {
+    const uint64_t nf = min(n, (uint64_t)kFuseMax) / 16;
+    const uint4* v = reinterpret_cast<const uint4*>(p);
+    for (uint64_t j = 0; j < nf; j++) {
+      uint4 q = __ldg(v + j);
+      uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+        code = S::template word<0>(img, smem, code, w[t]); acc += S::acc(code);
+        rcode = S::template word<0>(img, smem, rcode, w[t]); racc += S::acc(rcode);
+        code = S::template word<1>(img, smem, code, w[t]); acc += S::acc(code);
+        rcode = S::template word<1>(img, smem, rcode, w[t]); racc += S::acc(rcode);
+        code = S::template word<2>(img, smem, code, w[t]); acc += S::acc(code);
+        rcode = S::template word<2>(img, smem, rcode, w[t]); racc += S::acc(rcode);
+        code = S::template word<3>(img, smem, code, w[t]); acc += S::acc(code);
+        rcode = S::template word<3>(img, smem, rcode, w[t]); racc += S::acc(rcode);
+      }
+      if (code == rcode) {  // merged somewhere in these 16 bytes: identical from here on
+        *end_out = rend;
+        *cnt_out = rcnt - racc + acc;
+        return;
+      }
+    }
+    i = nf * 16;
+  }
+  code = walk_bytes<MODE>(img, smem, p + i, n - i, code, acc);
+  *end_out = S::tid(img, code);
+  *cnt_out = acc;
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
+                                                        uint64_t* btmp, uint32_t* chunk_ends) {
+  cg::grid_group grid = cg::this_grid();
+  extern __shared__ __align__(16) uint8_t smem[];
+  __shared__ uint32_t ws[3][kBS / 32];
+  __shared__ uint64_t red64[kBS / 32];
+  __shared__ uint64_t sh_pre[3];
+  __shared__ uint64_t sh_tot[3];
+  stage_table(img, smem);
+  __syncthreads();
+
+  const uint64_t N = rp.N;
+  const uint32_t G = gridDim.x, b = blockIdx.x;
+  const uint64_t lo = N * b / G, hi = N * (b + 1) / G;
+  const bool sre_like = rp.scheme == FSM_SCHEME_SRE || rp.scheme == FSM_SCHEME_RR || rp.scheme == FSM_SCHEME_NF;
+  const bool helpers = rp.scheme == FSM_SCHEME_RR || rp.scheme == FSM_SCHEME_NF;
+  volatile Ctl* vctl = ctl;
+
+  for (;;) {
+    const uint64_t f = vctl->f;
+    const uint32_t tf = vctl->tf;
+    // ---------------- V: verification by chaotic relaxation ----------------
+    if (b == 0 && threadIdx.x == 0) vctl->fmin = N;
+    uint32_t it = 0;
+    for (;;) {
+      if (b == 0 && threadIdx.x == 0) vctl->changed[(it + 1) % 3] = 0;
+      bool ch = false;
+      for (uint64_t c = max(lo, f) + threadIdx.x; c < hi; c += kBS) {
+        const uint32_t xin = (c == f) ? tf : ld_cg(rs.x + c);
+        uint32_t e;
+        const bool hit = vr_lookup(rs, rp.vr_end, rp.vr_oth, c, xin, &e, nullptr);
+        rs.found[c] = hit;
+        if (!hit) e = ld_cg(rs.cur_end + c);  // F_c default: the chunk's end as of the round start
+        if (ld_cg(rs.x + c + 1) != e) {
+          st_cg(rs.x + c + 1, e);
+          ch = true;
+        }
+      }
+      if (__syncthreads_or(ch) && threadIdx.x == 0) vctl->changed[it % 3] = 1;
+      grid.sync();
+      const bool any = vctl->changed[it % 3] != 0;
+      it++;
+      if (!any) break;
+    }
+    // ---------------- F: frontier + runtime accuracy counters ----------------
+    {
+      uint64_t fm = ~0ull;
+      uint64_t matches = 0, checks = 0;
+      for (uint64_t c = max(lo, f) + threadIdx.x; c < hi; c += kBS) {
+        const bool fd = __ldcg(rs.found + c);
+        st_cg(rs.cur_end + c, ld_cg(rs.x + c + 1));  // rear ripple result (Alg. 3 L10)
+        checks++;
+        matches += fd;
+        if (!fd) fm = min(fm, c);
+      }
+      fm = block_min(fm, red64);
+      checks = block_sum<uint64_t>(checks, red64);
+      matches = block_sum<uint64_t>(matches, red64);
+      if (threadIdx.x == 0) {
+        if (fm != ~0ull) atomicMin(reinterpret_cast<unsigned long long*>(&ctl->fmin), (unsigned long long)fm);
+        atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->verify_checks), (unsigned long long)checks);
+        atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->verify_matches), (unsigned long long)matches);
+        if (b == 0) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->jacobi_iters), (unsigned long long)it);
+      }
+    }
+    grid.sync();
+    const uint64_t f2 = vctl->fmin;
+    if (f2 >= N) break;
+    const uint32_t tf2 = ld_cg(rs.x + f2);
+    // ---------------- T: per-block counts of A-tasks and untried candidates -----
+    {
+      uint64_t cA = 0, cU = 0;
+      for (uint64_t c = max(lo, f2) + threadIdx.x; c < hi; c += kBS) {
+        const bool busy = (c == f2) || (sre_like && c > f2 && !__ldcg(rs.found + c));
+        cA += busy;
+        if (helpers && c > f2) {
+          const uint32_t u = untried(img, rp, rs, c, busy, busy ? ld_cg(rs.x + c) : 0, kNone, nullptr, nullptr);
+          rs.ulen[c] = (uint8_t)u;
+          cU += u;
+        }
+      }
+      cA = block_sum<uint64_t>(cA, red64);
+      cU = block_sum<uint64_t>(cU, red64);
+      if (threadIdx.x == 0) {
+        __stcg(reinterpret_cast<unsigned long long*>(btmp + 2 * b), (unsigned long long)cA);
+        __stcg(reinterpret_cast<unsigned long long*>(btmp + 2 * b + 1), (unsigned long long)cU);
+      }
+    }
+    grid.sync();
+    // block prefixes and totals
+    {
+      uint64_t pA = 0, pU = 0, tA = 0, tU = 0;
+      for (uint32_t j = threadIdx.x; j < G; j += kBS) {
+        const uint64_t a = ld_cg64(btmp + 2 * j), u = ld_cg64(btmp + 2 * j + 1);
+        tA += a;
+        tU += u;
+        if (j < b) { pA += a; pU += u; }
+      }
+      pA = block_sum<uint64_t>(pA, red64);
+      pU = block_sum<uint64_t>(pU, red64);
+      tA = block_sum<uint64_t>(tA, red64);
+      tU = block_sum<uint64_t>(tU, red64);
+      if (threadIdx.x == 0) {
+        sh_pre[0] = pA; sh_pre[1] = pU;
+        sh_tot[0] = tA; sh_tot[1] = tU;
+      }
+      __syncthreads();
+    }
+    const uint64_t nA = sh_tot[0], nU = sh_tot[1];
+    const uint64_t I = N - nA;  // idle workers (W = N logical workers)
+    const uint64_t M = N - f2 - 1;
+    // ---------------- H1: A-task slots, NF prefix of untried counts ------------
+    {
+      uint64_t runA = sh_pre[0], runU = sh_pre[1];
+      const uint64_t start = max(lo, f2);
+      for (uint64_t base = start; base < hi; base += kBS) {
+        const uint64_t c = base + threadIdx.x;
+        const bool in = c < hi;
+        const bool busy = in && ((c == f2) || (sre_like && c > f2 && !__ldcg(rs.found + c)));
+        const uint32_t u = (in && helpers && c > f2) ? __ldcg(rs.ulen + c) : 0u;
+        uint32_t v[2] = {busy ? 1u : 0u, u}, tot[2];
+        block_scan<2>(v, tot, ws);
+        if (busy) {
+          const uint64_t s = runA + v[0];
+          rs.task_chunk[s] = (uint32_t)c;
+          rs.task_start[s] = (c == f2) ? tf2 : ld_cg(rs.x + c);
+          rs.task_j[s] = 0;
+        }
+        if (in && helpers && c > f2) rs.prefU[c] = (uint32_t)(runU + v[1]);
+        runA += tot[0];
+        runU += tot[1];
+      }
+    }
+    grid.sync();
+    // ---------------- H2: helpers (worker rank k) + per-chunk helper counts -----
+    if (helpers) {
+      const uint64_t T = (uint64_t)G * kBS, gt = (uint64_t)b * kBS + threadIdx.x;
+      for (uint64_t k = gt; k < I; k += T) {
+        uint32_t cid = kNone, st = 0, j = 0;
+        if (M > 0) {
+          uint64_t c = 0;
+          bool ok = false;
+          if (rp.scheme == FSM_SCHEME_RR) {  // Alg. 4 L23 (0-indexed, reading R10)
+            c = f2 + 1 + k % M;
+            j = (uint32_t)(k / M);
+            ok = j < __ldcg(rs.ulen + c);
+          } else if (k < nU) {  // NF: k-th untried candidate of QS_{f+1} || QS_{f+2} || ...
+            uint64_t a = f2 + 1, z = N - 1;  // last c with prefU[c] <= k
+            while (a < z) {
+              const uint64_t mid = (a + z + 1) / 2;
+              if (ld_cg(rs.prefU + mid) <= k) a = mid; else z = mid - 1;
+            }
+            c = a;
+            j = (uint32_t)(k - ld_cg(rs.prefU + c));
+            ok = j < __ldcg(rs.ulen + c);
+          }
+          if (ok) {
+            const bool busy = !__ldcg(rs.found + c);  // c > f2: busy iff SRE task
+            uint32_t q = 0;
+            untried(img, rp, rs, c, busy, busy ? ld_cg(rs.x + c) : 0, j, &q, nullptr);
+            cid = (uint32_t)c;
+            st = q;
+          }
+        }
+        rs.task_chunk[nA + k] = cid;
+        rs.task_start[nA + k] = st;
+        rs.task_j[nA + k] = j;
+      }
+      // owners: helpers per chunk, next QS cursor, VR^others base
+      for (uint64_t c = max(lo, f2 + 1) + threadIdx.x; c < hi; c += kBS) {
+        const uint32_t ul = __ldcg(rs.ulen + c);
+        uint64_t h = 0;
+        if (rp.scheme == FSM_SCHEME_RR) {
+          const uint64_t u = c - f2 - 1;
+          const uint64_t ck = I > u ? (I - 1 - u) / M + 1 : 0;
+          h = min((uint64_t)ul, ck);
+        } else {
+          const uint64_t p = ld_cg(rs.prefU + c);
+          h = I > p ? min((uint64_t)ul, I - p) : 0;
+        }
+        uint8_t nx = __ldcg(rs.next_qs + c);
+        if (h > 0) {
+          const bool busy = !__ldcg(rs.found + c);
+          uint32_t pos = 0;
+          untried(img, rp, rs, c, busy, busy ? ld_cg(rs.x + c) : 0, (uint32_t)(h - 1), nullptr, &pos);
+          nx = (uint8_t)(pos + 1);
+        }
+        rs.next_new[c] = nx;
+        rs.oth_base[c] = ld_cg(rs.n_oth + c);
+        rs.hcnt[c] = (uint8_t)h;
+      }
+    }
+    grid.sync();
+    // ---------------- E: execute all tasks, append records --------------------
+    {
+      const uint64_t nslots = nA + (helpers ? I : 0);
+      const uint64_t T = (uint64_t)G * kBS, gt = (uint64_t)b * kBS + threadIdx.x;
+      uint64_t mustdo = 0, sre = 0, hel = 0, reread = 0;
+      for (uint64_t s = gt; s < nslots; s += T) {
+        const uint32_t c = __ldcg(rs.task_chunk + s);
+        if (c == kNone) continue;
+        const uint32_t st = __ldcg(rs.task_start + s);
+        uint32_t e, cnt;
+        task_walk<MODE>(img, smem, rp, rs, c, st, &e, &cnt);
+        reread += min((uint64_t)rp.B, rp.len - (uint64_t)c * rp.B);
+        if (s < nA) {  // VR^end: the chunk's own (must-do or SRE) record
+          const uint32_t ne = ld_cg(rs.n_end + c);
+          const uint64_t o = (uint64_t)(ne % rp.vr_end) * rs.cap + c;
+          st_cg(rs.start + o, st);
+          st_cg(rs.end + o, e);
+          st_cg(rs.cnt + o, cnt);
+          st_cg(rs.n_end + c, ne + 1);
+          st_cg(rs.x + c + 1, e);  // Alg. 3 L17: the recovering chunk's end_c
+          st_cg(rs.cur_end + c, e);
+          if (c == f2) mustdo++; else sre++;
+        } else {  // VR^others: helper record (Fig. 5 (2))
+          const uint32_t j = __ldcg(rs.task_j + s);
+          const uint64_t o = (uint64_t)(kVrMax + (ld_cg(rs.oth_base + c) + j) % rp.vr_oth) * rs.cap + c;
+          st_cg(rs.start + o, st);
+          st_cg(rs.end + o, e);
+          st_cg(rs.cnt + o, cnt);
+          hel++;
+        }
+      }
+      if (helpers)
+        for (uint64_t c = max(lo, f2 + 1) + threadIdx.x; c < hi; c += kBS) {
+          const uint32_t h = __ldcg(rs.hcnt + c);
+          if (h) st_cg(rs.n_oth + c, ld_cg(rs.n_oth + c) + h);
+          rs.next_qs[c] = __ldcg(rs.next_new + c);
+        }
+      mustdo = block_sum<uint64_t>(mustdo, red64);
+      sre = block_sum<uint64_t>(sre, red64);
+      hel = block_sum<uint64_t>(hel, red64);
+      reread = block_sum<uint64_t>(reread, red64);
+      if (threadIdx.x == 0) {
+        auto A = [](uint64_t* p, uint64_t v) {
+          if (v) atomicAdd(reinterpret_cast<unsigned long long*>(p), (unsigned long long)v);
+        };
+        A(&ctl->tasks_mustdo, mustdo);
+        A(&ctl->tasks_sre, sre);
+        A(&ctl->tasks_helper, hel);
+        A(&ctl->reread_bytes, reread);
+        A(&ctl->active_sum, mustdo + sre + hel);
+        if (b == 0) {
+          vctl->rounds = vctl->rounds + 1;
+          vctl->f = f2;
+          vctl->tf = tf2;
+        }
+      }
+    }
+    grid.sync();
+  }
+  // ---------------- Z: finalize (chunk ends, u64 accept count) ----------------
+  {
+    uint64_t total = 0;
+    for (uint64_t c = lo + threadIdx.x; c < hi; c += kBS) {
+      uint32_t e = 0, cnt = 0;
+      vr_lookup(rs, rp.vr_end, rp.vr_oth, c, ld_cg(rs.x + c), &e, &cnt);
+      total += cnt;
+      if (chunk_ends) chunk_ends[c] = __ldg(img.inv + ld_cg(rs.x + c + 1));
+    }
+    total = block_sum<uint64_t>(total, red64);
+    if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->accept_count), (unsigned long long)total);
+  }
+}
+
+template <int MODE>
+cudaError_t launch_m(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t* btmp,
+                     uint32_t* chunk_ends, cudaStream_t st, int sms) {
+  auto kern = k_verify_recover<MODE>;
+  const uint32_t smem = smem_bytes_for(img);
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBS, smem);
+  if (e != cudaSuccess) return e;
+  if (occ < 1) return cudaErrorInvalidConfiguration;
+  uint64_t grid = (uint64_t)sms * occ;
+  const uint64_t want = (rp.N + kBS - 1) / kBS;
+  if (want < grid) grid = want < 1 ? 1 : want;
+  DevImage a0 = img;
+  RunParams a1 = rp;
+  RecStore a2 = rs;
+  void* args[] = {&a0, &a1, &a2, &ctl, &btmp, &chunk_ends};
+  return cudaLaunchCooperativeKernel((const void*)kern, dim3((unsigned)grid), dim3(kBS), args, smem, st);
+}
+
+}  // namespace
+
+uint32_t verify_recover_max_grid();
+
+cudaError_t launch_verify_recover(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* d_ctl,
+                                  uint64_t* d_block_tmp, uint32_t* d_chunk_ends, cudaStream_t st, int sm_count) {
+  if (rp.N == 0) return cudaSuccess;
+  switch (img.mode) {
+    case MODE_U8: return launch_m<MODE_U8>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
+    case MODE_U16: return launch_m<MODE_U16>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
+    default: return launch_m<MODE_U32>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
+  }
+}
+
+}  // namespace gspec

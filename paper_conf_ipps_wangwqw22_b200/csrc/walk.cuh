@@ -1,0 +1,143 @@
+// walk.cuh — the state-transition step of every kernel ("state =
+// Table[state][symbol]"), specialised per table format, plus the shared-memory
+// staging of the hot part of the transformed table.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "internal.h"
+
+namespace gspec {
+
+// Copy the hot table prefix (and the class map) into dynamic shared memory.
+// Layout: [table: smem_table_bytes][cls: 256 B]
+__device__ __forceinline__ void stage_table(const DevImage& img, uint8_t* smem) {
+  const uint4* src = (img.mode == MODE_U8)    ? reinterpret_cast<const uint4*>(img.T8)
+                     : (img.mode == MODE_U16) ? reinterpret_cast<const uint4*>(img.T16)
+                                              : reinterpret_cast<const uint4*>(img.T32);
+  uint4* dst = reinterpret_cast<uint4*>(smem);
+  const uint32_t nv = img.smem_table_bytes / 16;
+  for (uint32_t i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(src + i);
+  if (img.mode != MODE_U8) {
+    const uint4* cs = reinterpret_cast<const uint4*>(img.cls);
+    uint4* cd = reinterpret_cast<uint4*>(smem + img.smem_table_bytes);
+    for (uint32_t i = threadIdx.x; i < 16; i += blockDim.x) cd[i] = __ldg(cs + i);
+  }
+}
+
+__host__ __device__ inline uint32_t smem_bytes_for(const DevImage& img) {
+  return img.smem_table_bytes + (img.mode == MODE_U8 ? 0u : 256u);
+}
+
+template <int MODE>
+struct Step;
+
+// MODE_U8: code < 256 with the accept flag in bit 7; the next code of (code, b)
+// sits at byte (code << 8) | b, so one PRMT forms the address from the packed
+// input word and the current code.
+template <>
+struct Step<MODE_U8> {
+  static constexpr uint32_t kShift = 7;
+  template <int K>
+  static __device__ __forceinline__ uint32_t word(const DevImage&, const uint8_t* s, uint32_t code, uint32_t w) {
+    return s[__byte_perm(w, code, 0x5540 | K)];
+  }
+  static __device__ __forceinline__ uint32_t byte(const DevImage&, const uint8_t* s, uint32_t code, uint32_t b) {
+    return s[(code << 8) | b];
+  }
+  static __device__ __forceinline__ uint32_t acc(uint32_t code) { return code >> 7; }
+  static __device__ __forceinline__ uint32_t tid(const DevImage& img, uint32_t code) { return __ldg(img.code2tid + code); }
+};
+
+// MODE_U16 / MODE_U32: classed rows; tid < H is hot (smem), else global/L2.
+template <typename CodeT, int SHIFT>
+struct StepClassed {
+  static constexpr uint32_t kShift = SHIFT;
+  static constexpr uint32_t kMask = (1u << SHIFT) - 1u;
+  static __device__ __forceinline__ uint32_t byte(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t b) {
+    const CodeT* st = reinterpret_cast<const CodeT*>(s);
+    const uint8_t* sc = s + img.smem_table_bytes;
+    uint32_t t = code & kMask;
+    uint32_t idx = t * img.C + sc[b];
+    if (t < img.H) return st[idx];
+    const CodeT* g = (sizeof(CodeT) == 2) ? reinterpret_cast<const CodeT*>(img.T16) : reinterpret_cast<const CodeT*>(img.T32);
+    return __ldg(g + idx);
+  }
+  template <int K>
+  static __device__ __forceinline__ uint32_t word(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t w) {
+    return byte(img, s, code, (w >> (8 * K)) & 0xffu);
+  }
+  static __device__ __forceinline__ uint32_t acc(uint32_t code) { return code >> SHIFT; }
+  static __device__ __forceinline__ uint32_t tid(const DevImage&, uint32_t code) { return code & kMask; }
+};
+
+template <>
+struct Step<MODE_U16> : StepClassed<uint16_t, 15> {};
+template <>
+struct Step<MODE_U32> : StepClassed<uint32_t, 31> {};
+
+// Walk one path over [p, p+n) bytes from `code`; returns end code, adds accepts.
+template <int MODE>
+__device__ __forceinline__ uint32_t walk_bytes(const DevImage& img, const uint8_t* s, const uint8_t* p, uint64_t n,
+                                               uint32_t code, uint32_t& acc) {
+  using S = Step<MODE>;
+  uint64_t i = 0;
+  // vector part when 16-byte aligned
+  if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
+    const uint4* v = reinterpret_cast<const uint4*>(p);
+    uint64_t nv = n / 16;
+    for (uint64_t j = 0; j < nv; j++) {
+      uint4 q = __ldg(v + j);
+      uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+        code = S::template word<0>(img, s, code, w[t]); acc += S::acc(code);
+        code = S::template word<1>(img, s, code, w[t]); acc += S::acc(code);
+        code = S::template word<2>(img, s, code, w[t]); acc += S::acc(code);
+        code = S::template word<3>(img, s, code, w[t]); acc += S::acc(code);
+      }
+    }
+    i = nv * 16;
+  }
+  for (; i < n; i++) {
+    code = S::byte(img, s, code, __ldg(p + i));
+    acc += S::acc(code);
+  }
+  return code;
+}
+
+// ---- coherent (L2) accessors for data written by other CTAs of a persistent kernel
+__device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) { return __ldcg(p); }
+__device__ __forceinline__ void st_cg(uint32_t* p, uint32_t v) { __stcg(p, v); }
+
+// Look x up in VR_c (END slots then OTH slots).  Returns true on a match.
+__device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, uint32_t vr_oth, uint64_t c,
+                                          uint32_t x, uint32_t* end, uint32_t* cnt) {
+  uint32_t ne = min(ld_cg(rs.n_end + c), vr_end);
+  for (uint32_t s = 0; s < ne; s++) {
+    if (ld_cg(rs.start + s * rs.cap + c) == x) {
+      *end = ld_cg(rs.end + s * rs.cap + c);
+      if (cnt) *cnt = ld_cg(rs.cnt + s * rs.cap + c);
+      return true;
+    }
+  }
+  uint32_t no = min(ld_cg(rs.n_oth + c), vr_oth);
+  for (uint32_t s = 0; s < no; s++) {
+    uint64_t o = (uint64_t)(kVrMax + s) * rs.cap + c;
+    if (ld_cg(rs.start + o) == x) {
+      *end = ld_cg(rs.end + o);
+      if (cnt) *cnt = ld_cg(rs.cnt + o);
+      return true;
+    }
+  }
+  return false;
+}
+
+// Ranked lookback candidates of chunk c >= 1 (lookback-2 pair table).
+__device__ __forceinline__ uint32_t qs_pair(const DevImage& img, const uint8_t* in, uint64_t c, uint32_t B) {
+  uint64_t e = c * (uint64_t)B;
+  uint32_t a = __ldg(in + e - 2), b = __ldg(in + e - 1);
+  return (uint32_t)__ldg(img.cls + a) * img.C + __ldg(img.cls + b);
+}
+
+}  // namespace gspec

@@ -1,0 +1,115 @@
+"""Multi-GPU contiguous sharding: one process per GPU.
+
+Rank g owns a contiguous, chunk-aligned shard of the stream.  It reduces the
+shard to a state map over the transformed states (fsm_shard_map: candidate
+starts = lookback image of the bytes before the shard, enumerated with
+path fusion, then the speculative pipeline), ONE allgather exchanges the maps
+(NCCL over NVLink on GPUs; any torch.distributed backend works), and every
+rank composes them from q0 and fixes its chunk ends (fsm_shard_finish).
+
+Map layout (fsm_map_bytes): uint32 end[nt] (0xFFFFFFFF = not a candidate),
+padded to 8 bytes, then uint64 count[nt]; nt = nstates + 1 (poison last).
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+
+from . import FSM, Result, _check, _lib, _run_opts, fsm_num_chunks, fsm_result
+
+NO_STATE = 0xFFFFFFFF
+
+
+def map_layout(nt: int):
+    off = (nt * 4 + 7) & ~7
+    return off, off + nt * 8
+
+
+def shard_bounds(total_len: int, world: int, rank: int, chunk_bytes: int = 4096):
+    """Chunk-aligned contiguous shard [lo, hi) of rank among world."""
+    nchunks = fsm_num_chunks(total_len, chunk_bytes)
+    c0 = nchunks * rank // world
+    c1 = nchunks * (rank + 1) // world
+    return min(total_len, c0 * chunk_bytes), min(total_len, c1 * chunk_bytes)
+
+
+def exchange_lookback(shard, group=None, L: int = 2):
+    """Each rank receives the last L bytes of the previous rank's shard (tiny allgather)."""
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    tail = torch.zeros(16, dtype=torch.uint8, device=shard.device)
+    n = min(L, shard.numel())
+    if n:
+        tail[16 - n:] = shard[shard.numel() - n:]
+    lens = torch.tensor([n], dtype=torch.int64, device=shard.device)
+    tails = [torch.empty_like(tail) for _ in range(world)]
+    allens = [torch.empty_like(lens) for _ in range(world)]
+    dist.all_gather(tails, tail, group=group)
+    dist.all_gather(allens, lens, group=group)
+    if rank == 0:
+        return tail[:0]
+    m = int(allens[rank - 1].item())
+    return tails[rank - 1][16 - m:]
+
+
+def run_sharded(fsm: FSM, shard, lookback, group=None, scheme="auto", chunk_bytes=4096, spec_k=4,
+                chunk_ends=True, stream=None) -> Result:
+    """fsm_shard_map -> all_gather_into_tensor(maps) -> fsm_shard_finish."""
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    o = _run_opts(scheme, chunk_bytes, spec_k, stream=stream)
+    mb = fsm.map_bytes()
+    local = torch.empty(mb, dtype=torch.uint8, device=shard.device)
+    n = fsm_num_chunks(shard.numel(), chunk_bytes)
+    ce = torch.empty(max(n, 1), dtype=torch.int32, device=shard.device) if chunk_ends else None
+    lb = lookback if lookback is not None and lookback.numel() else None
+    _check(_lib.fsm_shard_map(fsm.handle, shard.data_ptr() if shard.numel() else None, shard.numel(),
+                              lb.data_ptr() if lb is not None else None, lb.numel() if lb is not None else 0,
+                              ctypes.byref(o), local.data_ptr(), ce.data_ptr() if ce is not None else None),
+           "fsm_shard_map")
+    gathered = torch.empty(world * mb, dtype=torch.uint8, device=shard.device)
+    dist.all_gather_into_tensor(gathered, local, group=group)
+    r = fsm_result()
+    _check(_lib.fsm_shard_finish(fsm.handle, gathered.data_ptr(), world, rank, ctypes.byref(o),
+                                 ce.data_ptr() if ce is not None else None, ctypes.byref(r)), "fsm_shard_finish")
+    return Result.from_c(r, ce[:n] if ce is not None else None)
+
+
+# ---- host-side helpers (CPU process groups, tests) ----------------------------
+def pack_map(end: np.ndarray, count: np.ndarray) -> np.ndarray:
+    """Pack (end[nt] uint32, count[nt] uint64) into the wire layout."""
+    nt = len(end)
+    off, total = map_layout(nt)
+    buf = np.zeros(total, np.uint8)
+    buf[:nt * 4] = np.ascontiguousarray(end, np.uint32).view(np.uint8)
+    buf[off:off + nt * 8] = np.ascontiguousarray(count, np.uint64).view(np.uint8)
+    return buf
+
+
+def unpack_map(buf: np.ndarray, nt: int):
+    off, total = map_layout(nt)
+    b = np.ascontiguousarray(buf[:total])
+    return b[:nt * 4].view(np.uint32), b[off:off + nt * 8].view(np.uint64)
+
+
+def compose_maps_host(maps: np.ndarray, nt: int, q0t: int):
+    """s_0 = q0; s_{g+1} = M_g[s_g]; count = sum_g C_g[s_g].  Returns (starts[G+1], count)."""
+    G = maps.shape[0]
+    s = q0t
+    starts = [s]
+    total = 0
+    for g in range(G):
+        e, c = unpack_map(maps[g], nt)
+        if int(e[s]) == NO_STATE:
+            raise RuntimeError(f"shard {g}: start state {s} not in its candidate set")
+        total += int(c[s])
+        s = int(e[s])
+        starts.append(s)
+    return starts, total
