@@ -83,46 +83,57 @@ int ensure_records(fsm_t f, uint64_t N) {
   if (f->rs_cap >= N && f->rs_base) return FSM_OK;
   if (f->rs_base) cudaFree(f->rs_base);
   f->rs_base = nullptr;
+  f->rs_cap = 0;
   uint64_t cap = std::max<uint64_t>(N, 1024);
   cap = (cap + 255) & ~255ull;
-  // u32 arrays: start/end/cnt (kSlots each) + n_end, n_oth, oth_base, ref x3, x(+1), prefU, task x3 (+1)
-  const uint64_t u32s = cap * 3 * kSlots + cap * 11 + 8 + 3 * 8;
-  const uint64_t u8s = cap * 5;  // next_qs, found, ulen, next_new, hcnt
-  size_t bytes = u32s * 4 + u8s + 4096;
+  // carve the store: a dry run (base = null) sizes it, the second pass assigns pointers
+  RecStore r{};
+  auto carve = [&](uint8_t* base) -> uint64_t {
+    uint64_t off = 0;
+    auto take = [&](uint64_t bytes) -> uint8_t* {
+      uint8_t* q = base ? base + off : nullptr;
+      off += (bytes + 255) & ~255ull;
+      return q;
+    };
+    r.cap = cap;
+    r.start = (uint32_t*)take(4 * cap * kSlots);
+    r.end = (uint32_t*)take(4 * cap * kSlots);
+    r.cnt = (uint32_t*)take(4 * cap * kSlots);
+    r.n_end = (uint32_t*)take(4 * cap);
+    r.n_oth = (uint32_t*)take(4 * cap);
+    r.oth_base = (uint32_t*)take(4 * cap);
+    r.ref_start = (uint32_t*)take(4 * cap);
+    r.ref_end = (uint32_t*)take(4 * cap);
+    r.ref_cnt = (uint32_t*)take(4 * cap);
+    r.x = (uint32_t*)take(4 * (cap + 8));
+    r.cur_end = (uint32_t*)take(4 * cap);
+    r.prefU = (uint32_t*)take(4 * cap);
+    r.task_chunk = (uint32_t*)take(4 * (cap + 8));
+    r.task_start = (uint32_t*)take(4 * (cap + 8));
+    r.task_j = (uint32_t*)take(4 * (cap + 8));
+    r.next_qs = take(cap);
+    r.found = take(cap);
+    r.ulen = take(cap);
+    r.next_new = take(cap);
+    r.hcnt = take(cap);
+    return off;
+  };
+  const uint64_t bytes = carve(nullptr);
   void* p = nullptr;
   cudaError_t e = cudaMalloc(&p, bytes);
   if (e != cudaSuccess) return fail(FSM_ENOMEM, std::string("record store: ") + cudaGetErrorString(e));
+  carve(reinterpret_cast<uint8_t*>(p));
+  f->rs = r;
   f->rs_base = p;
   f->rs_cap = cap;
-  uint32_t* u = reinterpret_cast<uint32_t*>(p);
-  RecStore& r = f->rs;
-  r.cap = cap;
-  r.start = u; u += cap * kSlots;
-  r.end = u; u += cap * kSlots;
-  r.cnt = u; u += cap * kSlots;
-  r.n_end = u; u += cap;
-  r.n_oth = u; u += cap;
-  r.oth_base = u; u += cap;
-  r.ref_start = u; u += cap;
-  r.ref_end = u; u += cap;
-  r.ref_cnt = u; u += cap;
-  r.x = u; u += cap + 8;
-  r.cur_end = u; u += cap;
-  r.prefU = u; u += cap;
-  r.task_chunk = u; u += cap + 8;
-  r.task_start = u; u += cap + 8;
-  r.task_j = u; u += cap + 8;
-  uint8_t* b = reinterpret_cast<uint8_t*>(u);
-  r.next_qs = b; b += cap;
-  r.found = b; b += cap;
-  r.ulen = b; b += cap;
-  r.next_new = b; b += cap;
-  r.hcnt = b; b += cap;
   return FSM_OK;
 }
 
 int ensure_ctl(fsm_t f) {
   if (!f->d_ctl) CUDA_TRY(cudaMalloc(&f->d_ctl, sizeof(Ctl)));
+  if (!f->h_ctl) CUDA_TRY(cudaMallocHost(&f->h_ctl, sizeof(Ctl)));
+  for (auto& e : f->ev)
+    if (!e) CUDA_TRY(cudaEventCreate(&e));
   const size_t need = 2 * 4096 + 64;
   if (f->block_tmp_elems < need) {
     if (f->d_block_tmp) cudaFree(f->d_block_tmp);
@@ -169,15 +180,10 @@ int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_sche
   rp.qs_cap = o.qs_cap;
   rp.vr_end = o.vr_end;
   rp.vr_oth = o.vr_oth;
-  cudaEvent_t ev[3];
-  for (auto& e : ev) CUDA_TRY(cudaEventCreate(&e));
-  Ctl h{};
-  uint32_t xfin = 0;
+  cudaEvent_t* ev = f->ev;
+  Ctl& h = *f->h_ctl;
   if (scheme == FSM_SCHEME_ENUM) {
-    if (f->n + 1 > kEnumMax) {
-      for (auto& e : ev) cudaEventDestroy(e);
-      return fail(FSM_EUNSUPPORTED, "ENUM needs nstates + 1 <= 32");
-    }
+    if (f->n + 1 > kEnumMax) return fail(FSM_EUNSUPPORTED, "ENUM needs nstates + 1 <= 32");
     // sub-chunk size E | B: small enough for parallelism, bounded scratch
     uint32_t E = o.B;
     while (E % 32 == 0 && E > 256 && (len + E / 2 - 1) / (E / 2) <= (1ull << 22)) E /= 2;
@@ -192,21 +198,17 @@ int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_sche
     }
     CUDA_TRY(cudaMemsetAsync(f->d_ctl, 0, sizeof(Ctl), o.st));
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
-    if (!f->d_small) CUDA_TRY(cudaMalloc(&f->d_small, 64 * sizeof(uint32_t)));
-    CUDA_TRY(launch_enum_full(f->img, rp, E, f->enum_base, d_chunk_ends, f->d_ctl, f->d_small, o.st, f->sm_count));
+    CUDA_TRY(launch_enum_full(f->img, rp, E, f->enum_base, d_chunk_ends, f->d_ctl, &f->d_ctl->xfin, o.st,
+                              f->sm_count));
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   } else {
-    rc = ensure_records(f, N);
-    if (rc) {
-      for (auto& e : ev) cudaEventDestroy(e);
-      return rc;
-    }
-    Ctl init{};
-    init.f = 0;
-    init.tf = q0t;
-    init.fmin = N;
-    CUDA_TRY(cudaMemcpyAsync(f->d_ctl, &init, sizeof(Ctl), cudaMemcpyHostToDevice, o.st));
+    if ((rc = ensure_records(f, N))) return rc;
+    std::memset(&h, 0, sizeof(Ctl));
+    h.f = 0;
+    h.tf = q0t;
+    h.fmin = N;
+    CUDA_TRY(cudaMemcpyAsync(f->d_ctl, &h, sizeof(Ctl), cudaMemcpyHostToDevice, o.st));
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
     CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
@@ -214,20 +216,15 @@ int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_sche
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   }
   CUDA_TRY(cudaMemcpyAsync(&h, f->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, o.st));
-  if (scheme != FSM_SCHEME_ENUM)
-    CUDA_TRY(cudaMemcpyAsync(&xfin, f->rs.x + N, sizeof(uint32_t), cudaMemcpyDeviceToHost, o.st));
-  else
-    CUDA_TRY(cudaMemcpyAsync(&xfin, f->d_small, sizeof(uint32_t), cudaMemcpyDeviceToHost, o.st));
   CUDA_TRY(cudaStreamSynchronize(o.st));
   float t1 = 0, t2 = 0;
   cudaEventElapsedTime(&t1, ev[0], ev[1]);
   cudaEventElapsedTime(&t2, ev[1], ev[2]);
-  for (auto& e : ev) cudaEventDestroy(e);
   fill_result_stats(out, h);
   out->accept_count = h.accept_count;
   out->ms_spec = t1;
   out->ms_verify = t2;
-  *final_tid = xfin;
+  *final_tid = h.xfin;
   return FSM_OK;
 }
 
@@ -381,13 +378,14 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
       tid2code[t] = code;
       code2tid[code] = t;
     }
-    std::vector<uint8_t> T8(256 * 256, (uint8_t)tid2code[P]);
+    const uint32_t R = 260;  // row stride (walk.cuh kRow8): 4-byte pad rotates rows across banks
+    std::vector<uint8_t> T8(256 * R, (uint8_t)tid2code[P]);
     for (uint32_t code = 0; code < 256; code++) {
       const uint32_t t = code2tid[code];
-      for (uint32_t b = 0; b < 256; b++) T8[code * 256 + b] = (uint8_t)tid2code[ttc[(uint64_t)t * C + f->cls[b]]];
+      for (uint32_t b = 0; b < 256; b++) T8[code * R + b] = (uint8_t)tid2code[ttc[(uint64_t)t * C + f->cls[b]]];
     }
     img.H = nt;
-    img.smem_table_bytes = (n_acc > 0 ? 128 + n_acc : n_na) * 256;
+    img.smem_table_bytes = (((n_acc > 0 ? 128 + n_acc : n_na) * R) + 15) & ~15u;
     if ((rc = upload(f, &img.T8, T8))) return bail(rc);
   } else {
     const uint32_t shift = mode == MODE_U16 ? 15 : 31;
@@ -444,6 +442,9 @@ void fsm_free(fsm_t f) {
   for (void* p : f->owned) cudaFree(p);
   if (f->rs_base) cudaFree(f->rs_base);
   if (f->d_ctl) cudaFree(f->d_ctl);
+  if (f->h_ctl) cudaFreeHost(f->h_ctl);
+  for (auto& e : f->ev)
+    if (e) cudaEventDestroy(e);
   if (f->d_block_tmp) cudaFree(f->d_block_tmp);
   if (f->enum_base) cudaFree(f->enum_base);
   if (f->feat_base) cudaFree(f->feat_base);

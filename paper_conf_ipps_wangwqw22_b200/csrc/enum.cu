@@ -22,7 +22,7 @@ template <int MODE, int NE>
 __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* __restrict__ in, uint64_t len,
                                                   uint32_t E, uint64_t nsub, uint8_t* __restrict__ M,
                                                   uint64_t* __restrict__ Cn) {
-  extern __shared__ __align__(16) uint8_t smem[];
+  extern __shared__ __align__(1024) uint8_t smem[];
   stage_table(img, smem);
   __syncthreads();
   using S = Step<MODE>;
@@ -164,10 +164,11 @@ cudaError_t walk_m(const DevImage& img, const RunParams& rp, uint32_t E, uint64_
 
 // Scratch layout for the enumeration (levels of maps + per-level states).
 uint64_t enum_scratch_bytes(uint64_t nsub) {
+  auto r = [](uint64_t b) { return (b + 255) & ~255ull; };  // same rounding as the carve in launch_enum_full
   uint64_t tot = 0, cnt = nsub;
-  for (;;) {
-    tot += cnt * 32 * (1 + 8) + cnt * (4 + 8) + 64;
-    if (cnt <= kGroup) break;
+  for (int L = 0;; L++) {
+    tot += r(cnt * 32) + r(cnt * 32 * 8) + r(cnt * 4) + r(cnt * 8);
+    if (cnt <= kGroup || L + 1 == 16) break;
     cnt = (cnt + kGroup - 1) / kGroup;
   }
   return tot + 1024;

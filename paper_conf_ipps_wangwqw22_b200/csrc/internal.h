@@ -88,6 +88,8 @@ struct Ctl {
   uint64_t accept_count;
   uint64_t nA, I, nU;    // this round: A-tasks, idle workers, total untried candidates
   uint64_t jacobi_iters;
+  uint32_t xfin;         // transformed final state (written by the last kernel of a run)
+  uint32_t pad1;
 };
 
 struct RunParams {
@@ -159,6 +161,8 @@ struct fsm_s {
   uint32_t rs_slots_alloc = 0;
   void* rs_base = nullptr;
   gspec::Ctl* d_ctl = nullptr;
+  gspec::Ctl* h_ctl = nullptr;       // pinned host mirror (init + readback, async)
+  cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};
   uint64_t* d_block_tmp = nullptr;
   size_t block_tmp_elems = 0;
   void* enum_base = nullptr;

@@ -65,7 +65,7 @@ __global__ void __launch_bounds__(1024) k_fuse(DevImage img, const uint8_t* __re
                                                const uint32_t* __restrict__ cand, uint32_t ncand, uint32_t max_chunks,
                                                uint32_t* __restrict__ states, unsigned long long* __restrict__ cnt,
                                                uint32_t* __restrict__ info) {
-  extern __shared__ __align__(16) uint8_t smem[];
+  extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ uint32_t s0;
   stage_table(img, smem);
   __syncthreads();

@@ -28,7 +28,7 @@ namespace {
 
 template <int MODE, int NI, int KP>
 __global__ void __launch_bounds__(256) k_spec_exec(DevImage img, RunParams rp, RecStore rs, uint64_t c0) {
-  extern __shared__ __align__(16) uint8_t smem[];
+  extern __shared__ __align__(1024) uint8_t smem[];
   stage_table(img, smem);
   __syncthreads();
   using S = Step<MODE>;

@@ -3,7 +3,7 @@
 // The stream is viewed as a 2-D tensor [N_full chunks][B bytes].  Each warp
 // owns tiles of 32 consecutive chunks (lane = chunk, Alg. 2 L3 "Forall
 // thread i") and streams them through shared memory with a per-warp
-// multi-stage TMA pipeline: box = 32 rows x 128 B, SWIZZLE_128B so the 32
+// multi-stage TMA pipeline: box = 32 rows x 64 B, SWIZZLE_64B so the 32
 // lanes' 16-byte reads of their own rows are bank-conflict-free.  Lanes then
 // run register-resident transition chains over the staged bytes, the
 // transformed table resident in shared memory.  One CTA per SM.
@@ -18,7 +18,7 @@
 namespace gspec {
 namespace {
 
-constexpr uint32_t kRowBytes = 128;             // box inner extent (bytes per chunk per stage)
+constexpr uint32_t kRowBytes = 64;              // box inner extent (bytes per chunk per stage)
 constexpr uint32_t kStageBytes = 32 * kRowBytes;  // 32 rows (chunks) per box
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -54,15 +54,15 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
 }
 
 template <int MODE, int KP, int S>
-__global__ void __launch_bounds__(512, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
+__global__ void __launch_bounds__(1024, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
                                                     RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  // layout: [stages: nwarps * S * 4 KiB][mbarriers][table]
+  // layout: [table (at offset 0: the lookup address is one IMAD)][stages: nwarps * S * 2 KiB][mbarriers]
   const uint32_t nwarps = blockDim.x / 32;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  uint8_t* stages = smem_raw;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem_raw + (size_t)nwarps * S * kStageBytes);
-  uint8_t* table = smem_raw + table_off;
+  uint8_t* table = smem_raw;
+  uint8_t* stages = smem_raw + table_off;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(stages + (size_t)nwarps * S * kStageBytes);
   stage_table(img, table);
   if (lane == 0)
     for (int s = 0; s < S; s++) mbar_init(bars + warp * S + s, 1);
@@ -118,7 +118,7 @@ __global__ void __launch_bounds__(512, 1) k_spec_tma(const __grid_constant__ CUt
     const uint8_t* row = wst + (size_t)s * kStageBytes + lane * kRowBytes;
 #pragma unroll
     for (int u = 0; u < (int)(kRowBytes / 16); u++) {
-      const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ (lane & 7)) << 4));  // SWIZZLE_128B
+      const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ ((lane >> 1) & 3)) << 4));  // SWIZZLE_64B
       const uint32_t w[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
       for (int t = 0; t < 4; t++) {
@@ -184,7 +184,7 @@ uint32_t pick_warps(uint64_t ntiles, int sms, uint32_t wmax) {
     const double slots = (double)sms * w;
     const double rounds = std::ceil((double)ntiles / slots);
     const double eff = (double)ntiles / (rounds * slots);
-    const double score = eff * std::min(1.0, w / 12.0);  // throughput saturates around 12 warps/SM
+    const double score = eff * std::min(1.0, w / 24.0);  // ~24 one-chain warps hide the lookup latency
     if (score > best_score + 1e-9) { best_score = score; best = w; }
   }
   return best;
@@ -197,14 +197,13 @@ cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunPa
   const uint64_t ntiles = (n_full + 31) / 32;
   const uint32_t tbytes = smem_bytes_for(img);
   const uint32_t per_warp = S * kStageBytes + S * 8;
-  const uint32_t avail = 227 * 1024 - tbytes - 1024;
-  uint32_t wmax = std::min<uint32_t>(16, avail / per_warp);
+  const uint32_t avail = 227 * 1024 - ((tbytes + 1023) & ~1023u) - 64;
+  uint32_t wmax = std::min<uint32_t>(32, avail / per_warp);
   if (wmax < 4) return cudaErrorInvalidConfiguration;
   uint32_t w = pick_warps(ntiles, sms, wmax);
   if (wmax < 8) w = wmax;
-  const uint32_t stage_bytes = w * S * kStageBytes;
-  const uint32_t table_off = (stage_bytes + w * S * 8 + 127) & ~127u;
-  const uint32_t smem = table_off + tbytes;
+  const uint32_t table_off = (tbytes + 1023) & ~1023u;  // stages start 1 KiB-aligned (swizzle span)
+  const uint32_t smem = table_off + w * S * kStageBytes + w * S * 8;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   uint64_t grid = std::min<uint64_t>((uint64_t)sms, (ntiles + w - 1) / w);
@@ -217,7 +216,7 @@ template <int MODE, int KP>
 cudaError_t launch_tma_s(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
                          uint64_t n_full, int sms, cudaStream_t st) {
   const uint32_t tbytes = smem_bytes_for(img);
-  if (tbytes + 12 * (3 * kStageBytes) + 2048 <= 227 * 1024)
+  if (tbytes + 24 * (3 * kStageBytes) + 2048 <= 227 * 1024)
     return launch_tma_t<MODE, KP, 3>(tm, img, rp, rs, n_full, sms, st);
   return launch_tma_t<MODE, KP, 2>(tm, img, rp, rs, n_full, sms, st);
 }
@@ -249,7 +248,7 @@ cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecS
   cuuint32_t box[2] = {kRowBytes, 32};
   cuuint32_t es[2] = {1, 1};
   CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(rp.in), dims, strides, box, es,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return cudaErrorNotSupported;
   cudaError_t e;

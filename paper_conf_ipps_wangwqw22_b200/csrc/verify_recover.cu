@@ -167,7 +167,7 @@ template <int MODE>
 __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
                                                         uint64_t* btmp, uint32_t* chunk_ends) {
   cg::grid_group grid = cg::this_grid();
-  extern __shared__ __align__(16) uint8_t smem[];
+  extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ uint32_t ws[3][kBS / 32];
   __shared__ uint64_t red64[kBS / 32];
   __shared__ uint64_t sh_pre[3];
@@ -427,6 +427,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     }
     total = block_sum<uint64_t>(total, red64);
     if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->accept_count), (unsigned long long)total);
+    if (b == 0 && threadIdx.x == 0) ctl->xfin = ld_cg(rs.x + N);
   }
 }
 

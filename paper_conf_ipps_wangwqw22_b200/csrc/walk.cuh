@@ -32,18 +32,39 @@ __host__ __device__ inline uint32_t smem_bytes_for(const DevImage& img) {
 template <int MODE>
 struct Step;
 
-// MODE_U8: code < 256 with the accept flag in bit 7; the next code of (code, b)
-// sits at byte (code << 8) | b, so one PRMT forms the address from the packed
-// input word and the current code.
+// MODE_U8: code < 256 with the accept flag in bit 7 (acc += code >> 7).  Row
+// `code` starts at code * kRow8 bytes; the 4-byte pad rotates consecutive
+// rows by one bank, so lanes in different states that read the same byte hit
+// different banks (lanes in the same state read one row: broadcast or
+// distinct banks).
+constexpr uint32_t kRow8 = 260;
+
+__device__ __forceinline__ uint32_t lds_u8(uint32_t saddr) {
+  uint32_t v;
+  asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(saddr));
+  return v;
+}
+
+// (byte K of w) + base, for a 256-aligned base < 2^24: one PRMT
+template <int K>
+__device__ __forceinline__ uint32_t byte_plus(uint32_t w, uint32_t base) {
+  uint32_t b;
+  asm("prmt.b32 %0, %1, %2, %3;" : "=r"(b) : "r"(w), "r"(base), "n"(0x7650 | K));
+  return b;
+}
+
 template <>
 struct Step<MODE_U8> {
   static constexpr uint32_t kShift = 7;
+  // s (the smem table) must be 256-byte aligned: address = code*260 + (base | byte) = PRMT + IMAD
   template <int K>
   static __device__ __forceinline__ uint32_t word(const DevImage&, const uint8_t* s, uint32_t code, uint32_t w) {
-    return s[__byte_perm(w, code, 0x5540 | K)];
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
+    return lds_u8(code * kRow8 + byte_plus<K>(w, base));
   }
   static __device__ __forceinline__ uint32_t byte(const DevImage&, const uint8_t* s, uint32_t code, uint32_t b) {
-    return s[(code << 8) | b];
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
+    return lds_u8(base + code * kRow8 + b);
   }
   static __device__ __forceinline__ uint32_t acc(uint32_t code) { return code >> 7; }
   static __device__ __forceinline__ uint32_t tid(const DevImage& img, uint32_t code) { return __ldg(img.code2tid + code); }

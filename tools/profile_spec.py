@@ -1,0 +1,18 @@
+"""Run the bench workload's fsm_run a few times (for ncu captures).
+usage: python tools/profile_spec.py [config] [scheme] [reps]"""
+import sys
+sys.path.insert(0, '.')
+import torch
+import gen
+import paper_conf_ipps_wangwqw22_b200 as gs
+cfg = sys.argv[1] if len(sys.argv) > 1 else 'c2'
+scheme = sys.argv[2] if len(sys.argv) > 2 else 'sre'
+reps = int(sys.argv[3]) if len(sys.argv) > 3 else 3
+w = gen.workload(cfg)
+x = torch.empty(w.length, dtype=torch.uint8, device='cuda')
+w.device(x)
+fsm = gs.FSM.load(w.table, w.start, w.accept)
+for i in range(reps):
+    r = fsm.run(x, scheme=scheme)
+torch.cuda.synchronize()
+print(r.final_state, r.accept_count, r.stats['ms_spec'], r.stats['ms_verify'])
