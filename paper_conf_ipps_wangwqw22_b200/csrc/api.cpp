@@ -742,6 +742,28 @@ int fsm_shard_map(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* 
   f->shard_scheme = scheme;
   f->shard_grp.assign(ncand, 0);
   f->shard_dist.clear();
+  // 2a. fast path: fuse every candidate with the path of cand[0] (P:427 path
+  // fusion); the shard then runs once, from cand[0], through the normal pipeline
+  if (ncand > 1 && N > 0 && len > 0) {
+    long long* dcnt = reinterpret_cast<long long*>(S.prefix);
+    CUDA_TRY(launch_shard_fuse_ref(f->img, d_shard, len, o.B, S.cand, ncand, kFuseChunks, S.states, S.grp, dcnt,
+                                   o.st));
+    f->shard_merged.resize(ncand);
+    CUDA_TRY(cudaMemcpyAsync(f->shard_merged.data(), S.grp, 4ull * ncand, cudaMemcpyDeviceToHost, o.st));
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+    bool all = true;
+    for (uint32_t m : f->shard_merged) all &= m != kNoState;
+    if (all) {
+      fsm_result r;
+      uint32_t ft = 0;
+      rc = run_core(f, d_shard, len, o, scheme, f->shard_cand[0], d_chunk_ends_local, &r, &ft);
+      if (rc) return rc;
+      CUDA_TRY(launch_map_fused(S.cand, ncand, dcnt, ft, r.accept_count, mend, mcnt, o.st));
+      CUDA_TRY(cudaStreamSynchronize(o.st));
+      f->shard_mode = 3;
+      return FSM_OK;
+    }
+  }
   std::vector<uint32_t> last(f->shard_cand);
   uint32_t nj = 0;
   bool merged = ncand == 1;
@@ -845,6 +867,12 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
       rp.N = N;
       CUDA_TRY(launch_enum_full(f->img, rp, f->shard_E, f->enum_base, d_chunk_ends_local, f->d_ctl, f->d_small + 8,
                                 o.st, f->sm_count, 2));
+    } else if (f->shard_mode == 3) {
+      auto it = std::find(f->shard_cand.begin(), f->shard_cand.end(), srank);
+      if (it == f->shard_cand.end()) return fail(FSM_EINVAL, "rank start not among its candidates");
+      const uint32_t ci = (uint32_t)(it - f->shard_cand.begin());
+      const uint32_t nj = f->shard_merged[ci];  // chunks walked before merging with cand[0]
+      if (nj) CUDA_TRY(launch_fix_prefix(S.states, f->shard_ncand, ci, nj, f->img.inv, d_chunk_ends_local, o.st));
     } else {
       auto it = std::find(f->shard_cand.begin(), f->shard_cand.end(), srank);
       if (it == f->shard_cand.end()) return fail(FSM_EINVAL, "rank start not among its candidates");

@@ -128,6 +128,11 @@ cudaError_t launch_shard_fuse(const DevImage& img, const uint8_t* in, uint64_t l
                               uint32_t ncand, uint32_t max_chunks, uint32_t* states, unsigned long long* cnt,
                               uint32_t* info, cudaStream_t st);
 cudaError_t launch_map_init(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, cudaStream_t st);
+cudaError_t launch_shard_fuse_ref(const DevImage& img, const uint8_t* in, uint64_t len, uint32_t B,
+                                  const uint32_t* cand, uint32_t ncand, uint32_t max_chunks, uint32_t* states,
+                                  uint32_t* merged, long long* dcnt, cudaStream_t st);
+cudaError_t launch_map_fused(const uint32_t* cand, uint32_t ncand, const long long* dcnt, uint32_t fin,
+                             unsigned long long count0, uint32_t* mend, unsigned long long* mcnt, cudaStream_t st);
 cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_t* grp,
                              const unsigned long long* prefix, const uint32_t* pfinal, const unsigned long long* pcount,
                              uint32_t* mend, unsigned long long* mcnt, cudaStream_t st);
@@ -182,7 +187,8 @@ struct fsm_s {
   // sharded runs (state kept between fsm_shard_map and fsm_shard_finish)
   void* shard_base = nullptr;   // device scratch of the shard steps
   size_t shard_bytes = 0;
-  int shard_mode = -1;          // 0 fused/single path, 1 enum, 2 multi-path
+  int shard_mode = -1;          // 0 fused/single path, 1 enum, 2 multi-path, 3 fused with cand[0]
+  std::vector<uint32_t> shard_merged;  // mode 3: chunk where candidate i merged with cand[0]
   const uint8_t* shard_in = nullptr;
   uint64_t shard_len = 0;
   uint32_t shard_ncand = 0, shard_nj = 0;  // candidates; chunks covered by the fused prefix

@@ -7,6 +7,8 @@
 // chunks with path fusion (paths that meet stay merged), runs the normal
 // speculative pipeline from the merge point, and publishes a state map over
 // the transformed states; an allgather + composition fixes every start.
+#include <algorithm>
+
 #include "internal.h"
 #include "walk.cuh"
 
@@ -89,6 +91,61 @@ __global__ void __launch_bounds__(1024) k_fuse(DevImage img, const uint8_t* __re
   }
   if (i < ncand) cnt[i] = total;
   if (i == 0) { info[0] = merged; info[1] = j; }
+}
+
+// Path fusion against a reference candidate (cand[0]): thread i walks its
+// candidate and the reference in lockstep, 16 bytes at a time, until the two
+// states coincide (then the rest of the shard is shared, DFA determinism).
+// merged[i] = chunk in which it merged (kNoState if not within max_chunks),
+// dcnt[i] = accepts(own) - accepts(ref) up to the merge point, states[j][i] =
+// own state at the end of chunk j for chunks before the merge.
+template <int MODE>
+__global__ void __launch_bounds__(1024) k_fuse_ref(DevImage img, const uint8_t* __restrict__ in, uint64_t len,
+                                                   uint32_t B, const uint32_t* __restrict__ cand, uint32_t ncand,
+                                                   uint32_t max_chunks, uint32_t* __restrict__ states,
+                                                   uint32_t* __restrict__ merged, long long* __restrict__ dcnt) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  stage_table(img, smem);
+  __syncthreads();
+  using S = Step<MODE>;
+  for (uint32_t i = threadIdx.x; i < ncand; i += blockDim.x) {
+    uint32_t code = __ldg(img.tid2code + cand[i]), rcode = __ldg(img.tid2code + cand[0]);
+    long long d = 0;
+    uint32_t mj = code == rcode ? 0 : kNoState;
+    const uint64_t N = (len + B - 1) / B;
+    for (uint32_t j = 0; mj == kNoState && j < max_chunks && j < N; j++) {
+      const uint64_t lo = (uint64_t)j * B, n = min((uint64_t)B, len - lo);
+      const uint8_t* p = in + lo;
+      uint64_t t = 0;
+      while (t < n) {
+        const uint64_t m = min((uint64_t)16, n - t);
+        uint32_t a = 0, ra = 0;
+        for (uint64_t q = 0; q < m; q++) {
+          const uint32_t b = __ldg(p + t + q);
+          code = S::byte(img, smem, code, b);
+          a += S::acc(code);
+          rcode = S::byte(img, smem, rcode, b);
+          ra += S::acc(rcode);
+        }
+        d += (long long)a - (long long)ra;
+        t += m;
+        if (code == rcode) { mj = j; break; }
+      }
+      if (mj == kNoState) states[(uint64_t)j * ncand + i] = S::tid(img, code);
+    }
+    merged[i] = mj;
+    dcnt[i] = d;
+  }
+}
+
+// map[cand[i]] = (final, count0 + dcnt[i]) for candidates fused with cand[0]
+__global__ void k_map_fused(const uint32_t* __restrict__ cand, uint32_t ncand, const long long* __restrict__ dcnt,
+                            uint32_t fin, unsigned long long count0, uint32_t* __restrict__ mend,
+                            unsigned long long* __restrict__ mcnt) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x) {
+    mend[cand[i]] = fin;
+    mcnt[cand[i]] = (unsigned long long)((long long)count0 + dcnt[i]);
+  }
 }
 
 __global__ void k_map_init(uint32_t* __restrict__ mend, unsigned long long* __restrict__ mcnt, uint32_t nt) {
@@ -175,6 +232,35 @@ cudaError_t launch_shard_fuse(const DevImage& img, const uint8_t* in, uint64_t l
     case MODE_U16: return fuse_m<MODE_U16>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
     default: return fuse_m<MODE_U32>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
   }
+}
+
+cudaError_t launch_shard_fuse_ref(const DevImage& img, const uint8_t* in, uint64_t len, uint32_t B,
+                                  const uint32_t* cand, uint32_t ncand, uint32_t max_chunks, uint32_t* states,
+                                  uint32_t* merged, long long* dcnt, cudaStream_t st) {
+  const uint32_t smem = smem_bytes_for(img);
+  const uint32_t th = std::min<uint32_t>(1024, ((ncand + 31) / 32) * 32);
+  cudaError_t e;
+  switch (img.mode) {
+    case MODE_U8:
+      if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
+      k_fuse_ref<MODE_U8><<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, merged, dcnt);
+      break;
+    case MODE_U16:
+      if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
+      k_fuse_ref<MODE_U16><<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, merged, dcnt);
+      break;
+    default:
+      if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
+      k_fuse_ref<MODE_U32><<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, merged, dcnt);
+      break;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_map_fused(const uint32_t* cand, uint32_t ncand, const long long* dcnt, uint32_t fin,
+                             unsigned long long count0, uint32_t* mend, unsigned long long* mcnt, cudaStream_t st) {
+  k_map_fused<<<(ncand + 255) / 256, 256, 0, st>>>(cand, ncand, dcnt, fin, count0, mend, mcnt);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_map_init(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, cudaStream_t st) {

@@ -54,7 +54,7 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
 }
 
 template <int MODE, int KP, int S>
-__global__ void __launch_bounds__(1024, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
+__global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
                                                     RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // layout: [table (at offset 0: the lookup address is one IMAD)][stages: nwarps * S * 2 KiB][mbarriers]
@@ -198,7 +198,7 @@ cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunPa
   const uint32_t tbytes = smem_bytes_for(img);
   const uint32_t per_warp = S * kStageBytes + S * 8;
   const uint32_t avail = 227 * 1024 - ((tbytes + 1023) & ~1023u) - 64;
-  uint32_t wmax = std::min<uint32_t>(32, avail / per_warp);
+  uint32_t wmax = std::min<uint32_t>(28, avail / per_warp);  // launch bounds 896 -> 72 regs
   if (wmax < 4) return cudaErrorInvalidConfiguration;
   uint32_t w = pick_warps(ntiles, sms, wmax);
   if (wmax < 8) w = wmax;

@@ -34,6 +34,23 @@ def shard_bounds(total_len: int, world: int, rank: int, chunk_bytes: int = 4096)
     return min(total_len, c0 * chunk_bytes), min(total_len, c1 * chunk_bytes)
 
 
+def _all_gather_cat(t, group=None):
+    """all_gather of equal-size 1-D tensors, concatenated (NCCL: one in-place
+    all_gather_into_tensor on the device; other backends stage through host)."""
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    if dist.get_backend(group) == "nccl":
+        out = torch.empty(world * t.numel(), dtype=t.dtype, device=t.device)
+        dist.all_gather_into_tensor(out, t, group=group)
+        return out
+    h = t.cpu()
+    parts = [torch.empty_like(h) for _ in range(world)]
+    dist.all_gather(parts, h, group=group)
+    return torch.cat(parts).to(t.device)
+
+
 def exchange_lookback(shard, group=None, L: int = 2):
     """Each rank receives the last L bytes of the previous rank's shard (tiny allgather)."""
     import torch
@@ -41,19 +58,16 @@ def exchange_lookback(shard, group=None, L: int = 2):
 
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
-    tail = torch.zeros(16, dtype=torch.uint8, device=shard.device)
-    n = min(L, shard.numel())
+    tail = torch.zeros(17, dtype=torch.uint8, device=shard.device)
+    n = min(L, shard.numel(), 16)
     if n:
-        tail[16 - n:] = shard[shard.numel() - n:]
-    lens = torch.tensor([n], dtype=torch.int64, device=shard.device)
-    tails = [torch.empty_like(tail) for _ in range(world)]
-    allens = [torch.empty_like(lens) for _ in range(world)]
-    dist.all_gather(tails, tail, group=group)
-    dist.all_gather(allens, lens, group=group)
+        tail[16 - n:16] = shard[shard.numel() - n:]
+    tail[16] = n
+    tails = _all_gather_cat(tail, group).view(world, 17)
     if rank == 0:
         return tail[:0]
-    m = int(allens[rank - 1].item())
-    return tails[rank - 1][16 - m:]
+    m = int(tails[rank - 1, 16].item())
+    return tails[rank - 1, 16 - m:16].contiguous()
 
 
 def run_sharded(fsm: FSM, shard, lookback, group=None, scheme="auto", chunk_bytes=4096, spec_k=4,
@@ -74,8 +88,7 @@ def run_sharded(fsm: FSM, shard, lookback, group=None, scheme="auto", chunk_byte
                               lb.data_ptr() if lb is not None else None, lb.numel() if lb is not None else 0,
                               ctypes.byref(o), local.data_ptr(), ce.data_ptr() if ce is not None else None),
            "fsm_shard_map")
-    gathered = torch.empty(world * mb, dtype=torch.uint8, device=shard.device)
-    dist.all_gather_into_tensor(gathered, local, group=group)
+    gathered = _all_gather_cat(local, group)  # the single data-path collective
     r = fsm_result()
     _check(_lib.fsm_shard_finish(fsm.handle, gathered.data_ptr(), world, rank, ctypes.byref(o),
                                  ce.data_ptr() if ce is not None else None, ctypes.byref(r)), "fsm_shard_finish")
