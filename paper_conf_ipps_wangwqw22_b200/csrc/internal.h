@@ -4,6 +4,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <map>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -88,6 +90,7 @@ struct Ctl {
   uint64_t accept_count;
   uint64_t nA, I, nU;    // this round: A-tasks, idle workers, total untried candidates
   uint64_t jacobi_iters;
+  uint64_t ntask[2];     // fast path (SEQ/PM/SRE): per-round task-list length (alternating)
   uint32_t xfin;         // transformed final state (written by the last kernel of a run)
   uint32_t pad1;
 };
@@ -103,6 +106,38 @@ struct RunParams {
   uint32_t qs_cap;
   uint32_t vr_end, vr_oth;
 };
+
+// Host-side launch-config cache: sets the dynamic-smem attribute and queries
+// occupancy once per (kernel, smem, block) instead of on every launch.
+inline cudaError_t kernel_setup(const void* kern, uint32_t smem, int block, int* occ) {
+  struct Entry { uint32_t smem; int block; int occ; };
+  static std::mutex mu;
+  static std::map<const void*, Entry> cache;
+  std::lock_guard<std::mutex> g(mu);
+  auto it = cache.find(kern);
+  if (it != cache.end() && it->second.smem == smem && it->second.block == block) {
+    if (occ) *occ = it->second.occ;
+    return cudaSuccess;
+  }
+  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int o = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, block, smem);
+  if (e != cudaSuccess) return e;
+  cache[kern] = Entry{smem, block, o};
+  if (occ) *occ = o;
+  return cudaSuccess;
+}
+
+inline int device_sms() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  return sms;
+}
 
 // ---- launchers (each returns the cudaError_t of the launch) ------------------
 cudaError_t launch_build_qs2_raw(const uint32_t* d_ttc, uint32_t n, uint32_t C, uint32_t* scratch, uint32_t grid,

@@ -141,12 +141,9 @@ template <int MODE, int NI, int KP>
 cudaError_t launch_t(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st, uint64_t c0) {
   auto kern = k_spec_exec<MODE, NI, KP>;
   const uint32_t smem = smem_bytes_for(img);
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  int dev = 0, sms = 0, occ = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, 256, smem);
+  int occ = 0;
+  const int sms = device_sms();
+  cudaError_t e = kernel_setup((const void*)kern, smem, 256, &occ);
   if (e != cudaSuccess) return e;
   if (occ < 1) return cudaErrorInvalidConfiguration;
   const uint64_t groups = (rp.N - c0 + NI - 1) / NI;
@@ -180,9 +177,7 @@ cudaError_t launch_spec_generic(const DevImage& img, const RunParams& rp, const 
 
 cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st) {
   if (rp.N == 0) return cudaSuccess;
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int sms = device_sms();
   uint64_t done = 0;
   cudaError_t e = spec_path_generic_only() ? cudaErrorNotSupported : launch_spec_tma(img, rp, rs, sms, st, &done);
   if (e != cudaSuccess && e != cudaErrorNotSupported) return e;

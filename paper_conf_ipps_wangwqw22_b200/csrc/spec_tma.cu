@@ -204,7 +204,7 @@ cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunPa
   if (wmax < 8) w = wmax;
   const uint32_t table_off = (tbytes + 1023) & ~1023u;  // stages start 1 KiB-aligned (swizzle span)
   const uint32_t smem = table_off + w * S * kStageBytes + w * S * 8;
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = kernel_setup((const void*)kern, smem, (int)(w * 32), nullptr);
   if (e != cudaSuccess) return e;
   uint64_t grid = std::min<uint64_t>((uint64_t)sms, (ntiles + w - 1) / w);
   if (grid < 1) grid = 1;

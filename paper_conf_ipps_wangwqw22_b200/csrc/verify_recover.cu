@@ -182,11 +182,19 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   const bool helpers = rp.scheme == FSM_SCHEME_RR || rp.scheme == FSM_SCHEME_NF;
   volatile Ctl* vctl = ctl;
 
+  // fast path (SEQ/PM/SRE: no helpers): tasks are exactly the chunks without a
+  // matching record (SRE) or the frontier alone (SEQ/PM), so they are listed in
+  // phase F and executed in E: two grid barriers per round besides V.
+  const bool fast = !helpers;
   for (;;) {
     const uint64_t f = vctl->f;
     const uint32_t tf = vctl->tf;
+    const uint32_t rnd = (uint32_t)vctl->rounds;
     // ---------------- V: verification by chaotic relaxation ----------------
-    if (b == 0 && threadIdx.x == 0) vctl->fmin = N;
+    if (b == 0 && threadIdx.x == 0) {
+      vctl->fmin = N;
+      vctl->ntask[(rnd + 1) & 1] = 0;
+    }
     uint32_t it = 0;
     for (;;) {
       if (b == 0 && threadIdx.x == 0) vctl->changed[(it + 1) % 3] = 0;
@@ -218,6 +226,23 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         checks++;
         matches += fd;
         if (!fd) fm = min(fm, c);
+        if (fast && sre_like) {  // list every chunk without a match (warp-aggregated append)
+          const uint32_t am = __activemask();
+          const uint32_t bal = __ballot_sync(am, !fd);
+          if (bal) {
+            const uint32_t lane = threadIdx.x & 31, leader = __ffs(bal) - 1;
+            unsigned long long base = 0;
+            if (lane == leader)
+              base = atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->ntask[rnd & 1]),
+                               (unsigned long long)__popc(bal));
+            base = __shfl_sync(am, base, leader);
+            if (!fd) {
+              const uint64_t slot = base + __popc(bal & ((1u << lane) - 1));
+              rs.task_chunk[slot] = (uint32_t)c;
+              rs.task_start[slot] = ld_cg(rs.x + c);  // captured before E rewrites x
+            }
+          }
+        }
       }
       fm = block_min(fm, red64);
       checks = block_sum<uint64_t>(checks, red64);
@@ -233,6 +258,45 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     const uint64_t f2 = vctl->fmin;
     if (f2 >= N) break;
     const uint32_t tf2 = ld_cg(rs.x + f2);
+    if (fast) {
+      // ---------------- E (fast): must-do (+ SRE) tasks from the list --------------
+      const uint64_t T = (uint64_t)G * kBS, gt = (uint64_t)b * kBS + threadIdx.x;
+      const uint64_t nt = sre_like ? ld_cg64(&ctl->ntask[rnd & 1]) : 1;
+      uint64_t mustdo = 0, sre = 0, reread = 0;
+      for (uint64_t s = gt; s < nt; s += T) {
+        const uint32_t c = sre_like ? __ldcg(rs.task_chunk + s) : (uint32_t)f2;
+        const uint32_t st = sre_like ? __ldcg(rs.task_start + s) : tf2;
+        uint32_t e, cnt;
+        task_walk<MODE>(img, smem, rp, rs, c, st, &e, &cnt);
+        reread += min((uint64_t)rp.B, rp.len - (uint64_t)c * rp.B);
+        const uint32_t ne = ld_cg(rs.n_end + c);
+        const uint64_t o = (uint64_t)(ne % rp.vr_end) * rs.cap + c;
+        st_cg(rs.start + o, st);
+        st_cg(rs.end + o, e);
+        st_cg(rs.cnt + o, cnt);
+        st_cg(rs.n_end + c, ne + 1);
+        st_cg(rs.x + c + 1, e);
+        st_cg(rs.cur_end + c, e);
+        if (c == f2) mustdo++; else sre++;
+      }
+      mustdo = block_sum<uint64_t>(mustdo, red64);
+      sre = block_sum<uint64_t>(sre, red64);
+      reread = block_sum<uint64_t>(reread, red64);
+      if (threadIdx.x == 0) {
+        if (mustdo) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_mustdo), (unsigned long long)mustdo);
+        if (sre) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_sre), (unsigned long long)sre);
+        if (reread) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->reread_bytes), (unsigned long long)reread);
+        if (mustdo + sre)
+          atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->active_sum), (unsigned long long)(mustdo + sre));
+        if (b == 0) {
+          vctl->rounds = vctl->rounds + 1;
+          vctl->f = f2;
+          vctl->tf = tf2;
+        }
+      }
+      grid.sync();
+      continue;
+    }
     // ---------------- T: per-block counts of A-tasks and untried candidates -----
     {
       uint64_t cA = 0, cU = 0;
@@ -436,10 +500,8 @@ cudaError_t launch_m(const DevImage& img, const RunParams& rp, const RecStore& r
                      uint32_t* chunk_ends, cudaStream_t st, int sms) {
   auto kern = k_verify_recover<MODE>;
   const uint32_t smem = smem_bytes_for(img);
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
   int occ = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kBS, smem);
+  cudaError_t e = kernel_setup((const void*)kern, smem, kBS, &occ);
   if (e != cudaSuccess) return e;
   if (occ < 1) return cudaErrorInvalidConfiguration;
   uint64_t grid = (uint64_t)sms * occ;

@@ -132,19 +132,29 @@ __device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) { return __ldcg(p);
 __device__ __forceinline__ void st_cg(uint32_t* p, uint32_t v) { __stcg(p, v); }
 
 // Look x up in VR_c (END slots then OTH slots).  Returns true on a match.
+// Slot 0 and the ring counts are loaded together (one L2 round trip for the
+// common single-record chunk), the rest of the rings only if needed.
 __device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, uint32_t vr_oth, uint64_t c,
                                           uint32_t x, uint32_t* end, uint32_t* cnt) {
-  uint32_t ne = min(ld_cg(rs.n_end + c), vr_end);
-  for (uint32_t s = 0; s < ne; s++) {
+  const uint32_t ne_raw = ld_cg(rs.n_end + c), no_raw = ld_cg(rs.n_oth + c);
+  const uint32_t s0 = ld_cg(rs.start + c), e0 = ld_cg(rs.end + c);
+  const uint32_t c0 = cnt ? ld_cg(rs.cnt + c) : 0u;
+  if (ne_raw >= 1 && s0 == x) {
+    *end = e0;
+    if (cnt) *cnt = c0;
+    return true;
+  }
+  const uint32_t ne = min(ne_raw, vr_end);
+  for (uint32_t s = 1; s < ne; s++) {
     if (ld_cg(rs.start + s * rs.cap + c) == x) {
       *end = ld_cg(rs.end + s * rs.cap + c);
       if (cnt) *cnt = ld_cg(rs.cnt + s * rs.cap + c);
       return true;
     }
   }
-  uint32_t no = min(ld_cg(rs.n_oth + c), vr_oth);
+  const uint32_t no = min(no_raw, vr_oth);
   for (uint32_t s = 0; s < no; s++) {
-    uint64_t o = (uint64_t)(kVrMax + s) * rs.cap + c;
+    const uint64_t o = (uint64_t)(kVrMax + s) * rs.cap + c;
     if (ld_cg(rs.start + o) == x) {
       *end = ld_cg(rs.end + o);
       if (cnt) *cnt = ld_cg(rs.cnt + o);
