@@ -116,6 +116,17 @@ uint64_t fsm_num_chunks(uint64_t len, uint32_t chunk_bytes);
 int fsm_run(fsm_t fsm, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
             uint32_t* d_chunk_ends, fsm_result* out);
 
+/* Asynchronous fsm_run: enqueues the whole run (kernels + the small result
+ * readback into pinned memory) on opts->stream and returns a ticket at once;
+ * fsm_wait(ticket) blocks until that run is done and fills *out.  Up to 32
+ * runs may be in flight per handle (they execute in stream order and reuse
+ * the handle's scratch one after another).  d_input/d_chunk_ends must stay
+ * valid until the run completes.  With FSM_SCHEME_AUTO the first call may
+ * synchronously profile the input (selector). */
+int fsm_run_async(fsm_t fsm, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
+                  uint32_t* d_chunk_ends, uint64_t* ticket);
+int fsm_wait(fsm_t fsm, uint64_t ticket, fsm_result* out);
+
 /* Same as fsm_run with HOST buffers: copies h_input to the device (pinned
  * memory recommended), runs, and copies chunk ends back to h_chunk_ends
  * (nullable).  Used for end-to-end timing. */

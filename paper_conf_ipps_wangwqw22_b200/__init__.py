@@ -59,6 +59,8 @@ _lib.fsm_num_chunks.argtypes = [U64, U32]
 _lib.fsm_num_chunks.restype = U64
 _lib.fsm_run.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
 _lib.fsm_run_host.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
+_lib.fsm_run_async.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(U64)]
+_lib.fsm_wait.argtypes = [P, U64, ctypes.POINTER(fsm_result)]
 _lib.fsm_select_scheme.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), ctypes.POINTER(ctypes.c_int),
                                    ctypes.POINTER(fsm_features)]
 _lib.fsm_map_bytes.argtypes = [P]
@@ -172,6 +174,20 @@ class FSM:
         _check(_lib.fsm_run(self._h, x.data_ptr() if x.numel() else None, x.numel(), ctypes.byref(o),
                             ce.data_ptr() if ce is not None else None, ctypes.byref(r)), "fsm_run")
         return Result.from_c(r, ce[:n] if ce is not None else None)
+
+    def run_async(self, x, scheme="auto", chunk_bytes=4096, chunk_ends=None, spec_k=4, stream=None) -> int:
+        """fsm_run_async: enqueue a run (stream-ordered) and return a ticket for wait()."""
+        o = _run_opts(scheme, chunk_bytes, spec_k, stream=stream)
+        t = U64(0)
+        _check(_lib.fsm_run_async(self._h, x.data_ptr() if x.numel() else None, x.numel(), ctypes.byref(o),
+                                  chunk_ends.data_ptr() if chunk_ends is not None else None, ctypes.byref(t)),
+               "fsm_run_async")
+        return t.value
+
+    def wait(self, ticket: int) -> Result:
+        r = fsm_result()
+        _check(_lib.fsm_wait(self._h, ticket, ctypes.byref(r)), "fsm_wait")
+        return Result.from_c(r)
 
     def run_host(self, data: np.ndarray, scheme="auto", chunk_bytes=4096, chunk_ends=True, stream=None,
                  **kw) -> Result:

@@ -131,9 +131,11 @@ int ensure_records(fsm_t f, uint64_t N) {
 
 int ensure_ctl(fsm_t f) {
   if (!f->d_ctl) CUDA_TRY(cudaMalloc(&f->d_ctl, sizeof(Ctl)));
-  if (!f->h_ctl) CUDA_TRY(cudaMallocHost(&f->h_ctl, sizeof(Ctl)));
-  for (auto& e : f->ev)
-    if (!e) CUDA_TRY(cudaEventCreate(&e));
+  if (!f->h_ctl) {
+    CUDA_TRY(cudaMallocHost(&f->h_ctl, sizeof(Ctl) * fsm_s::kRing));
+    for (auto& slot : f->ev)
+      for (auto& e : slot) CUDA_TRY(cudaEventCreate(&e));
+  }
   const size_t need = 2 * 4096 + 64;
   if (f->block_tmp_elems < need) {
     if (f->d_block_tmp) cudaFree(f->d_block_tmp);
@@ -155,20 +157,21 @@ void fill_result_stats(fsm_result* out, const Ctl& h) {
   out->avg_active_workers = h.rounds ? (double)h.active_sum / (double)h.rounds : 0.0;
 }
 
-// Core device run over d_in[0..len) from transformed start q0t.  On success
-// leaves x[] (speculative/record path) in the handle for callers that need it.
-int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_scheme scheme, uint32_t q0t,
-             uint32_t* d_chunk_ends, fsm_result* out, uint32_t* final_tid) {
+// Enqueue one device run over d_in[0..len) from transformed start q0t on
+// o.st; returns a ticket.  Everything (init, kernels, readback) is stream
+// ordered, so runs on one handle may be queued back to back.
+int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_scheme scheme, uint32_t q0t,
+                uint32_t* d_chunk_ends, uint64_t* ticket) {
   const uint64_t N = (len + o.B - 1) / o.B;
-  std::memset(out, 0, sizeof(*out));
-  out->nchunks = N;
-  out->scheme_used = scheme;
-  if (N == 0) {
-    *final_tid = q0t;
-    return FSM_OK;
-  }
   int rc = ensure_ctl(f);
   if (rc) return rc;
+  const uint64_t seq = f->next_seq++;
+  const uint32_t slot = (uint32_t)(seq % fsm_s::kRing);
+  auto& pd = f->pend[slot];
+  if (pd.active) CUDA_TRY(cudaEventSynchronize(f->ev[slot][3]));  // ring wrapped: slot's readback must be done
+  pd = fsm_s::Pending{seq, N, scheme, q0t, true};
+  *ticket = seq;
+  if (N == 0) return FSM_OK;
   RunParams rp{};
   rp.in = d_in;
   rp.q0t = q0t;
@@ -180,34 +183,39 @@ int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_sche
   rp.qs_cap = o.qs_cap;
   rp.vr_end = o.vr_end;
   rp.vr_oth = o.vr_oth;
-  cudaEvent_t* ev = f->ev;
-  Ctl& h = *f->h_ctl;
+  cudaEvent_t* ev = f->ev[slot];
+  Ctl& h = f->h_ctl[slot];
+  std::memset(&h, 0, sizeof(Ctl));
+  h.f = 0;
+  h.tf = q0t;
+  h.fmin = N;
   if (scheme == FSM_SCHEME_ENUM) {
-    if (f->n + 1 > kEnumMax) return fail(FSM_EUNSUPPORTED, "ENUM needs nstates + 1 <= 32");
+    if (f->n + 1 > kEnumMax) {
+      pd.active = false;
+      return fail(FSM_EUNSUPPORTED, "ENUM needs nstates + 1 <= 32");
+    }
     // sub-chunk size E | B: small enough for parallelism, bounded scratch
     uint32_t E = o.B;
     while (E % 32 == 0 && E > 256 && (len + E / 2 - 1) / (E / 2) <= (1ull << 22)) E /= 2;
     const uint64_t nsub = (len + E - 1) / E;
     const uint64_t need = enum_scratch_bytes(nsub);
     if (f->enum_bytes < need) {
+      CUDA_TRY(cudaStreamSynchronize(o.st));  // earlier queued runs may still use the old scratch
       if (f->enum_base) cudaFree(f->enum_base);
       f->enum_base = nullptr;
       f->enum_bytes = 0;
       CUDA_TRY(cudaMalloc(&f->enum_base, need));
       f->enum_bytes = need;
     }
-    CUDA_TRY(cudaMemsetAsync(f->d_ctl, 0, sizeof(Ctl), o.st));
+    CUDA_TRY(cudaMemcpyAsync(f->d_ctl, &h, sizeof(Ctl), cudaMemcpyHostToDevice, o.st));
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
     CUDA_TRY(launch_enum_full(f->img, rp, E, f->enum_base, d_chunk_ends, f->d_ctl, &f->d_ctl->xfin, o.st,
                               f->sm_count));
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   } else {
+    if (f->rs_cap < N) CUDA_TRY(cudaStreamSynchronize(o.st));  // growing the store: drain queued runs
     if ((rc = ensure_records(f, N))) return rc;
-    std::memset(&h, 0, sizeof(Ctl));
-    h.f = 0;
-    h.tf = q0t;
-    h.fmin = N;
     CUDA_TRY(cudaMemcpyAsync(f->d_ctl, &h, sizeof(Ctl), cudaMemcpyHostToDevice, o.st));
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
     CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
@@ -216,16 +224,42 @@ int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_sche
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   }
   CUDA_TRY(cudaMemcpyAsync(&h, f->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, o.st));
-  CUDA_TRY(cudaStreamSynchronize(o.st));
+  CUDA_TRY(cudaEventRecord(ev[3], o.st));
+  return FSM_OK;
+}
+
+// Wait for a ticket and fill the result (transformed final state in *final_tid).
+int run_collect(fsm_t f, uint64_t ticket, fsm_result* out, uint32_t* final_tid) {
+  const uint32_t slot = (uint32_t)(ticket % fsm_s::kRing);
+  auto& pd = f->pend[slot];
+  if (!pd.active || pd.seq != ticket) return fail(FSM_EINVAL, "unknown or already collected ticket");
+  std::memset(out, 0, sizeof(*out));
+  out->nchunks = pd.N;
+  out->scheme_used = pd.scheme;
+  pd.active = false;
+  if (pd.N == 0) {
+    *final_tid = pd.q0t;
+    return FSM_OK;
+  }
+  CUDA_TRY(cudaEventSynchronize(f->ev[slot][3]));
+  const Ctl& h = f->h_ctl[slot];
   float t1 = 0, t2 = 0;
-  cudaEventElapsedTime(&t1, ev[0], ev[1]);
-  cudaEventElapsedTime(&t2, ev[1], ev[2]);
+  cudaEventElapsedTime(&t1, f->ev[slot][0], f->ev[slot][1]);
+  cudaEventElapsedTime(&t2, f->ev[slot][1], f->ev[slot][2]);
   fill_result_stats(out, h);
   out->accept_count = h.accept_count;
   out->ms_spec = t1;
   out->ms_verify = t2;
   *final_tid = h.xfin;
   return FSM_OK;
+}
+
+int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_scheme scheme, uint32_t q0t,
+             uint32_t* d_chunk_ends, fsm_result* out, uint32_t* final_tid) {
+  uint64_t t = 0;
+  int rc = run_enqueue(f, d_in, len, o, scheme, q0t, d_chunk_ends, &t);
+  if (rc) return rc;
+  return run_collect(f, t, out, final_tid);
 }
 
 fsm_scheme tree_select(const fsm_features& ft, uint32_t n) {
@@ -443,8 +477,9 @@ void fsm_free(fsm_t f) {
   if (f->rs_base) cudaFree(f->rs_base);
   if (f->d_ctl) cudaFree(f->d_ctl);
   if (f->h_ctl) cudaFreeHost(f->h_ctl);
-  for (auto& e : f->ev)
-    if (e) cudaEventDestroy(e);
+  for (auto& slot : f->ev)
+    for (auto& e : slot)
+      if (e) cudaEventDestroy(e);
   if (f->d_block_tmp) cudaFree(f->d_block_tmp);
   if (f->enum_base) cudaFree(f->enum_base);
   if (f->feat_base) cudaFree(f->feat_base);
@@ -478,6 +513,41 @@ int fsm_run(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* o
   fsm_result r;
   uint32_t fin = 0;
   rc = run_core(f, d_input, len, o, scheme, f->img.q0t, d_chunk_ends, &r, &fin);
+  if (rc) return rc;
+  if (fin == f->n) return fail(FSM_ESYMBOL, "input symbol >= nsyms");
+  r.final_state = f->inv[fin];
+  r.accept = f->accept[r.final_state];
+  *out = r;
+  return FSM_OK;
+}
+
+int fsm_run_async(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts, uint32_t* d_chunk_ends,
+                  uint64_t* ticket) {
+  if (!f || !ticket) return fail(FSM_EINVAL, "NULL handle/ticket");
+  if (!d_input && len > 0) return fail(FSM_EINVAL, "NULL input");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  fsm_scheme scheme = o.scheme;
+  if (scheme == FSM_SCHEME_AUTO) {
+    if (!f->auto_selected) {
+      fsm_run_opts so{};
+      if (opts) so = *opts;
+      so.scheme = FSM_SCHEME_SRE;
+      fsm_scheme pick;
+      if ((rc = fsm_select_scheme(f, d_input, std::min<uint64_t>(len, 1ull << 20), &so, &pick, nullptr))) return rc;
+    }
+    scheme = f->auto_scheme;
+    if (scheme == FSM_SCHEME_ENUM && f->n + 1 > kEnumMax) scheme = FSM_SCHEME_SRE;
+  }
+  return run_enqueue(f, d_input, len, o, scheme, f->img.q0t, d_chunk_ends, ticket);
+}
+
+int fsm_wait(fsm_t f, uint64_t ticket, fsm_result* out) {
+  if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
+  fsm_result r;
+  uint32_t fin = 0;
+  int rc = run_collect(f, ticket, &r, &fin);
   if (rc) return rc;
   if (fin == f->n) return fail(FSM_ESYMBOL, "input symbol >= nsyms");
   r.final_state = f->inv[fin];

@@ -201,8 +201,17 @@ struct fsm_s {
   uint32_t rs_slots_alloc = 0;
   void* rs_base = nullptr;
   gspec::Ctl* d_ctl = nullptr;
-  gspec::Ctl* h_ctl = nullptr;       // pinned host mirror (init + readback, async)
-  cudaEvent_t ev[3] = {nullptr, nullptr, nullptr};
+  // in-flight runs: pinned Ctl mirrors (init + readback) and events per ring slot
+  static constexpr uint32_t kRing = 32;
+  gspec::Ctl* h_ctl = nullptr;        // pinned [kRing]
+  cudaEvent_t ev[kRing][4] = {};      // start, after spec, after verify, after readback
+  struct Pending {
+    uint64_t seq = 0, N = 0;
+    fsm_scheme scheme = FSM_SCHEME_SRE;
+    uint32_t q0t = 0;
+    bool active = false;
+  } pend[kRing];
+  uint64_t next_seq = 1;
   uint64_t* d_block_tmp = nullptr;
   size_t block_tmp_elems = 0;
   void* enum_base = nullptr;

@@ -45,11 +45,20 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   }
 }
 
-__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int32_t x, int32_t y) {
+// The input is streamed exactly once: load it with an L2 evict-first policy so
+// it does not push the cold rows of a large transition table out of L2.
+__device__ __forceinline__ uint64_t evict_first_policy() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int32_t x, int32_t y,
+                                            uint64_t policy) {
   asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
-          smem_u32(dst)),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%2, %3}], [%4], %5;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar)), "l"(policy)
       : "memory");
 }
 
@@ -80,12 +89,13 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   uint8_t* wst = stages + (size_t)warp * S * kStageBytes;
   uint64_t* wbar = bars + warp * S;
 
+  const uint64_t pol = evict_first_policy();
   auto issue = [&](uint64_t it) {
     const uint64_t t = gw + (it / segs) * tw;
     const uint32_t sg = (uint32_t)(it % segs);
     const int s = (int)(it % S);
     mbar_expect_tx(wbar + s, kStageBytes);
-    tma_load_2d(wst + (size_t)s * kStageBytes, &tmap, wbar + s, (int32_t)(sg * kRowBytes), (int32_t)(t * 32));
+    tma_load_2d(wst + (size_t)s * kStageBytes, &tmap, wbar + s, (int32_t)(sg * kRowBytes), (int32_t)(t * 32), pol);
   };
   if (lane == 0)
     for (uint64_t it = 0; it < items && it < (uint64_t)S; it++) issue(it);

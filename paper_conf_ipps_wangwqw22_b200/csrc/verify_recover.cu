@@ -96,6 +96,50 @@ __device__ __forceinline__ uint64_t block_min(uint64_t v, uint64_t* red) {
   return s;
 }
 
+// Hierarchical result store, level 2 (Fig. 5 (2)): each CTA keeps the
+// ring counts and the first two VR^end records of the chunks it owns in shared
+// memory, refreshed from the global store (level 3) at every round start —
+// records produced by other CTAs' threads in phase E reach the owner through
+// that refresh.  Verification iterations then read shared memory; only
+// chunks with more records fall through to L2.
+struct VrCache {
+  uint8_t* ne;
+  uint8_t* no;
+  uint32_t *s0, *e0, *s1, *e1;
+};
+
+__device__ __forceinline__ VrCache vr_cache_at(uint8_t* base, uint32_t cap) {
+  VrCache v;
+  v.ne = base;
+  v.no = base + cap;
+  uint32_t* u = reinterpret_cast<uint32_t*>(base + ((2 * cap + 15) & ~15u));
+  v.s0 = u;
+  v.e0 = u + cap;
+  v.s1 = u + 2 * cap;
+  v.e1 = u + 3 * cap;
+  return v;
+}
+
+__host__ __device__ inline uint32_t vr_cache_bytes(uint32_t cap) { return ((2 * cap + 15) & ~15u) + 16 * cap; }
+
+__device__ __forceinline__ bool vr_lookup_cached(const VrCache& v, uint32_t i, const RecStore& rs, uint32_t vr_end,
+                                                 uint32_t vr_oth, uint64_t c, uint32_t x, uint32_t* end) {
+  const uint32_t ne = v.ne[i];
+  if (ne >= 1 && v.s0[i] == x) { *end = v.e0[i]; return true; }
+  if (ne >= 2 && vr_end >= 2 && v.s1[i] == x) { *end = v.e1[i]; return true; }
+  if (ne > 2 || v.no[i]) {  // rare: more records in the global rings
+    const uint32_t ne_all = min(ld_cg(rs.n_end + c), vr_end);
+    for (uint32_t sl = 2; sl < ne_all; sl++)
+      if (ld_cg(rs.start + sl * rs.cap + c) == x) { *end = ld_cg(rs.end + sl * rs.cap + c); return true; }
+    const uint32_t no = min(ld_cg(rs.n_oth + c), vr_oth);
+    for (uint32_t sl = 0; sl < no; sl++) {
+      const uint64_t o = (uint64_t)(kVrMax + sl) * rs.cap + c;
+      if (ld_cg(rs.start + o) == x) { *end = ld_cg(rs.end + o); return true; }
+    }
+  }
+  return false;
+}
+
 // Untried QS candidates of chunk c (Alg. 4 L24, Alg. 5 L30-32): QS_c entries
 // past the cursor that are neither in dom VR_c nor this round's task start.
 __device__ uint32_t untried(const DevImage& img, const RunParams& rp, const RecStore& rs, uint64_t c,
@@ -165,7 +209,7 @@ __device__ void task_walk(const DevImage& img, const uint8_t* smem, const RunPar
 
 template <int MODE>
 __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
-                                                        uint64_t* btmp, uint32_t* chunk_ends) {
+                                                        uint64_t* btmp, uint32_t* chunk_ends, uint32_t cache_cap) {
   cg::grid_group grid = cg::this_grid();
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ uint32_t ws[3][kBS / 32];
@@ -186,10 +230,24 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   // matching record (SRE) or the frontier alone (SEQ/PM), so they are listed in
   // phase F and executed in E: two grid barriers per round besides V.
   const bool fast = !helpers;
+  const bool cached = cache_cap != 0 && hi - lo <= cache_cap;
+  const VrCache vc = vr_cache_at(smem + ((smem_bytes_for(img) + 15) & ~15u), cache_cap);
   for (;;) {
     const uint64_t f = vctl->f;
     const uint32_t tf = vctl->tf;
     const uint32_t rnd = (uint32_t)vctl->rounds;
+    if (cached) {  // refresh level 2 from level 3 for the owned chunks
+      for (uint64_t c = max(lo, f) + threadIdx.x; c < hi; c += kBS) {
+        const uint32_t i = (uint32_t)(c - lo);
+        vc.ne[i] = (uint8_t)min(ld_cg(rs.n_end + c), 255u);
+        vc.no[i] = (uint8_t)min(ld_cg(rs.n_oth + c), 255u);
+        vc.s0[i] = ld_cg(rs.start + c);
+        vc.e0[i] = ld_cg(rs.end + c);
+        vc.s1[i] = ld_cg(rs.start + rs.cap + c);
+        vc.e1[i] = ld_cg(rs.end + rs.cap + c);
+      }
+      __syncthreads();
+    }
     // ---------------- V: verification by chaotic relaxation ----------------
     if (b == 0 && threadIdx.x == 0) {
       vctl->fmin = N;
@@ -202,7 +260,8 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       for (uint64_t c = max(lo, f) + threadIdx.x; c < hi; c += kBS) {
         const uint32_t xin = (c == f) ? tf : ld_cg(rs.x + c);
         uint32_t e;
-        const bool hit = vr_lookup(rs, rp.vr_end, rp.vr_oth, c, xin, &e, nullptr);
+        const bool hit = cached ? vr_lookup_cached(vc, (uint32_t)(c - lo), rs, rp.vr_end, rp.vr_oth, c, xin, &e)
+                                : vr_lookup(rs, rp.vr_end, rp.vr_oth, c, xin, &e, nullptr);
         rs.found[c] = hit;
         if (!hit) e = ld_cg(rs.cur_end + c);  // F_c default: the chunk's end as of the round start
         if (ld_cg(rs.x + c + 1) != e) {
@@ -499,18 +558,28 @@ template <int MODE>
 cudaError_t launch_m(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t* btmp,
                      uint32_t* chunk_ends, cudaStream_t st, int sms) {
   auto kern = k_verify_recover<MODE>;
-  const uint32_t smem = smem_bytes_for(img);
+  const uint32_t tsmem = (smem_bytes_for(img) + 15) & ~15u;
   int occ = 0;
-  cudaError_t e = kernel_setup((const void*)kern, smem, kBS, &occ);
+  cudaError_t e = kernel_setup((const void*)kern, tsmem, kBS, &occ);
   if (e != cudaSuccess) return e;
   if (occ < 1) return cudaErrorInvalidConfiguration;
   uint64_t grid = (uint64_t)sms * occ;
   const uint64_t want = (rp.N + kBS - 1) / kBS;
   if (want < grid) grid = want < 1 ? 1 : want;
+  // level-2 cache for the owned chunk range, if it fits without lowering occupancy
+  uint32_t cap = (uint32_t)((rp.N + grid - 1) / grid);
+  uint32_t smem = tsmem + vr_cache_bytes(cap);
+  int occ2 = 0;
+  if (cap > 16384 || kernel_setup((const void*)kern, smem, kBS, &occ2) != cudaSuccess ||
+      (uint64_t)sms * occ2 < grid) {
+    cap = 0;
+    smem = tsmem;
+    if ((e = kernel_setup((const void*)kern, smem, kBS, &occ)) != cudaSuccess) return e;
+  }
   DevImage a0 = img;
   RunParams a1 = rp;
   RecStore a2 = rs;
-  void* args[] = {&a0, &a1, &a2, &ctl, &btmp, &chunk_ends};
+  void* args[] = {&a0, &a1, &a2, &ctl, &btmp, &chunk_ends, &cap};
   return cudaLaunchCooperativeKernel((const void*)kern, dim3((unsigned)grid), dim3(kBS), args, smem, st);
 }
 

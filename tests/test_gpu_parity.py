@@ -227,3 +227,24 @@ def test_full_size_bench_config(gs, name, length):
     fsm = _fsm(gs, w)
     res = fsm.run(x, scheme="auto")
     check_equal(res, ref, 4096, w.nstates)
+
+
+def test_async_queue(gs):
+    """fsm_run_async/fsm_wait: runs queued back to back (different inputs and
+    schemes on one handle) each return exactly the sequential result."""
+    runs = []
+    fsm = None
+    for seed in range(6):
+        w, data = _wl("c2", (1 << 20) + seed * 4111, 100 + seed)
+        fsm = fsm or gs.FSM.load(w.table, w.start, w.accept)
+        x = torch.from_numpy(data).cuda()
+        ce = torch.empty(gs.fsm_num_chunks(len(data)), dtype=torch.int32, device="cuda")
+        scheme = ("sre", "pm", "seq", "rr", "nf", "sre")[seed]
+        runs.append((fsm.run_async(x, scheme=scheme, chunk_ends=ce), x, ce, data, w))
+    for t, x, ce, data, w in reversed(runs):
+        r = fsm.wait(t)
+        ref = oracle.run(w.table, w.start, w.accept, data, 4096)
+        assert r.final_state == ref["final"] and r.accept_count == ref["count"]
+        assert (ce.cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
+    with pytest.raises(gs.GSpecError):
+        fsm.wait(runs[0][0])  # already collected
