@@ -92,6 +92,16 @@ class ClockSampler:
                 "samples": len(self.samples)}
 
 
+def _max_over_ranks(dist, v: float) -> float:
+    """MAX over ranks (device timings are taken per rank, the job is as slow as the slowest)."""
+    import torch
+
+    on_gpu = dist.get_backend() == "nccl"
+    t = torch.tensor([v], dtype=torch.float64, device="cuda" if on_gpu else "cpu")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
 def cpu_baseline(w, budget_s=12.0):
     """The oracle (plain sequential C, oracle/) on host cores, bounded sample."""
     import numpy as np
@@ -172,12 +182,18 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
+    # one process per GPU; GSPEC_DIST_BACKEND=gloo lets several ranks share one GPU (tests only)
+    backend = os.environ.get("GSPEC_DIST_BACKEND", "nccl")
+    dev = local % max(1, torch.cuda.device_count()) if backend != "nccl" else local
+    torch.cuda.set_device(dev)
     dist = None
     if world > 1:
         import torch.distributed as dist
 
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group(backend)
     w = gen.workload(args.config)
     length = w.length
     B = args.chunk_bytes
@@ -222,7 +238,7 @@ def main():
         dist.barrier()
     torch.cuda.synchronize()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
+    with ClockSampler(dev) as clk:
         ev0.record(stream)
         for _ in range(args.steps):
             r_ = step()
@@ -240,28 +256,45 @@ def main():
         dist.barrier()
     ms = ev0.elapsed_time(ev1) / args.steps
     if dist:
-        t = torch.tensor([ms], device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms = _max_over_ranks(dist, ms)
     total_bytes = length * world
     value = total_bytes / (ms * 1e-3) / 1e9
 
     # end-to-end: host (pinned) bytes through the public API, H2D + D2H inside the timed region
     e2e = None
-    if args.e2e_steps > 0 and world == 1:
+    if args.e2e_steps > 0:
         h = torch.empty(length, dtype=torch.uint8, pin_memory=True)
-        h.copy_(x.cpu() if length <= (1 << 31) else x.cpu())
+        h.copy_(x)
         hn = h.numpy()
-        fsm.run_host(hn, scheme=scheme, chunk_bytes=B)
+        nch = gs.fsm_num_chunks(length, B)
+        if world == 1:
+            def e2e_step():
+                return fsm.run_host(hn, scheme=scheme, chunk_bytes=B)
+        else:
+            xd = torch.empty_like(x)
+            ce_h = torch.empty(nch, dtype=torch.int32, pin_memory=True)
+
+            def e2e_step():
+                xd.copy_(h, non_blocking=True)                     # H2D of this rank's shard
+                r = run_sharded(fsm, xd, lb, scheme=scheme, chunk_bytes=B)
+                ce_h.copy_(r.chunk_ends, non_blocking=True)       # D2H of the results
+                torch.cuda.current_stream().synchronize()
+                return r
+        e2e_step()
+        if dist:
+            dist.barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         for _ in range(args.e2e_steps):
-            r2 = fsm.run_host(hn, scheme=scheme, chunk_bytes=B)
+            r2 = e2e_step()
         torch.cuda.synchronize()
-        e2e_s = (time.perf_counter() - t0) / args.e2e_steps
+        e2e_s = time.perf_counter() - t0
+        if dist:
+            e2e_s = _max_over_ranks(dist, e2e_s)
+        e2e_s /= args.e2e_steps
         assert r2.final_state == res.final_state and r2.accept_count == res.accept_count
         e2e = {"value": round(total_bytes / e2e_s / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": length,
-               "d2h_bytes_per_step": int(gs.fsm_num_chunks(length, B) * 4 + 64), "ms_per_step": round(e2e_s * 1e3, 3)}
+               "d2h_bytes_per_step": int(nch * 4 + 64), "ms_per_step": round(e2e_s * 1e3, 3)}
 
     if not spec_ms:
         spec_ms = [r.stats["ms_spec"] for r in kr]

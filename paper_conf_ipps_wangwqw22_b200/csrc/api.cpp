@@ -111,6 +111,7 @@ int ensure_records(fsm_t f, uint64_t N) {
     r.task_chunk = (uint32_t*)take(4 * (cap + 8));
     r.task_start = (uint32_t*)take(4 * (cap + 8));
     r.task_j = (uint32_t*)take(4 * (cap + 8));
+    r.tstart = (uint32_t*)take(4 * (cap + 8));
     r.next_qs = take(cap);
     r.found = take(cap);
     r.ulen = take(cap);
@@ -218,9 +219,24 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     if ((rc = ensure_records(f, N))) return rc;
     CUDA_TRY(cudaMemcpyAsync(f->d_ctl, &h, sizeof(Ctl), cudaMemcpyHostToDevice, o.st));
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
+    // dense recovery rounds go to the TMA task kernel (SRE on low-accuracy DFAs); this
+    // needs a host check per verify launch, so it is off when the profile says the
+    // speculation is accurate (no dense rounds expected)
+    rp.dense = (scheme == FSM_SCHEME_SRE && len / o.B > 0 && o.B % 64 == 0 &&
+                (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0 && f->acc1_hint < 0.5) ? 1u : 0u;
     CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
-    CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
+    for (;;) {
+      CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
+      if (!rp.dense) break;
+      uint32_t pend = 0;
+      uint64_t fm = 0;
+      CUDA_TRY(cudaMemcpyAsync(&pend, &f->d_ctl->dense_pending, 4, cudaMemcpyDeviceToHost, o.st));
+      CUDA_TRY(cudaMemcpyAsync(&fm, &f->d_ctl->fmin, 8, cudaMemcpyDeviceToHost, o.st));
+      CUDA_TRY(cudaStreamSynchronize(o.st));
+      if (!pend) break;
+      CUDA_TRY(launch_task_dense(f->img, rp, f->rs, f->d_ctl, fm, f->sm_count, o.st));
+    }
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   }
   CUDA_TRY(cudaMemcpyAsync(&h, f->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, o.st));
@@ -430,6 +446,7 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
     if (H > nt) H = nt;
     img.H = (uint32_t)H;
     img.smem_table_bytes = (uint32_t)(((H * C * esz) + 15) & ~15ull);
+    if (mode == MODE_U16 && H == nt) img.mode = MODE_U16H;  // every row hot: no hot test
     if (mode == MODE_U16) {
       std::vector<uint16_t> T16((uint64_t)nt * C);
       for (uint64_t i = 0; i < T16.size(); i++) T16[i] = (uint16_t)tid2code[ttc[i]];
@@ -637,6 +654,7 @@ int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_
     if (len >= 10) ft.uniq10 = (double)h[20] / 64.0;
   }
   const fsm_scheme pick = tree_select(ft, f->n);
+  if (N > 1) f->acc1_hint = ft.acc1;
   f->auto_scheme = pick;
   f->auto_selected = true;
   *outp = pick;
@@ -650,7 +668,7 @@ int fsm_get_transform(fsm_t f, uint32_t* perm, uint32_t* inv, uint64_t* freq, ui
   if (perm) std::copy(f->perm.begin(), f->perm.end(), perm);
   if (inv) std::copy(f->inv.begin(), f->inv.end(), inv);
   if (freq) std::copy(f->freq.begin(), f->freq.end(), freq);
-  if (mode) *mode = f->img.mode;
+  if (mode) *mode = f->img.mode == MODE_U16H ? (uint32_t)MODE_U16 : f->img.mode;
   if (hot_rows) *hot_rows = f->img.H;
   if (nclasses) *nclasses = f->img.C;
   return FSM_OK;

@@ -206,6 +206,7 @@ cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t 
   switch (img.mode) {
     case MODE_U8: e = walk_m<MODE_U8>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
     case MODE_U16: e = walk_m<MODE_U16>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
+    case MODE_U16H: e = walk_m<MODE_U16H>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
     default: e = walk_m<MODE_U32>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
   }
   if (e != cudaSuccess) return e;

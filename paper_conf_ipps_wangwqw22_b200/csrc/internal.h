@@ -18,6 +18,7 @@ enum Mode : uint32_t {
   MODE_U8 = 1,   // raw-byte table, u8 codes, accept in bit 7, whole table in smem
   MODE_U16 = 2,  // classed table, u16 codes = tid | acc<<15, hot rows (tid < H) in smem
   MODE_U32 = 3,  // classed table, u32 codes = tid | acc<<31, hot rows in smem
+  MODE_U16H = 4, // MODE_U16 with every row in smem: no hot test on the lookup path
 };
 
 constexpr uint32_t kQsMax = 16;     // QS cap ("top 16 states")
@@ -73,6 +74,7 @@ struct RecStore {
   uint32_t* task_chunk;  // [cap+1] task slot -> chunk (0xFFFFFFFF = none)
   uint32_t* task_start;  // [cap+1]
   uint32_t* task_j;      // [cap+1] helper index within its chunk
+  uint32_t* tstart;      // [cap] dense rounds: task start of chunk c, 0xFFFFFFFF = no task
 };
 
 // Device control block of the verify/recover kernel.
@@ -91,6 +93,8 @@ struct Ctl {
   uint64_t nA, I, nU;    // this round: A-tasks, idle workers, total untried candidates
   uint64_t jacobi_iters;
   uint64_t ntask[2];     // fast path (SEQ/PM/SRE): per-round task-list length (alternating)
+  uint32_t dense_pending;  // verify exited: a dense task round (frontier fmin) must run first
+  uint32_t pad2;
   uint32_t xfin;         // transformed final state (written by the last kernel of a run)
   uint32_t pad1;
 };
@@ -105,6 +109,7 @@ struct RunParams {
   uint32_t k;      // paths per chunk in round 0
   uint32_t qs_cap;
   uint32_t vr_end, vr_oth;
+  uint32_t dense;  // 1: hand rounds with many SRE tasks to the TMA task kernel (verify exits)
 };
 
 // Host-side launch-config cache: sets the dynamic-smem attribute and queries
@@ -145,6 +150,10 @@ cudaError_t launch_build_qs2_raw(const uint32_t* d_ttc, uint32_t n, uint32_t C, 
 cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st);
 cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, int sms, cudaStream_t st,
                             uint64_t* n_done);
+// Dense recovery round: every chunk c >= f2 with rs.tstart[c] != none is re-walked from that
+// start by the TMA-staged kernel (full chunks) and the tail kernel; then the round is committed.
+cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
+                              int sms, cudaStream_t st);
 bool spec_path_generic_only();  // GSPEC_SPEC_PATH=generic forces the non-TMA kernel (A/B tests)
 cudaError_t launch_verify_recover(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* d_ctl,
                                   uint64_t* d_block_tmp, uint32_t* d_chunk_ends, cudaStream_t st, int sm_count);
@@ -221,6 +230,7 @@ struct fsm_s {
   int sm_count = 0;
   int device = 0;
   fsm_scheme auto_scheme = FSM_SCHEME_SRE;
+  double acc1_hint = 0.0;            // spec-1 accuracy from the selector's profile (dense-round gate)
   bool auto_selected = false;
   const uint32_t* d_ttc = nullptr;   // [nt][C] transformed tid x class table (prep/features)
   uint32_t* d_small = nullptr;       // small device scratch (ENUM final state, shard compose)

@@ -230,6 +230,7 @@ cudaError_t launch_shard_fuse(const DevImage& img, const uint8_t* in, uint64_t l
   switch (img.mode) {
     case MODE_U8: return fuse_m<MODE_U8>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
     case MODE_U16: return fuse_m<MODE_U16>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
+    case MODE_U16H: return fuse_m<MODE_U16H>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
     default: return fuse_m<MODE_U32>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
   }
 }
@@ -248,6 +249,10 @@ cudaError_t launch_shard_fuse_ref(const DevImage& img, const uint8_t* in, uint64
     case MODE_U16:
       if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
       k_fuse_ref<MODE_U16><<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, merged, dcnt);
+      break;
+    case MODE_U16H:
+      if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U16H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
+      k_fuse_ref<MODE_U16H><<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, merged, dcnt);
       break;
     default:
       if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;

@@ -62,9 +62,13 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       : "memory");
 }
 
-template <int MODE, int KP, int S>
+// TASKS = false: round 0 (starts from the lookback pair table).  TASKS = true: a dense
+// recovery round (Alg. 3 L16-18 for most chunks at once): chunk c >= f2 re-walks from
+// rs.tstart[c] (if set) and appends its record to VR^end.
+template <int MODE, int KP, int S, bool TASKS>
 __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
-                                                    RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off) {
+                                                    RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off,
+                                                    uint64_t tile0, uint64_t f2, Ctl* ctl) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // layout: [table (at offset 0: the lookup address is one IMAD)][stages: nwarps * S * 2 KiB][mbarriers]
   const uint32_t nwarps = blockDim.x / 32;
@@ -81,17 +85,18 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   using Sx = Step<MODE>;
 
   const uint32_t segs = rp.B / kRowBytes;
-  const uint64_t ntiles = (n_full + 31) / 32;
+  const uint64_t ntiles = (n_full + 31) / 32 - tile0;
   const uint64_t gw = (uint64_t)blockIdx.x * nwarps + warp, tw = (uint64_t)gridDim.x * nwarps;
   if (gw >= ntiles) return;
   const uint64_t my_tiles = (ntiles - gw + tw - 1) / tw;
+  uint64_t n_mustdo = 0, n_sre = 0;
   const uint64_t items = my_tiles * segs;  // (tile, segment) pairs streamed by this warp
   uint8_t* wst = stages + (size_t)warp * S * kStageBytes;
   uint64_t* wbar = bars + warp * S;
 
   const uint64_t pol = evict_first_policy();
   auto issue = [&](uint64_t it) {
-    const uint64_t t = gw + (it / segs) * tw;
+    const uint64_t t = tile0 + gw + (it / segs) * tw;
     const uint32_t sg = (uint32_t)(it % segs);
     const int s = (int)(it % S);
     mbar_expect_tx(wbar + s, kStageBytes);
@@ -105,8 +110,13 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   for (uint64_t it = 0; it < items; it++) {
     const uint32_t sg = (uint32_t)(it % segs);
     if (sg == 0) {  // new tile: predict this lane's chunk start (lookback-2 pair table)
-      c = (gw + (it / segs) * tw) * 32 + lane;
-      if (c == 0 || c >= n_full) {
+      c = (tile0 + gw + (it / segs) * tw) * 32 + lane;
+      if (TASKS) {
+        const uint32_t ts = (c < n_full && c >= f2) ? __ldcg(rs.tstart + c) : 0xFFFFFFFFu;
+        kc = ts != 0xFFFFFFFFu;  // 0: no task for this lane (walks the bytes, writes nothing)
+#pragma unroll
+        for (int p = 0; p < KP; p++) st[p] = kc ? ts : rp.q0t;
+      } else if (c == 0 || c >= n_full) {
         kc = 1;
 #pragma unroll
         for (int p = 0; p < KP; p++) st[p] = rp.q0t;
@@ -144,7 +154,19 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
     }
     __syncwarp();
     if (lane == 0 && it + S < items) issue(it + S);  // refill this stage
-    if (sg == segs - 1 && c < n_full) {  // tile done: round-0 records (VR^end)
+    if (TASKS && sg == segs - 1 && c < n_full && kc) {  // dense task done: append to VR^end
+      const uint32_t e = Sx::tid(img, code[0]);
+      const uint32_t ne = __ldcg(rs.n_end + c);
+      const uint64_t o = (uint64_t)(ne % rp.vr_end) * rs.cap + c;
+      __stcg(rs.start + o, st[0]);
+      __stcg(rs.end + o, e);
+      __stcg(rs.cnt + o, acc[0]);
+      __stcg(rs.n_end + c, ne + 1);
+      __stcg(rs.x + c + 1, e);  // Alg. 3 L17: the recovering chunk's end_c
+      __stcg(rs.cur_end + c, e);
+      if (c == f2) n_mustdo++; else n_sre++;
+    }
+    if (!TASKS && sg == segs - 1 && c < n_full) {  // tile done: round-0 records (VR^end)
       uint32_t e0 = 0;
 #pragma unroll
       for (int p = 0; p < KP; p++) {
@@ -165,6 +187,20 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
       rs.x[c + 1] = e0;
       rs.cur_end[c] = e0;
       if (c == 0) rs.x[0] = rp.q0t;
+    }
+  }
+  if (TASKS) {  // warp-level stats (warps may have returned early: no block barrier here)
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      n_mustdo += __shfl_down_sync(0xffffffffu, n_mustdo, o);
+      n_sre += __shfl_down_sync(0xffffffffu, n_sre, o);
+    }
+    if (lane == 0 && n_mustdo + n_sre) {
+      atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_mustdo), (unsigned long long)n_mustdo);
+      atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_sre), (unsigned long long)n_sre);
+      atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->active_sum), (unsigned long long)(n_mustdo + n_sre));
+      atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->reread_bytes),
+                (unsigned long long)((n_mustdo + n_sre) * rp.B));
     }
   }
 }
@@ -200,11 +236,11 @@ uint32_t pick_warps(uint64_t ntiles, int sms, uint32_t wmax) {
   return best;
 }
 
-template <int MODE, int KP, int S>
+template <int MODE, int KP, int S, bool TASKS>
 cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
-                         uint64_t n_full, int sms, cudaStream_t st) {
-  auto kern = k_spec_tma<MODE, KP, S>;
-  const uint64_t ntiles = (n_full + 31) / 32;
+                         uint64_t n_full, int sms, cudaStream_t st, uint64_t tile0, uint64_t f2, Ctl* ctl) {
+  auto kern = k_spec_tma<MODE, KP, S, TASKS>;
+  const uint64_t ntiles = (n_full + 31) / 32 - tile0;
   const uint32_t tbytes = smem_bytes_for(img);
   const uint32_t per_warp = S * kStageBytes + S * 8;
   const uint32_t avail = 227 * 1024 - ((tbytes + 1023) & ~1023u) - 64;
@@ -218,54 +254,79 @@ cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunPa
   if (e != cudaSuccess) return e;
   uint64_t grid = std::min<uint64_t>((uint64_t)sms, (ntiles + w - 1) / w);
   if (grid < 1) grid = 1;
-  kern<<<(unsigned)grid, w * 32, smem, st>>>(tm, img, rp, rs, n_full, table_off);
+  kern<<<(unsigned)grid, w * 32, smem, st>>>(tm, img, rp, rs, n_full, table_off, tile0, f2, ctl);
   return cudaGetLastError();
 }
 
-template <int MODE, int KP>
+template <int MODE, int KP, bool TASKS>
 cudaError_t launch_tma_s(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
-                         uint64_t n_full, int sms, cudaStream_t st) {
+                         uint64_t n_full, int sms, cudaStream_t st, uint64_t tile0, uint64_t f2, Ctl* ctl) {
   const uint32_t tbytes = smem_bytes_for(img);
   if (tbytes + 24 * (3 * kStageBytes) + 2048 <= 227 * 1024)
-    return launch_tma_t<MODE, KP, 3>(tm, img, rp, rs, n_full, sms, st);
-  return launch_tma_t<MODE, KP, 2>(tm, img, rp, rs, n_full, sms, st);
+    return launch_tma_t<MODE, KP, 3, TASKS>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl);
+  return launch_tma_t<MODE, KP, 2, TASKS>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl);
 }
 
 template <int MODE>
 cudaError_t launch_tma_m(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
                          uint64_t n_full, int sms, cudaStream_t st) {
-  if (rp.k <= 1) return launch_tma_s<MODE, 1>(tm, img, rp, rs, n_full, sms, st);
-  if (rp.k <= 2) return launch_tma_s<MODE, 2>(tm, img, rp, rs, n_full, sms, st);
-  if (rp.k <= 4) return launch_tma_s<MODE, 4>(tm, img, rp, rs, n_full, sms, st);
-  return launch_tma_s<MODE, 8>(tm, img, rp, rs, n_full, sms, st);
+  if (rp.k <= 1) return launch_tma_s<MODE, 1, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
+  if (rp.k <= 2) return launch_tma_s<MODE, 2, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
+  if (rp.k <= 4) return launch_tma_s<MODE, 4, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
+  return launch_tma_s<MODE, 8, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
+}
+
+bool encode_map(const RunParams& rp, uint64_t n_full, CUtensorMap* tm) {
+  EncodeFn enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {rp.B, n_full};
+  cuuint64_t strides[1] = {rp.B};
+  cuuint32_t box[2] = {kRowBytes, 32};
+  cuuint32_t es[2] = {1, 1};
+  return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(rp.in), dims, strides, box, es,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+bool tma_applies(const RunParams& rp, uint64_t n_full) {
+  return n_full > 0 && rp.B % kRowBytes == 0 && (reinterpret_cast<uintptr_t>(rp.in) & 15u) == 0 &&
+         n_full < (1ull << 31);
 }
 
 }  // namespace
 
 // Returns cudaErrorNotSupported when the TMA path does not apply (caller falls
-// back to the generic kernel): unaligned input, B % 128 != 0, no full chunks.
+// back to the generic kernel): unaligned input, B % 64 != 0, no full chunks.
 cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, int sms, cudaStream_t st,
                             uint64_t* n_done) {
   *n_done = 0;
   const uint64_t n_full = rp.len / rp.B;
-  if (n_full == 0 || rp.B % kRowBytes != 0 || (reinterpret_cast<uintptr_t>(rp.in) & 15u) != 0 || n_full >= (1ull << 31))
-    return cudaErrorNotSupported;
-  EncodeFn enc = get_encode();
-  if (!enc) return cudaErrorNotSupported;
   CUtensorMap tm;
-  cuuint64_t dims[2] = {rp.B, n_full};
-  cuuint64_t strides[1] = {rp.B};
-  cuuint32_t box[2] = {kRowBytes, 32};
-  cuuint32_t es[2] = {1, 1};
-  CUresult r = enc(&tm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(rp.in), dims, strides, box, es,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) return cudaErrorNotSupported;
+  if (!tma_applies(rp, n_full) || !encode_map(rp, n_full, &tm)) return cudaErrorNotSupported;
   cudaError_t e;
   switch (img.mode) {
     case MODE_U8: e = launch_tma_m<MODE_U8>(tm, img, rp, rs, n_full, sms, st); break;
     case MODE_U16: e = launch_tma_m<MODE_U16>(tm, img, rp, rs, n_full, sms, st); break;
+    case MODE_U16H: e = launch_tma_m<MODE_U16H>(tm, img, rp, rs, n_full, sms, st); break;
     default: e = launch_tma_m<MODE_U32>(tm, img, rp, rs, n_full, sms, st); break;
+  }
+  if (e == cudaSuccess) *n_done = n_full;
+  return e;
+}
+
+cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
+                            int sms, cudaStream_t st, uint64_t* n_done) {
+  *n_done = 0;
+  const uint64_t n_full = rp.len / rp.B;
+  CUtensorMap tm;
+  if (f2 >= n_full || !tma_applies(rp, n_full) || !encode_map(rp, n_full, &tm)) return cudaErrorNotSupported;
+  const uint64_t tile0 = f2 / 32;
+  cudaError_t e;
+  switch (img.mode) {
+    case MODE_U8: e = launch_tma_s<MODE_U8, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
+    case MODE_U16: e = launch_tma_s<MODE_U16, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
+    case MODE_U16H: e = launch_tma_s<MODE_U16H, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
+    default: e = launch_tma_s<MODE_U32, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
   }
   if (e == cudaSuccess) *n_done = n_full;
   return e;

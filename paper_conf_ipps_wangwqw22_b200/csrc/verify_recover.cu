@@ -180,8 +180,12 @@ __device__ void task_walk(const DevImage& img, const uint8_t* smem, const RunPar
   if (aligned) {
     const uint64_t nf = min(n, (uint64_t)kFuseMax) / 16;
     const uint4* v = reinterpret_cast<const uint4*>(p);
+    uint4 q0 = nf > 0 ? __ldg(v) : make_uint4(0, 0, 0, 0);
+    uint4 q1 = nf > 1 ? __ldg(v + 1) : make_uint4(0, 0, 0, 0);
     for (uint64_t j = 0; j < nf; j++) {
-      uint4 q = __ldg(v + j);
+      const uint4 q = q0;
+      q0 = q1;
+      if (j + 2 < nf) q1 = __ldg(v + j + 2);
       uint32_t w[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
       for (int t = 0; t < 4; t++) {
@@ -285,6 +289,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         checks++;
         matches += fd;
         if (!fd) fm = min(fm, c);
+        if (rp.dense) __stcg(rs.tstart + c, fd ? 0xFFFFFFFFu : ld_cg(rs.x + c));
         if (fast && sre_like) {  // list every chunk without a match (warp-aggregated append)
           const uint32_t am = __activemask();
           const uint32_t bal = __ballot_sync(am, !fd);
@@ -317,6 +322,15 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     const uint64_t f2 = vctl->fmin;
     if (f2 >= N) break;
     const uint32_t tf2 = ld_cg(rs.x + f2);
+    if (fast && sre_like && rp.dense) {
+      // dense round: most chunks need re-execution -> exit; the host runs the TMA-staged
+      // task kernel over chunk tiles (same tasks, same records) and relaunches us
+      const uint64_t nt = ld_cg64(&ctl->ntask[rnd & 1]);
+      if (nt >= 2048 && nt * 16 >= N - f2) {
+        if (b == 0 && threadIdx.x == 0) vctl->dense_pending = 1;
+        return;
+      }
+    }
     if (fast) {
       // ---------------- E (fast): must-do (+ SRE) tasks from the list --------------
       const uint64_t T = (uint64_t)G * kBS, gt = (uint64_t)b * kBS + threadIdx.x;
@@ -583,7 +597,72 @@ cudaError_t launch_m(const DevImage& img, const RunParams& rp, const RecStore& r
   return cudaLaunchCooperativeKernel((const void*)kern, dim3((unsigned)grid), dim3(kBS), args, smem, st);
 }
 
+// After the TMA task kernel: the partial tail chunk's task (if any), then commit
+// the round (Alg. 3 L14: the frontier advances to f2).
+template <int MODE>
+__global__ void __launch_bounds__(32) k_dense_finish(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
+                                                     uint64_t c_first_generic) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  stage_table(img, smem);
+  __syncwarp();
+  if (threadIdx.x != 0) return;
+  const uint64_t f2 = ctl->fmin;
+  for (uint64_t c = max(c_first_generic, f2); c < rp.N; c++) {
+    const uint32_t st = __ldcg(rs.tstart + c);
+    if (st == 0xFFFFFFFFu) continue;
+    uint32_t e, cnt;
+    task_walk<MODE>(img, smem, rp, rs, c, st, &e, &cnt);
+    const uint32_t ne = ld_cg(rs.n_end + c);
+    const uint64_t o = (uint64_t)(ne % rp.vr_end) * rs.cap + c;
+    st_cg(rs.start + o, st);
+    st_cg(rs.end + o, e);
+    st_cg(rs.cnt + o, cnt);
+    st_cg(rs.n_end + c, ne + 1);
+    st_cg(rs.x + c + 1, e);
+    st_cg(rs.cur_end + c, e);
+    if (c == f2) ctl->tasks_mustdo++; else ctl->tasks_sre++;
+    ctl->active_sum++;
+    ctl->reread_bytes += min((uint64_t)rp.B, rp.len - c * rp.B);
+  }
+  ctl->rounds++;
+  ctl->f = f2;
+  ctl->tf = ld_cg(rs.x + f2);
+  ctl->dense_pending = 0;
+}
+
+template <int MODE>
+cudaError_t launch_dense_finish(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl,
+                                uint64_t c_first_generic, cudaStream_t st) {
+  auto kern = k_dense_finish<MODE>;
+  const uint32_t smem = smem_bytes_for(img);
+  cudaError_t e = kernel_setup((const void*)kern, smem, 32, nullptr);
+  if (e != cudaSuccess) return e;
+  kern<<<1, 32, smem, st>>>(img, rp, rs, ctl, c_first_generic);
+  return cudaGetLastError();
+}
+
 }  // namespace
+
+cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
+                            int sms, cudaStream_t st, uint64_t* n_done);
+
+cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
+                              int sms, cudaStream_t st) {
+  uint64_t done = 0;
+  cudaError_t e = launch_task_tma(img, rp, rs, ctl, f2, sms, st, &done);
+  if (e == cudaErrorNotSupported) {
+    cudaGetLastError();
+    done = 0;  // the finish kernel walks everything (slow, but exact)
+  } else if (e != cudaSuccess) {
+    return e;
+  }
+  switch (img.mode) {
+    case MODE_U8: return launch_dense_finish<MODE_U8>(img, rp, rs, ctl, done, st);
+    case MODE_U16: return launch_dense_finish<MODE_U16>(img, rp, rs, ctl, done, st);
+    case MODE_U16H: return launch_dense_finish<MODE_U16H>(img, rp, rs, ctl, done, st);
+    default: return launch_dense_finish<MODE_U32>(img, rp, rs, ctl, done, st);
+  }
+}
 
 uint32_t verify_recover_max_grid();
 
@@ -593,6 +672,7 @@ cudaError_t launch_verify_recover(const DevImage& img, const RunParams& rp, cons
   switch (img.mode) {
     case MODE_U8: return launch_m<MODE_U8>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
     case MODE_U16: return launch_m<MODE_U16>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
+    case MODE_U16H: return launch_m<MODE_U16H>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
     default: return launch_m<MODE_U32>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
   }
 }

@@ -10,17 +10,19 @@
 namespace gspec {
 
 // Copy the hot table prefix (and the class map) into dynamic shared memory.
-// Layout: [table: smem_table_bytes][cls: 256 B]
+// Layout: u8 mode: [table]; classed modes: [cls: 256 B][table: smem_table_bytes]
+// (the class map first keeps it 256-aligned: its address is one PRMT away).
 __device__ __forceinline__ void stage_table(const DevImage& img, uint8_t* smem) {
-  const uint4* src = (img.mode == MODE_U8)    ? reinterpret_cast<const uint4*>(img.T8)
-                     : (img.mode == MODE_U16) ? reinterpret_cast<const uint4*>(img.T16)
-                                              : reinterpret_cast<const uint4*>(img.T32);
-  uint4* dst = reinterpret_cast<uint4*>(smem);
+  const uint4* src = (img.mode == MODE_U8)                                 ? reinterpret_cast<const uint4*>(img.T8)
+                     : (img.mode == MODE_U16 || img.mode == MODE_U16H) ? reinterpret_cast<const uint4*>(img.T16)
+                                                                         : reinterpret_cast<const uint4*>(img.T32);
+  const uint32_t off = img.mode == MODE_U8 ? 0u : 256u;
+  uint4* dst = reinterpret_cast<uint4*>(smem + off);
   const uint32_t nv = img.smem_table_bytes / 16;
   for (uint32_t i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(src + i);
   if (img.mode != MODE_U8) {
     const uint4* cs = reinterpret_cast<const uint4*>(img.cls);
-    uint4* cd = reinterpret_cast<uint4*>(smem + img.smem_table_bytes);
+    uint4* cd = reinterpret_cast<uint4*>(smem);
     for (uint32_t i = threadIdx.x; i < 16; i += blockDim.x) cd[i] = __ldg(cs + i);
   }
 }
@@ -70,32 +72,51 @@ struct Step<MODE_U8> {
   static __device__ __forceinline__ uint32_t tid(const DevImage& img, uint32_t code) { return __ldg(img.code2tid + code); }
 };
 
-// MODE_U16 / MODE_U32: classed rows; tid < H is hot (smem), else global/L2.
-template <typename CodeT, int SHIFT>
+__device__ __forceinline__ uint32_t lds_u16(uint32_t saddr) {
+  uint32_t v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=r"(v) : "r"(saddr));
+  return v;
+}
+
+__device__ __forceinline__ uint32_t lds_u32(uint32_t saddr) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(saddr));
+  return v;
+}
+
+// MODE_U16 / MODE_U16H / MODE_U32: classed rows (smem: [cls][rows]); tid < H is
+// hot (smem), else global/L2.  ALLHOT drops the hot test (every row in smem).
+template <typename CodeT, int SHIFT, bool ALLHOT>
 struct StepClassed {
   static constexpr uint32_t kShift = SHIFT;
   static constexpr uint32_t kMask = (1u << SHIFT) - 1u;
-  static __device__ __forceinline__ uint32_t byte(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t b) {
-    const CodeT* st = reinterpret_cast<const CodeT*>(s);
-    const uint8_t* sc = s + img.smem_table_bytes;
-    uint32_t t = code & kMask;
-    uint32_t idx = t * img.C + sc[b];
-    if (t < img.H) return st[idx];
+  static __device__ __forceinline__ uint32_t row(const DevImage& img, uint32_t base, uint32_t code, uint32_t cl) {
+    const uint32_t t = code & kMask;
+    const uint32_t idx = t * img.C + cl;
+    if (ALLHOT || t < img.H)
+      return sizeof(CodeT) == 2 ? lds_u16(base + 256 + idx * 2) : lds_u32(base + 256 + idx * 4);
     const CodeT* g = (sizeof(CodeT) == 2) ? reinterpret_cast<const CodeT*>(img.T16) : reinterpret_cast<const CodeT*>(img.T32);
     return __ldg(g + idx);
   }
+  static __device__ __forceinline__ uint32_t byte(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t b) {
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
+    return row(img, base, code, lds_u8(base + b));
+  }
   template <int K>
   static __device__ __forceinline__ uint32_t word(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t w) {
-    return byte(img, s, code, (w >> (8 * K)) & 0xffu);
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
+    return row(img, base, code, lds_u8(byte_plus<K>(w, base)));  // class map at the 256-aligned base
   }
   static __device__ __forceinline__ uint32_t acc(uint32_t code) { return code >> SHIFT; }
   static __device__ __forceinline__ uint32_t tid(const DevImage&, uint32_t code) { return code & kMask; }
 };
 
 template <>
-struct Step<MODE_U16> : StepClassed<uint16_t, 15> {};
+struct Step<MODE_U16> : StepClassed<uint16_t, 15, false> {};
 template <>
-struct Step<MODE_U32> : StepClassed<uint32_t, 31> {};
+struct Step<MODE_U16H> : StepClassed<uint16_t, 15, true> {};
+template <>
+struct Step<MODE_U32> : StepClassed<uint32_t, 31, false> {};
 
 // Walk one path over [p, p+n) bytes from `code`; returns end code, adds accepts.
 template <int MODE>
@@ -106,9 +127,14 @@ __device__ __forceinline__ uint32_t walk_bytes(const DevImage& img, const uint8_
   // vector part when 16-byte aligned
   if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
     const uint4* v = reinterpret_cast<const uint4*>(p);
-    uint64_t nv = n / 16;
+    const uint64_t nv = n / 16;
+    // software pipeline: two 16-byte loads in flight ahead of the dependent chain
+    uint4 q0 = nv > 0 ? __ldg(v) : make_uint4(0, 0, 0, 0);
+    uint4 q1 = nv > 1 ? __ldg(v + 1) : make_uint4(0, 0, 0, 0);
     for (uint64_t j = 0; j < nv; j++) {
-      uint4 q = __ldg(v + j);
+      const uint4 q = q0;
+      q0 = q1;
+      if (j + 2 < nv) q1 = __ldg(v + j + 2);
       uint32_t w[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
       for (int t = 0; t < 4; t++) {

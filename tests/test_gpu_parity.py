@@ -248,3 +248,20 @@ def test_async_queue(gs):
         assert (ce.cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
     with pytest.raises(gs.GSpecError):
         fsm.wait(runs[0][0])  # already collected
+
+
+@pytest.mark.parametrize("name,length,B", [("c3", 32 << 20, 4096), ("c3", (24 << 20) + 1000, 4096),
+                                           ("c3s", 160 << 20, 8192)])
+def test_dense_recovery_rounds(gs, name, length, B):
+    """SRE on a low-accuracy DFA: rounds where most chunks re-execute go to the
+    TMA-staged task kernel; results and round diagnostics stay identical."""
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    res = fsm.run(torch.from_numpy(data).cuda(), scheme="sre", chunk_bytes=B)
+    check_equal(res, ref, B, w.nstates)
+    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme="sre")
+    for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks",
+              "verify_matches"):
+        assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+    assert res.stats["tasks_sre"] > 2048  # the dense path really ran
