@@ -190,6 +190,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   h.f = 0;
   h.tf = q0t;
   h.fmin = N;
+  h.it_fm[0] = N;  // first relaxation pass slot
   if (scheme == FSM_SCHEME_ENUM) {
     if (f->n + 1 > kEnumMax) {
       pd.active = false;

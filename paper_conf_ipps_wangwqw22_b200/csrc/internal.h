@@ -92,7 +92,8 @@ struct Ctl {
   uint64_t accept_count;
   uint64_t nA, I, nU;    // this round: A-tasks, idle workers, total untried candidates
   uint64_t jacobi_iters;
-  uint64_t ntask[2];     // fast path (SEQ/PM/SRE): per-round task-list length (alternating)
+  uint64_t ntask[2];     // (unused, kept for layout)
+  uint64_t it_fm[3], it_checks[3], it_matches[3], it_ntask[3];  // per relaxation pass (rotating)
   uint32_t dense_pending;  // verify exited: a dense task round (frontier fmin) must run first
   uint32_t pad2;
   uint32_t xfin;         // transformed final state (written by the last kernel of a run)

@@ -95,22 +95,26 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   uint64_t* wbar = bars + warp * S;
 
   const uint64_t pol = evict_first_policy();
-  auto issue = [&](uint64_t it) {
-    const uint64_t t = tile0 + gw + (it / segs) * tw;
-    const uint32_t sg = (uint32_t)(it % segs);
-    const int s = (int)(it % S);
-    mbar_expect_tx(wbar + s, kStageBytes);
-    tma_load_2d(wst + (size_t)s * kStageBytes, &tmap, wbar + s, (int32_t)(sg * kRowBytes), (int32_t)(t * 32), pol);
+  // producer cursor (lane 0): the item S ahead of the consumer, tracked without divisions
+  uint64_t p_tile = 0;
+  uint32_t p_sg = 0, p_s = 0;
+  auto issue_next = [&]() {
+    const uint64_t t = tile0 + gw + p_tile * tw;
+    mbar_expect_tx(wbar + p_s, kStageBytes);
+    tma_load_2d(wst + (size_t)p_s * kStageBytes, &tmap, wbar + p_s, (int32_t)(p_sg * kRowBytes), (int32_t)(t * 32),
+                pol);
+    if (++p_sg == segs) { p_sg = 0; p_tile++; }
+    if (++p_s == (uint32_t)S) p_s = 0;
   };
   if (lane == 0)
-    for (uint64_t it = 0; it < items && it < (uint64_t)S; it++) issue(it);
+    for (uint64_t it = 0; it < items && it < (uint64_t)S; it++) issue_next();
 
   uint32_t st[KP], code[KP], acc[KP], kc = 1;
-  uint64_t c = 0;
+  uint64_t c = 0, tile_i = 0;
+  uint32_t sg = 0, s = 0, phase = 0;
   for (uint64_t it = 0; it < items; it++) {
-    const uint32_t sg = (uint32_t)(it % segs);
     if (sg == 0) {  // new tile: predict this lane's chunk start (lookback-2 pair table)
-      c = (tile0 + gw + (it / segs) * tw) * 32 + lane;
+      c = (tile0 + gw + tile_i * tw) * 32 + lane;
       if (TASKS) {
         const uint32_t ts = (c < n_full && c >= f2) ? __ldcg(rs.tstart + c) : 0xFFFFFFFFu;
         kc = ts != 0xFFFFFFFFu;  // 0: no task for this lane (walks the bytes, writes nothing)
@@ -133,8 +137,7 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
         acc[p] = 0;
       }
     }
-    const int s = (int)(it % S);
-    mbar_wait(wbar + s, (uint32_t)((it / S) & 1));
+    mbar_wait(wbar + s, phase);
     const uint8_t* row = wst + (size_t)s * kStageBytes + lane * kRowBytes;
 #pragma unroll
     for (int u = 0; u < (int)(kRowBytes / 16); u++) {
@@ -153,7 +156,7 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
       }
     }
     __syncwarp();
-    if (lane == 0 && it + S < items) issue(it + S);  // refill this stage
+    if (lane == 0 && it + S < items) issue_next();  // refill this stage
     if (TASKS && sg == segs - 1 && c < n_full && kc) {  // dense task done: append to VR^end
       const uint32_t e = Sx::tid(img, code[0]);
       const uint32_t ne = __ldcg(rs.n_end + c);
@@ -188,6 +191,8 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
       rs.cur_end[c] = e0;
       if (c == 0) rs.x[0] = rp.q0t;
     }
+    if (++sg == segs) { sg = 0; tile_i++; }
+    if (++s == (uint32_t)S) { s = 0; phase ^= 1u; }
   }
   if (TASKS) {  // warp-level stats (warps may have returned early: no block barrier here)
 #pragma unroll

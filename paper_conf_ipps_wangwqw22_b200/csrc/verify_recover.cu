@@ -19,6 +19,8 @@
 // thread keeps the record it is matching in registers.
 #include <cooperative_groups.h>
 
+#include <cstdlib>
+
 #include "internal.h"
 #include "walk.cuh"
 
@@ -234,6 +236,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   // matching record (SRE) or the frontier alone (SEQ/PM), so they are listed in
   // phase F and executed in E: two grid barriers per round besides V.
   const bool fast = !helpers;
+  uint32_t git = 0;  // relaxation passes since launch (identical in every CTA)
   const bool cached = cache_cap != 0 && hi - lo <= cache_cap;
   const VrCache vc = vr_cache_at(smem + ((smem_bytes_for(img) + 15) & ~15u), cache_cap);
   for (;;) {
@@ -252,15 +255,25 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       }
       __syncthreads();
     }
-    // ---------------- V: verification by chaotic relaxation ----------------
-    if (b == 0 && threadIdx.x == 0) {
-      vctl->fmin = N;
-      vctl->ntask[(rnd + 1) & 1] = 0;
-    }
-    uint32_t it = 0;
+    // ---------------- V+F: verification by chaotic relaxation ----------------
+    // Every pass also computes the frontier candidate, the accuracy counters and
+    // (fast path) the task list, into per-pass slots; the pass that changes
+    // nothing is the fixed point, and its slot is the round's result, so the
+    // frontier costs no extra barrier.
+    // pass slots rotate over a launch-wide pass counter (slot 0 is zeroed by the
+    // host init / the dense-round commit before a launch; slot p+1 is reset by
+    // CTA 0 at the start of pass p, two barriers before anyone reads it again)
+    uint32_t it = 0, slot = 0;
     for (;;) {
-      if (b == 0 && threadIdx.x == 0) vctl->changed[(it + 1) % 3] = 0;
+      slot = git % 3;
+      if (b == 0 && threadIdx.x == 0) {
+        const uint32_t nx = (git + 1) % 3;
+        vctl->changed[nx] = 0;
+        vctl->it_fm[nx] = N;
+        vctl->it_checks[nx] = vctl->it_matches[nx] = vctl->it_ntask[nx] = 0;
+      }
       bool ch = false;
+      uint64_t fm = ~0ull, matches = 0, checks = 0;
       for (uint64_t c = max(lo, f) + threadIdx.x; c < hi; c += kBS) {
         const uint32_t xin = (c == f) ? tf : ld_cg(rs.x + c);
         uint32_t e;
@@ -272,60 +285,62 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
           st_cg(rs.x + c + 1, e);
           ch = true;
         }
-      }
-      if (__syncthreads_or(ch) && threadIdx.x == 0) vctl->changed[it % 3] = 1;
-      grid.sync();
-      const bool any = vctl->changed[it % 3] != 0;
-      it++;
-      if (!any) break;
-    }
-    // ---------------- F: frontier + runtime accuracy counters ----------------
-    {
-      uint64_t fm = ~0ull;
-      uint64_t matches = 0, checks = 0;
-      for (uint64_t c = max(lo, f) + threadIdx.x; c < hi; c += kBS) {
-        const bool fd = __ldcg(rs.found + c);
-        st_cg(rs.cur_end + c, ld_cg(rs.x + c + 1));  // rear ripple result (Alg. 3 L10)
         checks++;
-        matches += fd;
-        if (!fd) fm = min(fm, c);
-        if (rp.dense) __stcg(rs.tstart + c, fd ? 0xFFFFFFFFu : ld_cg(rs.x + c));
+        matches += hit;
+        if (!hit) fm = min(fm, c);
+        if (rp.dense) __stcg(rs.tstart + c, hit ? 0xFFFFFFFFu : xin);
         if (fast && sre_like) {  // list every chunk without a match (warp-aggregated append)
           const uint32_t am = __activemask();
-          const uint32_t bal = __ballot_sync(am, !fd);
+          const uint32_t bal = __ballot_sync(am, !hit);
           if (bal) {
             const uint32_t lane = threadIdx.x & 31, leader = __ffs(bal) - 1;
             unsigned long long base = 0;
             if (lane == leader)
-              base = atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->ntask[rnd & 1]),
+              base = atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_ntask[slot]),
                                (unsigned long long)__popc(bal));
             base = __shfl_sync(am, base, leader);
-            if (!fd) {
-              const uint64_t slot = base + __popc(bal & ((1u << lane) - 1));
-              rs.task_chunk[slot] = (uint32_t)c;
-              rs.task_start[slot] = ld_cg(rs.x + c);  // captured before E rewrites x
+            if (!hit) {
+              const uint64_t q = base + __popc(bal & ((1u << lane) - 1));
+              rs.task_chunk[q] = (uint32_t)c;
+              rs.task_start[q] = xin;  // captured before E rewrites x
             }
           }
         }
       }
+      const bool bch = __syncthreads_or(ch);
       fm = block_min(fm, red64);
       checks = block_sum<uint64_t>(checks, red64);
       matches = block_sum<uint64_t>(matches, red64);
       if (threadIdx.x == 0) {
-        if (fm != ~0ull) atomicMin(reinterpret_cast<unsigned long long*>(&ctl->fmin), (unsigned long long)fm);
-        atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->verify_checks), (unsigned long long)checks);
-        atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->verify_matches), (unsigned long long)matches);
-        if (b == 0) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->jacobi_iters), (unsigned long long)it);
+        if (bch) vctl->changed[slot] = 1;
+        if (fm != ~0ull) atomicMin(reinterpret_cast<unsigned long long*>(&ctl->it_fm[slot]), (unsigned long long)fm);
+        if (checks) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_checks[slot]), (unsigned long long)checks);
+        if (matches)
+          atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_matches[slot]), (unsigned long long)matches);
       }
+      grid.sync();
+      const bool any = vctl->changed[slot] != 0;
+      it++;
+      git++;
+      if (!any) break;
     }
-    grid.sync();
-    const uint64_t f2 = vctl->fmin;
+    const uint64_t f2 = vctl->it_fm[slot];
+    if (b == 0 && threadIdx.x == 0) {
+      vctl->verify_checks = vctl->verify_checks + vctl->it_checks[slot];
+      vctl->verify_matches = vctl->verify_matches + vctl->it_matches[slot];
+      vctl->jacobi_iters = vctl->jacobi_iters + it;
+      vctl->fmin = f2;
+    }
     if (f2 >= N) break;
+    // rear ripple result (Alg. 3 L10): cur_end of matched chunks follows the chain
+    // (unmatched chunks keep theirs; their tasks set it in E)
+    for (uint64_t c = max(lo, f) + threadIdx.x; c < hi; c += kBS)
+      if (__ldcg(rs.found + c)) st_cg(rs.cur_end + c, ld_cg(rs.x + c + 1));
     const uint32_t tf2 = ld_cg(rs.x + f2);
     if (fast && sre_like && rp.dense) {
       // dense round: most chunks need re-execution -> exit; the host runs the TMA-staged
       // task kernel over chunk tiles (same tasks, same records) and relaunches us
-      const uint64_t nt = ld_cg64(&ctl->ntask[rnd & 1]);
+      const uint64_t nt = ld_cg64(&ctl->it_ntask[slot]);
       if (nt >= 2048 && nt * 16 >= N - f2) {
         if (b == 0 && threadIdx.x == 0) vctl->dense_pending = 1;
         return;
@@ -334,7 +349,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     if (fast) {
       // ---------------- E (fast): must-do (+ SRE) tasks from the list --------------
       const uint64_t T = (uint64_t)G * kBS, gt = (uint64_t)b * kBS + threadIdx.x;
-      const uint64_t nt = sre_like ? ld_cg64(&ctl->ntask[rnd & 1]) : 1;
+      const uint64_t nt = sre_like ? ld_cg64(&ctl->it_ntask[slot]) : 1;
       uint64_t mustdo = 0, sre = 0, reread = 0;
       for (uint64_t s = gt; s < nt; s += T) {
         const uint32_t c = sre_like ? __ldcg(rs.task_chunk + s) : (uint32_t)f2;
@@ -577,6 +592,12 @@ cudaError_t launch_m(const DevImage& img, const RunParams& rp, const RecStore& r
   cudaError_t e = kernel_setup((const void*)kern, tsmem, kBS, &occ);
   if (e != cudaSuccess) return e;
   if (occ < 1) return cudaErrorInvalidConfiguration;
+  static int bps = -1;  // CTAs per SM (GSPEC_VR_CTAS_PER_SM overrides; fewer CTAs = cheaper grid barriers)
+  if (bps < 0) {
+    const char* ev = getenv("GSPEC_VR_CTAS_PER_SM");
+    bps = ev ? atoi(ev) : 0;
+  }
+  if (bps > 0 && bps < occ) occ = bps;
   uint64_t grid = (uint64_t)sms * occ;
   const uint64_t want = (rp.N + kBS - 1) / kBS;
   if (want < grid) grid = want < 1 ? 1 : want;
@@ -628,6 +649,9 @@ __global__ void __launch_bounds__(32) k_dense_finish(DevImage img, RunParams rp,
   ctl->f = f2;
   ctl->tf = ld_cg(rs.x + f2);
   ctl->dense_pending = 0;
+  ctl->changed[0] = 0;  // the relaunched kernel starts its passes at slot 0
+  ctl->it_fm[0] = rp.N;
+  ctl->it_checks[0] = ctl->it_matches[0] = ctl->it_ntask[0] = 0;
 }
 
 template <int MODE>
