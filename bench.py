@@ -333,7 +333,8 @@ def main():
                          "verify_recover": round(sorted(ver_ms)[len(ver_ms) // 2], 4)},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": traffic,
-                     "kernel": "k_spec_exec", "peak_kind": peak_kind},
+                     "kernel": "k_spec_tma (speculative execution, TMA-staged)", "peak_kind": peak_kind,
+                     "achieved_def": "input bytes per launch / CUDA-event duration of the spec launch"},
         "diagnostics": {k: kr[-1].stats[k] for k in ("rounds", "tasks_total", "tasks_mustdo", "tasks_sre",
                                                      "tasks_helper", "reread_bytes", "verify_checks",
                                                      "verify_matches")},

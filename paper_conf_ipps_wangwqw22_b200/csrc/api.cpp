@@ -218,7 +218,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   } else {
     if (f->rs_cap < N) CUDA_TRY(cudaStreamSynchronize(o.st));  // growing the store: drain queued runs
     if ((rc = ensure_records(f, N))) return rc;
-    CUDA_TRY(cudaMemcpyAsync(f->d_ctl, &h, sizeof(Ctl), cudaMemcpyHostToDevice, o.st));
+    rp.ctl_init = f->d_ctl;  // the spec kernel initialises the control block
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
     // dense recovery rounds go to the TMA task kernel (SRE on low-accuracy DFAs); this
     // needs a host check per verify launch, so it is off when the profile says the

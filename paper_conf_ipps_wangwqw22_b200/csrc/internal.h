@@ -111,6 +111,7 @@ struct RunParams {
   uint32_t qs_cap;
   uint32_t vr_end, vr_oth;
   uint32_t dense;  // 1: hand rounds with many SRE tasks to the TMA task kernel (verify exits)
+  Ctl* ctl_init;   // non-null: the first spec kernel initialises this control block (no H2D copy)
 };
 
 // Host-side launch-config cache: sets the dynamic-smem attribute and queries

@@ -30,6 +30,7 @@ template <int MODE, int NI, int KP>
 __global__ void __launch_bounds__(256) k_spec_exec(DevImage img, RunParams rp, RecStore rs, uint64_t c0) {
   extern __shared__ __align__(1024) uint8_t smem[];
   stage_table(img, smem);
+  if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, rp.q0t, rp.N);
   __syncthreads();
   using S = Step<MODE>;
   const uint64_t N = rp.N, B = rp.B, len = rp.len;
@@ -182,11 +183,15 @@ cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const Rec
   uint64_t done = 0;
   cudaError_t e = spec_path_generic_only() ? cudaErrorNotSupported : launch_spec_tma(img, rp, rs, sms, st, &done);
   if (e != cudaSuccess && e != cudaErrorNotSupported) return e;
+  RunParams rp2 = rp;
   if (e == cudaErrorNotSupported) {
     cudaGetLastError();  // clear
     done = 0;
+  } else {
+    rp2.ctl_init = nullptr;  // already initialised by the TMA kernel
   }
-  return launch_spec_generic(img, rp, rs, st, done);  // tail chunk (or everything)
+  if (done >= rp.N) return cudaSuccess;
+  return launch_spec_generic(img, rp2, rs, st, done);  // tail chunk (or everything)
 }
 
 }  // namespace gspec

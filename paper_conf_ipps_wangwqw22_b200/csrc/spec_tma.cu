@@ -77,6 +77,7 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   uint8_t* stages = smem_raw + table_off;
   uint64_t* bars = reinterpret_cast<uint64_t*>(stages + (size_t)nwarps * S * kStageBytes);
   stage_table(img, table);
+  if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, rp.q0t, rp.N);
   if (lane == 0)
     for (int s = 0; s < S; s++) mbar_init(bars + warp * S + s, 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");

@@ -190,6 +190,19 @@ __device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, u
   return false;
 }
 
+// Initialise the verify/recover control block for a run (block 0 of the first kernel).
+__device__ __forceinline__ void init_ctl(Ctl* ctl, uint32_t q0t, uint64_t N) {
+  uint32_t* w = reinterpret_cast<uint32_t*>(ctl);
+  for (uint32_t i = threadIdx.x; i < sizeof(Ctl) / 4; i += blockDim.x) w[i] = 0;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    ctl->f = 0;
+    ctl->tf = q0t;
+    ctl->fmin = N;
+    ctl->it_fm[0] = N;
+  }
+}
+
 // Ranked lookback candidates of chunk c >= 1 (lookback-2 pair table).
 __device__ __forceinline__ uint32_t qs_pair(const DevImage& img, const uint8_t* in, uint64_t c, uint32_t B) {
   uint64_t e = c * (uint64_t)B;

@@ -265,3 +265,17 @@ def test_dense_recovery_rounds(gs, name, length, B):
               "verify_matches"):
         assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
     assert res.stats["tasks_sre"] > 2048  # the dense path really ran
+
+
+@pytest.mark.parametrize("name,length,scheme", [("c3", 1 << 30, "auto"), ("c3", 1 << 30, "sre"), ("c4", 4 << 30, "auto")])
+def test_full_size_other_configs(gs, name, length, scheme):
+    """BASELINE configs C3 (1 GB) and C4 (4 GB) at full size vs the oracle."""
+    w = gen.workload(name, length=length)
+    x = torch.empty(length, dtype=torch.uint8, device="cuda")
+    w.device(x)
+    h = w.host()
+    ref = oracle.run(w.table, w.start, w.accept, h, 4096)
+    del h
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    res = fsm.run(x, scheme=scheme)
+    check_equal(res, ref, 4096, w.nstates)
