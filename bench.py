@@ -228,6 +228,7 @@ def main():
 
     # kernel-level split (spec exec vs verify/recover) from single-shard runs on this GPU
     kr = [fsm.run(x, scheme=scheme, chunk_bytes=B) for _ in range(3)]
+    verify_phases = [round(float(v), 1) for v in fsm.phase_times()]
     for _ in range(max(3, args.warmup)):
         res = step()
     if world == 1:
@@ -329,6 +330,7 @@ def main():
                    else "single GPU"},
         "pct_hbm_roofline_8TBs": round(100 * value / world / 8000.0, 2),
         "latency_ms_per_GB": round(ms * 1e9 / length, 4),
+        "verify_phase_boundaries_us": verify_phases,
         "breakdown_ms": {"spec_exec": round(spec_med, 4),
                          "verify_recover": round(sorted(ver_ms)[len(ver_ms) // 2], 4)},
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",

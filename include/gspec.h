@@ -177,6 +177,11 @@ int fsm_get_qs(fsm_t fsm, uint8_t a, uint8_t b, uint32_t* qs, uint32_t* qs_len, 
 int fsm_get_records(fsm_t fsm, uint64_t nchunks, uint32_t* start, uint32_t* end, uint32_t* cnt, uint32_t* n_end,
                     uint32_t* n_oth, uint32_t* x);
 
+/* Phase timeline of the last collected run's verify/recover kernel (profiling):
+ * us[i] = microseconds since kernel start at phase boundary i (stage table,
+ * each relaxation pass, each recovery, finalize); up to 24 entries. */
+int fsm_get_phase_times(fsm_t fsm, double* us, uint32_t* n);
+
 void fsm_free(fsm_t fsm);
 const char* fsm_strerror(int status);
 const char* fsm_last_error(void);

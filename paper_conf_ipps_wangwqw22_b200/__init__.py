@@ -70,6 +70,7 @@ _lib.fsm_shard_finish.argtypes = [P, P, U32, U32, ctypes.POINTER(fsm_run_opts), 
 _lib.fsm_get_transform.argtypes = [P, P, P, P, P, P, P]
 _lib.fsm_get_qs.argtypes = [P, ctypes.c_uint8, ctypes.c_uint8, P, P, P]
 _lib.fsm_get_records.argtypes = [P, U64, P, P, P, P, P, P]
+_lib.fsm_get_phase_times.argtypes = [P, P, ctypes.POINTER(U32)]
 _lib.fsm_free.argtypes = [P]
 _lib.fsm_free.restype = None
 _lib.fsm_strerror.argtypes = [ctypes.c_int]
@@ -241,6 +242,13 @@ class FSM:
                "fsm_get_records")
         a.update(n_end=ne, n_oth=no, x=x)
         return a
+
+    def phase_times(self):
+        """Verify/recover phase boundaries (µs from kernel start) of the last collected run."""
+        us = np.zeros(24, np.float64)
+        n = U32(0)
+        _check(_lib.fsm_get_phase_times(self._h, us.ctypes.data, ctypes.byref(n)), "fsm_get_phase_times")
+        return us[:n.value].copy()
 
     def map_bytes(self) -> int:
         return int(_lib.fsm_map_bytes(self._h))

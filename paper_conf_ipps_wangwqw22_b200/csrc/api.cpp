@@ -162,7 +162,7 @@ void fill_result_stats(fsm_result* out, const Ctl& h) {
 // o.st; returns a ticket.  Everything (init, kernels, readback) is stream
 // ordered, so runs on one handle may be queued back to back.
 int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_scheme scheme, uint32_t q0t,
-                uint32_t* d_chunk_ends, uint64_t* ticket) {
+                uint32_t* d_chunk_ends, uint64_t* ticket, const uint32_t* q0_dev = nullptr) {
   const uint64_t N = (len + o.B - 1) / o.B;
   int rc = ensure_ctl(f);
   if (rc) return rc;
@@ -184,6 +184,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   rp.qs_cap = o.qs_cap;
   rp.vr_end = o.vr_end;
   rp.vr_oth = o.vr_oth;
+  rp.q0_dev = q0_dev;
   cudaEvent_t* ev = f->ev[slot];
   Ctl& h = f->h_ctl[slot];
   std::memset(&h, 0, sizeof(Ctl));
@@ -191,6 +192,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   h.tf = q0t;
   h.fmin = N;
   h.it_fm[0] = N;  // first relaxation pass slot
+  if (scheme == FSM_SCHEME_ENUM && q0_dev) scheme = FSM_SCHEME_SRE;  // device-resident start: pipeline path
   if (scheme == FSM_SCHEME_ENUM) {
     if (f->n + 1 > kEnumMax) {
       pd.active = false;
@@ -226,6 +228,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     rp.dense = (scheme == FSM_SCHEME_SRE && len / o.B > 0 && o.B % 64 == 0 &&
                 (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0 && f->acc1_hint < 0.5) ? 1u : 0u;
     CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
+    rp.ctl_init = nullptr;  // initialised by the spec kernel; later launches must not touch it
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
     for (;;) {
       CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
@@ -264,6 +267,8 @@ int run_collect(fsm_t f, uint64_t ticket, fsm_result* out, uint32_t* final_tid) 
   cudaEventElapsedTime(&t1, f->ev[slot][0], f->ev[slot][1]);
   cudaEventElapsedTime(&t2, f->ev[slot][1], f->ev[slot][2]);
   fill_result_stats(out, h);
+  f->last_nstamp = std::min<uint32_t>(h.nstamp, 24);
+  std::copy(h.stamp, h.stamp + 24, f->last_stamp);
   out->accept_count = h.accept_count;
   out->ms_spec = t1;
   out->ms_verify = t2;
@@ -703,6 +708,15 @@ int fsm_get_records(fsm_t f, uint64_t N, uint32_t* start, uint32_t* end, uint32_
   return FSM_OK;
 }
 
+int fsm_get_phase_times(fsm_t f, double* us, uint32_t* n) {
+  if (!f || !n) return fail(FSM_EINVAL, "NULL handle/n");
+  const uint32_t k = f->last_nstamp;
+  if (us)
+    for (uint32_t i = 0; i < k; i++) us[i] = (f->last_stamp[i] - f->last_stamp[0]) * 1e-3;
+  *n = k;
+  return FSM_OK;
+}
+
 uint64_t fsm_map_bytes(fsm_t f) {
   if (!f) return 0;
   const uint64_t nt = f->n + 1;
@@ -813,46 +827,58 @@ int fsm_shard_map(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* 
   unsigned long long* mcnt = reinterpret_cast<unsigned long long*>(reinterpret_cast<uint8_t*>(d_map) + map_cnt_off(nt));
   CUDA_TRY(launch_map_init(mend, mcnt, nt, o.st));
   // 1. candidate start states: the lookback image or q0 for the first shard
-  uint32_t ncand = 1;
-  if (lb_len == 0) {
-    CUDA_TRY(cudaMemcpyAsync(S.cand, &f->img.q0t, 4, cudaMemcpyHostToDevice, o.st));
-    f->shard_cand.assign(1, f->img.q0t);
-  } else {
-    CUDA_TRY(launch_shard_image(f->img, f->d_ttc, d_lookback, lb_len, S.mark, S.cand, S.info + 8, o.st));
-    CUDA_TRY(cudaMemcpyAsync(&ncand, S.info + 8, 4, cudaMemcpyDeviceToHost, o.st));
-    CUDA_TRY(cudaStreamSynchronize(o.st));
-    f->shard_cand.resize(ncand);
-    CUDA_TRY(cudaMemcpy(f->shard_cand.data(), S.cand, 4ull * ncand, cudaMemcpyDeviceToHost));
-  }
   f->shard_in = d_shard;
   f->shard_len = len;
-  f->shard_ncand = ncand;
   f->shard_nj = 0;
   f->shard_scheme = scheme;
-  f->shard_grp.assign(ncand, 0);
   f->shard_dist.clear();
+  uint32_t* d_ncand = S.info + 8;
+  uint32_t* d_unmerged = S.info + 9;
+  long long* dcnt = reinterpret_cast<long long*>(S.prefix);
+  if (lb_len == 0) {
+    CUDA_TRY(launch_set_u32(S.cand, f->img.q0t, d_ncand, 1, o.st));
+    CUDA_TRY(cudaMemsetAsync(S.grp, 0, 4, o.st));
+    CUDA_TRY(cudaMemsetAsync(dcnt, 0, 8, o.st));
+  } else {
+    CUDA_TRY(launch_shard_image(f->img, f->d_ttc, d_lookback, lb_len, S.mark, S.cand, d_ncand, o.st));
+  }
   // 2a. fast path: fuse every candidate with the path of cand[0] (P:427 path
-  // fusion); the shard then runs once, from cand[0], through the normal pipeline
-  if (ncand > 1 && N > 0 && len > 0) {
-    long long* dcnt = reinterpret_cast<long long*>(S.prefix);
-    CUDA_TRY(launch_shard_fuse_ref(f->img, d_shard, len, o.B, S.cand, ncand, kFuseChunks, S.states, S.grp, dcnt,
-                                   o.st));
-    f->shard_merged.resize(ncand);
-    CUDA_TRY(cudaMemcpyAsync(f->shard_merged.data(), S.grp, 4ull * ncand, cudaMemcpyDeviceToHost, o.st));
-    CUDA_TRY(cudaStreamSynchronize(o.st));
-    bool all = true;
-    for (uint32_t m : f->shard_merged) all &= m != kNoState;
-    if (all) {
-      fsm_result r;
-      uint32_t ft = 0;
-      rc = run_core(f, d_shard, len, o, scheme, f->shard_cand[0], d_chunk_ends_local, &r, &ft);
-      if (rc) return rc;
-      CUDA_TRY(launch_map_fused(S.cand, ncand, dcnt, ft, r.accept_count, mend, mcnt, o.st));
+  // fusion); the shard then runs once, from cand[0], through the normal pipeline.
+  // One host check (did every candidate merge?), the rest stays stream-ordered.
+  if (N > 0 && len > 0) {
+    uint32_t h2[2] = {1, 0};
+    if (lb_len != 0) {
+      CUDA_TRY(cudaMemsetAsync(d_unmerged, 0, 4, o.st));
+      CUDA_TRY(launch_shard_fuse_ref(f->img, d_shard, len, o.B, S.cand, d_ncand, kFuseChunks, S.states, S.grp, dcnt,
+                                     d_unmerged, o.st));
+      CUDA_TRY(cudaMemcpyAsync(h2, d_ncand, 8, cudaMemcpyDeviceToHost, o.st));
       CUDA_TRY(cudaStreamSynchronize(o.st));
+    }
+    f->shard_ncand = h2[0];
+    if (h2[1] == 0) {
+      if (f->shard_ticket) {  // a previous shard run that was never finished
+        fsm_result rr;
+        uint32_t ff;
+        run_collect(f, f->shard_ticket, &rr, &ff);
+        f->shard_ticket = 0;
+      }
+      if ((rc = run_enqueue(f, d_shard, len, o, scheme, f->img.q0t, d_chunk_ends_local, &f->shard_ticket, S.cand)))
+        return rc;
+      CUDA_TRY(launch_map_fused(S.cand, d_ncand, dcnt, &f->d_ctl->xfin,
+                                reinterpret_cast<const unsigned long long*>(&f->d_ctl->accept_count), mend, mcnt,
+                                o.st));
       f->shard_mode = 3;
       return FSM_OK;
     }
   }
+  // fallback: host-driven fusion / enumeration (candidate list needed on the host)
+  uint32_t ncand = 1;
+  CUDA_TRY(cudaMemcpyAsync(&ncand, d_ncand, 4, cudaMemcpyDeviceToHost, o.st));
+  CUDA_TRY(cudaStreamSynchronize(o.st));
+  f->shard_cand.resize(ncand);
+  CUDA_TRY(cudaMemcpy(f->shard_cand.data(), S.cand, 4ull * ncand, cudaMemcpyDeviceToHost));
+  f->shard_ncand = ncand;
+  f->shard_grp.assign(ncand, 0);
   std::vector<uint32_t> last(f->shard_cand);
   uint32_t nj = 0;
   bool merged = ncand == 1;
@@ -937,10 +963,26 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
   const uint32_t nt = f->n + 1;
   CUDA_TRY(launch_compose(reinterpret_cast<const uint8_t*>(d_maps), G, map_bytes_nt(nt), map_cnt_off(nt), f->img.q0t,
                           rank, f->d_small, o.st));
-  uint32_t h[5];
+  if (f->shard_mode == 3) {
+    // fused mode: this rank's chunk ends before the merge point are fixed on the device
+    ShardScratch S3;
+    if ((rc = ensure_shard(f, &S3))) return rc;
+    CUDA_TRY(cudaMemsetAsync(f->d_small + 5, 0, 4, o.st));
+    if (d_chunk_ends_local && f->shard_len)
+      CUDA_TRY(launch_fix_prefix_fused(S3.states, S3.cand, S3.info + 8, S3.grp, f->d_small, f->img.inv,
+                                       d_chunk_ends_local, f->d_small + 5, o.st));
+  }
+  uint32_t h[6] = {0, 0, 0, 0, 0, 0};
   CUDA_TRY(cudaMemcpyAsync(h, f->d_small, sizeof(h), cudaMemcpyDeviceToHost, o.st));
   CUDA_TRY(cudaStreamSynchronize(o.st));
-  if (h[2]) return fail(FSM_EINVAL, "a shard start state is outside its candidate set");
+  if (f->shard_mode == 3 && f->shard_ticket) {
+    fsm_result rr;
+    uint32_t ff;
+    rc = run_collect(f, f->shard_ticket, &rr, &ff);  // already complete: frees the ring slot
+    f->shard_ticket = 0;
+    if (rc) return rc;
+  }
+  if (h[2] || (f->shard_mode == 3 && h[5])) return fail(FSM_EINVAL, "a shard start state is outside its candidate set");
   const uint32_t srank = h[0], fin = h[1];
   const uint64_t count = (uint64_t)h[3] | ((uint64_t)h[4] << 32);
   const uint64_t N = (f->shard_len + o.B - 1) / o.B;
@@ -957,11 +999,7 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
       CUDA_TRY(launch_enum_full(f->img, rp, f->shard_E, f->enum_base, d_chunk_ends_local, f->d_ctl, f->d_small + 8,
                                 o.st, f->sm_count, 2));
     } else if (f->shard_mode == 3) {
-      auto it = std::find(f->shard_cand.begin(), f->shard_cand.end(), srank);
-      if (it == f->shard_cand.end()) return fail(FSM_EINVAL, "rank start not among its candidates");
-      const uint32_t ci = (uint32_t)(it - f->shard_cand.begin());
-      const uint32_t nj = f->shard_merged[ci];  // chunks walked before merging with cand[0]
-      if (nj) CUDA_TRY(launch_fix_prefix(S.states, f->shard_ncand, ci, nj, f->img.inv, d_chunk_ends_local, o.st));
+      (void)srank;  // located on the device
     } else {
       auto it = std::find(f->shard_cand.begin(), f->shard_cand.end(), srank);
       if (it == f->shard_cand.end()) return fail(FSM_EINVAL, "rank start not among its candidates");

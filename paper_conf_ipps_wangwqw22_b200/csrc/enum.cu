@@ -142,7 +142,7 @@ cudaError_t walk_t(const DevImage& img, const RunParams& rp, uint32_t E, uint64_
                    cudaStream_t st, int sms) {
   auto kern = k_enum_walk<MODE, NE>;
   const uint32_t smem = smem_bytes_for(img);
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = kernel_setup((const void*)kern, smem, 128, nullptr);
   if (e != cudaSuccess) return e;
   uint64_t grid = (nsub + 127) / 128;
   const uint64_t cap = (uint64_t)sms * 16;

@@ -95,6 +95,8 @@ struct Ctl {
   uint64_t ntask[2];     // (unused, kept for layout)
   uint64_t it_fm[3], it_checks[3], it_matches[3], it_ntask[3];  // per relaxation pass (rotating)
   uint32_t dense_pending;  // verify exited: a dense task round (frontier fmin) must run first
+  uint32_t nstamp;         // phase timestamps of the last verify launch (%globaltimer, ns)
+  uint64_t stamp[24];
   uint32_t pad2;
   uint32_t xfin;         // transformed final state (written by the last kernel of a run)
   uint32_t pad1;
@@ -112,27 +114,38 @@ struct RunParams {
   uint32_t vr_end, vr_oth;
   uint32_t dense;  // 1: hand rounds with many SRE tasks to the TMA task kernel (verify exits)
   Ctl* ctl_init;   // non-null: the first spec kernel initialises this control block (no H2D copy)
+  const uint32_t* q0_dev;  // non-null: chunk 0's start is read from the device (shard candidates)
 };
 
-// Host-side launch-config cache: sets the dynamic-smem attribute and queries
-// occupancy once per (kernel, smem, block) instead of on every launch.
+// Host-side launch-config cache: raises the kernel's dynamic-smem limit
+// (monotonically, so concurrent handles with different tables never lower it
+// under each other) and queries occupancy once per (kernel, smem, block).
 inline cudaError_t kernel_setup(const void* kern, uint32_t smem, int block, int* occ) {
-  struct Entry { uint32_t smem; int block; int occ; };
+  struct Key {
+    const void* k; uint32_t smem; int block;
+    bool operator<(const Key& o) const {
+      return k != o.k ? k < o.k : smem != o.smem ? smem < o.smem : block < o.block;
+    }
+  };
   static std::mutex mu;
-  static std::map<const void*, Entry> cache;
+  static std::map<Key, int> occ_cache;
+  static std::map<const void*, uint32_t> smem_max;
   std::lock_guard<std::mutex> g(mu);
-  auto it = cache.find(kern);
-  if (it != cache.end() && it->second.smem == smem && it->second.block == block) {
-    if (occ) *occ = it->second.occ;
-    return cudaSuccess;
+  uint32_t& mx = smem_max[kern];
+  if (smem > mx) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    mx = smem;
   }
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e != cudaSuccess) return e;
-  int o = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, block, smem);
-  if (e != cudaSuccess) return e;
-  cache[kern] = Entry{smem, block, o};
-  if (occ) *occ = o;
+  const Key key{kern, smem, block};
+  auto it = occ_cache.find(key);
+  if (it == occ_cache.end()) {
+    int o = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, kern, block, smem);
+    if (e != cudaSuccess) return e;
+    it = occ_cache.emplace(key, o).first;
+  }
+  if (occ) *occ = it->second;
   return cudaSuccess;
 }
 
@@ -175,10 +188,15 @@ cudaError_t launch_shard_fuse(const DevImage& img, const uint8_t* in, uint64_t l
                               uint32_t* info, cudaStream_t st);
 cudaError_t launch_map_init(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, cudaStream_t st);
 cudaError_t launch_shard_fuse_ref(const DevImage& img, const uint8_t* in, uint64_t len, uint32_t B,
-                                  const uint32_t* cand, uint32_t ncand, uint32_t max_chunks, uint32_t* states,
-                                  uint32_t* merged, long long* dcnt, cudaStream_t st);
-cudaError_t launch_map_fused(const uint32_t* cand, uint32_t ncand, const long long* dcnt, uint32_t fin,
-                             unsigned long long count0, uint32_t* mend, unsigned long long* mcnt, cudaStream_t st);
+                                  const uint32_t* cand, const uint32_t* ncand_p, uint32_t max_chunks, uint32_t* states,
+                                  uint32_t* merged, long long* dcnt, uint32_t* unmerged, cudaStream_t st);
+cudaError_t launch_map_fused(const uint32_t* cand, const uint32_t* ncand_p, const long long* dcnt, const uint32_t* fin_p,
+                             const unsigned long long* count_p, uint32_t* mend, unsigned long long* mcnt,
+                             cudaStream_t st);
+cudaError_t launch_fix_prefix_fused(const uint32_t* states, const uint32_t* cand, const uint32_t* ncand_p,
+                                    const uint32_t* merged, const uint32_t* srank_p, const uint32_t* inv,
+                                    uint32_t* chunk_ends, uint32_t* err, cudaStream_t st);
+cudaError_t launch_set_u32(uint32_t* p, uint32_t v, uint32_t* p2, uint32_t v2, cudaStream_t st);
 cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_t* grp,
                              const unsigned long long* prefix, const uint32_t* pfinal, const unsigned long long* pcount,
                              uint32_t* mend, unsigned long long* mcnt, cudaStream_t st);
@@ -244,7 +262,9 @@ struct fsm_s {
   void* shard_base = nullptr;   // device scratch of the shard steps
   size_t shard_bytes = 0;
   int shard_mode = -1;          // 0 fused/single path, 1 enum, 2 multi-path, 3 fused with cand[0]
-  std::vector<uint32_t> shard_merged;  // mode 3: chunk where candidate i merged with cand[0]
+  uint64_t shard_ticket = 0;
+  uint32_t last_nstamp = 0;            // verify phase timestamps of the last collected run
+  uint64_t last_stamp[24] = {};           // mode 3: the pending cand[0] pipeline run
   const uint8_t* shard_in = nullptr;
   uint64_t shard_len = 0;
   uint32_t shard_ncand = 0, shard_nj = 0;  // candidates; chunks covered by the fused prefix

@@ -101,13 +101,16 @@ __global__ void __launch_bounds__(1024) k_fuse(DevImage img, const uint8_t* __re
 // own state at the end of chunk j for chunks before the merge.
 template <int MODE>
 __global__ void __launch_bounds__(1024) k_fuse_ref(DevImage img, const uint8_t* __restrict__ in, uint64_t len,
-                                                   uint32_t B, const uint32_t* __restrict__ cand, uint32_t ncand,
-                                                   uint32_t max_chunks, uint32_t* __restrict__ states,
-                                                   uint32_t* __restrict__ merged, long long* __restrict__ dcnt) {
+                                                   uint32_t B, const uint32_t* __restrict__ cand,
+                                                   const uint32_t* __restrict__ ncand_p, uint32_t max_chunks,
+                                                   uint32_t* __restrict__ states, uint32_t* __restrict__ merged,
+                                                   long long* __restrict__ dcnt, uint32_t* __restrict__ unmerged) {
   extern __shared__ __align__(1024) uint8_t smem[];
   stage_table(img, smem);
   __syncthreads();
   using S = Step<MODE>;
+  const uint32_t ncand = *ncand_p;
+  uint32_t um = 0;
   for (uint32_t i = threadIdx.x; i < ncand; i += blockDim.x) {
     uint32_t code = __ldg(img.tid2code + cand[i]), rcode = __ldg(img.tid2code + cand[0]);
     long long d = 0;
@@ -135,17 +138,50 @@ __global__ void __launch_bounds__(1024) k_fuse_ref(DevImage img, const uint8_t* 
     }
     merged[i] = mj;
     dcnt[i] = d;
+    um += mj == kNoState;
+  }
+  if (um) atomicAdd(unmerged, um);
+}
+
+// map[cand[i]] = (final of the cand[0] pipeline, its count + dcnt[i]); the pipeline's
+// final state and count are read from its control block on the device
+__global__ void k_map_fused(const uint32_t* __restrict__ cand, const uint32_t* __restrict__ ncand_p,
+                            const long long* __restrict__ dcnt, const uint32_t* __restrict__ fin_p,
+                            const unsigned long long* __restrict__ count_p, uint32_t* __restrict__ mend,
+                            unsigned long long* __restrict__ mcnt) {
+  const uint32_t ncand = *ncand_p;
+  const uint32_t fin = *fin_p;
+  const unsigned long long c0 = *count_p;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x) {
+    mend[cand[i]] = fin;
+    mcnt[cand[i]] = (unsigned long long)((long long)c0 + dcnt[i]);
   }
 }
 
-// map[cand[i]] = (final, count0 + dcnt[i]) for candidates fused with cand[0]
-__global__ void k_map_fused(const uint32_t* __restrict__ cand, uint32_t ncand, const long long* __restrict__ dcnt,
-                            uint32_t fin, unsigned long long count0, uint32_t* __restrict__ mend,
-                            unsigned long long* __restrict__ mcnt) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x) {
-    mend[cand[i]] = fin;
-    mcnt[cand[i]] = (unsigned long long)((long long)count0 + dcnt[i]);
+// finish (fused mode): locate this rank's start among the candidates and write
+// the chunk ends walked before it merged with the reference path
+__global__ void k_fix_prefix_fused(const uint32_t* __restrict__ states, const uint32_t* __restrict__ cand,
+                                   const uint32_t* __restrict__ ncand_p, const uint32_t* __restrict__ merged,
+                                   const uint32_t* __restrict__ srank_p, const uint32_t* __restrict__ inv,
+                                   uint32_t* __restrict__ chunk_ends, uint32_t* __restrict__ err) {
+  __shared__ uint32_t ci;
+  const uint32_t ncand = *ncand_p, sr = *srank_p;
+  if (threadIdx.x == 0) ci = kNoState;
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < ncand; i += blockDim.x)
+    if (cand[i] == sr) atomicMin(&ci, i);
+  __syncthreads();
+  if (ci == kNoState) {
+    if (threadIdx.x == 0) *err = 1;
+    return;
   }
+  const uint32_t nj = merged[ci];
+  for (uint32_t j = threadIdx.x; j < nj; j += blockDim.x) chunk_ends[j] = inv[states[(uint64_t)j * ncand + ci]];
+}
+
+__global__ void k_set_u32(uint32_t* p, uint32_t v, uint32_t* p2, uint32_t v2) {
+  *p = v;
+  if (p2) *p2 = v2;
 }
 
 __global__ void k_map_init(uint32_t* __restrict__ mend, unsigned long long* __restrict__ mcnt, uint32_t nt) {
@@ -209,7 +245,7 @@ cudaError_t fuse_m(const DevImage& img, const uint8_t* in, uint64_t len, uint32_
                    cudaStream_t st) {
   auto kern = k_fuse<MODE>;
   const uint32_t smem = smem_bytes_for(img);
-  cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = kernel_setup((const void*)kern, smem, 1024, nullptr);
   if (e != cudaSuccess) return e;
   const uint32_t th = ((ncand + 31) / 32) * 32;
   kern<<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info);
@@ -236,35 +272,39 @@ cudaError_t launch_shard_fuse(const DevImage& img, const uint8_t* in, uint64_t l
 }
 
 cudaError_t launch_shard_fuse_ref(const DevImage& img, const uint8_t* in, uint64_t len, uint32_t B,
-                                  const uint32_t* cand, uint32_t ncand, uint32_t max_chunks, uint32_t* states,
-                                  uint32_t* merged, long long* dcnt, cudaStream_t st) {
+                                  const uint32_t* cand, const uint32_t* ncand_p, uint32_t max_chunks, uint32_t* states,
+                                  uint32_t* merged, long long* dcnt, uint32_t* unmerged, cudaStream_t st) {
   const uint32_t smem = smem_bytes_for(img);
-  const uint32_t th = std::min<uint32_t>(1024, ((ncand + 31) / 32) * 32);
   cudaError_t e;
+#define GS_FUSE_REF(M)                                                                                        \
+  if ((e = kernel_setup((const void*)k_fuse_ref<M>, smem, 1024, nullptr))) return e;                          \
+  k_fuse_ref<M><<<1, 1024, smem, st>>>(img, in, len, B, cand, ncand_p, max_chunks, states, merged, dcnt, unmerged)
   switch (img.mode) {
-    case MODE_U8:
-      if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
-      k_fuse_ref<MODE_U8><<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, merged, dcnt);
-      break;
-    case MODE_U16:
-      if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
-      k_fuse_ref<MODE_U16><<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, merged, dcnt);
-      break;
-    case MODE_U16H:
-      if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U16H>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
-      k_fuse_ref<MODE_U16H><<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, merged, dcnt);
-      break;
-    default:
-      if ((e = cudaFuncSetAttribute(k_fuse_ref<MODE_U32>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem))) return e;
-      k_fuse_ref<MODE_U32><<<1, th, smem, st>>>(img, in, len, B, cand, ncand, max_chunks, states, merged, dcnt);
-      break;
+    case MODE_U8: GS_FUSE_REF(MODE_U8); break;
+    case MODE_U16: GS_FUSE_REF(MODE_U16); break;
+    case MODE_U16H: GS_FUSE_REF(MODE_U16H); break;
+    default: GS_FUSE_REF(MODE_U32); break;
   }
+#undef GS_FUSE_REF
   return cudaGetLastError();
 }
 
-cudaError_t launch_map_fused(const uint32_t* cand, uint32_t ncand, const long long* dcnt, uint32_t fin,
-                             unsigned long long count0, uint32_t* mend, unsigned long long* mcnt, cudaStream_t st) {
-  k_map_fused<<<(ncand + 255) / 256, 256, 0, st>>>(cand, ncand, dcnt, fin, count0, mend, mcnt);
+cudaError_t launch_map_fused(const uint32_t* cand, const uint32_t* ncand_p, const long long* dcnt, const uint32_t* fin_p,
+                             const unsigned long long* count_p, uint32_t* mend, unsigned long long* mcnt,
+                             cudaStream_t st) {
+  k_map_fused<<<8, 256, 0, st>>>(cand, ncand_p, dcnt, fin_p, count_p, mend, mcnt);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_fix_prefix_fused(const uint32_t* states, const uint32_t* cand, const uint32_t* ncand_p,
+                                    const uint32_t* merged, const uint32_t* srank_p, const uint32_t* inv,
+                                    uint32_t* chunk_ends, uint32_t* err, cudaStream_t st) {
+  k_fix_prefix_fused<<<1, 256, 0, st>>>(states, cand, ncand_p, merged, srank_p, inv, chunk_ends, err);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_set_u32(uint32_t* p, uint32_t v, uint32_t* p2, uint32_t v2, cudaStream_t st) {
+  k_set_u32<<<1, 1, 0, st>>>(p, v, p2, v2);
   return cudaGetLastError();
 }
 

@@ -30,7 +30,7 @@ template <int MODE, int NI, int KP>
 __global__ void __launch_bounds__(256) k_spec_exec(DevImage img, RunParams rp, RecStore rs, uint64_t c0) {
   extern __shared__ __align__(1024) uint8_t smem[];
   stage_table(img, smem);
-  if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, rp.q0t, rp.N);
+  if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, q0_of(rp), rp.N);
   __syncthreads();
   using S = Step<MODE>;
   const uint64_t N = rp.N, B = rp.B, len = rp.len;
@@ -49,7 +49,7 @@ __global__ void __launch_bounds__(256) k_spec_exec(DevImage img, RunParams rp, R
       if (!valid || c[i] == 0) {
         kc[i] = 1;
 #pragma unroll
-        for (int p = 0; p < KP; p++) st[i][p] = rp.q0t;
+        for (int p = 0; p < KP; p++) st[i][p] = q0_of(rp);
       } else {
         const uint32_t pair = qs_pair(img, rp.in, c[i], rp.B);
         const uint32_t ql = __ldg(img.qs2_len + pair);
@@ -133,7 +133,7 @@ __global__ void __launch_bounds__(256) k_spec_exec(DevImage img, RunParams rp, R
       rs.ref_cnt[cc] = acc[i][0];
       rs.x[cc + 1] = e0;
       rs.cur_end[cc] = e0;
-      if (cc == 0) rs.x[0] = rp.q0t;
+      if (cc == 0) rs.x[0] = q0_of(rp);
     }
   }
 }

@@ -77,7 +77,7 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   uint8_t* stages = smem_raw + table_off;
   uint64_t* bars = reinterpret_cast<uint64_t*>(stages + (size_t)nwarps * S * kStageBytes);
   stage_table(img, table);
-  if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, rp.q0t, rp.N);
+  if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, q0_of(rp), rp.N);
   if (lane == 0)
     for (int s = 0; s < S; s++) mbar_init(bars + warp * S + s, 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -120,11 +120,11 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
         const uint32_t ts = (c < n_full && c >= f2) ? __ldcg(rs.tstart + c) : 0xFFFFFFFFu;
         kc = ts != 0xFFFFFFFFu;  // 0: no task for this lane (walks the bytes, writes nothing)
 #pragma unroll
-        for (int p = 0; p < KP; p++) st[p] = kc ? ts : rp.q0t;
+        for (int p = 0; p < KP; p++) st[p] = kc ? ts : q0_of(rp);
       } else if (c == 0 || c >= n_full) {
         kc = 1;
 #pragma unroll
-        for (int p = 0; p < KP; p++) st[p] = rp.q0t;
+        for (int p = 0; p < KP; p++) st[p] = q0_of(rp);
       } else {
         const uint32_t pair = qs_pair(img, rp.in, c, rp.B);
         const uint32_t ql = __ldg(img.qs2_len + pair);
@@ -190,7 +190,7 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
       rs.ref_cnt[c] = acc[0];
       rs.x[c + 1] = e0;
       rs.cur_end[c] = e0;
-      if (c == 0) rs.x[0] = rp.q0t;
+      if (c == 0) rs.x[0] = q0_of(rp);
     }
     if (++sg == segs) { sg = 0; tile_i++; }
     if (++s == (uint32_t)S) { s = 0; phase ^= 1u; }

@@ -213,6 +213,12 @@ __device__ void task_walk(const DevImage& img, const uint8_t* smem, const RunPar
   *cnt_out = acc;
 }
 
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
 template <int MODE>
 __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
                                                         uint64_t* btmp, uint32_t* chunk_ends, uint32_t cache_cap) {
@@ -222,8 +228,14 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   __shared__ uint64_t red64[kBS / 32];
   __shared__ uint64_t sh_pre[3];
   __shared__ uint64_t sh_tot[3];
+  uint32_t nst = 0;
+  auto stamp = [&]() {
+    if (blockIdx.x == 0 && threadIdx.x == 0 && nst < 24) { ctl->stamp[nst++] = gtimer(); ctl->nstamp = nst; }
+  };
+  stamp();
   stage_table(img, smem);
   __syncthreads();
+  stamp();
 
   const uint64_t N = rp.N;
   const uint32_t G = gridDim.x, b = blockIdx.x;
@@ -319,6 +331,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
           atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_matches[slot]), (unsigned long long)matches);
       }
       grid.sync();
+      stamp();
       const bool any = vctl->changed[slot] != 0;
       it++;
       git++;
@@ -383,6 +396,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         }
       }
       grid.sync();
+      stamp();
       continue;
     }
     // ---------------- T: per-block counts of A-tasks and untried candidates -----
@@ -580,6 +594,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     total = block_sum<uint64_t>(total, red64);
     if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->accept_count), (unsigned long long)total);
     if (b == 0 && threadIdx.x == 0) ctl->xfin = ld_cg(rs.x + N);
+    stamp();
   }
 }
 
@@ -670,8 +685,10 @@ cudaError_t launch_dense_finish(const DevImage& img, const RunParams& rp, const 
 cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
                             int sms, cudaStream_t st, uint64_t* n_done);
 
-cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
+cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp_in, const RecStore& rs, Ctl* ctl, uint64_t f2,
                               int sms, cudaStream_t st) {
+  RunParams rp = rp_in;
+  rp.ctl_init = nullptr;  // the control block is live: never re-initialise it mid-run
   uint64_t done = 0;
   cudaError_t e = launch_task_tma(img, rp, rs, ctl, f2, sms, st, &done);
   if (e == cudaErrorNotSupported) {

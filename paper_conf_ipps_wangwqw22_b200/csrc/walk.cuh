@@ -190,6 +190,9 @@ __device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, u
   return false;
 }
 
+// Chunk 0's start state (a shard's reference candidate may live on the device).
+__device__ __forceinline__ uint32_t q0_of(const RunParams& rp) { return rp.q0_dev ? __ldcg(rp.q0_dev) : rp.q0t; }
+
 // Initialise the verify/recover control block for a run (block 0 of the first kernel).
 __device__ __forceinline__ void init_ctl(Ctl* ctl, uint32_t q0t, uint64_t N) {
   uint32_t* w = reinterpret_cast<uint32_t*>(ctl);

@@ -16,3 +16,4 @@ for i in range(reps):
     r = fsm.run(x, scheme=scheme)
 torch.cuda.synchronize()
 print(r.final_state, r.accept_count, r.stats['ms_spec'], r.stats['ms_verify'])
+print("verify phase times (us):", [round(v, 1) for v in fsm.phase_times()])
