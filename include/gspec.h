@@ -162,6 +162,19 @@ int fsm_shard_map(fsm_t fsm, const uint8_t* d_shard, uint64_t len, const uint8_t
 int fsm_shard_finish(fsm_t fsm, const void* d_maps, uint32_t nranks, uint32_t rank,
                      const fsm_run_opts* opts, uint32_t* d_chunk_ends_local, fsm_result* out_global);
 
+/* ---- library-owned NCCL path (callers without torch.distributed) -------------
+ * fsm_comm_unique_id (one rank, 128 bytes, share out of band) -> fsm_comm_init
+ * on every rank (one GPU each) -> fsm_run_sharded = fsm_shard_map + one
+ * ncclAllGather of the maps on opts->stream + fsm_shard_finish.  NCCL is
+ * loaded at run time (libnccl.so.2); FSM_ENCCL if it is missing or fails. */
+typedef struct fsm_comm_s* fsm_comm_t;
+int fsm_comm_unique_id(void* id_out);
+int fsm_comm_init(int nranks, int rank, const void* unique_id, fsm_comm_t* out);
+int fsm_run_sharded(fsm_t fsm, fsm_comm_t comm, const uint8_t* d_shard, uint64_t shard_len,
+                    const uint8_t* d_lookback, uint32_t lookback_len, const fsm_run_opts* opts,
+                    uint32_t* d_chunk_ends_local, fsm_result* out_global);
+void fsm_comm_free(fsm_comm_t comm);
+
 /* ---- introspection (tests) ------------------------------------------------- */
 /* perm/inv: host uint32 [nstates+1] (poison = nstates last); freq: uint64
  * [nstates]; mode/H/C: table format, hot rows, classes. Any pointer nullable. */

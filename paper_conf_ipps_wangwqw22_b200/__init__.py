@@ -71,6 +71,11 @@ _lib.fsm_get_transform.argtypes = [P, P, P, P, P, P, P]
 _lib.fsm_get_qs.argtypes = [P, ctypes.c_uint8, ctypes.c_uint8, P, P, P]
 _lib.fsm_get_records.argtypes = [P, U64, P, P, P, P, P, P]
 _lib.fsm_get_phase_times.argtypes = [P, P, ctypes.POINTER(U32)]
+_lib.fsm_comm_unique_id.argtypes = [P]
+_lib.fsm_comm_init.argtypes = [ctypes.c_int, ctypes.c_int, P, ctypes.POINTER(P)]
+_lib.fsm_run_sharded.argtypes = [P, P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
+_lib.fsm_comm_free.argtypes = [P]
+_lib.fsm_comm_free.restype = None
 _lib.fsm_free.argtypes = [P]
 _lib.fsm_free.restype = None
 _lib.fsm_strerror.argtypes = [ctypes.c_int]
@@ -256,6 +261,50 @@ class FSM:
     @property
     def handle(self):
         return self._h
+
+
+class Comm:
+    """Library-owned NCCL communicator (fsm_comm_init); one per rank / GPU."""
+
+    def __init__(self, nranks: int, rank: int, unique_id: bytes):
+        h = P()
+        buf = ctypes.create_string_buffer(bytes(unique_id), 128)
+        _check(_lib.fsm_comm_init(nranks, rank, buf, ctypes.byref(h)), "fsm_comm_init")
+        self._h = h.value
+        self.nranks, self.rank = nranks, rank
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = ctypes.create_string_buffer(128)
+        _check(_lib.fsm_comm_unique_id(buf), "fsm_comm_unique_id")
+        return buf.raw
+
+    def run_sharded(self, fsm: "FSM", shard, lookback=None, scheme="auto", chunk_bytes=4096, spec_k=4,
+                    chunk_ends=True, stream=None) -> Result:
+        """fsm_run_sharded: shard map + one ncclAllGather + finish, all inside the library."""
+        import torch
+
+        o = _run_opts(scheme, chunk_bytes, spec_k, stream=stream)
+        n = fsm_num_chunks(shard.numel(), chunk_bytes)
+        ce = torch.empty(max(n, 1), dtype=torch.int32, device=shard.device) if chunk_ends else None
+        lb = lookback if lookback is not None and lookback.numel() else None
+        r = fsm_result()
+        _check(_lib.fsm_run_sharded(fsm.handle, self._h, shard.data_ptr() if shard.numel() else None, shard.numel(),
+                                    lb.data_ptr() if lb is not None else None, lb.numel() if lb is not None else 0,
+                                    ctypes.byref(o), ce.data_ptr() if ce is not None else None, ctypes.byref(r)),
+               "fsm_run_sharded")
+        return Result.from_c(r, ce[:n] if ce is not None else None)
+
+    def close(self):
+        if self._h:
+            _lib.fsm_comm_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 # C-ABI names (same entry points, argument marshalling only)

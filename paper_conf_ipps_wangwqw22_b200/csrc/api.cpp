@@ -297,6 +297,8 @@ fsm_scheme tree_select(const fsm_features& ft, uint32_t n) {
 
 extern "C" {
 
+int gspec_set_error(int code, const char* msg) { return fail(code, msg); }
+
 const char* fsm_last_error(void) { return g_err.c_str(); }
 
 const char* fsm_strerror(int s) {

@@ -122,3 +122,16 @@ def test_c5_16gib_shard_invariance(gs):
     h = w.host(0, 1 << 30)
     ref = oracle.run(w.table, w.start, w.accept, h, 4096)
     assert (ce_single[:len(ref["chunk_end"])] == ref["chunk_end"]).all()
+
+
+def test_library_nccl_single_rank(gs):
+    """fsm_comm_init + fsm_run_sharded with a real (1-rank) NCCL communicator."""
+    w = gen.workload("c2", length=8 << 20)
+    data = w.host()
+    ref = oracle.run(w.table, w.start, w.accept, data, 4096)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    comm = gs.Comm(1, 0, gs.Comm.unique_id())
+    r = comm.run_sharded(fsm, torch.from_numpy(data).cuda())
+    assert r.final_state == ref["final"] and r.accept_count == ref["count"]
+    assert (r.chunk_ends.cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
+    comm.close()
