@@ -221,6 +221,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     if (f->rs_cap < N) CUDA_TRY(cudaStreamSynchronize(o.st));  // growing the store: drain queued runs
     if ((rc = ensure_records(f, N))) return rc;
     rp.ctl_init = f->d_ctl;  // the spec kernel initialises the control block
+    rp.h_out = &h;           // ... and the verify kernel's finalize step writes it back (pinned, UVA)
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
     // dense recovery rounds go to the TMA task kernel (SRE on low-accuracy DFAs); this
     // needs a host check per verify launch, so it is off when the profile says the
@@ -243,7 +244,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     }
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   }
-  CUDA_TRY(cudaMemcpyAsync(&h, f->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, o.st));
+  if (!rp.h_out) CUDA_TRY(cudaMemcpyAsync(&h, f->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, o.st));
   CUDA_TRY(cudaEventRecord(ev[3], o.st));
   return FSM_OK;
 }

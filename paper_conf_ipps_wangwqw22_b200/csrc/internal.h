@@ -97,7 +97,7 @@ struct Ctl {
   uint32_t dense_pending;  // verify exited: a dense task round (frontier fmin) must run first
   uint32_t nstamp;         // phase timestamps of the last verify launch (%globaltimer, ns)
   uint64_t stamp[24];
-  uint32_t pad2;
+  uint32_t zdone;        // finalize tickets (the last CTA publishes the block to h_out)
   uint32_t xfin;         // transformed final state (written by the last kernel of a run)
   uint32_t pad1;
 };
@@ -115,6 +115,7 @@ struct RunParams {
   uint32_t dense;  // 1: hand rounds with many SRE tasks to the TMA task kernel (verify exits)
   Ctl* ctl_init;   // non-null: the first spec kernel initialises this control block (no H2D copy)
   const uint32_t* q0_dev;  // non-null: chunk 0's start is read from the device (shard candidates)
+  Ctl* h_out;      // non-null: pinned host slot; the finalize step writes the control block there
 };
 
 // Host-side launch-config cache: raises the kernel's dynamic-smem limit

@@ -632,6 +632,22 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->accept_count), (unsigned long long)total);
     if (b == 0 && threadIdx.x == 0) ctl->xfin = ld_cg(rs.x + N);
     stamp();
+    if (rp.h_out) {
+      // zero-copy result: the last CTA to finish publishes the control block to the
+      // pinned host slot (no device-to-host copy on the stream)
+      __shared__ uint32_t last;
+      if (threadIdx.x == 0) {
+        __threadfence();
+        last = atomicAdd(&ctl->zdone, 1u) == G - 1;
+      }
+      __syncthreads();
+      if (last) {
+        __threadfence();
+        const uint32_t* src = reinterpret_cast<const uint32_t*>(ctl);
+        uint32_t* dst = reinterpret_cast<uint32_t*>(rp.h_out);
+        for (uint32_t i = threadIdx.x; i < sizeof(Ctl) / 4; i += kBS) dst[i] = __ldcg(src + i);
+      }
+    }
   }
 }
 
