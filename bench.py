@@ -199,7 +199,12 @@ def main():
     B = args.chunk_bytes
     x = torch.empty(length, dtype=torch.uint8, device="cuda")
     w.device(x, offset=rank * length)  # weak scaling: rank r owns bytes [r*len, (r+1)*len)
-    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    # profile sample (a 1 MiB "training" trace): a disjoint slice of the same
+    # source, past every rank's shard; it places the u8 table rows bank-aware
+    prof = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")
+    w.device(prof, offset=world * length)
+    fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof.cpu().numpy())
+    del prof
     stream = torch.cuda.current_stream()
     scheme = args.scheme
     feats = None

@@ -56,7 +56,10 @@ typedef struct fsm_s* fsm_t;
 
 typedef struct {
   uint32_t freq_policy;          /* 0 = static in-degree (Fig. 4), 1 = profile visits */
-  const uint8_t* profile_sample; /* host bytes for freq_policy 1 (copied during the call)    */
+  const uint8_t* profile_sample; /* host bytes (read during the call only): freq_policy 1
+                                    ranks states by their visits on it; with any policy the
+                                    u8 format also places table rows bank-aware from it
+                                    (layout only, results unchanged); NULL = no profile    */
   uint64_t profile_len;
   uint32_t smem_budget_bytes;    /* hot-row budget in shared memory; 0 = auto        */
   uint32_t force_mode;           /* 0 auto; 1 u8 raw-byte table; 2 u16 classed; 3 u32 classed */

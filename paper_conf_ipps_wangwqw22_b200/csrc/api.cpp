@@ -53,6 +53,55 @@ int upload(fsm_t f, const T** dst, const std::vector<T>& v, size_t pad_bytes = 0
   return FSM_OK;
 }
 
+constexpr uint32_t kRow8Bytes = 260;  // walk.cuh kRow8: row r starts at bank (r * 65) % 32 = r % 32
+
+// MODE_U8 row placement from a profile sample (an extension of the transformation,
+// DESIGN.md §5.1): the lanes of a warp walk different chunks, so one warp-wide
+// lookup reads up to 32 rows; two lanes conflict when their (row, byte) words
+// fall in one bank.  Rows of frequently visited states are given codes (row
+// numbers, accept flag in bit 7) whose bank rotation keeps their hot words off
+// the banks already loaded by hotter rows: greedy over states by visits, cost =
+// sum over the state's word histogram of the bank load so far.  Codes are
+// drawn from [0, n_na + 32) and [128, 128 + n_acc + 32) so every rotation is
+// available at a bounded table size.  Purely a layout choice: tids, the
+// transformation and all results are unchanged.
+void place_rows_bank_aware(fsm_t f, const std::vector<uint32_t>& ttc, uint32_t C, const std::vector<uint8_t>& acc_t,
+                           uint32_t n_na, uint32_t n_acc, const uint8_t* sample, uint64_t len,
+                           std::vector<uint32_t>& tid2code, std::vector<uint32_t>& code2tid) {
+  const uint32_t nt = f->n + 1, P = f->n;
+  std::vector<double> visits(nt, 0.0), hist((size_t)nt * 64, 0.0);
+  uint32_t t = f->perm[f->q0];
+  for (uint64_t i = 0; i < len; i++) {
+    const uint8_t b = sample[i];
+    visits[t] += 1;
+    hist[(size_t)t * 64 + (b >> 2)] += 1;
+    t = t == P ? P : ttc[(uint64_t)t * C + f->cls[b]];
+  }
+  std::vector<uint32_t> order(nt);
+  std::iota(order.begin(), order.end(), 0u);
+  std::stable_sort(order.begin(), order.end(), [&](uint32_t a, uint32_t b) { return visits[a] > visits[b]; });
+  std::vector<uint8_t> used(256, 0);
+  const uint32_t lim_na = std::min(128u, n_na + 32), lim_acc = std::min(256u, 128 + n_acc + 32);
+  double load[32] = {0};
+  for (uint32_t q : order) {
+    const uint32_t lo = acc_t[q] ? 128 : 0, hi = acc_t[q] ? lim_acc : lim_na;
+    uint32_t best = 256;
+    double best_cost = 0;
+    for (uint32_t c = lo; c < hi; c++) {
+      if (used[c]) continue;
+      double cost = 0;
+      if (visits[q] > 0)
+        for (uint32_t w = 0; w < 64; w++) cost += hist[(size_t)q * 64 + w] * load[(w + c) % 32];
+      if (best == 256 || cost < best_cost) { best = c; best_cost = cost; }
+      if (visits[q] == 0) break;  // never visited: first free code
+    }
+    used[best] = 1;
+    tid2code[q] = best;
+    code2tid[best] = q;
+    for (uint32_t w = 0; w < 64; w++) load[(w + best) % 32] += hist[(size_t)q * 64 + w];
+  }
+}
+
 struct Opts {
   fsm_scheme scheme;
   uint32_t B, k, L, qs_cap, vr_end, vr_oth;
@@ -431,20 +480,27 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
   img.q0t = f->perm[start];
   std::vector<uint32_t> tid2code(nt), code2tid(256, P);
   if (mode == MODE_U8) {
-    uint32_t na = 0, ac = 0;
-    for (uint32_t t = 0; t < nt; t++) {
-      const uint32_t code = acc_t[t] ? 128 + ac++ : na++;
-      tid2code[t] = code;
-      code2tid[code] = t;
+    uint32_t max_code = 0;
+    if (opts && opts->profile_sample && opts->profile_len) {
+      place_rows_bank_aware(f, ttc, C, acc_t, n_na, n_acc, opts->profile_sample, opts->profile_len, tid2code,
+                            code2tid);
+    } else {
+      uint32_t na = 0, ac = 0;
+      for (uint32_t t = 0; t < nt; t++) {
+        const uint32_t code = acc_t[t] ? 128 + ac++ : na++;
+        tid2code[t] = code;
+        code2tid[code] = t;
+      }
     }
-    const uint32_t R = 260;  // row stride (walk.cuh kRow8): 4-byte pad rotates rows across banks
+    for (uint32_t t = 0; t < nt; t++) max_code = std::max(max_code, tid2code[t]);
+    const uint32_t R = kRow8Bytes;  // row stride (walk.cuh kRow8): 4-byte pad rotates rows across banks
     std::vector<uint8_t> T8(256 * R, (uint8_t)tid2code[P]);
     for (uint32_t code = 0; code < 256; code++) {
       const uint32_t t = code2tid[code];
       for (uint32_t b = 0; b < 256; b++) T8[code * R + b] = (uint8_t)tid2code[ttc[(uint64_t)t * C + f->cls[b]]];
     }
     img.H = nt;
-    img.smem_table_bytes = (((n_acc > 0 ? 128 + n_acc : n_na) * R) + 15) & ~15u;
+    img.smem_table_bytes = (((max_code + 1) * R) + 15) & ~15u;
     if ((rc = upload(f, &img.T8, T8))) return bail(rc);
   } else {
     const uint32_t shift = mode == MODE_U16 ? 15 : 31;

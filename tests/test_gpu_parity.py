@@ -169,6 +169,26 @@ def test_policies_and_transform(gs, policy):
     check_equal(res, ref, 4096, w.nstates)
 
 
+@pytest.mark.parametrize("name", ["c1", "c2", "rand:200:256:7", "rand:120:97:8"])
+def test_bank_aware_row_placement(gs, name):
+    """A profile sample with freq_policy 0 only moves u8 rows (codes); tids and every
+    result stay those of the plain load."""
+    w, data = _wl(name, 3 << 20, 7 if name.startswith("rand") else None)
+    ref = oracle.run(w.table, w.start, w.accept, data, 4096)
+    prof = gen.workload(name, length=1 << 20, seed=99).host()  # disjoint "training" trace
+    plain = gs.FSM.load(w.table, w.start, w.accept)
+    fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof)
+    tp, tr = plain.transform(), fsm.transform()
+    assert tr["mode"] == "u8"
+    assert (tp["perm"] == tr["perm"]).all() and (tp["inv"] == tr["inv"]).all()
+    x = torch.from_numpy(data).cuda()
+    for scheme in SCHEMES:
+        res = fsm.run(x, scheme=scheme)
+        check_equal(res, ref, 4096, w.nstates)
+        assert res.stats == plain.run(x, scheme=scheme).stats | {"ms_spec": res.stats["ms_spec"],
+                                                               "ms_verify": res.stats["ms_verify"]}
+
+
 def test_lookback_table_matches_oracle(gs):
     for name in ("c2", "c3", "c1"):
         w, data = _wl(name, 1 << 16)
