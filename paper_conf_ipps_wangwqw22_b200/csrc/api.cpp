@@ -218,7 +218,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   const uint64_t seq = f->next_seq++;
   const uint32_t slot = (uint32_t)(seq % fsm_s::kRing);
   auto& pd = f->pend[slot];
-  if (pd.active) CUDA_TRY(cudaEventSynchronize(f->ev[slot][3]));  // ring wrapped: slot's readback must be done
+  if (pd.active) CUDA_TRY(cudaEventSynchronize(f->ev[slot][pd.done_ev]));  // ring wrapped: slot's readback must be done
   pd = fsm_s::Pending{seq, N, scheme, q0t, true};
   *ticket = seq;
   if (N == 0) return FSM_OK;
@@ -293,8 +293,12 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     }
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   }
-  if (!rp.h_out) CUDA_TRY(cudaMemcpyAsync(&h, f->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, o.st));
-  CUDA_TRY(cudaEventRecord(ev[3], o.st));
+  if (rp.h_out) {
+    pd.done_ev = 2;  // the verify kernel wrote the result to the pinned slot
+  } else {
+    CUDA_TRY(cudaMemcpyAsync(&h, f->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, o.st));
+    CUDA_TRY(cudaEventRecord(ev[3], o.st));
+  }
   return FSM_OK;
 }
 
@@ -311,7 +315,7 @@ int run_collect(fsm_t f, uint64_t ticket, fsm_result* out, uint32_t* final_tid) 
     *final_tid = pd.q0t;
     return FSM_OK;
   }
-  CUDA_TRY(cudaEventSynchronize(f->ev[slot][3]));
+  CUDA_TRY(cudaEventSynchronize(f->ev[slot][pd.done_ev]));
   const Ctl& h = f->h_ctl[slot];
   float t1 = 0, t2 = 0;
   cudaEventElapsedTime(&t1, f->ev[slot][0], f->ev[slot][1]);

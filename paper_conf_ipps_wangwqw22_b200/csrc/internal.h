@@ -240,6 +240,7 @@ struct fsm_s {
     fsm_scheme scheme = FSM_SCHEME_SRE;
     uint32_t q0t = 0;
     bool active = false;
+    uint32_t done_ev = 3;  // event that marks the result readable (2: zero-copy result)
   } pend[kRing];
   uint64_t next_seq = 1;
   uint64_t* d_block_tmp = nullptr;

@@ -30,6 +30,7 @@ namespace gspec {
 namespace {
 
 constexpr int kBS = 256;
+constexpr int kU = 4;  // chunks per thread whose loads are issued together (batched passes)
 constexpr uint32_t kFuseMax = 256;  // bytes walked in lockstep with the reference path
 constexpr uint32_t kNone = 0xFFFFFFFFu;
 
@@ -295,14 +296,30 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     // verification of spec-1 records finishes in one pass, so it reads level 3 directly
     const bool use_cache = cached && (rnd > 0 || rp.k > 1);
     if (use_cache) {  // refresh level 2 from level 3 for the owned chunks
-      for (uint64_t c = max(lo, f) + threadIdx.x; c < hi; c += kBS) {
-        const uint32_t i = (uint32_t)(c - lo);
-        vc.ne[i] = (uint8_t)min(ld_cg(rs.n_end + c), 255u);
-        vc.no[i] = (uint8_t)min(ld_cg(rs.n_oth + c), 255u);
-        vc.s0[i] = ld_cg(rs.start + c);
-        vc.e0[i] = ld_cg(rs.end + c);
-        vc.s1[i] = ld_cg(rs.start + rs.cap + c);
-        vc.e1[i] = ld_cg(rs.end + rs.cap + c);
+      for (uint64_t cb = max(lo, f) + threadIdx.x; cb < hi; cb += kU * kBS) {
+        uint32_t ne[kU], no[kU], s0[kU], e0[kU], s1[kU], e1[kU];
+#pragma unroll
+        for (int u = 0; u < kU; u++) {  // all loads first: one L2 round trip for kU chunks
+          const uint64_t c = min(cb + u * kBS, hi - 1);
+          ne[u] = ld_cg(rs.n_end + c);
+          no[u] = ld_cg(rs.n_oth + c);
+          s0[u] = ld_cg(rs.start + c);
+          e0[u] = ld_cg(rs.end + c);
+          s1[u] = ld_cg(rs.start + rs.cap + c);
+          e1[u] = ld_cg(rs.end + rs.cap + c);
+        }
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+          const uint64_t c = cb + u * kBS;
+          if (c >= hi) break;
+          const uint32_t i = (uint32_t)(c - lo);
+          vc.ne[i] = (uint8_t)min(ne[u], 255u);
+          vc.no[i] = (uint8_t)min(no[u], 255u);
+          vc.s0[i] = s0[u];
+          vc.e0[i] = e0[u];
+          vc.s1[i] = s1[u];
+          vc.e1[i] = e1[u];
+        }
       }
       __syncthreads();
     }
@@ -325,35 +342,55 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       }
       bool ch = false;
       uint64_t fm = ~0ull, matches = 0, checks = 0;
-      for (uint64_t c = max(lo, f) + threadIdx.x; c < hi; c += kBS) {
-        const uint32_t xin = (c == f) ? tf : ld_cg(rs.x + c);
-        uint32_t e;
-        const bool hit = use_cache ? vr_lookup_cached(vc, (uint32_t)(c - lo), rs, rp.vr_end, rp.vr_oth, c, xin, &e)
-                                   : vr_lookup(rs, rp.vr_end, rp.vr_oth, c, xin, &e, nullptr);
-        rs.found[c] = hit;
-        if (!hit) e = ld_cg(rs.cur_end + c);  // F_c default: the chunk's end as of the round start
-        if (ld_cg(rs.x + c + 1) != e) {
-          st_cg(rs.x + c + 1, e);
-          ch = true;
+      // batched: a thread's kU chunks issue all their loads (incoming state, current
+      // outgoing state, default end, record slot 0) before any is resolved; reading
+      // x[c] early is allowed by the chaotic relaxation (a later write by chunk c-1's
+      // owner marks the pass as changed)
+      for (uint64_t cb = max(lo, f) + threadIdx.x; cb < hi; cb += kU * kBS) {
+        uint32_t xin[kU], xo[kU], ce[kU];
+        VrPre pre[kU];
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+          const uint64_t c = min(cb + u * kBS, hi - 1);
+          xin[u] = (c == f) ? tf : ld_cg(rs.x + c);
+          xo[u] = ld_cg(rs.x + c + 1);
+          ce[u] = ld_cg(rs.cur_end + c);
+          if (!use_cache) pre[u] = vr_prefetch(rs, c, false);
         }
-        checks++;
-        matches += hit;
-        if (!hit) fm = min(fm, c);
-        if (rp.dense) __stcg(rs.tstart + c, hit ? 0xFFFFFFFFu : xin);
-        if (fast && sre_like) {  // list every chunk without a match (warp-aggregated append)
-          const uint32_t am = __activemask();
-          const uint32_t bal = __ballot_sync(am, !hit);
-          if (bal) {
-            const uint32_t lane = threadIdx.x & 31, leader = __ffs(bal) - 1;
-            unsigned long long base = 0;
-            if (lane == leader)
-              base = atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_ntask[slot]),
-                               (unsigned long long)__popc(bal));
-            base = __shfl_sync(am, base, leader);
-            if (!hit) {
-              const uint64_t q = base + __popc(bal & ((1u << lane) - 1));
-              rs.task_chunk[q] = (uint32_t)c;
-              rs.task_start[q] = xin;  // captured before E rewrites x
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+          const uint64_t c = cb + u * kBS;
+          if (c >= hi) break;
+          const uint32_t xin_c = xin[u];
+          uint32_t e;
+          const bool hit = use_cache ? vr_lookup_cached(vc, (uint32_t)(c - lo), rs, rp.vr_end, rp.vr_oth, c, xin_c, &e)
+                                     : vr_resolve(pre[u], rs, rp.vr_end, rp.vr_oth, c, xin_c, &e, nullptr);
+          rs.found[c] = hit;
+          if (!hit) e = ce[u];  // F_c default: the chunk's end as of the round start
+          if (xo[u] != e) {
+            st_cg(rs.x + c + 1, e);
+            ch = true;
+          }
+          const uint32_t xin = xin_c;
+          checks++;
+          matches += hit;
+          if (!hit) fm = min(fm, c);
+          if (rp.dense) __stcg(rs.tstart + c, hit ? 0xFFFFFFFFu : xin);
+          if (fast && sre_like) {  // list every chunk without a match (warp-aggregated append)
+            const uint32_t am = __activemask();
+            const uint32_t bal = __ballot_sync(am, !hit);
+            if (bal) {
+              const uint32_t lane = threadIdx.x & 31, leader = __ffs(bal) - 1;
+              unsigned long long base = 0;
+              if (lane == leader)
+                base = atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_ntask[slot]),
+                                 (unsigned long long)__popc(bal));
+              base = __shfl_sync(am, base, leader);
+              if (!hit) {
+                const uint64_t q = base + __popc(bal & ((1u << lane) - 1));
+                rs.task_chunk[q] = (uint32_t)c;
+                rs.task_start[q] = xin;  // captured before E rewrites x
+              }
             }
           }
         }
@@ -622,11 +659,25 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   // ---------------- Z: finalize (chunk ends, u64 accept count) ----------------
   {
     uint64_t total = 0;
-    for (uint64_t c = lo + threadIdx.x; c < hi; c += kBS) {
-      uint32_t e = 0, cnt = 0;
-      vr_lookup(rs, rp.vr_end, rp.vr_oth, c, ld_cg(rs.x + c), &e, &cnt);
-      total += cnt;
-      if (chunk_ends) chunk_ends[c] = __ldg(img.inv + ld_cg(rs.x + c + 1));
+    for (uint64_t cb = lo + threadIdx.x; cb < hi; cb += kU * kBS) {
+      uint32_t xin[kU], xo[kU];
+      VrPre pre[kU];
+#pragma unroll
+      for (int u = 0; u < kU; u++) {
+        const uint64_t c = min(cb + u * kBS, hi - 1);
+        xin[u] = ld_cg(rs.x + c);
+        xo[u] = ld_cg(rs.x + c + 1);
+        pre[u] = vr_prefetch(rs, c, true);
+      }
+#pragma unroll
+      for (int u = 0; u < kU; u++) {
+        const uint64_t c = cb + u * kBS;
+        if (c >= hi) break;
+        uint32_t e = 0, cnt = 0;
+        vr_resolve(pre[u], rs, rp.vr_end, rp.vr_oth, c, xin[u], &e, &cnt);
+        total += cnt;
+        if (chunk_ends) chunk_ends[c] = __ldg(img.inv + xo[u]);
+      }
     }
     total = block_sum<uint64_t>(total, red64);
     if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->accept_count), (unsigned long long)total);

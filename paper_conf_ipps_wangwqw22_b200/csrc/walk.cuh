@@ -159,18 +159,31 @@ __device__ __forceinline__ void st_cg(uint32_t* p, uint32_t v) { __stcg(p, v); }
 
 // Look x up in VR_c (END slots then OTH slots).  Returns true on a match.
 // Slot 0 and the ring counts are loaded together (one L2 round trip for the
-// common single-record chunk), the rest of the rings only if needed.
-__device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, uint32_t vr_oth, uint64_t c,
-                                          uint32_t x, uint32_t* end, uint32_t* cnt) {
-  const uint32_t ne_raw = ld_cg(rs.n_end + c), no_raw = ld_cg(rs.n_oth + c);
-  const uint32_t s0 = ld_cg(rs.start + c), e0 = ld_cg(rs.end + c);
-  const uint32_t c0 = cnt ? ld_cg(rs.cnt + c) : 0u;
-  if (ne_raw >= 1 && s0 == x) {
-    *end = e0;
-    if (cnt) *cnt = c0;
+// common single-record chunk), the rest of the rings only if needed.  The
+// prefetch half depends on c only, so a thread can issue it for several
+// chunks before resolving any (batched relaxation passes).
+struct VrPre {
+  uint32_t ne, no, s0, e0, c0;
+};
+
+__device__ __forceinline__ VrPre vr_prefetch(const RecStore& rs, uint64_t c, bool want_cnt) {
+  VrPre p;
+  p.ne = ld_cg(rs.n_end + c);
+  p.no = ld_cg(rs.n_oth + c);
+  p.s0 = ld_cg(rs.start + c);
+  p.e0 = ld_cg(rs.end + c);
+  p.c0 = want_cnt ? ld_cg(rs.cnt + c) : 0u;
+  return p;
+}
+
+__device__ __forceinline__ bool vr_resolve(const VrPre& p, const RecStore& rs, uint32_t vr_end, uint32_t vr_oth,
+                                           uint64_t c, uint32_t x, uint32_t* end, uint32_t* cnt) {
+  if (p.ne >= 1 && p.s0 == x) {
+    *end = p.e0;
+    if (cnt) *cnt = p.c0;
     return true;
   }
-  const uint32_t ne = min(ne_raw, vr_end);
+  const uint32_t ne = min(p.ne, vr_end);
   for (uint32_t s = 1; s < ne; s++) {
     if (ld_cg(rs.start + s * rs.cap + c) == x) {
       *end = ld_cg(rs.end + s * rs.cap + c);
@@ -178,7 +191,7 @@ __device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, u
       return true;
     }
   }
-  const uint32_t no = min(no_raw, vr_oth);
+  const uint32_t no = min(p.no, vr_oth);
   for (uint32_t s = 0; s < no; s++) {
     const uint64_t o = (uint64_t)(kVrMax + s) * rs.cap + c;
     if (ld_cg(rs.start + o) == x) {
@@ -188,6 +201,11 @@ __device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, u
     }
   }
   return false;
+}
+
+__device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, uint32_t vr_oth, uint64_t c,
+                                          uint32_t x, uint32_t* end, uint32_t* cnt) {
+  return vr_resolve(vr_prefetch(rs, c, cnt != nullptr), rs, vr_end, vr_oth, c, x, end, cnt);
 }
 
 // Chunk 0's start state (a shard's reference candidate may live on the device).
