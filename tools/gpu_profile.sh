@@ -1,0 +1,9 @@
+# Round profile capture: GPU tests, default bench line, ncu launch list of the bench
+# command, ncu --set full of the two kernels of a run.  Usage (from gpurun):
+#   bash tools/gpu_profile.sh
+cd $GRAFT_REPO_ROOT; mkdir -p gpurun_out
+timeout 2400 python -m pytest tests -m gpu -q --timeout 1200 -p no:cacheprovider > gpurun_out/pytest_gpu_all.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu_all.log
+timeout 900 python bench.py > gpurun_out/bench_default.log 2>&1
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches_c2.csv python bench.py --steps 2 --warmup 3 --e2e-steps 0 --no-cpu-baseline > gpurun_out/ncu_launch.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_spec_tma -s 2 -c 1 -o gpurun_out/spec_tma_c2 -f python tools/profile_spec.py c2 sre 3 > gpurun_out/ncu_spec.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:k_verify_recover -s 2 -c 1 -o gpurun_out/verify_c2 -f python tools/profile_spec.py c2 sre 3 > gpurun_out/ncu_verify.log 2>&1

@@ -11,7 +11,9 @@ reps = int(sys.argv[3]) if len(sys.argv) > 3 else 3
 w = gen.workload(cfg)
 x = torch.empty(w.length, dtype=torch.uint8, device='cuda')
 w.device(x)
-fsm = gs.FSM.load(w.table, w.start, w.accept)
+prof = torch.empty(1 << 20, dtype=torch.uint8, device='cuda')
+w.device(prof, offset=w.length)  # disjoint training trace, as bench.py
+fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof.cpu().numpy())
 for i in range(reps):
     r = fsm.run(x, scheme=scheme)
 torch.cuda.synchronize()
