@@ -53,6 +53,15 @@ int upload(fsm_t f, const T** dst, const std::vector<T>& v, size_t pad_bytes = 0
   return FSM_OK;
 }
 
+// Every entry point starts by clearing a stale (non-sticky) CUDA error left by a
+// failed runtime call elsewhere in this thread, so it is not reported by our own
+// launch checks; GSPEC_DEBUG_ERR=1 prints it.
+void entry_clear(const char* name) {
+  const cudaError_t e = cudaGetLastError();
+  static const bool dbg = getenv("GSPEC_DEBUG_ERR") != nullptr;
+  if (e != cudaSuccess && dbg) fprintf(stderr, "gspec: stale CUDA error at %s entry: %s\n", name, cudaGetErrorString(e));
+}
+
 constexpr uint32_t kRow8Bytes = 260;  // walk.cuh kRow8: row r starts at bank (r * 65) % 32 = r % 32
 
 // MODE_U8 row placement from a profile sample (an extension of the transformation,
@@ -375,6 +384,7 @@ uint64_t fsm_num_chunks(uint64_t len, uint32_t chunk_bytes) {
 
 int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, const uint8_t* accept,
              const fsm_load_opts* opts, fsm_t* out) {
+  entry_clear("fsm_load");
   if (!table || !accept || !out) return fail(FSM_EINVAL, "NULL table/accept/out");
   if (n == 0 || nsyms == 0 || nsyms > 256 || start >= n) return fail(FSM_EINVAL, "bad nstates/nsyms/start");
   if (n >= (1u << 24)) return fail(FSM_EUNSUPPORTED, "nstates >= 2^24");
@@ -578,6 +588,7 @@ void fsm_free(fsm_t f) {
 
 int fsm_run(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts, uint32_t* d_chunk_ends,
             fsm_result* out) {
+  entry_clear("fsm_run");
   if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
   if (!d_input && len > 0) return fail(FSM_EINVAL, "NULL input");
   Opts o;
@@ -609,6 +620,7 @@ int fsm_run(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* o
 
 int fsm_run_async(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts, uint32_t* d_chunk_ends,
                   uint64_t* ticket) {
+  entry_clear("fsm_run_async");
   if (!f || !ticket) return fail(FSM_EINVAL, "NULL handle/ticket");
   if (!d_input && len > 0) return fail(FSM_EINVAL, "NULL input");
   Opts o;
@@ -630,6 +642,7 @@ int fsm_run_async(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_o
 }
 
 int fsm_wait(fsm_t f, uint64_t ticket, fsm_result* out) {
+  entry_clear("fsm_wait");
   if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
   fsm_result r;
   uint32_t fin = 0;
@@ -644,6 +657,7 @@ int fsm_wait(fsm_t f, uint64_t ticket, fsm_result* out) {
 
 int fsm_run_host(fsm_t f, const uint8_t* h_input, uint64_t len, const fsm_run_opts* opts, uint32_t* h_chunk_ends,
                  fsm_result* out) {
+  entry_clear("fsm_run_host");
   if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
   if (!h_input && len > 0) return fail(FSM_EINVAL, "NULL input");
   Opts o;
@@ -676,6 +690,7 @@ int fsm_run_host(fsm_t f, const uint8_t* h_input, uint64_t len, const fsm_run_op
 
 int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_run_opts* opts, fsm_scheme* outp,
                       fsm_features* feat) {
+  entry_clear("fsm_select_scheme");
   if (!f || !outp) return fail(FSM_EINVAL, "NULL handle/out");
   if (!d_sample && len > 0) return fail(FSM_EINVAL, "NULL sample");
   Opts o;
@@ -872,6 +887,7 @@ extern "C" {
 
 int fsm_shard_map(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
                   const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local) {
+  entry_clear("fsm_shard_map");
   if (!f || !d_map) return fail(FSM_EINVAL, "NULL handle/map");
   if (!d_shard && len > 0) return fail(FSM_EINVAL, "NULL shard");
   if (lb_len > 16 || (lb_len && !d_lookback)) return fail(FSM_EINVAL, "lookback_len must be <= 16 with bytes");
@@ -1018,6 +1034,7 @@ int fsm_shard_map(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* 
 
 int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, const fsm_run_opts* opts,
                      uint32_t* d_chunk_ends_local, fsm_result* out) {
+  entry_clear("fsm_shard_finish");
   if (!f || !d_maps || !out || rank >= G) return fail(FSM_EINVAL, "bad finish arguments");
   if (f->shard_mode < 0) return fail(FSM_EINVAL, "fsm_shard_map was not called");
   Opts o;

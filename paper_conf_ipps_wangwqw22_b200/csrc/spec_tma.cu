@@ -76,8 +76,10 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   uint8_t* table = smem_raw;
   uint8_t* stages = smem_raw + table_off;
   uint64_t* bars = reinterpret_cast<uint64_t*>(stages + (size_t)nwarps * S * kStageBytes);
-  stage_table(img, table);
+  stage_table(img, table);  // load-time data: staged before the dependency wait
+  pdl_wait();                // the previous kernel in the stream (e.g. the last run's verify) is done
   if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, q0_of(rp), rp.N);
+  pdl_launch_dependents();   // the verify kernel may launch now; it waits for our completion
   if (lane == 0)
     for (int s = 0; s < S; s++) mbar_init(bars + warp * S + s, 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -260,8 +262,17 @@ cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunPa
   if (e != cudaSuccess) return e;
   uint64_t grid = std::min<uint64_t>((uint64_t)sms, (ntiles + w - 1) / w);
   if (grid < 1) grid = 1;
-  kern<<<(unsigned)grid, w * 32, smem, st>>>(tm, img, rp, rs, n_full, table_off, tile0, f2, ctl);
-  return cudaGetLastError();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(w * 32);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, tm, img, rp, rs, n_full, table_off, tile0, f2, ctl);
 }
 
 template <int MODE, int KP, bool TASKS>

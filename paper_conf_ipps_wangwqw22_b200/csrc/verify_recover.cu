@@ -269,8 +269,10 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   auto stamp = [&]() {
     if (blockIdx.x == 0 && threadIdx.x == 0 && nst < 24) { ctl->stamp[nst++] = gtimer(); ctl->nstamp = nst; }
   };
+  stage_table(img, smem);  // the table is load-time data: staged before the dependency wait
+  pdl_wait();               // the spec kernel's records are complete and visible
+  pdl_launch_dependents();  // the next run's spec kernel may launch (it waits for us the same way)
   stamp();
-  stage_table(img, smem);
   __syncthreads();
   stamp();
 
@@ -733,8 +735,19 @@ cudaError_t launch_m(const DevImage& img, const RunParams& rp, const RecStore& r
   DevImage a0 = img;
   RunParams a1 = rp;
   RecStore a2 = rs;
-  void* args[] = {&a0, &a1, &a2, &ctl, &btmp, &chunk_ends, &cap};
-  return cudaLaunchCooperativeKernel((const void*)kern, dim3((unsigned)grid), dim3(kBS), args, smem, st);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3(kBS);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 2 : 1;
+  return cudaLaunchKernelEx(&cfg, kern, a0, a1, a2, ctl, btmp, chunk_ends, cap);
 }
 
 // After the TMA task kernel: the partial tail chunk's task (if any), then commit

@@ -153,6 +153,11 @@ __device__ __forceinline__ uint32_t walk_bytes(const DevImage& img, const uint8_
   return code;
 }
 
+// PDL (see internal.h): wait for the preceding grid (a no-op without a
+// programmatic dependency), and let the next grid in the stream launch.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_launch_dependents() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
 // ---- coherent (L2) accessors for data written by other CTAs of a persistent kernel
 __device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) { return __ldcg(p); }
 __device__ __forceinline__ void st_cg(uint32_t* p, uint32_t v) { __stcg(p, v); }
