@@ -198,6 +198,13 @@ int fsm_get_records(fsm_t fsm, uint64_t nchunks, uint32_t* start, uint32_t* end,
  * each relaxation pass, each recovery, finalize); up to 24 entries. */
 int fsm_get_phase_times(fsm_t fsm, double* us, uint32_t* n);
 
+/* Run timeline of the last collected run (profiling; recorded only when the
+ * environment has GSPEC_STAMPS=1 at library load, otherwise every entry is -1):
+ * us[0] = speculative-execution kernel (entry of CTA 0 -> last warp done),
+ * us[1] = gap until the verify/recover kernel's entry, us[2] = verify/recover
+ * kernel (entry -> last CTA done).  us: caller-owned, 3 doubles. */
+int fsm_get_timeline(fsm_t fsm, double* us);
+
 void fsm_free(fsm_t fsm);
 const char* fsm_strerror(int status);
 const char* fsm_last_error(void);

@@ -71,6 +71,7 @@ _lib.fsm_get_transform.argtypes = [P, P, P, P, P, P, P]
 _lib.fsm_get_qs.argtypes = [P, ctypes.c_uint8, ctypes.c_uint8, P, P, P]
 _lib.fsm_get_records.argtypes = [P, U64, P, P, P, P, P, P]
 _lib.fsm_get_phase_times.argtypes = [P, P, ctypes.POINTER(U32)]
+_lib.fsm_get_timeline.argtypes = [P, P]
 _lib.fsm_comm_unique_id.argtypes = [P]
 _lib.fsm_comm_init.argtypes = [ctypes.c_int, ctypes.c_int, P, ctypes.POINTER(P)]
 _lib.fsm_run_sharded.argtypes = [P, P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
@@ -254,6 +255,12 @@ class FSM:
         n = U32(0)
         _check(_lib.fsm_get_phase_times(self._h, us.ctypes.data, ctypes.byref(n)), "fsm_get_phase_times")
         return us[:n.value].copy()
+
+    def timeline(self):
+        """(spec kernel, gap, verify kernel) in µs of the last collected run; -1 unless GSPEC_STAMPS=1."""
+        us = np.zeros(3, np.float64)
+        _check(_lib.fsm_get_timeline(self._h, us.ctypes.data), "fsm_get_timeline")
+        return us.copy()
 
     def map_bytes(self) -> int:
         return int(_lib.fsm_map_bytes(self._h))

@@ -243,6 +243,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   rp.vr_end = o.vr_end;
   rp.vr_oth = o.vr_oth;
   rp.q0_dev = q0_dev;
+  rp.stamps = stamps_enabled() ? 1u : 0u;
   cudaEvent_t* ev = f->ev[slot];
   Ctl& h = f->h_ctl[slot];
   std::memset(&h, 0, sizeof(Ctl));
@@ -332,6 +333,7 @@ int run_collect(fsm_t f, uint64_t ticket, fsm_result* out, uint32_t* final_tid) 
   fill_result_stats(out, h);
   f->last_nstamp = std::min<uint32_t>(h.nstamp, 24);
   std::copy(h.stamp, h.stamp + 24, f->last_stamp);
+  std::copy(h.tl, h.tl + 4, f->last_tl);
   out->accept_count = h.accept_count;
   out->ms_spec = t1;
   out->ms_verify = t2;
@@ -352,6 +354,9 @@ fsm_scheme tree_select(const fsm_features& ft, uint32_t n) {
   if (n <= 31 && ft.uniq10 >= n / 2.0) return FSM_SCHEME_ENUM;
   if (ft.uniq10 <= 4.0) return FSM_SCHEME_SRE;
   if (ft.acck >= 0.9 && ft.acck - ft.acc1 >= 0.2) return FSM_SCHEME_PM;
+  // R19b: helpers cost a full chunk walk on a saturated GPU; RR/NF only when the
+  // extra lookback candidates catch most mispredictions
+  if (ft.acck - ft.acc1 < 0.5) return FSM_SCHEME_SRE;
   if (ft.input_sensitivity >= 0.2) return FSM_SCHEME_NF;
   return FSM_SCHEME_RR;
 }
@@ -792,6 +797,14 @@ int fsm_get_phase_times(fsm_t f, double* us, uint32_t* n) {
   if (us)
     for (uint32_t i = 0; i < k; i++) us[i] = (f->last_stamp[i] - f->last_stamp[0]) * 1e-3;
   *n = k;
+  return FSM_OK;
+}
+
+int fsm_get_timeline(fsm_t f, double* us) {
+  if (!f || !us) return fail(FSM_EINVAL, "NULL handle/us");
+  const uint64_t* t = f->last_tl;
+  const bool ok = t[0] && t[1] >= t[0] && t[2] >= t[1] && t[3] >= t[2];
+  for (int i = 0; i < 3; i++) us[i] = ok ? (t[i + 1] - t[i]) * 1e-3 : -1.0;
   return FSM_OK;
 }
 

@@ -95,12 +95,16 @@ struct Ctl {
   uint64_t jacobi_iters;
   uint64_t ntask[2];     // (unused, kept for layout)
   uint64_t it_fm[3], it_checks[3], it_matches[3], it_ntask[3];  // per relaxation pass (rotating)
+  uint64_t it_reread[3];  // round-0 SRE pass with inline tasks: bytes re-walked (rotating)
   uint32_t dense_pending;  // verify exited: a dense task round (frontier fmin) must run first
   uint32_t nstamp;         // phase timestamps of the last verify launch (%globaltimer, ns)
   uint64_t stamp[24];
   uint32_t zdone;        // finalize tickets (the last CTA publishes the block to h_out)
   uint32_t xfin;         // transformed final state (written by the last kernel of a run)
   uint32_t pad1;
+  // run timeline (%globaltimer ns; GSPEC_STAMPS=1): spec entry, last spec warp done,
+  // verify entry (before table staging), verify exit (last CTA, before the host publish)
+  uint64_t tl[4];
 };
 
 struct RunParams {
@@ -117,7 +121,18 @@ struct RunParams {
   Ctl* ctl_init;   // non-null: the first spec kernel initialises this control block (no H2D copy)
   const uint32_t* q0_dev;  // non-null: chunk 0's start is read from the device (shard candidates)
   Ctl* h_out;      // non-null: pinned host slot; the finalize step writes the control block there
+  uint32_t stamps; // 1: record the run timeline (Ctl::tl), profiling only
 };
+
+// GSPEC_STAMPS=1: kernels record the run timeline in Ctl::tl (one extra atomic per warp).
+inline bool stamps_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("GSPEC_STAMPS");
+    v = e ? atoi(e) : 0;
+  }
+  return v != 0;
+}
 
 // Programmatic dependent launch (PDL) between the two kernels of a run and
 // between consecutive runs: the next kernel is launched while the previous one
@@ -295,7 +310,8 @@ struct fsm_s {
   int shard_mode = -1;          // 0 fused/single path, 1 enum, 2 multi-path, 3 fused with cand[0]
   uint64_t shard_ticket = 0;
   uint32_t last_nstamp = 0;            // verify phase timestamps of the last collected run
-  uint64_t last_stamp[24] = {};           // mode 3: the pending cand[0] pipeline run
+  uint64_t last_stamp[24] = {};
+  uint64_t last_tl[4] = {};             // run timeline of the last collected run (GSPEC_STAMPS=1)
   const uint8_t* shard_in = nullptr;
   uint64_t shard_len = 0;
   uint32_t shard_ncand = 0, shard_nj = 0;  // candidates; chunks covered by the fused prefix

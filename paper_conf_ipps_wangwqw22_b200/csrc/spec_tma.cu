@@ -78,7 +78,10 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   uint64_t* bars = reinterpret_cast<uint64_t*>(stages + (size_t)nwarps * S * kStageBytes);
   stage_table(img, table);  // load-time data: staged before the dependency wait
   pdl_wait();                // the previous kernel in the stream (e.g. the last run's verify) is done
-  if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, q0_of(rp), rp.N);
+  if (rp.ctl_init && blockIdx.x == 0) {
+    init_ctl(rp.ctl_init, q0_of(rp), rp.N);
+    if (rp.stamps && threadIdx.x == 0) rp.ctl_init->tl[0] = gtimer();
+  }
   pdl_launch_dependents();   // the verify kernel may launch now; it waits for our completion
   if (lane == 0)
     for (int s = 0; s < S; s++) mbar_init(bars + warp * S + s, 1);
@@ -91,6 +94,12 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   const uint64_t ntiles = (n_full + 31) / 32 - tile0;
   const uint64_t gw = (uint64_t)blockIdx.x * nwarps + warp, tw = (uint64_t)gridDim.x * nwarps;
   if (gw >= ntiles) return;
+  struct StampEnd {  // timeline: the last warp to finish (profiling only)
+    bool on; Ctl* c; uint32_t lane;
+    __device__ ~StampEnd() {
+      if (on && lane == 0) atomicMax(reinterpret_cast<unsigned long long*>(&c->tl[1]), (unsigned long long)gtimer());
+    }
+  } stamp_end{rp.stamps != 0 && rp.ctl_init != nullptr && !TASKS, rp.ctl_init, lane};
   const uint64_t my_tiles = (ntiles - gw + tw - 1) / tw;
   uint64_t n_mustdo = 0, n_sre = 0;
   const uint64_t items = my_tiles * segs;  // (tile, segment) pairs streamed by this warp

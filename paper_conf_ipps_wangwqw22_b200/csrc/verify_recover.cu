@@ -249,12 +249,6 @@ __device__ void task_walk(const DevImage& img, const uint8_t* smem, const RunPar
   *cnt_out = acc;
 }
 
-__device__ __forceinline__ uint64_t gtimer() {
-  uint64_t t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
-
 template <int MODE>
 __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
                                                         uint64_t* btmp, uint32_t* chunk_ends, uint32_t cache_cap) {
@@ -269,6 +263,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   auto stamp = [&]() {
     if (blockIdx.x == 0 && threadIdx.x == 0 && nst < 24) { ctl->stamp[nst++] = gtimer(); ctl->nstamp = nst; }
   };
+  if (rp.stamps && blockIdx.x == 0 && threadIdx.x == 0 && ctl->tl[2] == 0) ctl->tl[2] = gtimer();
   stage_table(img, smem);  // the table is load-time data: staged before the dependency wait
   pdl_wait();               // the spec kernel's records are complete and visible
   pdl_launch_dependents();  // the next run's spec kernel may launch (it waits for us the same way)
@@ -290,13 +285,106 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   uint32_t git = 0;  // relaxation passes since launch (identical in every CTA)
   const bool cached = cache_cap != 0 && hi - lo <= cache_cap;
   const VrCache vc = vr_cache_at(smem + ((smem_bytes_for(img) + 15) & ~15u), cache_cap);
+  // round state, kept identically by every CTA (block 0 mirrors it into the control block)
+  uint64_t f = vctl->f;
+  uint32_t tf = vctl->tf;
+  uint32_t rnd = (uint32_t)vctl->rounds;
+  uint64_t last_tasks = 0;  // tasks of the previous round (this launch)
   for (;;) {
-    const uint64_t f = vctl->f;
-    const uint32_t tf = vctl->tf;
-    const uint32_t rnd = (uint32_t)vctl->rounds;
-    // level 2 pays off when a round's relaxation makes several passes; the first
-    // verification of spec-1 records finishes in one pass, so it reads level 3 directly
-    const bool use_cache = cached && (rnd > 0 || rp.k > 1);
+    // ---- round 0 of SRE with spec-1 records: verification + inline recovery --------
+    // With one record per chunk and cur_end = that record's end, F_c(x) = end_c for
+    // every x, so x_{c+1} = end_c is already the fixed point: the pass cannot change
+    // anything and each chunk's incoming state x_c = end_{c-1} is final.  The SRE
+    // task of an unmatched chunk (start x_c, Alg. 3 L16-18) is therefore run right
+    // where the mismatch is found, instead of being listed for a separate phase.
+    // Records and every counter are those of the listed-task rounds; x[c+1] is left
+    // to the next relaxation pass (it reads the new record), so this pass only reads
+    // round-0 values.
+    if (fast && rp.scheme == FSM_SCHEME_SRE && rp.k == 1 && rnd == 0 && f == 0 && !rp.dense) {
+      const uint32_t slot = git % 3;
+      if (b == 0 && threadIdx.x == 0) {
+        const uint32_t nx = (git + 1) % 3;
+        vctl->changed[nx] = 0;
+        vctl->it_fm[nx] = N;
+        vctl->it_checks[nx] = vctl->it_matches[nx] = vctl->it_ntask[nx] = vctl->it_reread[nx] = 0;
+      }
+      uint64_t fm = ~0ull, matches = 0, checks = 0, ntask = 0, reread = 0;
+      for (uint64_t cb = lo + threadIdx.x; cb < hi; cb += kU * kBS) {
+        uint32_t xin[kU], s0[kU];
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+          const uint64_t c = min(cb + u * kBS, hi - 1);
+          xin[u] = (c == 0) ? tf : ld_cg(rs.x + c);
+          s0[u] = ld_cg(rs.start + c);
+        }
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+          const uint64_t c = cb + u * kBS;
+          if (c >= hi) break;
+          const bool hit = xin[u] == s0[u];
+          rs.found[c] = hit;
+          checks++;
+          matches += hit;
+          if (!hit) {
+            fm = min(fm, c);
+            uint32_t e, cnt;
+            task_walk<MODE>(img, smem, rp, rs, c, xin[u], &e, &cnt);
+            const uint32_t ne = ld_cg(rs.n_end + c);
+            const uint64_t o = (uint64_t)(ne % rp.vr_end) * rs.cap + c;
+            st_cg(rs.start + o, xin[u]);
+            st_cg(rs.end + o, e);
+            st_cg(rs.cnt + o, cnt);
+            st_cg(rs.n_end + c, ne + 1);
+            st_cg(rs.cur_end + c, e);
+            ntask++;
+            reread += min((uint64_t)rp.B, rp.len - c * rp.B);
+          }
+        }
+      }
+      bool bch = false;
+      block_reduce_pass(false, fm, checks, matches, red4, &bch);
+      ntask = block_sum<uint64_t>(ntask, red64);
+      reread = block_sum<uint64_t>(reread, red64);
+      if (threadIdx.x == 0) {
+        if (fm != ~0ull) atomicMin(reinterpret_cast<unsigned long long*>(&ctl->it_fm[slot]), (unsigned long long)fm);
+        if (checks) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_checks[slot]), (unsigned long long)checks);
+        if (matches)
+          atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_matches[slot]), (unsigned long long)matches);
+        if (ntask) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_ntask[slot]), (unsigned long long)ntask);
+        if (reread) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_reread[slot]), (unsigned long long)reread);
+      }
+      grid.sync();
+      stamp();
+      git++;
+      const uint64_t f2 = vctl->it_fm[slot];
+      const uint64_t nt = vctl->it_ntask[slot];
+      if (b == 0 && threadIdx.x == 0) {
+        vctl->verify_checks = vctl->verify_checks + vctl->it_checks[slot];
+        vctl->verify_matches = vctl->verify_matches + vctl->it_matches[slot];
+        vctl->jacobi_iters = vctl->jacobi_iters + 1;
+        vctl->fmin = f2;
+      }
+      if (f2 >= N) break;
+      const uint32_t tf2 = ld_cg(rs.x + f2);  // = end_{f2-1}: not rewritten by the tasks
+      if (b == 0 && threadIdx.x == 0) {      // commit the round (the must-do is chunk f2)
+        vctl->tasks_mustdo = vctl->tasks_mustdo + 1;
+        vctl->tasks_sre = vctl->tasks_sre + (nt - 1);
+        vctl->reread_bytes = vctl->reread_bytes + vctl->it_reread[slot];
+        vctl->active_sum = vctl->active_sum + nt;
+        vctl->rounds = vctl->rounds + 1;
+        vctl->f = f2;
+        vctl->tf = tf2;
+      }
+      f = f2;
+      tf = tf2;
+      rnd++;
+      last_tasks = nt;
+      continue;  // round 1 verification: the tasks' records are visible (grid barrier above)
+    }
+    // level 2 pays off when a round's relaxation makes several passes: spec-k records,
+    // or a round after many tasks; a verification after a few tasks (high speculation
+    // accuracy) finishes in one pass and reads level 3 directly
+    const bool use_cache = cached && (rp.k > 1 || (rnd > 0 && (!fast || last_tasks * 64 >= N - f)));
     if (use_cache) {  // refresh level 2 from level 3 for the owned chunks
       for (uint64_t cb = max(lo, f) + threadIdx.x; cb < hi; cb += kU * kBS) {
         uint32_t ne[kU], no[kU], s0[kU], e0[kU], s1[kU], e1[kU];
@@ -340,7 +428,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         const uint32_t nx = (git + 1) % 3;
         vctl->changed[nx] = 0;
         vctl->it_fm[nx] = N;
-        vctl->it_checks[nx] = vctl->it_matches[nx] = vctl->it_ntask[nx] = 0;
+        vctl->it_checks[nx] = vctl->it_matches[nx] = vctl->it_ntask[nx] = vctl->it_reread[nx] = 0;
       }
       bool ch = false;
       uint64_t fm = ~0ull, matches = 0, checks = 0;
@@ -471,6 +559,10 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
           vctl->tf = tf2;
         }
       }
+      f = f2;
+      tf = tf2;
+      rnd++;
+      last_tasks = nt;
       grid.sync();
       stamp();
       continue;
@@ -655,6 +747,10 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
           vctl->tf = tf2;
         }
       }
+      f = f2;
+      tf = tf2;
+      rnd++;
+      last_tasks = nslots;
     }
     grid.sync();
   }
@@ -695,6 +791,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       }
       __syncthreads();
       if (last) {
+        if (rp.stamps && threadIdx.x == 0) ctl->tl[3] = gtimer();
         __threadfence();
         const uint32_t* src = reinterpret_cast<const uint32_t*>(ctl);
         uint32_t* dst = reinterpret_cast<uint32_t*>(rp.h_out);
@@ -783,7 +880,7 @@ __global__ void __launch_bounds__(32) k_dense_finish(DevImage img, RunParams rp,
   ctl->dense_pending = 0;
   ctl->changed[0] = 0;  // the relaunched kernel starts its passes at slot 0
   ctl->it_fm[0] = rp.N;
-  ctl->it_checks[0] = ctl->it_matches[0] = ctl->it_ntask[0] = 0;
+  ctl->it_checks[0] = ctl->it_matches[0] = ctl->it_ntask[0] = ctl->it_reread[0] = 0;
 }
 
 template <int MODE>

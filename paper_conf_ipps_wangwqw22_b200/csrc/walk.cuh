@@ -213,6 +213,12 @@ __device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, u
   return vr_resolve(vr_prefetch(rs, c, cnt != nullptr), rs, vr_end, vr_oth, c, x, end, cnt);
 }
 
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
 // Chunk 0's start state (a shard's reference candidate may live on the device).
 __device__ __forceinline__ uint32_t q0_of(const RunParams& rp) { return rp.q0_dev ? __ldcg(rp.q0_dev) : rp.q0t; }
 

@@ -203,7 +203,7 @@ def test_lookback_table_matches_oracle(gs):
 
 
 def test_selector_features_match_oracle(gs):
-    for name, expect in (("c1", {"enum"}), ("c2", {"sre"}), ("c3", {"rr", "nf"})):
+    for name, expect in (("c1", {"enum"}), ("c2", {"sre"}), ("c3", {"sre"})):  # R19b
         w, data = _wl(name, 1 << 20)
         fsm = gs.FSM.load(w.table, w.start, w.accept)
         pick, ft = fsm.select_scheme(torch.from_numpy(data).cuda())
@@ -299,3 +299,24 @@ def test_full_size_other_configs(gs, name, length, scheme):
     fsm = gs.FSM.load(w.table, w.start, w.accept)
     res = fsm.run(x, scheme=scheme)
     check_equal(res, ref, 4096, w.nstates)
+
+
+@pytest.mark.parametrize("name,length,vr_end", [("c2", 16 << 20, 16), ("c4", 16 << 20, 16), ("c4", 8 << 20, 1),
+                                                ("rand:40:7:3", 4 << 20, 16)])
+def test_inline_round0_recovery(gs, name, length, vr_end):
+    """SRE with a high-accuracy profile hint: round 0's verification runs the SRE tasks
+    inline (verify_recover.cu, round 0 of SRE); results and round diagnostics must
+    equal the listed-task semantics of the oracle's simulator exactly."""
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, 4096)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    x = torch.from_numpy(data).cuda()
+    fsm.select_scheme(x[: 1 << 20])  # sets the accuracy hint: no dense rounds
+    res = fsm.run(x, scheme="sre", vr_end=vr_end)
+    check_equal(res, ref, 4096, w.nstates)
+    sim = oracle.simulate(w.table, w.start, w.accept, data, 4096, scheme="sre", vr_end=vr_end)
+    for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks",
+              "verify_matches"):
+        assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+    if name != "c2":
+        assert res.stats["tasks_sre"] > 0  # mispredictions really happened

@@ -393,7 +393,11 @@ def test_features_closed_forms():
             img = {int(tac[q, ch]) for q in img}
         tot += len(img) * (1 if gen.RESET_BYTE in win else 16)
     assert f["uniq10"] == tot / 64 and f["uniq10"] > 8
-    assert oracle.select(f, w.nstates) in (oracle.RR, oracle.NF)
+    # spec-4 adds ~0.2 accuracy: helpers would mostly miss -> SRE (R19b)
+    assert f["acck"] - f["acc1"] < 0.5 and oracle.select(f, w.nstates) == oracle.SRE
+    g = dict(f, acc1=0.1, acck=0.7)  # helpers catch most mispredictions -> RR / NF by sensitivity
+    assert oracle.select(dict(g, sens=0.0), w.nstates) == oracle.RR
+    assert oracle.select(dict(g, sens=0.3), w.nstates) == oracle.NF
 
 
 def test_features_accuracy_bruteforce():
