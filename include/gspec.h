@@ -62,7 +62,11 @@ typedef struct {
                                     (layout only, results unchanged); NULL = no profile    */
   uint64_t profile_len;
   uint32_t smem_budget_bytes;    /* hot-row budget in shared memory; 0 = auto        */
-  uint32_t force_mode;           /* 0 auto; 1 u8 raw-byte table; 2 u16 classed; 3 u32 classed */
+  uint32_t force_mode;           /* 0 auto; 1 u8 raw-byte table; 2 u16 classed (hot rows in smem,
+                                    cold rows in L2); 3 u32 classed; 4 u16 classed whose cold rows
+                                    are delta rows in smem (hot base row + <= 2 exceptions, rows that
+                                    do not compress stay in L2).  Auto picks 4 over 2 when the delta
+                                    rows keep more frequency mass on chip. */
 } fsm_load_opts;
 
 typedef struct {
@@ -129,6 +133,32 @@ int fsm_run(fsm_t fsm, const uint8_t* d_input, uint64_t len, const fsm_run_opts*
 int fsm_run_async(fsm_t fsm, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
                   uint32_t* d_chunk_ends, uint64_t* ticket);
 int fsm_wait(fsm_t fsm, uint64_t ticket, fsm_result* out);
+
+/* ---- stream-level batching (Alg. 1 L2-3) ------------------------
+ * Runs the DFA over nstreams independent streams, stream s = d_input[h_offsets[s]
+ * .. h_offsets[s+1]) (host array of nstreams+1 non-decreasing byte offsets; any
+ * alignment; empty streams allowed).  Each stream is split into chunks of
+ * opts->chunk_bytes (its last chunk may be short); its first chunk starts at q0,
+ * the others at the lookback-2 prediction; one thread per stream then
+ * verifies its chain and re-executes each mispredicted chunk from the verified
+ * state (Alg. 2 L7-11, with path fusion).  Outputs (device, caller-owned):
+ * d_final[s] (uint32 original id; == nstates marks a stream with a byte >= nsyms),
+ * d_count[s] (uint64 accept count, R3), d_chunk_ends (nullable; uint32 per chunk,
+ * streams' chunks in order, fsm_batch_chunks() entries).  Synchronous; returns
+ * FSM_ESYMBOL (outputs still written) if any stream saw an invalid byte. */
+typedef struct {
+  uint64_t nstreams, nchunks;
+  uint64_t recoveries;       /* mispredicted chunks re-executed (== chunks whose lookback
+                                prediction differs from the true start state)           */
+  uint64_t reread_bytes;     /* bytes those recoveries covered (nominal)                 */
+  uint64_t invalid_streams;  /* streams that saw an input byte >= nsyms                  */
+  float ms;                  /* device time of the call (CUDA events)                    */
+} fsm_batch_result;
+
+uint64_t fsm_batch_chunks(const uint64_t* h_offsets, uint32_t nstreams, uint32_t chunk_bytes);
+int fsm_run_batch(fsm_t fsm, const uint8_t* d_input, const uint64_t* h_offsets, uint32_t nstreams,
+                  const fsm_run_opts* opts, uint32_t* d_final, uint64_t* d_count, uint32_t* d_chunk_ends,
+                  fsm_batch_result* out);
 
 /* Same as fsm_run with HOST buffers: copies h_input to the device (pinned
  * memory recommended), runs, and copies chunk ends back to h_chunk_ends

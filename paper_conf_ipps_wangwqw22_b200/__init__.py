@@ -26,7 +26,7 @@ _lib = ctypes.CDLL(_LIB_PATH)
 FSM_OK, FSM_EINVAL, FSM_ENOMEM, FSM_ECUDA, FSM_ESYMBOL, FSM_ENCCL, FSM_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 SCHEMES = {"auto": 0, "seq": 1, "pm": 2, "sre": 3, "rr": 4, "nf": 5, "enum": 6}
 SCHEME_NAMES = {v: k for k, v in SCHEMES.items()}
-MODES = {1: "u8", 2: "u16", 3: "u32"}
+MODES = {1: "u8", 2: "u16", 3: "u32", 4: "u16d"}
 
 U32, U64, P = ctypes.c_uint32, ctypes.c_uint64, ctypes.c_void_p
 
@@ -49,6 +49,11 @@ class fsm_result(ctypes.Structure):
                 ("ms_verify", ctypes.c_double)]
 
 
+class fsm_batch_result(ctypes.Structure):
+    _fields_ = [("nstreams", U64), ("nchunks", U64), ("recoveries", U64), ("reread_bytes", U64),
+                ("invalid_streams", U64), ("ms", ctypes.c_float)]
+
+
 class fsm_features(ctypes.Structure):
     _fields_ = [("acc1", ctypes.c_double), ("acck", ctypes.c_double), ("input_sensitivity", ctypes.c_double),
                 ("uniq10", ctypes.c_double), ("nstates", U32)]
@@ -61,6 +66,9 @@ _lib.fsm_run.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POIN
 _lib.fsm_run_host.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
 _lib.fsm_run_async.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(U64)]
 _lib.fsm_wait.argtypes = [P, U64, ctypes.POINTER(fsm_result)]
+_lib.fsm_batch_chunks.argtypes = [P, U32, U32]
+_lib.fsm_batch_chunks.restype = U64
+_lib.fsm_run_batch.argtypes = [P, P, P, U32, ctypes.POINTER(fsm_run_opts), P, P, P, ctypes.POINTER(fsm_batch_result)]
 _lib.fsm_select_scheme.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), ctypes.POINTER(ctypes.c_int),
                                    ctypes.POINTER(fsm_features)]
 _lib.fsm_map_bytes.argtypes = [P]
@@ -255,6 +263,30 @@ class FSM:
         n = U32(0)
         _check(_lib.fsm_get_phase_times(self._h, us.ctypes.data, ctypes.byref(n)), "fsm_get_phase_times")
         return us[:n.value].copy()
+
+    def run_batch(self, x, offsets, chunk_bytes=4096, chunk_ends=False, stream=None):
+        """fsm_run_batch: independent streams x[offsets[s]:offsets[s+1]] (x: uint8 CUDA tensor,
+        offsets: host ints, len nstreams+1).  Returns (final int32 CUDA [ns], count int64 CUDA [ns],
+        chunk_ends int32 CUDA or None, stats dict).  final == nstates marks a stream with an
+        invalid byte (the call then raises GSpecError after filling the outputs)."""
+        import torch
+
+        assert x.is_cuda and x.dtype == torch.uint8 and x.is_contiguous()
+        off = np.ascontiguousarray(offsets, dtype=np.uint64)
+        ns = off.size - 1
+        assert ns >= 0 and (ns == 0 or int(off[-1]) <= x.numel())
+        o = _run_opts("sre", chunk_bytes, stream=stream)
+        nch = int(_lib.fsm_batch_chunks(off.ctypes.data, ns, chunk_bytes))
+        fin = torch.empty(max(ns, 1), dtype=torch.int32, device=x.device)
+        cnt = torch.empty(max(ns, 1), dtype=torch.int64, device=x.device)
+        ce = torch.empty(max(nch, 1), dtype=torch.int32, device=x.device) if chunk_ends else None
+        r = fsm_batch_result()
+        rc = _lib.fsm_run_batch(self._h, x.data_ptr() if x.numel() else None, off.ctypes.data, ns, ctypes.byref(o),
+                                fin.data_ptr(), cnt.data_ptr(), ce.data_ptr() if ce is not None else None,
+                                ctypes.byref(r))
+        stats = {k: getattr(r, k) for k, _ in fsm_batch_result._fields_}
+        _check(rc, "fsm_run_batch")
+        return fin[:ns], cnt[:ns], (ce[:nch] if ce is not None else None), stats
 
     def timeline(self):
         """(spec kernel, gap, verify kernel) in µs of the last collected run; -1 unless GSPEC_STAMPS=1."""

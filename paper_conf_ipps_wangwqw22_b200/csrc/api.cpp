@@ -349,6 +349,87 @@ int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_sche
   return run_collect(f, t, out, final_tid);
 }
 
+// Delta rows for MODE_U16D: a cold row of the transformed table
+// is stored as (hot base row, <= kDeltaExc exception classes) when it differs from
+// some hot row in that few columns — the rows of a literal/regex DFA's deep states
+// are their failure state's row plus a goto or two.  Picks the hot-row count H
+// that keeps the most frequency mass on chip within the smem budget
+// (hot rows C*2 B each + 8 B per delta row); used only when every cold real
+// row compresses.  The poison row (all poison) is stored once as hot row H.
+// Output: the shared-memory image [hot rows 0..H-1][poison row][pad][delta rows].
+bool plan_delta_rows(fsm_t f, const std::vector<uint32_t>& ttc, uint32_t nt, uint32_t C,
+                     const std::vector<uint32_t>& tid2code, uint32_t budget_in, DevImage* img,
+                     std::vector<uint2>* out) {
+  const uint32_t budget = budget_in ? budget_in : 128 * 1024;
+  const uint64_t row_b = (uint64_t)C * 2;
+  const uint32_t nr = nt - 1;  // real states (the poison tid nr is handled apart)
+  if (nr < 2 || row_b <= 8 || (uint64_t)nr * 8 + 2 * row_b + 32 > budget) return false;
+  uint64_t hmax = (budget - (uint64_t)nr * 8 - row_b - 32) / (row_b - 8);  // (H+1)*row + (nr-H)*8 <= budget
+  hmax = std::min<uint64_t>(hmax, std::min<uint64_t>(nr - 1, 0xFFFEu));  // base tids are 16-bit
+  if (hmax < 1) return false;
+  // first[t][d] = smallest j < min(t, hmax) whose row differs from row t in <= d columns
+  const uint32_t kNo = 0xFFFFFFFFu;
+  std::vector<uint32_t> first((uint64_t)nr * (kDeltaExc + 1), kNo);
+  for (uint32_t t = 1; t < nr; t++) {
+    const uint32_t* rt = &ttc[(uint64_t)t * C];
+    uint32_t* ft = &first[(uint64_t)t * (kDeltaExc + 1)];
+    const uint32_t jm = (uint32_t)std::min<uint64_t>(t, hmax);
+    for (uint32_t j = 0; j < jm && ft[0] == kNo; j++) {
+      const uint32_t* rj = &ttc[(uint64_t)j * C];
+      uint32_t d = 0;
+      for (uint32_t c = 0; c < C && d <= kDeltaExc; c++) d += rt[c] != rj[c];
+      for (uint32_t e = d; e <= kDeltaExc; e++)
+        if (ft[e] == kNo) ft[e] = j;
+    }
+  }
+  // smallest H with every real row hot or compressible (more room for TMA stages)
+  uint64_t H = 0;
+  for (uint64_t h = 1; h <= hmax && !H; h++) {
+    bool ok = true;
+    for (uint64_t t = h; t < nr && ok; t++) ok = first[t * (kDeltaExc + 1) + kDeltaExc] < h;
+    if (ok) H = h;
+  }
+  if (!H) return false;
+  if (const char* e = getenv("GSPEC_DELTA_H")) {  // experiments: a larger hot set (fewer delta lookups)
+    const uint64_t want = strtoull(e, nullptr, 10);
+    if (want > H) H = std::min<uint64_t>(want, hmax);
+  }
+  const uint64_t hot_b = (H + 1) * row_b;  // + the poison row as row H
+  const uint64_t delta_off = (hot_b + 15) & ~15ull;
+  const uint64_t bytes = (delta_off + (uint64_t)(nt - H) * 8 + 15) & ~15ull;
+  std::vector<uint16_t> im(bytes / 2, 0);
+  for (uint64_t t = 0; t < H; t++)
+    for (uint32_t c = 0; c < C; c++) im[t * C + c] = (uint16_t)tid2code[ttc[t * C + c]];
+  for (uint32_t c = 0; c < C; c++) im[H * C + c] = (uint16_t)tid2code[nr];
+  uint2* dl = reinterpret_cast<uint2*>(im.data() + delta_off / 2);
+  for (uint32_t t = (uint32_t)H; t < nt; t++) {
+    if (t == nr) {  // poison: base = the poison row, no exceptions
+      dl[t - H] = make_uint2((uint32_t)H | 0xFFFF0000u, 0);
+      continue;
+    }
+    const uint32_t* ft = &first[(uint64_t)t * (kDeltaExc + 1)];
+    uint32_t j = kNo;
+    for (uint32_t e = 0; e <= kDeltaExc && j == kNo; e++)
+      if (ft[e] < H) j = ft[e];
+    if (j == kNo) return false;  // unreachable (checked above)
+    uint32_t cls[kDeltaExc] = {0xFF, 0xFF}, code[kDeltaExc] = {0, 0}, k = 0;
+    for (uint32_t c = 0; c < C; c++)
+      if (ttc[(uint64_t)t * C + c] != ttc[(uint64_t)j * C + c]) {
+        cls[k] = c;
+        code[k] = tid2code[ttc[(uint64_t)t * C + c]];
+        k++;
+      }
+    dl[t - H] = make_uint2(j | (cls[0] << 16) | (cls[1] << 24), (code[0] & 0xFFFFu) | (code[1] << 16));
+  }
+  out->assign(reinterpret_cast<const uint2*>(im.data()), reinterpret_cast<const uint2*>(im.data()) + bytes / 8);
+  img->H = (uint32_t)H;
+  img->D = nt - (uint32_t)H;
+  img->delta_off = (uint32_t)delta_off;
+  img->smem_table_bytes = (uint32_t)bytes;
+  (void)f;
+  return true;
+}
+
 fsm_scheme tree_select(const fsm_features& ft, uint32_t n) {
   // Fig. 6 (image lost) reconstructed from P:284-290, P:339-345, P:383 (R19)
   if (n <= 31 && ft.uniq10 >= n / 2.0) return FSM_SCHEME_ENUM;
@@ -483,6 +564,9 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
   for (uint32_t t = 0; t < nt; t++) n_acc += acc_t[t];
   const uint32_t n_na = nt - n_acc;
   uint32_t force = opts ? opts->force_mode : 0;
+  if (force > 4) return bail(fail(FSM_EINVAL, "force_mode must be 0..4"));
+  const bool want_delta = force == 0 || force == 4;  // 4: u16 classed with delta rows
+  if (force == 4) force = MODE_U16;
   uint32_t mode;
   if (force) mode = force;
   else if (n_na <= 128 && n_acc <= 128) mode = MODE_U8;
@@ -531,6 +615,12 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
     img.H = (uint32_t)H;
     img.smem_table_bytes = (uint32_t)(((H * C * esz) + 15) & ~15ull);
     if (mode == MODE_U16 && H == nt) img.mode = MODE_U16H;  // every row hot: no hot test
+    std::vector<uint2> delta;
+    if (mode == MODE_U16 && H < nt && want_delta && C < 256 &&
+        plan_delta_rows(f, ttc, nt, C, tid2code, opts ? opts->smem_budget_bytes : 0, &img, &delta)) {
+      img.mode = MODE_U16D;
+      if ((rc = upload(f, &img.Dl, delta))) return bail(rc);
+    }
     if (mode == MODE_U16) {
       std::vector<uint16_t> T16((uint64_t)nt * C);
       for (uint64_t i = 0; i < T16.size(); i++) T16[i] = (uint16_t)tid2code[ttc[i]];
@@ -588,6 +678,9 @@ void fsm_free(fsm_t f) {
   if (f->h_dev_ce) cudaFree(f->h_dev_ce);
   if (f->d_small) cudaFree(f->d_small);
   if (f->shard_base) cudaFree(f->shard_base);
+  if (f->batch_base) cudaFree(f->batch_base);
+  for (auto& e : f->batch_ev)
+    if (e) cudaEventDestroy(e);
   delete f;
 }
 
@@ -657,6 +750,78 @@ int fsm_wait(fsm_t f, uint64_t ticket, fsm_result* out) {
   r.final_state = f->inv[fin];
   r.accept = f->accept[r.final_state];
   *out = r;
+  return FSM_OK;
+}
+
+uint64_t fsm_batch_chunks(const uint64_t* h_offsets, uint32_t nstreams, uint32_t chunk_bytes) {
+  if (!h_offsets) return 0;
+  const uint32_t B = chunk_bytes ? chunk_bytes : 4096;
+  uint64_t n = 0;
+  for (uint32_t s = 0; s < nstreams; s++)
+    if (h_offsets[s + 1] > h_offsets[s]) n += (h_offsets[s + 1] - h_offsets[s] + B - 1) / B;
+  return n;
+}
+
+int fsm_run_batch(fsm_t f, const uint8_t* d_input, const uint64_t* h_offsets, uint32_t nstreams,
+                  const fsm_run_opts* opts, uint32_t* d_final, uint64_t* d_count, uint32_t* d_chunk_ends,
+                  fsm_batch_result* out) {
+  entry_clear("fsm_run_batch");
+  if (!f || !out || !h_offsets) return fail(FSM_EINVAL, "NULL handle/offsets/out");
+  std::memset(out, 0, sizeof(*out));
+  if (nstreams == 0) return FSM_OK;
+  if (!d_final || !d_count) return fail(FSM_EINVAL, "NULL d_final/d_count");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  const uint32_t B = o.B;
+  std::vector<uint64_t> hb(2 * ((uint64_t)nstreams + 1));  // [offsets | chunk bases]
+  uint64_t N = 0;
+  for (uint32_t s = 0; s <= nstreams; s++) {
+    if (s < nstreams && h_offsets[s + 1] < h_offsets[s]) return fail(FSM_EINVAL, "offsets must be non-decreasing");
+    hb[s] = h_offsets[s];
+    hb[nstreams + 1 + s] = N;
+    if (s < nstreams) N += (h_offsets[s + 1] - h_offsets[s] + B - 1) / B;
+  }
+  if (N && !d_input) return fail(FSM_EINVAL, "NULL input");
+  auto al = [](uint64_t b) { return (b + 255) & ~255ull; };
+  const uint64_t need = al(hb.size() * 8) + 4 * al(N * 4 + 16) + al(gspec::batch_totals_bytes());
+  if (f->batch_bytes < need) {
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+    if (f->batch_base) cudaFree(f->batch_base);
+    f->batch_base = nullptr;
+    f->batch_bytes = 0;
+    CUDA_TRY(cudaMalloc(&f->batch_base, need));
+    f->batch_bytes = need;
+  }
+  if (!f->batch_ev[0]) {
+    CUDA_TRY(cudaEventCreate(&f->batch_ev[0]));
+    CUDA_TRY(cudaEventCreate(&f->batch_ev[1]));
+  }
+  uint8_t* p = reinterpret_cast<uint8_t*>(f->batch_base);
+  uint64_t* d_off = reinterpret_cast<uint64_t*>(p);
+  uint64_t* d_cb = d_off + nstreams + 1;
+  p += al(hb.size() * 8);
+  uint32_t* rs = reinterpret_cast<uint32_t*>(p); p += al(N * 4 + 16);
+  uint32_t* re = reinterpret_cast<uint32_t*>(p); p += al(N * 4 + 16);
+  uint32_t* rcn = reinterpret_cast<uint32_t*>(p); p += al(N * 4 + 16);
+  uint32_t* cs = reinterpret_cast<uint32_t*>(p); p += al(N * 4 + 16);  // chunk -> stream
+  void* tot = p;
+  CUDA_TRY(cudaMemcpyAsync(d_off, hb.data(), hb.size() * 8, cudaMemcpyHostToDevice, o.st));
+  CUDA_TRY(cudaMemsetAsync(tot, 0, gspec::batch_totals_bytes(), o.st));
+  CUDA_TRY(cudaEventRecord(f->batch_ev[0], o.st));
+  CUDA_TRY(gspec::launch_batch(f->img, d_input, d_off, d_cb, nstreams, N, B, cs, rs, re, rcn, d_final,
+                               reinterpret_cast<unsigned long long*>(d_count), d_chunk_ends, tot, o.st, f->sm_count));
+  CUDA_TRY(cudaEventRecord(f->batch_ev[1], o.st));
+  uint64_t t[3] = {0, 0, 0};  // recoveries, reread, invalid (BatchTotals layout)
+  CUDA_TRY(cudaMemcpyAsync(t, tot, sizeof(t), cudaMemcpyDeviceToHost, o.st));
+  CUDA_TRY(cudaStreamSynchronize(o.st));
+  out->nstreams = nstreams;
+  out->nchunks = N;
+  out->recoveries = t[0];
+  out->reread_bytes = t[1];
+  out->invalid_streams = t[2];
+  cudaEventElapsedTime(&out->ms, f->batch_ev[0], f->batch_ev[1]);
+  if (t[2]) return fail(FSM_ESYMBOL, "input symbol >= nsyms in some stream");
   return FSM_OK;
 }
 
@@ -757,7 +922,7 @@ int fsm_get_transform(fsm_t f, uint32_t* perm, uint32_t* inv, uint64_t* freq, ui
   if (perm) std::copy(f->perm.begin(), f->perm.end(), perm);
   if (inv) std::copy(f->inv.begin(), f->inv.end(), inv);
   if (freq) std::copy(f->freq.begin(), f->freq.end(), freq);
-  if (mode) *mode = f->img.mode == MODE_U16H ? (uint32_t)MODE_U16 : f->img.mode;
+  if (mode) *mode = f->img.mode == MODE_U16H ? (uint32_t)MODE_U16 : f->img.mode == MODE_U16D ? 4u : f->img.mode;
   if (hot_rows) *hot_rows = f->img.H;
   if (nclasses) *nclasses = f->img.C;
   return FSM_OK;

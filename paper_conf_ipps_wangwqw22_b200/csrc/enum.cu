@@ -71,7 +71,10 @@ __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* 
 }
 
 // K2: warp per group of kGroup maps: in-place inclusive prefix P_j = M_j o ... o M_g0,
-// and the group total written as one map of the next level.
+// and the group total written as one map of the next level.  The maps are loaded in
+// batches of kBatch (independent loads in flight) before the dependent shuffle chain
+// consumes them, so a group costs kGroup / kBatch memory round trips, not kGroup.
+constexpr int kBatch = 8;
 __global__ void __launch_bounds__(128) k_enum_group(uint8_t* __restrict__ M, uint64_t* __restrict__ Cn, uint64_t cnt,
                                                    uint8_t* __restrict__ Mup, uint64_t* __restrict__ Cup) {
   const uint32_t lane = threadIdx.x & 31;
@@ -81,19 +84,24 @@ __global__ void __launch_bounds__(128) k_enum_group(uint8_t* __restrict__ M, uin
     uint32_t P = lane;
     uint64_t PC = 0;
     const uint64_t j0 = g * kGroup, j1 = min(cnt, j0 + kGroup);
-    uint32_t m = M[j0 * 32 + lane];
-    uint64_t c = Cn[j0 * 32 + lane];
-    for (uint64_t j = j0; j < j1; j++) {
-      uint32_t mn = 0;
-      uint64_t cn = 0;
-      if (j + 1 < j1) { mn = M[(j + 1) * 32 + lane]; cn = Cn[(j + 1) * 32 + lane]; }  // prefetch
-      const uint32_t nP = __shfl_sync(0xffffffffu, m, P);
-      PC += __shfl_sync(0xffffffffu, c, P);
-      P = nP;
-      M[j * 32 + lane] = (uint8_t)P;
-      Cn[j * 32 + lane] = PC;
-      m = mn;
-      c = cn;
+    for (uint64_t jb = j0; jb < j1; jb += kBatch) {
+      uint32_t m[kBatch];
+      uint64_t c[kBatch];
+#pragma unroll
+      for (int u = 0; u < kBatch; u++) {
+        const uint64_t j = min(jb + u, j1 - 1);
+        m[u] = M[j * 32 + lane];
+        c[u] = Cn[j * 32 + lane];
+      }
+#pragma unroll
+      for (int u = 0; u < kBatch; u++) {
+        if (jb + u >= j1) break;
+        const uint32_t nP = __shfl_sync(0xffffffffu, m[u], P);
+        PC += __shfl_sync(0xffffffffu, c[u], P);
+        P = nP;
+        M[(jb + u) * 32 + lane] = (uint8_t)P;
+        Cn[(jb + u) * 32 + lane] = PC;
+      }
     }
     if (Mup) {
       Mup[g * 32 + lane] = (uint8_t)P;
@@ -207,6 +215,7 @@ cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t 
     case MODE_U8: e = walk_m<MODE_U8>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
     case MODE_U16: e = walk_m<MODE_U16>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
     case MODE_U16H: e = walk_m<MODE_U16H>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
+    case MODE_U16D: e = walk_m<MODE_U16D>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
     default: e = walk_m<MODE_U32>(img, rp, E, nsub, lv[0].M, lv[0].C, st, sms); break;
   }
   if (e != cudaSuccess) return e;

@@ -20,7 +20,11 @@ enum Mode : uint32_t {
   MODE_U16 = 2,  // classed table, u16 codes = tid | acc<<15, hot rows (tid < H) in smem
   MODE_U32 = 3,  // classed table, u32 codes = tid | acc<<31, hot rows in smem
   MODE_U16H = 4, // MODE_U16 with every row in smem: no hot test on the lookup path
+  MODE_U16D = 5, // MODE_U16 whose cold rows are delta rows in smem: a hot base row + <= 2
+                 // exceptions (8 B each); chosen only when every cold row compresses
 };
+
+constexpr uint32_t kDeltaExc = 2;        // exceptions per delta row
 
 constexpr uint32_t kQsMax = 16;     // QS cap ("top 16 states")
 constexpr uint32_t kVrMax = 16;     // VR^end / VR^others slots
@@ -47,6 +51,12 @@ struct DevImage {
   const uint32_t* code2tid;   // MODE_U8: [256]
   const uint32_t* inv;        // [nt] tid -> original id (poison -> n)
   const uint8_t* acc;         // [nt] accept by tid
+  // MODE_U16D: the whole shared-memory table image [hot rows 0..H-1][poison row (= row H)]
+  // [pad][delta rows of tids H..nt-1]; delta row: x = base tid | cls0 << 16 | cls1 << 24,
+  // y = code0 | code1 << 16 (unused exception: class 0xFF)
+  const uint2* Dl;
+  uint32_t delta_off;         // byte offset of the delta rows behind the hot rows (16-aligned)
+  uint32_t D;                 // delta rows (= nt - H)
 };
 
 // Global record store (hierarchical store, level 3).
@@ -226,6 +236,12 @@ cudaError_t launch_features_raw(const DevImage& img, const uint32_t* d_ttc, cons
                                 unsigned long long* d_counts, uint32_t* d_seen, unsigned long long* d_uniq,
                                 cudaStream_t st);
 
+uint64_t batch_totals_bytes();
+cudaError_t launch_batch(const DevImage& img, const uint8_t* in, const uint64_t* off, const uint64_t* cbase,
+                         uint32_t ns, uint64_t N, uint32_t B, uint32_t* cs, uint32_t* rs, uint32_t* re, uint32_t* rc,
+                         uint32_t* fin,
+                         unsigned long long* count, uint32_t* chunk_ends, void* tot, cudaStream_t st, int sms);
+
 cudaError_t launch_shard_image(const DevImage& img, const uint32_t* ttc, const uint8_t* w, uint32_t L, uint32_t* mark,
                                uint32_t* list, uint32_t* count, cudaStream_t st);
 cudaError_t launch_shard_fuse(const DevImage& img, const uint8_t* in, uint64_t len, uint32_t B, const uint32_t* cand,
@@ -312,6 +328,9 @@ struct fsm_s {
   uint32_t last_nstamp = 0;            // verify phase timestamps of the last collected run
   uint64_t last_stamp[24] = {};
   uint64_t last_tl[4] = {};             // run timeline of the last collected run (GSPEC_STAMPS=1)
+  void* batch_base = nullptr;            // fsm_run_batch scratch (offsets, chunk bases, records, totals)
+  size_t batch_bytes = 0;
+  cudaEvent_t batch_ev[2] = {nullptr, nullptr};
   const uint8_t* shard_in = nullptr;
   uint64_t shard_len = 0;
   uint32_t shard_ncand = 0, shard_nj = 0;  // candidates; chunks covered by the fused prefix

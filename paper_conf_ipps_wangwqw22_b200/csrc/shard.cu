@@ -267,6 +267,7 @@ cudaError_t launch_shard_fuse(const DevImage& img, const uint8_t* in, uint64_t l
     case MODE_U8: return fuse_m<MODE_U8>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
     case MODE_U16: return fuse_m<MODE_U16>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
     case MODE_U16H: return fuse_m<MODE_U16H>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
+    case MODE_U16D: return fuse_m<MODE_U16D>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
     default: return fuse_m<MODE_U32>(img, in, len, B, cand, ncand, max_chunks, states, cnt, info, st);
   }
 }
@@ -283,6 +284,7 @@ cudaError_t launch_shard_fuse_ref(const DevImage& img, const uint8_t* in, uint64
     case MODE_U8: GS_FUSE_REF(MODE_U8); break;
     case MODE_U16: GS_FUSE_REF(MODE_U16); break;
     case MODE_U16H: GS_FUSE_REF(MODE_U16H); break;
+    case MODE_U16D: GS_FUSE_REF(MODE_U16D); break;
     default: GS_FUSE_REF(MODE_U32); break;
   }
 #undef GS_FUSE_REF

@@ -173,6 +173,7 @@ cudaError_t launch_spec_generic(const DevImage& img, const RunParams& rp, const 
     case MODE_U8: return launch_mode<MODE_U8>(img, rp, rs, st, c0);
     case MODE_U16: return launch_mode<MODE_U16>(img, rp, rs, st, c0);
     case MODE_U16H: return launch_mode<MODE_U16H>(img, rp, rs, st, c0);
+    case MODE_U16D: return launch_mode<MODE_U16D>(img, rp, rs, st, c0);
     default: return launch_mode<MODE_U32>(img, rp, rs, st, c0);
   }
 }

@@ -334,6 +334,7 @@ cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecS
     case MODE_U8: e = launch_tma_m<MODE_U8>(tm, img, rp, rs, n_full, sms, st); break;
     case MODE_U16: e = launch_tma_m<MODE_U16>(tm, img, rp, rs, n_full, sms, st); break;
     case MODE_U16H: e = launch_tma_m<MODE_U16H>(tm, img, rp, rs, n_full, sms, st); break;
+    case MODE_U16D: e = launch_tma_m<MODE_U16D>(tm, img, rp, rs, n_full, sms, st); break;
     default: e = launch_tma_m<MODE_U32>(tm, img, rp, rs, n_full, sms, st); break;
   }
   if (e == cudaSuccess) *n_done = n_full;
@@ -352,6 +353,7 @@ cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecS
     case MODE_U8: e = launch_tma_s<MODE_U8, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
     case MODE_U16: e = launch_tma_s<MODE_U16, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
     case MODE_U16H: e = launch_tma_s<MODE_U16H, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
+    case MODE_U16D: e = launch_tma_s<MODE_U16D, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
     default: e = launch_tma_s<MODE_U32, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
   }
   if (e == cudaSuccess) *n_done = n_full;

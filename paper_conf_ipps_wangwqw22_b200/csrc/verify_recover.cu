@@ -915,6 +915,7 @@ cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp_in, const
     case MODE_U8: return launch_dense_finish<MODE_U8>(img, rp, rs, ctl, done, st);
     case MODE_U16: return launch_dense_finish<MODE_U16>(img, rp, rs, ctl, done, st);
     case MODE_U16H: return launch_dense_finish<MODE_U16H>(img, rp, rs, ctl, done, st);
+    case MODE_U16D: return launch_dense_finish<MODE_U16D>(img, rp, rs, ctl, done, st);
     default: return launch_dense_finish<MODE_U32>(img, rp, rs, ctl, done, st);
   }
 }
@@ -928,6 +929,7 @@ cudaError_t launch_verify_recover(const DevImage& img, const RunParams& rp, cons
     case MODE_U8: return launch_m<MODE_U8>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
     case MODE_U16: return launch_m<MODE_U16>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
     case MODE_U16H: return launch_m<MODE_U16H>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
+    case MODE_U16D: return launch_m<MODE_U16D>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
     default: return launch_m<MODE_U32>(img, rp, rs, d_ctl, d_block_tmp, d_chunk_ends, st, sm_count);
   }
 }

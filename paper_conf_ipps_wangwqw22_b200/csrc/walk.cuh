@@ -14,12 +14,13 @@ namespace gspec {
 // (the class map first keeps it 256-aligned: its address is one PRMT away).
 __device__ __forceinline__ void stage_table(const DevImage& img, uint8_t* smem) {
   const uint4* src = (img.mode == MODE_U8)                                 ? reinterpret_cast<const uint4*>(img.T8)
-                     : (img.mode == MODE_U16 || img.mode == MODE_U16H) ? reinterpret_cast<const uint4*>(img.T16)
+                     : (img.mode == MODE_U16 || img.mode == MODE_U16H || img.mode == MODE_U16D) ? reinterpret_cast<const uint4*>(img.T16)
                                                                          : reinterpret_cast<const uint4*>(img.T32);
   const uint32_t off = img.mode == MODE_U8 ? 0u : 256u;
   uint4* dst = reinterpret_cast<uint4*>(smem + off);
+  const uint4* from = img.mode == MODE_U16D ? reinterpret_cast<const uint4*>(img.Dl) : src;  // u16d: its own image
   const uint32_t nv = img.smem_table_bytes / 16;
-  for (uint32_t i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(src + i);
+  for (uint32_t i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(from + i);
   if (img.mode != MODE_U8) {
     const uint4* cs = reinterpret_cast<const uint4*>(img.cls);
     uint4* cd = reinterpret_cast<uint4*>(smem);
@@ -111,8 +112,54 @@ struct StepClassed {
   static __device__ __forceinline__ uint32_t tid(const DevImage&, uint32_t code) { return code & kMask; }
 };
 
+__device__ __forceinline__ uint2 lds_u64(uint32_t saddr) {
+  uint2 v;
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(saddr));
+  return v;
+}
+
+// MODE_U16D: a cold tid (>= H) reads its 8-byte delta row {hot base tid, 2 exception
+// classes, 2 exception codes}; a hot tid acts as its own base with no exceptions.
+// Branch-free: the delta-row load is predicated on the cold lanes only (hot lanes
+// generate no shared-memory traffic for it), then every lane reads one row entry
+// (its own row or its base row) and the exceptions override by select — two
+// dependent shared-memory loads, no L2 trip, no divergence.  fsm_load picks this
+// mode only when every cold row compresses.  (Measured on C4: a hot/cold branch
+// cost 28 instructions per warp-step with 90% of warp-steps divergent; loading a
+// descriptor for every lane cost 4.7 wavefronts per LDS.64.)
+struct StepDelta {
+  static constexpr uint32_t kShift = 15;
+  static constexpr uint32_t kMask = 0x7FFFu;
+  static __device__ __forceinline__ uint32_t row(const DevImage& img, uint32_t base, uint32_t code, uint32_t cl) {
+    const uint32_t t = code & kMask;
+    uint32_t dx = t | 0xFFFF0000u, dy = 0;  // hot: base = t, exception classes 0xFF (none)
+    const uint32_t da = base + 256 + img.delta_off + (t - img.H) * 8;
+    asm volatile(
+        "{\n .reg .pred p;\n setp.ge.u32 p, %2, %3;\n @p ld.shared.v2.u32 {%0, %1}, [%4];\n}\n"
+        : "+r"(dx), "+r"(dy)
+        : "r"(t), "r"(img.H), "r"(da));
+    uint32_t v = lds_u16(base + 256 + ((dx & 0xFFFFu) * img.C + cl) * 2);
+    v = (cl == (dx >> 24)) ? (dy >> 16) : v;
+    v = (cl == ((dx >> 16) & 0xFFu)) ? (dy & 0xFFFFu) : v;
+    return v;
+  }
+  static __device__ __forceinline__ uint32_t byte(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t b) {
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
+    return row(img, base, code, lds_u8(base + b));
+  }
+  template <int K>
+  static __device__ __forceinline__ uint32_t word(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t w) {
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
+    return row(img, base, code, lds_u8(byte_plus<K>(w, base)));
+  }
+  static __device__ __forceinline__ uint32_t acc(uint32_t code) { return code >> 15; }
+  static __device__ __forceinline__ uint32_t tid(const DevImage&, uint32_t code) { return code & kMask; }
+};
+
 template <>
 struct Step<MODE_U16> : StepClassed<uint16_t, 15, false> {};
+template <>
+struct Step<MODE_U16D> : StepDelta {};
 template <>
 struct Step<MODE_U16H> : StepClassed<uint16_t, 15, true> {};
 template <>
@@ -124,8 +171,17 @@ __device__ __forceinline__ uint32_t walk_bytes(const DevImage& img, const uint8_
                                                uint32_t code, uint32_t& acc) {
   using S = Step<MODE>;
   uint64_t i = 0;
-  // vector part when 16-byte aligned
-  if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
+  // unaligned start: walk the head bytes one by one up to the next 16-byte boundary
+  const uint64_t head = min(n, (uint64_t)((16u - (reinterpret_cast<uintptr_t>(p) & 15u)) & 15u));
+  for (; i < head; i++) {
+    code = S::byte(img, s, code, __ldg(p + i));
+    acc += S::acc(code);
+  }
+  p += head;
+  n -= head;
+  i = 0;
+  // vector part (16-byte aligned now)
+  {
     const uint4* v = reinterpret_cast<const uint4*>(p);
     const uint64_t nv = n / 16;
     // software pipeline: two 16-byte loads in flight ahead of the dependent chain

@@ -55,6 +55,12 @@ def test_host_only_calls(lib):
     assert lib.fsm_num_chunks(4097, 4096) == 2
     assert lib.fsm_num_chunks(100, 0) == 1  # 0 -> default 4096
     assert lib._lib.fsm_strerror(-4) == b"input symbol out of range"
+    import numpy as np
+
+    off = np.array([0, 0, 1, 4096, 4096 + 4097, 9000, 9000], np.uint64)  # empty, 1 B, 1 chunk, 2 chunks, short, empty
+    assert lib._lib.fsm_batch_chunks(off.ctypes.data, 6, 4096) == 0 + 1 + 1 + 2 + 1 + 0
+    assert lib._lib.fsm_batch_chunks(off.ctypes.data, 6, 16) == sum(
+        (int(off[i + 1]) - int(off[i]) + 15) // 16 for i in range(6))
 
 
 def test_binding_never_imports_oracle():

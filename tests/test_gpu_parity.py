@@ -320,3 +320,31 @@ def test_inline_round0_recovery(gs, name, length, vr_end):
         assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
     if name != "c2":
         assert res.stats["tasks_sre"] > 0  # mispredictions really happened
+
+
+@pytest.mark.parametrize("name,length,budget", [("c4", 4 << 20, 0), ("c4", 2 << 20, 48 * 1024), ("c3", 2 << 20, 0),
+                                                ("c2", 2 << 20, 0), ("c2", 1 << 20, 2048),
+                                                ("rand:300:60:7", 1 << 20, 8192)])
+def test_delta_rows(gs, name, length, budget):
+    """u16 table whose cold rows are delta rows in smem (hot base row + <= 2 exceptions,
+    the poison row as an extra hot row); when some row does not compress within the
+    budget the plain hot/cold split is used — every scheme stays bit-exact."""
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, 4096)
+    fsm = gs.FSM.load(w.table, w.start, w.accept, force_mode=4, smem_budget=budget)
+    tr = fsm.transform()
+    if tr["mode"] == "u16d":
+        assert tr["hot_rows"] < w.nstates + 1
+    x = torch.from_numpy(data).cuda()
+    for scheme in ("sre", "nf", "pm"):
+        res = fsm.run(x, scheme=scheme)
+        check_equal(res, ref, 4096, w.nstates)
+    res = fsm.run(x[5:], scheme="sre", chunk_bytes=48)  # generic (unaligned) kernel, many tasks
+    ref2 = oracle.run(w.table, w.start, w.accept, data[5:], 48)
+    check_equal(res, ref2, 48, w.nstates)
+
+
+def test_c4_auto_picks_delta_rows(gs):
+    w, _ = _wl("c4", 1 << 16)
+    tr = gs.FSM.load(w.table, w.start, w.accept).transform()
+    assert tr["mode"] == "u16d" and tr["hot_rows"] < 2048
