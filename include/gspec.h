@@ -92,6 +92,7 @@ typedef struct {
   uint64_t verify_checks, verify_matches; /* runtime speculation accuracy    */
   double avg_active_workers; /* mean active workers per round (Table III analogue)    */
   double ms_spec, ms_verify; /* device time of speculative execution / verify+recover */
+  uint32_t kernel_launches;  /* kernels this run launched (spec, verify, dense rounds, ENUM levels) */
 } fsm_result;
 
 typedef struct {

@@ -46,7 +46,7 @@ class fsm_result(ctypes.Structure):
                 ("scheme_used", ctypes.c_int), ("rounds", U32), ("tasks_total", U64), ("tasks_mustdo", U64),
                 ("tasks_sre", U64), ("tasks_helper", U64), ("reread_bytes", U64), ("verify_checks", U64),
                 ("verify_matches", U64), ("avg_active_workers", ctypes.c_double), ("ms_spec", ctypes.c_double),
-                ("ms_verify", ctypes.c_double)]
+                ("ms_verify", ctypes.c_double), ("kernel_launches", U32)]
 
 
 class fsm_batch_result(ctypes.Structure):

@@ -274,6 +274,9 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
     CUDA_TRY(launch_enum_full(f->img, rp, E, f->enum_base, d_chunk_ends, f->d_ctl, &f->d_ctl->xfin, o.st,
                               f->sm_count));
+    uint32_t L = 1;  // map levels: walk + L group scans + L descents + outputs
+    for (uint64_t c = nsub; c > 64 && L < 16; c = (c + 63) / 64) L++;
+    pd.launches = 2 + 2 * L;
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   } else {
@@ -288,10 +291,16 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     rp.dense = (scheme == FSM_SCHEME_SRE && len / o.B > 0 && o.B % 64 == 0 &&
                 (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0 && f->acc1_hint < 0.5) ? 1u : 0u;
     CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
+    {  // TMA kernel over the full chunks + the generic kernel for a tail chunk (or everything)
+      const bool tma = !spec_path_generic_only() && len / o.B > 0 && o.B % 64 == 0 &&
+                       (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0;
+      pd.launches = tma ? 1 + (len % o.B != 0) : 1;
+    }
     rp.ctl_init = nullptr;  // initialised by the spec kernel; later launches must not touch it
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
     for (;;) {
       CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
+      pd.launches++;
       if (!rp.dense) break;
       uint32_t pend = 0;
       uint64_t fm = 0;
@@ -300,6 +309,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       CUDA_TRY(cudaStreamSynchronize(o.st));
       if (!pend) break;
       CUDA_TRY(launch_task_dense(f->img, rp, f->rs, f->d_ctl, fm, f->sm_count, o.st));
+      pd.launches += 2;  // TMA task kernel + finish
     }
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   }
@@ -337,6 +347,7 @@ int run_collect(fsm_t f, uint64_t ticket, fsm_result* out, uint32_t* final_tid) 
   out->accept_count = h.accept_count;
   out->ms_spec = t1;
   out->ms_verify = t2;
+  out->kernel_launches = pd.launches;
   *final_tid = h.xfin;
   return FSM_OK;
 }

@@ -37,20 +37,35 @@ __global__ void __launch_bounds__(256) k_batch_spec(DevImage img, const uint8_t*
   stage_table(img, smem);
   __syncthreads();
   using S = Step<MODE>;
-  for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < N; c += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t s = __ldg(cs + c);
-    const uint64_t k = c - __ldg(cbase + s);
-    const uint64_t lo = __ldg(off + s) + k * B, hi = min(lo + B, __ldg(off + s + 1));
-    uint32_t st = q0t;
-    if (k > 0) {  // lookback-2 over the previous chunk's last two bytes (same stream, B >= 16)
-      const uint32_t pair = (uint32_t)__ldg(img.cls + __ldg(in + lo - 2)) * img.C + __ldg(img.cls + __ldg(in + lo - 1));
-      st = __ldg(img.qs2 + (uint64_t)pair * kQsMax);
+  // two chunks per thread (2g, 2g+1), walked interleaved for ILP
+  for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; 2 * g < N; g += (uint64_t)gridDim.x * blockDim.x) {
+    uint64_t lo[2], hi[2];
+    uint32_t st[2], code[2], acc[2] = {0, 0};
+#pragma unroll
+    for (int i = 0; i < 2; i++) {
+      const uint64_t c = min(2 * g + i, N - 1);  // odd N: the last thread walks its chunk twice
+      const uint32_t s = __ldg(cs + c);
+      const uint64_t k = c - __ldg(cbase + s);
+      lo[i] = __ldg(off + s) + k * B;
+      hi[i] = min(lo[i] + B, __ldg(off + s + 1));
+      st[i] = q0t;
+      if (k > 0) {  // lookback-2 over the previous chunk's last two bytes (same stream, B >= 16)
+        const uint32_t pair =
+            (uint32_t)__ldg(img.cls + __ldg(in + lo[i] - 2)) * img.C + __ldg(img.cls + __ldg(in + lo[i] - 1));
+        st[i] = __ldg(img.qs2 + (uint64_t)pair * kQsMax);
+      }
+      code[i] = __ldg(img.tid2code + st[i]);
     }
-    uint32_t acc = 0;
-    const uint32_t code = walk_bytes<MODE>(img, smem, in + lo, hi - lo, __ldg(img.tid2code + st), acc);
-    rstart[c] = st;
-    rend[c] = S::tid(img, code);
-    rcnt[c] = acc;
+    walk2_bytes<MODE>(img, smem, in + lo[0], hi[0] - lo[0], code[0], acc[0], in + lo[1], hi[1] - lo[1], code[1],
+                      acc[1]);
+#pragma unroll
+    for (int i = 0; i < 2; i++) {
+      const uint64_t c = 2 * g + i;
+      if (c >= N) break;
+      rstart[c] = st[i];
+      rend[c] = S::tid(img, code[i]);
+      rcnt[c] = acc[i];
+    }
   }
 }
 
@@ -190,7 +205,7 @@ cudaError_t launch_batch_m(const DevImage& img, const uint8_t* in, const uint64_
   if (N > 0) {
     k_batch_map<<<(unsigned)std::min<uint64_t>((ns + 255) / 256, (uint64_t)sms * 8), 256, 0, st>>>(cbase, ns, cs);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
-    uint64_t grid = std::min<uint64_t>((N + 255) / 256, (uint64_t)sms * std::max(occ, 1));
+    uint64_t grid = std::min<uint64_t>((N / 2 + 256) / 256, (uint64_t)sms * std::max(occ, 1));
     k1<<<(unsigned)std::max<uint64_t>(grid, 1), 256, smem, st>>>(img, in, off, cbase, cs, N, B, img.q0t, rs, re, rc);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }

@@ -209,6 +209,43 @@ __device__ __forceinline__ uint32_t walk_bytes(const DevImage& img, const uint8_
   return code;
 }
 
+// Two independent walks interleaved (ILP 2) over arbitrarily aligned ranges: heads
+// byte by byte, then both 16-byte-aligned bodies in lockstep, then each one's rest.
+template <int MODE>
+__device__ __forceinline__ void walk2_bytes(const DevImage& img, const uint8_t* s, const uint8_t* p0, uint64_t n0,
+                                            uint32_t& c0, uint32_t& a0, const uint8_t* p1, uint64_t n1, uint32_t& c1,
+                                            uint32_t& a1) {
+  using S = Step<MODE>;
+  const uint64_t h0 = min(n0, (uint64_t)((16u - (reinterpret_cast<uintptr_t>(p0) & 15u)) & 15u));
+  const uint64_t h1 = min(n1, (uint64_t)((16u - (reinterpret_cast<uintptr_t>(p1) & 15u)) & 15u));
+  for (uint64_t i = 0; i < h0; i++) { c0 = S::byte(img, s, c0, __ldg(p0 + i)); a0 += S::acc(c0); }
+  for (uint64_t i = 0; i < h1; i++) { c1 = S::byte(img, s, c1, __ldg(p1 + i)); a1 += S::acc(c1); }
+  p0 += h0; n0 -= h0;
+  p1 += h1; n1 -= h1;
+  const uint64_t nb = min(n0, n1) / 16;
+  const uint4* v0 = reinterpret_cast<const uint4*>(p0);
+  const uint4* v1 = reinterpret_cast<const uint4*>(p1);
+  uint4 q0 = nb > 0 ? __ldg(v0) : make_uint4(0, 0, 0, 0), q1 = nb > 0 ? __ldg(v1) : make_uint4(0, 0, 0, 0);
+  for (uint64_t j = 0; j < nb; j++) {
+    const uint4 x0 = q0, x1 = q1;
+    if (j + 1 < nb) { q0 = __ldg(v0 + j + 1); q1 = __ldg(v1 + j + 1); }
+    const uint32_t w0[4] = {x0.x, x0.y, x0.z, x0.w}, w1[4] = {x1.x, x1.y, x1.z, x1.w};
+#pragma unroll
+    for (int t = 0; t < 4; t++) {
+      c0 = S::template word<0>(img, s, c0, w0[t]); a0 += S::acc(c0);
+      c1 = S::template word<0>(img, s, c1, w1[t]); a1 += S::acc(c1);
+      c0 = S::template word<1>(img, s, c0, w0[t]); a0 += S::acc(c0);
+      c1 = S::template word<1>(img, s, c1, w1[t]); a1 += S::acc(c1);
+      c0 = S::template word<2>(img, s, c0, w0[t]); a0 += S::acc(c0);
+      c1 = S::template word<2>(img, s, c1, w1[t]); a1 += S::acc(c1);
+      c0 = S::template word<3>(img, s, c0, w0[t]); a0 += S::acc(c0);
+      c1 = S::template word<3>(img, s, c1, w1[t]); a1 += S::acc(c1);
+    }
+  }
+  c0 = walk_bytes<MODE>(img, s, p0 + nb * 16, n0 - nb * 16, c0, a0);
+  c1 = walk_bytes<MODE>(img, s, p1 + nb * 16, n1 - nb * 16, c1, a1);
+}
+
 // PDL (see internal.h): wait for the preceding grid (a no-op without a
 // programmatic dependency), and let the next grid in the stream launch.
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
