@@ -10,6 +10,7 @@ Usage: python build.py [--force] [--only gen|oracle|gspec]
 """
 from __future__ import annotations
 
+import concurrent.futures
 import glob
 import os
 import shutil
@@ -70,14 +71,19 @@ def build_gspec(force=False):
         return
     objdir = os.path.join(ROOT, "build", "gspec")
     os.makedirs(objdir, exist_ok=True)
-    objs = []
+    objs, cmds = [], []
+    hdrs = glob.glob(os.path.join(csrc, "*.h")) + glob.glob(os.path.join(csrc, "*.cuh")) + \
+        [os.path.join(ROOT, "include", "gspec.h")]
     for s in srcs:
         o = os.path.join(objdir, os.path.basename(s) + ".o")
-        hdrs = glob.glob(os.path.join(csrc, "*.h")) + glob.glob(os.path.join(csrc, "*.cuh")) + \
-            [os.path.join(ROOT, "include", "gspec.h")]
         if force or _stale(o, [s] + hdrs):
-            _run([NVCC] + NVFLAGS + ["-I", os.path.join(ROOT, "include"), "-I", csrc, "-rdc=false", "-c", s, "-o", o])
+            cmds.append([NVCC] + NVFLAGS + ["-I", os.path.join(ROOT, "include"), "-I", csrc, "-rdc=false", "-c", s,
+                                            "-o", o])
         objs.append(o)
+    # translation units are independent: compile them in parallel
+    with concurrent.futures.ThreadPoolExecutor(max_workers=max(1, min(len(cmds), os.cpu_count() or 1))) as ex:
+        for fut in [ex.submit(_run, c) for c in cmds]:
+            fut.result()
     _run([NVCC] + ARCH + ["-shared", "-o", out] + objs + ["-ldl"])
 
 

@@ -303,12 +303,13 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       pd.launches++;
       if (!rp.dense) break;
       uint32_t pend = 0;
-      uint64_t fm = 0;
+      uint64_t fm = 0, nt = 0;
       CUDA_TRY(cudaMemcpyAsync(&pend, &f->d_ctl->dense_pending, 4, cudaMemcpyDeviceToHost, o.st));
       CUDA_TRY(cudaMemcpyAsync(&fm, &f->d_ctl->fmin, 8, cudaMemcpyDeviceToHost, o.st));
+      CUDA_TRY(cudaMemcpyAsync(&nt, &f->d_ctl->ntask[0], 8, cudaMemcpyDeviceToHost, o.st));
       CUDA_TRY(cudaStreamSynchronize(o.st));
       if (!pend) break;
-      CUDA_TRY(launch_task_dense(f->img, rp, f->rs, f->d_ctl, fm, f->sm_count, o.st));
+      CUDA_TRY(launch_task_dense(f->img, rp, f->rs, f->d_ctl, fm, nt, f->sm_count, o.st));
       pd.launches += 2;  // TMA task kernel + finish
     }
     CUDA_TRY(cudaEventRecord(ev[2], o.st));

@@ -103,7 +103,7 @@ struct Ctl {
   uint64_t accept_count;
   uint64_t nA, I, nU;    // this round: A-tasks, idle workers, total untried candidates
   uint64_t jacobi_iters;
-  uint64_t ntask[2];     // (unused, kept for layout)
+  uint64_t ntask[2];     // [0]: length of the task list handed to a dense round; [1] unused
   uint64_t it_fm[3], it_checks[3], it_matches[3], it_ntask[3];  // per relaxation pass (rotating)
   uint64_t it_reread[3];  // round-0 SRE pass with inline tasks: bytes re-walked (rotating)
   uint32_t dense_pending;  // verify exited: a dense task round (frontier fmin) must run first
@@ -220,10 +220,11 @@ cudaError_t launch_build_qs2_raw(const uint32_t* d_ttc, uint32_t n, uint32_t C, 
 cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st);
 cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, int sms, cudaStream_t st,
                             uint64_t* n_done);
-// Dense recovery round: every chunk c >= f2 with rs.tstart[c] != none is re-walked from that
-// start by the TMA-staged kernel (full chunks) and the tail kernel; then the round is committed.
+// Dense recovery round: the round's task list (rs.task_chunk/task_start, ntask entries, all
+// chunks >= f2) is re-walked by the TMA-gather task kernel (full chunks) and the tail kernel
+// (rs.tstart of the partial last chunk); then the round is committed.
 cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
-                              int sms, cudaStream_t st);
+                              uint64_t ntask, int sms, cudaStream_t st);
 bool spec_path_generic_only();  // GSPEC_SPEC_PATH=generic forces the non-TMA kernel (A/B tests)
 cudaError_t launch_verify_recover(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* d_ctl,
                                   uint64_t* d_block_tmp, uint32_t* d_chunk_ends, cudaStream_t st, int sm_count);

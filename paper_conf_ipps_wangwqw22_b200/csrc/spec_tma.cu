@@ -62,13 +62,30 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       : "memory");
 }
 
+// Blackwell TMA gather: 4 arbitrary rows (chunks) x one 64 B box column.  With
+// SWIZZLE_64B the rows land with the same address-based XOR pattern as a 32-row
+// 2-D box (tools/gather4_probe.cu verified this at 256 B destination offsets), so
+// 8 gathers fill a stage exactly like one tile box and the readers are unchanged.
+__device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, uint64_t* bar, int32_t x, uint4 r,
+                                            uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%2, %3, %4, %5, %6}], [%7], %8;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(r.x), "r"(r.y), "r"(r.z), "r"(r.w), "r"(smem_u32(bar)),
+      "l"(policy)
+      : "memory");
+}
+
 // TASKS = false: round 0 (starts from the lookback pair table).  TASKS = true: a dense
-// recovery round (Alg. 3 L16-18 for most chunks at once): chunk c >= f2 re-walks from
-// rs.tstart[c] (if set) and appends its record to VR^end.
+// recovery round (Alg. 3 L16-18 for many chunks at once): the round's task list
+// (rs.task_chunk / rs.task_start, ntask entries, listed by the verification pass) is
+// cut into groups of 32 tasks, one per lane; each stage gathers the 32 chunks' next
+// 64 B with 8 TMA gather4 loads (tmap is then the {64 B x 1 row} gather map), so a
+// round walks only the chunks that have a task.  Each task appends its record to VR^end.
 template <int MODE, int KP, int S, bool TASKS>
 __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
                                                     RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off,
-                                                    uint64_t tile0, uint64_t f2, Ctl* ctl) {
+                                                    uint64_t tile0, uint64_t f2, Ctl* ctl, uint64_t ntask) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // layout: [table (at offset 0: the lookup address is one IMAD)][stages: nwarps * S * 2 KiB][mbarriers]
   const uint32_t nwarps = blockDim.x / 32;
@@ -76,6 +93,7 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   uint8_t* table = smem_raw;
   uint8_t* stages = smem_raw + table_off;
   uint64_t* bars = reinterpret_cast<uint64_t*>(stages + (size_t)nwarps * S * kStageBytes);
+  uint32_t* prow = reinterpret_cast<uint32_t*>(bars + ((nwarps * S + 1) & ~1u)) + warp * 32;  // TASKS: producer group's chunks
   stage_table(img, table);  // load-time data: staged before the dependency wait
   pdl_wait();                // the previous kernel in the stream (e.g. the last run's verify) is done
   if (rp.ctl_init && blockIdx.x == 0) {
@@ -91,7 +109,7 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   using Sx = Step<MODE>;
 
   const uint32_t segs = rp.B / kRowBytes;
-  const uint64_t ntiles = (n_full + 31) / 32 - tile0;
+  const uint64_t ntiles = TASKS ? (ntask + 31) / 32 : (n_full + 31) / 32 - tile0;
   const uint64_t gw = (uint64_t)blockIdx.x * nwarps + warp, tw = (uint64_t)gridDim.x * nwarps;
   if (gw >= ntiles) return;
   struct StampEnd {  // timeline: the last warp to finish (profiling only)
@@ -110,16 +128,31 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   // producer cursor (lane 0): the item S ahead of the consumer, tracked without divisions
   uint64_t p_tile = 0;
   uint32_t p_sg = 0, p_s = 0;
-  auto issue_next = [&]() {
+  auto issue_next = [&]() {  // called by every lane of the warp (lane 0 issues)
     const uint64_t t = tile0 + gw + p_tile * tw;
-    mbar_expect_tx(wbar + p_s, kStageBytes);
-    tma_load_2d(wst + (size_t)p_s * kStageBytes, &tmap, wbar + p_s, (int32_t)(p_sg * kRowBytes), (int32_t)(t * 32),
-                pol);
+    if (TASKS && p_sg == 0) {  // new task group: its 32 chunks (the tail chunk / no task -> any full row)
+      const uint64_t idx = t * 32 + lane;
+      const uint32_t pc = idx < ntask ? __ldcg(rs.task_chunk + idx) : 0u;
+      __syncwarp();
+      prow[lane] = (uint32_t)min((uint64_t)pc, n_full - 1);
+      __syncwarp();
+    }
+    if (lane == 0) {
+      mbar_expect_tx(wbar + p_s, kStageBytes);
+      if (TASKS) {
+#pragma unroll
+        for (int g = 0; g < 8; g++)
+          tma_gather4(wst + (size_t)p_s * kStageBytes + g * 4 * kRowBytes, &tmap, wbar + p_s,
+                      (int32_t)(p_sg * kRowBytes), reinterpret_cast<const uint4*>(prow)[g], pol);
+      } else {
+        tma_load_2d(wst + (size_t)p_s * kStageBytes, &tmap, wbar + p_s, (int32_t)(p_sg * kRowBytes),
+                    (int32_t)(t * 32), pol);
+      }
+    }
     if (++p_sg == segs) { p_sg = 0; p_tile++; }
     if (++p_s == (uint32_t)S) p_s = 0;
   };
-  if (lane == 0)
-    for (uint64_t it = 0; it < items && it < (uint64_t)S; it++) issue_next();
+  for (uint64_t it = 0; it < items && it < (uint64_t)S; it++) issue_next();
 
   uint32_t st[KP], code[KP], acc[KP], kc = 1;
   uint64_t c = 0, tile_i = 0;
@@ -127,9 +160,11 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   for (uint64_t it = 0; it < items; it++) {
     if (sg == 0) {  // new tile: predict this lane's chunk start (lookback-2 pair table)
       c = (tile0 + gw + tile_i * tw) * 32 + lane;
-      if (TASKS) {
-        const uint32_t ts = (c < n_full && c >= f2) ? __ldcg(rs.tstart + c) : 0xFFFFFFFFu;
-        kc = ts != 0xFFFFFFFFu;  // 0: no task for this lane (walks the bytes, writes nothing)
+      if (TASKS) {  // c = this lane's task index until the chunk is known
+        const uint32_t tc = c < ntask ? __ldcg(rs.task_chunk + c) : 0xFFFFFFFFu;
+        const uint32_t ts = (tc < n_full && tc >= f2) ? __ldcg(rs.task_start + c) : 0xFFFFFFFFu;
+        c = tc;
+        kc = ts != 0xFFFFFFFFu;  // 0: no task for this lane (walks a row's bytes, writes nothing)
 #pragma unroll
         for (int p = 0; p < KP; p++) st[p] = kc ? ts : q0_of(rp);
       } else if (c == 0 || c >= n_full) {
@@ -168,7 +203,7 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
       }
     }
     __syncwarp();
-    if (lane == 0 && it + S < items) issue_next();  // refill this stage
+    if (it + S < items) issue_next();  // refill this stage
     if (TASKS && sg == segs - 1 && c < n_full && kc) {  // dense task done: append to VR^end
       const uint32_t e = Sx::tid(img, code[0]);
       const uint32_t ne = __ldcg(rs.n_end + c);
@@ -255,18 +290,20 @@ uint32_t pick_warps(uint64_t ntiles, int sms, uint32_t wmax) {
 
 template <int MODE, int KP, int S, bool TASKS>
 cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
-                         uint64_t n_full, int sms, cudaStream_t st, uint64_t tile0, uint64_t f2, Ctl* ctl) {
+                         uint64_t n_full, int sms, cudaStream_t st, uint64_t tile0, uint64_t f2, Ctl* ctl,
+                         uint64_t ntask) {
   auto kern = k_spec_tma<MODE, KP, S, TASKS>;
-  const uint64_t ntiles = (n_full + 31) / 32 - tile0;
+  const uint64_t ntiles = TASKS ? (ntask + 31) / 32 : (n_full + 31) / 32 - tile0;
+  if (ntiles == 0) return cudaSuccess;
   const uint32_t tbytes = smem_bytes_for(img);
-  const uint32_t per_warp = S * kStageBytes + S * 8;
+  const uint32_t per_warp = S * kStageBytes + S * 8 + 128;
   const uint32_t avail = 227 * 1024 - ((tbytes + 1023) & ~1023u) - 64;
   uint32_t wmax = std::min<uint32_t>(28, avail / per_warp);  // launch bounds 896 -> 72 regs
   if (wmax < 4) return cudaErrorInvalidConfiguration;
   uint32_t w = pick_warps(ntiles, sms, wmax);
   if (wmax < 8) w = wmax;
   const uint32_t table_off = (tbytes + 1023) & ~1023u;  // stages start 1 KiB-aligned (swizzle span)
-  const uint32_t smem = table_off + w * S * kStageBytes + w * S * 8;
+  const uint32_t smem = table_off + w * S * kStageBytes + ((w * S + 1) & ~1u) * 8 + w * 128;
   cudaError_t e = kernel_setup((const void*)kern, smem, (int)(w * 32), nullptr);
   if (e != cudaSuccess) return e;
   uint64_t grid = std::min<uint64_t>((uint64_t)sms, (ntiles + w - 1) / w);
@@ -281,16 +318,17 @@ cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunPa
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = pdl_enabled() ? 1 : 0;
-  return cudaLaunchKernelEx(&cfg, kern, tm, img, rp, rs, n_full, table_off, tile0, f2, ctl);
+  return cudaLaunchKernelEx(&cfg, kern, tm, img, rp, rs, n_full, table_off, tile0, f2, ctl, ntask);
 }
 
 template <int MODE, int KP, bool TASKS>
 cudaError_t launch_tma_s(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
-                         uint64_t n_full, int sms, cudaStream_t st, uint64_t tile0, uint64_t f2, Ctl* ctl) {
+                         uint64_t n_full, int sms, cudaStream_t st, uint64_t tile0, uint64_t f2, Ctl* ctl,
+                         uint64_t ntask = 0) {
   const uint32_t tbytes = smem_bytes_for(img);
-  if (tbytes + 24 * (3 * kStageBytes) + 2048 <= 227 * 1024)
-    return launch_tma_t<MODE, KP, 3, TASKS>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl);
-  return launch_tma_t<MODE, KP, 2, TASKS>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl);
+  if (tbytes + 24 * (3 * kStageBytes) + 2048 + 24 * 128 <= 227 * 1024)
+    return launch_tma_t<MODE, KP, 3, TASKS>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask);
+  return launch_tma_t<MODE, KP, 2, TASKS>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask);
 }
 
 template <int MODE>
@@ -302,12 +340,14 @@ cudaError_t launch_tma_m(const CUtensorMap& tm, const DevImage& img, const RunPa
   return launch_tma_s<MODE, 8, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
 }
 
-bool encode_map(const RunParams& rp, uint64_t n_full, CUtensorMap* tm) {
+// gather = false: box {64 B, 32 chunks} (tiles of consecutive chunks);
+// gather = true: box {64 B, 1 chunk} for tile::gather4 (4 arbitrary chunks per load)
+bool encode_map(const RunParams& rp, uint64_t n_full, CUtensorMap* tm, bool gather = false) {
   EncodeFn enc = get_encode();
   if (!enc) return false;
   cuuint64_t dims[2] = {rp.B, n_full};
   cuuint64_t strides[1] = {rp.B};
-  cuuint32_t box[2] = {kRowBytes, 32};
+  cuuint32_t box[2] = {kRowBytes, gather ? 1u : 32u};
   cuuint32_t es[2] = {1, 1};
   return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(rp.in), dims, strides, box, es,
              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -341,20 +381,22 @@ cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecS
   return e;
 }
 
+// Dense recovery round over the task list (ntask entries): chunks < n_full are walked
+// here; the tail chunk (if its task is listed) is left to the finish kernel.
 cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
-                            int sms, cudaStream_t st, uint64_t* n_done) {
+                            uint64_t ntask, int sms, cudaStream_t st, uint64_t* n_done) {
   *n_done = 0;
   const uint64_t n_full = rp.len / rp.B;
   CUtensorMap tm;
-  if (f2 >= n_full || !tma_applies(rp, n_full) || !encode_map(rp, n_full, &tm)) return cudaErrorNotSupported;
-  const uint64_t tile0 = f2 / 32;
+  if (f2 >= n_full || !tma_applies(rp, n_full) || !encode_map(rp, n_full, &tm, true)) return cudaErrorNotSupported;
+  const uint64_t tile0 = 0;
   cudaError_t e;
   switch (img.mode) {
-    case MODE_U8: e = launch_tma_s<MODE_U8, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
-    case MODE_U16: e = launch_tma_s<MODE_U16, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
-    case MODE_U16H: e = launch_tma_s<MODE_U16H, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
-    case MODE_U16D: e = launch_tma_s<MODE_U16D, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
-    default: e = launch_tma_s<MODE_U32, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl); break;
+    case MODE_U8: e = launch_tma_s<MODE_U8, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
+    case MODE_U16: e = launch_tma_s<MODE_U16, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
+    case MODE_U16H: e = launch_tma_s<MODE_U16H, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
+    case MODE_U16D: e = launch_tma_s<MODE_U16D, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
+    default: e = launch_tma_s<MODE_U32, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
   }
   if (e == cudaSuccess) *n_done = n_full;
   return e;

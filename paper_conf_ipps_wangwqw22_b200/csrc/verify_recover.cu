@@ -519,7 +519,10 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       // task kernel over chunk tiles (same tasks, same records) and relaunches us
       const uint64_t nt = ld_cg64(&ctl->it_ntask[slot]);
       if (nt >= 2048 && nt * 16 >= N - f2) {
-        if (b == 0 && threadIdx.x == 0) vctl->dense_pending = 1;
+        if (b == 0 && threadIdx.x == 0) {
+          vctl->ntask[0] = nt;  // the task list's length (this pass's slot) for the host launch
+          vctl->dense_pending = 1;
+        }
         return;
       }
     }
@@ -897,14 +900,14 @@ cudaError_t launch_dense_finish(const DevImage& img, const RunParams& rp, const 
 }  // namespace
 
 cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
-                            int sms, cudaStream_t st, uint64_t* n_done);
+                            uint64_t ntask, int sms, cudaStream_t st, uint64_t* n_done);
 
 cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp_in, const RecStore& rs, Ctl* ctl, uint64_t f2,
-                              int sms, cudaStream_t st) {
+                              uint64_t ntask, int sms, cudaStream_t st) {
   RunParams rp = rp_in;
   rp.ctl_init = nullptr;  // the control block is live: never re-initialise it mid-run
   uint64_t done = 0;
-  cudaError_t e = launch_task_tma(img, rp, rs, ctl, f2, sms, st, &done);
+  cudaError_t e = launch_task_tma(img, rp, rs, ctl, f2, ntask, sms, st, &done);
   if (e == cudaErrorNotSupported) {
     cudaGetLastError();
     done = 0;  // the finish kernel walks everything (slow, but exact)
