@@ -370,14 +370,17 @@ int run_core(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_sche
 // row compresses.  The poison row (all poison) is stored once as hot row H.
 // Output: the shared-memory image [hot rows 0..H-1][poison row][pad][delta rows].
 bool plan_delta_rows(fsm_t f, const std::vector<uint32_t>& ttc, uint32_t nt, uint32_t C,
-                     const std::vector<uint32_t>& tid2code, uint32_t budget_in, DevImage* img,
-                     std::vector<uint2>* out) {
+                     std::vector<uint32_t>& tid2code, std::vector<uint32_t>& code2tid, uint32_t budget_in,
+                     DevImage* img, std::vector<uint2>* out) {
   const uint32_t budget = budget_in ? budget_in : 128 * 1024;
   const uint64_t row_b = (uint64_t)C * 2;
   const uint32_t nr = nt - 1;  // real states (the poison tid nr is handled apart)
-  if (nr < 2 || row_b <= 8 || (uint64_t)nr * 8 + 2 * row_b + 32 > budget) return false;
-  uint64_t hmax = (budget - (uint64_t)nr * 8 - row_b - 32) / (row_b - 8);  // (H+1)*row + (nr-H)*8 <= budget
-  hmax = std::min<uint64_t>(hmax, std::min<uint64_t>(nr - 1, 0xFFFEu));  // base tids are 16-bit
+  if (nr < 2 || row_b <= 8 || 2 * C > 254 || (uint64_t)nr * 8 + 2 * row_b + 512 > budget) return false;
+  uint64_t hmax = (budget - (uint64_t)nr * 8 - row_b - 512) / (row_b - 8);  // (H+1)*row + (nr-H)*8 <= budget
+  hmax = std::min<uint64_t>(hmax, nr - 1);
+  // pre-multiplied codes: (H+1)*C + cold tids < 2^15, hot byte offsets + the smem base < 2^16
+  while (hmax >= 1 && ((hmax + 1) * C + (nr - hmax) > 0x7FFFu || 2 * (hmax + 1) * C + kDeltaBaseMax > 0xFFFFu))
+    hmax--;
   if (hmax < 1) return false;
   // first[t][d] = smallest j < min(t, hmax) whose row differs from row t in <= d columns
   const uint32_t kNo = 0xFFFFFFFFu;
@@ -406,39 +409,51 @@ bool plan_delta_rows(fsm_t f, const std::vector<uint32_t>& ttc, uint32_t nt, uin
     const uint64_t want = strtoull(e, nullptr, 10);
     if (want > H) H = std::min<uint64_t>(want, hmax);
   }
-  const uint64_t hot_b = (H + 1) * row_b;  // + the poison row as row H
-  const uint64_t delta_off = (hot_b + 15) & ~15ull;
-  const uint64_t bytes = (delta_off + (uint64_t)(nt - H) * 8 + 15) & ~15ull;
+  // codes: hot t -> t*C, poison -> H*C (stored as hot row H), cold t -> HC1 + (t - H)
+  const uint64_t HC1 = (H + 1) * C;
+  std::vector<uint32_t> code(nt);
+  for (uint32_t t = 0; t < nt; t++) {
+    const uint32_t a = tid2code[t] >> 15;  // accept flag of the plain u16 code
+    const uint64_t c = t < H ? (uint64_t)t * C : t == nr ? H * C : HC1 + (t - H);
+    code[t] = (uint32_t)c | (a << 15);
+  }
+  const uint64_t hot_b = HC1 * 2;
+  const uint64_t cls_off = (hot_b + 255) & ~255ull;
+  const uint64_t delta_off = cls_off + 256;
+  const uint64_t bytes = (delta_off + (uint64_t)(nr - H) * 8 + 15) & ~15ull;
+  if (bytes > budget) return false;
   std::vector<uint16_t> im(bytes / 2, 0);
   for (uint64_t t = 0; t < H; t++)
-    for (uint32_t c = 0; c < C; c++) im[t * C + c] = (uint16_t)tid2code[ttc[t * C + c]];
-  for (uint32_t c = 0; c < C; c++) im[H * C + c] = (uint16_t)tid2code[nr];
-  uint2* dl = reinterpret_cast<uint2*>(im.data() + delta_off / 2);
-  for (uint32_t t = (uint32_t)H; t < nt; t++) {
-    if (t == nr) {  // poison: base = the poison row, no exceptions
-      dl[t - H] = make_uint2((uint32_t)H | 0xFFFF0000u, 0);
-      continue;
-    }
+    for (uint32_t c = 0; c < C; c++) im[t * C + c] = (uint16_t)code[ttc[t * C + c]];
+  for (uint32_t c = 0; c < C; c++) im[H * C + c] = (uint16_t)code[nr];
+  uint8_t* cm = reinterpret_cast<uint8_t*>(im.data()) + cls_off;
+  for (uint32_t b = 0; b < 256; b++) cm[b] = (uint8_t)(2 * f->cls[b]);
+  uint2* dl = reinterpret_cast<uint2*>(reinterpret_cast<uint8_t*>(im.data()) + delta_off);
+  for (uint32_t t = (uint32_t)H; t < nr; t++) {
     const uint32_t* ft = &first[(uint64_t)t * (kDeltaExc + 1)];
     uint32_t j = kNo;
     for (uint32_t e = 0; e <= kDeltaExc && j == kNo; e++)
       if (ft[e] < H) j = ft[e];
     if (j == kNo) return false;  // unreachable (checked above)
-    uint32_t cls[kDeltaExc] = {0xFF, 0xFF}, code[kDeltaExc] = {0, 0}, k = 0;
+    uint32_t ex[kDeltaExc] = {0xFF, 0xFF}, ec[kDeltaExc] = {0, 0}, k = 0;
     for (uint32_t c = 0; c < C; c++)
       if (ttc[(uint64_t)t * C + c] != ttc[(uint64_t)j * C + c]) {
-        cls[k] = c;
-        code[k] = tid2code[ttc[(uint64_t)t * C + c]];
+        ex[k] = 2 * c;
+        ec[k] = code[ttc[(uint64_t)t * C + c]];
         k++;
       }
-    dl[t - H] = make_uint2(j | (cls[0] << 16) | (cls[1] << 24), (code[0] & 0xFFFFu) | (code[1] << 16));
+    dl[t - H] = make_uint2((uint32_t)(2 * C * j) << 16 | ex[1] << 8 | ex[0], (ec[0] & 0xFFFFu) | (ec[1] << 16));
   }
   out->assign(reinterpret_cast<const uint2*>(im.data()), reinterpret_cast<const uint2*>(im.data()) + bytes / 8);
+  tid2code = code;
+  code2tid.assign(0x8000, nr);
+  for (uint32_t t = 0; t < nt; t++) code2tid[code[t] & 0x7FFFu] = t;
   img->H = (uint32_t)H;
-  img->D = nt - (uint32_t)H;
+  img->D = nr - (uint32_t)H;
+  img->HC1 = (uint32_t)HC1;
+  img->cls_off = (uint32_t)cls_off;
   img->delta_off = (uint32_t)delta_off;
   img->smem_table_bytes = (uint32_t)bytes;
-  (void)f;
   return true;
 }
 
@@ -628,8 +643,8 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
     img.smem_table_bytes = (uint32_t)(((H * C * esz) + 15) & ~15ull);
     if (mode == MODE_U16 && H == nt) img.mode = MODE_U16H;  // every row hot: no hot test
     std::vector<uint2> delta;
-    if (mode == MODE_U16 && H < nt && want_delta && C < 256 &&
-        plan_delta_rows(f, ttc, nt, C, tid2code, opts ? opts->smem_budget_bytes : 0, &img, &delta)) {
+    if (mode == MODE_U16 && H < nt && want_delta && C < 128 &&
+        plan_delta_rows(f, ttc, nt, C, tid2code, code2tid, opts ? opts->smem_budget_bytes : 0, &img, &delta)) {
       img.mode = MODE_U16D;
       if ((rc = upload(f, &img.Dl, delta))) return bail(rc);
     }

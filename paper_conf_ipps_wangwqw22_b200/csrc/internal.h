@@ -25,6 +25,7 @@ enum Mode : uint32_t {
 };
 
 constexpr uint32_t kDeltaExc = 2;        // exceptions per delta row
+constexpr uint32_t kDeltaBaseMax = 8192;  // MODE_U16D: max shared-window offset of the staged table
 
 constexpr uint32_t kQsMax = 16;     // QS cap ("top 16 states")
 constexpr uint32_t kVrMax = 16;     // VR^end / VR^others slots
@@ -51,12 +52,17 @@ struct DevImage {
   const uint32_t* code2tid;   // MODE_U8: [256]
   const uint32_t* inv;        // [nt] tid -> original id (poison -> n)
   const uint8_t* acc;         // [nt] accept by tid
-  // MODE_U16D: the whole shared-memory table image [hot rows 0..H-1][poison row (= row H)]
-  // [pad][delta rows of tids H..nt-1]; delta row: x = base tid | cls0 << 16 | cls1 << 24,
-  // y = code0 | code1 << 16 (unused exception: class 0xFF)
+  // MODE_U16D: the whole shared-memory table image
+  //   [hot rows 0..H-1][poison row (= row H)][pad to 256][class map: 2*class, 256 B][delta rows]
+  // Codes are pre-multiplied: hot tid t -> t*C, poison -> H*C, cold tid t -> HC1 + (t - H),
+  // accept flag in bit 15.  Delta row of a cold tid: x = (2*C*base tid) << 16 | e1 << 8 | e0
+  // (e = 2*exception class, 0xFF = none; the row offset is made absolute at staging),
+  // y = code0 | code1 << 16.
   const uint2* Dl;
-  uint32_t delta_off;         // byte offset of the delta rows behind the hot rows (16-aligned)
-  uint32_t D;                 // delta rows (= nt - H)
+  uint32_t delta_off;         // byte offset of the delta rows (16-aligned)
+  uint32_t D;                 // delta rows (cold real tids)
+  uint32_t cls_off;           // byte offset of the doubled class map (256-aligned)
+  uint32_t HC1;               // (H + 1) * C: the first cold code
 };
 
 // Global record store (hierarchical store, level 3).

@@ -851,16 +851,23 @@ cudaError_t launch_m(const DevImage& img, const RunParams& rp, const RecStore& r
 }
 
 // After the TMA task kernel: the partial tail chunk's task (if any), then commit
-// the round (Alg. 3 L14: the frontier advances to f2).
+// the round (Alg. 3 L14: the frontier advances to f2).  The table is staged only
+// when a chunk is left to walk (a stream whose length is a multiple of B has none).
 template <int MODE>
-__global__ void __launch_bounds__(32) k_dense_finish(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
-                                                     uint64_t c_first_generic) {
+__global__ void __launch_bounds__(256) k_dense_finish(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
+                                                      uint64_t c_first_generic) {
   extern __shared__ __align__(1024) uint8_t smem[];
-  stage_table(img, smem);
-  __syncwarp();
-  if (threadIdx.x != 0) return;
+  __shared__ uint32_t any;
   const uint64_t f2 = ctl->fmin;
-  for (uint64_t c = max(c_first_generic, f2); c < rp.N; c++) {
+  if (threadIdx.x == 0) {
+    any = 0;
+    for (uint64_t c = max(c_first_generic, f2); c < rp.N && !any; c++) any = __ldcg(rs.tstart + c) != 0xFFFFFFFFu;
+  }
+  __syncthreads();
+  if (any) stage_table(img, smem);
+  __syncthreads();
+  if (threadIdx.x != 0) return;
+  for (uint64_t c = max(c_first_generic, f2); any && c < rp.N; c++) {
     const uint32_t st = __ldcg(rs.tstart + c);
     if (st == 0xFFFFFFFFu) continue;
     uint32_t e, cnt;
@@ -891,9 +898,9 @@ cudaError_t launch_dense_finish(const DevImage& img, const RunParams& rp, const 
                                 uint64_t c_first_generic, cudaStream_t st) {
   auto kern = k_dense_finish<MODE>;
   const uint32_t smem = smem_bytes_for(img);
-  cudaError_t e = kernel_setup((const void*)kern, smem, 32, nullptr);
+  cudaError_t e = kernel_setup((const void*)kern, smem, 256, nullptr);
   if (e != cudaSuccess) return e;
-  kern<<<1, 32, smem, st>>>(img, rp, rs, ctl, c_first_generic);
+  kern<<<1, 256, smem, st>>>(img, rp, rs, ctl, c_first_generic);
   return cudaGetLastError();
 }
 

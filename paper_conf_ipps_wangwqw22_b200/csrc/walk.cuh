@@ -13,14 +13,29 @@ namespace gspec {
 // Layout: u8 mode: [table]; classed modes: [cls: 256 B][table: smem_table_bytes]
 // (the class map first keeps it 256-aligned: its address is one PRMT away).
 __device__ __forceinline__ void stage_table(const DevImage& img, uint8_t* smem) {
+  if (img.mode == MODE_U16D) {  // one image [hot rows][class map][delta rows]; delta offsets made absolute
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
+    if (base + 2 * img.HC1 > 0xFFFFu) __trap();  // fsm_load bounds the hot bytes by 64 KiB - kDeltaBaseMax
+    const uint4* from = reinterpret_cast<const uint4*>(img.Dl);
+    uint4* dst = reinterpret_cast<uint4*>(smem);
+    const uint32_t nv = img.smem_table_bytes / 16, d0 = img.delta_off / 16;
+    for (uint32_t i = threadIdx.x; i < nv; i += blockDim.x) {
+      uint4 v = __ldg(from + i);
+      if (i >= d0) {
+        v.x += base << 16;
+        v.z += base << 16;
+      }
+      dst[i] = v;
+    }
+    return;
+  }
   const uint4* src = (img.mode == MODE_U8)                                 ? reinterpret_cast<const uint4*>(img.T8)
-                     : (img.mode == MODE_U16 || img.mode == MODE_U16H || img.mode == MODE_U16D) ? reinterpret_cast<const uint4*>(img.T16)
+                     : (img.mode == MODE_U16 || img.mode == MODE_U16H) ? reinterpret_cast<const uint4*>(img.T16)
                                                                          : reinterpret_cast<const uint4*>(img.T32);
   const uint32_t off = img.mode == MODE_U8 ? 0u : 256u;
   uint4* dst = reinterpret_cast<uint4*>(smem + off);
-  const uint4* from = img.mode == MODE_U16D ? reinterpret_cast<const uint4*>(img.Dl) : src;  // u16d: its own image
   const uint32_t nv = img.smem_table_bytes / 16;
-  for (uint32_t i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(from + i);
+  for (uint32_t i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(src + i);
   if (img.mode != MODE_U8) {
     const uint4* cs = reinterpret_cast<const uint4*>(img.cls);
     uint4* cd = reinterpret_cast<uint4*>(smem);
@@ -29,7 +44,7 @@ __device__ __forceinline__ void stage_table(const DevImage& img, uint8_t* smem) 
 }
 
 __host__ __device__ inline uint32_t smem_bytes_for(const DevImage& img) {
-  return img.smem_table_bytes + (img.mode == MODE_U8 ? 0u : 256u);
+  return img.smem_table_bytes + (img.mode == MODE_U8 || img.mode == MODE_U16D ? 0u : 256u);
 }
 
 template <int MODE>
@@ -118,42 +133,46 @@ __device__ __forceinline__ uint2 lds_u64(uint32_t saddr) {
   return v;
 }
 
-// MODE_U16D: a cold tid (>= H) reads its 8-byte delta row {hot base tid, 2 exception
-// classes, 2 exception codes}; a hot tid acts as its own base with no exceptions.
-// Branch-free: the delta-row load is predicated on the cold lanes only (hot lanes
-// generate no shared-memory traffic for it), then every lane reads one row entry
-// (its own row or its base row) and the exceptions override by select — two
-// dependent shared-memory loads, no L2 trip, no divergence.  fsm_load picks this
-// mode only when every cold row compresses.  (Measured on C4: a hot/cold branch
-// cost 28 instructions per warp-step with 90% of warp-steps divergent; loading a
-// descriptor for every lane cost 4.7 wavefronts per LDS.64.)
+// MODE_U16D: pre-multiplied codes.  c = code & 0x7FFF; a hot code is
+// its row's entry index (t*C), a cold code c >= HC1 owns the 8-byte delta row
+// {x = absolute row byte offset << 16 | e1 << 8 | e0, y = code0 | code1 << 16}.  Every
+// lane starts from the hot default x = (base + 2c) << 16 | 0xFFFF (no exceptions); the
+// delta-row load is predicated on the cold lanes only (hot lanes generate no
+// shared-memory traffic for it), then one row entry is read at (x >> 16) + 2*class
+// and the exceptions override by select — two dependent shared-memory loads, no L2
+// trip, no divergence, and no multiply by C on the path (the class map holds 2*class).
+// The step is ALU-pipe-bound on C4 (math_pipe_throttle): this form needs ~10 ALU-pipe
+// and ~3 FMA-pipe instructions per symbol.
 struct StepDelta {
   static constexpr uint32_t kShift = 15;
-  static constexpr uint32_t kMask = 0x7FFFu;
-  static __device__ __forceinline__ uint32_t row(const DevImage& img, uint32_t base, uint32_t code, uint32_t cl) {
-    const uint32_t t = code & kMask;
-    uint32_t dx = t | 0xFFFF0000u, dy = 0;  // hot: base = t, exception classes 0xFF (none)
-    const uint32_t da = base + 256 + img.delta_off + (t - img.H) * 8;
+  static __device__ __forceinline__ uint32_t row(const DevImage& img, uint32_t base, uint32_t code, uint32_t cl2) {
+    const uint32_t c = code & 0x7FFFu;
+    uint32_t dx = c * 0x20000u + ((base << 16) | 0xFFFFu), dy = 0;
+    uint32_t da;  // c*8 + const on the FMA pipe (the ALU pipe is the bound)
+    asm("mad.lo.u32 %0, %1, 8, %2;" : "=r"(da) : "r"(c), "r"(base + img.delta_off - img.HC1 * 8u));
     asm volatile(
         "{\n .reg .pred p;\n setp.ge.u32 p, %2, %3;\n @p ld.shared.v2.u32 {%0, %1}, [%4];\n}\n"
         : "+r"(dx), "+r"(dy)
-        : "r"(t), "r"(img.H), "r"(da));
-    uint32_t v = lds_u16(base + 256 + ((dx & 0xFFFFu) * img.C + cl) * 2);
-    v = (cl == (dx >> 24)) ? (dy >> 16) : v;
-    v = (cl == ((dx >> 16) & 0xFFu)) ? (dy & 0xFFFFu) : v;
+        : "r"(c), "r"(img.HC1), "r"(da));
+    uint32_t v = lds_u16((dx >> 16) + cl2);
+    const uint32_t x = dx ^ (cl2 * 0x101u);
+    v = (x & 0xFFu) == 0 ? (dy & 0xFFFFu) : v;
+    v = (x & 0xFF00u) == 0 ? (dy >> 16) : v;
     return v;
   }
   static __device__ __forceinline__ uint32_t byte(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t b) {
     const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
-    return row(img, base, code, lds_u8(base + b));
+    return row(img, base, code, lds_u8(base + img.cls_off + b));
   }
   template <int K>
   static __device__ __forceinline__ uint32_t word(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t w) {
     const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
-    return row(img, base, code, lds_u8(byte_plus<K>(w, base)));
+    return row(img, base, code, lds_u8(byte_plus<K>(w, base + img.cls_off)));  // class map 256-aligned
   }
   static __device__ __forceinline__ uint32_t acc(uint32_t code) { return code >> 15; }
-  static __device__ __forceinline__ uint32_t tid(const DevImage&, uint32_t code) { return code & kMask; }
+  static __device__ __forceinline__ uint32_t tid(const DevImage& img, uint32_t code) {
+    return __ldg(img.code2tid + (code & 0x7FFFu));
+  }
 };
 
 template <>
