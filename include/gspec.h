@@ -49,7 +49,13 @@ typedef enum {
   FSM_SCHEME_SRE = 3,  /* Alg. 3: recovery activated by the predecessor's end    */
   FSM_SCHEME_RR = 4,   /* Alg. 4: SRE + round-robin helpers over QS              */
   FSM_SCHEME_NF = 5,   /* Alg. 5: SRE + nearest-first helpers over QS            */
-  FSM_SCHEME_ENUM = 6  /* enumerative: all-state chunk maps + composition scan  */
+  FSM_SCHEME_ENUM = 6, /* enumerative: all-state chunk maps + composition scan  */
+  FSM_SCHEME_CSE = 7   /* convergence-set enumeration (P:300, P:427 [21][24]):
+                          round 0 walks every lookback-2 candidate of each chunk up to
+                          spec_k (default 8) — the whole image, which contains the true
+                          start, whenever it has <= spec_k states — with path fusion
+                          (paths that meet are walked once); SRE rounds recover what a
+                          capped image missed.  Not chosen by FSM_SCHEME_AUTO. */
 } fsm_scheme;
 
 typedef struct fsm_s* fsm_t;
@@ -72,7 +78,7 @@ typedef struct {
 typedef struct {
   fsm_scheme scheme;    /* FSM_SCHEME_*                                                  */
   uint32_t chunk_bytes; /* B: chunk c = [cB, min(len,(c+1)B)); multiple of 16; 0 = 4096   */
-  uint32_t spec_k;      /* paths per chunk for PM (4); 1..8; 0 = 4                 */
+  uint32_t spec_k;      /* paths per chunk: PM (4) / CSE (8); 1..8; 0 = default    */
   uint32_t lookback;    /* lookback symbols (2); only 2 is supported; 0 = 2        */
   uint32_t qs_cap;      /* K: ranked candidates kept per chunk (16); 1..16; 0 = 16 */
   uint32_t vr_end;      /* VR^end slots per chunk (16); 1..16; 0 = 16              */

@@ -15,8 +15,8 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB = None
 
 OR_OK, OR_EINVAL, OR_ESYMBOL, OR_EUNSUPPORTED = 0, -1, -4, -6
-SEQ, PM, SRE, RR, NF, ENUM = 1, 2, 3, 4, 5, 6
-SCHEME_IDS = {"seq": SEQ, "pm": PM, "sre": SRE, "rr": RR, "nf": NF, "enum": ENUM}
+SEQ, PM, SRE, RR, NF, ENUM, CSE = 1, 2, 3, 4, 5, 6, 7
+SCHEME_IDS = {"seq": SEQ, "pm": PM, "sre": SRE, "rr": RR, "nf": NF, "enum": ENUM, "cse": CSE}
 
 P = ctypes.c_void_p
 U32, U64 = ctypes.c_uint32, ctypes.c_uint64
@@ -138,9 +138,12 @@ def compose(M1, C1, M2, C2):
     return M, C
 
 
-def simulate(table, start, accept, data, B=4096, scheme="sre", spec_k=4, qs_cap=16, vr_end=16, vr_oth=16,
+def simulate(table, start, accept, data, B=4096, scheme="sre", spec_k=None, qs_cap=16, vr_end=16, vr_oth=16,
              policy=0, max_tasks=0):
-    """Round semantics of Alg. 2-5. Works on the transformed DFA."""
+    """Round semantics of Alg. 2-5. Works on the transformed DFA.
+    spec_k: round-0 paths per chunk for PM (default 4) and CSE (default 8)."""
+    if spec_k is None:
+        spec_k = 8 if scheme == "cse" else 4
     perm, inv, _, tt, acc = transform(table, accept, policy, data if policy == 1 else None, start)
     t = _c(table, np.uint32)
     n, ns = t.shape

@@ -65,6 +65,12 @@ void or_compose(uint32_t n, const uint32_t* M1, const uint64_t* C1, const uint32
 #define OR_RR 4
 #define OR_NF 5
 #define OR_ENUM 6
+/* Convergence-set enumeration (the exact-coverage methods the
+ * paper cites beside SRE, P:427 [21][24]): round 0 runs EVERY lookback candidate
+ * of QS_c up to spec_k (the whole lookback image when it has <= spec_k states,
+ * which contains the true start), then SRE rounds for whatever a capped
+ * image missed. */
+#define OR_CSE 7
 
 typedef struct {
   uint32_t final_state; /* original id */

@@ -24,7 +24,7 @@ if not os.path.exists(_LIB_PATH):
 _lib = ctypes.CDLL(_LIB_PATH)
 
 FSM_OK, FSM_EINVAL, FSM_ENOMEM, FSM_ECUDA, FSM_ESYMBOL, FSM_ENCCL, FSM_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
-SCHEMES = {"auto": 0, "seq": 1, "pm": 2, "sre": 3, "rr": 4, "nf": 5, "enum": 6}
+SCHEMES = {"auto": 0, "seq": 1, "pm": 2, "sre": 3, "rr": 4, "nf": 5, "enum": 6, "cse": 7}
 SCHEME_NAMES = {v: k for k, v in SCHEMES.items()}
 MODES = {1: "u8", 2: "u16", 3: "u32", 4: "u16d"}
 
@@ -112,7 +112,7 @@ def fsm_num_chunks(length: int, chunk_bytes: int = 4096) -> int:
     return int(_lib.fsm_num_chunks(length, chunk_bytes))
 
 
-def _run_opts(scheme="auto", chunk_bytes=4096, spec_k=4, qs_cap=16, vr_end=16, vr_others=16, stream=None):
+def _run_opts(scheme="auto", chunk_bytes=4096, spec_k=0, qs_cap=16, vr_end=16, vr_others=16, stream=None):
     if isinstance(scheme, str):
         scheme = SCHEMES[scheme]
     if stream is None:
@@ -176,7 +176,7 @@ class FSM:
             pass
 
     # ---- runs -----------------------------------------------------------------
-    def run(self, x, scheme="auto", chunk_bytes=4096, spec_k=4, qs_cap=16, vr_end=16, vr_others=16,
+    def run(self, x, scheme="auto", chunk_bytes=4096, spec_k=0, qs_cap=16, vr_end=16, vr_others=16,
             chunk_ends=True, stream=None) -> Result:
         """fsm_run over a uint8 CUDA tensor; chunk_ends -> int64-free uint32 CUDA tensor (as torch.int32 view)."""
         import torch
@@ -190,7 +190,7 @@ class FSM:
                             ce.data_ptr() if ce is not None else None, ctypes.byref(r)), "fsm_run")
         return Result.from_c(r, ce[:n] if ce is not None else None)
 
-    def run_async(self, x, scheme="auto", chunk_bytes=4096, chunk_ends=None, spec_k=4, stream=None) -> int:
+    def run_async(self, x, scheme="auto", chunk_bytes=4096, chunk_ends=None, spec_k=0, stream=None) -> int:
         """fsm_run_async: enqueue a run (stream-ordered) and return a ticket for wait()."""
         o = _run_opts(scheme, chunk_bytes, spec_k, stream=stream)
         t = U64(0)
@@ -318,7 +318,7 @@ class Comm:
         _check(_lib.fsm_comm_unique_id(buf), "fsm_comm_unique_id")
         return buf.raw
 
-    def run_sharded(self, fsm: "FSM", shard, lookback=None, scheme="auto", chunk_bytes=4096, spec_k=4,
+    def run_sharded(self, fsm: "FSM", shard, lookback=None, scheme="auto", chunk_bytes=4096, spec_k=0,
                     chunk_ends=True, stream=None) -> Result:
         """fsm_run_sharded: shard map + one ncclAllGather + finish, all inside the library."""
         import torch

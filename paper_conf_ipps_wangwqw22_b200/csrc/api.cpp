@@ -113,7 +113,7 @@ void place_rows_bank_aware(fsm_t f, const std::vector<uint32_t>& ttc, uint32_t C
 
 struct Opts {
   fsm_scheme scheme;
-  uint32_t B, k, L, qs_cap, vr_end, vr_oth;
+  uint32_t B, k, k_cse, L, qs_cap, vr_end, vr_oth;
   cudaStream_t st;
 };
 
@@ -121,6 +121,7 @@ int resolve_opts(const fsm_run_opts* o, Opts* r) {
   r->scheme = o ? o->scheme : FSM_SCHEME_AUTO;
   r->B = (o && o->chunk_bytes) ? o->chunk_bytes : 4096;
   r->k = (o && o->spec_k) ? o->spec_k : 4;
+  r->k_cse = (o && o->spec_k) ? o->spec_k : 8;  // CSE: up to 8 lookback candidates per chunk
   r->L = (o && o->lookback) ? o->lookback : 2;
   r->qs_cap = (o && o->qs_cap) ? o->qs_cap : 16;
   r->vr_end = (o && o->vr_end) ? o->vr_end : 16;
@@ -132,7 +133,7 @@ int resolve_opts(const fsm_run_opts* o, Opts* r) {
   if (r->qs_cap < 1 || r->qs_cap > kQsMax) return fail(FSM_EINVAL, "qs_cap must be in [1,16]");
   if (r->vr_end < 1 || r->vr_end > kVrMax || r->vr_oth < 1 || r->vr_oth > kVrMax)
     return fail(FSM_EINVAL, "vr_end / vr_others must be in [1,16]");
-  if ((int)r->scheme < 0 || (int)r->scheme > FSM_SCHEME_ENUM) return fail(FSM_EINVAL, "unknown scheme");
+  if ((int)r->scheme < 0 || (int)r->scheme > FSM_SCHEME_CSE) return fail(FSM_EINVAL, "unknown scheme");
   return FSM_OK;
 }
 
@@ -238,7 +239,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   rp.B = o.B;
   rp.N = N;
   rp.scheme = scheme;
-  rp.k = scheme == FSM_SCHEME_PM ? o.k : 1;
+  rp.k = scheme == FSM_SCHEME_PM ? o.k : scheme == FSM_SCHEME_CSE ? o.k_cse : 1;
   rp.qs_cap = o.qs_cap;
   rp.vr_end = o.vr_end;
   rp.vr_oth = o.vr_oth;
@@ -288,7 +289,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     // dense recovery rounds go to the TMA task kernel (SRE on low-accuracy DFAs); this
     // needs a host check per verify launch, so it is off when the profile says the
     // speculation is accurate (no dense rounds expected)
-    rp.dense = (scheme == FSM_SCHEME_SRE && len / o.B > 0 && o.B % 64 == 0 &&
+    rp.dense = ((scheme == FSM_SCHEME_SRE || scheme == FSM_SCHEME_CSE) && len / o.B > 0 && o.B % 64 == 0 &&
                 (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0 && f->acc1_hint < 0.5) ? 1u : 0u;
     CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
     {  // TMA kernel over the full chunks + the generic kernel for a tail chunk (or everything)

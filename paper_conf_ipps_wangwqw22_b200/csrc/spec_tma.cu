@@ -154,7 +154,8 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   };
   for (uint64_t it = 0; it < items && it < (uint64_t)S; it++) issue_next();
 
-  uint32_t st[KP], code[KP], acc[KP], kc = 1;
+  uint32_t st[KP], code[KP], acc[KP], dacc[KP], kc = 1;
+  bool single = false;  // spec-k: all paths of the warp's lanes merged (path fusion, P:427 [21])
   uint64_t c = 0, tile_i = 0;
   uint32_t sg = 0, s = 0, phase = 0;
   for (uint64_t it = 0; it < items; it++) {
@@ -182,24 +183,51 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
       for (int p = 0; p < KP; p++) {
         code[p] = __ldg(img.tid2code + st[p]);
         acc[p] = 0;
+        dacc[p] = 0;
       }
+      single = false;
     }
     mbar_wait(wbar + s, phase);
     const uint8_t* row = wst + (size_t)s * kStageBytes + lane * kRowBytes;
+    if (KP > 1 && single) {  // path fusion: every path of every lane has merged into path 0
 #pragma unroll
-    for (int u = 0; u < (int)(kRowBytes / 16); u++) {
-      const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ ((lane >> 1) & 3)) << 4));  // SWIZZLE_64B
-      const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+      for (int u = 0; u < (int)(kRowBytes / 16); u++) {
+        const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ ((lane >> 1) & 3)) << 4));  // SWIZZLE_64B
+        const uint32_t w[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
-      for (int t = 0; t < 4; t++) {
+        for (int t = 0; t < 4; t++) {
+          code[0] = Sx::template word<0>(img, table, code[0], w[t]); acc[0] += Sx::acc(code[0]);
+          code[0] = Sx::template word<1>(img, table, code[0], w[t]); acc[0] += Sx::acc(code[0]);
+          code[0] = Sx::template word<2>(img, table, code[0], w[t]); acc[0] += Sx::acc(code[0]);
+          code[0] = Sx::template word<3>(img, table, code[0], w[t]); acc[0] += Sx::acc(code[0]);
+        }
+      }
+    } else {
 #pragma unroll
-        for (int p = 0; p < KP; p++) { code[p] = Sx::template word<0>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+      for (int u = 0; u < (int)(kRowBytes / 16); u++) {
+        const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ ((lane >> 1) & 3)) << 4));  // SWIZZLE_64B
+        const uint32_t w[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
-        for (int p = 0; p < KP; p++) { code[p] = Sx::template word<1>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+        for (int t = 0; t < 4; t++) {
 #pragma unroll
-        for (int p = 0; p < KP; p++) { code[p] = Sx::template word<2>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+          for (int p = 0; p < KP; p++) { code[p] = Sx::template word<0>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
 #pragma unroll
-        for (int p = 0; p < KP; p++) { code[p] = Sx::template word<3>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+          for (int p = 0; p < KP; p++) { code[p] = Sx::template word<1>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+#pragma unroll
+          for (int p = 0; p < KP; p++) { code[p] = Sx::template word<2>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+#pragma unroll
+          for (int p = 0; p < KP; p++) { code[p] = Sx::template word<3>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+        }
+      }
+      if (KP > 1) {  // DFA determinism: paths that meet stay together; once all have met, walk one
+        bool merged = true;
+#pragma unroll
+        for (int p = 1; p < KP; p++) merged = merged && code[p] == code[0];
+        if (__all_sync(0xffffffffu, merged)) {
+          single = true;
+#pragma unroll
+          for (int p = 0; p < KP; p++) dacc[p] = acc[p] - acc[0];
+        }
       }
     }
     __syncwarp();
@@ -220,12 +248,12 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
       uint32_t e0 = 0;
 #pragma unroll
       for (int p = 0; p < KP; p++) {
-        const uint32_t e = Sx::tid(img, code[p]);
+        const uint32_t e = Sx::tid(img, code[(KP > 1 && single) ? 0 : p]);
         if (p == 0) e0 = e;
         if ((uint32_t)p < kc) {
           rs.start[p * rs.cap + c] = st[p];
           rs.end[p * rs.cap + c] = e;
-          rs.cnt[p * rs.cap + c] = acc[p];
+          rs.cnt[p * rs.cap + c] = (KP > 1 && single) ? acc[0] + dacc[p] : acc[p];
         }
       }
       rs.n_end[c] = kc;

@@ -274,7 +274,8 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   const uint64_t N = rp.N;
   const uint32_t G = gridDim.x, b = blockIdx.x;
   const uint64_t lo = N * b / G, hi = N * (b + 1) / G;
-  const bool sre_like = rp.scheme == FSM_SCHEME_SRE || rp.scheme == FSM_SCHEME_RR || rp.scheme == FSM_SCHEME_NF;
+  const bool sre_like = rp.scheme == FSM_SCHEME_SRE || rp.scheme == FSM_SCHEME_RR || rp.scheme == FSM_SCHEME_NF ||
+                        rp.scheme == FSM_SCHEME_CSE;
   const bool helpers = rp.scheme == FSM_SCHEME_RR || rp.scheme == FSM_SCHEME_NF;
   volatile Ctl* vctl = ctl;
 

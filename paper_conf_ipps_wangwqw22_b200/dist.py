@@ -70,7 +70,7 @@ def exchange_lookback(shard, group=None, L: int = 2):
     return tails[rank - 1, 16 - m:16].contiguous()
 
 
-def run_sharded(fsm: FSM, shard, lookback, group=None, scheme="auto", chunk_bytes=4096, spec_k=4,
+def run_sharded(fsm: FSM, shard, lookback, group=None, scheme="auto", chunk_bytes=4096, spec_k=0,
                 chunk_ends=True, stream=None) -> Result:
     """fsm_shard_map -> all_gather_into_tensor(maps) -> fsm_shard_finish."""
     import torch

@@ -51,7 +51,7 @@ def check_equal(res, ref, B, n):
     assert bad.size == 0, f"first mismatching chunk {bad[:5]} of {len(ce)}"
 
 
-SCHEMES = ["seq", "pm", "sre", "rr", "nf"]
+SCHEMES = ["seq", "pm", "sre", "rr", "nf", "cse"]
 
 
 @pytest.mark.parametrize("scheme", SCHEMES + ["enum", "auto"])
@@ -62,6 +62,8 @@ def test_div7_c1(gs, scheme):
     x = torch.from_numpy(data).cuda()
     res = fsm.run(x, scheme=scheme)
     check_equal(res, ref, 4096, w.nstates)
+    if scheme == "cse":  # every lookback image is all 7 states (<= 8): exact coverage, no recovery
+        assert res.stats["rounds"] == 0 and res.stats["verify_matches"] == res.stats["verify_checks"] == 256
     big_mod = ref["final"]  # pinned separately against int(bits,2) % 7 in the oracle tests
     assert res.accept == (big_mod == 0)
 
@@ -270,17 +272,18 @@ def test_async_queue(gs):
         fsm.wait(runs[0][0])  # already collected
 
 
-@pytest.mark.parametrize("name,length,B", [("c3", 32 << 20, 4096), ("c3", (24 << 20) + 1000, 4096),
-                                           ("c3s", 160 << 20, 8192)])
-def test_dense_recovery_rounds(gs, name, length, B):
-    """SRE on a low-accuracy DFA: rounds where most chunks re-execute go to the
-    TMA-staged task kernel; results and round diagnostics stay identical."""
+@pytest.mark.parametrize("name,length,B,scheme", [("c3", 32 << 20, 4096, "sre"), ("c3", (24 << 20) + 1000, 4096, "sre"),
+                                                  ("c3s", 160 << 20, 8192, "sre"), ("c3", 32 << 20, 4096, "cse")])
+def test_dense_recovery_rounds(gs, name, length, B, scheme):
+    """SRE (and CSE's SRE rounds) on a low-accuracy DFA: rounds where many chunks
+    re-execute go to the TMA-gather task kernel over the round's task list; results
+    and round diagnostics stay identical."""
     w, data = _wl(name, length)
     ref = oracle.run(w.table, w.start, w.accept, data, B)
     fsm = gs.FSM.load(w.table, w.start, w.accept)
-    res = fsm.run(torch.from_numpy(data).cuda(), scheme="sre", chunk_bytes=B)
+    res = fsm.run(torch.from_numpy(data).cuda(), scheme=scheme, chunk_bytes=B)
     check_equal(res, ref, B, w.nstates)
-    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme="sre")
+    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme=scheme)
     for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks",
               "verify_matches"):
         assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])

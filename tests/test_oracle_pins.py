@@ -284,7 +284,7 @@ def test_lookback_containment(seed):
 
 
 # ----------------------------------------------------------- simulate -------
-@pytest.mark.parametrize("scheme", ["seq", "pm", "sre", "rr", "nf"])
+@pytest.mark.parametrize("scheme", ["seq", "pm", "sre", "rr", "nf", "cse"])
 @pytest.mark.parametrize("seed", range(6))
 def test_simulate_equals_sequential(scheme, seed):
     rng = random.Random(seed * 31 + len(scheme))
@@ -359,10 +359,41 @@ def test_simulate_rr_bound_and_nf_order():
                 assert [c for c, _ in helpers] == sorted(c for c, _ in helpers)
 
 
+def test_simulate_cse_exact_coverage():
+    """CSE: when a chunk's lookback-2 image has <= spec_k states, round 0
+    ran every state of it, and the true start is in it (pinned by
+    test_lookback_containment), so verification needs no recovery there.  div7:
+    every 2-symbol image is all 7 states (closed form above) -> zero rounds, every
+    check matches.  Tiny random DFAs (n <= 8): every image has <= n states -> zero
+    rounds.  C3 (counter images > 8): recovery rounds remain, result still exact."""
+    t, s, a = gen.dfa_div7()
+    data = gen.workload("c1", length=50000, seed=3).host()
+    for B in (16, 256, 4096):
+        o = oracle.simulate(t, s, a, data, B, scheme="cse")
+        N = oracle.nchunks(len(data), B)
+        assert o["rounds"] == 0 and o["tasks_total"] == 0
+        assert o["verify_checks"] == o["verify_matches"] == N
+        pm = oracle.simulate(t, s, a, data, B, scheme="pm", spec_k=4)  # 4 of 7: must recover
+        assert pm["rounds"] > 0
+    for seed in range(8):
+        rng = random.Random(seed)
+        n, ns = rng.randint(1, 8), rng.randint(1, 6)
+        t, s, a = gen.dfa_random(seed + 11, n, ns)
+        data = gen.workload(f"rand:{n}:{ns}:{seed}", length=20000, seed=seed).host()
+        o = oracle.simulate(t, s, a, data, 64, scheme="cse")
+        r = oracle.run(t, s, a, data, 64)
+        assert o["rounds"] == 0 and o["final_state"] == r["final"] and o["accept_count"] == r["count"]
+    w = gen.workload("c3", length=1 << 18, seed=2)
+    data = w.host()
+    o = oracle.simulate(w.table, w.start, w.accept, data, 4096, scheme="cse")
+    r = oracle.run(w.table, w.start, w.accept, data, 4096)
+    assert o["rounds"] > 0 and o["final_state"] == r["final"] and (o["chunk_end"] == r["chunk_end"]).all()
+
+
 def test_simulate_invalid_symbol():
     t, s, a = gen.dfa_div7()
     data = np.array([1, 0, 1] * 100 + [3] + [1] * 50, np.uint8)
-    for scheme in ("seq", "sre", "rr", "nf", "pm"):
+    for scheme in ("seq", "sre", "rr", "nf", "pm", "cse"):
         o = oracle.simulate(t, s, a, data, 16, scheme=scheme)
         assert o["status"] == oracle.OR_ESYMBOL
 

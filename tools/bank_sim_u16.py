@@ -49,7 +49,43 @@ def wf(words):
     return m
 
 
-res = {k: 0 for k in ("row", "rowpad", "col", "cold_lanes", "any_cold")}
+# greedy bank-aware row placement (the u8 placement of fsm_load, on class words):
+# states by profile visits; each takes the free row slot whose bank rotation
+# (slot * padw mod 32) puts its word histogram on the least-loaded banks
+prof = data[: 1 << 20]
+visits = np.zeros(nt)
+hist = np.zeros((nt, padw))
+t0 = perm[w.start]
+pcl = cls[prof]
+tcur = t0
+for i in range(len(prof)):
+    visits[tcur] += 1
+    hist[tcur, pcl[i] // 2] += 1
+    tcur = tt[tcur, prof[i]]
+slot_of = np.zeros(nt, np.int64)
+nslots = ((nt + 31) // 32 + 1) * 32
+free = np.ones(nslots, bool)
+load = np.zeros(32)
+for q in np.argsort(-visits, kind='stable'):
+    if visits[q] == 0:
+        r = int(np.nonzero(free)[0][0])
+    else:
+        best, bc = -1, 0
+        for rot in range(32):
+            cand = np.nonzero(free[rot::32])[0]
+            if len(cand) == 0:
+                continue
+            r0 = rot + 32 * int(cand[0])
+            cost = sum(hist[q, wd] * load[(wd + r0 * padw) % 32] for wd in range(padw))
+            if best < 0 or cost < bc:
+                best, bc = r0, cost
+        r = best
+    free[r] = False
+    slot_of[q] = r
+    for wd in range(padw):
+        load[(wd + r * padw) % 32] += hist[q, wd]
+
+res = {k: 0 for k in ("row", "rowpad", "col", "greedy", "cold_lanes", "any_cold")}
 for s in range(steps):
     cl = cls[byts[:, :, s]]
     for wi in range(nw):
@@ -60,6 +96,7 @@ for s in range(steps):
         res["row"] += wf(((th * C + c) * 2) // 4)
         res["rowpad"] += wf(th * padw + (c * 2) // 4)
         res["col"] += wf(((c * Hp + th) * 2) // 4)
+        res["greedy"] += wf(slot_of[t] * padw + (c * 2) // 4)
         res["cold_lanes"] += (~hot).sum()
         res["any_cold"] += (~hot).any()
     st = tt[st, byts[:, :, s]]
