@@ -111,6 +111,14 @@ void place_rows_bank_aware(fsm_t f, const std::vector<uint32_t>& ttc, uint32_t C
   }
 }
 
+// ENUM sub-chunk size E | B: halve down to 256 B while the map count stays <= 4 M (measured
+// on C1: going further, to 64 B, made the scan levels cost more than the walk saved).
+uint32_t enum_sub_bytes(uint32_t B, uint64_t len) {
+  uint32_t E = B;
+  while (E % 32 == 0 && E > 256 && (len + E / 2 - 1) / (E / 2) <= (1ull << 22)) E /= 2;
+  return E;
+}
+
 struct Opts {
   fsm_scheme scheme;
   uint32_t B, k, k_cse, L, qs_cap, vr_end, vr_oth;
@@ -259,8 +267,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       return fail(FSM_EUNSUPPORTED, "ENUM needs nstates + 1 <= 32");
     }
     // sub-chunk size E | B: small enough for parallelism, bounded scratch
-    uint32_t E = o.B;
-    while (E % 32 == 0 && E > 256 && (len + E / 2 - 1) / (E / 2) <= (1ull << 22)) E /= 2;
+    const uint32_t E = enum_sub_bytes(o.B, len);
     const uint64_t nsub = (len + E - 1) / E;
     const uint64_t need = enum_scratch_bytes(nsub);
     if (f->enum_bytes < need) {
@@ -271,7 +278,8 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       CUDA_TRY(cudaMalloc(&f->enum_base, need));
       f->enum_bytes = need;
     }
-    CUDA_TRY(cudaMemcpyAsync(f->d_ctl, &h, sizeof(Ctl), cudaMemcpyHostToDevice, o.st));
+    rp.ctl_init = f->d_ctl;  // the walk kernel initialises the control block (no H2D copy)
+    rp.h_out = &h;           // ... and the output kernel writes it back (pinned, UVA)
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
     CUDA_TRY(launch_enum_full(f->img, rp, E, f->enum_base, d_chunk_ends, f->d_ctl, &f->d_ctl->xfin, o.st,
                               f->sm_count));
@@ -1068,11 +1076,6 @@ int resolve_scheme(fsm_t f, const uint8_t* d_in, uint64_t len, const fsm_run_opt
   return FSM_OK;
 }
 
-uint32_t enum_sub_bytes(uint32_t B, uint64_t len) {
-  uint32_t E = B;
-  while (E % 32 == 0 && E > 256 && (len + E / 2 - 1) / (E / 2) <= (1ull << 22)) E /= 2;
-  return E;
-}
 
 int ensure_enum_scratch(fsm_t f, uint64_t nsub) {
   const uint64_t need = enum_scratch_bytes(nsub);

@@ -21,8 +21,9 @@ constexpr uint32_t kGroup = 64;
 template <int MODE, int NE>
 __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* __restrict__ in, uint64_t len,
                                                   uint32_t E, uint64_t nsub, uint8_t* __restrict__ M,
-                                                  uint64_t* __restrict__ Cn) {
+                                                  uint64_t* __restrict__ Cn, Ctl* ctl_init, uint32_t q0t, uint64_t N) {
   extern __shared__ __align__(1024) uint8_t smem[];
+  if (ctl_init && blockIdx.x == 0) init_ctl(ctl_init, q0t, N);  // the run's control block (no H2D copy)
   stage_table(img, smem);
   __syncthreads();
   using S = Step<MODE>;
@@ -132,7 +133,7 @@ __global__ void k_enum_descend(const uint8_t* __restrict__ P, const uint64_t* __
 __global__ void k_enum_out(DevImage img, const uint32_t* __restrict__ st0, const uint8_t* __restrict__ P0top,
                            const uint64_t* __restrict__ PC0top, uint64_t top_last, uint32_t q0t, uint64_t nsub,
                            uint32_t per_chunk, uint64_t N, uint32_t* __restrict__ chunk_ends, Ctl* ctl,
-                           uint32_t* __restrict__ x_final) {
+                           uint32_t* __restrict__ x_final, void* h_out) {
   const uint32_t fin = P0top[top_last * 32 + q0t];
   for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < N; c += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t jn = (c + 1) * per_chunk;  // first sub-chunk after chunk c
@@ -142,6 +143,12 @@ __global__ void k_enum_out(DevImage img, const uint32_t* __restrict__ st0, const
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     *x_final = fin;
     ctl->accept_count = PC0top[top_last * 32 + q0t];
+    if (h_out) {  // zero-copy result: publish the control block to the run's pinned host slot
+      __threadfence();
+      const uint32_t* src = reinterpret_cast<const uint32_t*>(ctl);
+      uint32_t* dst = reinterpret_cast<uint32_t*>(h_out);
+      for (uint32_t i = 0; i < sizeof(Ctl) / 4; i++) dst[i] = __ldcg(src + i);
+    }
   }
 }
 
@@ -155,7 +162,7 @@ cudaError_t walk_t(const DevImage& img, const RunParams& rp, uint32_t E, uint64_
   uint64_t grid = (nsub + 127) / 128;
   const uint64_t cap = (uint64_t)sms * 16;
   if (grid > cap) grid = cap;
-  kern<<<(unsigned)grid, 128, smem, st>>>(img, rp.in, rp.len, E, nsub, M, Cn);
+  kern<<<(unsigned)grid, 128, smem, st>>>(img, rp.in, rp.len, E, nsub, M, Cn, rp.ctl_init, rp.q0t, rp.N);
   return cudaGetLastError();
 }
 
@@ -240,7 +247,7 @@ cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t 
   if (grid > (uint64_t)sms * 16) grid = (uint64_t)sms * 16;
   if (grid < 1) grid = 1;
   k_enum_out<<<(unsigned)grid, 256, 0, st>>>(img, lv[0].s, lv[L - 1].M, lv[L - 1].C, top_last, rp.q0t, nsub,
-                                             rp.B / E, rp.N, d_chunk_ends, d_ctl, d_x_final);
+                                             rp.B / E, rp.N, d_chunk_ends, d_ctl, d_x_final, rp.h_out);
   return cudaGetLastError();
 }
 
