@@ -199,6 +199,55 @@ __device__ uint32_t untried(const DevImage& img, const RunParams& rp, const RecS
   return m;
 }
 
+// Chained (Gauss-Seidel) relaxation pass over chunks [c0, hi) by one warp (see the
+// pass loop): x_{c+1} = F_c(x_c), F_c(x) = VR_c(x).end if x in dom VR_c else cur_end[c].
+// Returns whether any x_{c+1} changed.  Lane l holds chunk (b0 + l)'s default end and up
+// to kChainRec END records in registers; chunks with more records (or VR^others records)
+// fall back to the full lookup for their own step.
+constexpr int kChainRec = 8;
+__device__ bool chain_pass(const RecStore& rs, const RunParams& rp, uint64_t c0, uint64_t hi, uint64_t f,
+                           uint32_t tf) {
+  const uint32_t lane = threadIdx.x & 31;
+  bool ch = false;
+  if (c0 >= hi) return false;
+  uint32_t x = (c0 == f) ? tf : ld_cg(rs.x + c0);
+  for (uint64_t b0 = c0; b0 < hi; b0 += 32) {
+    const uint64_t c = b0 + lane;
+    const bool in = c < hi;
+    const uint64_t cc = in ? c : hi - 1;
+    const uint32_t dflt = ld_cg(rs.cur_end + cc);
+    const uint32_t ne = min(ld_cg(rs.n_end + cc), rp.vr_end), no = min(ld_cg(rs.n_oth + cc), rp.vr_oth);
+    const uint32_t xo = ld_cg(rs.x + cc + 1);
+    uint32_t s[kChainRec], e[kChainRec];
+#pragma unroll
+    for (int j = 0; j < kChainRec; j++) {
+      s[j] = (uint32_t)j < ne ? ld_cg(rs.start + (uint64_t)j * rs.cap + cc) : kNone;
+      e[j] = (uint32_t)j < ne ? ld_cg(rs.end + (uint64_t)j * rs.cap + cc) : 0u;
+    }
+    const bool spill = ne > (uint32_t)kChainRec || no > 0;
+    const uint32_t steps = (uint32_t)min((uint64_t)32, hi - b0);
+    uint32_t mine = 0;
+    for (uint32_t i = 0; i < steps; i++) {  // lane i resolves chunk b0 + i
+      uint32_t y = dflt;
+      bool hit = false;
+#pragma unroll
+      for (int j = 0; j < kChainRec; j++)
+        if (s[j] == x) { y = e[j]; hit = true; }
+      if (lane == i && !hit && spill) {
+        uint32_t y2;
+        if (vr_lookup(rs, rp.vr_end, rp.vr_oth, cc, x, &y2, nullptr)) y = y2;
+      }
+      x = __shfl_sync(0xffffffffu, y, i);
+      if (lane == i) mine = x;
+    }
+    if (in && mine != xo) {
+      st_cg(rs.x + c + 1, mine);
+      ch = true;
+    }
+  }
+  return ch;
+}
+
 // FSM_Processing over chunk c from `start` with path fusion: walk in lockstep
 // with the chunk's round-0 path; once the two states coincide the rest of the
 // path is known (DFA determinism), so end/count follow from the reference.
@@ -433,6 +482,19 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       }
       bool ch = false;
       uint64_t fm = ~0ull, matches = 0, checks = 0;
+      // A chaotic pass moves a value one chunk per pass through chunks whose records
+      // all match (a non-convergent DFA with several records per chunk: PM/CSE/RR/NF on
+      // div7-like machines needs ~N passes).  From the 4th pass of a round on, every
+      // other pass is a CHAINED (Gauss-Seidel) pass: warp 0 of each CTA propagates
+      // x_{c+1} = F_c(x_c) through the CTA's whole range in order — one warp step per
+      // chunk, each lane holding its chunk's function (default end + kChainRec records)
+      // in registers, the running value passed lane to lane by shuffle — so a pass
+      // crosses a whole CTA range.  Same unique fixed point; the pass that ends the
+      // round is always a normal pass (it does the bookkeeping below).
+      const bool chain = it >= 3 && (it & 1u);
+      if (chain) {
+        if (threadIdx.x < 32) ch = chain_pass(rs, rp, max(lo, f), hi, f, tf);
+      } else
       // batched: a thread's kU chunks issue all their loads (incoming state, current
       // outgoing state, default end, record slot 0) before any is resolved; reading
       // x[c] early is allowed by the chaotic relaxation (a later write by chunk c-1's
@@ -500,7 +562,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       const bool any = vctl->changed[slot] != 0;
       it++;
       git++;
-      if (!any) break;
+      if (!any && !chain) break;  // a chained pass did no bookkeeping: a normal pass ends the round
     }
     const uint64_t f2 = vctl->it_fm[slot];
     if (b == 0 && threadIdx.x == 0) {

@@ -6,6 +6,9 @@
   * Table III analogue: runtime speculation accuracy = verify matches / checks
     and average active workers per recovery round
   * Fig. 7 analogue: VR^others slots sweep for RR
+  * Fig. 9 analogue: verification+recovery time per recovered chunk, normalised to SRE
+    (RR/NF activate more threads per round; is a recovery cheaper or dearer?)
+  * CSE (extension): every lookback candidate up to 8 with path fusion
 
 Datasets are the synthetic configs of DESIGN.md §4 (the paper's Snort/ClamAV/PowerEN
 FSMs are out of scope).  Every run is checked against the oracle on a sample.
@@ -45,7 +48,7 @@ def main():
                 best = (t, r)
         return best
 
-    for cfg in ("c2", "c3", "c3s"):
+    for cfg in ("c2", "c3", "c3s", "c4"):
         w = gen.workload(cfg, length=length)
         x = torch.empty(length, dtype=torch.uint8, device="cuda")
         w.device(x)
@@ -54,8 +57,9 @@ def main():
         ref = None
         rows = []
         base_t = None
-        for scheme in ("pm", "sre", "rr", "nf", "auto"):
-            if scheme == "pm" and cfg != "c2":
+        fig9 = {}
+        for scheme in ("pm", "sre", "rr", "nf", "cse", "auto"):
+            if scheme == "pm" and cfg in ("c3", "c3s"):
                 # PM's stage 2 is sequential (one must-do per round): on low-accuracy
                 # DFAs it needs ~N rounds, so it is timed on a 1/64 prefix and scaled
                 xs = x[: length // 64]
@@ -63,11 +67,13 @@ def main():
                 t *= 64
             else:
                 t, r = timed(fsm, x, scheme=scheme)
-            if not (scheme == "pm" and cfg != "c2"):
+            if not (scheme == "pm" and cfg in ("c3", "c3s")):
                 if ref is None:
                     ref = (r.final_state, r.accept_count)
                 assert (r.final_state, r.accept_count) == ref, (cfg, scheme)
             st = r.stats
+            if st["tasks_total"] and scheme in ("sre", "rr", "nf"):
+                fig9[scheme] = st["ms_verify"] / st["tasks_total"]
             acc = st["verify_matches"] / max(1, st["verify_checks"])
             if scheme == "pm":
                 base_t = t
@@ -83,6 +89,12 @@ def main():
                   "| rounds | tasks | re-read MiB |\n|---|---|---|---|---|---|---|---|")
         for row in rows:
             md.append("| %s | %.3f | %.2fx | %.1f | %.1f | %d | %d | %d |" % row)
+        if "sre" in fig9:
+            md.append("\nrecovery time per recovered chunk, normalised to SRE (Fig. 9 analogue): " +
+                      ", ".join(f"{k}: {v / fig9['sre']:.2f}" for k, v in fig9.items()))
+            for k, v in fig9.items():
+                lines.append({"exp": "fig9_recovery_per_chunk", "config": cfg, "scheme": k,
+                              "us_per_task": 1e3 * v, "vs_sre": v / fig9["sre"]})
         # Fig. 3: alpha_k (speculative execution time only)
         t1 = None
         al = []
