@@ -290,6 +290,21 @@ def test_dense_recovery_rounds(gs, name, length, B, scheme):
     assert res.stats["tasks_sre"] > 2048  # the dense path really ran
 
 
+@pytest.mark.parametrize("scheme,B", [("cse", 64), ("cse", 16), ("rr", 64), ("nf", 256)])
+def test_chained_verification_passes(gs, scheme, B):
+    """div7 with several records per chunk: non-convergent chains that a chaotic pass
+    advances one chunk at a time; the chained (Gauss-Seidel) passes cross whole CTA
+    ranges (16 K-64 K chunks over many CTAs).  Results and round diagnostics stay exact."""
+    w, data = _wl("c1", 1 << 20)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    fsm = _fsm(gs, w)
+    res = fsm.run(torch.from_numpy(data).cuda(), scheme=scheme, chunk_bytes=B)
+    check_equal(res, ref, B, w.nstates)
+    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme=scheme)
+    for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "verify_checks", "verify_matches"):
+        assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+
+
 @pytest.mark.parametrize("name,length,scheme", [("c3", 1 << 30, "auto"), ("c3", 1 << 30, "sre"), ("c4", 4 << 30, "auto")])
 def test_full_size_other_configs(gs, name, length, scheme):
     """BASELINE configs C3 (1 GB) and C4 (4 GB) at full size vs the oracle."""
