@@ -307,20 +307,21 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     }
     rp.ctl_init = nullptr;  // initialised by the spec kernel; later launches must not touch it
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
-    for (;;) {
+    // dense rounds are device-driven: `slots` (task kernel + finish + verify) triples are
+    // queued behind the first verify launch; a verify launch that needs a dense round
+    // hands it to the next triple, or runs it in-kernel when none is left; launches after
+    // the run completed return at once.  No host round trip: runs stay queued back to back.
+    const uint32_t slots = rp.dense ? f->dense_hint : 0;
+    rp.dense_slots = slots;
+    CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
+    pd.launches++;
+    for (uint32_t r = 0; r < slots; r++) {
+      CUDA_TRY(launch_task_dense(f->img, rp, f->rs, f->d_ctl, f->sm_count, o.st));
+      rp.dense_slots = slots - 1 - r;
       CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
-      pd.launches++;
-      if (!rp.dense) break;
-      uint32_t pend = 0;
-      uint64_t fm = 0, nt = 0;
-      CUDA_TRY(cudaMemcpyAsync(&pend, &f->d_ctl->dense_pending, 4, cudaMemcpyDeviceToHost, o.st));
-      CUDA_TRY(cudaMemcpyAsync(&fm, &f->d_ctl->fmin, 8, cudaMemcpyDeviceToHost, o.st));
-      CUDA_TRY(cudaMemcpyAsync(&nt, &f->d_ctl->ntask[0], 8, cudaMemcpyDeviceToHost, o.st));
-      CUDA_TRY(cudaStreamSynchronize(o.st));
-      if (!pend) break;
-      CUDA_TRY(launch_task_dense(f->img, rp, f->rs, f->d_ctl, fm, nt, f->sm_count, o.st));
-      pd.launches += 2;  // TMA task kernel + finish
+      pd.launches += 3;  // task kernel + finish + verify (no-ops once the run is complete)
     }
+    pd.dense_slots = slots;
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   }
   if (rp.h_out) {
@@ -351,6 +352,10 @@ int run_collect(fsm_t f, uint64_t ticket, fsm_result* out, uint32_t* final_tid) 
   cudaEventElapsedTime(&t1, f->ev[slot][0], f->ev[slot][1]);
   cudaEventElapsedTime(&t2, f->ev[slot][1], f->ev[slot][2]);
   fill_result_stats(out, h);
+  if (pd.dense_slots) {  // size the next run's dense slots to the rounds this one used
+    const uint32_t used = h.dense_rounds + (h.dense_denied ? 1u : 0u);
+    f->dense_hint = std::min<uint32_t>(16u, std::max<uint32_t>(1u, used));
+  }
   f->last_nstamp = std::min<uint32_t>(h.nstamp, 24);
   std::copy(h.stamp, h.stamp + 24, f->last_stamp);
   std::copy(h.tl, h.tl + 4, f->last_tl);

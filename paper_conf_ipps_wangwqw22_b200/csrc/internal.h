@@ -121,6 +121,11 @@ struct Ctl {
   // run timeline (%globaltimer ns; GSPEC_STAMPS=1): spec entry, last spec warp done,
   // verify entry (before table staging), verify exit (last CTA, before the host publish)
   uint64_t tl[4];
+  // device-driven dense rounds (no host round trip): the verify finalize sets `finished`
+  // (later launches of the run return at once); the finish kernel counts dense rounds;
+  // `dense_denied` = a verify launch ran a dense round in-kernel because the run had no
+  // task-kernel slot left (the host raises its slot count for the next run)
+  uint32_t finished, dense_rounds, dense_denied, pad2;
 };
 
 struct RunParams {
@@ -134,6 +139,7 @@ struct RunParams {
   uint32_t qs_cap;
   uint32_t vr_end, vr_oth;
   uint32_t dense;  // 1: hand rounds with many SRE tasks to the TMA task kernel (verify exits)
+  uint32_t dense_slots;  // task-kernel launches still queued behind this verify launch
   Ctl* ctl_init;   // non-null: the first spec kernel initialises this control block (no H2D copy)
   const uint32_t* q0_dev;  // non-null: chunk 0's start is read from the device (shard candidates)
   Ctl* h_out;      // non-null: pinned host slot; the finalize step writes the control block there
@@ -226,11 +232,13 @@ cudaError_t launch_build_qs2_raw(const uint32_t* d_ttc, uint32_t n, uint32_t C, 
 cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st);
 cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, int sms, cudaStream_t st,
                             uint64_t* n_done);
-// Dense recovery round: the round's task list (rs.task_chunk/task_start, ntask entries, all
-// chunks >= f2) is re-walked by the TMA-gather task kernel (full chunks) and the tail kernel
-// (rs.tstart of the partial last chunk); then the round is committed.
-cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
-                              uint64_t ntask, int sms, cudaStream_t st);
+// Dense recovery round, device-driven: if the preceding verify launch left a dense round
+// pending (ctl->dense_pending), its task list (rs.task_chunk/task_start, ctl->ntask[0]
+// entries, all chunks >= ctl->fmin) is re-walked by the TMA-gather task kernel (full
+// chunks) and the finish kernel (tail chunk, round commit); otherwise both return at once.
+// Enqueued without any host synchronisation.
+cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, int sms,
+                              cudaStream_t st);
 bool spec_path_generic_only();  // GSPEC_SPEC_PATH=generic forces the non-TMA kernel (A/B tests)
 cudaError_t launch_verify_recover(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* d_ctl,
                                   uint64_t* d_block_tmp, uint32_t* d_chunk_ends, cudaStream_t st, int sm_count);
@@ -309,6 +317,7 @@ struct fsm_s {
     bool active = false;
     uint32_t done_ev = 3;  // event that marks the result readable (2: zero-copy result)
     uint32_t launches = 0; // kernels enqueued for this run
+    uint32_t dense_slots = 0;  // dense task-kernel slots queued for this run
   } pend[kRing];
   uint64_t next_seq = 1;
   uint64_t* d_block_tmp = nullptr;
@@ -321,6 +330,7 @@ struct fsm_s {
   int device = 0;
   fsm_scheme auto_scheme = FSM_SCHEME_SRE;
   double acc1_hint = 0.0;            // spec-1 accuracy from the selector's profile (dense-round gate)
+  uint32_t dense_hint = 4;           // task-kernel slots queued per dense run (dense rounds last seen)
   bool auto_selected = false;
   const uint32_t* d_ttc = nullptr;   // [nt][C] transformed tid x class table (prep/features)
   uint32_t* d_small = nullptr;       // small device scratch (ENUM final state, shard compose)

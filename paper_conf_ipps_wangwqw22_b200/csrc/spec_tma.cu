@@ -96,6 +96,11 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   uint32_t* prow = reinterpret_cast<uint32_t*>(bars + ((nwarps * S + 1) & ~1u)) + warp * 32;  // TASKS: producer group's chunks
   stage_table(img, table);  // load-time data: staged before the dependency wait
   pdl_wait();                // the previous kernel in the stream (e.g. the last run's verify) is done
+  if (TASKS) {  // device-driven dense round: the task list and frontier come from the control block
+    if (!__ldcg(&ctl->dense_pending)) return;  // the verify launch before us handed no round over
+    ntask = __ldcg(reinterpret_cast<const unsigned long long*>(&ctl->ntask[0]));
+    f2 = __ldcg(reinterpret_cast<const unsigned long long*>(&ctl->fmin));
+  }
   if (rp.ctl_init && blockIdx.x == 0) {
     init_ctl(rp.ctl_init, q0_of(rp), rp.N);
     if (rp.stamps && threadIdx.x == 0) rp.ctl_init->tl[0] = gtimer();
@@ -110,7 +115,10 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
 
   const uint32_t segs = rp.B / kRowBytes;
   const uint64_t ntiles = TASKS ? (ntask + 31) / 32 : (n_full + 31) / 32 - tile0;
-  const uint64_t gw = (uint64_t)blockIdx.x * nwarps + warp, tw = (uint64_t)gridDim.x * nwarps;
+  // TASKS: the task list may cover only part of the grid; warp-major numbering spreads
+  // its groups over every SM (CTA-major would pack them into the first CTAs)
+  const uint64_t gw = TASKS ? (uint64_t)warp * gridDim.x + blockIdx.x : (uint64_t)blockIdx.x * nwarps + warp;
+  const uint64_t tw = (uint64_t)gridDim.x * nwarps;
   if (gw >= ntiles) return;
   struct StampEnd {  // timeline: the last warp to finish (profiling only)
     bool on; Ctl* c; uint32_t lane;
@@ -409,15 +417,16 @@ cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecS
   return e;
 }
 
-// Dense recovery round over the task list (ntask entries): chunks < n_full are walked
-// here; the tail chunk (if its task is listed) is left to the finish kernel.
-cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
-                            uint64_t ntask, int sms, cudaStream_t st, uint64_t* n_done) {
+// Dense recovery round over the task list (ctl->ntask[0] entries, read on the device):
+// chunks < n_full are walked here; the tail chunk (if its task is listed) is left to the
+// finish kernel.  Launched with the grid of a full list (one CTA per SM, persistent).
+cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, int sms,
+                            cudaStream_t st, uint64_t* n_done) {
   *n_done = 0;
   const uint64_t n_full = rp.len / rp.B;
   CUtensorMap tm;
-  if (f2 >= n_full || !tma_applies(rp, n_full) || !encode_map(rp, n_full, &tm, true)) return cudaErrorNotSupported;
-  const uint64_t tile0 = 0;
+  if (!tma_applies(rp, n_full) || !encode_map(rp, n_full, &tm, true)) return cudaErrorNotSupported;
+  const uint64_t tile0 = 0, f2 = 0, ntask = n_full;  // launch-shape hints; the kernel reads the real values
   cudaError_t e;
   switch (img.mode) {
     case MODE_U8: e = launch_tma_s<MODE_U8, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;

@@ -316,6 +316,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   stage_table(img, smem);  // the table is load-time data: staged before the dependency wait
   pdl_wait();               // the spec kernel's records are complete and visible
   pdl_launch_dependents();  // the next run's spec kernel may launch (it waits for us the same way)
+  if (ctl->finished) return;  // an earlier launch of this run completed it (spare dense slot)
   stamp();
   __syncthreads();
   stamp();
@@ -582,11 +583,14 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       // task kernel over chunk tiles (same tasks, same records) and relaunches us
       const uint64_t nt = ld_cg64(&ctl->it_ntask[slot]);
       if (nt >= 2048 && nt * 16 >= N - f2) {
-        if (b == 0 && threadIdx.x == 0) {
-          vctl->ntask[0] = nt;  // the task list's length (this pass's slot) for the host launch
-          vctl->dense_pending = 1;
+        if (rp.dense_slots > 0) {  // a task kernel is queued behind us: hand the round over
+          if (b == 0 && threadIdx.x == 0) {
+            vctl->ntask[0] = nt;  // the task list's length (this pass's slot) for the task kernel
+            vctl->dense_pending = 1;
+          }
+          return;
         }
-        return;
+        if (b == 0 && threadIdx.x == 0) vctl->dense_denied = 1;  // run it here (phase E below)
       }
     }
     if (fast) {
@@ -845,7 +849,10 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     }
     total = block_sum<uint64_t>(total, red64);
     if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->accept_count), (unsigned long long)total);
-    if (b == 0 && threadIdx.x == 0) ctl->xfin = ld_cg(rs.x + N);
+    if (b == 0 && threadIdx.x == 0) {
+      ctl->xfin = ld_cg(rs.x + N);
+      ctl->finished = 1;  // before this CTA's fence + ticket: the publishing CTA sees it
+    }
     stamp();
     if (rp.h_out) {
       // zero-copy result: the last CTA to finish publishes the control block to the
@@ -921,6 +928,7 @@ __global__ void __launch_bounds__(256) k_dense_finish(DevImage img, RunParams rp
                                                       uint64_t c_first_generic) {
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ uint32_t any;
+  if (!ctl->dense_pending) return;  // no dense round was handed over (spare slot)
   const uint64_t f2 = ctl->fmin;
   if (threadIdx.x == 0) {
     any = 0;
@@ -948,6 +956,7 @@ __global__ void __launch_bounds__(256) k_dense_finish(DevImage img, RunParams rp
     ctl->reread_bytes += min((uint64_t)rp.B, rp.len - c * rp.B);
   }
   ctl->rounds++;
+  ctl->dense_rounds++;
   ctl->f = f2;
   ctl->tf = ld_cg(rs.x + f2);
   ctl->dense_pending = 0;
@@ -969,15 +978,15 @@ cudaError_t launch_dense_finish(const DevImage& img, const RunParams& rp, const 
 
 }  // namespace
 
-cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint64_t f2,
-                            uint64_t ntask, int sms, cudaStream_t st, uint64_t* n_done);
+cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, int sms,
+                            cudaStream_t st, uint64_t* n_done);
 
-cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp_in, const RecStore& rs, Ctl* ctl, uint64_t f2,
-                              uint64_t ntask, int sms, cudaStream_t st) {
+cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp_in, const RecStore& rs, Ctl* ctl, int sms,
+                              cudaStream_t st) {
   RunParams rp = rp_in;
   rp.ctl_init = nullptr;  // the control block is live: never re-initialise it mid-run
   uint64_t done = 0;
-  cudaError_t e = launch_task_tma(img, rp, rs, ctl, f2, ntask, sms, st, &done);
+  cudaError_t e = launch_task_tma(img, rp, rs, ctl, sms, st, &done);
   if (e == cudaErrorNotSupported) {
     cudaGetLastError();
     done = 0;  // the finish kernel walks everything (slow, but exact)
