@@ -167,6 +167,18 @@ int fsm_run_batch(fsm_t fsm, const uint8_t* d_input, const uint64_t* h_offsets, 
                   const fsm_run_opts* opts, uint32_t* d_final, uint64_t* d_count, uint32_t* d_chunk_ends,
                   fsm_batch_result* out);
 
+/* Paper-literal SRE (Alg. 2 L2-6 + Alg. 3, P:98-102, P:162-179,
+ * verbatim): ONE CTA, one thread per chunk, a shared `mark`, one frontier step per
+ * iteration with a CTA barrier, exactly N iterations; a must-do recovery is one
+ * thread's walk of its chunk.  A reference point for fsm_run's batched-frontier
+ * design (same results; R13).  Only opts->chunk_bytes, vr_end and stream
+ * are used (VR_tid = one FIFO list of vr_end records).  d_input / d_chunk_ends as in
+ * fsm_run.  Synchronous.  Errors: FSM_EUNSUPPORTED when ceil(len / chunk_bytes) >
+ * 1024; FSM_ESYMBOL as fsm_run.  Stats: rounds = iterations with a must-do recovery,
+ * tasks_* = re-executions, verify_* over all N iterations, ms_verify = kernel time. */
+int fsm_run_literal(fsm_t fsm, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
+                    uint32_t* d_chunk_ends, fsm_result* out);
+
 /* Same as fsm_run with HOST buffers: copies h_input to the device (pinned
  * memory recommended), runs, and copies chunk ends back to h_chunk_ends
  * (nullable).  Used for end-to-end timing. */

@@ -56,6 +56,8 @@ def lib():
         L.or_compose.argtypes = [U32, P, P, P, P, P, P]
         L.or_simulate.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, ctypes.c_int, U32, U32, U32, U32,
                                   P, ctypes.POINTER(SimResult), P, U64, P]
+        L.or_simulate_literal_sre.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, U32, P,
+                                              ctypes.POINTER(SimResult)]
         L.or_features_compute.argtypes = [P, U32, U32, U32, P, P, U64, U32, U32, U32, ctypes.POINTER(Features)]
         L.or_select.argtypes = [ctypes.POINTER(Features), U32]
         _LIB = L
@@ -162,6 +164,22 @@ def simulate(table, start, accept, data, B=4096, scheme="sre", spec_k=None, qs_c
                     for i in range(min(nt.value, max_tasks))]
     out["ntasks"] = nt.value
     out["perm"] = perm
+    return out
+
+
+def simulate_literal_sre(table, start, accept, data, B=4096, vr_cap=16, policy=0):
+    """Paper-literal SRE: Alg. 2 L2-6 then Alg. 3 verbatim, N iterations."""
+    perm, inv, _, tt, acc = transform(table, accept, policy, data if policy == 1 else None, start)
+    t = _c(table, np.uint32)
+    n, ns = t.shape
+    d = _c(data, np.uint8)
+    ce = np.zeros(max(1, nchunks(d.size, B)), np.uint32)
+    res = SimResult()
+    rc = lib().or_simulate_literal_sre(tt.ctypes.data, n, ns, int(perm[start]), acc.ctypes.data, inv.ctypes.data,
+                                       d.ctypes.data, d.size, B, vr_cap, ce.ctypes.data, ctypes.byref(res))
+    out = res.as_dict()
+    out["status"] = rc
+    out["chunk_end"] = ce[:nchunks(d.size, B)]
     return out
 
 

@@ -98,6 +98,13 @@ int or_simulate(const uint32_t* tt, uint32_t nt, uint32_t nsyms, uint32_t q0t, c
                 uint32_t* chunk_end, or_sim_result* res, or_task* tasks, uint64_t max_tasks,
                 uint64_t* ntasks);
 
+/* Paper-literal SRE (Alg. 2 L2-6 + Alg. 3 verbatim, one frontier step per iteration,
+ * exactly N iterations).  Same outputs as or_run; diagnostics: rounds =
+ * iterations with a must-do recovery, tasks_total = re-executions. */
+int or_simulate_literal_sre(const uint32_t* tt, uint32_t nt, uint32_t nsyms, uint32_t q0t, const uint8_t* acc_t,
+                            const uint32_t* inv, const uint8_t* in, uint64_t len, uint32_t B, uint32_t vr_cap,
+                            uint32_t* chunk_end, or_sim_result* res);
+
 typedef struct {
   double acc1, acck, sens, uniq10;
 } or_features;

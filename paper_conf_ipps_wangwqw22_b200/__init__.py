@@ -64,6 +64,7 @@ _lib.fsm_num_chunks.argtypes = [U64, U32]
 _lib.fsm_num_chunks.restype = U64
 _lib.fsm_run.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
 _lib.fsm_run_host.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
+_lib.fsm_run_literal.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
 _lib.fsm_run_async.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(U64)]
 _lib.fsm_wait.argtypes = [P, U64, ctypes.POINTER(fsm_result)]
 _lib.fsm_batch_chunks.argtypes = [P, U32, U32]
@@ -203,6 +204,19 @@ class FSM:
         r = fsm_result()
         _check(_lib.fsm_wait(self._h, ticket, ctypes.byref(r)), "fsm_wait")
         return Result.from_c(r)
+
+    def run_literal(self, x, chunk_bytes=4096, vr_end=16, stream=None) -> Result:
+        """fsm_run_literal: the paper-literal single-CTA SRE kernel (Alg. 2 L2-6 + Alg. 3
+        verbatim, <= 1024 chunks) on a uint8 CUDA tensor."""
+        o = _run_opts("sre", chunk_bytes, vr_end=vr_end, stream=stream)
+        n = fsm_num_chunks(x.numel(), chunk_bytes)
+        import torch
+
+        ce = torch.empty(max(n, 1), dtype=torch.int32, device=x.device)
+        r = fsm_result()
+        _check(_lib.fsm_run_literal(self._h, x.data_ptr() if x.numel() else None, x.numel(), ctypes.byref(o),
+                                    ce.data_ptr(), ctypes.byref(r)), "fsm_run_literal")
+        return Result.from_c(r, ce[:n])
 
     def run_host(self, data: np.ndarray, scheme="auto", chunk_bytes=4096, chunk_ends=True, stream=None,
                  **kw) -> Result:

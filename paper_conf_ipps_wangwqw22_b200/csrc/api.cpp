@@ -866,6 +866,58 @@ int fsm_run_batch(fsm_t f, const uint8_t* d_input, const uint64_t* h_offsets, ui
   return FSM_OK;
 }
 
+int fsm_run_literal(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
+                    uint32_t* d_chunk_ends, fsm_result* out) {
+  entry_clear("fsm_run_literal");
+  if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
+  if (!d_input && len > 0) return fail(FSM_EINVAL, "NULL input");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  const uint64_t N = fsm_num_chunks(len, o.B);
+  if (N > literal_max_chunks()) return fail(FSM_EUNSUPPORTED, "paper-literal kernel: at most 1024 chunks (one CTA)");
+  std::memset(out, 0, sizeof(*out));
+  out->nchunks = N;
+  out->scheme_used = FSM_SCHEME_SRE;
+  uint32_t fin = f->img.q0t;
+  if (N) {
+    if ((rc = ensure_ctl(f))) return rc;
+    CUDA_TRY(cudaStreamSynchronize(o.st));  // queued runs may still use the record store
+    if ((rc = ensure_records(f, N))) return rc;
+    RunParams rp{};
+    rp.in = d_input;
+    rp.q0t = f->img.q0t;
+    rp.len = len;
+    rp.B = o.B;
+    rp.N = N;
+    rp.scheme = FSM_SCHEME_SRE;
+    rp.k = 1;
+    rp.vr_end = o.vr_end;
+    rp.vr_oth = o.vr_oth;
+    for (auto& e : f->batch_ev)
+      if (!e) CUDA_TRY(cudaEventCreate(&e));
+    cudaEvent_t e0 = f->batch_ev[0], e1 = f->batch_ev[1];
+    CUDA_TRY(cudaMemsetAsync(f->d_ctl, 0, sizeof(Ctl), o.st));
+    CUDA_TRY(cudaEventRecord(e0, o.st));
+    CUDA_TRY(launch_literal_sre(f->img, rp, f->rs, f->d_ctl, d_chunk_ends, o.st));
+    CUDA_TRY(cudaEventRecord(e1, o.st));
+    Ctl h;
+    CUDA_TRY(cudaMemcpyAsync(&h, f->d_ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, o.st));
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+    fill_result_stats(out, h);
+    out->accept_count = h.accept_count;
+    float t = 0;
+    cudaEventElapsedTime(&t, e0, e1);
+    out->ms_verify = t;
+    out->kernel_launches = 1;
+    fin = h.xfin;
+  }
+  if (fin == f->n) return fail(FSM_ESYMBOL, "input symbol >= nsyms");
+  out->final_state = f->inv[fin];
+  out->accept = f->accept[out->final_state];
+  return FSM_OK;
+}
+
 int fsm_run_host(fsm_t f, const uint8_t* h_input, uint64_t len, const fsm_run_opts* opts, uint32_t* h_chunk_ends,
                  fsm_result* out) {
   entry_clear("fsm_run_host");

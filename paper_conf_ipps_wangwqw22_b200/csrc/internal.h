@@ -239,6 +239,11 @@ cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecS
 // Enqueued without any host synchronisation.
 cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, int sms,
                               cudaStream_t st);
+// Paper-literal SRE: one CTA, one thread per chunk (N <= literal_max_chunks()),
+// Alg. 2 L2-6 + Alg. 3 verbatim; results and stats in *ctl (zeroed by the caller).
+uint32_t literal_max_chunks();
+cudaError_t launch_literal_sre(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl,
+                               uint32_t* d_chunk_ends, cudaStream_t st);
 bool spec_path_generic_only();  // GSPEC_SPEC_PATH=generic forces the non-TMA kernel (A/B tests)
 cudaError_t launch_verify_recover(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* d_ctl,
                                   uint64_t* d_block_tmp, uint32_t* d_chunk_ends, cudaStream_t st, int sm_count);

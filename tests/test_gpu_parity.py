@@ -290,6 +290,27 @@ def test_dense_recovery_rounds(gs, name, length, B, scheme):
     assert res.stats["tasks_sre"] > 2048  # the dense path really ran
 
 
+@pytest.mark.parametrize("name,length,B", [("c1", 1 << 20, 4096), ("c2", 4 << 20, 16384), ("c3", 2 << 20, 8192),
+                                           ("c4", 2 << 20, 4096), ("c2", (1 << 20) + 77, 2048), ("c1", 100, 16),
+                                           ("c2", 0, 4096)])
+def test_paper_literal_sre(gs, name, length, B):
+    """The paper-literal single-CTA kernel: bit-exact results, and Alg. 3's
+    per-iteration accounting equal to the oracle's literal simulation."""
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    fsm = _fsm(gs, w)
+    x = torch.from_numpy(data).cuda() if length else torch.empty(0, dtype=torch.uint8, device="cuda")
+    res = fsm.run_literal(x, chunk_bytes=B)
+    assert res.final_state == ref["final"] and res.accept_count == ref["count"]
+    if length:
+        assert (res.chunk_ends.cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
+        sim = oracle.simulate_literal_sre(w.table, w.start, w.accept, data, B)
+        for k in ("rounds", "tasks_mustdo", "tasks_sre", "reread_bytes", "verify_checks", "verify_matches"):
+            assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+    with pytest.raises(gs.GSpecError):
+        fsm.run_literal(torch.zeros(1025 * 16, dtype=torch.uint8, device="cuda"), chunk_bytes=16)
+
+
 @pytest.mark.parametrize("scheme,B", [("cse", 64), ("cse", 16), ("rr", 64), ("nf", 256)])
 def test_chained_verification_passes(gs, scheme, B):
     """div7 with several records per chunk: non-convergent chains that a chaotic pass

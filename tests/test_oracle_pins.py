@@ -390,6 +390,32 @@ def test_simulate_cse_exact_coverage():
     assert o["rounds"] > 0 and o["final_state"] == r["final"] and (o["chunk_end"] == r["chunk_end"]).all()
 
 
+@pytest.mark.parametrize("seed", range(6))
+def test_simulate_literal_sre(seed):
+    """Paper-literal SRE (Alg. 2 L2-6 + Alg. 3 verbatim) reaches the sequential
+    result (the invariant of Alg. 3: after the iteration with frontier f every chunk <= f
+    holds its true end) on random DFAs and chunkings; Alg. 3's accounting: one must-do per
+    iteration whose frontier missed, at most N of them, every re-execution is a task."""
+    rng = random.Random(seed * 7 + 1)
+    n, ns = rng.randint(1, 24), rng.randint(1, 5)
+    t, s, a = gen.dfa_random(seed + 21, n, ns)
+    data = gen.workload(f"rand:{n}:{ns}:{seed}", length=rng.randint(0, 4000), seed=seed).host()
+    for B in (16, 48, 256):
+        r = oracle.run(t, s, a, data, B)
+        o = oracle.simulate_literal_sre(t, s, a, data, B, vr_cap=rng.randint(1, 16))
+        N = oracle.nchunks(len(data), B)
+        assert o["status"] == 0
+        assert o["final_state"] == r["final"] and o["accept_count"] == r["count"]
+        assert (o["chunk_end"] == r["chunk_end"]).all()
+        assert o["rounds"] == o["tasks_mustdo"] <= max(N, 0)
+        assert o["tasks_total"] >= o["rounds"] and o["verify_checks"] == N * N
+    # a DFA whose lookback always predicts right (one state): no recovery at all
+    t1 = np.zeros((1, 3), np.uint32)
+    d1 = np.array([0, 1, 2] * 300, np.uint8)
+    o = oracle.simulate_literal_sre(t1, 0, np.array([1], np.uint8), d1, 16)
+    assert o["rounds"] == 0 and o["accept_count"] == len(d1)
+
+
 def test_simulate_invalid_symbol():
     t, s, a = gen.dfa_div7()
     data = np.array([1, 0, 1] * 100 + [3] + [1] * 50, np.uint8)
