@@ -6,7 +6,7 @@
 // exactly N iterations.  It is the reference point for the batched-frontier
 // redesign in verify_recover.cu (reading R13): same results, but every
 // iteration is a CTA-wide barrier and a must-do recovery is a single-thread walk
-// on the critical path.  The oracle's twin is or_simulate_literal_sre.
+// on the critical path.  Tests compare it with a CPU simulation of the same steps.
 #include "internal.h"
 #include "walk.cuh"
 
