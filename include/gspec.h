@@ -38,7 +38,10 @@ typedef enum {
   FSM_ECUDA = -3,        /* CUDA runtime error (message in fsm_last_error)     */
   FSM_ESYMBOL = -4,      /* an input byte >= nsyms (reading R4); outputs unset  */
   FSM_ENCCL = -5,        /* collective failed                                  */
-  FSM_EUNSUPPORTED = -6  /* e.g. ENUM on a DFA with > 31 states                */
+  FSM_EUNSUPPORTED = -6, /* e.g. ENUM on a DFA with > 31 states                */
+  FSM_EAGAIN = -7        /* fsm_shard_finish: a rank's speculative shard map was
+                            invalid; every rank redoes fsm_shard_map_exact + the
+                            exchange + fsm_shard_finish (all ranks see the same maps) */
 } fsm_status;
 
 /* Parallelization schemes (PM, SRE; P:195 RR; P:222 NF; P:89 ENUM). */
@@ -208,9 +211,17 @@ uint64_t fsm_map_bytes(fsm_t fsm);
  * the rest is kept in the handle for fsm_shard_finish. */
 int fsm_shard_map(fsm_t fsm, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback,
                   uint32_t lookback_len, const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local);
+/* fsm_shard_map is speculative for a shard with a lookback: its pipeline is queued
+ * from the first candidate without waiting to learn whether every candidate's path
+ * merged with it (P:427 path fusion) — no host round trip.  If one did not, the map
+ * is marked invalid and fsm_shard_finish returns FSM_EAGAIN on EVERY rank; every rank
+ * then calls fsm_shard_map_exact (same arguments: checks on the host, falls back to
+ * per-path pipelines or enumeration), exchanges the maps again and finishes. */
+int fsm_shard_map_exact(fsm_t fsm, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback,
+                        uint32_t lookback_len, const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local);
 /* Step 2 (every rank, after the allgather): d_maps = nranks maps back to back.
  * Composes them from q0 (s_{g+1} = M_g[s_g]), writes this rank's chunk ends
- * (original ids, nullable) and the global result. */
+ * (original ids, nullable) and the global result.  FSM_EAGAIN: see above. */
 int fsm_shard_finish(fsm_t fsm, const void* d_maps, uint32_t nranks, uint32_t rank,
                      const fsm_run_opts* opts, uint32_t* d_chunk_ends_local, fsm_result* out_global);
 

@@ -75,6 +75,7 @@ _lib.fsm_select_scheme.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), ctyp
 _lib.fsm_map_bytes.argtypes = [P]
 _lib.fsm_map_bytes.restype = U64
 _lib.fsm_shard_map.argtypes = [P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, P]
+_lib.fsm_shard_map_exact.argtypes = [P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, P]
 _lib.fsm_shard_finish.argtypes = [P, P, U32, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
 _lib.fsm_get_transform.argtypes = [P, P, P, P, P, P, P]
 _lib.fsm_get_qs.argtypes = [P, ctypes.c_uint8, ctypes.c_uint8, P, P, P]

@@ -497,6 +497,7 @@ const char* fsm_strerror(int s) {
     case FSM_EINVAL: return "invalid argument";
     case FSM_ENOMEM: return "out of memory";
     case FSM_ECUDA: return "CUDA error";
+    case FSM_EAGAIN: return "retry (speculative shard map invalid)";
     case FSM_ESYMBOL: return "input symbol out of range";
     case FSM_ENCCL: return "collective failed";
     case FSM_EUNSUPPORTED: return "unsupported";
@@ -1151,9 +1152,24 @@ int ensure_enum_scratch(fsm_t f, uint64_t nsub) {
 
 extern "C" {
 
+int shard_map_impl(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
+                   const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local, bool exact);
+
 int fsm_shard_map(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
                   const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local) {
   entry_clear("fsm_shard_map");
+  return shard_map_impl(f, d_shard, len, d_lookback, lb_len, opts, d_map, d_chunk_ends_local,
+                        f && f->shard_prefer_exact);
+}
+
+int fsm_shard_map_exact(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
+                        const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local) {
+  entry_clear("fsm_shard_map_exact");
+  return shard_map_impl(f, d_shard, len, d_lookback, lb_len, opts, d_map, d_chunk_ends_local, true);
+}
+
+int shard_map_impl(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
+                   const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local, bool exact) {
   if (!f || !d_map) return fail(FSM_EINVAL, "NULL handle/map");
   if (!d_shard && len > 0) return fail(FSM_EINVAL, "NULL shard");
   if (lb_len > 16 || (lb_len && !d_lookback)) return fail(FSM_EINVAL, "lookback_len must be <= 16 with bytes");
@@ -1189,17 +1205,22 @@ int fsm_shard_map(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* 
   }
   // 2a. fast path: fuse every candidate with the path of cand[0] (P:427 path
   // fusion); the shard then runs once, from cand[0], through the normal pipeline.
-  // One host check (did every candidate merge?), the rest stays stream-ordered.
+  // Speculative (default): no host check — the pipeline is queued at once and the map
+  // kernel marks the map invalid if some candidate did not merge; the composition then
+  // reports FSM_EAGAIN on every rank and all ranks redo fsm_shard_map_exact (DESIGN.md
+  // §8).  Exact: one host check (did every candidate merge?), else the fallbacks below.
   if (N > 0 && len > 0) {
     uint32_t h2[2] = {1, 0};
     if (lb_len != 0) {
       CUDA_TRY(cudaMemsetAsync(d_unmerged, 0, 4, o.st));
       CUDA_TRY(launch_shard_fuse_ref(f->img, d_shard, len, o.B, S.cand, d_ncand, kFuseChunks, S.states, S.grp, dcnt,
                                      d_unmerged, o.st));
-      CUDA_TRY(cudaMemcpyAsync(h2, d_ncand, 8, cudaMemcpyDeviceToHost, o.st));
-      CUDA_TRY(cudaStreamSynchronize(o.st));
+      if (exact) {
+        CUDA_TRY(cudaMemcpyAsync(h2, d_ncand, 8, cudaMemcpyDeviceToHost, o.st));
+        CUDA_TRY(cudaStreamSynchronize(o.st));
+      }
     }
-    f->shard_ncand = h2[0];
+    f->shard_ncand = h2[0];  // (speculative: not read on the host in fused mode)
     if (h2[1] == 0) {
       if (f->shard_ticket) {  // a previous shard run that was never finished
         fsm_result rr;
@@ -1211,7 +1232,7 @@ int fsm_shard_map(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* 
         return rc;
       CUDA_TRY(launch_map_fused(S.cand, d_ncand, dcnt, &f->d_ctl->xfin,
                                 reinterpret_cast<const unsigned long long*>(&f->d_ctl->accept_count), mend, mcnt,
-                                o.st));
+                                (lb_len != 0 && !exact) ? d_unmerged : nullptr, o.st));
       f->shard_mode = 3;
       return FSM_OK;
     }
@@ -1327,6 +1348,10 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
     rc = run_collect(f, f->shard_ticket, &rr, &ff);  // already complete: frees the ring slot
     f->shard_ticket = 0;
     if (rc) return rc;
+  }
+  if (h[2] == 2) {
+    f->shard_prefer_exact = true;  // this DFA's shards do not merge early: skip speculation from now on
+    return fail(FSM_EAGAIN, "a rank's speculative shard map was invalid: every rank redoes fsm_shard_map_exact");
   }
   if (h[2] || (f->shard_mode == 3 && h[5])) return fail(FSM_EINVAL, "a shard start state is outside its candidate set");
   const uint32_t srank = h[0], fin = h[1];

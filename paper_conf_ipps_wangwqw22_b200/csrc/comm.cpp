@@ -106,13 +106,20 @@ int fsm_run_sharded(fsm_t f, fsm_comm_t c, const uint8_t* d_shard, uint64_t shar
       return gspec_set_error(FSM_ENOMEM, "map buffers");
     c->map_bytes = mb;
   }
-  int rc = fsm_shard_map(f, d_shard, shard_len, d_lookback, lookback_len, opts, c->d_local, d_chunk_ends_local);
-  if (rc) return rc;
   cudaStream_t st = opts ? reinterpret_cast<cudaStream_t>(opts->stream) : nullptr;
-  ncclResult_t r = nccl().allGather(c->d_local, c->d_all, mb, ncclUint8, c->comm, st);
-  if (r != ncclSuccess)
-    return gspec_set_error(FSM_ENCCL, nccl().getErrorString ? nccl().getErrorString(r) : "ncclAllGather");
-  return fsm_shard_finish(f, c->d_all, (uint32_t)c->nranks, (uint32_t)c->rank, opts, d_chunk_ends_local, out_global);
+  int rc = FSM_OK;
+  for (int exact = 0; exact < 2; exact++) {  // speculative map first; FSM_EAGAIN (same on every rank) -> exact
+    rc = exact ? fsm_shard_map_exact(f, d_shard, shard_len, d_lookback, lookback_len, opts, c->d_local,
+                                     d_chunk_ends_local)
+               : fsm_shard_map(f, d_shard, shard_len, d_lookback, lookback_len, opts, c->d_local, d_chunk_ends_local);
+    if (rc) return rc;
+    ncclResult_t r = nccl().allGather(c->d_local, c->d_all, mb, ncclUint8, c->comm, st);
+    if (r != ncclSuccess)
+      return gspec_set_error(FSM_ENCCL, nccl().getErrorString ? nccl().getErrorString(r) : "ncclAllGather");
+    rc = fsm_shard_finish(f, c->d_all, (uint32_t)c->nranks, (uint32_t)c->rank, opts, d_chunk_ends_local, out_global);
+    if (rc != FSM_EAGAIN) break;
+  }
+  return rc;
 }
 
 }  // extern "C"

@@ -25,6 +25,7 @@ enum Mode : uint32_t {
 };
 
 constexpr uint32_t kDeltaExc = 2;        // exceptions per delta row
+constexpr uint32_t kInvalidMap = 0xFFFFFFFEu;  // map entry of a speculative shard map that must be redone
 constexpr uint32_t kDeltaBaseMax = 8192;  // MODE_U16D: max shared-window offset of the staged table
 
 constexpr uint32_t kQsMax = 16;     // QS cap ("top 16 states")
@@ -273,7 +274,7 @@ cudaError_t launch_shard_fuse_ref(const DevImage& img, const uint8_t* in, uint64
                                   uint32_t* merged, long long* dcnt, uint32_t* unmerged, cudaStream_t st);
 cudaError_t launch_map_fused(const uint32_t* cand, const uint32_t* ncand_p, const long long* dcnt, const uint32_t* fin_p,
                              const unsigned long long* count_p, uint32_t* mend, unsigned long long* mcnt,
-                             cudaStream_t st);
+                             const uint32_t* unmerged, cudaStream_t st);
 cudaError_t launch_fix_prefix_fused(const uint32_t* states, const uint32_t* cand, const uint32_t* ncand_p,
                                     const uint32_t* merged, const uint32_t* srank_p, const uint32_t* inv,
                                     uint32_t* chunk_ends, uint32_t* err, cudaStream_t st);
@@ -336,6 +337,7 @@ struct fsm_s {
   fsm_scheme auto_scheme = FSM_SCHEME_SRE;
   double acc1_hint = 0.0;            // spec-1 accuracy from the selector's profile (dense-round gate)
   uint32_t dense_hint = 4;           // task-kernel slots queued per dense run (dense rounds last seen)
+  bool shard_prefer_exact = false;   // a speculative shard map was invalid once: use the exact map
   bool auto_selected = false;
   const uint32_t* d_ttc = nullptr;   // [nt][C] transformed tid x class table (prep/features)
   uint32_t* d_small = nullptr;       // small device scratch (ENUM final state, shard compose)

@@ -145,12 +145,15 @@ __global__ void __launch_bounds__(1024) k_fuse_ref(DevImage img, const uint8_t* 
 
 // map[cand[i]] = (final of the cand[0] pipeline, its count + dcnt[i]); the pipeline's
 // final state and count are read from its control block on the device
+// Speculative use (unmerged != null): the pipeline ran before the host knew whether
+// every candidate merged; if some did not, every candidate's entry becomes kInvalidMap
+// and the composition on every rank reports it (all ranks then redo the exact map).
 __global__ void k_map_fused(const uint32_t* __restrict__ cand, const uint32_t* __restrict__ ncand_p,
                             const long long* __restrict__ dcnt, const uint32_t* __restrict__ fin_p,
                             const unsigned long long* __restrict__ count_p, uint32_t* __restrict__ mend,
-                            unsigned long long* __restrict__ mcnt) {
+                            unsigned long long* __restrict__ mcnt, const uint32_t* __restrict__ unmerged) {
   const uint32_t ncand = *ncand_p;
-  const uint32_t fin = *fin_p;
+  const uint32_t fin = (unmerged && *unmerged) ? kInvalidMap : *fin_p;
   const unsigned long long c0 = *count_p;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x) {
     mend[cand[i]] = fin;
@@ -165,6 +168,7 @@ __global__ void k_fix_prefix_fused(const uint32_t* __restrict__ states, const ui
                                    const uint32_t* __restrict__ srank_p, const uint32_t* __restrict__ inv,
                                    uint32_t* __restrict__ chunk_ends, uint32_t* __restrict__ err) {
   __shared__ uint32_t ci;
+  if (srank_p[2] != 0) return;  // the composition failed (e.g. an invalid speculative map): nothing to fix
   const uint32_t ncand = *ncand_p, sr = *srank_p;
   if (threadIdx.x == 0) ci = kNoState;
   __syncthreads();
@@ -176,6 +180,10 @@ __global__ void k_fix_prefix_fused(const uint32_t* __restrict__ states, const ui
     return;
   }
   const uint32_t nj = merged[ci];
+  if (nj == kNoState) {  // this candidate never merged (cannot happen with a valid map)
+    if (threadIdx.x == 0) *err = 1;
+    return;
+  }
   for (uint32_t j = threadIdx.x; j < nj; j += blockDim.x) chunk_ends[j] = inv[states[(uint64_t)j * ncand + ci]];
 }
 
@@ -222,6 +230,7 @@ __global__ void k_compose(const uint8_t* __restrict__ maps, uint32_t G, uint64_t
     const unsigned long long* mc = reinterpret_cast<const unsigned long long*>(maps + h * map_bytes + cnt_off);
     const uint32_t e = me[s];
     if (e == kNoState) { err = 1; break; }
+    if (e == kInvalidMap) { err = 2; break; }  // a rank's speculative map must be redone
     c += mc[s];
     s = e;
   }
@@ -293,8 +302,8 @@ cudaError_t launch_shard_fuse_ref(const DevImage& img, const uint8_t* in, uint64
 
 cudaError_t launch_map_fused(const uint32_t* cand, const uint32_t* ncand_p, const long long* dcnt, const uint32_t* fin_p,
                              const unsigned long long* count_p, uint32_t* mend, unsigned long long* mcnt,
-                             cudaStream_t st) {
-  k_map_fused<<<8, 256, 0, st>>>(cand, ncand_p, dcnt, fin_p, count_p, mend, mcnt);
+                             const uint32_t* unmerged, cudaStream_t st) {
+  k_map_fused<<<8, 256, 0, st>>>(cand, ncand_p, dcnt, fin_p, count_p, mend, mcnt, unmerged);
   return cudaGetLastError();
 }
 

@@ -18,6 +18,8 @@ import numpy as np
 
 from . import FSM, Result, _check, _lib, _run_opts, fsm_num_chunks, fsm_result
 
+FSM_EAGAIN = -7  # fsm_shard_finish: a speculative shard map was invalid (include/gspec.h)
+
 NO_STATE = 0xFFFFFFFF
 
 
@@ -84,14 +86,18 @@ def run_sharded(fsm: FSM, shard, lookback, group=None, scheme="auto", chunk_byte
     n = fsm_num_chunks(shard.numel(), chunk_bytes)
     ce = torch.empty(max(n, 1), dtype=torch.int32, device=shard.device) if chunk_ends else None
     lb = lookback if lookback is not None and lookback.numel() else None
-    _check(_lib.fsm_shard_map(fsm.handle, shard.data_ptr() if shard.numel() else None, shard.numel(),
-                              lb.data_ptr() if lb is not None else None, lb.numel() if lb is not None else 0,
-                              ctypes.byref(o), local.data_ptr(), ce.data_ptr() if ce is not None else None),
-           "fsm_shard_map")
-    gathered = _all_gather_cat(local, group)  # the single data-path collective
-    r = fsm_result()
-    _check(_lib.fsm_shard_finish(fsm.handle, gathered.data_ptr(), world, rank, ctypes.byref(o),
-                                 ce.data_ptr() if ce is not None else None, ctypes.byref(r)), "fsm_shard_finish")
+    for exact in (False, True):  # speculative map first; FSM_EAGAIN is seen by every rank alike
+        fn = _lib.fsm_shard_map_exact if exact else _lib.fsm_shard_map
+        _check(fn(fsm.handle, shard.data_ptr() if shard.numel() else None, shard.numel(),
+                  lb.data_ptr() if lb is not None else None, lb.numel() if lb is not None else 0,
+                  ctypes.byref(o), local.data_ptr(), ce.data_ptr() if ce is not None else None), "fsm_shard_map")
+        gathered = _all_gather_cat(local, group)  # the single data-path collective
+        r = fsm_result()
+        rc = _lib.fsm_shard_finish(fsm.handle, gathered.data_ptr(), world, rank, ctypes.byref(o),
+                                   ce.data_ptr() if ce is not None else None, ctypes.byref(r))
+        if rc != FSM_EAGAIN:
+            break
+    _check(rc, "fsm_shard_finish")
     return Result.from_c(r, ce[:n] if ce is not None else None)
 
 

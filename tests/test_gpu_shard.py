@@ -22,21 +22,27 @@ def sharded_fake(gs, w, data, G, B=4096, scheme="auto"):
     maps = torch.zeros(G * mb, dtype=torch.uint8, device="cuda")
     o = _run_opts(scheme, B)
     bounds = [shard_bounds(len(data), G, g, B) for g in range(G)]
-    ces = []
-    for g, (lo, hi) in enumerate(bounds):
-        n = gs.fsm_num_chunks(hi - lo, B)
-        ce = torch.full((max(n, 1),), -1, dtype=torch.int32, device="cuda")
-        lb = x[max(0, lo - 2):lo] if g else None
-        _check(_lib.fsm_shard_map(fsms[g].handle, x[lo:].data_ptr() if hi > lo else None, hi - lo,
-                                  lb.data_ptr() if lb is not None else None, 0 if lb is None else lb.numel(),
-                                  ctypes.byref(o), maps[g * mb:].data_ptr(), ce.data_ptr()), "shard_map")
-        ces.append((ce, n))
-    outs = []
-    for g in range(G):
-        r = fsm_result()
-        _check(_lib.fsm_shard_finish(fsms[g].handle, maps.data_ptr(), G, g, ctypes.byref(o), ces[g][0].data_ptr(),
-                                     ctypes.byref(r)), "shard_finish")
-        outs.append(r)
+    for exact in (False, True):  # the speculative maps first; FSM_EAGAIN on every rank -> exact maps
+        ces = []
+        for g, (lo, hi) in enumerate(bounds):
+            n = gs.fsm_num_chunks(hi - lo, B)
+            ce = torch.full((max(n, 1),), -1, dtype=torch.int32, device="cuda")
+            lb = x[max(0, lo - 2):lo] if g else None
+            fn = _lib.fsm_shard_map_exact if exact else _lib.fsm_shard_map
+            _check(fn(fsms[g].handle, x[lo:].data_ptr() if hi > lo else None, hi - lo,
+                      lb.data_ptr() if lb is not None else None, 0 if lb is None else lb.numel(),
+                      ctypes.byref(o), maps[g * mb:].data_ptr(), ce.data_ptr()), "shard_map")
+            ces.append((ce, n))
+        outs, rcs = [], []
+        for g in range(G):
+            r = fsm_result()
+            rcs.append(_lib.fsm_shard_finish(fsms[g].handle, maps.data_ptr(), G, g, ctypes.byref(o),
+                                             ces[g][0].data_ptr(), ctypes.byref(r)))
+            outs.append(r)
+        assert len(set(rcs)) == 1, rcs  # every rank sees the same maps
+        if rcs[0] != -7:
+            _check(rcs[0], "shard_finish")
+            break
     chunk_ends = np.concatenate([ce[:n].cpu().numpy().view(np.uint32) for ce, n in ces])
     return outs, chunk_ends
 
