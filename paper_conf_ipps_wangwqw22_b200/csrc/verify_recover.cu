@@ -360,6 +360,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         vctl->it_checks[nx] = vctl->it_matches[nx] = vctl->it_ntask[nx] = vctl->it_reread[nx] = 0;
       }
       uint64_t fm = ~0ull, matches = 0, checks = 0, ntask = 0, reread = 0;
+      bool tch = false;  // some task's chunk end differs from its round-0 end
       for (uint64_t cb = lo + threadIdx.x; cb < hi; cb += kU * kBS) {
         uint32_t xin[kU], s0[kU];
 #pragma unroll
@@ -387,13 +388,15 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
             st_cg(rs.cnt + o, cnt);
             st_cg(rs.n_end + c, ne + 1);
             st_cg(rs.cur_end + c, e);
+            tch |= e != ld_cg(rs.x + c + 1);  // x[c+1] still holds the round-0 end here
             ntask++;
             reread += min((uint64_t)rp.B, rp.len - c * rp.B);
           }
         }
       }
       bool bch = false;
-      block_reduce_pass(false, fm, checks, matches, red4, &bch);
+      block_reduce_pass(tch, fm, checks, matches, red4, &bch);
+      if (threadIdx.x == 0 && bch) vctl->changed[slot] = 1;
       ntask = block_sum<uint64_t>(ntask, red64);
       reread = block_sum<uint64_t>(reread, red64);
       if (threadIdx.x == 0) {
@@ -430,6 +433,20 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       tf = tf2;
       rnd++;
       last_tasks = nt;
+      if (vctl->changed[slot] == 0) {
+        // No task changed its chunk's end (every recovery merged with the round-0 path —
+        // the usual case for convergent DFAs): the incoming states x are those of round 0,
+        // and every chunk now holds a record for its incoming state (its round-0 record, or
+        // the task's from x_c).  Round 1's verification therefore matches every chunk from
+        // f2 on: count its N - f2 checks (all matches, as the oracle does) and finish
+        // without the pass.
+        if (b == 0 && threadIdx.x == 0) {
+          vctl->verify_checks = vctl->verify_checks + (N - f2);
+          vctl->verify_matches = vctl->verify_matches + (N - f2);
+          vctl->fmin = N;
+        }
+        break;
+      }
       continue;  // round 1 verification: the tasks' records are visible (grid barrier above)
     }
     // level 2 pays off when a round's relaxation makes several passes: spec-k records,
