@@ -322,6 +322,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       pd.launches += 3;  // task kernel + finish + verify (no-ops once the run is complete)
     }
     pd.dense_slots = slots;
+    pd.dense = rp.dense != 0;
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   }
   if (rp.h_out) {
@@ -352,9 +353,10 @@ int run_collect(fsm_t f, uint64_t ticket, fsm_result* out, uint32_t* final_tid) 
   cudaEventElapsedTime(&t1, f->ev[slot][0], f->ev[slot][1]);
   cudaEventElapsedTime(&t2, f->ev[slot][1], f->ev[slot][2]);
   fill_result_stats(out, h);
-  if (pd.dense_slots) {  // size the next run's dense slots to the rounds this one used
+  if (pd.dense) {  // size the next run's dense slots to the rounds this one used (0: none queued;
+                   // a run that then needs one runs it in-kernel and sets dense_denied)
     const uint32_t used = h.dense_rounds + (h.dense_denied ? 1u : 0u);
-    f->dense_hint = std::min<uint32_t>(16u, std::max<uint32_t>(1u, used));
+    f->dense_hint = std::min<uint32_t>(16u, used);
   }
   f->last_nstamp = std::min<uint32_t>(h.nstamp, 24);
   std::copy(h.stamp, h.stamp + 24, f->last_stamp);

@@ -324,6 +324,7 @@ struct fsm_s {
     uint32_t done_ev = 3;  // event that marks the result readable (2: zero-copy result)
     uint32_t launches = 0; // kernels enqueued for this run
     uint32_t dense_slots = 0;  // dense task-kernel slots queued for this run
+    bool dense = false;        // dense rounds were enabled for this run
   } pend[kRing];
   uint64_t next_seq = 1;
   uint64_t* d_block_tmp = nullptr;

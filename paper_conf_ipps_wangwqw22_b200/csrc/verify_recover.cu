@@ -351,7 +351,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     // Records and every counter are those of the listed-task rounds; x[c+1] is left
     // to the next relaxation pass (it reads the new record), so this pass only reads
     // round-0 values.
-    if (fast && rp.scheme == FSM_SCHEME_SRE && rp.k == 1 && rnd == 0 && f == 0 && !rp.dense) {
+    if (fast && rp.scheme == FSM_SCHEME_SRE && rp.k == 1 && rnd == 0 && f == 0 && rp.dense_slots == 0) {
       const uint32_t slot = git % 3;
       if (b == 0 && threadIdx.x == 0) {
         const uint32_t nx = (git + 1) % 3;
@@ -413,6 +413,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       const uint64_t f2 = vctl->it_fm[slot];
       const uint64_t nt = vctl->it_ntask[slot];
       if (b == 0 && threadIdx.x == 0) {
+        if (rp.dense && nt >= 2048 && nt * 16 >= N) vctl->dense_denied = 1;  // a dense round ran here
         vctl->verify_checks = vctl->verify_checks + vctl->it_checks[slot];
         vctl->verify_matches = vctl->verify_matches + vctl->it_matches[slot];
         vctl->jacobi_iters = vctl->jacobi_iters + 1;
