@@ -341,6 +341,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   uint32_t tf = vctl->tf;
   uint32_t rnd = (uint32_t)vctl->rounds;
   uint64_t last_tasks = 0;  // tasks of the previous round (this launch)
+  bool z_early = false;     // the round-0 pass already wrote the chunk ends and summed the counts
   for (;;) {
     // ---- round 0 of SRE with spec-1 records: verification + inline recovery --------
     // With one record per chunk and cur_end = that record's end, F_c(x) = end_c for
@@ -359,15 +360,17 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         vctl->it_fm[nx] = N;
         vctl->it_checks[nx] = vctl->it_matches[nx] = vctl->it_ntask[nx] = vctl->it_reread[nx] = 0;
       }
-      uint64_t fm = ~0ull, matches = 0, checks = 0, ntask = 0, reread = 0;
+      uint64_t fm = ~0ull, matches = 0, checks = 0, ntask = 0, reread = 0, ztot = 0;
       bool tch = false;  // some task's chunk end differs from its round-0 end
       for (uint64_t cb = lo + threadIdx.x; cb < hi; cb += kU * kBS) {
-        uint32_t xin[kU], s0[kU];
+        uint32_t xin[kU], s0[kU], xo[kU], c0[kU];
 #pragma unroll
         for (int u = 0; u < kU; u++) {
           const uint64_t c = min(cb + u * kBS, hi - 1);
           xin[u] = (c == 0) ? tf : ld_cg(rs.x + c);
           s0[u] = ld_cg(rs.start + c);
+          xo[u] = ld_cg(rs.x + c + 1);  // the round-0 end of chunk c
+          c0[u] = ld_cg(rs.cnt + c);
         }
 #pragma unroll
         for (int u = 0; u < kU; u++) {
@@ -377,6 +380,10 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
           rs.found[c] = hit;
           checks++;
           matches += hit;
+          // speculative finalize (phase Z): exact whenever this round ends the run (no task
+          // changes an end), which is decided after the barrier below
+          if (chunk_ends) chunk_ends[c] = __ldg(img.inv + xo[u]);
+          if (hit) ztot += c0[u];
           if (!hit) {
             fm = min(fm, c);
             uint32_t e, cnt;
@@ -388,7 +395,8 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
             st_cg(rs.cnt + o, cnt);
             st_cg(rs.n_end + c, ne + 1);
             st_cg(rs.cur_end + c, e);
-            tch |= e != ld_cg(rs.x + c + 1);  // x[c+1] still holds the round-0 end here
+            tch |= e != xo[u];  // x[c+1] still holds the round-0 end here
+            ztot += cnt;
             ntask++;
             reread += min((uint64_t)rp.B, rp.len - c * rp.B);
           }
@@ -399,7 +407,9 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       if (threadIdx.x == 0 && bch) vctl->changed[slot] = 1;
       ntask = block_sum<uint64_t>(ntask, red64);
       reread = block_sum<uint64_t>(reread, red64);
+      ztot = block_sum<uint64_t>(ztot, red64);
       if (threadIdx.x == 0) {
+        if (ztot) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->ntask[1]), (unsigned long long)ztot);
         if (fm != ~0ull) atomicMin(reinterpret_cast<unsigned long long*>(&ctl->it_fm[slot]), (unsigned long long)fm);
         if (checks) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->it_checks[slot]), (unsigned long long)checks);
         if (matches)
@@ -419,7 +429,10 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         vctl->jacobi_iters = vctl->jacobi_iters + 1;
         vctl->fmin = f2;
       }
-      if (f2 >= N) break;
+      if (f2 >= N) {
+        z_early = true;
+        break;
+      }
       const uint32_t tf2 = ld_cg(rs.x + f2);  // = end_{f2-1}: not rewritten by the tasks
       if (b == 0 && threadIdx.x == 0) {      // commit the round (the must-do is chunk f2)
         vctl->tasks_mustdo = vctl->tasks_mustdo + 1;
@@ -446,6 +459,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
           vctl->verify_matches = vctl->verify_matches + (N - f2);
           vctl->fmin = N;
         }
+        z_early = true;
         break;
       }
       continue;  // round 1 verification: the tasks' records are visible (grid barrier above)
@@ -845,7 +859,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   // ---------------- Z: finalize (chunk ends, u64 accept count) ----------------
   {
     uint64_t total = 0;
-    for (uint64_t cb = lo + threadIdx.x; cb < hi; cb += kU * kBS) {
+    for (uint64_t cb = lo + threadIdx.x; !z_early && cb < hi; cb += kU * kBS) {
       uint32_t xin[kU], xo[kU];
       VrPre pre[kU];
 #pragma unroll
@@ -865,8 +879,13 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         if (chunk_ends) chunk_ends[c] = __ldg(img.inv + xo[u]);
       }
     }
-    total = block_sum<uint64_t>(total, red64);
-    if (threadIdx.x == 0) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->accept_count), (unsigned long long)total);
+    if (z_early) {  // counts summed by the round-0 pass (complete: every CTA added before its barrier)
+      if (b == 0 && threadIdx.x == 0) ctl->accept_count = ld_cg64(&ctl->ntask[1]);
+    } else {
+      total = block_sum<uint64_t>(total, red64);
+      if (threadIdx.x == 0)
+        atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->accept_count), (unsigned long long)total);
+    }
     if (b == 0 && threadIdx.x == 0) {
       ctl->xfin = ld_cg(rs.x + N);
       ctl->finished = 1;  // before this CTA's fence + ticket: the publishing CTA sees it
