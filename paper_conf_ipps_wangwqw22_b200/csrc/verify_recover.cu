@@ -452,7 +452,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         // the usual case for convergent DFAs): the incoming states x are those of round 0,
         // and every chunk now holds a record for its incoming state (its round-0 record, or
         // the task's from x_c).  Round 1's verification therefore matches every chunk from
-        // f2 on: count its N - f2 checks (all matches, as the oracle does) and finish
+        // f2 on: count its N - f2 checks (all matches, per the round semantics) and finish
         // without the pass.
         if (b == 0 && threadIdx.x == 0) {
           vctl->verify_checks = vctl->verify_checks + (N - f2);
