@@ -182,6 +182,22 @@ int fsm_run_batch(fsm_t fsm, const uint8_t* d_input, const uint64_t* h_offsets, 
 int fsm_run_literal(fsm_t fsm, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
                     uint32_t* d_chunk_ends, fsm_result* out);
 
+/* FSM-level batching (Alg. 1 L2-3): npairs (DFA, stream)
+ * pairs — fsms[i] over d_inputs[i][0, lens[i]) (device pointers, any alignment) — in ONE
+ * launch per table format: one CTA per pair stages that DFA's table in shared memory and
+ * runs lookback-2 speculation + SRE rounds over the pair's stream in waves of 256 chunks
+ * (opts->chunk_bytes; other opts ignored).  Handles may repeat.  Writes h_final[i]
+ * (original id; 0xFFFFFFFF when the stream holds a symbol >= nsyms, and the call then
+ * returns FSM_ESYMBOL after filling every output) and h_count[i] (accept count).  out
+ * (nullable): re-walks, SRE rounds, kernel milliseconds.  Synchronous on opts->stream. */
+typedef struct {
+  uint64_t rewalks;  /* chunk re-executions over all pairs          */
+  uint64_t rounds;   /* SRE rounds with a re-execution, summed       */
+  float ms;          /* device time of the launches (CUDA events)    */
+} fsm_multi_result;
+int fsm_run_multi(const fsm_t* fsms, uint32_t npairs, const uint8_t* const* d_inputs, const uint64_t* lens,
+                  const fsm_run_opts* opts, uint32_t* h_final, uint64_t* h_count, fsm_multi_result* out);
+
 /* Same as fsm_run with HOST buffers: copies h_input to the device (pinned
  * memory recommended), runs, and copies chunk ends back to h_chunk_ends
  * (nullable).  Used for end-to-end timing. */

@@ -54,6 +54,10 @@ class fsm_batch_result(ctypes.Structure):
                 ("invalid_streams", U64), ("ms", ctypes.c_float)]
 
 
+class fsm_multi_result(ctypes.Structure):
+    _fields_ = [("rewalks", U64), ("rounds", U64), ("ms", ctypes.c_float)]
+
+
 class fsm_features(ctypes.Structure):
     _fields_ = [("acc1", ctypes.c_double), ("acck", ctypes.c_double), ("input_sensitivity", ctypes.c_double),
                 ("uniq10", ctypes.c_double), ("nstates", U32)]
@@ -70,6 +74,7 @@ _lib.fsm_wait.argtypes = [P, U64, ctypes.POINTER(fsm_result)]
 _lib.fsm_batch_chunks.argtypes = [P, U32, U32]
 _lib.fsm_batch_chunks.restype = U64
 _lib.fsm_run_batch.argtypes = [P, P, P, U32, ctypes.POINTER(fsm_run_opts), P, P, P, ctypes.POINTER(fsm_batch_result)]
+_lib.fsm_run_multi.argtypes = [P, U32, P, P, ctypes.POINTER(fsm_run_opts), P, P, ctypes.POINTER(fsm_multi_result)]
 _lib.fsm_select_scheme.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), ctypes.POINTER(ctypes.c_int),
                                    ctypes.POINTER(fsm_features)]
 _lib.fsm_map_bytes.argtypes = [P]
@@ -112,6 +117,24 @@ def lib_path() -> str:
 
 def fsm_num_chunks(length: int, chunk_bytes: int = 4096) -> int:
     return int(_lib.fsm_num_chunks(length, chunk_bytes))
+
+
+def run_multi(fsms, inputs, chunk_bytes=4096, stream=None):
+    """fsm_run_multi (FSM-level batching): fsms[i] over the uint8 CUDA tensor inputs[i], all
+    pairs in one launch per table format.  Returns (finals uint32 [n], counts uint64 [n],
+    stats dict); a final of 0xFFFFFFFF marks a stream with an invalid symbol (and raises)."""
+    n = len(fsms)
+    assert len(inputs) == n
+    hs = (ctypes.c_void_p * max(n, 1))(*[f.handle for f in fsms])
+    ptrs = (ctypes.c_void_p * max(n, 1))(*[x.data_ptr() if x.numel() else 0 for x in inputs])
+    lens = np.array([x.numel() for x in inputs] or [0], np.uint64)
+    fin = np.zeros(max(n, 1), np.uint32)
+    cnt = np.zeros(max(n, 1), np.uint64)
+    o = _run_opts("sre", chunk_bytes, stream=stream)
+    r = fsm_multi_result()
+    _check(_lib.fsm_run_multi(hs, n, ptrs, lens.ctypes.data, ctypes.byref(o), fin.ctypes.data, cnt.ctypes.data,
+                              ctypes.byref(r)), "fsm_run_multi")
+    return fin[:n], cnt[:n], {k: getattr(r, k) for k, _ in fsm_multi_result._fields_}
 
 
 def _run_opts(scheme="auto", chunk_bytes=4096, spec_k=0, qs_cap=16, vr_end=16, vr_others=16, stream=None):

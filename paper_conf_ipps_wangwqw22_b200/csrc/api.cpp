@@ -869,6 +869,97 @@ int fsm_run_batch(fsm_t f, const uint8_t* d_input, const uint64_t* h_offsets, ui
   return FSM_OK;
 }
 
+int fsm_run_multi(const fsm_t* fsms, uint32_t npairs, const uint8_t* const* d_inputs, const uint64_t* lens,
+                  const fsm_run_opts* opts, uint32_t* h_final, uint64_t* h_count, fsm_multi_result* out) {
+  entry_clear("fsm_run_multi");
+  if (out) std::memset(out, 0, sizeof(*out));
+  if (npairs == 0) return FSM_OK;
+  if (!fsms || !d_inputs || !lens || !h_final || !h_count) return fail(FSM_EINVAL, "NULL argument");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  std::vector<DevImage> imgs(npairs);
+  std::vector<const uint8_t*> ins(npairs);
+  std::vector<uint32_t> order;
+  order.reserve(npairs);
+  for (uint32_t i = 0; i < npairs; i++) {
+    if (!fsms[i]) return fail(FSM_EINVAL, "NULL handle");
+    if (!d_inputs[i] && lens[i]) return fail(FSM_EINVAL, "NULL input");
+    imgs[i] = fsms[i]->img;
+    ins[i] = d_inputs[i];
+  }
+  // group the pairs by table format: one launch per format present
+  const int modes[5] = {MODE_U8, MODE_U16, MODE_U16H, MODE_U16D, MODE_U32};
+  std::vector<std::pair<int, uint32_t>> groups;  // (mode, count)
+  std::vector<uint32_t> smem_of;
+  for (int m : modes) {
+    uint32_t cnt = 0, sm = 0;
+    for (uint32_t i = 0; i < npairs; i++)
+      if ((int)imgs[i].mode == m) {
+        order.push_back(i);
+        cnt++;
+        sm = std::max(sm, imgs[i].smem_table_bytes + ((m == MODE_U8 || m == MODE_U16D) ? 0u : 256u));  // walk.cuh smem_bytes_for
+      }
+    if (cnt) {
+      groups.push_back({m, cnt});
+      smem_of.push_back(sm);
+    }
+  }
+  // device scratch: [images][inputs][lengths][pair order][finals][counts][stats]
+  static thread_local void* base = nullptr;
+  static thread_local size_t cap = 0;
+  auto al = [](size_t b) { return (b + 255) & ~size_t(255); };
+  const size_t b_img = al(sizeof(DevImage) * npairs), b_in = al(8 * npairs), b_len = al(8 * npairs),
+               b_ord = al(4 * npairs), b_fin = al(4 * npairs), b_cnt = al(8 * npairs), b_st = 256;
+  const size_t need = b_img + b_in + b_len + b_ord + b_fin + b_cnt + b_st;
+  cudaStream_t st = o.st;
+  if (cap < need) {
+    CUDA_TRY(cudaStreamSynchronize(st));
+    if (base) cudaFree(base);
+    base = nullptr;
+    cap = 0;
+    CUDA_TRY(cudaMalloc(&base, need));
+    cap = need;
+  }
+  uint8_t* p = static_cast<uint8_t*>(base);
+  DevImage* d_imgs = reinterpret_cast<DevImage*>(p);
+  const uint8_t** d_ins = reinterpret_cast<const uint8_t**>(p + b_img);
+  uint64_t* d_lens = reinterpret_cast<uint64_t*>(p + b_img + b_in);
+  uint32_t* d_ord = reinterpret_cast<uint32_t*>(p + b_img + b_in + b_len);
+  uint32_t* d_fin = reinterpret_cast<uint32_t*>(p + b_img + b_in + b_len + b_ord);
+  unsigned long long* d_cnt = reinterpret_cast<unsigned long long*>(p + b_img + b_in + b_len + b_ord + b_fin);
+  unsigned long long* d_st = reinterpret_cast<unsigned long long*>(p + b_img + b_in + b_len + b_ord + b_fin + b_cnt);
+  CUDA_TRY(cudaMemcpyAsync(d_imgs, imgs.data(), sizeof(DevImage) * npairs, cudaMemcpyHostToDevice, st));
+  CUDA_TRY(cudaMemcpyAsync(d_ins, ins.data(), 8ull * npairs, cudaMemcpyHostToDevice, st));
+  CUDA_TRY(cudaMemcpyAsync(d_lens, lens, 8ull * npairs, cudaMemcpyHostToDevice, st));
+  CUDA_TRY(cudaMemcpyAsync(d_ord, order.data(), 4ull * npairs, cudaMemcpyHostToDevice, st));
+  CUDA_TRY(cudaMemsetAsync(d_st, 0, 16, st));
+  static thread_local cudaEvent_t ev[2] = {nullptr, nullptr};
+  for (auto& e : ev)
+    if (!e) CUDA_TRY(cudaEventCreate(&e));
+  CUDA_TRY(cudaEventRecord(ev[0], st));
+  uint32_t off = 0;
+  for (size_t g = 0; g < groups.size(); g++) {
+    CUDA_TRY(launch_multi(groups[g].first, d_imgs, d_ins, d_lens, d_ord + off, groups[g].second, smem_of[g], o.B,
+                          d_fin, d_cnt, d_st, st));
+    off += groups[g].second;
+  }
+  CUDA_TRY(cudaEventRecord(ev[1], st));
+  unsigned long long hst[2];
+  CUDA_TRY(cudaMemcpyAsync(h_final, d_fin, 4ull * npairs, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(cudaMemcpyAsync(h_count, d_cnt, 8ull * npairs, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(cudaMemcpyAsync(hst, d_st, 16, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(cudaStreamSynchronize(st));
+  if (out) {
+    out->rewalks = hst[0];
+    out->rounds = hst[1];
+    cudaEventElapsedTime(&out->ms, ev[0], ev[1]);
+  }
+  for (uint32_t i = 0; i < npairs; i++)
+    if (h_final[i] == 0xFFFFFFFFu) return fail(FSM_ESYMBOL, "input symbol >= nsyms in some stream");
+  return FSM_OK;
+}
+
 int fsm_run_literal(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
                     uint32_t* d_chunk_ends, fsm_result* out) {
   entry_clear("fsm_run_literal");

@@ -242,6 +242,10 @@ cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp, const Re
                               cudaStream_t st);
 // Paper-literal SRE: one CTA, one thread per chunk (N <= literal_max_chunks()),
 // Alg. 2 L2-6 + Alg. 3 verbatim; results and stats in *ctl (zeroed by the caller).
+// FSM-level batching: one CTA per (DFA, stream) pair of one table format.
+cudaError_t launch_multi(int mode, const DevImage* d_imgs, const uint8_t* const* d_ins, const uint64_t* d_lens,
+                         const uint32_t* d_pairs, uint32_t npairs, uint32_t smem, uint32_t B, uint32_t* d_fin,
+                         unsigned long long* d_cnt, unsigned long long* d_stats, cudaStream_t st);
 uint32_t literal_max_chunks();
 cudaError_t launch_literal_sre(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl,
                                uint32_t* d_chunk_ends, cudaStream_t st);

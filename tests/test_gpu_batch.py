@@ -121,3 +121,27 @@ def test_batch_empty_and_single(gs):
     r = fsm.run(x, scheme="sre")
     assert int(fin[0]) == r.final_state and int(cnt[0]) == r.accept_count
     assert (ce.cpu() == r.chunk_ends.cpu()).all()
+
+
+def test_fsm_level_batching(gs):
+    """FSM-level batching (Alg. 1 L2-3): many (DFA, stream) pairs of mixed
+    table formats (u8, u16, u16 delta rows) in one call; every pair's final state and
+    accept count equal the oracle's sequential run."""
+    rng = np.random.default_rng(7)
+    specs = [("c1", 0), ("c2", 0), ("c3", 0), ("c4", 0)] + [(f"rand:{int(rng.integers(1, 300))}:"
+                                                             f"{int(rng.integers(1, 257))}:{s}", s) for s in range(10)]
+    fsms, xs, refs = [], [], []
+    for k, (name, seed) in enumerate(specs * 3):
+        length = int(rng.integers(0, 300000))
+        w = gen.workload(name, length=length, seed=seed + k)
+        h = w.host()
+        fsms.append(gs.FSM.load(w.table, w.start, w.accept))
+        xs.append(torch.from_numpy(h).cuda() if length else torch.empty(0, dtype=torch.uint8, device="cuda"))
+        refs.append(oracle.run(w.table, w.start, w.accept, h, 4096))
+    fin, cnt, st = gs.run_multi(fsms, xs, chunk_bytes=4096)
+    for i, ref in enumerate(refs):
+        assert fin[i] == ref["final"] and cnt[i] == ref["count"], (i, specs[i % len(specs)])
+    modes = {f.transform()["mode"] for f in fsms}
+    assert len(modes) >= 2, modes  # several table formats in one call
+    for f in fsms:
+        f.close()
