@@ -48,7 +48,7 @@ def _peaks():
 
 
 class ClockSampler:
-    """SM clocks + throttle reasons sampled DURING the timed region: NVML every 2 ms (a
+    """SM clocks + throttle reasons sampled DURING the timed region: NVML every 0.5 ms (a
     short timed region still gets many samples), nvidia-smi every 100 ms as a fallback."""
 
     REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown", 0x4: "sw_power_cap"}
@@ -99,7 +99,7 @@ class ClockSampler:
                 self.samples.append(self._sample_nvml() if self._nvml else self._sample_smi())
             except Exception:
                 pass
-            self._stop.wait(0.002 if self._nvml else 0.1)
+            self._stop.wait(0.0005 if self._nvml else 0.1)
 
     def __enter__(self):
         self._t = threading.Thread(target=self._run, daemon=True)
