@@ -145,3 +145,20 @@ def test_fsm_level_batching(gs):
     assert len(modes) >= 2, modes  # several table formats in one call
     for f in fsms:
         f.close()
+
+
+def test_fsm_level_batching_invalid_symbol(gs):
+    """A stream with a symbol >= nsyms: its final is 0xFFFFFFFF (R4) and the call raises
+    FSM_ESYMBOL after filling every output; the other pairs are still exact."""
+    t, s_, a = gen.dfa_div7()
+    good = np.array([1, 0, 1, 1] * 5000, np.uint8)
+    bad = good.copy()
+    bad[777] = 5
+    fsm = gs.FSM.load(t, s_, a)
+    xs = [torch.from_numpy(good).cuda(), torch.from_numpy(bad).cuda()]
+    with pytest.raises(gs.GSpecError):
+        gs.run_multi([fsm, fsm], xs)
+    ref = oracle.run(t, s_, a, good, 4096)
+    fin, cnt, _ = gs.run_multi([fsm], xs[:1])
+    assert fin[0] == ref["final"] and cnt[0] == ref["count"]
+    fsm.close()

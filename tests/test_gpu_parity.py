@@ -309,6 +309,11 @@ def test_paper_literal_sre(gs, name, length, B):
             assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
     with pytest.raises(gs.GSpecError):
         fsm.run_literal(torch.zeros(1025 * 16, dtype=torch.uint8, device="cuda"), chunk_bytes=16)
+    if name == "c1" and length > 1000:  # an invalid symbol ends on the poison state (R4)
+        bad = data.copy()
+        bad[length // 2] = 9
+        with pytest.raises(gs.GSpecError):
+            fsm.run_literal(torch.from_numpy(bad).cuda(), chunk_bytes=B)
 
 
 @pytest.mark.parametrize("scheme,B", [("cse", 64), ("cse", 16), ("rr", 64), ("nf", 256)])
