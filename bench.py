@@ -131,8 +131,10 @@ def _max_over_ranks(dist, v: float) -> float:
     return float(t.item())
 
 
-def cpu_baseline(w, budget_s=12.0):
-    """The oracle (plain sequential C, oracle/) on host cores, bounded sample."""
+def cpu_baseline(w, budget_s=12.0, check=None):
+    """The oracle (plain sequential C, oracle/) on host cores, bounded sample.  check
+    (nullable): callable(sample_len) -> the GPU result on the same prefix, compared with
+    the oracle's bit for bit (final state, accept count, every chunk end)."""
     import numpy as np
 
     import oracle
@@ -143,6 +145,13 @@ def cpu_baseline(w, budget_s=12.0):
     r = oracle.run(w.table, w.start, w.accept, data, 4096)
     dt = time.perf_counter() - t0
     assert r["status"] == 0
+    parity = None
+    if check is not None:
+        g = check(sample)
+        ce = g.chunk_ends.cpu().numpy().view(np.uint32)
+        ok = g.final_state == r["final"] and g.accept_count == r["count"] and (ce == r["chunk_end"]).all()
+        parity = {"bit_exact": bool(ok), "sample": f"first {sample >> 20} MiB, same scheme and chunking",
+                  "chunks": int(len(ce))}
     # grow the sample if it was too quick to time well (bounded by budget)
     if dt < 1.0 and sample < w.length:
         reps = max(1, min(int(budget_s / max(dt, 1e-3)), 8))
@@ -150,9 +159,17 @@ def cpu_baseline(w, budget_s=12.0):
         for _ in range(reps):
             oracle.run(w.table, w.start, w.accept, data, 4096)
         dt = (time.perf_counter() - t0) / reps
-    return {"value": round(sample / dt / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-            "sample": f"first {sample >> 20} MiB of the {w.name} stream, oracle.run (Alg. 1), 1 thread",
-            "seconds": round(dt, 3)}
+    out = {"value": round(sample / dt / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+           "sample": f"first {sample >> 20} MiB of the {w.name} stream, oracle.run (Alg. 1), 1 thread",
+           "seconds": round(dt, 3), "host_nproc": os.cpu_count()}
+    try:
+        import platform
+
+        out["cpu_model"] = next((l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo")
+                                 if l.startswith("model name")), platform.processor())
+    except OSError:
+        pass
+    return out, parity
 
 
 def run_reference(args):
@@ -381,10 +398,22 @@ def main():
         "clocks": clk.summary(),
         "e2e": e2e,
     }
+    st0 = kr[-1].stats
+    line["diagnostics"]["runtime_speculation_accuracy"] = round(st0["verify_matches"] / max(1, st0["verify_checks"]), 6)
+    line["diagnostics"]["avg_active_workers"] = round(float(st0.get("avg_active_workers", 0.0)), 2)
+    line["pct_measured_hbm_whole_step"] = round(100 * value / world / peak, 2)
+    try:
+        tr = fsm.transform()
+        line["config"]["table"] = {"format": tr["mode"], "nclasses": int(tr["nclasses"]), "hot_rows": int(tr["hot_rows"])}
+    except Exception:
+        pass
     if feats:
         line["config"]["features"] = {k: round(v, 4) if isinstance(v, float) else v for k, v in feats.items()}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(w)
+        line["cpu_baseline"], parity = cpu_baseline(
+            w, check=lambda n: fsm.run(x[:n], scheme=scheme, chunk_bytes=B))
+        if parity is not None:
+            line["parity"] = parity
     if rank == 0:
         print(json.dumps(line), flush=True)
     if dist:
