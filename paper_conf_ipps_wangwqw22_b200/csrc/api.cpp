@@ -266,10 +266,14 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       pd.active = false;
       return fail(FSM_EUNSUPPORTED, "ENUM needs nstates + 1 <= 32");
     }
-    // sub-chunk size E | B: small enough for parallelism, bounded scratch
-    const uint32_t E = enum_sub_bytes(o.B, len);
+    // sub-chunk size E | B: small enough for parallelism, bounded scratch.  A stream of at
+    // most enum_small_max_sub() sub-chunks of >= 64 B runs as ONE launch (k_enum_small)
+    uint32_t Es = o.B;
+    while (Es % 32 == 0 && Es > 64 && (len + Es / 2 - 1) / (Es / 2) <= enum_small_max_sub()) Es /= 2;
+    const bool small = len > 0 && (len + Es - 1) / Es <= enum_small_max_sub();
+    const uint32_t E = small ? Es : enum_sub_bytes(o.B, len);
     const uint64_t nsub = (len + E - 1) / E;
-    const uint64_t need = enum_scratch_bytes(nsub);
+    const uint64_t need = small ? enum_small_scratch_bytes(nsub) : enum_scratch_bytes(nsub);
     if (f->enum_bytes < need) {
       CUDA_TRY(cudaStreamSynchronize(o.st));  // earlier queued runs may still use the old scratch
       if (f->enum_base) cudaFree(f->enum_base);
@@ -280,12 +284,21 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     }
     rp.ctl_init = f->d_ctl;  // the walk kernel initialises the control block (no H2D copy)
     rp.h_out = &h;           // ... and the output kernel writes it back (pinned, UVA)
+    if (small && !f->enum_ticket) {
+      CUDA_TRY(cudaMalloc(&f->enum_ticket, 256));
+      CUDA_TRY(cudaMemset(f->enum_ticket, 0, 256));
+    }
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
-    CUDA_TRY(launch_enum_full(f->img, rp, E, f->enum_base, d_chunk_ends, f->d_ctl, &f->d_ctl->xfin, o.st,
-                              f->sm_count));
-    uint32_t L = 1;  // map levels: walk + L group scans + L descents + outputs
-    for (uint64_t c = nsub; c > 64 && L < 16; c = (c + 63) / 64) L++;
-    pd.launches = 2 + 2 * L;
+    if (small) {
+      CUDA_TRY(launch_enum_small(f->img, rp, E, f->enum_base, f->enum_ticket, d_chunk_ends, f->d_ctl, o.st));
+      pd.launches = 1;
+    } else {
+      CUDA_TRY(launch_enum_full(f->img, rp, E, f->enum_base, d_chunk_ends, f->d_ctl, &f->d_ctl->xfin, o.st,
+                                f->sm_count));
+      uint32_t L = 1;  // map levels: walk + L group scans + L descents + outputs
+      for (uint64_t c = nsub; c > 64 && L < 16; c = (c + 63) / 64) L++;
+      pd.launches = 2 + 2 * L;
+    }
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   } else {
@@ -717,6 +730,7 @@ void fsm_free(fsm_t f) {
       if (e) cudaEventDestroy(e);
   if (f->d_block_tmp) cudaFree(f->d_block_tmp);
   if (f->enum_base) cudaFree(f->enum_base);
+  if (f->enum_ticket) cudaFree(f->enum_ticket);
   if (f->feat_base) cudaFree(f->feat_base);
   if (f->h_dev_in) cudaFree(f->h_dev_in);
   if (f->h_dev_ce) cudaFree(f->h_dev_ce);

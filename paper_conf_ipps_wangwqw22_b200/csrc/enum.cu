@@ -175,7 +175,179 @@ cudaError_t walk_m(const DevImage& img, const RunParams& rp, uint32_t E, uint64_
   return walk_t<MODE, 32>(img, rp, E, nsub, M, Cn, st, sms);
 }
 
+// ---- small streams: the whole enumeration in ONE launch -------------------------
+// K1+K2+descend+outputs fused for nsub <= kSmallCTAs * kSmallT sub-chunks: each CTA walks
+// kSmallT sub-chunks (one per thread, NE chains), one warp scans the CTA's maps in shared
+// memory (lane q holds entry q; a composition is one shuffle), the CTA publishes
+// its aggregate map, and the last CTA to finish (ticket) composes the aggregates from q0,
+// writes every chunk end, the accept count and the control block (zero-copy to the host).
+constexpr int kSmallT = 128;
+constexpr int kSmallCTAs = 64;
+
+template <int MODE, int NE>
+__global__ void __launch_bounds__(kSmallT) k_enum_small(DevImage img, RunParams rp, uint32_t E, uint64_t nsub,
+                                                       uint8_t* __restrict__ P, uint64_t* __restrict__ PC,
+                                                       uint8_t* __restrict__ AM, uint64_t* __restrict__ AC,
+                                                       uint32_t* __restrict__ ticket, uint32_t* __restrict__ chunk_ends,
+                                                       Ctl* ctl) {
+  extern __shared__ __align__(1024) uint8_t smem[];
+  __shared__ uint8_t sM[kSmallT][32];
+  __shared__ unsigned long long sC[kSmallT][32];
+  __shared__ uint8_t s_in[kSmallCTAs];
+  __shared__ uint32_t last;
+  if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, rp.q0t, rp.N);
+  stage_table(img, smem);
+  __syncthreads();
+  using S = Step<MODE>;
+  const uint32_t nt = img.n + 1, t = threadIdx.x;
+  const uint64_t j = (uint64_t)blockIdx.x * kSmallT + t;
+  {  // walk sub-chunk j from every state (ILP = NE chains)
+    uint32_t code[NE], acc[NE];
+#pragma unroll
+    for (int q = 0; q < NE; q++) {
+      code[q] = __ldg(img.tid2code + ((uint32_t)q < nt ? q : 0));
+      acc[q] = 0;
+    }
+    if (j < nsub) {
+      const uint64_t lo = j * E, n = min((uint64_t)E, rp.len - lo);
+      const uint8_t* p = rp.in + lo;
+      const uint4* v = reinterpret_cast<const uint4*>(p);
+      uint64_t i = 0;
+      if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
+        for (uint64_t t16 = 0; t16 < n / 16; t16++) {
+          const uint4 qv = __ldg(v + t16);
+          const uint32_t w[4] = {qv.x, qv.y, qv.z, qv.w};
+#pragma unroll
+          for (int k = 0; k < 4; k++) {
+#pragma unroll
+            for (int q = 0; q < NE; q++) { code[q] = S::template word<0>(img, smem, code[q], w[k]); acc[q] += S::acc(code[q]); }
+#pragma unroll
+            for (int q = 0; q < NE; q++) { code[q] = S::template word<1>(img, smem, code[q], w[k]); acc[q] += S::acc(code[q]); }
+#pragma unroll
+            for (int q = 0; q < NE; q++) { code[q] = S::template word<2>(img, smem, code[q], w[k]); acc[q] += S::acc(code[q]); }
+#pragma unroll
+            for (int q = 0; q < NE; q++) { code[q] = S::template word<3>(img, smem, code[q], w[k]); acc[q] += S::acc(code[q]); }
+          }
+        }
+        i = (n / 16) * 16;
+      }
+      for (; i < n; i++) {
+        const uint32_t bb = __ldg(p + i);
+#pragma unroll
+        for (int q = 0; q < NE; q++) { code[q] = S::byte(img, smem, code[q], bb); acc[q] += S::acc(code[q]); }
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < 32; q++) {
+      const bool real = q < NE && (uint32_t)q < nt && j < nsub;
+      sM[t][q] = (uint8_t)(real ? S::tid(img, code[q < NE ? q : 0]) : q);  // identity past the stream
+      sC[t][q] = real ? acc[q < NE ? q : 0] : 0;
+    }
+  }
+  __syncthreads();
+  const uint64_t G = (nsub + kSmallT - 1) / kSmallT;
+  if (t < 32) {  // in-CTA inclusive prefix: P_i = M_i o ... o M_0 (lane t holds entry t)
+    uint32_t x = t;
+    unsigned long long c = 0;
+    for (int i = 0; i < kSmallT; i++) {
+      const uint32_t y = __shfl_sync(0xffffffffu, (uint32_t)sM[i][t], x);
+      c += __shfl_sync(0xffffffffu, sC[i][t], x);
+      x = y;
+      const uint64_t ji = (uint64_t)blockIdx.x * kSmallT + i;
+      if (ji < nsub) {
+        P[ji * 32 + t] = (uint8_t)x;
+        PC[ji * 32 + t] = c;
+      }
+    }
+    AM[blockIdx.x * 32 + t] = (uint8_t)x;
+    AC[blockIdx.x * 32 + t] = c;
+  }
+  __threadfence();
+  __syncthreads();
+  if (t == 0) last = atomicAdd(ticket, 1u) == G - 1;
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  if (t < 32) {  // compose the CTA aggregates from q0: incoming state of every CTA
+    uint32_t s = rp.q0t;
+    unsigned long long total = 0;
+    for (uint64_t g = 0; g < G; g++) {
+      if (t == 0) s_in[g] = (uint8_t)s;
+      total += __ldcg(reinterpret_cast<const unsigned long long*>(AC) + g * 32 + s);
+      s = __ldcg(AM + g * 32 + s);
+    }
+    if (t == 0) {
+      ctl->accept_count = total;
+      ctl->xfin = s;
+      *ticket = 0;  // re-armed for the next run
+    }
+  }
+  __syncthreads();
+  const uint32_t per = rp.B / E;  // sub-chunks per chunk
+  for (uint64_t c = t; c < rp.N; c += kSmallT) {
+    const uint64_t jl = min((c + 1) * per, nsub) - 1;
+    const uint32_t sin = s_in[jl / kSmallT];
+    if (chunk_ends) chunk_ends[c] = __ldg(img.inv + __ldcg(P + jl * 32 + sin));
+  }
+  __syncthreads();
+  if (t == 0 && rp.h_out) {
+    __threadfence();
+    ctl->finished = 1;
+    const uint32_t* src = reinterpret_cast<const uint32_t*>(ctl);
+    uint32_t* dst = reinterpret_cast<uint32_t*>(rp.h_out);
+    for (uint32_t i = 0; i < sizeof(Ctl) / 4; i++) dst[i] = __ldcg(src + i);
+  }
+}
+
+template <int MODE, int NE>
+cudaError_t small_t(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, void* scratch,
+                    uint32_t* ticket, uint32_t* chunk_ends, Ctl* ctl, cudaStream_t st) {
+  auto kern = k_enum_small<MODE, NE>;
+  const uint32_t smem = smem_bytes_for(img);
+  cudaError_t e = kernel_setup((const void*)kern, smem, kSmallT, nullptr);
+  if (e != cudaSuccess) return e;
+  uint8_t* p = reinterpret_cast<uint8_t*>(scratch);
+  auto take = [&](uint64_t bytes) { uint8_t* r = p; p += (bytes + 255) & ~255ull; return r; };
+  uint8_t* P = take(nsub * 32);
+  uint64_t* PC = reinterpret_cast<uint64_t*>(take(nsub * 32 * 8));
+  uint8_t* AM = take(kSmallCTAs * 32);
+  uint64_t* AC = reinterpret_cast<uint64_t*>(take(kSmallCTAs * 32 * 8));
+  const uint64_t G = (nsub + kSmallT - 1) / kSmallT;
+  kern<<<(unsigned)G, kSmallT, smem, st>>>(img, rp, E, nsub, P, PC, AM, AC, ticket, chunk_ends, ctl);
+  return cudaGetLastError();
+}
+
+template <int MODE>
+cudaError_t small_m(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, void* scratch,
+                    uint32_t* ticket, uint32_t* chunk_ends, Ctl* ctl, cudaStream_t st) {
+  const uint32_t nt = img.n + 1;
+  if (nt <= 8) return small_t<MODE, 8>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
+  if (nt <= 16) return small_t<MODE, 16>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
+  return small_t<MODE, 32>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
+}
+
 }  // namespace
+
+uint64_t enum_small_max_sub() { return (uint64_t)kSmallCTAs * kSmallT; }
+
+uint64_t enum_small_scratch_bytes(uint64_t nsub) {
+  auto r = [](uint64_t b) { return (b + 255) & ~255ull; };
+  return r(nsub * 32) + r(nsub * 32 * 8) + r(kSmallCTAs * 32) + r(kSmallCTAs * 32 * 8);
+}
+
+// `ticket` (device u32, zero before the first launch) counts finished CTAs; the last CTA
+// re-arms it, so runs queued back to back on one stream reuse it.
+cudaError_t launch_enum_small(const DevImage& img, const RunParams& rp, uint32_t E, void* scratch, uint32_t* ticket,
+                              uint32_t* d_chunk_ends, Ctl* d_ctl, cudaStream_t st) {
+  const uint64_t nsub = (rp.len + E - 1) / E;
+  switch (img.mode) {
+    case MODE_U8: return small_m<MODE_U8>(img, rp, E, nsub, scratch, ticket, d_chunk_ends, d_ctl, st);
+    case MODE_U16: return small_m<MODE_U16>(img, rp, E, nsub, scratch, ticket, d_chunk_ends, d_ctl, st);
+    case MODE_U16H: return small_m<MODE_U16H>(img, rp, E, nsub, scratch, ticket, d_chunk_ends, d_ctl, st);
+    case MODE_U16D: return small_m<MODE_U16D>(img, rp, E, nsub, scratch, ticket, d_chunk_ends, d_ctl, st);
+    default: return small_m<MODE_U32>(img, rp, E, nsub, scratch, ticket, d_chunk_ends, d_ctl, st);
+  }
+}
 
 // Scratch layout for the enumeration (levels of maps + per-level states).
 uint64_t enum_scratch_bytes(uint64_t nsub) {

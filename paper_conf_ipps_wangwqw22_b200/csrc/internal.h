@@ -253,6 +253,11 @@ bool spec_path_generic_only();  // GSPEC_SPEC_PATH=generic forces the non-TMA ke
 cudaError_t launch_verify_recover(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* d_ctl,
                                   uint64_t* d_block_tmp, uint32_t* d_chunk_ends, cudaStream_t st, int sm_count);
 uint64_t enum_scratch_bytes(uint64_t nsub);
+// ENUM of a small stream (nsub <= enum_small_max_sub() sub-chunks) in ONE launch
+uint64_t enum_small_max_sub();
+uint64_t enum_small_scratch_bytes(uint64_t nsub);
+cudaError_t launch_enum_small(const DevImage& img, const RunParams& rp, uint32_t E, void* scratch, uint32_t* ticket,
+                              uint32_t* d_chunk_ends, Ctl* d_ctl, cudaStream_t st);
 cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t E, void* scratch,
                              uint32_t* d_chunk_ends, Ctl* d_ctl, uint32_t* d_x_final, cudaStream_t st, int sms,
                              int phases = 3, const uint8_t** top_M = nullptr, const uint64_t** top_C = nullptr);
@@ -343,6 +348,7 @@ struct fsm_s {
   double acc1_hint = 0.0;            // spec-1 accuracy from the selector's profile (dense-round gate)
   uint32_t dense_hint = 4;           // task-kernel slots queued per dense run (dense rounds last seen)
   bool shard_prefer_exact = false;   // a speculative shard map was invalid once: use the exact map
+  uint32_t* enum_ticket = nullptr;   // single-launch ENUM: finished-CTA counter (zeroed once)
   bool auto_selected = false;
   const uint32_t* d_ttc = nullptr;   // [nt][C] transformed tid x class table (prep/features)
   uint32_t* d_small = nullptr;       // small device scratch (ENUM final state, shard compose)
