@@ -140,14 +140,17 @@ __global__ void k_enum_out(DevImage img, const uint32_t* __restrict__ st0, const
     const uint32_t s = jn < nsub ? st0[jn] : fin;
     if (chunk_ends) chunk_ends[c] = img.inv[s];
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    *x_final = fin;
-    ctl->accept_count = PC0top[top_last * 32 + q0t];
-    if (h_out) {  // zero-copy result: publish the control block to the run's pinned host slot
+  if (blockIdx.x == 0) {
+    if (threadIdx.x == 0) {
+      *x_final = fin;
+      ctl->accept_count = PC0top[top_last * 32 + q0t];
       __threadfence();
+    }
+    __syncthreads();
+    if (h_out) {  // zero-copy result: the block publishes the control block to the pinned host slot
       const uint32_t* src = reinterpret_cast<const uint32_t*>(ctl);
       uint32_t* dst = reinterpret_cast<uint32_t*>(h_out);
-      for (uint32_t i = 0; i < sizeof(Ctl) / 4; i++) dst[i] = __ldcg(src + i);
+      for (uint32_t i = threadIdx.x; i < sizeof(Ctl) / 4; i += blockDim.x) dst[i] = __ldcg(src + i);
     }
   }
 }
@@ -268,13 +271,20 @@ __global__ void __launch_bounds__(kSmallT) k_enum_small(DevImage img, RunParams 
   __syncthreads();
   if (!last) return;
   __threadfence();
+  // the CTA aggregates into shared memory first (independent loads), then the dependent
+  // composition chain runs on shared memory instead of G dependent L2 round trips
+  for (uint32_t i = t; i < G * 32; i += kSmallT) {
+    sM[i / 32][i % 32] = __ldcg(AM + i);
+    sC[i / 32][i % 32] = __ldcg(reinterpret_cast<const unsigned long long*>(AC) + i);
+  }
+  __syncthreads();
   if (t < 32) {  // compose the CTA aggregates from q0: incoming state of every CTA
     uint32_t s = rp.q0t;
     unsigned long long total = 0;
     for (uint64_t g = 0; g < G; g++) {
       if (t == 0) s_in[g] = (uint8_t)s;
-      total += __ldcg(reinterpret_cast<const unsigned long long*>(AC) + g * 32 + s);
-      s = __ldcg(AM + g * 32 + s);
+      total += sC[g][s];
+      s = sM[g][s];
     }
     if (t == 0) {
       ctl->accept_count = total;
@@ -289,13 +299,13 @@ __global__ void __launch_bounds__(kSmallT) k_enum_small(DevImage img, RunParams 
     const uint32_t sin = s_in[jl / kSmallT];
     if (chunk_ends) chunk_ends[c] = __ldg(img.inv + __ldcg(P + jl * 32 + sin));
   }
+  if (t == 0) ctl->finished = 1;
+  __threadfence();
   __syncthreads();
-  if (t == 0 && rp.h_out) {
-    __threadfence();
-    ctl->finished = 1;
+  if (rp.h_out) {  // zero-copy result, copied by the whole CTA (one thread would serialise ~130 L2 loads)
     const uint32_t* src = reinterpret_cast<const uint32_t*>(ctl);
     uint32_t* dst = reinterpret_cast<uint32_t*>(rp.h_out);
-    for (uint32_t i = 0; i < sizeof(Ctl) / 4; i++) dst[i] = __ldcg(src + i);
+    for (uint32_t i = t; i < sizeof(Ctl) / 4; i += kSmallT) dst[i] = __ldcg(src + i);
   }
 }
 
