@@ -194,8 +194,8 @@ __global__ void __launch_bounds__(kSmallT) k_enum_small(DevImage img, RunParams 
                                                        uint32_t* __restrict__ ticket, uint32_t* __restrict__ chunk_ends,
                                                        Ctl* ctl) {
   extern __shared__ __align__(1024) uint8_t smem[];
-  __shared__ uint8_t sM[kSmallT][32];
-  __shared__ unsigned long long sC[kSmallT][32];
+  __shared__ uint8_t sM[kSmallT][33];  // +1 pad: a thread's 32 writes of its own map hit
+  __shared__ unsigned long long sC[kSmallT][33];  // different banks from its neighbours' writes
   __shared__ uint8_t s_in[kSmallCTAs];
   __shared__ uint32_t last;
   if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, rp.q0t, rp.N);
