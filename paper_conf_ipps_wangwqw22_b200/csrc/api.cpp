@@ -270,7 +270,9 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     // most enum_small_max_sub() sub-chunks of >= 64 B runs as ONE launch (k_enum_small)
     uint32_t Es = o.B;
     while (Es % 32 == 0 && Es > 64 && (len + Es / 2 - 1) / (Es / 2) <= enum_small_max_sub()) Es /= 2;
-    const bool small = len > 0 && (len + Es - 1) / Es <= enum_small_max_sub();
+    // (only for short sub-chunks: 8192 threads walking long sub-chunks would be latency-bound;
+    // longer streams keep the multi-level scan with many more threads)
+    const bool small = len > 0 && Es <= 256 && (len + Es - 1) / Es <= enum_small_max_sub();
     const uint32_t E = small ? Es : enum_sub_bytes(o.B, len);
     const uint64_t nsub = (len + E - 1) / E;
     const uint64_t need = small ? enum_small_scratch_bytes(nsub) : enum_scratch_bytes(nsub);
