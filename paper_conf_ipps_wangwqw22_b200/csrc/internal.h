@@ -46,6 +46,7 @@ struct DevImage {
   const uint16_t* T16;        // MODE_U16: [nt][C]
   const uint32_t* T32;        // MODE_U32: [nt][C]
   const uint8_t* cls;         // [256] byte -> class
+  const uint8_t* cls2;        // MODE_U16H: [256] byte -> 2*class (staged instead of cls)
   const uint32_t* qs2;        // [C*C][kQsMax] ranked lookback candidates (tids)
   const uint8_t* qs2_len;     // [C*C]
   const uint32_t* qs2_img;    // [C*C] image size

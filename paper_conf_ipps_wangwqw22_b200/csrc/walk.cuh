@@ -37,7 +37,7 @@ __device__ __forceinline__ void stage_table(const DevImage& img, uint8_t* smem) 
   const uint32_t nv = img.smem_table_bytes / 16;
   for (uint32_t i = threadIdx.x; i < nv; i += blockDim.x) dst[i] = __ldg(src + i);
   if (img.mode != MODE_U8) {
-    const uint4* cs = reinterpret_cast<const uint4*>(img.cls);
+    const uint4* cs = reinterpret_cast<const uint4*>(img.mode == MODE_U16H ? img.cls2 : img.cls);
     uint4* cd = reinterpret_cast<uint4*>(smem);
     for (uint32_t i = threadIdx.x; i < 16; i += blockDim.x) cd[i] = __ldg(cs + i);
   }
@@ -179,8 +179,31 @@ template <>
 struct Step<MODE_U16> : StepClassed<uint16_t, 15, false> {};
 template <>
 struct Step<MODE_U16D> : StepDelta {};
+// MODE_U16H: every row in shared memory, pre-multiplied codes (code & 0x7FFF = t*C, the
+// row's entry index; accept flag in bit 15) and a doubled class map, so the entry address
+// is (c << 1) + (base + 256 + 2*class): LOP3 + LEA on the dependent chain.
+struct StepPM {
+  static constexpr uint32_t kShift = 15;
+  static __device__ __forceinline__ uint32_t row(uint32_t base, uint32_t code, uint32_t cl2) {
+    return lds_u16(((code & 0x7FFFu) << 1) + (base + 256 + cl2));
+  }
+  static __device__ __forceinline__ uint32_t byte(const DevImage&, const uint8_t* s, uint32_t code, uint32_t b) {
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
+    return row(base, code, lds_u8(base + b));
+  }
+  template <int K>
+  static __device__ __forceinline__ uint32_t word(const DevImage&, const uint8_t* s, uint32_t code, uint32_t w) {
+    const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
+    return row(base, code, lds_u8(byte_plus<K>(w, base)));  // class map at the 256-aligned base
+  }
+  static __device__ __forceinline__ uint32_t acc(uint32_t code) { return code >> 15; }
+  static __device__ __forceinline__ uint32_t tid(const DevImage& img, uint32_t code) {
+    return __ldg(img.code2tid + (code & 0x7FFFu));
+  }
+};
+
 template <>
-struct Step<MODE_U16H> : StepClassed<uint16_t, 15, true> {};
+struct Step<MODE_U16H> : StepPM {};
 template <>
 struct Step<MODE_U32> : StepClassed<uint32_t, 31, false> {};
 
