@@ -218,9 +218,20 @@ __global__ void k_map_enum(const uint8_t* __restrict__ topM, const unsigned long
   if (s < nt) { mend[s] = topM[s]; mcnt[s] = topC[s]; }
 }
 
-// s_0 = q0; s_{h+1} = M_h[s_h]: out = {s_rank, final, err, count_lo, count_hi}
-__global__ void k_compose(const uint8_t* __restrict__ maps, uint32_t G, uint64_t map_bytes, uint64_t cnt_off,
-                          uint32_t q0t, uint32_t rank, uint32_t* __restrict__ out) {
+// s_0 = q0; s_{h+1} = M_h[s_h]: out = {s_rank, final, err, count_lo, count_hi}.  With
+// `staged` the G maps are first copied into shared memory by the whole block (coalesced),
+// so the dependent chain of G lookups runs on shared memory instead of G L2 round trips.
+__global__ void k_compose(const uint8_t* __restrict__ maps_g, uint32_t G, uint64_t map_bytes, uint64_t cnt_off,
+                          uint32_t q0t, uint32_t rank, uint32_t* __restrict__ out, uint32_t staged) {
+  extern __shared__ __align__(16) uint8_t sm_maps[];
+  const uint8_t* maps = maps_g;
+  if (staged) {
+    const uint64_t words = G * map_bytes / 4;
+    for (uint64_t i = threadIdx.x; i < words; i += blockDim.x)
+      reinterpret_cast<uint32_t*>(sm_maps)[i] = __ldcg(reinterpret_cast<const uint32_t*>(maps_g) + i);
+    __syncthreads();
+    maps = sm_maps;
+  }
   if (threadIdx.x || blockIdx.x) return;
   uint32_t s = q0t, srank = q0t, err = 0;
   unsigned long long c = 0;
@@ -339,7 +350,13 @@ cudaError_t launch_map_enum(const uint8_t* topM, const unsigned long long* topC,
 
 cudaError_t launch_compose(const uint8_t* maps, uint32_t G, uint64_t map_bytes, uint64_t cnt_off, uint32_t q0t,
                            uint32_t rank, uint32_t* out, cudaStream_t st) {
-  k_compose<<<1, 32, 0, st>>>(maps, G, map_bytes, cnt_off, q0t, rank, out);
+  const uint64_t bytes = (uint64_t)G * map_bytes;
+  uint32_t staged = bytes <= 96 * 1024 && map_bytes % 8 == 0;
+  if (staged && kernel_setup((const void*)k_compose, (uint32_t)bytes, 256, nullptr) != cudaSuccess) staged = 0;
+  if (staged)
+    k_compose<<<1, 256, (uint32_t)bytes, st>>>(maps, G, map_bytes, cnt_off, q0t, rank, out, 1u);
+  else
+    k_compose<<<1, 32, 0, st>>>(maps, G, map_bytes, cnt_off, q0t, rank, out, 0u);
   return cudaGetLastError();
 }
 
