@@ -674,13 +674,13 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
     img.H = (uint32_t)H;
     img.smem_table_bytes = (uint32_t)(((H * C * esz) + 15) & ~15ull);
     if (mode == MODE_U16 && H == nt && (uint64_t)nt * C <= 0x7FFFu && C < 128) {
-      // every row hot: no hot test, and pre-multiplied codes (code = t*C = the row's entry
-      // index, accept flag in bit 15; the staged class map holds 2*class), so a step is
-      // LOP3 + LEA on the dependent chain instead of LOP3 + IMAD + IADD3
+      // every row hot: no hot test, and pre-multiplied codes (code = 2*t*C = the row's byte
+      // offset, accept flag in bit 0; the staged class map holds 2*class), so a step is
+      // LOP3 + IADD3 on the dependent chain instead of LOP3 + IMAD + IADD3
       img.mode = MODE_U16H;
       code2tid.assign(0x8000, P);
       for (uint32_t t = 0; t < nt; t++) {
-        tid2code[t] = t * C | ((uint32_t)acc_t[t] << 15);
+        tid2code[t] = 2 * t * C | (uint32_t)acc_t[t];  // row byte offset | accept flag (bit 0)
         code2tid[t * C] = t;
       }
       std::vector<uint8_t> cls2(256);

@@ -179,13 +179,13 @@ template <>
 struct Step<MODE_U16> : StepClassed<uint16_t, 15, false> {};
 template <>
 struct Step<MODE_U16D> : StepDelta {};
-// MODE_U16H: every row in shared memory, pre-multiplied codes (code & 0x7FFF = t*C, the
-// row's entry index; accept flag in bit 15) and a doubled class map, so the entry address
-// is (c << 1) + (base + 256 + 2*class): LOP3 + LEA on the dependent chain.
+// MODE_U16H: every row in shared memory, pre-multiplied codes (code = 2*t*C | accept: the
+// row's byte offset with the accept flag in bit 0) and a doubled class map, so the entry
+// address is code - (code & 1) + (base + 256 + 2*class): LOP3 + IADD3 on the dependent chain.
 struct StepPM {
-  static constexpr uint32_t kShift = 15;
+  static constexpr uint32_t kShift = 0;
   static __device__ __forceinline__ uint32_t row(uint32_t base, uint32_t code, uint32_t cl2) {
-    return lds_u16(((code & 0x7FFFu) << 1) + (base + 256 + cl2));
+    return lds_u16(code - (code & 1u) + (base + 256 + cl2));
   }
   static __device__ __forceinline__ uint32_t byte(const DevImage&, const uint8_t* s, uint32_t code, uint32_t b) {
     const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
@@ -196,9 +196,9 @@ struct StepPM {
     const uint32_t base = static_cast<uint32_t>(__cvta_generic_to_shared(s));
     return row(base, code, lds_u8(byte_plus<K>(w, base)));  // class map at the 256-aligned base
   }
-  static __device__ __forceinline__ uint32_t acc(uint32_t code) { return code >> 15; }
+  static __device__ __forceinline__ uint32_t acc(uint32_t code) { return code & 1u; }
   static __device__ __forceinline__ uint32_t tid(const DevImage& img, uint32_t code) {
-    return __ldg(img.code2tid + (code & 0x7FFFu));
+    return __ldg(img.code2tid + (code >> 1));
   }
 };
 
