@@ -91,6 +91,40 @@ def run(table, start, accept, data, B=4096):
             "chunk_end": ce[:nchunks(d.size, B)]}
 
 
+def run_stream(table, start, accept, fill, length, B=4096, block=64 << 20, prefetch=2):
+    """Alg. 1 FSM_PROCESSING over a stream too large for one host buffer
+    (16 GiB in 64 MiB blocks).  Alg. 1 is a left fold over the input,
+    so the walk is or_run block after block, each block starting from the previous
+    block's final state; block is a multiple of B, so every chunk lies in one block.
+    fill(offset, n) -> uint8 array of the stream's bytes [offset, offset + n), e.g. the
+    host generator; the next `prefetch` blocks are generated in background threads.
+    Returns the same dict as run()."""
+    import concurrent.futures
+
+    assert block % B == 0
+    t = _c(table, np.uint32)
+    a = _c(accept, np.uint8)
+    n, ns = t.shape
+    ce = np.zeros(max(1, nchunks(length, B)), np.uint32)
+    s, total = int(start), 0
+    offs = list(range(0, length, block))
+    with concurrent.futures.ThreadPoolExecutor(max(1, prefetch)) as ex:
+        futs = {}
+        for i, off in enumerate(offs):
+            for j in range(i, min(len(offs), i + prefetch + 1)):
+                if j not in futs:
+                    futs[j] = ex.submit(fill, offs[j], min(block, length - offs[j]))
+            d = _c(futs.pop(i).result(), np.uint8)
+            fin, cnt = U32(0), U64(0)
+            rc = lib().or_run(t.ctypes.data, n, ns, s, a.ctypes.data, d.ctypes.data, d.size, B,
+                              ce[off // B:].ctypes.data, ctypes.byref(fin), ctypes.byref(cnt))
+            if rc != OR_OK:
+                return {"status": rc}
+            s = int(fin.value)
+            total += int(cnt.value)
+    return {"status": 0, "final": s, "accept": int(a[s]), "count": total, "chunk_end": ce[:nchunks(length, B)]}
+
+
 def transform(table, accept, policy=0, profile=None, start=0):
     """Frequency-based transformation. Returns (perm[n+1], inv[n+1], freq[n], tt[n+1,ns], acc_t[n+1])."""
     t = _c(table, np.uint32)

@@ -392,3 +392,76 @@ def test_c4_auto_picks_delta_rows(gs):
     w, _ = _wl("c4", 1 << 16)
     tr = gs.FSM.load(w.table, w.start, w.accept).transform()
     assert tr["mode"] == "u16d" and tr["hot_rows"] < 2048
+
+
+def _perm_dfa(n, nsyms, seed):
+    """Permutation DFA (every column a permutation): no convergence, uniq10 = n."""
+    rng = np.random.default_rng(seed)
+    t = np.stack([rng.permutation(n) for _ in range(nsyms)], axis=1).astype(np.uint32)
+    a = (rng.random(n) < 0.5).astype(np.uint8)
+    return t, 0, a
+
+
+@pytest.mark.parametrize("n", [31, 32])
+def test_selector_enum_bound(gs, n):
+    """R19's ENUM leaf: n <= 31.  The GPU selector and the oracle pick the same scheme
+    on permutation DFAs of 31 and 32 states, and the picked scheme is exact."""
+    t, s, a = _perm_dfa(n, 3, n)
+    rng = np.random.default_rng(n)
+    data = rng.integers(0, 3, 1 << 18).astype(np.uint8)
+    fsm = gs.FSM.load(t, s, a)
+    x = torch.from_numpy(data).cuda()
+    pick, ft = fsm.select_scheme(x)
+    of = oracle.features(t, s, a, data, B=4096)
+    assert ft["uniq10"] == pytest.approx(of["uniq10"]) == n
+    assert ft["acc1"] == pytest.approx(of["acc1"]) and ft["acck"] == pytest.approx(of["acck"])
+    assert ft["input_sensitivity"] == pytest.approx(of["sens"])
+    assert oracle.select(of, n) == gs.SCHEMES[pick]
+    assert pick == ("enum" if n == 31 else "sre")
+    ref = oracle.run(t, s, a, data, 4096)
+    check_equal(fsm.run(x, scheme="auto"), ref, 4096, n)
+
+
+def test_selector_features_input_sensitive(gs):
+    """GPU features equal the oracle's on inputs whose segments provably differ: the
+    designed div7 stream of test_oracle_pins (sens > 0.5) and a C3s slice across a
+    region boundary (normal / vowel-free halves)."""
+    import test_oracle_pins as pins
+
+    w = gen.workload("c1")
+    rng = np.random.default_rng(7)
+    B, m = 16, 8
+    N = 8 * m + 1
+    res = [0] * (N + 1)
+    for c in range(1, N):
+        res[c] = 0 if (c - 1) // m in (0, 2, 4) and rng.random() < 0.9 else int(rng.integers(1, 7))
+    bits = pins._div7_designed_bits(res, B, rng)
+    cases = [(w, bits, B)]
+    w3 = gen.workload("c3s")
+    cases.append((w3, w3.host((1 << 26) - 33 * 4096, 65 * 4096), 4096))
+    for wl, data, BB in cases:
+        fsm = gs.FSM.load(wl.table, wl.start, wl.accept)
+        pick, ft = fsm.select_scheme(torch.from_numpy(data).cuda(), chunk_bytes=BB)
+        of = oracle.features(wl.table, wl.start, wl.accept, data, B=BB)
+        assert of["sens"] >= 0.2
+        assert ft["acc1"] == pytest.approx(of["acc1"]) and ft["acck"] == pytest.approx(of["acck"])
+        assert ft["input_sensitivity"] == pytest.approx(of["sens"])
+        assert ft["uniq10"] == pytest.approx(of["uniq10"])
+        assert gs.SCHEMES[pick] == oracle.select(of, wl.nstates)
+
+
+@pytest.mark.parametrize("vr_others", [1, 2, 4])
+@pytest.mark.parametrize("scheme", ["rr", "nf"])
+def test_vr_others_capacity(gs, vr_others, scheme):
+    """Helper records go to VR^others; with 1/2/4 slots the FIFO eviction
+    (R16) runs on the GPU: results exact, round diagnostics equal the oracle's."""
+    w, data = _wl("c3", 4 << 20)
+    ref = oracle.run(w.table, w.start, w.accept, data, 4096)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    res = fsm.run(torch.from_numpy(data).cuda(), scheme=scheme, vr_others=vr_others)
+    check_equal(res, ref, 4096, w.nstates)
+    sim = oracle.simulate(w.table, w.start, w.accept, data, 4096, scheme=scheme, vr_oth=vr_others)
+    for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks",
+              "verify_matches"):
+        assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+    assert res.stats["tasks_helper"] > 0

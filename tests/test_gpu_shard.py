@@ -88,48 +88,6 @@ def test_single_rank_nccl_group(gs):
         dist.destroy_process_group()
 
 
-def test_c5_16gib_shard_invariance(gs):
-    """C5: a 16 GiB stream sharded 8 ways (fake collective, one GPU) gives exactly the
-    single-GPU result (G-invariance), and the single-GPU result matches the oracle on
-    its first 1 GiB prefix (chunk ends are prefix states)."""
-    import ctypes
-
-    from paper_conf_ipps_wangwqw22_b200 import _check, _lib, _run_opts, fsm_result
-    from paper_conf_ipps_wangwqw22_b200.dist import shard_bounds
-
-    L = 16 << 30
-    w = gen.workload("c2", length=L)
-    x = torch.empty(L, dtype=torch.uint8, device="cuda")
-    w.device(x)
-    fsm = gs.FSM.load(w.table, w.start, w.accept)
-    single = fsm.run(x, scheme="sre")
-    ce_single = single.chunk_ends.cpu().numpy().view(np.uint32)
-    G = 8
-    fsms = [gs.FSM.load(w.table, w.start, w.accept) for _ in range(G)]
-    mb = fsms[0].map_bytes()
-    maps = torch.zeros(G * mb, dtype=torch.uint8, device="cuda")
-    o = _run_opts("sre", 4096)
-    ces = []
-    for g in range(G):
-        lo, hi = shard_bounds(L, G, g)
-        n = gs.fsm_num_chunks(hi - lo)
-        ce = torch.empty(n, dtype=torch.int32, device="cuda")
-        lb = x[lo - 2:lo] if g else None
-        _check(_lib.fsm_shard_map(fsms[g].handle, x[lo:].data_ptr(), hi - lo, lb.data_ptr() if g else None,
-                                  2 if g else 0, ctypes.byref(o), maps[g * mb:].data_ptr(), ce.data_ptr()), "map")
-        ces.append(ce)
-    for g in range(G):
-        r = fsm_result()
-        _check(_lib.fsm_shard_finish(fsms[g].handle, maps.data_ptr(), G, g, ctypes.byref(o), ces[g].data_ptr(),
-                                     ctypes.byref(r)), "finish")
-        assert r.final_state == single.final_state and r.accept_count == single.accept_count
-    ce_sharded = np.concatenate([c.cpu().numpy().view(np.uint32) for c in ces])
-    assert (ce_sharded == ce_single).all()
-    h = w.host(0, 1 << 30)
-    ref = oracle.run(w.table, w.start, w.accept, h, 4096)
-    assert (ce_single[:len(ref["chunk_end"])] == ref["chunk_end"]).all()
-
-
 def test_library_nccl_single_rank(gs):
     """fsm_comm_init + fsm_run_sharded with a real (1-rank) NCCL communicator."""
     w = gen.workload("c2", length=8 << 20)

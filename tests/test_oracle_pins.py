@@ -472,3 +472,115 @@ def test_features_accuracy_bruteforce():
         hitk += int(truth in list(qs[:4]))
     f = oracle.features(t, s, a, data, B=B)
     assert f["acc1"] == pytest.approx(hit1 / (N - 1)) and f["acck"] == pytest.approx(hitk / (N - 1))
+
+
+# ------------------------------------------------ input sensitivity (sens) --
+def _div7_designed_bits(residues, B, rng):
+    """Bits of a div7 stream whose prefix value at every chunk boundary c*B (c >= 1)
+    is residues[c] mod 7: the first B-3 bits of a chunk are random, its last 3 bits
+    are chosen so that value(prefix) = 8*v + b = v + b (mod 7) hits the target."""
+    N = len(residues) - 1  # residues[0..N]: entry c is the target at boundary c*B
+    bits = np.zeros(N * B, np.uint8)
+    v = 0
+    for c in range(N):
+        body = rng.integers(0, 2, B - 3)
+        for b in body:
+            v = (2 * v + int(b)) % 7
+        bits[c * B:c * B + B - 3] = body
+        target = residues[c + 1] if c + 1 < N else int(rng.integers(0, 7))
+        last = (target - v) % 7  # 0..6 < 8: three bits
+        bits[c * B + B - 3:c * B + B] = [(last >> 2) & 1, (last >> 1) & 1, last & 1]
+        v = (v + last) % 7
+    return bits
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2, 3])
+def test_features_sens_div7_designed(seed):
+    """Input sensitivity pinned by construction (R19: max - min of the per-segment
+    spec-1 accuracy over 8 equal segments of the profile chunks c >= 1).
+
+    div7's lookback-2 image is every state at multiplicity 1 (a bijection), its static
+    in-degrees all equal 2 so the transformation is the identity, hence QS = [0..6] and
+    spec-1 hits chunk c iff the big-integer value of the prefix before it is = 0 (mod 7),
+    spec-4 iff it is < 4.  The residues are drawn here, per segment, so the expected
+    acc1 / acc4 / sens come from the design, not from the oracle."""
+    rng = np.random.default_rng(seed)
+    B, m = 16, 6 + seed          # N - 1 = 8m profile chunks: 8 equal segments of m chunks
+    N = 8 * m + 1
+    p_hit = np.roll([0.8, 0.2, 0.7, 0.3, 0.9, 0.1, 0.6, 0.4], seed)  # high / low alternate
+    res = [0] * (N + 1)
+    for c in range(1, N):
+        seg = (c - 1) // m
+        res[c] = 0 if rng.random() < p_hit[seg] else int(rng.integers(1, 7))
+    # segment edges carry the opposite outcome of their neighbour's majority so that a
+    # segment formula off by one chunk changes some segment's accuracy
+    for j in range(8):
+        first, last = 1 + j * m, (j + 1) * m
+        res[first] = 0 if p_hit[j] >= 0.5 else 3
+        res[last] = 0 if p_hit[j] >= 0.5 else 5
+    bits = _div7_designed_bits(res, B, rng)
+    # the construction really produces those residues (Python big integers)
+    for c in range(1, N):
+        assert int("".join(map(str, bits[:c * B])), 2) % 7 == res[c]
+    seg_acc = []
+    for j in range(8):
+        cs = range(1 + j * m, 1 + (j + 1) * m)
+        seg_acc.append(sum(res[c] == 0 for c in cs) / m)
+    acc1 = sum(res[c] == 0 for c in range(1, N)) / (N - 1)
+    acc4 = sum(res[c] < 4 for c in range(1, N)) / (N - 1)
+    w = gen.workload("c1")
+    f = oracle.features(w.table, w.start, w.accept, bits, B=B, k=4)
+    assert f["acc1"] == pytest.approx(acc1, abs=1e-12)
+    assert f["acck"] == pytest.approx(acc4, abs=1e-12)
+    assert f["sens"] == pytest.approx(max(seg_acc) - min(seg_acc), abs=1e-12)
+    assert f["sens"] > 0.5
+
+
+def test_features_sens_c3s_region_boundary():
+    """Input sensitivity on the input-sensitive C3 stream: a profile slice whose first
+    half lies in a normal region and second half in a vowel-free region.
+    Expected per-segment accuracy by brute force: true chunk starts from the sequential
+    run (pinned above), predictions from the lookback ranking (pinned above), 8 equal
+    segments of the N - 1 = 64 profile chunks."""
+    w = gen.workload("c3s")
+    B, N = 4096, 65
+    region = 1 << 26
+    lo = region - 33 * B         # chunks 1..32 normal, 33..64 vowel-free
+    data = w.host(lo, N * B)
+    perm, inv, _, tt, acc = oracle.transform(w.table, w.accept)
+    r = oracle.run(w.table, w.start, w.accept, data, B)
+    m = (N - 1) // 8
+    seg = [0] * 8
+    for c in range(1, N):
+        qs, _ = oracle.lookback(tt, w.nstates, data[c * B - 2:c * B], K=16)
+        seg[(c - 1) // m] += int(qs[0] == perm[r["chunk_end"][c - 1]])
+    seg_acc = [s / m for s in seg]
+    f = oracle.features(w.table, w.start, w.accept, data, B=B)
+    assert f["sens"] == pytest.approx(max(seg_acc) - min(seg_acc), abs=1e-12)
+    assert f["acc1"] == pytest.approx(sum(seg) / (N - 1), abs=1e-12)
+    assert max(seg_acc[4:]) > min(seg_acc[:4]) and f["sens"] >= 0.2  # the regions really differ
+
+
+def test_select_enum_bound_31_32():
+    """R19: the ENUM leaf needs n <= 31 real states (n + poison in one warp)."""
+    f = {"acc1": 0.0, "acck": 0.0, "sens": 0.0, "uniq10": 31.0}
+    assert oracle.select(f, 31) == oracle.ENUM
+    assert oracle.select(dict(f, uniq10=15.5), 31) == oracle.ENUM
+    assert oracle.select(dict(f, uniq10=15.4), 31) != oracle.ENUM
+    assert oracle.select(dict(f, uniq10=32.0), 32) != oracle.ENUM
+    assert oracle.select(dict(f, uniq10=32.0), 32) == oracle.SRE  # acck - acc1 < 0.5 (R19b)
+
+
+def test_run_stream_div7_closed_form():
+    """The streamed oracle (blocks folded left) against the div7 closed
+    form: every chunk end = prefix value mod 7, final accept = big integer mod 7 == 0."""
+    w = gen.workload("c1", length=50000)
+    bits = w.host()
+    B = 16
+    r = oracle.run_stream(w.table, w.start, w.accept, w.host, bits.size, B, block=4096, prefetch=2)
+    res = div7_prefix_residues(bits)
+    ends = np.minimum(np.arange(1, oracle.nchunks(bits.size, B) + 1) * B, bits.size) - 1
+    assert (r["chunk_end"] == res[ends]).all()
+    assert r["final"] == int("".join(map(str, bits)), 2) % 7
+    assert r["accept"] == int(r["final"] == 0)
+    assert r["count"] == int((res == 0).sum())
