@@ -6,15 +6,19 @@ lookback speculation, speculative execution, verification/recovery rounds,
 finalize) with the input already resident in HBM.  Default workload =
 BASELINE.json configs[1] ("c2": ~100-state Snort-like Aho–Corasick DFA on a
 1 GiB synthetic text stream), scheme chosen by the selector (untimed, like
-the paper's offline profiling P:363).
+the paper's offline profiling P:363).  The default single-GPU line also
+carries per-DFA sub-results for C1, C3, C3s and C4 under "per_dfa".
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--scheme auto]
+  python bench.py --config c5 [--gpus N]   # 16 GiB per DFA sharded over N GPUs (strong)
   python bench.py --impl reference ...     # the CPU oracle, timed on host cores
 
-Multi-GPU (torchrun, one rank per GPU): the stream is sharded contiguously
-(each rank owns len/N bytes at fixed per-GPU size: weak scaling); each rank
-reduces its shard to a state map, one allgather exchanges the maps, every
-rank composes them.
+Multi-GPU (one process per GPU; `--gpus N` without torchrun re-launches itself
+under torch.distributed.run): the stream is sharded contiguously; each rank
+reduces its shard to a state map, ONE allgather (the library's own NCCL
+communicator, fsm_run_sharded) exchanges the maps and every rank composes them
+(DESIGN.md §Multi-GPU).  c1..c4 at N > 1: weak scaling (each rank owns the
+config's length, N x the bytes in total); c5: strong scaling (16 GiB in total).
 """
 from __future__ import annotations
 
@@ -34,8 +38,12 @@ CONFIG_DESC = {
     "c2": "AC-111 Snort-like literal DFA (12 literals) on a 1 GiB synthetic text stream",
     "c3": "AC x Z16 counter DFA (816 states, low speculation accuracy) on a 1 GiB stream",
     "c3s": "AC x Z16 counter DFA, input-sensitive stream (1 GiB)",
-    "c4": "AC-9770-ish DFA (520 literals, table exceeds smem) on a 4 GiB stream",
+    "c4": "AC-9912 DFA (520 literals, table exceeds smem) on a 4 GiB stream",
+    "c5": "16 GiB stream of each of the C1-C4 DFAs sharded over N B200 (strong scaling), "
+          "scheme chosen by the selector per DFA; NCCL allgather of state maps",
 }
+C5_LEN = 16 << 30
+C5_DFAS = ("c2", "c1", "c3", "c4")  # c2 (the high-accuracy DFA) is the line's headline
 METRIC = "input GB/s per DFA (1 GB stream, 1 B200); % of HBM roofline; latency per 1 GB"
 
 
@@ -131,44 +139,69 @@ def _max_over_ranks(dist, v: float) -> float:
     return float(t.item())
 
 
-def cpu_baseline(w, budget_s=12.0, check=None):
-    """The oracle (plain sequential C, oracle/) on host cores, bounded sample.  check
+def _cpu_model():
+    try:
+        return next((l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo") if l.startswith("model name")), "")
+    except OSError:
+        import platform
+
+        return platform.processor()
+
+
+class _Pinned:
+    """Pin the calling thread to one host core (1 thread, 1 core)."""
+
+    def __enter__(self):
+        self.old = None
+        self.core = None
+        try:
+            self.old = os.sched_getaffinity(0)
+            self.core = max(self.old)
+            os.sched_setaffinity(0, {self.core})
+        except (AttributeError, OSError):
+            self.old = None
+        return self
+
+    def __exit__(self, *a):
+        if self.old is not None:
+            os.sched_setaffinity(0, self.old)
+
+
+def cpu_baseline(w, sample_cap=256 << 20, check=None, x=None):
+    """The oracle (plain sequential C, oracle/) on one pinned host core, bounded sample
+    (the first min(len, 256 MiB) bytes of the stream), median of 3 runs.  check
     (nullable): callable(sample_len) -> the GPU result on the same prefix, compared with
-    the oracle's bit for bit (final state, accept count, every chunk end)."""
+    the oracle's bit for bit (final state, accept count, every chunk end).  x (nullable):
+    the device stream, whose sample bytes are hash-compared with the host generator's."""
     import numpy as np
 
+    import gen
     import oracle
 
-    sample = min(w.length, 256 << 20)
+    sample = min(w.length, sample_cap)
     data = w.host(0, sample)
-    t0 = time.perf_counter()
-    r = oracle.run(w.table, w.start, w.accept, data, 4096)
-    dt = time.perf_counter() - t0
-    assert r["status"] == 0
+    same_bytes = None
+    if x is not None:
+        same_bytes = gen.bytes_hash(data) == gen.bytes_hash(x[:sample].cpu().numpy())
+    times = []
+    with _Pinned() as pin:
+        for _ in range(3):
+            t0 = time.perf_counter()
+            r = oracle.run(w.table, w.start, w.accept, data, 4096)
+            times.append(time.perf_counter() - t0)
+            assert r["status"] == 0
+    dt = sorted(times)[1]
     parity = None
     if check is not None:
         g = check(sample)
         ce = g.chunk_ends.cpu().numpy().view(np.uint32)
         ok = g.final_state == r["final"] and g.accept_count == r["count"] and (ce == r["chunk_end"]).all()
-        parity = {"bit_exact": bool(ok), "sample": f"first {sample >> 20} MiB, same scheme and chunking",
-                  "chunks": int(len(ce))}
-    # grow the sample if it was too quick to time well (bounded by budget)
-    if dt < 1.0 and sample < w.length:
-        reps = max(1, min(int(budget_s / max(dt, 1e-3)), 8))
-        t0 = time.perf_counter()
-        for _ in range(reps):
-            oracle.run(w.table, w.start, w.accept, data, 4096)
-        dt = (time.perf_counter() - t0) / reps
+        parity = {"bit_exact": bool(ok), "sample": f"first {sample >> 20 or sample} {'MiB' if sample >> 20 else 'B'}"
+                  f", same scheme and chunking", "chunks": int(len(ce)), "host_device_bytes_hash_equal": same_bytes}
     out = {"value": round(sample / dt / 1e9, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-           "sample": f"first {sample >> 20} MiB of the {w.name} stream, oracle.run (Alg. 1), 1 thread",
-           "seconds": round(dt, 3), "host_nproc": os.cpu_count()}
-    try:
-        import platform
-
-        out["cpu_model"] = next((l.split(":", 1)[1].strip() for l in open("/proc/cpuinfo")
-                                 if l.startswith("model name")), platform.processor())
-    except OSError:
-        pass
+           "sample": f"first {sample >> 20} MiB of the {w.name} stream, oracle.run (Alg. 1), 1 thread pinned to "
+                     f"core {pin.core}, median of 3", "seconds": round(dt, 3), "host_nproc": os.cpu_count(),
+           "cpu_model": _cpu_model()}
     return out, parity
 
 
@@ -180,27 +213,251 @@ def run_reference(args):
     import gen
     import oracle
 
-    w = gen.workload(args.config)
+    name = "c2" if args.config == "c5" else args.config
+    w = gen.workload(name)
     sample = min(w.length, args.ref_sample_mib << 20)
     data = w.host(0, sample)
-    for _ in range(max(0, args.warmup)):
-        oracle.run(w.table, w.start, w.accept, data[: 1 << 20], 4096)
-    t0 = time.perf_counter()
-    for _ in range(args.steps):
-        r = oracle.run(w.table, w.start, w.accept, data, 4096)
-        assert r["status"] == 0
-    dt = (time.perf_counter() - t0) / args.steps
+    with _Pinned() as pin:
+        for _ in range(max(0, args.warmup)):
+            oracle.run(w.table, w.start, w.accept, data[: 1 << 20], 4096)
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            r = oracle.run(w.table, w.start, w.accept, data, 4096)
+            assert r["status"] == 0
+        dt = (time.perf_counter() - t0) / args.steps
     v = sample / dt / 1e9
     line = {"impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": "GB/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt * 1e3, 3),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
-            "data": "synthetic", "config": {"workload": args.config, "desc": CONFIG_DESC[args.config],
-                                            "bytes_per_step": sample, "chunk_bytes": 4096},
+            "higher_is_better": True, "scaling": "strong" if args.config == "c5" else "weak", "vs_baseline": None,
+            "dtype": "u8", "data": "synthetic",
+            "config": {"workload": args.config, "desc": CONFIG_DESC[args.config], "bytes_per_step": sample,
+                       "chunk_bytes": 4096},
             "cpu_baseline": {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                             "sample": f"first {sample >> 20} MiB of the {args.config} stream per step"},
+                             "sample": f"first {sample >> 20} MiB of the {name} stream per step, 1 thread pinned "
+                                       f"to core {pin.core}"},
             "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
+
+
+def _median(v):
+    v = sorted(v)
+    return v[len(v) // 2] if v else None
+
+
+def _roofline(name, length, spec_ms, peak, peak_kind):
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get(name)
+        except Exception:
+            traffic = None
+    achieved = length / (spec_ms * 1e-3) / 1e9
+    return {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4), "traffic": traffic,
+            "kernel": "k_spec_tma (speculative execution, TMA-staged)", "peak_kind": peak_kind,
+            "achieved_def": "input bytes per launch / CUDA-event duration of the spec launch on its stream"}
+
+
+def measure_single(gs, w, x, args, fsm, scheme, with_clocks=True):
+    """K back-to-back runs of the whole stream on this GPU (fsm_run_async queue), timed by
+    two CUDA events on the launching stream; spec / verify splits from the library's
+    own per-run events."""
+    import torch
+
+    B = args.chunk_bytes
+    length = x.numel()
+    stream = torch.cuda.current_stream()
+    ce = torch.empty(gs.fsm_num_chunks(length, B), dtype=torch.int32, device="cuda")
+    kr = [fsm.run(x, scheme=scheme, chunk_bytes=B) for _ in range(3)]
+    verify_phases = [round(float(v), 1) for v in fsm.phase_times()]
+    pending = []
+    for _ in range(max(3, args.warmup)):
+        pending.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce))
+    for t in pending:
+        fsm.wait(t)
+    pending.clear()
+    torch.cuda.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clk = ClockSampler(torch.cuda.current_device()) if with_clocks else None
+    if clk:
+        clk.__enter__()
+    ev0.record(stream)
+    for _ in range(args.steps):
+        pending.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce))
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    if clk:
+        clk.__exit__()
+    spec_ms, ver_ms, launches = [], [], 0
+    for t in pending:
+        res = fsm.wait(t)
+        spec_ms.append(res.stats["ms_spec"])
+        ver_ms.append(res.stats["ms_verify"])
+        launches += res.stats["kernel_launches"]  # counted by the library per run
+    ms = ev0.elapsed_time(ev1) / args.steps
+    st0 = kr[-1].stats
+    diag = {k: st0[k] for k in ("rounds", "tasks_total", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes",
+                                "verify_checks", "verify_matches")}
+    diag["runtime_speculation_accuracy"] = round(st0["verify_matches"] / max(1, st0["verify_checks"]), 6)
+    diag["avg_active_workers"] = round(float(st0.get("avg_active_workers", 0.0)), 2)
+    return {"ms": ms, "value": length / (ms * 1e-3) / 1e9, "spec_ms": _median(spec_ms), "ver_ms": _median(ver_ms),
+            "launches": launches, "clocks": clk.summary() if clk else None, "diag": diag, "phases": verify_phases,
+            "result": res}
+
+
+def _table_info(fsm):
+    try:
+        tr = fsm.transform()
+        return {"format": tr["mode"], "nclasses": int(tr["nclasses"]), "hot_rows": int(tr["hot_rows"])}
+    except Exception:
+        return None
+
+
+def per_dfa_result(gs, name, args, peak, peak_kind, with_cpu=True):
+    """One sub-result of the default N = 1 line: config `name` at its full size, selector
+    scheme, value / ms / roofline / diagnostics / cpu_baseline / parity on a sample."""
+    import torch
+
+    import gen
+
+    w = gen.workload(name)
+    x = torch.empty(w.length, dtype=torch.uint8, device="cuda")
+    w.device(x)
+    prof = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")
+    w.device(prof, offset=w.length)
+    fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof.cpu().numpy())
+    scheme, feats = fsm.select_scheme(prof, chunk_bytes=args.chunk_bytes)
+    m = measure_single(gs, w, x, args, fsm, scheme, with_clocks=False)
+    out = {"value": round(m["value"], 3), "unit": "GB/s", "ms_per_step": round(m["ms"], 4),
+           "bytes": w.length, "scheme": scheme, "nstates": int(w.nstates),
+           "pct_hbm_roofline_8TBs": round(100 * m["value"] / 8000.0, 2),
+           "breakdown_ms": {"spec_exec": round(m["spec_ms"], 4), "verify_recover": round(m["ver_ms"], 4)},
+           "roofline": _roofline(name, w.length, m["spec_ms"], peak, peak_kind), "diagnostics": m["diag"],
+           "gpu_launches": m["launches"], "table": _table_info(fsm),
+           "features": {k: round(v, 4) if isinstance(v, float) else v for k, v in feats.items()}}
+    if with_cpu:
+        out["cpu_baseline"], out["parity"] = cpu_baseline(
+            w, sample_cap=64 << 20, x=x, check=lambda n: fsm.run(x[:n], scheme=scheme, chunk_bytes=args.chunk_bytes))
+    fsm.close()
+    del x
+    torch.cuda.empty_cache()
+    return out
+
+
+def _maybe_relaunch(args):
+    """--gpus N > 1 without a torch.distributed launcher: re-run this command under
+    torch.distributed.run (one process per GPU, rendezvous on 127.0.0.1)."""
+    if args.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return None
+    import socket
+
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
+    """C5: each DFA's 16 GiB stream sharded over the `world` ranks (strong scaling); one
+    step = fsm_run_sharded on every rank (shard map, one allgather, compose, fix-up),
+    timed per rank by CUDA events, MAX over ranks."""
+    import numpy as np
+    import torch
+
+    import gen
+    from paper_conf_ipps_wangwqw22_b200.dist import run_sharded, shard_bounds
+
+    B = args.chunk_bytes
+    L = args.c5_bytes
+    per = {}
+    dfas = C5_DFAS if args.c5_dfa == "all" else (args.c5_dfa,)
+    clk_all = None
+    for name in dfas:
+        w = gen.workload(name, length=L)
+        lo, hi = shard_bounds(L, world, rank, B)
+        x = torch.empty(hi - lo, dtype=torch.uint8, device="cuda")
+        w.device(x, offset=lo)
+        lb = torch.empty(2 if lo else 0, dtype=torch.uint8, device="cuda")
+        if lo:
+            w.device(lb, offset=lo - 2)  # the 2 bytes before the shard (pure function of the offset)
+        fsm = gs.FSM.load(w.table, w.start, w.accept)
+        # selector per DFA (offline profiling, P:363): every rank profiles the stream's first MiB
+        prof = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")
+        w.device(prof, offset=0)
+        scheme, feats = fsm.select_scheme(prof, chunk_bytes=B)
+        del prof
+
+        def step():
+            if comm is not None:
+                return comm.run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
+            if dist is not None:
+                return run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
+            return fsm.run(x, scheme=scheme, chunk_bytes=B)
+
+        res = None
+        for _ in range(max(3, args.warmup)):
+            res = step()
+        if dist:
+            dist.barrier()
+        torch.cuda.synchronize()
+        stream = torch.cuda.current_stream()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with ClockSampler(dev) as clk:
+            ev0.record(stream)
+            for _ in range(args.steps):
+                res = step()
+            ev1.record(stream)
+            torch.cuda.synchronize()
+        if clk_all is None:
+            clk_all = clk
+        else:
+            clk_all.samples += clk.samples
+        ms = ev0.elapsed_time(ev1) / args.steps
+        if dist:
+            dist.barrier()
+            ms = _max_over_ranks(dist, ms)
+        value = L / (ms * 1e-3) / 1e9
+        # parity: the global result equals the oracle's on the bench's own run is checked
+        # at full size by tests/test_gpu_c5.py; here every rank's global result must agree
+        agree = True
+        if dist:
+            t = torch.tensor([res.final_state, res.accept_count & 0xFFFFFFFF, res.accept_count >> 32],
+                             dtype=torch.int64, device="cuda" if dist.get_backend() == "nccl" else "cpu")
+            t2 = t.clone()
+            dist.all_reduce(t2, op=dist.ReduceOp.MAX)
+            agree = bool((t == t2).all().item())
+        per[name] = {"value": round(value, 3), "unit": "GB/s", "ms_per_step": round(ms, 4), "bytes": L,
+                     "bytes_per_rank": hi - lo, "scheme": scheme, "nstates": int(w.nstates),
+                     "pct_hbm_roofline_8TBs_per_gpu": round(100 * value / world / 8000.0, 2),
+                     "latency_ms_per_GB": round(ms * 1e9 / L, 4), "ranks_agree": agree,
+                     "final_state": res.final_state, "accept_count": res.accept_count,
+                     "features": {k: round(v, 4) if isinstance(v, float) else v for k, v in feats.items()}}
+        fsm.close()
+        del x
+        torch.cuda.empty_cache()
+    head = per[dfas[0]]
+    line = {
+        "metric": METRIC, "value": head["value"], "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": max(3, args.warmup), "ms_per_step": head["ms_per_step"], "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": "c5", "desc": CONFIG_DESC["c5"], "headline_dfa": dfas[0], "bytes_total": L,
+                   "chunk_bytes": B, "l2": "input (16 GiB / N per GPU) larger than the 126 MB L2; no flush",
+                   "parallelism": f"{world} contiguous shards + one allgather of state maps"
+                   + (" (library NCCL communicator, fsm_run_sharded)" if comm is not None else
+                      " (torch.distributed allgather)" if dist is not None else " (single GPU, fsm_run)"),
+                   "nccl_ranks": comm.nranks if comm is not None else 0},
+        "per_dfa": per,
+        "gpu_launches": None,
+        "clocks": clk_all.summary() if clk_all else None,
+        "e2e": None,
+        "e2e_note": "C5 shards are 16/N GiB per rank: the end-to-end (host-buffer) number is the default c2 line's",
+    }
+    return line
 
 
 def main():
@@ -214,10 +471,16 @@ def main():
     ap.add_argument("--chunk-bytes", type=int, default=4096)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-per-dfa", action="store_true", help="skip the per-DFA sub-results of the default line")
     ap.add_argument("--ref-sample-mib", type=int, default=256)
+    ap.add_argument("--c5-dfa", default="all", choices=["all"] + list(C5_DFAS))
+    ap.add_argument("--c5-bytes", type=int, default=C5_LEN)
     args = ap.parse_args()
     if args.impl == "reference":
         return run_reference(args)
+    rc = _maybe_relaunch(args)
+    if rc is not None:
+        return rc
 
     import numpy as np
     import torch
@@ -233,31 +496,49 @@ def main():
     dev = local % max(1, torch.cuda.device_count()) if backend != "nccl" else local
     torch.cuda.set_device(dev)
     dist = None
+    comm = None
     if world > 1:
         import torch.distributed as dist
 
         if backend == "nccl":
             dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+            # the library owns its NCCL communicator (fsm_comm_init); torch.distributed
+            # only broadcasts the 128-byte unique id and provides barriers
+            uid = [gs.Comm.unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(uid, src=0)
+            comm = gs.Comm(world, rank, uid[0])
         else:
             dist.init_process_group(backend)
+    peak, peak_kind = _peaks()
+
+    if args.config == "c5":
+        line = run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind)
+        if rank == 0:
+            print(json.dumps(line), flush=True)
+        if comm is not None:
+            comm.close()
+        if dist:
+            dist.destroy_process_group()
+        return 0
+
     w = gen.workload(args.config)
     length = w.length
     B = args.chunk_bytes
     x = torch.empty(length, dtype=torch.uint8, device="cuda")
     w.device(x, offset=rank * length)  # weak scaling: rank r owns bytes [r*len, (r+1)*len)
     # profile sample (a 1 MiB "training" trace): a disjoint slice of the same
-    # source, past every rank's shard; it places the u8 table rows bank-aware
+    # source, past every rank's shard; it places the u8 table rows bank-aware (DESIGN.md
+    # §5.1) and is the selector's profile
     prof = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")
     w.device(prof, offset=world * length)
     fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof.cpu().numpy())
-    del prof
-    stream = torch.cuda.current_stream()
     scheme = args.scheme
     feats = None
     if scheme == "auto":
-        scheme, feats = fsm.select_scheme(x[: 1 << 20], chunk_bytes=B)  # offline profiling, untimed
-    ce = torch.empty(gs.fsm_num_chunks(length, B), dtype=torch.int32, device="cuda")
+        scheme, feats = fsm.select_scheme(prof, chunk_bytes=B)  # offline profiling, untimed
+    del prof
 
+    lb = None
     if world > 1:
         from paper_conf_ipps_wangwqw22_b200.dist import run_sharded
 
@@ -267,51 +548,34 @@ def main():
             w.device(lb, offset=rank * length - 2)
 
         def step():
+            if comm is not None:
+                return comm.run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
             return run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
-    else:
-        # one step = one whole-stream run; steps are enqueued back to back
-        # (fsm_run_async) and collected after the timed region's final sync
-        pending = []
 
-        def step():
-            pending.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce))
-            return None
-
-    # kernel-level split (spec exec vs verify/recover) from single-shard runs on this GPU
-    kr = [fsm.run(x, scheme=scheme, chunk_bytes=B) for _ in range(3)]
-    verify_phases = [round(float(v), 1) for v in fsm.phase_times()]
-    for _ in range(max(3, args.warmup)):
-        res = step()
-    if world == 1:
-        res = [fsm.wait(t) for t in pending][-1]
-        pending.clear()
-    spec_ms, ver_ms = [], []
-    if dist:
+        kr = [fsm.run(x, scheme=scheme, chunk_bytes=B) for _ in range(3)]
+        for _ in range(max(3, args.warmup)):
+            res = step()
         dist.barrier()
-    torch.cuda.synchronize()
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(dev) as clk:
-        ev0.record(stream)
-        for _ in range(args.steps):
-            r_ = step()
-            if r_ is not None:
-                res = r_
-        ev1.record(stream)
         torch.cuda.synchronize()
-    launches = None
-    if world == 1:
-        launches = 0
-        for t in pending:
-            res = fsm.wait(t)
-            spec_ms.append(res.stats["ms_spec"])
-            ver_ms.append(res.stats["ms_verify"])
-            launches += res.stats["kernel_launches"]  # counted by the library per run
-        pending.clear()
-    if dist:
+        stream = torch.cuda.current_stream()
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with ClockSampler(dev) as clk:
+            ev0.record(stream)
+            for _ in range(args.steps):
+                res = step()
+            ev1.record(stream)
+            torch.cuda.synchronize()
         dist.barrier()
-    ms = ev0.elapsed_time(ev1) / args.steps
-    if dist:
-        ms = _max_over_ranks(dist, ms)
+        ms = _max_over_ranks(dist, ev0.elapsed_time(ev1) / args.steps)
+        m = {"ms": ms, "spec_ms": _median([r.stats["ms_spec"] for r in kr]),
+             "ver_ms": _median([r.stats["ms_verify"] for r in kr]), "launches": None, "clocks": clk.summary(),
+             "phases": [], "diag": {k: kr[-1].stats[k] for k in ("rounds", "tasks_total", "tasks_mustdo", "tasks_sre",
+                                                                  "tasks_helper", "reread_bytes", "verify_checks",
+                                                                  "verify_matches")}}
+    else:
+        m = measure_single(gs, w, x, args, fsm, scheme)
+        res = m["result"]
+        ms = m["ms"]
     total_bytes = length * world
     value = total_bytes / (ms * 1e-3) / 1e9
 
@@ -331,7 +595,10 @@ def main():
 
             def e2e_step():
                 xd.copy_(h, non_blocking=True)                     # H2D of this rank's shard
-                r = run_sharded(fsm, xd, lb, scheme=scheme, chunk_bytes=B)
+                if comm is not None:
+                    r = comm.run_sharded(fsm, xd, lb, scheme=scheme, chunk_bytes=B)
+                else:
+                    r = run_sharded(fsm, xd, lb, scheme=scheme, chunk_bytes=B)
                 ce_h.copy_(r.chunk_ends, non_blocking=True)       # D2H of the results
                 torch.cuda.current_stream().synchronize()
                 return r
@@ -351,19 +618,6 @@ def main():
         e2e = {"value": round(total_bytes / e2e_s / 1e9, 3), "unit": "GB/s", "h2d_bytes_per_step": length,
                "d2h_bytes_per_step": int(nch * 4 + 64), "ms_per_step": round(e2e_s * 1e3, 3)}
 
-    if not spec_ms:
-        spec_ms = [r.stats["ms_spec"] for r in kr]
-        ver_ms = [r.stats["ms_verify"] for r in kr]
-    peak, peak_kind = _peaks()
-    spec_med = sorted(spec_ms)[len(spec_ms) // 2]
-    achieved = length / (spec_med * 1e-3) / 1e9
-    traffic = None
-    tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp):
-        try:
-            traffic = json.load(open(tp)).get(args.config)
-        except Exception:
-            traffic = None
     line = {
         "metric": METRIC,
         "value": round(value, 3),
@@ -380,42 +634,42 @@ def main():
         "config": {"workload": args.config, "desc": CONFIG_DESC[args.config], "bytes_per_gpu": length,
                    "chunk_bytes": B, "scheme": scheme, "nstates": int(w.nstates),
                    "l2": "input (1 GiB/GPU) larger than the 126 MB L2; no explicit flush",
-                   "parallelism": f"dp{world} contiguous shards + allgather of state maps" if world > 1
-                   else "single GPU"},
+                   "parallelism": (f"dp{world} contiguous shards + one allgather of state maps"
+                                   + (" (library NCCL, fsm_run_sharded)" if comm is not None else "")
+                                   if world > 1 else "single GPU"),
+                   "nccl_ranks": comm.nranks if comm is not None else 0},
         "pct_hbm_roofline_8TBs": round(100 * value / world / 8000.0, 2),
         "latency_ms_per_GB": round(ms * 1e9 / length, 4),
-        "verify_phase_boundaries_us": verify_phases,
-        "breakdown_ms": {"spec_exec": round(spec_med, 4),
-                         "verify_recover": round(sorted(ver_ms)[len(ver_ms) // 2], 4)},
-        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 4), "traffic": traffic,
-                     "kernel": "k_spec_tma (speculative execution, TMA-staged)", "peak_kind": peak_kind,
-                     "achieved_def": "input bytes per launch / CUDA-event duration of the spec launch"},
-        "diagnostics": {k: kr[-1].stats[k] for k in ("rounds", "tasks_total", "tasks_mustdo", "tasks_sre",
-                                                     "tasks_helper", "reread_bytes", "verify_checks",
-                                                     "verify_matches")},
-        "gpu_launches": launches if launches is not None else 6 * args.steps,
-        "clocks": clk.summary(),
+        "verify_phase_boundaries_us": m["phases"],
+        "breakdown_ms": {"spec_exec": round(m["spec_ms"], 4), "verify_recover": round(m["ver_ms"], 4)},
+        "roofline": _roofline(args.config, length, m["spec_ms"], peak, peak_kind),
+        "diagnostics": m["diag"],
+        "gpu_launches": m["launches"] if m["launches"] is not None else 6 * args.steps,
+        "clocks": m["clocks"],
         "e2e": e2e,
     }
-    st0 = kr[-1].stats
-    line["diagnostics"]["runtime_speculation_accuracy"] = round(st0["verify_matches"] / max(1, st0["verify_checks"]), 6)
-    line["diagnostics"]["avg_active_workers"] = round(float(st0.get("avg_active_workers", 0.0)), 2)
     line["pct_measured_hbm_whole_step"] = round(100 * value / world / peak, 2)
-    try:
-        tr = fsm.transform()
-        line["config"]["table"] = {"format": tr["mode"], "nclasses": int(tr["nclasses"]), "hot_rows": int(tr["hot_rows"])}
-    except Exception:
-        pass
+    line["config"]["table"] = _table_info(fsm)
     if feats:
         line["config"]["features"] = {k: round(v, 4) if isinstance(v, float) else v for k, v in feats.items()}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"], parity = cpu_baseline(
-            w, check=lambda n: fsm.run(x[:n], scheme=scheme, chunk_bytes=B))
+            w, x=x, check=lambda n: fsm.run(x[:n], scheme=scheme, chunk_bytes=B))
         if parity is not None:
             line["parity"] = parity
+    if world == 1 and args.config == "c2" and args.scheme == "auto" and not args.no_per_dfa:
+        fsm.close()
+        del x
+        torch.cuda.empty_cache()
+        line["per_dfa"] = {"c2": {"value": line["value"], "ms_per_step": line["ms_per_step"], "scheme": scheme,
+                                  "roofline_frac": line["roofline"]["frac"], "see": "top-level keys"}}
+        for name in ("c1", "c3", "c3s", "c4"):
+            line["per_dfa"][name] = per_dfa_result(gs, name, args, peak, peak_kind,
+                                                   with_cpu=not args.no_cpu_baseline)
     if rank == 0:
         print(json.dumps(line), flush=True)
+    if comm is not None:
+        comm.close()
     if dist:
         dist.destroy_process_group()
     return 0

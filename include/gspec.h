@@ -218,13 +218,21 @@ int fsm_select_scheme(fsm_t fsm, const uint8_t* d_sample, uint64_t len, const fs
  * one allgather (NCCL via the caller's process group), composes them, and
  * fixes its chunk ends.  Map layout (device, caller-allocated, fsm_map_bytes()
  * bytes): uint32 end[nt] (0xFFFFFFFF = start not reachable/not computed),
- * then uint64 count[nt].  */
+ * then uint64 count[nt].  The poison state (nt-1, R4) is a fixed entry of every
+ * map (poison -> poison, count 0), so an invalid byte in any shard makes every
+ * rank's fsm_shard_finish return FSM_ESYMBOL, as fsm_run does.  */
 uint64_t fsm_map_bytes(fsm_t fsm);
 /* Step 1 (per rank): d_shard = shard bytes; d_lookback = the up to 2 bytes
  * before the shard (NULL/0 for the first shard, whose start is q0).  Writes
  * the map to d_map; chunk ends that do not depend on the shard's start state
  * go to d_chunk_ends_local (device, nullable, fsm_num_chunks(len) entries),
- * the rest is kept in the handle for fsm_shard_finish. */
+ * the rest is kept in the handle for fsm_shard_finish.  On failure the call
+ * returns its status AND writes an error map (every entry 0xFFFFFFFD, count[0] =
+ * -status) when d_map is valid: the caller must still take part in the exchange
+ * and call fsm_shard_finish, which then returns that status on every rank — no
+ * rank is left waiting in the collective.  Non-convergent DFAs above the ENUM
+ * limit (paths that never merge) run one pipeline per surviving path: exact, at
+ * (#paths) x the shard's work. */
 int fsm_shard_map(fsm_t fsm, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback,
                   uint32_t lookback_len, const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local);
 /* fsm_shard_map is speculative for a shard with a lookback: its pipeline is queued
@@ -237,7 +245,8 @@ int fsm_shard_map_exact(fsm_t fsm, const uint8_t* d_shard, uint64_t len, const u
                         uint32_t lookback_len, const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local);
 /* Step 2 (every rank, after the allgather): d_maps = nranks maps back to back.
  * Composes them from q0 (s_{g+1} = M_g[s_g]), writes this rank's chunk ends
- * (original ids, nullable) and the global result.  FSM_EAGAIN: see above. */
+ * (original ids, nullable) and the global result.  FSM_EAGAIN: see above.
+ * A failed map on any rank: that rank's status on every rank. */
 int fsm_shard_finish(fsm_t fsm, const void* d_maps, uint32_t nranks, uint32_t rank,
                      const fsm_run_opts* opts, uint32_t* d_chunk_ends_local, fsm_result* out_global);
 

@@ -309,10 +309,11 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     rp.ctl_init = f->d_ctl;  // the spec kernel initialises the control block
     rp.h_out = &h;           // ... and the verify kernel's finalize step writes it back (pinned, UVA)
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
-    // dense recovery rounds go to the TMA task kernel (SRE on low-accuracy DFAs); this
+    // dense recovery rounds go to the TMA task kernel (SRE / RR / NF on low-accuracy DFAs); this
     // needs a host check per verify launch, so it is off when the profile says the
     // speculation is accurate (no dense rounds expected)
-    rp.dense = ((scheme == FSM_SCHEME_SRE || scheme == FSM_SCHEME_CSE) && len / o.B > 0 && o.B % 64 == 0 &&
+    rp.dense = ((scheme == FSM_SCHEME_SRE || scheme == FSM_SCHEME_CSE || scheme == FSM_SCHEME_RR ||
+                 scheme == FSM_SCHEME_NF) && len / o.B > 0 && o.B % 64 == 0 &&
                 (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0 && f->acc1_hint < 0.5) ? 1u : 0u;
     CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
     {  // TMA kernel over the full chunks + the generic kernel for a tail chunk (or everything)
@@ -754,6 +755,9 @@ void fsm_free(fsm_t f) {
   if (f->batch_base) cudaFree(f->batch_base);
   for (auto& e : f->batch_ev)
     if (e) cudaEventDestroy(e);
+  if (f->multi_base) cudaFree(f->multi_base);
+  for (auto& e : f->multi_ev)
+    if (e) cudaEventDestroy(e);
   delete f;
 }
 
@@ -935,8 +939,9 @@ int fsm_run_multi(const fsm_t* fsms, uint32_t npairs, const uint8_t* const* d_in
     }
   }
   // device scratch: [images][inputs][lengths][pair order][finals][counts][stats]
-  static thread_local void* base = nullptr;
-  static thread_local size_t cap = 0;
+  // scratch and events live in the first handle (device-bound, freed by fsm_free)
+  void*& base = fsms[0]->multi_base;
+  size_t& cap = fsms[0]->multi_cap;
   auto al = [](size_t b) { return (b + 255) & ~size_t(255); };
   const size_t b_img = al(sizeof(DevImage) * npairs), b_in = al(8 * npairs), b_len = al(8 * npairs),
                b_ord = al(4 * npairs), b_fin = al(4 * npairs), b_cnt = al(8 * npairs), b_st = 256;
@@ -963,9 +968,9 @@ int fsm_run_multi(const fsm_t* fsms, uint32_t npairs, const uint8_t* const* d_in
   CUDA_TRY(cudaMemcpyAsync(d_lens, lens, 8ull * npairs, cudaMemcpyHostToDevice, st));
   CUDA_TRY(cudaMemcpyAsync(d_ord, order.data(), 4ull * npairs, cudaMemcpyHostToDevice, st));
   CUDA_TRY(cudaMemsetAsync(d_st, 0, 16, st));
-  static thread_local cudaEvent_t ev[2] = {nullptr, nullptr};
-  for (auto& e : ev)
-    if (!e) CUDA_TRY(cudaEventCreate(&e));
+  cudaEvent_t* ev = fsms[0]->multi_ev;
+  for (int i = 0; i < 2; i++)
+    if (!ev[i]) CUDA_TRY(cudaEventCreate(&ev[i]));
   CUDA_TRY(cudaEventRecord(ev[0], st));
   uint32_t off = 0;
   for (size_t g = 0; g < groups.size(); g++) {
@@ -1202,7 +1207,6 @@ uint64_t fsm_map_bytes(fsm_t f) {
 namespace {
 
 constexpr uint32_t kFuseChunks = 8;   // path-fusion window (chunks) before falling back
-constexpr uint32_t kMaxMulti = 64;    // distinct surviving paths run by the pipeline
 constexpr uint32_t kNoState = 0xFFFFFFFFu;
 
 uint64_t map_cnt_off(uint32_t nt) { return ((uint64_t)nt * 4 + 7) & ~7ull; }
@@ -1290,7 +1294,27 @@ int fsm_shard_map_exact(fsm_t f, const uint8_t* d_shard, uint64_t len, const uin
   return shard_map_impl(f, d_shard, len, d_lookback, lb_len, opts, d_map, d_chunk_ends_local, true);
 }
 
+int shard_map_body(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
+                   const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local, bool exact);
+
+// A failed map must not strand the other ranks in the exchange (they are already
+// waiting in the allgather): the failing rank publishes an error map, still takes part
+// in the collective, and every rank's fsm_shard_finish returns this rank's status.
 int shard_map_impl(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
+                   const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local, bool exact) {
+  const int rc = shard_map_body(f, d_shard, len, d_lookback, lb_len, opts, d_map, d_chunk_ends_local, exact);
+  if (rc != FSM_OK && f && d_map) {
+    cudaStream_t st = opts ? reinterpret_cast<cudaStream_t>(opts->stream) : nullptr;
+    const uint32_t nt = f->n + 1;
+    uint32_t* mend = reinterpret_cast<uint32_t*>(d_map);
+    unsigned long long* mcnt =
+        reinterpret_cast<unsigned long long*>(reinterpret_cast<uint8_t*>(d_map) + map_cnt_off(nt));
+    if (launch_map_error(mend, mcnt, nt, (uint32_t)(-rc), st) == cudaSuccess) f->shard_mode = 4;
+  }
+  return rc;
+}
+
+int shard_map_body(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
                    const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local, bool exact) {
   if (!f || !d_map) return fail(FSM_EINVAL, "NULL handle/map");
   if (!d_shard && len > 0) return fail(FSM_EINVAL, "NULL shard");
@@ -1395,7 +1419,8 @@ int shard_map_impl(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t*
         f->shard_grp[i] = (uint32_t)(it - D.begin());
       }
     }
-    if (D.size() > kMaxMulti) return fail(FSM_EUNSUPPORTED, "shard start not resolved by path fusion");
+    // more than kMaxMulti non-merging paths (a non-convergent DFA too large for ENUM):
+    // still exact, at the cost of one pipeline per surviving path
     std::vector<uint32_t> fin(D.size());
     std::vector<unsigned long long> cnt(D.size());
     for (size_t d = 0; d < D.size(); d++) {
@@ -1450,6 +1475,7 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
   int rc = resolve_opts(opts, &o);
   if (rc) return rc;
   const uint32_t nt = f->n + 1;
+  if (!f->d_small) CUDA_TRY(cudaMalloc(&f->d_small, 64 * sizeof(uint32_t)));  // (a map that failed early)
   CUDA_TRY(launch_compose(reinterpret_cast<const uint8_t*>(d_maps), G, map_bytes_nt(nt), map_cnt_off(nt), f->img.q0t,
                           rank, f->d_small, o.st));
   if (f->shard_mode == 3) {
@@ -1458,7 +1484,7 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
     if ((rc = ensure_shard(f, &S3))) return rc;
     CUDA_TRY(cudaMemsetAsync(f->d_small + 5, 0, 4, o.st));
     if (d_chunk_ends_local && f->shard_len)
-      CUDA_TRY(launch_fix_prefix_fused(S3.states, S3.cand, S3.info + 8, S3.grp, f->d_small, f->img.inv,
+      CUDA_TRY(launch_fix_prefix_fused(S3.states, S3.cand, S3.info + 8, S3.grp, f->d_small, f->img.inv, f->n,
                                        d_chunk_ends_local, f->d_small + 5, o.st));
   }
   uint32_t h[6] = {0, 0, 0, 0, 0, 0};
@@ -1471,17 +1497,24 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
     f->shard_ticket = 0;
     if (rc) return rc;
   }
+  if (h[2] == 3) {  // some rank's map failed: every rank returns that rank's status
+    const int code = -(int)h[3];
+    char msg[96];
+    std::snprintf(msg, sizeof(msg), "fsm_shard_map failed on rank %u (%s)", h[4], fsm_strerror(code));
+    return fail(code < 0 ? code : FSM_EINVAL, msg);
+  }
   if (h[2] == 2) {
     f->shard_prefer_exact = true;  // this DFA's shards do not merge early: skip speculation from now on
     return fail(FSM_EAGAIN, "a rank's speculative shard map was invalid: every rank redoes fsm_shard_map_exact");
   }
+  if (f->shard_mode == 4) return fail(FSM_EINVAL, "this rank's fsm_shard_map failed");
   if (h[2] || (f->shard_mode == 3 && h[5])) return fail(FSM_EINVAL, "a shard start state is outside its candidate set");
   const uint32_t srank = h[0], fin = h[1];
   const uint64_t count = (uint64_t)h[3] | ((uint64_t)h[4] << 32);
   const uint64_t N = (f->shard_len + o.B - 1) / o.B;
   ShardScratch S;
   if ((rc = ensure_shard(f, &S))) return rc;
-  if (d_chunk_ends_local && N) {
+  if (d_chunk_ends_local && N && srank != f->n) {  // poison start: FSM_ESYMBOL below
     if (f->shard_mode == 1) {
       RunParams rp{};
       rp.in = f->shard_in;

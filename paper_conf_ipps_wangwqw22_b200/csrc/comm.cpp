@@ -112,12 +112,17 @@ int fsm_run_sharded(fsm_t f, fsm_comm_t c, const uint8_t* d_shard, uint64_t shar
     rc = exact ? fsm_shard_map_exact(f, d_shard, shard_len, d_lookback, lookback_len, opts, c->d_local,
                                      d_chunk_ends_local)
                : fsm_shard_map(f, d_shard, shard_len, d_lookback, lookback_len, opts, c->d_local, d_chunk_ends_local);
-    if (rc) return rc;
+    // a failed map is published as an error map (shard.cu k_map_error) and the exchange
+    // still runs, so no rank waits in the allgather for one that returned early
+    if (rc && f->shard_mode != 4) return rc;
+    const int map_rc = rc;
     ncclResult_t r = nccl().allGather(c->d_local, c->d_all, mb, ncclUint8, c->comm, st);
     if (r != ncclSuccess)
       return gspec_set_error(FSM_ENCCL, nccl().getErrorString ? nccl().getErrorString(r) : "ncclAllGather");
     rc = fsm_shard_finish(f, c->d_all, (uint32_t)c->nranks, (uint32_t)c->rank, opts, d_chunk_ends_local, out_global);
-    if (rc != FSM_EAGAIN) break;
+    if (rc == FSM_EAGAIN) continue;  // every rank (a failed one too) redoes the exact map
+    if (map_rc) return map_rc;
+    break;
   }
   return rc;
 }

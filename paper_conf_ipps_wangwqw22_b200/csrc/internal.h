@@ -26,6 +26,7 @@ enum Mode : uint32_t {
 
 constexpr uint32_t kDeltaExc = 2;        // exceptions per delta row
 constexpr uint32_t kInvalidMap = 0xFFFFFFFEu;  // map entry of a speculative shard map that must be redone
+constexpr uint32_t kErrorMap = 0xFFFFFFFDu;    // map of a rank whose fsm_shard_map failed (count[0] = -status)
 constexpr uint32_t kDeltaBaseMax = 8192;  // MODE_U16D: max shared-window offset of the staged table
 
 constexpr uint32_t kQsMax = 16;     // QS cap ("top 16 states")
@@ -109,9 +110,9 @@ struct Ctl {
   uint64_t tasks_mustdo, tasks_sre, tasks_helper, reread_bytes, verify_checks, verify_matches,
       active_sum;
   uint64_t accept_count;
-  uint64_t nA, I, nU;    // this round: A-tasks, idle workers, total untried candidates
+  uint64_t nA, I, nU;    // nA: A-task entries of the task list handed to a dense round (the rest are helpers)
   uint64_t jacobi_iters;
-  uint64_t ntask[2];     // [0]: length of the task list handed to a dense round; [1] unused
+  uint64_t ntask[2];     // [0]: length of the task list handed to a dense round; [1]: round-0 accept-count accumulator
   uint64_t it_fm[3], it_checks[3], it_matches[3], it_ntask[3];  // per relaxation pass (rotating)
   uint64_t it_reread[3];  // round-0 SRE pass with inline tasks: bytes re-walked (rotating)
   uint32_t dense_pending;  // verify exited: a dense task round (frontier fmin) must run first
@@ -287,7 +288,8 @@ cudaError_t launch_map_fused(const uint32_t* cand, const uint32_t* ncand_p, cons
                              const uint32_t* unmerged, cudaStream_t st);
 cudaError_t launch_fix_prefix_fused(const uint32_t* states, const uint32_t* cand, const uint32_t* ncand_p,
                                     const uint32_t* merged, const uint32_t* srank_p, const uint32_t* inv,
-                                    uint32_t* chunk_ends, uint32_t* err, cudaStream_t st);
+                                    uint32_t poison, uint32_t* chunk_ends, uint32_t* err, cudaStream_t st);
+cudaError_t launch_map_error(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, uint32_t code, cudaStream_t st);
 cudaError_t launch_set_u32(uint32_t* p, uint32_t v, uint32_t* p2, uint32_t v2, cudaStream_t st);
 cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_t* grp,
                              const unsigned long long* prefix, const uint32_t* pfinal, const unsigned long long* pcount,
@@ -360,7 +362,7 @@ struct fsm_s {
   // sharded runs (state kept between fsm_shard_map and fsm_shard_finish)
   void* shard_base = nullptr;   // device scratch of the shard steps
   size_t shard_bytes = 0;
-  int shard_mode = -1;          // 0 fused/single path, 1 enum, 2 multi-path, 3 fused with cand[0]
+  int shard_mode = -1;          // 0 fused/single path, 1 enum, 2 multi-path, 3 fused with cand[0], 4 map failed
   uint64_t shard_ticket = 0;
   uint32_t last_nstamp = 0;            // verify phase timestamps of the last collected run
   uint64_t last_stamp[24] = {};
@@ -368,6 +370,9 @@ struct fsm_s {
   void* batch_base = nullptr;            // fsm_run_batch scratch (offsets, chunk bases, records, totals)
   size_t batch_bytes = 0;
   cudaEvent_t batch_ev[2] = {nullptr, nullptr};
+  void* multi_base = nullptr;            // fsm_run_multi scratch when this handle is fsms[0] (its device)
+  size_t multi_cap = 0;
+  cudaEvent_t multi_ev[2] = {nullptr, nullptr};
   const uint8_t* shard_in = nullptr;
   uint64_t shard_len = 0;
   uint32_t shard_ncand = 0, shard_nj = 0;  // candidates; chunks covered by the fused prefix

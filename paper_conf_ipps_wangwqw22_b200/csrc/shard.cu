@@ -166,10 +166,11 @@ __global__ void k_map_fused(const uint32_t* __restrict__ cand, const uint32_t* _
 __global__ void k_fix_prefix_fused(const uint32_t* __restrict__ states, const uint32_t* __restrict__ cand,
                                    const uint32_t* __restrict__ ncand_p, const uint32_t* __restrict__ merged,
                                    const uint32_t* __restrict__ srank_p, const uint32_t* __restrict__ inv,
-                                   uint32_t* __restrict__ chunk_ends, uint32_t* __restrict__ err) {
+                                   uint32_t poison, uint32_t* __restrict__ chunk_ends, uint32_t* __restrict__ err) {
   __shared__ uint32_t ci;
   if (srank_p[2] != 0) return;  // the composition failed (e.g. an invalid speculative map): nothing to fix
   const uint32_t ncand = *ncand_p, sr = *srank_p;
+  if (sr == poison) return;  // an invalid byte before this shard: the run reports FSM_ESYMBOL
   if (threadIdx.x == 0) ci = kNoState;
   __syncthreads();
   for (uint32_t i = threadIdx.x; i < ncand; i += blockDim.x)
@@ -192,10 +193,23 @@ __global__ void k_set_u32(uint32_t* p, uint32_t v, uint32_t* p2, uint32_t v2) {
   if (p2) *p2 = v2;
 }
 
+// every entry "not a candidate", except the poison state (transformed id nt - 1), which
+// is absorbing and non-accepting (R4): poison -> poison with count 0 on every shard, so
+// an invalid byte in an earlier shard composes to the poison final state (FSM_ESYMBOL)
 __global__ void k_map_init(uint32_t* __restrict__ mend, unsigned long long* __restrict__ mcnt, uint32_t nt) {
   for (uint32_t s = blockIdx.x * blockDim.x + threadIdx.x; s < nt; s += gridDim.x * blockDim.x) {
-    mend[s] = kNoState;
+    mend[s] = s == nt - 1 ? s : kNoState;
     mcnt[s] = 0;
+  }
+}
+
+// the map of a rank whose fsm_shard_map failed: the exchange still runs (every rank
+// reaches the collective) and every rank's composition reports the failure
+__global__ void k_map_error(uint32_t* __restrict__ mend, unsigned long long* __restrict__ mcnt, uint32_t nt,
+                            uint32_t code) {
+  for (uint32_t s = blockIdx.x * blockDim.x + threadIdx.x; s < nt; s += gridDim.x * blockDim.x) {
+    mend[s] = kErrorMap;
+    mcnt[s] = s == 0 ? code : 0ull;
   }
 }
 
@@ -240,6 +254,14 @@ __global__ void k_compose(const uint8_t* __restrict__ maps_g, uint32_t G, uint64
     const uint32_t* me = reinterpret_cast<const uint32_t*>(maps + h * map_bytes);
     const unsigned long long* mc = reinterpret_cast<const unsigned long long*>(maps + h * map_bytes + cnt_off);
     const uint32_t e = me[s];
+    if (e == kErrorMap) {  // rank h's fsm_shard_map failed: report its status and rank
+      out[0] = q0t;
+      out[1] = q0t;
+      out[2] = 3;
+      out[3] = (uint32_t)mc[0];
+      out[4] = h;
+      return;
+    }
     if (e == kNoState) { err = 1; break; }
     if (e == kInvalidMap) { err = 2; break; }  // a rank's speculative map must be redone
     c += mc[s];
@@ -320,8 +342,8 @@ cudaError_t launch_map_fused(const uint32_t* cand, const uint32_t* ncand_p, cons
 
 cudaError_t launch_fix_prefix_fused(const uint32_t* states, const uint32_t* cand, const uint32_t* ncand_p,
                                     const uint32_t* merged, const uint32_t* srank_p, const uint32_t* inv,
-                                    uint32_t* chunk_ends, uint32_t* err, cudaStream_t st) {
-  k_fix_prefix_fused<<<1, 256, 0, st>>>(states, cand, ncand_p, merged, srank_p, inv, chunk_ends, err);
+                                    uint32_t poison, uint32_t* chunk_ends, uint32_t* err, cudaStream_t st) {
+  k_fix_prefix_fused<<<1, 256, 0, st>>>(states, cand, ncand_p, merged, srank_p, inv, poison, chunk_ends, err);
   return cudaGetLastError();
 }
 
@@ -332,6 +354,11 @@ cudaError_t launch_set_u32(uint32_t* p, uint32_t v, uint32_t* p2, uint32_t v2, c
 
 cudaError_t launch_map_init(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, cudaStream_t st) {
   k_map_init<<<(nt + 255) / 256, 256, 0, st>>>(mend, mcnt, nt);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_map_error(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, uint32_t code, cudaStream_t st) {
+  k_map_error<<<(nt + 255) / 256, 256, 0, st>>>(mend, mcnt, nt, code);
   return cudaGetLastError();
 }
 

@@ -81,7 +81,10 @@ __device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, u
 // (rs.task_chunk / rs.task_start, ntask entries, listed by the verification pass) is
 // cut into groups of 32 tasks, one per lane; each stage gathers the 32 chunks' next
 // 64 B with 8 TMA gather4 loads (tmap is then the {64 B x 1 row} gather map), so a
-// round walks only the chunks that have a task.  Each task appends its record to VR^end.
+// round walks only the chunks that have a task.  Entries [0, nA) are A-tasks (must-do
+// + SRE rear tasks: record to VR^end, the chunk's end moves); entries from nA on are
+// RR / NF helper tasks (Alg. 4 L23-27, Alg. 5 L19-21): record to VR^others at the
+// helper's precomputed ring position (oth_base[c] + task_j), nothing else changes.
 template <int MODE, int KP, int S, bool TASKS>
 __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
                                                     RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off,
@@ -96,10 +99,12 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   uint32_t* prow = reinterpret_cast<uint32_t*>(bars + ((nwarps * S + 1) & ~1u)) + warp * 32;  // TASKS: producer group's chunks
   stage_table(img, table);  // load-time data: staged before the dependency wait
   pdl_wait();                // the previous kernel in the stream (e.g. the last run's verify) is done
+  uint64_t nA = 0;  // TASKS: entries [0, nA) of the list are A-tasks, the rest helpers
   if (TASKS) {  // device-driven dense round: the task list and frontier come from the control block
     if (!__ldcg(&ctl->dense_pending)) return;  // the verify launch before us handed no round over
     ntask = __ldcg(reinterpret_cast<const unsigned long long*>(&ctl->ntask[0]));
     f2 = __ldcg(reinterpret_cast<const unsigned long long*>(&ctl->fmin));
+    nA = __ldcg(reinterpret_cast<const unsigned long long*>(&ctl->nA));
   }
   if (rp.ctl_init && blockIdx.x == 0) {
     init_ctl(rp.ctl_init, q0_of(rp), rp.N);
@@ -127,7 +132,9 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
     }
   } stamp_end{rp.stamps != 0 && rp.ctl_init != nullptr && !TASKS, rp.ctl_init, lane};
   const uint64_t my_tiles = (ntiles - gw + tw - 1) / tw;
-  uint64_t n_mustdo = 0, n_sre = 0;
+  uint64_t n_mustdo = 0, n_sre = 0, n_hel = 0;
+  bool helper = false;  // TASKS: this lane's task is a helper (VR^others)
+  uint32_t hslot = 0;   // ... and its ring position in VR^others
   const uint64_t items = my_tiles * segs;  // (tile, segment) pairs streamed by this warp
   uint8_t* wst = stages + (size_t)warp * S * kStageBytes;
   uint64_t* wbar = bars + warp * S;
@@ -170,10 +177,18 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
     if (sg == 0) {  // new tile: predict this lane's chunk start (lookback-2 pair table)
       c = (tile0 + gw + tile_i * tw) * 32 + lane;
       if (TASKS) {  // c = this lane's task index until the chunk is known
+        const uint64_t tix = c;
         const uint32_t tc = c < ntask ? __ldcg(rs.task_chunk + c) : 0xFFFFFFFFu;
         const uint32_t ts = (tc < n_full && tc >= f2) ? __ldcg(rs.task_start + c) : 0xFFFFFFFFu;
         c = tc;
         kc = ts != 0xFFFFFFFFu;  // 0: no task for this lane (walks a row's bytes, writes nothing)
+        helper = tix >= nA;
+        if (helper && kc) {
+          const uint32_t j = __ldcg(rs.task_j + tix);
+          // FIFO in task order (R16): a later helper of this round on the same chunk that
+          // lands in the same ring slot evicts this record -> it is not stored (kNone)
+          hslot = j + rp.vr_oth >= __ldcg(rs.hcnt + tc) ? (__ldcg(rs.oth_base + tc) + j) % rp.vr_oth : 0xFFFFFFFFu;
+        }
 #pragma unroll
         for (int p = 0; p < KP; p++) st[p] = kc ? ts : q0_of(rp);
       } else if (c == 0 || c >= n_full) {
@@ -240,7 +255,16 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
     }
     __syncwarp();
     if (it + S < items) issue_next();  // refill this stage
-    if (TASKS && sg == segs - 1 && c < n_full && kc) {  // dense task done: append to VR^end
+    if (TASKS && sg == segs - 1 && c < n_full && kc && helper) {  // helper done: append to VR^others
+      if (hslot != 0xFFFFFFFFu) {
+        const uint64_t o = (uint64_t)(kVrMax + hslot) * rs.cap + c;
+        __stcg(rs.start + o, st[0]);
+        __stcg(rs.end + o, Sx::tid(img, code[0]));
+        __stcg(rs.cnt + o, acc[0]);
+      }
+      n_hel++;
+    }
+    if (TASKS && sg == segs - 1 && c < n_full && kc && !helper) {  // dense task done: append to VR^end
       const uint32_t e = Sx::tid(img, code[0]);
       const uint32_t ne = __ldcg(rs.n_end + c);
       const uint64_t o = (uint64_t)(ne % rp.vr_end) * rs.cap + c;
@@ -282,13 +306,16 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
     for (int o = 16; o > 0; o >>= 1) {
       n_mustdo += __shfl_down_sync(0xffffffffu, n_mustdo, o);
       n_sre += __shfl_down_sync(0xffffffffu, n_sre, o);
+      n_hel += __shfl_down_sync(0xffffffffu, n_hel, o);
     }
-    if (lane == 0 && n_mustdo + n_sre) {
+    if (lane == 0 && n_mustdo + n_sre + n_hel) {
       atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_mustdo), (unsigned long long)n_mustdo);
       atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_sre), (unsigned long long)n_sre);
-      atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->active_sum), (unsigned long long)(n_mustdo + n_sre));
+      if (n_hel) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_helper), (unsigned long long)n_hel);
+      atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->active_sum),
+                (unsigned long long)(n_mustdo + n_sre + n_hel));
       atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->reread_bytes),
-                (unsigned long long)((n_mustdo + n_sre) * rp.B));
+                (unsigned long long)((n_mustdo + n_sre + n_hel) * rp.B));
     }
   }
 }

@@ -618,6 +618,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         if (rp.dense_slots > 0) {  // a task kernel is queued behind us: hand the round over
           if (b == 0 && threadIdx.x == 0) {
             vctl->ntask[0] = nt;  // the task list's length (this pass's slot) for the task kernel
+            vctl->nA = nt;        // every entry is an A-task (no helpers)
             vctl->dense_pending = 1;
           }
           return;
@@ -793,6 +794,27 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       }
     }
     grid.sync();
+    // RR / NF dense round: the slot list [0, nA + I) (A-tasks, then one helper per idle
+    // worker, kNone where a worker found no candidate) goes to the TMA task kernel queued
+    // behind us, like SRE's dense rounds.  The per-chunk helper bookkeeping that E does
+    // after its walks (VR^others counts, QS cursors) is committed here first; the task
+    // kernel writes each helper record at its precomputed ring slot oth_base[c] + j.
+    if (helpers && rp.dense && rp.dense_slots > 0) {
+      const uint64_t nslots = nA + I;
+      if (nslots >= 2048 && nslots * 16 >= N - f2) {
+        for (uint64_t c = max(lo, f2 + 1) + threadIdx.x; c < hi; c += kBS) {
+          const uint32_t h = __ldcg(rs.hcnt + c);
+          if (h) st_cg(rs.n_oth + c, ld_cg(rs.n_oth + c) + h);
+          rs.next_qs[c] = __ldcg(rs.next_new + c);
+        }
+        if (b == 0 && threadIdx.x == 0) {
+          vctl->ntask[0] = nslots;
+          vctl->nA = nA;
+          vctl->dense_pending = 1;
+        }
+        return;
+      }
+    }
     // ---------------- E: execute all tasks, append records --------------------
     {
       const uint64_t nslots = nA + (helpers ? I : 0);
@@ -817,10 +839,14 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
           if (c == f2) mustdo++; else sre++;
         } else {  // VR^others: helper record (Fig. 5 (2))
           const uint32_t j = __ldcg(rs.task_j + s);
-          const uint64_t o = (uint64_t)(kVrMax + (ld_cg(rs.oth_base + c) + j) % rp.vr_oth) * rs.cap + c;
-          st_cg(rs.start + o, st);
-          st_cg(rs.end + o, e);
-          st_cg(rs.cnt + o, cnt);
+          // FIFO in task order (R16): a record that a later helper of this round evicts
+          // again (same ring slot) is not stored — the slot's last writer is the survivor
+          if (j + rp.vr_oth >= __ldcg(rs.hcnt + c)) {
+            const uint64_t o = (uint64_t)(kVrMax + (ld_cg(rs.oth_base + c) + j) % rp.vr_oth) * rs.cap + c;
+            st_cg(rs.start + o, st);
+            st_cg(rs.end + o, e);
+            st_cg(rs.cnt + o, cnt);
+          }
           hel++;
         }
       }
@@ -960,21 +986,59 @@ cudaError_t launch_m(const DevImage& img, const RunParams& rp, const RecStore& r
 // After the TMA task kernel: the partial tail chunk's task (if any), then commit
 // the round (Alg. 3 L14: the frontier advances to f2).  The table is staged only
 // when a chunk is left to walk (a stream whose length is a multiple of B has none).
+// RR / NF rounds: helper tasks of the list (entries >= nA) whose chunk is the partial tail
+// are walked here too (records to VR^others at their precomputed ring slots).
 template <int MODE>
 __global__ void __launch_bounds__(256) k_dense_finish(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
                                                       uint64_t c_first_generic) {
   extern __shared__ __align__(1024) uint8_t smem[];
   __shared__ uint32_t any;
+  __shared__ uint32_t nh;
+  __shared__ uint32_t hslot[64];
   if (!ctl->dense_pending) return;  // no dense round was handed over (spare slot)
   const uint64_t f2 = ctl->fmin;
+  const uint64_t ntask = ctl->ntask[0], nA = ctl->nA;
   if (threadIdx.x == 0) {
     any = 0;
+    nh = 0;
     for (uint64_t c = max(c_first_generic, f2); c < rp.N && !any; c++) any = __ldcg(rs.tstart + c) != 0xFFFFFFFFu;
+  }
+  __syncthreads();
+  if (c_first_generic < rp.N && ntask > nA) {  // helpers on the tail chunk(s): find their slots
+    for (uint64_t s = nA + threadIdx.x; s < ntask; s += blockDim.x) {
+      const uint32_t c = __ldcg(rs.task_chunk + s);
+      if (c != kNone && c >= c_first_generic) {
+        const uint32_t i = atomicAdd(&nh, 1u);
+        if (i < 64) hslot[i] = (uint32_t)s;
+      }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && nh) any = 1;
   }
   __syncthreads();
   if (any) stage_table(img, smem);
   __syncthreads();
   if (threadIdx.x != 0) return;
+  // (one partial tail chunk has <= qs_cap <= 16 helpers; more only if the task kernel
+  // walked nothing — then every helper of the list is visited here, in list order)
+  const uint64_t nvisit = nh <= 64 ? nh : ntask - nA;
+  for (uint64_t i = 0; i < nvisit; i++) {
+    const uint64_t s = nh <= 64 ? hslot[i] : nA + i;
+    const uint32_t c = __ldcg(rs.task_chunk + s), st = __ldcg(rs.task_start + s);
+    if (c == kNone || c < c_first_generic) continue;
+    uint32_t e, cnt;
+    task_walk<MODE>(img, smem, rp, rs, c, st, &e, &cnt);
+    const uint32_t j = __ldcg(rs.task_j + s);
+    if (j + rp.vr_oth >= __ldcg(rs.hcnt + c)) {  // evicted again by a later helper of the round: not stored
+      const uint64_t o = (uint64_t)(kVrMax + (ld_cg(rs.oth_base + c) + j) % rp.vr_oth) * rs.cap + c;
+      st_cg(rs.start + o, st);
+      st_cg(rs.end + o, e);
+      st_cg(rs.cnt + o, cnt);
+    }
+    ctl->tasks_helper++;
+    ctl->active_sum++;
+    ctl->reread_bytes += min((uint64_t)rp.B, rp.len - (uint64_t)c * rp.B);
+  }
   for (uint64_t c = max(c_first_generic, f2); any && c < rp.N; c++) {
     const uint32_t st = __ldcg(rs.tstart + c);
     if (st == 0xFFFFFFFFu) continue;

@@ -54,22 +54,28 @@ def _all_gather_cat(t, group=None):
 
 
 def exchange_lookback(shard, group=None, L: int = 2):
-    """Each rank receives the last L bytes of the previous rank's shard (tiny allgather)."""
+    """The last L (<= 16) bytes of the stream before this rank's shard (tiny allgather of
+    every rank's tail).  They come from the nearest preceding non-empty shards: a shard
+    shorter than L (or empty, when there are fewer chunks than ranks) contributes what it
+    has and the ranks before it the rest.  Empty only for a shard that starts the stream."""
     import torch
     import torch.distributed as dist
 
+    assert 0 < L <= 16
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
     tail = torch.zeros(17, dtype=torch.uint8, device=shard.device)
-    n = min(L, shard.numel(), 16)
+    n = min(L, shard.numel())
     if n:
         tail[16 - n:16] = shard[shard.numel() - n:]
     tail[16] = n
-    tails = _all_gather_cat(tail, group).view(world, 17)
-    if rank == 0:
-        return tail[:0]
-    m = int(tails[rank - 1, 16].item())
-    return tails[rank - 1, 16 - m:16].contiguous()
+    tails = _all_gather_cat(tail, group).view(world, 17).cpu()
+    parts = []
+    for r in range(rank):
+        m = int(tails[r, 16].item())
+        parts.append(tails[r, 16 - m:16])
+    before = torch.cat(parts) if parts else tail[:0].cpu()
+    return before[max(0, before.numel() - L):].contiguous().to(shard.device)
 
 
 def run_sharded(fsm: FSM, shard, lookback, group=None, scheme="auto", chunk_bytes=4096, spec_k=0,
@@ -88,15 +94,19 @@ def run_sharded(fsm: FSM, shard, lookback, group=None, scheme="auto", chunk_byte
     lb = lookback if lookback is not None and lookback.numel() else None
     for exact in (False, True):  # speculative map first; FSM_EAGAIN is seen by every rank alike
         fn = _lib.fsm_shard_map_exact if exact else _lib.fsm_shard_map
-        _check(fn(fsm.handle, shard.data_ptr() if shard.numel() else None, shard.numel(),
-                  lb.data_ptr() if lb is not None else None, lb.numel() if lb is not None else 0,
-                  ctypes.byref(o), local.data_ptr(), ce.data_ptr() if ce is not None else None), "fsm_shard_map")
+        map_rc = fn(fsm.handle, shard.data_ptr() if shard.numel() else None, shard.numel(),
+                    lb.data_ptr() if lb is not None else None, lb.numel() if lb is not None else 0,
+                    ctypes.byref(o), local.data_ptr(), ce.data_ptr() if ce is not None else None)
+        # a failed map is published as an error map (every rank's finish reports it), so
+        # this rank still joins the collective the others are waiting in
         gathered = _all_gather_cat(local, group)  # the single data-path collective
         r = fsm_result()
         rc = _lib.fsm_shard_finish(fsm.handle, gathered.data_ptr(), world, rank, ctypes.byref(o),
                                    ce.data_ptr() if ce is not None else None, ctypes.byref(r))
-        if rc != FSM_EAGAIN:
-            break
+        if rc == FSM_EAGAIN:
+            continue
+        _check(map_rc, "fsm_shard_map")
+        break
     _check(rc, "fsm_shard_finish")
     return Result.from_c(r, ce[:n] if ce is not None else None)
 
@@ -116,19 +126,3 @@ def unpack_map(buf: np.ndarray, nt: int):
     off, total = map_layout(nt)
     b = np.ascontiguousarray(buf[:total])
     return b[:nt * 4].view(np.uint32), b[off:off + nt * 8].view(np.uint64)
-
-
-def compose_maps_host(maps: np.ndarray, nt: int, q0t: int):
-    """s_0 = q0; s_{g+1} = M_g[s_g]; count = sum_g C_g[s_g].  Returns (starts[G+1], count)."""
-    G = maps.shape[0]
-    s = q0t
-    starts = [s]
-    total = 0
-    for g in range(G):
-        e, c = unpack_map(maps[g], nt)
-        if int(e[s]) == NO_STATE:
-            raise RuntimeError(f"shard {g}: start state {s} not in its candidate set")
-        total += int(c[s])
-        s = int(e[s])
-        starts.append(s)
-    return starts, total

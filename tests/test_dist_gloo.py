@@ -44,10 +44,25 @@ def oracle_shard_map(w, data, lo, hi, B):
     return pack_map(end, cnt), perm, inv
 
 
+def compose_maps(maps, nt, q0t):
+    """Test-side composition of the gathered maps (the library's is k_compose, shard.cu):
+    s_0 = q0; s_{g+1} = M_g[s_g]; count = sum_g C_g[s_g]."""
+    from paper_conf_ipps_wangwqw22_b200.dist import NO_STATE, unpack_map
+
+    s, total, starts = q0t, 0, [q0t]
+    for g in range(maps.shape[0]):
+        e, c = unpack_map(maps[g], nt)
+        assert int(e[s]) != NO_STATE, f"shard {g}: start state {s} not in its candidate set"
+        total += int(c[s])
+        s = int(e[s])
+        starts.append(s)
+    return starts, total
+
+
 def _worker(rank, world, port, name, length, B, q):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    from paper_conf_ipps_wangwqw22_b200.dist import compose_maps_host, shard_bounds
+    from paper_conf_ipps_wangwqw22_b200.dist import shard_bounds
 
     w = gen.workload(name, length=length)
     data = w.host()
@@ -57,7 +72,7 @@ def _worker(rank, world, port, name, length, B, q):
     gathered = [torch.empty_like(local) for _ in range(world)]
     dist.all_gather(gathered, local)  # the single data-path collective
     maps = torch.stack(gathered).numpy()
-    starts, count = compose_maps_host(maps, w.nstates + 1, int(perm[w.start]))
+    starts, count = compose_maps(maps, w.nstates + 1, int(perm[w.start]))
     q.put((rank, int(inv[starts[-1]]), count, int(inv[starts[rank]]), lo))
     dist.barrier()
     dist.destroy_process_group()
@@ -101,3 +116,44 @@ def test_shard_bounds_and_wire_format():
     assert len(buf) == map_layout(3)[1]
     e, c = unpack_map(buf, 3)
     assert (e == end).all() and (c == cnt).all()
+
+
+def _lb_worker(rank, world, port, data, bounds, L, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_wangwqw22_b200.dist import exchange_lookback
+
+    lo, hi = bounds[rank]
+    lb = exchange_lookback(torch.from_numpy(data[lo:hi].copy()), L=L)
+    q.put((rank, lb.numpy().tobytes()))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("L", [2, 5])
+@pytest.mark.parametrize("layout", ["bounds", "ragged"])
+def test_exchange_lookback_empty_shards(L, layout):
+    """Fewer chunks than ranks: some shards are empty (and some shorter than L); every
+    rank still receives the L bytes just before its shard."""
+    from paper_conf_ipps_wangwqw22_b200.dist import shard_bounds
+
+    world, B = 8, 16
+    data = np.arange(5 * B - 3, dtype=np.uint8)  # 5 chunks over 8 ranks
+    if layout == "bounds":
+        bounds = [shard_bounds(len(data), world, r, B) for r in range(world)]
+    else:  # contiguous, with empty and 1-byte shards
+        cuts = [0, 0, 3, 3, 4, 20, 20, 21, len(data)]
+        bounds = list(zip(cuts[:-1], cuts[1:]))
+    assert any(lo == hi and lo > 0 for lo, hi in bounds)
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_lb_worker, args=(r, world, port, data, bounds, L, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    outs = dict(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for r, (lo, hi) in enumerate(bounds):
+        assert outs[r] == data[max(0, lo - L):lo].tobytes(), (r, lo)

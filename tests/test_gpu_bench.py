@@ -1,0 +1,41 @@
+"""bench.py's own launch paths on one GPU: the C5 line (per-DFA sharded runs) at N = 1 and,
+with ranks sharing cuda:0 over gloo, at N = 2 through bench.py's self-relaunch under
+torch.distributed.run (the driver's 8-GPU run uses the same code with NCCL)."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _bench(*args, env=None):
+    e = dict(os.environ)
+    e.update(env or {})
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py")] + list(args), capture_output=True, text=True,
+                         timeout=900, env=e, cwd=ROOT)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout[-2000:]
+    return json.loads(lines[0])
+
+
+@pytest.mark.parametrize("gpus", [1, 2])
+def test_bench_c5_line(gpus):
+    import gen
+    import oracle
+
+    L = 64 << 20
+    d = _bench("--config", "c5", "--gpus", str(gpus), "--steps", "2", "--warmup", "3", "--c5-bytes", str(L),
+               env={"GSPEC_DIST_BACKEND": "gloo"} if gpus > 1 else None)
+    assert d["n_gpus"] == gpus and d["scaling"] == "strong" and d["config"]["workload"] == "c5"
+    assert set(d["per_dfa"]) == {"c1", "c2", "c3", "c4"}
+    for name, r in d["per_dfa"].items():
+        assert r["value"] > 0 and r["ranks_agree"]
+        w = gen.workload(name, length=L)
+        ref = oracle.run(w.table, w.start, w.accept, w.host(), 4096)
+        assert r["final_state"] == ref["final"] and r["accept_count"] == ref["count"], name
+        assert r["scheme"] == {"c1": "enum", "c2": "sre", "c3": "sre", "c4": "sre"}[name]

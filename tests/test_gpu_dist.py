@@ -64,3 +64,47 @@ def test_run_sharded_multi_rank(name, length, world):
         assert fin == ref["final"] and cnt == ref["count"]
     ce_all = np.concatenate([o[4] for o in outs])
     assert (ce_all == ref["chunk_end"]).all()
+
+
+def _fail_worker(rank, world, port, q):
+    import torch.distributed as dist
+
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import paper_conf_ipps_wangwqw22_b200 as gs
+    from paper_conf_ipps_wangwqw22_b200.dist import run_sharded, shard_bounds
+
+    torch.cuda.set_device(0)
+    w = gen.workload("c2", length=3 << 20)
+    lo, hi = shard_bounds(w.length, world, rank)
+    x = torch.empty(hi - lo, dtype=torch.uint8, device="cuda")
+    w.device(x, offset=lo)
+    lb = torch.zeros(17 if rank == 1 else (2 if rank else 0), dtype=torch.uint8, device="cuda")  # rank 1: bad
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    try:
+        run_sharded(fsm, x, lb)
+        q.put((rank, 0))
+    except gs.GSpecError as e:
+        q.put((rank, e.status))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_run_sharded_failed_rank_is_collective():
+    """One rank's fsm_shard_map fails: it publishes an error map and still joins the
+    allgather, so every rank raises the same status instead of hanging."""
+    import paper_conf_ipps_wangwqw22_b200 as gs
+    import torch.multiprocessing as mp
+
+    world = 3
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _port()
+    ps = [ctx.Process(target=_fail_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in ps:
+        p.start()
+    outs = dict(q.get(timeout=600) for _ in range(world))
+    for p in ps:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    assert outs == {r: gs.FSM_EINVAL for r in range(world)}

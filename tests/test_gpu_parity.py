@@ -272,22 +272,31 @@ def test_async_queue(gs):
         fsm.wait(runs[0][0])  # already collected
 
 
-@pytest.mark.parametrize("name,length,B,scheme", [("c3", 32 << 20, 4096, "sre"), ("c3", (24 << 20) + 1000, 4096, "sre"),
-                                                  ("c3s", 160 << 20, 8192, "sre"), ("c3", 32 << 20, 4096, "cse")])
-def test_dense_recovery_rounds(gs, name, length, B, scheme):
-    """SRE (and CSE's SRE rounds) on a low-accuracy DFA: rounds where many chunks
-    re-execute go to the TMA-gather task kernel over the round's task list; results
-    and round diagnostics stay identical."""
+@pytest.mark.parametrize("name,length,B,scheme,vr_oth", [
+    ("c3", 32 << 20, 4096, "sre", 16), ("c3", (24 << 20) + 1000, 4096, "sre", 16), ("c3s", 160 << 20, 8192, "sre", 16),
+    ("c3", 32 << 20, 4096, "cse", 16), ("c3", 32 << 20, 4096, "rr", 16), ("c3", 32 << 20, 4096, "nf", 16),
+    ("c3", (24 << 20) + 1000, 4096, "rr", 16), ("c3", (24 << 20) + 1000, 4096, "nf", 2),
+    ("c3s", 160 << 20, 8192, "nf", 16), ("c3", 16 << 20, 4096, "nf", 1)])
+def test_dense_recovery_rounds(gs, name, length, B, scheme, vr_oth):
+    """SRE / RR / NF (and CSE's SRE rounds) on a low-accuracy DFA: rounds where many
+    chunks re-execute go to the TMA-gather task kernel over the round's task list (RR /
+    NF: A-tasks to VR^end, helpers to VR^others at their precomputed ring slots); results
+    and round diagnostics stay identical to the oracle's, twice in a row (the second run
+    queues as many task-kernel slots as the first used)."""
     w, data = _wl(name, length)
     ref = oracle.run(w.table, w.start, w.accept, data, B)
     fsm = gs.FSM.load(w.table, w.start, w.accept)
-    res = fsm.run(torch.from_numpy(data).cuda(), scheme=scheme, chunk_bytes=B)
-    check_equal(res, ref, B, w.nstates)
-    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme=scheme)
-    for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks",
-              "verify_matches"):
-        assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme=scheme, vr_oth=vr_oth)
+    x = torch.from_numpy(data).cuda()
+    for _ in range(2):
+        res = fsm.run(x, scheme=scheme, chunk_bytes=B, vr_others=vr_oth)
+        check_equal(res, ref, B, w.nstates)
+        for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks",
+                  "verify_matches"):
+            assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
     assert res.stats["tasks_sre"] > 2048  # the dense path really ran
+    if scheme in ("rr", "nf"):
+        assert res.stats["tasks_helper"] > 2048
 
 
 @pytest.mark.parametrize("name,length,B", [("c1", 1 << 20, 4096), ("c2", 4 << 20, 16384), ("c3", 2 << 20, 8192),

@@ -99,3 +99,87 @@ def test_library_nccl_single_rank(gs):
     assert r.final_state == ref["final"] and r.accept_count == ref["count"]
     assert (r.chunk_ends.cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
     comm.close()
+
+
+def _maps_and_finish(gs, w, x, G, scheme="auto", B=4096, bad_rank=None, exact=False):
+    """Fake-collective round returning the raw status codes: (map rcs, finish rcs, results,
+    chunk ends).  bad_rank passes an over-long lookback (17 bytes -> FSM_EINVAL)."""
+    import ctypes
+
+    from paper_conf_ipps_wangwqw22_b200 import _lib, _run_opts, fsm_result
+    from paper_conf_ipps_wangwqw22_b200.dist import shard_bounds
+
+    L = x.numel()
+    fsms = [gs.FSM.load(w.table, w.start, w.accept) for _ in range(G)]
+    mb = fsms[0].map_bytes()
+    maps = torch.zeros(G * mb, dtype=torch.uint8, device="cuda")
+    o = _run_opts(scheme, B)
+    ce_all = torch.full((max(1, gs.fsm_num_chunks(L, B)),), -1, dtype=torch.int32, device="cuda")
+    map_rc, fin_rc, outs = [], [], []
+    for attempt in range(2):
+        map_rc = []
+        for g in range(G):
+            lo, hi = shard_bounds(L, G, g, B)
+            lbn = 17 if g == bad_rank else (2 if g else 0)
+            lb = x[max(0, lo - lbn):lo] if g else None
+            fn = _lib.fsm_shard_map_exact if (exact or attempt) else _lib.fsm_shard_map
+            map_rc.append(fn(fsms[g].handle, x[lo:].data_ptr() if hi > lo else None, hi - lo,
+                             lb.data_ptr() if lb is not None else None, lbn, ctypes.byref(o),
+                             maps[g * mb:].data_ptr(), ce_all[lo // B:].data_ptr()))
+        fin_rc, outs = [], []
+        for g in range(G):
+            r = fsm_result()
+            fin_rc.append(_lib.fsm_shard_finish(fsms[g].handle, maps.data_ptr(), G, g, ctypes.byref(o),
+                                                ce_all[shard_bounds(L, G, g, B)[0] // B:].data_ptr(), ctypes.byref(r)))
+            outs.append(r)
+        if fin_rc[0] != -7:
+            break
+    return map_rc, fin_rc, outs, ce_all
+
+
+def test_invalid_symbol_in_earlier_shard(gs):
+    """An invalid byte (>= nsyms, R4) inside shard 0 of 3: the poison state is a fixed
+    entry of every map, so every rank's composition reaches it and reports FSM_ESYMBOL,
+    as fsm_run does on one GPU."""
+    w = gen.workload("rand:50:7:3", length=3 * 64 * 4096)
+    data = w.host()
+    data[1000] = 9  # nsyms = 7
+    x = torch.from_numpy(data).cuda()
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    with pytest.raises(gs.GSpecError) as e:
+        fsm.run(x, scheme="sre")
+    assert e.value.status == gs.FSM_ESYMBOL
+    for exact in (False, True):
+        map_rc, fin_rc, _, _ = _maps_and_finish(gs, w, x, 3, scheme="sre", exact=exact)
+        assert map_rc == [0, 0, 0]
+        assert fin_rc == [gs.FSM_ESYMBOL] * 3, fin_rc
+
+
+def test_failed_map_is_collective(gs):
+    """A rank whose fsm_shard_map fails publishes an error map; every rank's finish
+    returns that rank's status (nobody is left waiting in the exchange)."""
+    w = gen.workload("c2", length=6 << 20)
+    x = torch.from_numpy(w.host()).cuda()
+    map_rc, fin_rc, _, _ = _maps_and_finish(gs, w, x, 3, scheme="sre", bad_rank=1)
+    assert map_rc[1] == gs.FSM_EINVAL and map_rc[0] == 0 and map_rc[2] == 0
+    assert fin_rc == [gs.FSM_EINVAL] * 3, fin_rc
+
+
+@pytest.mark.parametrize("n,G", [(100, 3), (40, 2)])
+def test_many_nonmerging_paths(gs, n, G):
+    """A non-convergent DFA above the ENUM limit (permutation columns, n = 100: 100
+    candidate paths that never merge) shards exactly (one pipeline per surviving path)."""
+    rng = np.random.default_rng(n)
+    t = np.stack([rng.permutation(n) for _ in range(3)], axis=1).astype(np.uint32)
+    a = (rng.random(n) < 0.5).astype(np.uint8)
+    data = rng.integers(0, 3, 24 * 4096 + 77).astype(np.uint8)
+    ref = oracle.run(t, 0, a, data, 4096)
+
+    class W:
+        table, start, accept = t, 0, a
+
+    map_rc, fin_rc, outs, ce = _maps_and_finish(gs, W, torch.from_numpy(data).cuda(), G, scheme="sre")
+    assert map_rc == [0] * G and fin_rc == [0] * G, (map_rc, fin_rc)
+    for r in outs:
+        assert r.final_state == ref["final"] and r.accept_count == ref["count"]
+    assert (ce[:len(ref["chunk_end"])].cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
