@@ -58,6 +58,8 @@ def lib():
                                   P, ctypes.POINTER(SimResult), P, U64, P]
         L.or_simulate_literal_sre.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, U32, P,
                                               ctypes.POINTER(SimResult)]
+        L.or_simulate_literal.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, ctypes.c_int, U32, U32, P,
+                                          ctypes.POINTER(SimResult), P, U64, P]
         L.or_features_compute.argtypes = [P, U32, U32, U32, P, P, U64, U32, U32, U32, ctypes.POINTER(Features)]
         L.or_select.argtypes = [ctypes.POINTER(Features), U32]
         _LIB = L
@@ -214,6 +216,29 @@ def simulate_literal_sre(table, start, accept, data, B=4096, vr_cap=16, policy=0
     out = res.as_dict()
     out["status"] = rc
     out["chunk_end"] = ce[:nchunks(d.size, B)]
+    return out
+
+
+def simulate_literal(table, start, accept, data, B=4096, scheme="rr", qs_cap=16, vr_cap=16, policy=0,
+                     max_tasks=0):
+    """Paper-literal SRE / RR / NF (Alg. 3 / 4 / 5 verbatim, N iterations)."""
+    perm, inv, _, tt, acc = transform(table, accept, policy, data if policy == 1 else None, start)
+    t = _c(table, np.uint32)
+    n, ns = t.shape
+    d = _c(data, np.uint8)
+    ce = np.zeros(max(1, nchunks(d.size, B)), np.uint32)
+    res = SimResult()
+    tasks = (Task * max(1, max_tasks))()
+    nt = U64(0)
+    rc = lib().or_simulate_literal(tt.ctypes.data, n, ns, int(perm[start]), acc.ctypes.data, inv.ctypes.data,
+                                   d.ctypes.data, d.size, B, SCHEME_IDS[scheme], qs_cap, vr_cap, ce.ctypes.data,
+                                   ctypes.byref(res), tasks, max_tasks, ctypes.byref(nt))
+    out = res.as_dict()
+    out["status"] = rc
+    out["chunk_end"] = ce[:nchunks(d.size, B)]
+    out["tasks"] = [(tasks[i].round, tasks[i].chunk, tasks[i].start, tasks[i].kind)
+                    for i in range(min(nt.value, max_tasks))]
+    out["perm"] = perm
     return out
 
 

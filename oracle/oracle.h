@@ -105,6 +105,15 @@ int or_simulate_literal_sre(const uint32_t* tt, uint32_t nt, uint32_t nsyms, uin
                             const uint32_t* inv, const uint8_t* in, uint64_t len, uint32_t B, uint32_t vr_cap,
                             uint32_t* chunk_end, or_sim_result* res);
 
+/* Paper-literal RR (Alg. 4) and NF (Alg. 5) — and SRE (Alg. 3)
+ * through the same loop: N iterations of Alg. 3's frontier step, the recovery step of
+ * the chosen algorithm when mark == false.  Per-iteration task log (nullable):
+ * tasks[i] = {iteration, chunk, start, kind 0 must-do / 1 rear / 2 helper}. */
+int or_simulate_literal(const uint32_t* tt, uint32_t nt, uint32_t nsyms, uint32_t q0t, const uint8_t* acc_t,
+                        const uint32_t* inv, const uint8_t* in, uint64_t len, uint32_t B, int scheme,
+                        uint32_t qs_cap, uint32_t vr_cap, uint32_t* chunk_end, or_sim_result* res, or_task* tasks,
+                        uint64_t max_tasks, uint64_t* ntasks);
+
 typedef struct {
   double acc1, acck, sens, uniq10;
 } or_features;

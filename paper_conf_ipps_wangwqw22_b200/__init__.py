@@ -229,10 +229,10 @@ class FSM:
         _check(_lib.fsm_wait(self._h, ticket, ctypes.byref(r)), "fsm_wait")
         return Result.from_c(r)
 
-    def run_literal(self, x, chunk_bytes=4096, vr_end=16, stream=None) -> Result:
-        """fsm_run_literal: the paper-literal single-CTA SRE kernel (Alg. 2 L2-6 + Alg. 3
-        verbatim, <= 1024 chunks) on a uint8 CUDA tensor."""
-        o = _run_opts("sre", chunk_bytes, vr_end=vr_end, stream=stream)
+    def run_literal(self, x, chunk_bytes=4096, vr_end=16, scheme="sre", qs_cap=16, stream=None) -> Result:
+        """fsm_run_literal: the paper-literal single-CTA kernel (Alg. 2 L2-6 + Alg. 3 SRE /
+        Alg. 4 RR / Alg. 5 NF verbatim, <= 1024 chunks) on a uint8 CUDA tensor."""
+        o = _run_opts(scheme, chunk_bytes, qs_cap=qs_cap, vr_end=vr_end, stream=stream)
         n = fsm_num_chunks(x.numel(), chunk_bytes)
         import torch
 

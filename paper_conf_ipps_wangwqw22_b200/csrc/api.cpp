@@ -12,6 +12,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "gspec.h"
 #include "internal.h"
 
@@ -61,6 +63,21 @@ void entry_clear(const char* name) {
   static const bool dbg = getenv("GSPEC_DEBUG_ERR") != nullptr;
   if (e != cudaSuccess && dbg) fprintf(stderr, "gspec: stale CUDA error at %s entry: %s\n", name, cudaGetErrorString(e));
 }
+
+// One NVTX range per C-ABI call (tracing: nsys / ncu --nvtx show which entry point and
+// phase enqueued each kernel); NVTX v3 is header-only and a no-op without a tool attached.
+struct ApiScope {
+  explicit ApiScope(const char* name) {
+    entry_clear(name);
+    nvtxRangePushA(name);
+  }
+  ~ApiScope() { nvtxRangePop(); }
+};
+
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 constexpr uint32_t kRow8Bytes = 260;  // walk.cuh kRow8: row r starts at bank (r * 65) % 32 = r % 32
 
@@ -182,6 +199,7 @@ int ensure_records(fsm_t f, uint64_t N) {
     r.next_qs = take(cap);
     r.found = take(cap);
     r.ulen = take(cap);
+    r.upos = take(cap * kQsMax);
     r.next_new = take(cap);
     r.hcnt = take(cap);
     return off;
@@ -291,6 +309,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       CUDA_TRY(cudaMemset(f->enum_ticket, 0, 256));
     }
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
+    NvtxRange nv_("enum (walk + composition scan)");
     if (small) {
       CUDA_TRY(launch_enum_small(f->img, rp, E, f->enum_base, f->enum_ticket, d_chunk_ends, f->d_ctl, o.st));
       pd.launches = 1;
@@ -315,7 +334,10 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     rp.dense = ((scheme == FSM_SCHEME_SRE || scheme == FSM_SCHEME_CSE || scheme == FSM_SCHEME_RR ||
                  scheme == FSM_SCHEME_NF) && len / o.B > 0 && o.B % 64 == 0 &&
                 (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0 && f->acc1_hint < 0.5) ? 1u : 0u;
-    CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
+    {
+      NvtxRange nv_("speculative execution (round 0)");
+      CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
+    }
     {  // TMA kernel over the full chunks + the generic kernel for a tail chunk (or everything)
       const bool tma = !spec_path_generic_only() && len / o.B > 0 && o.B % 64 == 0 &&
                        (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0;
@@ -329,6 +351,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     // the run completed return at once.  No host round trip: runs stay queued back to back.
     const uint32_t slots = rp.dense ? f->dense_hint : 0;
     rp.dense_slots = slots;
+    NvtxRange nv_("verification + recovery (+ dense-round slots)");
     CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
     pd.launches++;
     for (uint32_t r = 0; r < slots; r++) {
@@ -530,7 +553,7 @@ uint64_t fsm_num_chunks(uint64_t len, uint32_t chunk_bytes) {
 
 int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, const uint8_t* accept,
              const fsm_load_opts* opts, fsm_t* out) {
-  entry_clear("fsm_load");
+  ApiScope api_scope_("fsm_load");
   if (!table || !accept || !out) return fail(FSM_EINVAL, "NULL table/accept/out");
   if (n == 0 || nsyms == 0 || nsyms > 256 || start >= n) return fail(FSM_EINVAL, "bad nstates/nsyms/start");
   if (n >= (1u << 24)) return fail(FSM_EUNSUPPORTED, "nstates >= 2^24");
@@ -763,7 +786,7 @@ void fsm_free(fsm_t f) {
 
 int fsm_run(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts, uint32_t* d_chunk_ends,
             fsm_result* out) {
-  entry_clear("fsm_run");
+  ApiScope api_scope_("fsm_run");
   if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
   if (!d_input && len > 0) return fail(FSM_EINVAL, "NULL input");
   Opts o;
@@ -795,7 +818,7 @@ int fsm_run(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* o
 
 int fsm_run_async(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts, uint32_t* d_chunk_ends,
                   uint64_t* ticket) {
-  entry_clear("fsm_run_async");
+  ApiScope api_scope_("fsm_run_async");
   if (!f || !ticket) return fail(FSM_EINVAL, "NULL handle/ticket");
   if (!d_input && len > 0) return fail(FSM_EINVAL, "NULL input");
   Opts o;
@@ -817,7 +840,7 @@ int fsm_run_async(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_o
 }
 
 int fsm_wait(fsm_t f, uint64_t ticket, fsm_result* out) {
-  entry_clear("fsm_wait");
+  ApiScope api_scope_("fsm_wait");
   if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
   fsm_result r;
   uint32_t fin = 0;
@@ -842,7 +865,7 @@ uint64_t fsm_batch_chunks(const uint64_t* h_offsets, uint32_t nstreams, uint32_t
 int fsm_run_batch(fsm_t f, const uint8_t* d_input, const uint64_t* h_offsets, uint32_t nstreams,
                   const fsm_run_opts* opts, uint32_t* d_final, uint64_t* d_count, uint32_t* d_chunk_ends,
                   fsm_batch_result* out) {
-  entry_clear("fsm_run_batch");
+  ApiScope api_scope_("fsm_run_batch");
   if (!f || !out || !h_offsets) return fail(FSM_EINVAL, "NULL handle/offsets/out");
   std::memset(out, 0, sizeof(*out));
   if (nstreams == 0) return FSM_OK;
@@ -904,7 +927,7 @@ int fsm_run_batch(fsm_t f, const uint8_t* d_input, const uint64_t* h_offsets, ui
 
 int fsm_run_multi(const fsm_t* fsms, uint32_t npairs, const uint8_t* const* d_inputs, const uint64_t* lens,
                   const fsm_run_opts* opts, uint32_t* h_final, uint64_t* h_count, fsm_multi_result* out) {
-  entry_clear("fsm_run_multi");
+  ApiScope api_scope_("fsm_run_multi");
   if (out) std::memset(out, 0, sizeof(*out));
   if (npairs == 0) return FSM_OK;
   if (!fsms || !d_inputs || !lens || !h_final || !h_count) return fail(FSM_EINVAL, "NULL argument");
@@ -996,7 +1019,7 @@ int fsm_run_multi(const fsm_t* fsms, uint32_t npairs, const uint8_t* const* d_in
 
 int fsm_run_literal(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
                     uint32_t* d_chunk_ends, fsm_result* out) {
-  entry_clear("fsm_run_literal");
+  ApiScope api_scope_("fsm_run_literal");
   if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
   if (!d_input && len > 0) return fail(FSM_EINVAL, "NULL input");
   Opts o;
@@ -1004,9 +1027,13 @@ int fsm_run_literal(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run
   if (rc) return rc;
   const uint64_t N = fsm_num_chunks(len, o.B);
   if (N > literal_max_chunks()) return fail(FSM_EUNSUPPORTED, "paper-literal kernel: at most 1024 chunks (one CTA)");
+  // SRE (Alg. 3, the default for AUTO), RR (Alg. 4) or NF (Alg. 5)
+  const fsm_scheme lscheme = (o.scheme == FSM_SCHEME_RR || o.scheme == FSM_SCHEME_NF) ? o.scheme : FSM_SCHEME_SRE;
+  if (o.scheme != FSM_SCHEME_AUTO && o.scheme != lscheme)
+    return fail(FSM_EUNSUPPORTED, "paper-literal kernel: SRE, RR or NF (Alg. 3-5)");
   std::memset(out, 0, sizeof(*out));
   out->nchunks = N;
-  out->scheme_used = FSM_SCHEME_SRE;
+  out->scheme_used = lscheme;
   uint32_t fin = f->img.q0t;
   if (N) {
     if ((rc = ensure_ctl(f))) return rc;
@@ -1018,8 +1045,9 @@ int fsm_run_literal(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run
     rp.len = len;
     rp.B = o.B;
     rp.N = N;
-    rp.scheme = FSM_SCHEME_SRE;
+    rp.scheme = lscheme;
     rp.k = 1;
+    rp.qs_cap = o.qs_cap;
     rp.vr_end = o.vr_end;
     rp.vr_oth = o.vr_oth;
     for (auto& e : f->batch_ev)
@@ -1048,7 +1076,7 @@ int fsm_run_literal(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run
 
 int fsm_run_host(fsm_t f, const uint8_t* h_input, uint64_t len, const fsm_run_opts* opts, uint32_t* h_chunk_ends,
                  fsm_result* out) {
-  entry_clear("fsm_run_host");
+  ApiScope api_scope_("fsm_run_host");
   if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
   if (!h_input && len > 0) return fail(FSM_EINVAL, "NULL input");
   Opts o;
@@ -1081,7 +1109,7 @@ int fsm_run_host(fsm_t f, const uint8_t* h_input, uint64_t len, const fsm_run_op
 
 int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_run_opts* opts, fsm_scheme* outp,
                       fsm_features* feat) {
-  entry_clear("fsm_select_scheme");
+  ApiScope api_scope_("fsm_select_scheme");
   if (!f || !outp) return fail(FSM_EINVAL, "NULL handle/out");
   if (!d_sample && len > 0) return fail(FSM_EINVAL, "NULL sample");
   Opts o;
@@ -1283,14 +1311,14 @@ int shard_map_impl(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t*
 
 int fsm_shard_map(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
                   const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local) {
-  entry_clear("fsm_shard_map");
+  ApiScope api_scope_("fsm_shard_map");
   return shard_map_impl(f, d_shard, len, d_lookback, lb_len, opts, d_map, d_chunk_ends_local,
                         f && f->shard_prefer_exact);
 }
 
 int fsm_shard_map_exact(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t* d_lookback, uint32_t lb_len,
                         const fsm_run_opts* opts, void* d_map, uint32_t* d_chunk_ends_local) {
-  entry_clear("fsm_shard_map_exact");
+  ApiScope api_scope_("fsm_shard_map_exact");
   return shard_map_impl(f, d_shard, len, d_lookback, lb_len, opts, d_map, d_chunk_ends_local, true);
 }
 
@@ -1468,7 +1496,7 @@ int shard_map_body(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t*
 
 int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, const fsm_run_opts* opts,
                      uint32_t* d_chunk_ends_local, fsm_result* out) {
-  entry_clear("fsm_shard_finish");
+  ApiScope api_scope_("fsm_shard_finish");
   if (!f || !d_maps || !out || rank >= G) return fail(FSM_EINVAL, "bad finish arguments");
   if (f->shard_mode < 0) return fail(FSM_EINVAL, "fsm_shard_map was not called");
   Opts o;

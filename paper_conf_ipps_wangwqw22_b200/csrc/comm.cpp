@@ -5,6 +5,7 @@
 // sharded method is one ncclAllGather of the per-shard state maps.
 #include <dlfcn.h>
 #include <nccl.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <cstring>
 #include <mutex>
@@ -116,7 +117,9 @@ int fsm_run_sharded(fsm_t f, fsm_comm_t c, const uint8_t* d_shard, uint64_t shar
     // still runs, so no rank waits in the allgather for one that returned early
     if (rc && f->shard_mode != 4) return rc;
     const int map_rc = rc;
+    nvtxRangePushA("ncclAllGather (shard maps)");
     ncclResult_t r = nccl().allGather(c->d_local, c->d_all, mb, ncclUint8, c->comm, st);
+    nvtxRangePop();
     if (r != ncclSuccess)
       return gspec_set_error(FSM_ENCCL, nccl().getErrorString ? nccl().getErrorString(r) : "ncclAllGather");
     rc = fsm_shard_finish(f, c->d_all, (uint32_t)c->nranks, (uint32_t)c->rank, opts, d_chunk_ends_local, out_global);

@@ -88,6 +88,7 @@ struct RecStore {
   uint8_t* found;      // [cap]
   // per-round scratch of the verify/recover kernel
   uint8_t* ulen;       // [cap] untried QS candidates of chunk c
+  uint8_t* upos;       // [cap][kQsMax] their QS positions (phase T), for H2 and the cursor
   uint8_t* next_new;   // [cap] QS cursor after this round's helpers
   uint8_t* hcnt;       // [cap] helpers assigned to chunk c this round
   uint32_t* prefU;     // [cap] NF: exclusive prefix of ulen over c > f

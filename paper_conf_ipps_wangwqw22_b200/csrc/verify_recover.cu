@@ -178,22 +178,29 @@ __device__ __forceinline__ bool vr_lookup_cached(const VrCache& v, uint32_t i, c
   return false;
 }
 
-// Untried QS candidates of chunk c (Alg. 4 L24, Alg. 5 L30-32): QS_c entries
-// past the cursor that are neither in dom VR_c nor this round's task start.
-__device__ uint32_t untried(const DevImage& img, const RunParams& rp, const RecStore& rs, uint64_t c,
-                            bool busy, uint32_t tstart, uint32_t want_j, uint32_t* q_out, uint32_t* pos_out) {
+// Untried QS candidates of chunk c (Alg. 4 L24, Alg. 5 L30-32): QS_c entries past the
+// cursor that are neither in dom VR_c nor this round's task start.  Computed once per
+// round (phase T): the chunk's record starts (VR^end then VR^others ring) are read once,
+// QS_c is scanned against them, and the QS positions of the untried candidates are kept
+// in rs.upos[c][0..m) for the helper assignment (H2) and the cursor update.
+__device__ uint32_t untried_scan(const DevImage& img, const RunParams& rp, const RecStore& rs, uint64_t c, bool busy,
+                                 uint32_t tstart) {
   const uint32_t pair = qs_pair(img, rp.in, c, rp.B);
   const uint32_t ql = min((uint32_t)__ldg(img.qs2_len + pair), rp.qs_cap);
   const uint32_t nx = __ldcg(rs.next_qs + c);
-  uint32_t m = 0, e;
+  if (nx >= ql) return 0;
+  const uint32_t ne = min(ld_cg(rs.n_end + c), rp.vr_end), no = min(ld_cg(rs.n_oth + c), rp.vr_oth);
+  uint32_t rec[2 * kVrMax];
+  for (uint32_t i = 0; i < ne; i++) rec[i] = ld_cg(rs.start + (uint64_t)i * rs.cap + c);
+  for (uint32_t i = 0; i < no; i++) rec[ne + i] = ld_cg(rs.start + (uint64_t)(kVrMax + i) * rs.cap + c);
+  uint32_t m = 0;
   for (uint32_t j = nx; j < ql; j++) {
     const uint32_t q = __ldg(img.qs2 + (uint64_t)pair * kQsMax + j);
     if (busy && q == tstart) continue;
-    if (vr_lookup(rs, rp.vr_end, rp.vr_oth, c, q, &e, nullptr)) continue;
-    if (m == want_j) {
-      if (q_out) *q_out = q;
-      if (pos_out) *pos_out = j;
-    }
+    bool in = false;
+    for (uint32_t i = 0; i < ne + no; i++) in |= rec[i] == q;
+    if (in) continue;
+    rs.upos[c * kQsMax + m] = (uint8_t)j;
     m++;
   }
   return m;
@@ -677,7 +684,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         const bool busy = (c == f2) || (sre_like && c > f2 && !__ldcg(rs.found + c));
         cA += busy;
         if (helpers && c > f2) {
-          const uint32_t u = untried(img, rp, rs, c, busy, busy ? ld_cg(rs.x + c) : 0, kNone, nullptr, nullptr);
+          const uint32_t u = untried_scan(img, rp, rs, c, busy, busy ? ld_cg(rs.x + c) : 0);
           rs.ulen[c] = (uint8_t)u;
           cU += u;
         }
@@ -757,12 +764,10 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
             j = (uint32_t)(k - ld_cg(rs.prefU + c));
             ok = j < __ldcg(rs.ulen + c);
           }
-          if (ok) {
-            const bool busy = !__ldcg(rs.found + c);  // c > f2: busy iff SRE task
-            uint32_t q = 0;
-            untried(img, rp, rs, c, busy, busy ? ld_cg(rs.x + c) : 0, j, &q, nullptr);
+          if (ok) {  // the j-th untried candidate of chunk c (positions listed in phase T)
+            const uint32_t pair = qs_pair(img, rp.in, c, rp.B);
             cid = (uint32_t)c;
-            st = q;
+            st = __ldg(img.qs2 + (uint64_t)pair * kQsMax + __ldcg(rs.upos + c * kQsMax + j));
           }
         }
         rs.task_chunk[nA + k] = cid;
@@ -782,12 +787,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
           h = I > p ? min((uint64_t)ul, I - p) : 0;
         }
         uint8_t nx = __ldcg(rs.next_qs + c);
-        if (h > 0) {
-          const bool busy = !__ldcg(rs.found + c);
-          uint32_t pos = 0;
-          untried(img, rp, rs, c, busy, busy ? ld_cg(rs.x + c) : 0, (uint32_t)(h - 1), nullptr, &pos);
-          nx = (uint8_t)(pos + 1);
-        }
+        if (h > 0) nx = (uint8_t)(__ldcg(rs.upos + c * kQsMax + (h - 1)) + 1);  // past the last tried
         rs.next_new[c] = nx;
         rs.oth_base[c] = ld_cg(rs.n_oth + c);
         rs.hcnt[c] = (uint8_t)h;

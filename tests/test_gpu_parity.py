@@ -325,6 +325,29 @@ def test_paper_literal_sre(gs, name, length, B):
             fsm.run_literal(torch.from_numpy(bad).cuda(), chunk_bytes=B)
 
 
+@pytest.mark.parametrize("name,length,B", [("c1", 1 << 18, 1024), ("c3", 2 << 20, 8192), ("c2", (1 << 20) + 77, 2048),
+                                           ("c4", 2 << 20, 4096), ("rand:40:7:3", 60000, 64), ("rand:200:30:5", 30000, 48)])
+@pytest.mark.parametrize("scheme", ["rr", "nf"])
+def test_paper_literal_rr_nf(gs, name, length, B, scheme):
+    """Paper-literal Alg. 4 (RR) / Alg. 5 (NF) single-CTA kernels: bit-exact
+    results, and the per-iteration accounting (must-do, rear re-executions, helpers,
+    re-read bytes, checks, matches) equal to the oracle's literal simulation."""
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    fsm = _fsm(gs, w)
+    for vr in (16, 2):
+        res = fsm.run_literal(torch.from_numpy(data).cuda(), chunk_bytes=B, scheme=scheme, vr_end=vr)
+        assert res.scheme == scheme
+        assert res.final_state == ref["final"] and res.accept_count == ref["count"]
+        assert (res.chunk_ends.cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
+        sim = oracle.simulate_literal(w.table, w.start, w.accept, data, B, scheme=scheme, vr_cap=vr)
+        for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks",
+                  "verify_matches"):
+            assert res.stats[k] == sim[k], (k, vr, res.stats[k], sim[k])
+    if name.startswith("rand") or name == "c3":
+        assert res.stats["tasks_helper"] > 0
+
+
 @pytest.mark.parametrize("scheme,B", [("cse", 64), ("cse", 16), ("rr", 64), ("nf", 256)])
 def test_chained_verification_passes(gs, scheme, B):
     """div7 with several records per chunk: non-convergent chains that a chaotic pass

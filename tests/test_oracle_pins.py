@@ -416,6 +416,70 @@ def test_simulate_literal_sre(seed):
     assert o["rounds"] == 0 and o["accept_count"] == len(d1)
 
 
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("scheme", ["sre", "rr", "nf"])
+def test_simulate_literal_rr_nf(seed, scheme):
+    """Paper-literal Alg. 3 / 4 / 5 on random DFAs and chunkings:
+    * results equal the sequential run (P:89, P:334);
+    * N iterations with N checks each; one must-do per iteration whose frontier missed;
+    * the literal SRE loop equals the separate literal-SRE simulator exactly;
+    * RR: at most 1 + ceil((i-1)/(T-i)) threads work on a chunk in an iteration with
+      frontier i (P:195, 1-indexed; here i = fr + 1, T = N);
+    * NF: helpers fill QS_{f+1} before QS_{f+2}: in every iteration the helper
+      targets are non-decreasing in tid order and every chunk before the last targeted
+      one gets all its remaining candidates (counted from the lookback ranking, whose
+      ranking is pinned above, and the dequeues logged in earlier iterations)."""
+    rng = random.Random(seed * 13 + 5)
+    n, ns = rng.randint(2, 24), rng.randint(2, 5)
+    t, s, a = gen.dfa_random(seed + 41, n, ns)
+    data = gen.workload(f"rand:{n}:{ns}:{seed}", length=rng.randint(1, 6000), seed=seed + 3).host()
+    perm, inv, _, tt, acc = oracle.transform(t, a)
+    for B in (16, 48, 256):
+        vr_cap = rng.randint(1, 16)
+        r = oracle.run(t, s, a, data, B)
+        o = oracle.simulate_literal(t, s, a, data, B, scheme=scheme, vr_cap=vr_cap, max_tasks=1 << 20)
+        N = oracle.nchunks(len(data), B)
+        assert o["status"] == 0
+        assert o["final_state"] == r["final"] and o["accept_count"] == r["count"]
+        assert (o["chunk_end"] == r["chunk_end"]).all()
+        assert o["verify_checks"] == N * N and o["rounds"] == o["tasks_mustdo"] <= N
+        assert o["tasks_total"] == o["tasks_mustdo"] + o["tasks_sre"] + o["tasks_helper"] == len(o["tasks"])
+        if scheme == "sre":
+            ls = oracle.simulate_literal_sre(t, s, a, data, B, vr_cap=vr_cap)
+            for k in ("rounds", "tasks_total", "tasks_mustdo", "tasks_sre", "reread_bytes", "verify_checks",
+                      "verify_matches", "accept_count"):
+                assert o[k] == ls[k], k
+            assert o["tasks_helper"] == 0
+            continue
+        qlen = [1] + [len(oracle.lookback(tt, n, data[c * B - 2:c * B], K=16)[0]) for c in range(1, N)]
+        taken = [1] * N  # round 0 ran QS.front()
+        by_it = {}
+        for it, cid, st, kind in o["tasks"]:
+            by_it.setdefault(it, []).append((cid, st, kind))
+        for it, ts in sorted(by_it.items()):
+            fr = [cid for cid, _, k in ts if k == 0]
+            assert len(fr) == 1
+            fr = fr[0]
+            per = {}
+            for cid, _, _ in ts:
+                per[cid] = per.get(cid, 0) + 1
+            if scheme == "rr" and N - fr - 1 > 0:
+                bound = 1 + -(-fr // (N - fr - 1))
+                assert max(per.values()) <= bound
+            helpers = [cid for cid, _, k in ts if k == 2]
+            assert all(h > fr for h in helpers)
+            if scheme == "nf":
+                assert helpers == sorted(helpers)
+                if helpers:
+                    last = helpers[-1]
+                    for d in range(fr + 1, last):
+                        assert helpers.count(d) == qlen[d] - taken[d], (it, d)
+                    assert len(helpers) == min(fr, sum(qlen[d] - taken[d] for d in range(fr + 1, N)))
+            for h in helpers:
+                taken[h] += 1
+            assert all(taken[d] <= qlen[d] for d in range(N))
+
+
 def test_simulate_invalid_symbol():
     t, s, a = gen.dfa_div7()
     data = np.array([1, 0, 1] * 100 + [3] + [1] * 50, np.uint8)
