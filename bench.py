@@ -307,6 +307,24 @@ def measure_single(gs, w, x, args, fsm, scheme, with_clocks=True):
             "result": res}
 
 
+def spread_profile(w, total_len):
+    """The selector's profile of a stream of total_len bytes (reading R20, as
+    fsm_select_scheme builds it from a long trace): 8 portions of 128 KiB spread evenly
+    from the start to the end of the stream, generated on the device from their global
+    offsets (so every rank of a sharded run profiles the same global portions)."""
+    import torch
+
+    S = 128 << 10
+    buf = torch.empty(8 * S, dtype=torch.uint8, device="cuda")
+    if total_len <= 8 * S:
+        buf = buf[:total_len]
+        w.device(buf, offset=0)
+        return buf
+    for i in range(8):
+        w.device(buf[i * S:(i + 1) * S], offset=(i * (total_len - S) // 7) & ~4095)
+    return buf
+
+
 def _table_info(fsm):
     try:
         tr = fsm.transform()
@@ -328,7 +346,7 @@ def per_dfa_result(gs, name, args, peak, peak_kind, with_cpu=True):
     prof = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")
     w.device(prof, offset=w.length)
     fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof.cpu().numpy())
-    scheme, feats = fsm.select_scheme(prof, chunk_bytes=args.chunk_bytes)
+    scheme, feats = fsm.select_scheme(x, chunk_bytes=args.chunk_bytes)  # spread profile (R20)
     m = measure_single(gs, w, x, args, fsm, scheme, with_clocks=False)
     out = {"value": round(m["value"], 3), "unit": "GB/s", "ms_per_step": round(m["ms"], 4),
            "bytes": w.length, "scheme": scheme, "nstates": int(w.nstates),
@@ -386,9 +404,9 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         if lo:
             w.device(lb, offset=lo - 2)  # the 2 bytes before the shard (pure function of the offset)
         fsm = gs.FSM.load(w.table, w.start, w.accept)
-        # selector per DFA (offline profiling): every rank profiles the stream's first MiB
-        prof = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")
-        w.device(prof, offset=0)
+        # selector per DFA (offline profiling): every rank profiles the same 8 spread
+        # portions of the global stream (R20), so every rank picks the same scheme
+        prof = spread_profile(w, L)
         scheme, feats = fsm.select_scheme(prof, chunk_bytes=B)
         del prof
 
@@ -534,9 +552,11 @@ def main():
     fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof.cpu().numpy())
     scheme = args.scheme
     feats = None
-    if scheme == "auto":
-        scheme, feats = fsm.select_scheme(prof, chunk_bytes=B)  # offline profiling, untimed
     del prof
+    if scheme == "auto":  # offline profiling, untimed: 8 spread portions of the stream (R20)
+        sp = spread_profile(w, length * world)
+        scheme, feats = fsm.select_scheme(sp, chunk_bytes=B)
+        del sp
 
     lb = None
     if world > 1:

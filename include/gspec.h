@@ -53,12 +53,20 @@ typedef enum {
   FSM_SCHEME_RR = 4,   /* Alg. 4: SRE + round-robin helpers over QS              */
   FSM_SCHEME_NF = 5,   /* Alg. 5: SRE + nearest-first helpers over QS            */
   FSM_SCHEME_ENUM = 6, /* enumerative: all-state chunk maps + composition scan  */
-  FSM_SCHEME_CSE = 7   /* convergence-set enumeration (P:300, P:427 [21][24]):
+  FSM_SCHEME_CSE = 7,  /* convergence-set enumeration (P:300, P:427 [21][24]):
                           round 0 walks every lookback-2 candidate of each chunk up to
                           spec_k (default 8) — the whole image, which contains the true
                           start, whenever it has <= spec_k states — with path fusion
                           (paths that meet are walked once); SRE rounds recover what a
                           capped image missed.  Not chosen by FSM_SCHEME_AUTO. */
+  FSM_SCHEME_PM_TREE = 8 /* faithful PM as published (Xia et al.; Fig. 2, Eq. 2
+                          P:266-268): spec-k, ceil(log2 N) rounds of parallel
+                          tree-like merging of k-entry chunk maps where a mismatch marks
+                          the path invalid (delayed recovery), then a sequential stage from
+                          q0 over the merged segments that recovers a chunk at once when
+                          its incoming state has no valid record.  The paper's comparison
+                          baseline (Fig. 8 "PM spec-4"); FSM_SCHEME_PM is the B200 reading
+                          R17 chosen by the selector.  Not chosen by FSM_SCHEME_AUTO. */
 } fsm_scheme;
 
 typedef struct fsm_s* fsm_t;
@@ -102,6 +110,11 @@ typedef struct {
   double avg_active_workers; /* mean active workers per round (Table III analogue)    */
   double ms_spec, ms_verify; /* device time of speculative execution / verify+recover */
   uint32_t kernel_launches;  /* kernels this run launched (spec, verify, dense rounds, ENUM levels) */
+  /* FSM_SCHEME_PM_TREE only (0 otherwise): stage-1 entry lookups, entries marked invalid
+   * (delayed recoveries), stage-2 segments taken through their merged maps.  For that
+   * scheme rounds = merge rounds, tasks_mustdo = stage-2 recoveries, verify_checks =
+   * stage-2 steps, verify_matches = stage-2 jumps. */
+  uint64_t pm_merge_checks, pm_invalid_marks, pm_jumps;
 } fsm_result;
 
 typedef struct {
@@ -207,7 +220,11 @@ int fsm_run_host(fsm_t fsm, const uint8_t* h_input, uint64_t len, const fsm_run_
 /* Scheme selector: profile the device sample (the paper uses a
  * 1 MB trace), compute the features, walk the decision tree (Fig. 6,
  * reconstructed: DESIGN.md R19) and cache the choice for FSM_SCHEME_AUTO.
- * feat nullable. */
+ * A sample longer than 1 MiB (e.g. the whole stream) is profiled on 8 portions
+ * of 128 KiB spread evenly over it — portion i at floor(i (len - 128 KiB) / 7)
+ * rounded down to 4 KiB — gathered into one 1 MiB sample (reading R20: input
+ * sensitivity compares "different portions").  FSM_SCHEME_AUTO without a
+ * cached choice profiles the run's own input this way.  feat nullable. */
 int fsm_select_scheme(fsm_t fsm, const uint8_t* d_sample, uint64_t len, const fsm_run_opts* opts,
                       fsm_scheme* out, fsm_features* feat);
 

@@ -36,6 +36,11 @@ class Task(ctypes.Structure):
     _fields_ = [("round", U32), ("chunk", U32), ("start", U32), ("kind", U32)]
 
 
+class PmStats(ctypes.Structure):
+    _fields_ = [("levels", U32), ("merge_checks", U64), ("invalid_marks", U64), ("jumps", U64),
+                ("recoveries", U64), ("reread_bytes", U64)]
+
+
 class Features(ctypes.Structure):
     _fields_ = [("acc1", ctypes.c_double), ("acck", ctypes.c_double), ("sens", ctypes.c_double),
                 ("uniq10", ctypes.c_double)]
@@ -60,6 +65,8 @@ def lib():
                                               ctypes.POINTER(SimResult)]
         L.or_simulate_literal.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, ctypes.c_int, U32, U32, P,
                                           ctypes.POINTER(SimResult), P, U64, P]
+        L.or_simulate_pm_tree.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, U32, U32, P,
+                                          ctypes.POINTER(SimResult), ctypes.POINTER(PmStats)]
         L.or_features_compute.argtypes = [P, U32, U32, U32, P, P, U64, U32, U32, U32, ctypes.POINTER(Features)]
         L.or_select.argtypes = [ctypes.POINTER(Features), U32]
         _LIB = L
@@ -239,6 +246,24 @@ def simulate_literal(table, start, accept, data, B=4096, scheme="rr", qs_cap=16,
     out["tasks"] = [(tasks[i].round, tasks[i].chunk, tasks[i].start, tasks[i].kind)
                     for i in range(min(nt.value, max_tasks))]
     out["perm"] = perm
+    return out
+
+
+def simulate_pm_tree(table, start, accept, data, B=4096, k=4, qs_cap=16, policy=0):
+    """Faithful PM (Eq. 2): spec-k, tree merge with delayed recovery, sequential stage 2."""
+    perm, inv, _, tt, acc = transform(table, accept, policy, data if policy == 1 else None, start)
+    t = _c(table, np.uint32)
+    n, ns = t.shape
+    d = _c(data, np.uint8)
+    ce = np.zeros(max(1, nchunks(d.size, B)), np.uint32)
+    res, pm = SimResult(), PmStats()
+    rc = lib().or_simulate_pm_tree(tt.ctypes.data, n, ns, int(perm[start]), acc.ctypes.data, inv.ctypes.data,
+                                   d.ctypes.data, d.size, B, k, qs_cap, ce.ctypes.data, ctypes.byref(res),
+                                   ctypes.byref(pm))
+    out = res.as_dict()
+    out.update({"pm_" + k_: getattr(pm, k_) for k_, _ in PmStats._fields_})
+    out["status"] = rc
+    out["chunk_end"] = ce[:nchunks(d.size, B)]
     return out
 
 

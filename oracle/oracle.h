@@ -114,6 +114,25 @@ int or_simulate_literal(const uint32_t* tt, uint32_t nt, uint32_t nsyms, uint32_
                         uint32_t qs_cap, uint32_t vr_cap, uint32_t* chunk_end, or_sim_result* res, or_task* tasks,
                         uint64_t max_tasks, uint64_t* ntasks);
 
+/* Faithful PM (Parallel Merge, Xia et al., the paper's prior state of the art; P:120-127,
+ * Fig. 2, Eq. 2).  spec-k round 0; stage 1: log N rounds of a
+ * parallel tree-like verification and merge of the chunks' k-entry maps, a mismatch
+ * marking the path invalid (delayed recovery, no re-execution); stage 2: sequential
+ * verification from q0 over the merged segments, with an immediate recovery of a chunk
+ * whose incoming state has no (valid) record.  Same outputs as or_run. */
+typedef struct {
+  uint32_t levels;          /* tree rounds = ceil(log2 N) */
+  uint64_t merge_checks;    /* left entries looked up among a right segment's starts */
+  uint64_t invalid_marks;   /* entries marked invalid by a merge (delayed recovery) */
+  uint64_t jumps;           /* stage 2: segments taken through their merged map */
+  uint64_t recoveries;      /* stage 2: must-be-done re-executions (P_i^PM events) */
+  uint64_t reread_bytes;
+} or_pm_stats;
+
+int or_simulate_pm_tree(const uint32_t* tt, uint32_t nt, uint32_t nsyms, uint32_t q0t, const uint8_t* acc_t,
+                        const uint32_t* inv, const uint8_t* in, uint64_t len, uint32_t B, uint32_t k,
+                        uint32_t qs_cap, uint32_t* chunk_end, or_sim_result* res, or_pm_stats* pm);
+
 typedef struct {
   double acc1, acck, sens, uniq10;
 } or_features;

@@ -24,7 +24,7 @@ if not os.path.exists(_LIB_PATH):
 _lib = ctypes.CDLL(_LIB_PATH)
 
 FSM_OK, FSM_EINVAL, FSM_ENOMEM, FSM_ECUDA, FSM_ESYMBOL, FSM_ENCCL, FSM_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
-SCHEMES = {"auto": 0, "seq": 1, "pm": 2, "sre": 3, "rr": 4, "nf": 5, "enum": 6, "cse": 7}
+SCHEMES = {"auto": 0, "seq": 1, "pm": 2, "sre": 3, "rr": 4, "nf": 5, "enum": 6, "cse": 7, "pm_tree": 8}
 SCHEME_NAMES = {v: k for k, v in SCHEMES.items()}
 MODES = {1: "u8", 2: "u16", 3: "u32", 4: "u16d"}
 
@@ -46,7 +46,8 @@ class fsm_result(ctypes.Structure):
                 ("scheme_used", ctypes.c_int), ("rounds", U32), ("tasks_total", U64), ("tasks_mustdo", U64),
                 ("tasks_sre", U64), ("tasks_helper", U64), ("reread_bytes", U64), ("verify_checks", U64),
                 ("verify_matches", U64), ("avg_active_workers", ctypes.c_double), ("ms_spec", ctypes.c_double),
-                ("ms_verify", ctypes.c_double), ("kernel_launches", U32)]
+                ("ms_verify", ctypes.c_double), ("kernel_launches", U32), ("pm_merge_checks", U64),
+                ("pm_invalid_marks", U64), ("pm_jumps", U64)]
 
 
 class fsm_batch_result(ctypes.Structure):

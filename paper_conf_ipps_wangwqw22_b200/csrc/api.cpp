@@ -158,7 +158,7 @@ int resolve_opts(const fsm_run_opts* o, Opts* r) {
   if (r->qs_cap < 1 || r->qs_cap > kQsMax) return fail(FSM_EINVAL, "qs_cap must be in [1,16]");
   if (r->vr_end < 1 || r->vr_end > kVrMax || r->vr_oth < 1 || r->vr_oth > kVrMax)
     return fail(FSM_EINVAL, "vr_end / vr_others must be in [1,16]");
-  if ((int)r->scheme < 0 || (int)r->scheme > FSM_SCHEME_CSE) return fail(FSM_EINVAL, "unknown scheme");
+  if ((int)r->scheme < 0 || (int)r->scheme > FSM_SCHEME_PM_TREE) return fail(FSM_EINVAL, "unknown scheme");
   return FSM_OK;
 }
 
@@ -241,7 +241,12 @@ void fill_result_stats(fsm_result* out, const Ctl& h) {
   out->verify_checks = h.verify_checks;
   out->verify_matches = h.verify_matches;
   out->avg_active_workers = h.rounds ? (double)h.active_sum / (double)h.rounds : 0.0;
+  out->pm_merge_checks = h.pm_merge_checks;
+  out->pm_invalid_marks = h.pm_invalid_marks;
+  out->pm_jumps = h.pm_jumps;
 }
+
+int select_auto(fsm_t f, const uint8_t* d_in, uint64_t len, const fsm_run_opts* opts);
 
 // Enqueue one device run over d_in[0..len) from transformed start q0t on
 // o.st; returns a ticket.  Everything (init, kernels, readback) is stream
@@ -265,7 +270,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   rp.B = o.B;
   rp.N = N;
   rp.scheme = scheme;
-  rp.k = scheme == FSM_SCHEME_PM ? o.k : scheme == FSM_SCHEME_CSE ? o.k_cse : 1;
+  rp.k = (scheme == FSM_SCHEME_PM || scheme == FSM_SCHEME_PM_TREE) ? o.k : scheme == FSM_SCHEME_CSE ? o.k_cse : 1;
   rp.qs_cap = o.qs_cap;
   rp.vr_end = o.vr_end;
   rp.vr_oth = o.vr_oth;
@@ -278,7 +283,8 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   h.tf = q0t;
   h.fmin = N;
   h.it_fm[0] = N;  // first relaxation pass slot
-  if (scheme == FSM_SCHEME_ENUM && q0_dev) scheme = FSM_SCHEME_SRE;  // device-resident start: pipeline path
+  if ((scheme == FSM_SCHEME_ENUM || scheme == FSM_SCHEME_PM_TREE) && q0_dev)
+    scheme = FSM_SCHEME_SRE;  // device-resident start: pipeline path
   if (scheme == FSM_SCHEME_ENUM) {
     if (f->n + 1 > kEnumMax) {
       pd.active = false;
@@ -321,6 +327,36 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       pd.launches = 2 + 2 * L;
     }
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
+    CUDA_TRY(cudaEventRecord(ev[2], o.st));
+  } else if (scheme == FSM_SCHEME_PM_TREE) {
+    // faithful PM (pm_tree.cu): spec-k round 0, tree merge rounds, sequential stage 2, descent
+    if (f->rs_cap < N) CUDA_TRY(cudaStreamSynchronize(o.st));
+    if ((rc = ensure_records(f, N))) return rc;
+    const size_t need = pm_tree_scratch_bytes(N, o.k, nullptr);
+    if (f->pm_bytes < need) {
+      CUDA_TRY(cudaStreamSynchronize(o.st));
+      if (f->pm_base) cudaFree(f->pm_base);
+  if (f->prof_buf) cudaFree(f->prof_buf);
+      f->pm_base = nullptr;
+      f->pm_bytes = 0;
+      CUDA_TRY(cudaMalloc(&f->pm_base, need));
+      f->pm_bytes = need;
+    }
+    rp.ctl_init = f->d_ctl;
+    CUDA_TRY(cudaEventRecord(ev[0], o.st));
+    {
+      NvtxRange nv_("speculative execution spec-k (PM round 0)");
+      CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
+    }
+    pd.launches = 1 + (len % o.B != 0 && len / o.B > 0);
+    rp.ctl_init = nullptr;
+    CUDA_TRY(cudaEventRecord(ev[1], o.st));
+    uint32_t nl = 0;
+    {
+      NvtxRange nv_("PM tree merge + sequential stage 2");
+      CUDA_TRY(launch_pm_tree(f->img, rp, f->rs, o.k, f->pm_base, f->d_ctl, d_chunk_ends, f->sm_count, o.st, &nl));
+    }
+    pd.launches += nl;
     CUDA_TRY(cudaEventRecord(ev[2], o.st));
   } else {
     if (f->rs_cap < N) CUDA_TRY(cudaStreamSynchronize(o.st));  // growing the store: drain queued runs
@@ -779,6 +815,8 @@ void fsm_free(fsm_t f) {
   for (auto& e : f->batch_ev)
     if (e) cudaEventDestroy(e);
   if (f->multi_base) cudaFree(f->multi_base);
+  if (f->pm_base) cudaFree(f->pm_base);
+  if (f->prof_buf) cudaFree(f->prof_buf);
   for (auto& e : f->multi_ev)
     if (e) cudaEventDestroy(e);
   delete f;
@@ -799,7 +837,7 @@ int fsm_run(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_opts* o
       if (opts) so = *opts;
       so.scheme = FSM_SCHEME_SRE;
       fsm_scheme pick;
-      rc = fsm_select_scheme(f, d_input, std::min<uint64_t>(len, 1ull << 20), &so, &pick, nullptr);
+      rc = select_auto(f, d_input, len, &so);
       if (rc) return rc;
     }
     scheme = f->auto_scheme;
@@ -831,7 +869,7 @@ int fsm_run_async(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run_o
       if (opts) so = *opts;
       so.scheme = FSM_SCHEME_SRE;
       fsm_scheme pick;
-      if ((rc = fsm_select_scheme(f, d_input, std::min<uint64_t>(len, 1ull << 20), &so, &pick, nullptr))) return rc;
+      if ((rc = select_auto(f, d_input, len, &so))) return rc;
     }
     scheme = f->auto_scheme;
     if (scheme == FSM_SCHEME_ENUM && f->n + 1 > kEnumMax) scheme = FSM_SCHEME_SRE;
@@ -1115,6 +1153,21 @@ int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_
   Opts o;
   int rc = resolve_opts(opts, &o);
   if (rc) return rc;
+  // Reading R20 ("a randomly selected 1 MB trace"; "similarity of speculation
+  // results over different portions"): a trace longer than 1 MiB is profiled on 8
+  // portions of 128 KiB spread evenly from its start to its end (portion i at
+  // i (len - 128 KiB) / 7, 4 KiB-aligned), gathered into one 1 MiB sample, so the
+  // input-sensitivity feature compares different portions of the stream.
+  constexpr uint64_t kSlice = 128 << 10, kSample = 8 * kSlice;
+  if (len > kSample) {
+    if (!f->prof_buf) CUDA_TRY(cudaMalloc(&f->prof_buf, kSample));
+    for (uint64_t i = 0; i < 8; i++) {
+      const uint64_t off = (i * (len - kSlice) / 7) & ~4095ull;
+      CUDA_TRY(cudaMemcpyAsync(f->prof_buf + i * kSlice, d_sample + off, kSlice, cudaMemcpyDeviceToDevice, o.st));
+    }
+    d_sample = f->prof_buf;
+    len = kSample;
+  }
   // 1. true chunk starts by an exact scheme on the sample
   fsm_result r;
   uint32_t fin = 0;
@@ -1278,7 +1331,7 @@ int resolve_scheme(fsm_t f, const uint8_t* d_in, uint64_t len, const fsm_run_opt
       if (opts) so = *opts;
       so.scheme = FSM_SCHEME_SRE;
       fsm_scheme pick;
-      int rc = fsm_select_scheme(f, d_in, std::min<uint64_t>(len, 1ull << 20), &so, &pick, nullptr);
+      int rc = select_auto(f, d_in, len, &so);
       if (rc) return rc;
     }
     scheme = f->auto_scheme;
@@ -1584,3 +1637,13 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
 }
 
 }  // extern "C"
+
+namespace {
+
+// FSM_SCHEME_AUTO: profile the stream itself (fsm_select_scheme spreads a long one).
+int select_auto(fsm_t f, const uint8_t* d_in, uint64_t len, const fsm_run_opts* opts) {
+  fsm_scheme pick;
+  return fsm_select_scheme(f, d_in, len, opts, &pick, nullptr);
+}
+
+}  // namespace

@@ -130,6 +130,8 @@ struct Ctl {
   // `dense_denied` = a verify launch ran a dense round in-kernel because the run had no
   // task-kernel slot left (the host raises its slot count for the next run)
   uint32_t finished, dense_rounds, dense_denied, pad2;
+  // FSM_SCHEME_PM_TREE (pm_tree.cu): stage-1 lookups, entries marked invalid, stage-2 jumps
+  uint64_t pm_merge_checks, pm_invalid_marks, pm_jumps;
 };
 
 struct RunParams {
@@ -290,6 +292,9 @@ cudaError_t launch_map_fused(const uint32_t* cand, const uint32_t* ncand_p, cons
 cudaError_t launch_fix_prefix_fused(const uint32_t* states, const uint32_t* cand, const uint32_t* ncand_p,
                                     const uint32_t* merged, const uint32_t* srank_p, const uint32_t* inv,
                                     uint32_t poison, uint32_t* chunk_ends, uint32_t* err, cudaStream_t st);
+uint64_t pm_tree_scratch_bytes(uint64_t N, uint32_t k, uint32_t* levels);
+cudaError_t launch_pm_tree(const DevImage& img, const RunParams& rp, const RecStore& rs, uint32_t k, void* scratch,
+                           Ctl* ctl, uint32_t* d_chunk_ends, int sms, cudaStream_t st, uint32_t* launches);
 cudaError_t launch_map_error(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, uint32_t code, cudaStream_t st);
 cudaError_t launch_set_u32(uint32_t* p, uint32_t v, uint32_t* p2, uint32_t v2, cudaStream_t st);
 cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_t* grp,
@@ -371,6 +376,9 @@ struct fsm_s {
   void* batch_base = nullptr;            // fsm_run_batch scratch (offsets, chunk bases, records, totals)
   size_t batch_bytes = 0;
   cudaEvent_t batch_ev[2] = {nullptr, nullptr};
+  uint8_t* prof_buf = nullptr;           // FSM_SCHEME_AUTO's spread 1 MiB profile sample
+  void* pm_base = nullptr;               // FSM_SCHEME_PM_TREE scratch (level maps, jump list)
+  size_t pm_bytes = 0;
   void* multi_base = nullptr;            // fsm_run_multi scratch when this handle is fsms[0] (its device)
   size_t multi_cap = 0;
   cudaEvent_t multi_ev[2] = {nullptr, nullptr};

@@ -497,3 +497,58 @@ def test_vr_others_capacity(gs, vr_others, scheme):
               "verify_matches"):
         assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
     assert res.stats["tasks_helper"] > 0
+
+
+@pytest.mark.parametrize("name,length,B,k", [("c1", 1 << 20, 4096, 4), ("c2", 4 << 20, 4096, 4),
+                                             ("c3", 2 << 20, 4096, 4), ("c4", 4 << 20, 4096, 4),
+                                             ("c2", (1 << 20) + 77, 2048, 2), ("c3s", 1 << 20, 1024, 8),
+                                             ("rand:40:7:3", 200000, 48, 4), ("rand:200:30:5", 100000, 16, 1),
+                                             ("c2", 3000, 4096, 4), ("c1", 16, 16, 4)])
+def test_pm_tree(gs, name, length, B, k):
+    """Faithful PM (FSM_SCHEME_PM_TREE): bit-exact results and every stage
+    counter (merge rounds, merge lookups, invalid marks, stage-2 jumps and recoveries,
+    re-read bytes) equal to the oracle twin or_simulate_pm_tree."""
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    fsm = _fsm(gs, w)
+    res = fsm.run(torch.from_numpy(data).cuda(), scheme="pm_tree", chunk_bytes=B, spec_k=k)
+    check_equal(res, ref, B, w.nstates)
+    assert res.scheme == "pm_tree"
+    sim = oracle.simulate_pm_tree(w.table, w.start, w.accept, data, B, k=k)
+    st = res.stats
+    pairs = [("rounds", "pm_levels"), ("tasks_mustdo", "pm_recoveries"), ("reread_bytes", "pm_reread_bytes"),
+             ("pm_merge_checks", "pm_merge_checks"), ("pm_invalid_marks", "pm_invalid_marks"), ("pm_jumps", "pm_jumps"),
+             ("verify_checks", "verify_checks"), ("verify_matches", "verify_matches")]
+    for a, b in pairs:
+        assert st[a] == sim[b], (a, st[a], sim[b])
+
+
+def _spread_host(w, total):
+    """The 1 MiB selector profile of a long stream (reading R20, include/gspec.h): 8
+    portions of 128 KiB at floor(i (len - 128 KiB) / 7) rounded down to 4 KiB."""
+    S = 128 << 10
+    return np.concatenate([w.host((i * (total - S) // 7) & ~4095, S) for i in range(8)])
+
+
+@pytest.mark.parametrize("name", ["c3s", "c3", "c2"])
+def test_selector_spread_profile(gs, name):
+    """fsm_select_scheme on a whole 1 GiB stream profiles 8 spread portions of it (R20):
+    the GPU features equal the oracle's on the same portions, and on the input-sensitive
+    stream the sensitivity feature now sees its normal and vowel-free regions."""
+    L = 1 << 30
+    w = gen.workload(name, length=L)
+    x = torch.empty(L, dtype=torch.uint8, device="cuda")
+    w.device(x)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    pick, ft = fsm.select_scheme(x)
+    sample = _spread_host(w, L)
+    of = oracle.features(w.table, w.start, w.accept, sample, B=4096)
+    assert ft["acc1"] == pytest.approx(of["acc1"]) and ft["acck"] == pytest.approx(of["acck"])
+    assert ft["input_sensitivity"] == pytest.approx(of["sens"]) and ft["uniq10"] == pytest.approx(of["uniq10"])
+    assert gs.SCHEMES[pick] == oracle.select(of, w.nstates)
+    if name == "c3s":
+        assert of["sens"] >= 0.2
+    res = fsm.run(x[:64 << 20], scheme="auto")  # the cached choice
+    assert res.scheme == pick
+    del x
+    torch.cuda.empty_cache()

@@ -480,6 +480,52 @@ def test_simulate_literal_rr_nf(seed, scheme):
             assert all(taken[d] <= qlen[d] for d in range(N))
 
 
+@pytest.mark.parametrize("seed", range(8))
+def test_simulate_pm_tree(seed):
+    """Faithful PM (Eq. 2) on random DFAs and chunkings:
+    * results equal the sequential run;
+    * ceil(log2 N) merge rounds;
+    * stage-2 recoveries = chunks whose true start is not among their k speculated
+      states (Eq. 2: P_i^PM = 1 - accu_i^spec-k), counted by brute force from the
+      sequential run's chunk ends and the lookback ranking (both pinned above)."""
+    rng = random.Random(seed * 31 + 7)
+    n, ns = rng.randint(1, 40), rng.randint(1, 6)
+    t, s, a = gen.dfa_random(seed + 61, n, ns)
+    data = gen.workload(f"rand:{n}:{ns}:{seed}", length=rng.randint(0, 20000), seed=seed + 5).host()
+    perm, inv, _, tt, acc = oracle.transform(t, a)
+    for B in (16, 48, 256):
+        for k in (1, 2, 4):
+            r = oracle.run(t, s, a, data, B)
+            o = oracle.simulate_pm_tree(t, s, a, data, B, k=k)
+            N = oracle.nchunks(len(data), B)
+            assert o["status"] == 0
+            assert o["final_state"] == r["final"] and o["accept_count"] == r["count"]
+            assert (o["chunk_end"] == r["chunk_end"]).all()
+            assert o["pm_levels"] == (max(N - 1, 0)).bit_length()
+            miss = 0
+            for c in range(1, N):
+                qs, _ = oracle.lookback(tt, n, data[c * B - 2:c * B], K=16)
+                miss += int(perm[r["chunk_end"][c - 1]]) not in [int(q) for q in qs[:k]]
+            assert o["pm_recoveries"] == miss
+            assert o["pm_reread_bytes"] <= miss * B
+
+
+def test_simulate_pm_tree_special_cases():
+    """div7 (every lookback image is all 7 states): with k = 7 every path merges
+    (no invalid mark, one stage-2 jump, no recovery); a one-state DFA likewise."""
+    w = gen.workload("c1", length=1 << 14)
+    d = w.host()
+    o = oracle.simulate_pm_tree(w.table, w.start, w.accept, d, 64, k=7)
+    assert o["pm_invalid_marks"] == 0 and o["pm_jumps"] == 1 and o["pm_recoveries"] == 0
+    o4 = oracle.simulate_pm_tree(w.table, w.start, w.accept, d, 64, k=4)
+    assert o4["pm_invalid_marks"] > 0 and o4["pm_recoveries"] > 0
+    assert o4["final_state"] == o["final_state"] and o4["accept_count"] == o["accept_count"]
+    t1 = np.zeros((1, 3), np.uint32)
+    d1 = np.array([0, 1, 2] * 300, np.uint8)
+    o = oracle.simulate_pm_tree(t1, 0, np.array([1], np.uint8), d1, 16, k=4)
+    assert o["pm_recoveries"] == 0 and o["pm_jumps"] == 1 and o["accept_count"] == len(d1)
+
+
 def test_simulate_invalid_symbol():
     t, s, a = gen.dfa_div7()
     data = np.array([1, 0, 1] * 100 + [3] + [1] * 50, np.uint8)
