@@ -270,11 +270,12 @@ def measure_single(gs, w, x, args, fsm, scheme, with_clocks=True):
     length = x.numel()
     stream = torch.cuda.current_stream()
     ce = torch.empty(gs.fsm_num_chunks(length, B), dtype=torch.int32, device="cuda")
-    kr = [fsm.run(x, scheme=scheme, chunk_bytes=B) for _ in range(3)]
+    kw = {"spec_k": args.spec_k, "lookback": args.lookback}
+    kr = [fsm.run(x, scheme=scheme, chunk_bytes=B, **kw) for _ in range(3)]
     verify_phases = [round(float(v), 1) for v in fsm.phase_times()]
     pending = []
     for _ in range(max(3, args.warmup)):
-        pending.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce))
+        pending.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce, **kw))
     for t in pending:
         fsm.wait(t)
     pending.clear()
@@ -285,7 +286,7 @@ def measure_single(gs, w, x, args, fsm, scheme, with_clocks=True):
         clk.__enter__()
     ev0.record(stream)
     for _ in range(args.steps):
-        pending.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce))
+        pending.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce, **kw))
     ev1.record(stream)
     torch.cuda.synchronize()
     if clk:
@@ -400,9 +401,9 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         lo, hi = shard_bounds(L, world, rank, B)
         x = torch.empty(hi - lo, dtype=torch.uint8, device="cuda")
         w.device(x, offset=lo)
-        lb = torch.empty(2 if lo else 0, dtype=torch.uint8, device="cuda")
-        if lo:
-            w.device(lb, offset=lo - 2)  # the 2 bytes before the shard (pure function of the offset)
+        lb = torch.empty(min(16, lo), dtype=torch.uint8, device="cuda")
+        if lo:  # the 16 bytes before the shard (pure function of the offset): its candidate set
+            w.device(lb, offset=lo - lb.numel())
         fsm = gs.FSM.load(w.table, w.start, w.accept)
         # selector per DFA (offline profiling): every rank profiles the same 8 spread
         # portions of the global stream (R20), so every rank picks the same scheme
@@ -487,6 +488,8 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(CONFIG_DESC))
     ap.add_argument("--scheme", default="auto")
     ap.add_argument("--chunk-bytes", type=int, default=4096)
+    ap.add_argument("--spec-k", type=int, default=0, help="paths per chunk for pm / pm_tree / cse (0 = default)")
+    ap.add_argument("--lookback", type=int, default=2, help="lookback symbols per chunk prediction (2..16, R25)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-per-dfa", action="store_true", help="skip the per-DFA sub-results of the default line")
@@ -562,10 +565,11 @@ def main():
     if world > 1:
         from paper_conf_ipps_wangwqw22_b200.dist import run_sharded
 
-        # the 2 bytes before this rank's shard (pure function of the offset): lookback image
-        lb = torch.empty(2 if rank else 0, dtype=torch.uint8, device="cuda")
+        # the 16 bytes before this rank's shard (pure function of the offset): its candidate
+        # start set is their lookback image, the smallest one fsm_shard_map accepts
+        lb = torch.empty(16 if rank else 0, dtype=torch.uint8, device="cuda")
         if rank:
-            w.device(lb, offset=rank * length - 2)
+            w.device(lb, offset=rank * length - 16)
 
         def step():
             if comm is not None:
@@ -652,7 +656,8 @@ def main():
         "dtype": "u8",
         "data": "synthetic",
         "config": {"workload": args.config, "desc": CONFIG_DESC[args.config], "bytes_per_gpu": length,
-                   "chunk_bytes": B, "scheme": scheme, "nstates": int(w.nstates),
+                   "chunk_bytes": B, "scheme": scheme, "nstates": int(w.nstates), "spec_k": args.spec_k or None,
+                   "lookback": args.lookback,
                    "l2": "input (1 GiB/GPU) larger than the 126 MB L2; no explicit flush",
                    "parallelism": (f"dp{world} contiguous shards + one allgather of state maps"
                                    + (" (library NCCL, fsm_run_sharded)" if comm is not None else "")

@@ -89,7 +89,7 @@ typedef struct {
 typedef struct {
   fsm_scheme scheme;    /* FSM_SCHEME_*                                                  */
   uint32_t chunk_bytes; /* B: chunk c = [cB, min(len,(c+1)B)); multiple of 16; 0 = 4096   */
-  uint32_t spec_k;      /* paths per chunk: PM (4) / CSE (8); 1..8; 0 = default    */
+  uint32_t spec_k;      /* paths per chunk: PM (4) / CSE (8); 1..16; 0 = default   */
   uint32_t lookback;    /* lookback symbols (2); only 2 is supported; 0 = 2        */
   uint32_t qs_cap;      /* K: ranked candidates kept per chunk (16); 1..16; 0 = 16 */
   uint32_t vr_end;      /* VR^end slots per chunk (16); 1..16; 0 = 16              */

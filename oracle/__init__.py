@@ -59,8 +59,10 @@ def lib():
         L.or_lookback.restype = U32
         L.or_enum.argtypes = [P, U32, U32, P, P, U64, P, P]
         L.or_compose.argtypes = [U32, P, P, P, P, P, P]
-        L.or_simulate.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, ctypes.c_int, U32, U32, U32, U32,
+        L.or_simulate.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, ctypes.c_int, U32, U32, U32, U32, U32,
                                   P, ctypes.POINTER(SimResult), P, U64, P]
+        L.or_lookback_long.argtypes = [P, U32, U32, P, U32, U32, P, P]
+        L.or_lookback_long.restype = U32
         L.or_simulate_literal_sre.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, U32, P,
                                               ctypes.POINTER(SimResult)]
         L.or_simulate_literal.argtypes = [P, U32, U32, U32, P, P, P, U64, U32, ctypes.c_int, U32, U32, P,
@@ -183,8 +185,19 @@ def compose(M1, C1, M2, C2):
     return M, C
 
 
+def lookback_long(t, nq, w, K=16):
+    """Lookback over the len(w) in [2, 16] symbols w before a chunk (reading R25)."""
+    t = _c(t, np.uint32)
+    w = _c(w, np.uint8)
+    qs = np.zeros(max(1, K), np.uint32)
+    ql = U32(0)
+    img = lib().or_lookback_long(t.ctypes.data, nq, t.shape[1], w.ctypes.data, w.size, K, qs.ctypes.data,
+                                 ctypes.byref(ql))
+    return qs[:ql.value].copy(), int(img)
+
+
 def simulate(table, start, accept, data, B=4096, scheme="sre", spec_k=None, qs_cap=16, vr_end=16, vr_oth=16,
-             policy=0, max_tasks=0):
+             policy=0, max_tasks=0, lookback=2):
     """Round semantics of Alg. 2-5. Works on the transformed DFA.
     spec_k: round-0 paths per chunk for PM (default 4) and CSE (default 8)."""
     if spec_k is None:
@@ -198,7 +211,7 @@ def simulate(table, start, accept, data, B=4096, scheme="sre", spec_k=None, qs_c
     tasks = (Task * max(1, max_tasks))()
     nt = U64(0)
     rc = lib().or_simulate(tt.ctypes.data, n, ns, int(perm[start]), acc.ctypes.data, inv.ctypes.data,
-                           d.ctypes.data, d.size, B, SCHEME_IDS[scheme], spec_k, qs_cap, vr_end, vr_oth,
+                           d.ctypes.data, d.size, B, SCHEME_IDS[scheme], spec_k, qs_cap, lookback, vr_end, vr_oth,
                            ce.ctypes.data, ctypes.byref(res), tasks, max_tasks, ctypes.byref(nt))
     out = res.as_dict()
     out["status"] = rc

@@ -49,6 +49,13 @@ int or_transform(const uint32_t* table, uint32_t n, uint32_t nsyms, const uint8_
 uint32_t or_lookback(const uint32_t* t, uint32_t nq, uint32_t nsyms, const uint8_t* w, uint32_t L,
                      uint32_t K, uint32_t* qs, uint32_t* qs_len);
 
+/* Lookback of L in [2, 16] symbols (P:300 with L > 2; reading R25): or_lookback over the
+ * L symbols w[0..L) before a chunk, except that when the image of the first two of them
+ * already has more than 64 states the lookback-2 ranking of the last two (w[L-2..L)) is
+ * used — the cost bound of the GPU path; both images contain the true start. */
+uint32_t or_lookback_long(const uint32_t* t, uint32_t nq, uint32_t nsyms, const uint8_t* w, uint32_t L,
+                          uint32_t K, uint32_t* qs, uint32_t* qs_len);
+
 /* Enumeration: M[q] = state after the chunk from q, C[q] = accepts
  * along that path, for every q < n.  Returns OR_ESYMBOL on an invalid byte. */
 int or_enum(const uint32_t* table, uint32_t n, uint32_t nsyms, const uint8_t* accept,
@@ -94,7 +101,7 @@ typedef struct {
  * tasks (nullable) receives up to max_tasks task records. */
 int or_simulate(const uint32_t* tt, uint32_t nt, uint32_t nsyms, uint32_t q0t, const uint8_t* acc_t,
                 const uint32_t* inv, const uint8_t* in, uint64_t len, uint32_t B, int scheme,
-                uint32_t spec_k, uint32_t qs_cap, uint32_t vr_end, uint32_t vr_oth,
+                uint32_t spec_k, uint32_t qs_cap, uint32_t lookback, uint32_t vr_end, uint32_t vr_oth,
                 uint32_t* chunk_end, or_sim_result* res, or_task* tasks, uint64_t max_tasks,
                 uint64_t* ntasks);
 

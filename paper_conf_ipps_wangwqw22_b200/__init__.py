@@ -138,14 +138,15 @@ def run_multi(fsms, inputs, chunk_bytes=4096, stream=None):
     return fin[:n], cnt[:n], {k: getattr(r, k) for k, _ in fsm_multi_result._fields_}
 
 
-def _run_opts(scheme="auto", chunk_bytes=4096, spec_k=0, qs_cap=16, vr_end=16, vr_others=16, stream=None):
+def _run_opts(scheme="auto", chunk_bytes=4096, spec_k=0, qs_cap=16, vr_end=16, vr_others=16, stream=None,
+              lookback=2):
     if isinstance(scheme, str):
         scheme = SCHEMES[scheme]
     if stream is None:
         import torch
 
         stream = torch.cuda.current_stream().cuda_stream if torch.cuda.is_available() else 0
-    return fsm_run_opts(scheme=scheme, chunk_bytes=chunk_bytes, spec_k=spec_k, lookback=2, qs_cap=qs_cap,
+    return fsm_run_opts(scheme=scheme, chunk_bytes=chunk_bytes, spec_k=spec_k, lookback=lookback, qs_cap=qs_cap,
                         vr_end=vr_end, vr_others=vr_others, stream=stream)
 
 
@@ -203,12 +204,13 @@ class FSM:
 
     # ---- runs -----------------------------------------------------------------
     def run(self, x, scheme="auto", chunk_bytes=4096, spec_k=0, qs_cap=16, vr_end=16, vr_others=16,
-            chunk_ends=True, stream=None) -> Result:
-        """fsm_run over a uint8 CUDA tensor; chunk_ends -> int64-free uint32 CUDA tensor (as torch.int32 view)."""
+            chunk_ends=True, stream=None, lookback=2) -> Result:
+        """fsm_run over a uint8 CUDA tensor; chunk_ends -> uint32 chunk end states (a torch.int32
+        CUDA tensor); lookback = symbols before each chunk used for its prediction (2..16)."""
         import torch
 
         assert x.is_cuda and x.dtype == torch.uint8 and x.is_contiguous()
-        o = _run_opts(scheme, chunk_bytes, spec_k, qs_cap, vr_end, vr_others, stream)
+        o = _run_opts(scheme, chunk_bytes, spec_k, qs_cap, vr_end, vr_others, stream, lookback)
         n = fsm_num_chunks(x.numel(), chunk_bytes)
         ce = torch.empty(max(n, 1), dtype=torch.int32, device=x.device) if chunk_ends else None
         r = fsm_result()
@@ -216,9 +218,10 @@ class FSM:
                             ce.data_ptr() if ce is not None else None, ctypes.byref(r)), "fsm_run")
         return Result.from_c(r, ce[:n] if ce is not None else None)
 
-    def run_async(self, x, scheme="auto", chunk_bytes=4096, chunk_ends=None, spec_k=0, stream=None) -> int:
+    def run_async(self, x, scheme="auto", chunk_bytes=4096, chunk_ends=None, spec_k=0, stream=None,
+                  lookback=2) -> int:
         """fsm_run_async: enqueue a run (stream-ordered) and return a ticket for wait()."""
-        o = _run_opts(scheme, chunk_bytes, spec_k, stream=stream)
+        o = _run_opts(scheme, chunk_bytes, spec_k, stream=stream, lookback=lookback)
         t = U64(0)
         _check(_lib.fsm_run_async(self._h, x.data_ptr() if x.numel() else None, x.numel(), ctypes.byref(o),
                                   chunk_ends.data_ptr() if chunk_ends is not None else None, ctypes.byref(t)),

@@ -153,8 +153,8 @@ int resolve_opts(const fsm_run_opts* o, Opts* r) {
   r->vr_oth = (o && o->vr_others) ? o->vr_others : 16;
   r->st = o ? reinterpret_cast<cudaStream_t>(o->stream) : nullptr;
   if (r->B % 16 != 0) return fail(FSM_EINVAL, "chunk_bytes must be a multiple of 16");
-  if (r->k < 1 || r->k > 8) return fail(FSM_EINVAL, "spec_k must be in [1,8]");
-  if (r->L != 2) return fail(FSM_EUNSUPPORTED, "only lookback = 2 is supported (P:300)");
+  if (r->k < 1 || r->k > kQsMax) return fail(FSM_EINVAL, "spec_k must be in [1,16]");
+  if (r->L < 2 || r->L > kLookbackMax) return fail(FSM_EUNSUPPORTED, "lookback must be in [2,16] (P:300, R25)");
   if (r->qs_cap < 1 || r->qs_cap > kQsMax) return fail(FSM_EINVAL, "qs_cap must be in [1,16]");
   if (r->vr_end < 1 || r->vr_end > kVrMax || r->vr_oth < 1 || r->vr_oth > kVrMax)
     return fail(FSM_EINVAL, "vr_end / vr_others must be in [1,16]");
@@ -196,6 +196,8 @@ int ensure_records(fsm_t f, uint64_t N) {
     r.task_start = (uint32_t*)take(4 * (cap + 8));
     r.task_j = (uint32_t*)take(4 * (cap + 8));
     r.tstart = (uint32_t*)take(4 * (cap + 8));
+    r.bflag = (uint32_t*)take(4 * (cap / 32 + 8) + 64);
+    r.v0c = base ? reinterpret_cast<unsigned long long*>(r.bflag + cap / 32 + 8) : nullptr;
     r.next_qs = take(cap);
     r.found = take(cap);
     r.ulen = take(cap);
@@ -209,6 +211,8 @@ int ensure_records(fsm_t f, uint64_t N) {
   cudaError_t e = cudaMalloc(&p, bytes);
   if (e != cudaSuccess) return fail(FSM_ENOMEM, std::string("record store: ") + cudaGetErrorString(e));
   carve(reinterpret_cast<uint8_t*>(p));
+  e = cudaMemset(r.bflag, 0, 4 * (cap / 32 + 8) + 64);  // boundary counters start even (never reset), v0c zero
+  if (e != cudaSuccess) return fail(FSM_ECUDA, std::string("record store: ") + cudaGetErrorString(e));
   f->rs = r;
   f->rs_base = p;
   f->rs_cap = cap;
@@ -247,6 +251,46 @@ void fill_result_stats(fsm_result* out, const Ctl& h) {
 }
 
 int select_auto(fsm_t f, const uint8_t* d_in, uint64_t len, const fsm_run_opts* opts);
+
+// Lookback L > 2 (reading R25): the per-pair full images with multiplicities (built once,
+// at the first such run) and the per-run table QS_c for every chunk (k_qs_long).
+int prepare_long_lookback(fsm_t f, const uint8_t* d_in, uint64_t N, const Opts& o, RunParams* rp,
+                          uint32_t* launches) {
+  if (o.L <= 2) return FSM_OK;
+  const uint32_t C = f->img.C, nt = f->n + 1;
+  const uint64_t npairs = (uint64_t)C * C;
+  if (!f->img2_base) {
+    CUDA_TRY(cudaMalloc(&f->img2_base, npairs * kImgFull * 8 + npairs + 16));
+    f->img2_s = reinterpret_cast<uint32_t*>(f->img2_base);
+    f->img2_m = f->img2_s + npairs * kImgFull;
+    f->img2_n = reinterpret_cast<uint8_t*>(f->img2_m + npairs * kImgFull);
+    uint32_t grid = (uint32_t)std::min<uint64_t>(npairs, (uint64_t)f->sm_count * 4);
+    if ((uint64_t)grid * nt > (1ull << 28)) grid = (uint32_t)std::max<uint64_t>(1, (1ull << 28) / nt);
+    void* scratch = nullptr;
+    CUDA_TRY(cudaMalloc(&scratch, (uint64_t)grid * nt * 4));
+    cudaError_t ce = launch_build_img2_raw(f->d_ttc, f->n, C, (uint32_t*)scratch, grid, f->img2_s, f->img2_m,
+                                           f->img2_n, o.st);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(o.st);
+    cudaFree(scratch);
+    CUDA_TRY(ce);
+  }
+  if (f->qsc_cap < N) {
+    CUDA_TRY(cudaStreamSynchronize(o.st));  // queued runs may still read the old table
+    if (f->qsc_base) cudaFree(f->qsc_base);
+    f->qsc_base = nullptr;
+    f->qsc_cap = 0;
+    CUDA_TRY(cudaMalloc(&f->qsc_base, N * (kQsMax * 4 + 1) + 16));
+    f->qsc_cap = N;
+  }
+  uint32_t* qsc = reinterpret_cast<uint32_t*>(f->qsc_base);
+  uint8_t* qsl = reinterpret_cast<uint8_t*>(qsc + f->qsc_cap * kQsMax);
+  CUDA_TRY(launch_qs_long(f->img, f->d_ttc, d_in, o.B, N, o.L, f->img2_s, f->img2_m, f->img2_n, qsc, qsl,
+                          f->sm_count, o.st));
+  rp->qsc = qsc;
+  rp->qsc_len = qsl;
+  *launches += 1;
+  return FSM_OK;
+}
 
 // Enqueue one device run over d_in[0..len) from transformed start q0t on
 // o.st; returns a ticket.  Everything (init, kernels, readback) is stream
@@ -336,7 +380,6 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     if (f->pm_bytes < need) {
       CUDA_TRY(cudaStreamSynchronize(o.st));
       if (f->pm_base) cudaFree(f->pm_base);
-  if (f->prof_buf) cudaFree(f->prof_buf);
       f->pm_base = nullptr;
       f->pm_bytes = 0;
       CUDA_TRY(cudaMalloc(&f->pm_base, need));
@@ -344,11 +387,13 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     }
     rp.ctl_init = f->d_ctl;
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
+    uint32_t lq = 0;
+    if ((rc = prepare_long_lookback(f, d_in, N, o, &rp, &lq))) return rc;
     {
       NvtxRange nv_("speculative execution spec-k (PM round 0)");
       CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
     }
-    pd.launches = 1 + (len % o.B != 0 && len / o.B > 0);
+    pd.launches = lq + 1 + (len % o.B != 0 && len / o.B > 0);
     rp.ctl_init = nullptr;
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
     uint32_t nl = 0;
@@ -364,6 +409,8 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     rp.ctl_init = f->d_ctl;  // the spec kernel initialises the control block
     rp.h_out = &h;           // ... and the verify kernel's finalize step writes it back (pinned, UVA)
     CUDA_TRY(cudaEventRecord(ev[0], o.st));
+    uint32_t lq = 0;
+    if ((rc = prepare_long_lookback(f, d_in, N, o, &rp, &lq))) return rc;
     // dense recovery rounds go to the TMA task kernel (SRE / RR / NF on low-accuracy DFAs); this
     // needs a host check per verify launch, so it is off when the profile says the
     // speculation is accurate (no dense rounds expected)
@@ -371,13 +418,22 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
                  scheme == FSM_SCHEME_NF) && len / o.B > 0 && o.B % 64 == 0 &&
                 (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0 && f->acc1_hint < 0.5) ? 1u : 0u;
     {
+      // accurate SRE (no dense rounds expected): round 0's verification and its inline
+      // recoveries run inside the TMA spec kernel as its tiles finish (RunParams::v0); the
+      // verify launch then returns at once unless a recovery moved an end
+      const bool tma_full = !spec_path_generic_only() && len % o.B == 0 && len / o.B > 0 && o.B % 64 == 0 &&
+                            (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0 && len / o.B < (1ull << 31);
+      rp.v0 = (scheme == FSM_SCHEME_SRE && rp.k == 1 && !rp.dense && tma_full && !v0_disabled()) ? 1u : 0u;
+      rp.v0_ctl = f->d_ctl;
+      rp.v0_bflag = f->rs.bflag;
+      rp.v0_chunk_ends = d_chunk_ends;
       NvtxRange nv_("speculative execution (round 0)");
       CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
     }
     {  // TMA kernel over the full chunks + the generic kernel for a tail chunk (or everything)
       const bool tma = !spec_path_generic_only() && len / o.B > 0 && o.B % 64 == 0 &&
                        (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0;
-      pd.launches = tma ? 1 + (len % o.B != 0) : 1;
+      pd.launches = lq + (tma ? 1 + (len % o.B != 0) : 1);
     }
     rp.ctl_init = nullptr;  // initialised by the spec kernel; later launches must not touch it
     CUDA_TRY(cudaEventRecord(ev[1], o.st));
@@ -817,6 +873,8 @@ void fsm_free(fsm_t f) {
   if (f->multi_base) cudaFree(f->multi_base);
   if (f->pm_base) cudaFree(f->pm_base);
   if (f->prof_buf) cudaFree(f->prof_buf);
+  if (f->img2_base) cudaFree(f->img2_base);
+  if (f->qsc_base) cudaFree(f->qsc_base);
   for (auto& e : f->multi_ev)
     if (e) cudaEventDestroy(e);
   delete f;
@@ -911,6 +969,7 @@ int fsm_run_batch(fsm_t f, const uint8_t* d_input, const uint64_t* h_offsets, ui
   Opts o;
   int rc = resolve_opts(opts, &o);
   if (rc) return rc;
+  if (o.L != 2) return fail(FSM_EUNSUPPORTED, "fsm_run_batch: lookback 2 only (the pair table, P:300)");
   const uint32_t B = o.B;
   std::vector<uint64_t> hb(2 * ((uint64_t)nstreams + 1));  // [offsets | chunk bases]
   uint64_t N = 0;
@@ -972,6 +1031,7 @@ int fsm_run_multi(const fsm_t* fsms, uint32_t npairs, const uint8_t* const* d_in
   Opts o;
   int rc = resolve_opts(opts, &o);
   if (rc) return rc;
+  if (o.L != 2) return fail(FSM_EUNSUPPORTED, "fsm_run_multi: lookback 2 only (the pair table, P:300)");
   std::vector<DevImage> imgs(npairs);
   std::vector<const uint8_t*> ins(npairs);
   std::vector<uint32_t> order;
@@ -1063,6 +1123,7 @@ int fsm_run_literal(fsm_t f, const uint8_t* d_input, uint64_t len, const fsm_run
   Opts o;
   int rc = resolve_opts(opts, &o);
   if (rc) return rc;
+  if (o.L != 2) return fail(FSM_EUNSUPPORTED, "fsm_run_literal: lookback 2 only (the pair table, P:300)");
   const uint64_t N = fsm_num_chunks(len, o.B);
   if (N > literal_max_chunks()) return fail(FSM_EUNSUPPORTED, "paper-literal kernel: at most 1024 chunks (one CTA)");
   // SRE (Alg. 3, the default for AUTO), RR (Alg. 4) or NF (Alg. 5)

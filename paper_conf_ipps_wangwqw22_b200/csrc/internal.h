@@ -30,6 +30,8 @@ constexpr uint32_t kErrorMap = 0xFFFFFFFDu;    // map of a rank whose fsm_shard_
 constexpr uint32_t kDeltaBaseMax = 8192;  // MODE_U16D: max shared-window offset of the staged table
 
 constexpr uint32_t kQsMax = 16;     // QS cap ("top 16 states")
+constexpr uint32_t kImgFull = 64;   // lookback > 2: pair images kept with multiplicities up to this size (R25)
+constexpr uint32_t kLookbackMax = 16;
 constexpr uint32_t kVrMax = 16;     // VR^end / VR^others slots
 constexpr uint32_t kSlots = 2 * kVrMax;
 constexpr uint32_t kEnumMax = 32;   // ENUM: transformed states incl. poison
@@ -96,6 +98,10 @@ struct RecStore {
   uint32_t* task_start;  // [cap+1]
   uint32_t* task_j;      // [cap+1] helper index within its chunk
   uint32_t* tstart;      // [cap] dense rounds: task start of chunk c, 0xFFFFFFFF = no task
+  uint32_t* bflag;       // [cap / 32 + 1] fused round-0 verification: tile-boundary arrivals
+  // fused round-0 verification counters {checks, matches, tasks, reread, ztot, ~first task
+  // chunk (0 = none), moved, warps}: zero between runs (the last warp of a run clears them)
+  unsigned long long* v0c;
 };
 
 // Device control block of the verify/recover kernel.
@@ -150,6 +156,15 @@ struct RunParams {
   const uint32_t* q0_dev;  // non-null: chunk 0's start is read from the device (shard candidates)
   Ctl* h_out;      // non-null: pinned host slot; the finalize step writes the control block there
   uint32_t stamps; // 1: record the run timeline (Ctl::tl), profiling only
+  const uint32_t* qsc;     // non-null: per-chunk QS [N][kQsMax] of a lookback > 2 (k_qs_long)
+  const uint8_t* qsc_len;  // [N]
+  // fused round-0 verification (SRE, spec-1, accurate speculation): the TMA spec kernel
+  // checks every chunk against its predecessor's round-0 end as its tiles finish, runs the
+  // mismatches' recoveries inline and, when no recovery changed an end, completes the run
+  uint32_t v0;             // 1: fused (v0_ctl, v0_bflag set)
+  Ctl* v0_ctl;
+  uint32_t* v0_bflag;      // [tiles] tile-boundary arrival counters (+2 per run, never reset)
+  uint32_t* v0_chunk_ends; // nullable: the run's chunk ends (original ids)
 };
 
 // GSPEC_STAMPS=1: kernels record the run timeline in Ctl::tl (one extra atomic per warp).
@@ -168,6 +183,16 @@ inline bool stamps_enabled() {
 // previous grid's completion and memory flush.  Opt-in (GSPEC_PDL=1): measured on
 // c2 it does not shorten the step (0.3237 vs 0.3232 ms) — the verify CTAs cannot
 // become resident before the spec CTAs (full shared memory) exit.
+// GSPEC_V0=0 turns the fused round-0 verification off (A/B measurements).
+inline bool v0_disabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("GSPEC_V0");
+    v = (e && atoi(e) == 0) ? 1 : 0;
+  }
+  return v != 0;
+}
+
 inline bool pdl_enabled() {
   static int v = -1;
   if (v < 0) {
@@ -292,6 +317,11 @@ cudaError_t launch_map_fused(const uint32_t* cand, const uint32_t* ncand_p, cons
 cudaError_t launch_fix_prefix_fused(const uint32_t* states, const uint32_t* cand, const uint32_t* ncand_p,
                                     const uint32_t* merged, const uint32_t* srank_p, const uint32_t* inv,
                                     uint32_t poison, uint32_t* chunk_ends, uint32_t* err, cudaStream_t st);
+cudaError_t launch_build_img2_raw(const uint32_t* d_ttc, uint32_t n, uint32_t C, uint32_t* scratch, uint32_t grid,
+                                  uint32_t* img_s, uint32_t* img_m, uint8_t* img_n, cudaStream_t st);
+cudaError_t launch_qs_long(const DevImage& img, const uint32_t* d_ttc, const uint8_t* in, uint32_t B, uint64_t N,
+                           uint32_t L, const uint32_t* img_s, const uint32_t* img_m, const uint8_t* img_n,
+                           uint32_t* qsc, uint8_t* qsc_len, int sms, cudaStream_t st);
 uint64_t pm_tree_scratch_bytes(uint64_t N, uint32_t k, uint32_t* levels);
 cudaError_t launch_pm_tree(const DevImage& img, const RunParams& rp, const RecStore& rs, uint32_t k, void* scratch,
                            Ctl* ctl, uint32_t* d_chunk_ends, int sms, cudaStream_t st, uint32_t* launches);
@@ -376,7 +406,12 @@ struct fsm_s {
   void* batch_base = nullptr;            // fsm_run_batch scratch (offsets, chunk bases, records, totals)
   size_t batch_bytes = 0;
   cudaEvent_t batch_ev[2] = {nullptr, nullptr};
-  uint8_t* prof_buf = nullptr;           // FSM_SCHEME_AUTO's spread 1 MiB profile sample
+  uint8_t* prof_buf = nullptr;
+  void* img2_base = nullptr;             // lookback > 2: full pair images (built at first use)
+  uint32_t *img2_s = nullptr, *img2_m = nullptr;
+  uint8_t* img2_n = nullptr;
+  void* qsc_base = nullptr;              // lookback > 2: per-run QS table [N][kQsMax] + lengths
+  uint64_t qsc_cap = 0;           // FSM_SCHEME_AUTO's spread 1 MiB profile sample
   void* pm_base = nullptr;               // FSM_SCHEME_PM_TREE scratch (level maps, jump list)
   size_t pm_bytes = 0;
   void* multi_base = nullptr;            // fsm_run_multi scratch when this handle is fsms[0] (its device)

@@ -73,7 +73,7 @@ __global__ void k_pm_merge(const PmEnt* __restrict__ prev, uint64_t nprev, PmEnt
     }
     const PmEnt* re = prev + (2 * g + 1) * k;
     const uint64_t m1 = (2 * g + 1) << (l - 1);  // first chunk of the right segment
-    uint32_t rs_[8];
+    uint32_t rs_[kQsMax];
     for (uint32_t r = 0; r < k; r++) rs_[r] = starts[m1 * k + r];
     for (uint32_t j = 0; j < k; j++) {
       const PmEnt a = le[j];

@@ -51,11 +51,11 @@ __global__ void __launch_bounds__(256) k_spec_exec(DevImage img, RunParams rp, R
 #pragma unroll
         for (int p = 0; p < KP; p++) st[i][p] = q0_of(rp);
       } else {
-        const uint32_t pair = qs_pair(img, rp.in, c[i], rp.B);
-        const uint32_t ql = __ldg(img.qs2_len + pair);
+        uint32_t ql;
+        const uint32_t* qs = qs_chunk(img, rp, c[i], &ql);
         kc[i] = min(rp.k, min(ql, rp.qs_cap));
 #pragma unroll
-        for (int p = 0; p < KP; p++) st[i][p] = __ldg(img.qs2 + (uint64_t)pair * kQsMax + min((uint32_t)p, kc[i] - 1));
+        for (int p = 0; p < KP; p++) st[i][p] = __ldg(qs + min((uint32_t)p, kc[i] - 1));
       }
 #pragma unroll
       for (int p = 0; p < KP; p++) {
@@ -161,7 +161,8 @@ cudaError_t launch_mode(const DevImage& img, const RunParams& rp, const RecStore
   if (rp.k <= 1) return launch_t<MODE, 2, 1>(img, rp, rs, st, c0);
   if (rp.k <= 2) return launch_t<MODE, 1, 2>(img, rp, rs, st, c0);
   if (rp.k <= 4) return launch_t<MODE, 1, 4>(img, rp, rs, st, c0);
-  return launch_t<MODE, 1, 8>(img, rp, rs, st, c0);
+  if (rp.k <= 8) return launch_t<MODE, 1, 8>(img, rp, rs, st, c0);
+  return launch_t<MODE, 1, 16>(img, rp, rs, st, c0);
 }
 
 }  // namespace

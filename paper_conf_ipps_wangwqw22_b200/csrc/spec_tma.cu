@@ -76,6 +76,118 @@ __device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, u
       : "memory");
 }
 
+// Fused round-0 verification (SRE with spec-1 records, accurate speculation; RunParams::v0).
+// Round 0's verification cannot change an incoming state (one record per chunk: x_c is the
+// predecessor's round-0 end), so every chunk is checked as soon as its own and its
+// predecessor's walks are done: inside a tile by shuffle, across tiles by whichever of the
+// two warps finishes second (tile-boundary arrival counters, no spinning).  A mismatch is
+// recovered at once from x_c (Alg. 3 L16-18) with path fusion, exactly as the verify
+// kernel's round-0 pass does; the counters go to the same pass slot.
+// Returns bit 0 = hit, bit 1 = recovered (a task ran), bit 2 = the task moved the end;
+// *cnt = the chunk's accept count on the true path (round-0 count, or the task's).
+template <int MODE>
+__device__ __noinline__ uint32_t v0_check(const DevImage& img, const uint8_t* table, const RunParams& rp,
+                                          const RecStore& rs, uint64_t c, uint32_t xin, uint32_t s0, uint32_t xo,
+                                          uint32_t c0, uint32_t* cnt_out) {
+  const bool hit = xin == s0;
+  rs.found[c] = hit;
+  if (rp.v0_chunk_ends) rp.v0_chunk_ends[c] = __ldg(img.inv + xo);  // speculative: exact unless a task moves an end
+  if (hit) {
+    *cnt_out = c0;
+    return 1u;
+  }
+  uint32_t e, cnt;
+  task_walk<MODE>(img, table, rp, rs, c, xin, &e, &cnt);
+  const uint32_t ne = __ldcg(rs.n_end + c);
+  const uint64_t o = (uint64_t)(ne % rp.vr_end) * rs.cap + c;
+  __stcg(rs.start + o, xin);
+  __stcg(rs.end + o, e);
+  __stcg(rs.cnt + o, cnt);
+  __stcg(rs.n_end + c, ne + 1);
+  __stcg(rs.cur_end + c, e);
+  *cnt_out = cnt;
+  return 2u | (e != xo ? 4u : 0u);
+}
+
+// chunk c checked from the global record store (the other warp of its tile boundary)
+template <int MODE>
+__device__ __forceinline__ uint32_t v0_check_global(const DevImage& img, const uint8_t* table, const RunParams& rp,
+                                                    const RecStore& rs, uint64_t c, uint32_t* cnt) {
+  return v0_check<MODE>(img, table, rp, rs, c, __ldcg(rs.x + c), __ldcg(rs.start + c), __ldcg(rs.x + c + 1),
+                        __ldcg(rs.cnt + c), cnt);
+}
+
+// atomicAdd with acquire-release semantics at GPU scope (PTX memory model): the release
+// half publishes every write that happens-before it — the warp's lanes' record stores,
+// ordered before lane 0 by __syncwarp — and the acquire half lets the second arrival read
+// the first one's records; no full fence per tile.
+__device__ __forceinline__ uint32_t atom_add_acq_rel(uint32_t* p, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.add.acq_rel.gpu.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
+
+__device__ __forceinline__ unsigned long long atom_add_acq_rel64(unsigned long long* p, unsigned long long v) {
+  unsigned long long old;
+  asm volatile("atom.add.acq_rel.gpu.u64 %0, [%1], %2;" : "=l"(old) : "l"(p), "l"(v) : "memory");
+  return old;
+}
+
+// per-warp fused-round-0 counters in shared memory (no registers held across the walk)
+struct V0Sh {
+  unsigned long long checks, matches, ntask, reread, ztot, fm;
+  uint32_t tch, pad;
+};
+
+// The last warp of the spec kernel (all 32 lanes): commit round 0 as the verify kernel's
+// round-0 pass would, and complete the run when no recovery changed an end (then the
+// verify launch queued behind returns at once).  Lane 0 decides and clears the counters
+// for the next run; the whole warp publishes the zero-copy result (one thread would
+// serialise ~180 L2 reads).
+__device__ __noinline__ void v0_finalize(const RunParams& rp, const RecStore& rs, uint32_t lane) {
+  Ctl* ctl = rp.v0_ctl;
+  uint32_t finished = 0;
+  if (lane == 0) {
+    volatile Ctl* v = ctl;
+    volatile unsigned long long* k = rs.v0c;
+    const uint64_t N = rp.N;
+    const uint64_t f2 = k[5] ? ~k[5] : N, nt = k[2];
+    v->verify_checks = k[0];
+    v->verify_matches = k[1];
+    v->jacobi_iters = 1;
+    v->fmin = f2;
+    finished = f2 >= N;
+    if (!finished) {  // commit round 1's tasks (the must-do is chunk f2)
+      v->tasks_mustdo = 1;
+      v->tasks_sre = nt - 1;
+      v->reread_bytes = k[3];
+      v->active_sum = nt;
+      v->rounds = 1;
+      v->f = f2;
+      v->tf = __ldcg(rs.x + f2);
+      if (k[6] == 0) {  // no task moved an end: round 1 verifies every chunk from f2
+        v->verify_checks = v->verify_checks + (N - f2);
+        v->verify_matches = v->verify_matches + (N - f2);
+        v->fmin = N;
+        finished = 1;
+      }
+    }
+    if (finished) {
+      v->accept_count = k[4];
+      v->xfin = __ldcg(rs.x + N);
+    }
+    for (int i = 0; i < 8; i++) k[i] = 0;
+    if (finished) v->finished = 1;
+    __threadfence();
+  }
+  finished = __shfl_sync(0xffffffffu, finished, 0);
+  if (finished && rp.h_out) {  // zero-copy result (as the verify kernel's finalize would publish it)
+    const uint32_t* src = reinterpret_cast<const uint32_t*>(ctl);
+    uint32_t* dst = reinterpret_cast<uint32_t*>(rp.h_out);
+    for (uint32_t i = lane; i < sizeof(Ctl) / 4; i += 32) dst[i] = __ldcg(src + i);
+  }
+}
+
 // TASKS = false: round 0 (starts from the lookback pair table).  TASKS = true: a dense
 // recovery round (Alg. 3 L16-18 for many chunks at once): the round's task list
 // (rs.task_chunk / rs.task_start, ntask entries, listed by the verification pass) is
@@ -85,8 +197,10 @@ __device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, u
 // + SRE rear tasks: record to VR^end, the chunk's end moves); entries from nA on are
 // RR / NF helper tasks (Alg. 4 L23-27, Alg. 5 L19-21): record to VR^others at the
 // helper's precomputed ring position (oth_base[c] + task_j), nothing else changes.
-template <int MODE, int KP, int S, bool TASKS>
-__global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
+// up to 28 warps (896 threads, 72 registers) for <= 8 paths per lane; 16 paths (CSE with
+// spec_k 16: the whole lookback image of a 16-state convergence set) need 128 registers
+template <int MODE, int KP, int S, bool TASKS, bool V0 = false>
+__global__ void __launch_bounds__(KP > 8 ? 512 : 896, 1) k_spec_tma(const __grid_constant__ CUtensorMap tmap, DevImage img,
                                                     RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off,
                                                     uint64_t tile0, uint64_t f2, Ctl* ctl, uint64_t ntask) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -169,6 +283,9 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
   };
   for (uint64_t it = 0; it < items && it < (uint64_t)S; it++) issue_next();
 
+  constexpr bool v0 = V0 && !TASKS && KP == 1;  // fused round-0 verification compiled in
+  V0Sh* vsh = reinterpret_cast<V0Sh*>(prow + (blockDim.x / 32 - warp) * 32) + warp;  // after the prow block
+  if (v0 && lane == 0) *vsh = V0Sh{0ull, 0ull, 0ull, 0ull, 0ull, ~0ull, 0u, 0u};
   uint32_t st[KP], code[KP], acc[KP], dacc[KP], kc = 1;
   bool single = false;  // spec-k: all paths of the warp's lanes merged (path fusion, P:427 [21])
   uint64_t c = 0, tile_i = 0;
@@ -196,11 +313,11 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
 #pragma unroll
         for (int p = 0; p < KP; p++) st[p] = q0_of(rp);
       } else {
-        const uint32_t pair = qs_pair(img, rp.in, c, rp.B);
-        const uint32_t ql = __ldg(img.qs2_len + pair);
+        uint32_t ql;
+        const uint32_t* qs = qs_chunk(img, rp, c, &ql);
         kc = min(rp.k, min(ql, rp.qs_cap));
 #pragma unroll
-        for (int p = 0; p < KP; p++) st[p] = __ldg(img.qs2 + (uint64_t)pair * kQsMax + min((uint32_t)p, kc - 1));
+        for (int p = 0; p < KP; p++) st[p] = __ldg(qs + min((uint32_t)p, kc - 1));
       }
 #pragma unroll
       for (int p = 0; p < KP; p++) {
@@ -298,8 +415,74 @@ __global__ void __launch_bounds__(896, 1) k_spec_tma(const __grid_constant__ CUt
       rs.cur_end[c] = e0;
       if (c == 0) rs.x[0] = q0_of(rp);
     }
+    if (v0 && sg == segs - 1) {  // fused round-0 verification of this tile
+      const bool mine = c < n_full;
+      const uint32_t e_me = mine ? Sx::tid(img, code[0]) : 0u;
+      const uint32_t prev = __shfl_up_sync(0xffffffffu, e_me, 1);
+      uint32_t fl = 0, ct = 0;
+      uint64_t fmc = ~0ull;
+      if (mine && (lane > 0 || c == 0)) {
+        fl = v0_check<MODE>(img, table, rp, rs, c, lane > 0 ? prev : q0_of(rp), st[0], e_me, acc[0], &ct);
+        if (fl & 2u) fmc = c;
+      }
+      __syncwarp();  // the lanes' record stores happen-before lane 0's release below
+      uint32_t xc = 0, xh = 0, xt = 0, xm = 0, ct2 = 0;  // lane 0: the boundary checks it ran
+      if (lane == 0) {
+        const uint64_t t = c / 32;  // this tile
+        for (int side = 0; side < 2; side++) {
+          const uint64_t tb = t + side;  // boundary tb: between tiles tb - 1 and tb
+          const bool exists = side == 0 ? t > 0 : (t + 1) * 32 < n_full;
+          if (!exists || !(atom_add_acq_rel(rp.v0_bflag + tb, 1u) & 1u)) continue;  // first: the other checks
+          uint32_t cb = 0;
+          const uint32_t f = v0_check_global<MODE>(img, table, rp, rs, tb * 32, &cb);
+          xc++;
+          xh += f & 1u;
+          if (f & 2u) {
+            xt++;
+            fmc = min(fmc, (uint64_t)(tb * 32));
+          }
+          xm |= (f >> 2) & 1u;
+          ct2 += cb;
+        }
+      }
+      // tile totals -> the warp's shared counters (lane 0)
+      const uint32_t chk = __popc(__ballot_sync(0xffffffffu, fl != 0));
+      const uint32_t hits = __popc(__ballot_sync(0xffffffffu, fl & 1u));
+      const uint32_t tasks = __popc(__ballot_sync(0xffffffffu, (fl & 2u) != 0));
+      const uint32_t moved = __ballot_sync(0xffffffffu, (fl & 4u) != 0);
+      uint32_t zs = ct;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        zs += __shfl_down_sync(0xffffffffu, zs, o);
+        fmc = min(fmc, (uint64_t)__shfl_down_sync(0xffffffffu, (unsigned long long)fmc, o));
+      }
+      if (lane == 0) {
+        vsh->checks += chk + xc;
+        vsh->matches += hits + xh;
+        vsh->ntask += tasks + xt;
+        vsh->reread += (unsigned long long)(tasks + xt) * rp.B;
+        vsh->ztot += (unsigned long long)zs + ct2;
+        vsh->fm = min(vsh->fm, (unsigned long long)fmc);
+        vsh->tch |= (moved != 0) | xm;
+      }
+      __syncwarp();
+    }
     if (++sg == segs) { sg = 0; tile_i++; }
     if (++s == (uint32_t)S) { s = 0; phase ^= 1u; }
+  }
+  if (v0) {  // fused round 0: the warp's counters; the last warp finalises
+    uint32_t last = 0;
+    if (lane == 0) {
+      unsigned long long* k = rs.v0c;
+      const unsigned long long w[5] = {vsh->checks, vsh->matches, vsh->ntask, vsh->reread, vsh->ztot};
+      for (int i = 0; i < 5; i++)
+        if (w[i]) atomicAdd(k + i, w[i]);
+      if (vsh->fm != ~0ull) atomicMax(k + 5, ~vsh->fm);  // ~chunk: the largest is the first task chunk
+      if (vsh->tch) atomicOr(k + 6, 1ull);
+      const uint64_t warps = min(ntiles, tw);  // warps that walk tiles
+      last = atom_add_acq_rel64(k + 7, 1ull) == warps - 1;
+    }
+    if (__shfl_sync(0xffffffffu, last, 0)) v0_finalize(rp, rs, lane);
   }
   if (TASKS) {  // warp-level stats (warps may have returned early: no block barrier here)
 #pragma unroll
@@ -351,22 +534,22 @@ uint32_t pick_warps(uint64_t ntiles, int sms, uint32_t wmax) {
   return best;
 }
 
-template <int MODE, int KP, int S, bool TASKS>
+template <int MODE, int KP, int S, bool TASKS, bool V0 = false>
 cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
                          uint64_t n_full, int sms, cudaStream_t st, uint64_t tile0, uint64_t f2, Ctl* ctl,
                          uint64_t ntask) {
-  auto kern = k_spec_tma<MODE, KP, S, TASKS>;
+  auto kern = k_spec_tma<MODE, KP, S, TASKS, V0>;
   const uint64_t ntiles = TASKS ? (ntask + 31) / 32 : (n_full + 31) / 32 - tile0;
   if (ntiles == 0) return cudaSuccess;
   const uint32_t tbytes = smem_bytes_for(img);
-  const uint32_t per_warp = S * kStageBytes + S * 8 + 128;
+  const uint32_t per_warp = S * kStageBytes + S * 8 + 128 + 64;
   const uint32_t avail = 227 * 1024 - ((tbytes + 1023) & ~1023u) - 64;
-  uint32_t wmax = std::min<uint32_t>(28, avail / per_warp);  // launch bounds 896 -> 72 regs
+  uint32_t wmax = std::min<uint32_t>(KP > 8 ? 16 : 28, avail / per_warp);  // launch bounds 896 / 512
   if (wmax < 4) return cudaErrorInvalidConfiguration;
   uint32_t w = pick_warps(ntiles, sms, wmax);
   if (wmax < 8) w = wmax;
   const uint32_t table_off = (tbytes + 1023) & ~1023u;  // stages start 1 KiB-aligned (swizzle span)
-  const uint32_t smem = table_off + w * S * kStageBytes + ((w * S + 1) & ~1u) * 8 + w * 128;
+  const uint32_t smem = table_off + w * S * kStageBytes + ((w * S + 1) & ~1u) * 8 + w * 128 + w * 64;
   cudaError_t e = kernel_setup((const void*)kern, smem, (int)(w * 32), nullptr);
   if (e != cudaSuccess) return e;
   uint64_t grid = std::min<uint64_t>((uint64_t)sms, (ntiles + w - 1) / w);
@@ -384,23 +567,25 @@ cudaError_t launch_tma_t(const CUtensorMap& tm, const DevImage& img, const RunPa
   return cudaLaunchKernelEx(&cfg, kern, tm, img, rp, rs, n_full, table_off, tile0, f2, ctl, ntask);
 }
 
-template <int MODE, int KP, bool TASKS>
+template <int MODE, int KP, bool TASKS, bool V0 = false>
 cudaError_t launch_tma_s(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
                          uint64_t n_full, int sms, cudaStream_t st, uint64_t tile0, uint64_t f2, Ctl* ctl,
                          uint64_t ntask = 0) {
   const uint32_t tbytes = smem_bytes_for(img);
   if (tbytes + 24 * (3 * kStageBytes) + 2048 + 24 * 128 <= 227 * 1024)
-    return launch_tma_t<MODE, KP, 3, TASKS>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask);
-  return launch_tma_t<MODE, KP, 2, TASKS>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask);
+    return launch_tma_t<MODE, KP, 3, TASKS, V0>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask);
+  return launch_tma_t<MODE, KP, 2, TASKS, V0>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask);
 }
 
 template <int MODE>
 cudaError_t launch_tma_m(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
                          uint64_t n_full, int sms, cudaStream_t st) {
+  if (rp.k <= 1 && rp.v0) return launch_tma_s<MODE, 1, false, true>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
   if (rp.k <= 1) return launch_tma_s<MODE, 1, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
   if (rp.k <= 2) return launch_tma_s<MODE, 2, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
   if (rp.k <= 4) return launch_tma_s<MODE, 4, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
-  return launch_tma_s<MODE, 8, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
+  if (rp.k <= 8) return launch_tma_s<MODE, 8, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
+  return launch_tma_s<MODE, 16, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
 }
 
 // gather = false: box {64 B, 32 chunks} (tiles of consecutive chunks);

@@ -31,7 +31,6 @@ namespace {
 
 constexpr int kBS = 256;
 constexpr int kU = 4;  // chunks per thread whose loads are issued together (batched passes)
-constexpr uint32_t kFuseMax = 256;  // bytes walked in lockstep with the reference path
 constexpr uint32_t kNone = 0xFFFFFFFFu;
 
 __device__ __forceinline__ uint64_t ld_cg64(const uint64_t* p) { return __ldcg(reinterpret_cast<const unsigned long long*>(p)); }
@@ -185,8 +184,9 @@ __device__ __forceinline__ bool vr_lookup_cached(const VrCache& v, uint32_t i, c
 // in rs.upos[c][0..m) for the helper assignment (H2) and the cursor update.
 __device__ uint32_t untried_scan(const DevImage& img, const RunParams& rp, const RecStore& rs, uint64_t c, bool busy,
                                  uint32_t tstart) {
-  const uint32_t pair = qs_pair(img, rp.in, c, rp.B);
-  const uint32_t ql = min((uint32_t)__ldg(img.qs2_len + pair), rp.qs_cap);
+  uint32_t ql;
+  const uint32_t* qs = qs_chunk(img, rp, c, &ql);
+  ql = min(ql, rp.qs_cap);
   const uint32_t nx = __ldcg(rs.next_qs + c);
   if (nx >= ql) return 0;
   const uint32_t ne = min(ld_cg(rs.n_end + c), rp.vr_end), no = min(ld_cg(rs.n_oth + c), rp.vr_oth);
@@ -195,7 +195,7 @@ __device__ uint32_t untried_scan(const DevImage& img, const RunParams& rp, const
   for (uint32_t i = 0; i < no; i++) rec[ne + i] = ld_cg(rs.start + (uint64_t)(kVrMax + i) * rs.cap + c);
   uint32_t m = 0;
   for (uint32_t j = nx; j < ql; j++) {
-    const uint32_t q = __ldg(img.qs2 + (uint64_t)pair * kQsMax + j);
+    const uint32_t q = __ldg(qs + j);
     if (busy && q == tstart) continue;
     bool in = false;
     for (uint32_t i = 0; i < ne + no; i++) in |= rec[i] == q;
@@ -255,56 +255,6 @@ __device__ bool chain_pass(const RecStore& rs, const RunParams& rp, uint64_t c0,
   return ch;
 }
 
-// FSM_Processing over chunk c from `start` with path fusion: walk in lockstep
-// with the chunk's round-0 path; once the two states coincide the rest of the
-// path is known (DFA determinism), so end/count follow from the reference.
-template <int MODE>
-__device__ void task_walk(const DevImage& img, const uint8_t* smem, const RunParams& rp, const RecStore& rs,
-                          uint64_t c, uint32_t start, uint32_t* end_out, uint32_t* cnt_out) {
-  using S = Step<MODE>;
-  const uint64_t lo = c * rp.B, n = min((uint64_t)rp.B, rp.len - lo);
-  const uint8_t* p = rp.in + lo;
-  const uint32_t rstart = __ldcg(rs.ref_start + c);
-  const uint32_t rend = __ldcg(rs.ref_end + c), rcnt = __ldcg(rs.ref_cnt + c);
-  if (rstart == start) { *end_out = rend; *cnt_out = rcnt; return; }
-  uint32_t code = __ldg(img.tid2code + start), rcode = __ldg(img.tid2code + rstart);
-  uint32_t acc = 0, racc = 0;
-  uint64_t i = 0;
-  const bool aligned = (reinterpret_cast<uintptr_t>(p) & 15u) == 0;
-  if (aligned) {
-    const uint64_t nf = min(n, (uint64_t)kFuseMax) / 16;
-    const uint4* v = reinterpret_cast<const uint4*>(p);
-    uint4 q0 = nf > 0 ? __ldg(v) : make_uint4(0, 0, 0, 0);
-    uint4 q1 = nf > 1 ? __ldg(v + 1) : make_uint4(0, 0, 0, 0);
-    for (uint64_t j = 0; j < nf; j++) {
-      const uint4 q = q0;
-      q0 = q1;
-      if (j + 2 < nf) q1 = __ldg(v + j + 2);
-      uint32_t w[4] = {q.x, q.y, q.z, q.w};
-#pragma unroll
-      for (int t = 0; t < 4; t++) {
-        code = S::template word<0>(img, smem, code, w[t]); acc += S::acc(code);
-        rcode = S::template word<0>(img, smem, rcode, w[t]); racc += S::acc(rcode);
-        code = S::template word<1>(img, smem, code, w[t]); acc += S::acc(code);
-        rcode = S::template word<1>(img, smem, rcode, w[t]); racc += S::acc(rcode);
-        code = S::template word<2>(img, smem, code, w[t]); acc += S::acc(code);
-        rcode = S::template word<2>(img, smem, rcode, w[t]); racc += S::acc(rcode);
-        code = S::template word<3>(img, smem, code, w[t]); acc += S::acc(code);
-        rcode = S::template word<3>(img, smem, rcode, w[t]); racc += S::acc(rcode);
-      }
-      if (code == rcode) {  // merged somewhere in these 16 bytes: identical from here on
-        *end_out = rend;
-        *cnt_out = rcnt - racc + acc;
-        return;
-      }
-    }
-    i = nf * 16;
-  }
-  code = walk_bytes<MODE>(img, smem, p + i, n - i, code, acc);
-  *end_out = S::tid(img, code);
-  *cnt_out = acc;
-}
-
 template <int MODE>
 __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
                                                         uint64_t* btmp, uint32_t* chunk_ends, uint32_t cache_cap) {
@@ -319,6 +269,9 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
   auto stamp = [&]() {
     if (blockIdx.x == 0 && threadIdx.x == 0 && nst < 24) { ctl->stamp[nst++] = gtimer(); ctl->nstamp = nst; }
   };
+  // fused round 0 completed the run in the spec kernel (without PDL the spec kernel is done
+  // here; with PDL a 0 read falls through to the authoritative check after the wait)
+  if (rp.v0 && *reinterpret_cast<volatile uint32_t*>(&ctl->finished)) return;
   if (rp.stamps && blockIdx.x == 0 && threadIdx.x == 0 && ctl->tl[2] == 0) ctl->tl[2] = gtimer();
   stage_table(img, smem);  // the table is load-time data: staged before the dependency wait
   pdl_wait();               // the spec kernel's records are complete and visible
@@ -765,9 +718,10 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
             ok = j < __ldcg(rs.ulen + c);
           }
           if (ok) {  // the j-th untried candidate of chunk c (positions listed in phase T)
-            const uint32_t pair = qs_pair(img, rp.in, c, rp.B);
+            uint32_t ql;
+            const uint32_t* qs = qs_chunk(img, rp, c, &ql);
             cid = (uint32_t)c;
-            st = __ldg(img.qs2 + (uint64_t)pair * kQsMax + __ldcg(rs.upos + c * kQsMax + j));
+            st = __ldg(qs + __ldcg(rs.upos + c * kQsMax + j));
           }
         }
         rs.task_chunk[nA + k] = cid;

@@ -348,6 +348,58 @@ __device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, u
   return vr_resolve(vr_prefetch(rs, c, cnt != nullptr), rs, vr_end, vr_oth, c, x, end, cnt);
 }
 
+// FSM_Processing over chunk c from `start` with path fusion: walk in lockstep
+// with the chunk's round-0 path; once the two states coincide the rest of the
+// path is known (DFA determinism), so end/count follow from the reference.
+constexpr uint32_t kFuseMax = 256;  // bytes walked in lockstep with the reference path
+
+template <int MODE>
+__device__ __noinline__ void task_walk(const DevImage& img, const uint8_t* smem, const RunParams& rp, const RecStore& rs,
+                          uint64_t c, uint32_t start, uint32_t* end_out, uint32_t* cnt_out) {
+  using S = Step<MODE>;
+  const uint64_t lo = c * rp.B, n = min((uint64_t)rp.B, rp.len - lo);
+  const uint8_t* p = rp.in + lo;
+  const uint32_t rstart = __ldcg(rs.ref_start + c);
+  const uint32_t rend = __ldcg(rs.ref_end + c), rcnt = __ldcg(rs.ref_cnt + c);
+  if (rstart == start) { *end_out = rend; *cnt_out = rcnt; return; }
+  uint32_t code = __ldg(img.tid2code + start), rcode = __ldg(img.tid2code + rstart);
+  uint32_t acc = 0, racc = 0;
+  uint64_t i = 0;
+  const bool aligned = (reinterpret_cast<uintptr_t>(p) & 15u) == 0;
+  if (aligned) {
+    const uint64_t nf = min(n, (uint64_t)kFuseMax) / 16;
+    const uint4* v = reinterpret_cast<const uint4*>(p);
+    uint4 q0 = nf > 0 ? __ldg(v) : make_uint4(0, 0, 0, 0);
+    uint4 q1 = nf > 1 ? __ldg(v + 1) : make_uint4(0, 0, 0, 0);
+    for (uint64_t j = 0; j < nf; j++) {
+      const uint4 q = q0;
+      q0 = q1;
+      if (j + 2 < nf) q1 = __ldg(v + j + 2);
+      uint32_t w[4] = {q.x, q.y, q.z, q.w};
+#pragma unroll
+      for (int t = 0; t < 4; t++) {
+        code = S::template word<0>(img, smem, code, w[t]); acc += S::acc(code);
+        rcode = S::template word<0>(img, smem, rcode, w[t]); racc += S::acc(rcode);
+        code = S::template word<1>(img, smem, code, w[t]); acc += S::acc(code);
+        rcode = S::template word<1>(img, smem, rcode, w[t]); racc += S::acc(rcode);
+        code = S::template word<2>(img, smem, code, w[t]); acc += S::acc(code);
+        rcode = S::template word<2>(img, smem, rcode, w[t]); racc += S::acc(rcode);
+        code = S::template word<3>(img, smem, code, w[t]); acc += S::acc(code);
+        rcode = S::template word<3>(img, smem, rcode, w[t]); racc += S::acc(rcode);
+      }
+      if (code == rcode) {  // merged somewhere in these 16 bytes: identical from here on
+        *end_out = rend;
+        *cnt_out = rcnt - racc + acc;
+        return;
+      }
+    }
+    i = nf * 16;
+  }
+  code = walk_bytes<MODE>(img, smem, p + i, n - i, code, acc);
+  *end_out = S::tid(img, code);
+  *cnt_out = acc;
+}
+
 __device__ __forceinline__ uint64_t gtimer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -375,6 +427,20 @@ __device__ __forceinline__ uint32_t qs_pair(const DevImage& img, const uint8_t* 
   uint64_t e = c * (uint64_t)B;
   uint32_t a = __ldg(in + e - 2), b = __ldg(in + e - 1);
   return (uint32_t)__ldg(img.cls + a) * img.C + __ldg(img.cls + b);
+}
+
+// QS_c of chunk c >= 1: the lookback-2 pair table, or — with a longer lookback
+// (fsm_run_opts.lookback > 2, reading R25) — the per-run table rp.qsc built by
+// k_qs_long.  Returns the ranked candidates; *ql = their number (<= kQsMax).
+__device__ __forceinline__ const uint32_t* qs_chunk(const DevImage& img, const RunParams& rp, uint64_t c,
+                                                    uint32_t* ql) {
+  if (rp.qsc) {
+    *ql = __ldg(rp.qsc_len + c);
+    return rp.qsc + c * kQsMax;
+  }
+  const uint32_t pair = qs_pair(img, rp.in, c, rp.B);
+  *ql = __ldg(img.qs2_len + pair);
+  return img.qs2 + (uint64_t)pair * kQsMax;
 }
 
 }  // namespace gspec

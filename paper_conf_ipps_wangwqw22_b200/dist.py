@@ -53,9 +53,11 @@ def _all_gather_cat(t, group=None):
     return torch.cat(parts).to(t.device)
 
 
-def exchange_lookback(shard, group=None, L: int = 2):
+def exchange_lookback(shard, group=None, L: int = 16):
     """The last L (<= 16) bytes of the stream before this rank's shard (tiny allgather of
-    every rank's tail).  They come from the nearest preceding non-empty shards: a shard
+    every rank's tail).  The shard's candidate start set is the image of all states over
+    them; a longer window can only shrink it (delta*(Q, uv) is a subset of
+    delta*(Q, v)), so the default takes the 16 bytes fsm_shard_map accepts.  They come from the nearest preceding non-empty shards: a shard
     shorter than L (or empty, when there are fewer chunks than ranks) contributes what it
     has and the ranks before it the rest.  Empty only for a shard that starts the stream."""
     import torch

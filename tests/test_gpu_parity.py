@@ -552,3 +552,56 @@ def test_selector_spread_profile(gs, name):
     assert res.scheme == pick
     del x
     torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("name,length,B", [("c2", 4 << 20, 4096), ("c3", 4 << 20, 4096), ("c4", 2 << 20, 4096),
+                                           ("rand:40:7:3", 300000, 48), ("rand:150:3:9", 200000, 64),
+                                           ("c1", 1 << 18, 1024), ("c3", (3 << 20) + 555, 2048)])
+@pytest.mark.parametrize("scheme,L", [("sre", 3), ("sre", 16), ("rr", 8), ("nf", 5), ("pm", 16), ("cse", 8),
+                                      ("pm_tree", 4)])
+def test_lookback_long(gs, name, length, B, scheme, L):
+    """Lookback over L > 2 symbols (reading R25: per-chunk QS from the pair image
+    with multiplicities walked over the extra symbols, k_qs_long): bit-exact results and
+    round diagnostics equal to the oracle's simulation with the same lookback."""
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    fsm = _fsm(gs, w)
+    res = fsm.run(torch.from_numpy(data).cuda(), scheme=scheme, chunk_bytes=B, lookback=L)
+    check_equal(res, ref, B, w.nstates)
+    if scheme == "pm_tree":
+        return
+    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme=scheme, lookback=L)
+    for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks",
+              "verify_matches"):
+        assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+
+
+def test_lookback_long_wide_fallback(gs):
+    """A permutation DFA (every 2-symbol image has all 100 states > 64): lookback 8 keeps
+    the lookback-2 ranking (R25), exactly as the oracle does."""
+    t, s, a = _perm_dfa(100, 3, 5)
+    rng = np.random.default_rng(5)
+    data = rng.integers(0, 3, 20 * 4096).astype(np.uint8)
+    ref = oracle.run(t, s, a, data, 1024)
+    fsm = gs.FSM.load(t, s, a)
+    res = fsm.run(torch.from_numpy(data).cuda(), scheme="sre", chunk_bytes=1024, lookback=8)
+    check_equal(res, ref, 1024, 100)
+    sim = oracle.simulate(t, s, a, data, 1024, scheme="sre", lookback=8)
+    sim2 = oracle.simulate(t, s, a, data, 1024, scheme="sre", lookback=2)
+    assert res.stats["verify_matches"] == sim["verify_matches"] == sim2["verify_matches"]
+
+
+@pytest.mark.parametrize("name,length,B,k", [("c3", 8 << 20, 4096, 16), ("c1", 1 << 20, 4096, 16),
+                                             ("c2", 4 << 20, 4096, 12), ("rand:60:5:2", 300000, 64, 16)])
+def test_cse_spec16(gs, name, length, B, k):
+    """CSE with up to 16 paths per chunk (the whole lookback image of C3's
+    16-value counter; the 16-path TMA kernel runs 16 warps of 128 registers): exact, and
+    its rounds equal the oracle's simulation with the same spec_k."""
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    fsm = _fsm(gs, w)
+    res = fsm.run(torch.from_numpy(data).cuda(), scheme="cse", chunk_bytes=B, spec_k=k)
+    check_equal(res, ref, B, w.nstates)
+    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme="cse", spec_k=k)
+    for key in ("rounds", "tasks_mustdo", "tasks_sre", "reread_bytes", "verify_checks", "verify_matches"):
+        assert res.stats[key] == sim[key], (key, res.stats[key], sim[key])

@@ -11,7 +11,7 @@ pytestmark = pytest.mark.gpu
 torch = pytest.importorskip("torch")
 
 
-def sharded_fake(gs, w, data, G, B=4096, scheme="auto"):
+def sharded_fake(gs, w, data, G, B=4096, scheme="auto", L=2):
     from paper_conf_ipps_wangwqw22_b200 import _check, _lib, _run_opts, fsm_result
     from paper_conf_ipps_wangwqw22_b200.dist import shard_bounds
     import ctypes
@@ -27,7 +27,7 @@ def sharded_fake(gs, w, data, G, B=4096, scheme="auto"):
         for g, (lo, hi) in enumerate(bounds):
             n = gs.fsm_num_chunks(hi - lo, B)
             ce = torch.full((max(n, 1),), -1, dtype=torch.int32, device="cuda")
-            lb = x[max(0, lo - 2):lo] if g else None
+            lb = x[max(0, lo - L):lo] if g else None
             fn = _lib.fsm_shard_map_exact if exact else _lib.fsm_shard_map
             _check(fn(fsms[g].handle, x[lo:].data_ptr() if hi > lo else None, hi - lo,
                       lb.data_ptr() if lb is not None else None, 0 if lb is None else lb.numel(),
@@ -56,12 +56,14 @@ def gs():
 
 @pytest.mark.parametrize("name,length", [("c1", 1 << 20), ("c2", 8 << 20), ("c3", 4 << 20), ("c3s", 2 << 20),
                                          ("c4", 4 << 20), ("rand:40:3:5", 300000), ("rand:300:7:2", 200000)])
-@pytest.mark.parametrize("G", [1, 2, 3, 8])
-def test_fake_collective(gs, name, length, G):
+@pytest.mark.parametrize("G,L", [(1, 2), (2, 2), (3, 2), (8, 2), (3, 16), (8, 16)])
+def test_fake_collective(gs, name, length, G, L):
+    """L = bytes before each shard whose lookback image is its candidate start set:
+    16 gives the smallest sets (a subset of the 2-byte image)."""
     w = gen.workload(name, length=length)
     data = w.host()
     ref = oracle.run(w.table, w.start, w.accept, data, 4096)
-    outs, ce = sharded_fake(gs, w, data, G)
+    outs, ce = sharded_fake(gs, w, data, G, L=L)
     for r in outs:
         assert r.final_state == ref["final"] and r.accept_count == ref["count"]
         assert bool(r.accept) == bool(ref["accept"])

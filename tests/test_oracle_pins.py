@@ -283,6 +283,58 @@ def test_lookback_containment(seed):
     assert list(qs) == expect
 
 
+@pytest.mark.parametrize("seed", range(4))
+def test_lookback_long(seed):
+    """Lookback over L in [2, 16] symbols (reading R25): the true start is in the
+    image (containment) for every L; the image over the last L symbols is a subset of the
+    image over the last 2 (delta*(Q, uv) is a subset of delta*(Q, v)); the ranking is the
+    brute-force multiplicity ranking over all states; a DFA whose 2-symbol images exceed 64
+    states (a permutation DFA) falls back to the lookback-2 ranking of the last two symbols."""
+    rng = random.Random(seed + 100)
+    n, ns = rng.randint(2, 40), rng.randint(1, 6)
+    t, s, a = gen.dfa_random(seed + 77, n, ns)
+    data = gen.workload(f"rand:{n}:{ns}:{seed}", length=4000, seed=seed).host()
+    B = 64
+    r = oracle.run(t, s, a, data, B)
+    for L in (2, 3, 5, 9, 16):
+        for c in range(1, oracle.nchunks(len(data), B)):
+            w = data[c * B - L:c * B]
+            qs, img = oracle.lookback_long(t, n, w, K=n)
+            q2, img2 = oracle.lookback(t, n, w[-2:], K=n)
+            assert r["chunk_end"][c - 1] in set(qs.tolist())
+            assert set(qs.tolist()) <= set(q2.tolist()) and img <= img2
+            if c % 7 == 0:  # brute force ranking
+                mult = {}
+                for q in range(n):
+                    e = q
+                    for ch in w:
+                        e = int(t[e, ch])
+                    mult[e] = mult.get(e, 0) + 1
+                assert list(qs) == sorted(mult, key=lambda e: (-mult[e], e))
+    rng2 = np.random.default_rng(seed)
+    nperm = 100
+    tp = np.stack([rng2.permutation(nperm) for _ in range(3)], axis=1).astype(np.uint32)
+    w = np.array([0, 1, 2, 1, 0, 2], np.uint8)
+    qs, img = oracle.lookback_long(tp, nperm, w, K=16)
+    q2, img2 = oracle.lookback(tp, nperm, w[-2:], K=16)
+    assert list(qs) == list(q2) and img == img2 == nperm
+
+
+@pytest.mark.parametrize("scheme", ["sre", "rr", "pm", "cse"])
+@pytest.mark.parametrize("L", [3, 8, 16])
+def test_simulate_lookback_long(scheme, L):
+    """Every scheme with a longer lookback still reaches the sequential result."""
+    rng = random.Random(L)
+    n, ns = rng.randint(2, 30), rng.randint(2, 5)
+    t, s, a = gen.dfa_random(L + 3, n, ns)
+    data = gen.workload(f"rand:{n}:{ns}:{L}", length=30000, seed=L).host()
+    for B in (16, 64):
+        r = oracle.run(t, s, a, data, B)
+        o = oracle.simulate(t, s, a, data, B, scheme=scheme, lookback=L)
+        assert o["status"] == 0 and o["final_state"] == r["final"] and o["accept_count"] == r["count"]
+        assert (o["chunk_end"] == r["chunk_end"]).all()
+
+
 # ----------------------------------------------------------- simulate -------
 @pytest.mark.parametrize("scheme", ["seq", "pm", "sre", "rr", "nf", "cse"])
 @pytest.mark.parametrize("seed", range(6))
