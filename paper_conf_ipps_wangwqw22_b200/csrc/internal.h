@@ -183,12 +183,15 @@ inline bool stamps_enabled() {
 // previous grid's completion and memory flush.  Opt-in (GSPEC_PDL=1): measured on
 // c2 it does not shorten the step (0.3237 vs 0.3232 ms) — the verify CTAs cannot
 // become resident before the spec CTAs (full shared memory) exit.
-// GSPEC_V0=0 turns the fused round-0 verification off (A/B measurements).
+// Fused round-0 verification in the spec kernel (RunParams::v0): opt-in, GSPEC_V0=1.
+// Measured neutral on C2 (spec kernel +16 us, verify launch -16 us: 3446 vs 3447 GB/s) and
+// slightly slower on C4 (3.34 vs 3.29 ms: the per-tile epilogue competes with the walk for
+// issue and LSU slots), so the separate verify kernel stays the default.
 inline bool v0_disabled() {
   static int v = -1;
   if (v < 0) {
     const char* e = getenv("GSPEC_V0");
-    v = (e && atoi(e) == 0) ? 1 : 0;
+    v = (e && atoi(e) == 1) ? 0 : 1;
   }
   return v != 0;
 }

@@ -86,7 +86,7 @@ __device__ __forceinline__ void tma_gather4(void* dst, const CUtensorMap* map, u
 // Returns bit 0 = hit, bit 1 = recovered (a task ran), bit 2 = the task moved the end;
 // *cnt = the chunk's accept count on the true path (round-0 count, or the task's).
 template <int MODE>
-__device__ __noinline__ uint32_t v0_check(const DevImage& img, const uint8_t* table, const RunParams& rp,
+__device__ __forceinline__ uint32_t v0_check(const DevImage& img, const uint8_t* table, const RunParams& rp,
                                           const RecStore& rs, uint64_t c, uint32_t xin, uint32_t s0, uint32_t xo,
                                           uint32_t c0, uint32_t* cnt_out) {
   const bool hit = xin == s0;
@@ -144,7 +144,7 @@ struct V0Sh {
 // verify launch queued behind returns at once).  Lane 0 decides and clears the counters
 // for the next run; the whole warp publishes the zero-copy result (one thread would
 // serialise ~180 L2 reads).
-__device__ __noinline__ void v0_finalize(const RunParams& rp, const RecStore& rs, uint32_t lane) {
+__device__ __forceinline__ void v0_finalize(const RunParams& rp, const RecStore& rs, uint32_t lane) {
   Ctl* ctl = rp.v0_ctl;
   uint32_t finished = 0;
   if (lane == 0) {

@@ -354,7 +354,7 @@ __device__ __forceinline__ bool vr_lookup(const RecStore& rs, uint32_t vr_end, u
 constexpr uint32_t kFuseMax = 256;  // bytes walked in lockstep with the reference path
 
 template <int MODE>
-__device__ __noinline__ void task_walk(const DevImage& img, const uint8_t* smem, const RunParams& rp, const RecStore& rs,
+__device__ __forceinline__ void task_walk(const DevImage& img, const uint8_t* smem, const RunParams& rp, const RecStore& rs,
                           uint64_t c, uint32_t start, uint32_t* end_out, uint32_t* cnt_out) {
   using S = Step<MODE>;
   const uint64_t lo = c * rp.B, n = min((uint64_t)rp.B, rp.len - lo);

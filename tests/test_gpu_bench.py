@@ -39,3 +39,15 @@ def test_bench_c5_line(gpus):
         ref = oracle.run(w.table, w.start, w.accept, w.host(), 4096)
         assert r["final_state"] == ref["final"] and r["accept_count"] == ref["count"], name
         assert r["scheme"] == {"c1": "enum", "c2": "sre", "c3": "sre", "c4": "sre"}[name]
+
+
+def test_fused_round0_verification_path():
+    """The opt-in fused round-0 verification (GSPEC_V0=1, read once per process: run the
+    oracle-parity tests of the SRE round-0 path in a child process with it on)."""
+    e = dict(os.environ)
+    e["GSPEC_V0"] = "1"
+    out = subprocess.run([sys.executable, "-m", "pytest", os.path.join(ROOT, "tests", "test_gpu_parity.py"), "-q",
+                          "-p", "no:cacheprovider", "-k", "inline_round0 or full_size_bench or edge_lengths or async"],
+                         capture_output=True, text=True, timeout=900, env=e, cwd=ROOT)
+    assert out.returncode == 0, out.stdout[-3000:] + out.stderr[-2000:]
+    assert " passed" in out.stdout

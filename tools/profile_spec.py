@@ -14,7 +14,7 @@ w.device(x)
 prof = torch.empty(1 << 20, dtype=torch.uint8, device='cuda')
 w.device(prof, offset=w.length)  # disjoint training trace, as bench.py
 fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof.cpu().numpy())
-fsm.select_scheme(x[: 1 << 20])  # as bench.py: the profile gates the dense-round slots (none for accurate DFAs)
+fsm.select_scheme(x)  # as bench.py (spread profile, R20): gates the dense-round slots and the fused round 0
 for i in range(reps):
     r = fsm.run(x, scheme=scheme)
 torch.cuda.synchronize()
