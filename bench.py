@@ -365,6 +365,32 @@ def per_dfa_result(gs, name, args, peak, peak_kind, with_cpu=True):
     return out
 
 
+def async_sharded_steps(gs, comm, fsm, x, lb, scheme, B, ce, k, window=16):
+    """k sharded steps queued back to back (fsm_run_sharded_async: map, ncclAllGather and
+    finish without a host wait), collected window by window; returns the last result.  A
+    step that reports FSM_EAGAIN (a speculative shard map was invalid) is redone
+    synchronously, as every rank sees the same EAGAIN."""
+    res, pend = None, []
+
+    def drain():
+        nonlocal res
+        for t in pend:
+            try:
+                res = gs.Comm.wait(fsm, t)
+            except gs.GSpecError as e:
+                if e.status != gs.FSM_EAGAIN:
+                    raise
+                res = comm.run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
+        pend.clear()
+
+    for _ in range(k):
+        pend.append(comm.run_sharded_async(fsm, x, lb, scheme=scheme, chunk_bytes=B, chunk_ends=ce))
+        if len(pend) >= window:
+            drain()
+    drain()
+    return res
+
+
 def _maybe_relaunch(args):
     """--gpus N > 1 without a torch.distributed launcher: re-run this command under
     torch.distributed.run (one process per GPU, rendezvous on 127.0.0.1)."""
@@ -421,6 +447,7 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         res = None
         for _ in range(max(3, args.warmup)):
             res = step()
+        ce = torch.empty(max(1, gs.fsm_num_chunks(x.numel(), B)), dtype=torch.int32, device="cuda")
         if dist:
             dist.barrier()
         torch.cuda.synchronize()
@@ -428,8 +455,11 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         with ClockSampler(dev) as clk:
             ev0.record(stream)
-            for _ in range(args.steps):
-                res = step()
+            if comm is not None:  # steps queued back to back: no host wait between them
+                res = async_sharded_steps(gs, comm, fsm, x, lb, scheme, B, ce, args.steps)
+            else:
+                for _ in range(args.steps):
+                    res = step()
             ev1.record(stream)
             torch.cuda.synchronize()
         if clk_all is None:
@@ -579,14 +609,18 @@ def main():
         kr = [fsm.run(x, scheme=scheme, chunk_bytes=B) for _ in range(3)]
         for _ in range(max(3, args.warmup)):
             res = step()
+        ce_sh = torch.empty(max(1, gs.fsm_num_chunks(length, B)), dtype=torch.int32, device="cuda")
         dist.barrier()
         torch.cuda.synchronize()
         stream = torch.cuda.current_stream()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         with ClockSampler(dev) as clk:
             ev0.record(stream)
-            for _ in range(args.steps):
-                res = step()
+            if comm is not None:  # steps queued back to back: no host wait between them
+                res = async_sharded_steps(gs, comm, fsm, x, lb, scheme, B, ce_sh, args.steps)
+            else:
+                for _ in range(args.steps):
+                    res = step()
             ev1.record(stream)
             torch.cuda.synchronize()
         dist.barrier()

@@ -38,7 +38,7 @@ typedef enum {
   FSM_ECUDA = -3,        /* CUDA runtime error (message in fsm_last_error)     */
   FSM_ESYMBOL = -4,      /* an input byte >= nsyms (reading R4); outputs unset  */
   FSM_ENCCL = -5,        /* collective failed                                  */
-  FSM_EUNSUPPORTED = -6, /* e.g. ENUM on a DFA with > 31 states                */
+  FSM_EUNSUPPORTED = -6, /* e.g. ENUM on a DFA with > 63 states                */
   FSM_EAGAIN = -7        /* fsm_shard_finish: a rank's speculative shard map was
                             invalid; every rank redoes fsm_shard_map_exact + the
                             exchange + fsm_shard_finish (all ranks see the same maps) */
@@ -142,7 +142,7 @@ uint64_t fsm_num_chunks(uint64_t len, uint32_t chunk_bytes);
  * ids: the state after each chunk's last symbol.  opts nullable (defaults).
  * Errors: FSM_EINVAL (bad opts, NULL input with len > 0), FSM_ESYMBOL (an input
  * byte >= nsyms; detected through the absorbing poison state), FSM_ENOMEM,
- * FSM_ECUDA, FSM_EUNSUPPORTED (ENUM with nstates > 31). */
+ * FSM_ECUDA, FSM_EUNSUPPORTED (ENUM with nstates > 63). */
 int fsm_run(fsm_t fsm, const uint8_t* d_input, uint64_t len, const fsm_run_opts* opts,
             uint32_t* d_chunk_ends, fsm_result* out);
 
@@ -267,6 +267,16 @@ int fsm_shard_map_exact(fsm_t fsm, const uint8_t* d_shard, uint64_t len, const u
 int fsm_shard_finish(fsm_t fsm, const void* d_maps, uint32_t nranks, uint32_t rank,
                      const fsm_run_opts* opts, uint32_t* d_chunk_ends_local, fsm_result* out_global);
 
+/* Asynchronous step 2: queues the composition and the fix-up on opts->stream and
+ * returns a ticket at once (the host fix-up modes of non-merging shards finish here and
+ * the ticket carries the outcome); fsm_shard_wait blocks until that step is done and
+ * fills *out.  Steps on one handle may be queued back to back (up to 32 in flight), so
+ * the host never stalls the GPU between steps.  FSM_EAGAIN from the wait: redo the step
+ * synchronously (fsm_run_sharded / fsm_shard_map_exact) on every rank. */
+int fsm_shard_finish_async(fsm_t fsm, const void* d_maps, uint32_t nranks, uint32_t rank,
+                           const fsm_run_opts* opts, uint32_t* d_chunk_ends_local, uint64_t* ticket);
+int fsm_shard_wait(fsm_t fsm, uint64_t ticket, fsm_result* out);
+
 /* ---- library-owned NCCL path (callers without torch.distributed) -------------
  * fsm_comm_unique_id (one rank, 128 bytes, share out of band) -> fsm_comm_init
  * on every rank (one GPU each) -> fsm_run_sharded = fsm_shard_map + one
@@ -278,6 +288,11 @@ int fsm_comm_init(int nranks, int rank, const void* unique_id, fsm_comm_t* out);
 int fsm_run_sharded(fsm_t fsm, fsm_comm_t comm, const uint8_t* d_shard, uint64_t shard_len,
                     const uint8_t* d_lookback, uint32_t lookback_len, const fsm_run_opts* opts,
                     uint32_t* d_chunk_ends_local, fsm_result* out_global);
+/* fsm_run_sharded without the host wait: map + ncclAllGather + fsm_shard_finish_async;
+ * collect with fsm_shard_wait(fsm, ticket, out). */
+int fsm_run_sharded_async(fsm_t fsm, fsm_comm_t comm, const uint8_t* d_shard, uint64_t shard_len,
+                          const uint8_t* d_lookback, uint32_t lookback_len, const fsm_run_opts* opts,
+                          uint32_t* d_chunk_ends_local, uint64_t* ticket);
 void fsm_comm_free(fsm_comm_t comm);
 
 /* ---- introspection (tests) ------------------------------------------------- */

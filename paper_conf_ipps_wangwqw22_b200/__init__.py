@@ -24,6 +24,7 @@ if not os.path.exists(_LIB_PATH):
 _lib = ctypes.CDLL(_LIB_PATH)
 
 FSM_OK, FSM_EINVAL, FSM_ENOMEM, FSM_ECUDA, FSM_ESYMBOL, FSM_ENCCL, FSM_EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
+FSM_EAGAIN = -7
 SCHEMES = {"auto": 0, "seq": 1, "pm": 2, "sre": 3, "rr": 4, "nf": 5, "enum": 6, "cse": 7, "pm_tree": 8}
 SCHEME_NAMES = {v: k for k, v in SCHEMES.items()}
 MODES = {1: "u8", 2: "u16", 3: "u32", 4: "u16d"}
@@ -91,6 +92,9 @@ _lib.fsm_get_timeline.argtypes = [P, P]
 _lib.fsm_comm_unique_id.argtypes = [P]
 _lib.fsm_comm_init.argtypes = [ctypes.c_int, ctypes.c_int, P, ctypes.POINTER(P)]
 _lib.fsm_run_sharded.argtypes = [P, P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
+_lib.fsm_run_sharded_async.argtypes = [P, P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(U64)]
+_lib.fsm_shard_finish_async.argtypes = [P, P, U32, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(U64)]
+_lib.fsm_shard_wait.argtypes = [P, U64, ctypes.POINTER(fsm_result)]
 _lib.fsm_comm_free.argtypes = [P]
 _lib.fsm_comm_free.restype = None
 _lib.fsm_free.argtypes = [P]
@@ -375,6 +379,28 @@ class Comm:
                                     ctypes.byref(o), ce.data_ptr() if ce is not None else None, ctypes.byref(r)),
                "fsm_run_sharded")
         return Result.from_c(r, ce[:n] if ce is not None else None)
+
+    def run_sharded_async(self, fsm: "FSM", shard, lookback=None, scheme="auto", chunk_bytes=4096, spec_k=0,
+                          chunk_ends=None, stream=None) -> int:
+        """fsm_run_sharded_async: queue one sharded step (map, ncclAllGather, finish) without a
+        host wait; returns a ticket for wait().  chunk_ends: an int32 CUDA tensor or None."""
+        o = _run_opts(scheme, chunk_bytes, spec_k, stream=stream)
+        lb = lookback if lookback is not None and lookback.numel() else None
+        t = U64(0)
+        _check(_lib.fsm_run_sharded_async(fsm.handle, self._h, shard.data_ptr() if shard.numel() else None,
+                                          shard.numel(), lb.data_ptr() if lb is not None else None,
+                                          lb.numel() if lb is not None else 0, ctypes.byref(o),
+                                          chunk_ends.data_ptr() if chunk_ends is not None else None,
+                                          ctypes.byref(t)), "fsm_run_sharded_async")
+        return t.value
+
+    @staticmethod
+    def wait(fsm: "FSM", ticket: int) -> Result:
+        """fsm_shard_wait: block until a queued sharded step is done (GSpecError FSM_EAGAIN:
+        redo the step with run_sharded on every rank)."""
+        r = fsm_result()
+        _check(_lib.fsm_shard_wait(fsm.handle, ticket, ctypes.byref(r)), "fsm_shard_wait")
+        return Result.from_c(r)
 
     def close(self):
         if self._h:

@@ -332,7 +332,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   if (scheme == FSM_SCHEME_ENUM) {
     if (f->n + 1 > kEnumMax) {
       pd.active = false;
-      return fail(FSM_EUNSUPPORTED, "ENUM needs nstates + 1 <= 32");
+      return fail(FSM_EUNSUPPORTED, "ENUM needs nstates + 1 <= 64");
     }
     // sub-chunk size E | B: small enough for parallelism, bounded scratch.  A stream of at
     // most enum_small_max_sub() sub-chunks of >= 64 B runs as ONE launch (k_enum_small)
@@ -340,7 +340,8 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     while (Es % 32 == 0 && Es > 64 && (len + Es / 2 - 1) / (Es / 2) <= enum_small_max_sub()) Es /= 2;
     // (only for short sub-chunks: 8192 threads walking long sub-chunks would be latency-bound;
     // longer streams keep the multi-level scan with many more threads)
-    const bool small = len > 0 && Es <= 256 && (len + Es - 1) / Es <= enum_small_max_sub();
+    const bool small = len > 0 && Es <= 256 && (len + Es - 1) / Es <= enum_small_max_sub() &&
+                       f->n + 1 <= kEnumSmallMax;
     const uint32_t E = small ? Es : enum_sub_bytes(o.B, len);
     const uint64_t nsub = (len + E - 1) / E;
     const uint64_t need = small ? enum_small_scratch_bytes(nsub) : enum_scratch_bytes(nsub);
@@ -427,6 +428,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       rp.v0_ctl = f->d_ctl;
       rp.v0_bflag = f->rs.bflag;
       rp.v0_chunk_ends = d_chunk_ends;
+      rp.tma_evict_normal = tma_evict_mode() == 1 ? 1u : 0u;
       NvtxRange nv_("speculative execution (round 0)");
       CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
     }
@@ -606,7 +608,7 @@ bool plan_delta_rows(fsm_t f, const std::vector<uint32_t>& ttc, uint32_t nt, uin
 
 fsm_scheme tree_select(const fsm_features& ft, uint32_t n) {
   // Fig. 6 (image lost) reconstructed from P:284-290, P:339-345, P:383 (R19)
-  if (n <= 31 && ft.uniq10 >= n / 2.0) return FSM_SCHEME_ENUM;
+  if (n <= 63 && ft.uniq10 >= n / 2.0) return FSM_SCHEME_ENUM;  // n + poison <= 64 map entries
   if (ft.uniq10 <= 4.0) return FSM_SCHEME_SRE;
   if (ft.acck >= 0.9 && ft.acck - ft.acc1 >= 0.2) return FSM_SCHEME_PM;
   // R19b: helpers cost a full chunk walk on a saturated GPU; RR/NF only when the
@@ -875,6 +877,9 @@ void fsm_free(fsm_t f) {
   if (f->prof_buf) cudaFree(f->prof_buf);
   if (f->img2_base) cudaFree(f->img2_base);
   if (f->qsc_base) cudaFree(f->qsc_base);
+  if (f->h_sh) cudaFreeHost(f->h_sh);
+  for (auto& e : f->sh_ev)
+    if (e) cudaEventDestroy(e);
   for (auto& e : f->multi_ev)
     if (e) cudaEventDestroy(e);
   delete f;
@@ -1694,6 +1699,95 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
   out->final_state = f->inv[fin];
   out->accept = f->accept[out->final_state];
   out->accept_count = count;
+  return FSM_OK;
+}
+
+// Asynchronous finish (stream-ordered): in the fused mode the composition, the prefix
+// fix-up and a copy of the 6 result words into a pinned ring slot are queued and the call
+// returns a ticket at once; the modes whose fix-up runs on the host finish synchronously
+// (the ticket then carries the outcome).  fsm_shard_wait blocks for a ticket and decodes.
+int fsm_shard_finish_async(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, const fsm_run_opts* opts,
+                           uint32_t* d_chunk_ends_local, uint64_t* ticket) {
+  ApiScope api_scope_("fsm_shard_finish_async");
+  if (!f || !d_maps || !ticket || rank >= G) return fail(FSM_EINVAL, "bad finish arguments");
+  if (f->shard_mode < 0) return fail(FSM_EINVAL, "fsm_shard_map was not called");
+  Opts o;
+  int rc = resolve_opts(opts, &o);
+  if (rc) return rc;
+  if (!f->h_sh) {
+    CUDA_TRY(cudaMallocHost(&f->h_sh, fsm_s::kRing * 8 * sizeof(uint32_t)));
+    for (auto& e : f->sh_ev) CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  }
+  const uint64_t seq = f->sh_next++;
+  const uint32_t slot = (uint32_t)(seq % fsm_s::kRing);
+  auto& sp = f->spend[slot];
+  if (sp.active) CUDA_TRY(cudaEventSynchronize(f->sh_ev[slot]));  // ring wrapped
+  sp = fsm_s::ShardPend{};
+  sp.active = true;
+  sp.seq = seq;
+  sp.N = (f->shard_len + o.B - 1) / o.B;
+  sp.scheme = f->shard_scheme;
+  *ticket = seq;
+  if (f->shard_mode != 3) {  // host fix-up modes: finish now
+    sp.done = true;
+    sp.rc = fsm_shard_finish(f, d_maps, G, rank, opts, d_chunk_ends_local, &sp.res);
+    return FSM_OK;
+  }
+  const uint32_t nt = f->n + 1;
+  if (!f->d_small) CUDA_TRY(cudaMalloc(&f->d_small, 64 * sizeof(uint32_t)));
+  CUDA_TRY(launch_compose(reinterpret_cast<const uint8_t*>(d_maps), G, map_bytes_nt(nt), map_cnt_off(nt), f->img.q0t,
+                          rank, f->d_small, o.st));
+  ShardScratch S3;
+  if ((rc = ensure_shard(f, &S3))) return rc;
+  CUDA_TRY(cudaMemsetAsync(f->d_small + 5, 0, 4, o.st));
+  if (d_chunk_ends_local && f->shard_len)
+    CUDA_TRY(launch_fix_prefix_fused(S3.states, S3.cand, S3.info + 8, S3.grp, f->d_small, f->img.inv, f->n,
+                                     d_chunk_ends_local, f->d_small + 5, o.st));
+  CUDA_TRY(cudaMemcpyAsync(f->h_sh + slot * 8, f->d_small, 6 * sizeof(uint32_t), cudaMemcpyDeviceToHost, o.st));
+  CUDA_TRY(cudaEventRecord(f->sh_ev[slot], o.st));
+  sp.pipe_ticket = f->shard_ticket;  // the shard's pipeline run: collected by the wait
+  f->shard_ticket = 0;
+  return FSM_OK;
+}
+
+int fsm_shard_wait(fsm_t f, uint64_t ticket, fsm_result* out) {
+  ApiScope api_scope_("fsm_shard_wait");
+  if (!f || !out) return fail(FSM_EINVAL, "NULL handle/out");
+  const uint32_t slot = (uint32_t)(ticket % fsm_s::kRing);
+  auto& sp = f->spend[slot];
+  if (!sp.active || sp.seq != ticket) return fail(FSM_EINVAL, "unknown or already collected shard ticket");
+  sp.active = false;
+  if (sp.done) {
+    *out = sp.res;
+    return sp.rc;
+  }
+  CUDA_TRY(cudaEventSynchronize(f->sh_ev[slot]));
+  const uint32_t* h = f->h_sh + slot * 8;
+  if (sp.pipe_ticket) {
+    fsm_result rr;
+    uint32_t ff;
+    const int rc = run_collect(f, sp.pipe_ticket, &rr, &ff);  // complete: frees its ring slot
+    if (rc) return rc;
+  }
+  if (h[2] == 3) {
+    const int code = -(int)h[3];
+    char msg[96];
+    std::snprintf(msg, sizeof(msg), "fsm_shard_map failed on rank %u (%s)", h[4], fsm_strerror(code));
+    return fail(code < 0 ? code : FSM_EINVAL, msg);
+  }
+  if (h[2] == 2) {
+    f->shard_prefer_exact = true;
+    return fail(FSM_EAGAIN, "a rank's speculative shard map was invalid: redo the step with fsm_run_sharded");
+  }
+  if (h[2] || h[5]) return fail(FSM_EINVAL, "a shard start state is outside its candidate set");
+  std::memset(out, 0, sizeof(*out));
+  out->nchunks = sp.N;
+  out->scheme_used = sp.scheme;
+  const uint32_t fin = h[1];
+  if (fin == f->n) return fail(FSM_ESYMBOL, "input symbol >= nsyms");
+  out->final_state = f->inv[fin];
+  out->accept = f->accept[out->final_state];
+  out->accept_count = (uint64_t)h[3] | ((uint64_t)h[4] << 32);
   return FSM_OK;
 }
 

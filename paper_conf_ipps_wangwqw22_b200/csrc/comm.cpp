@@ -130,4 +130,32 @@ int fsm_run_sharded(fsm_t f, fsm_comm_t c, const uint8_t* d_shard, uint64_t shar
   return rc;
 }
 
+// Asynchronous step: map + allgather + queued finish; fsm_shard_wait(ticket) collects.  A
+// failed map still joins the exchange (error map) and its status reaches every rank's wait.
+int fsm_run_sharded_async(fsm_t f, fsm_comm_t c, const uint8_t* d_shard, uint64_t shard_len,
+                          const uint8_t* d_lookback, uint32_t lookback_len, const fsm_run_opts* opts,
+                          uint32_t* d_chunk_ends_local, uint64_t* ticket) {
+  if (!f || !c || !ticket) return gspec_set_error(FSM_EINVAL, "NULL handle/comm/ticket");
+  const size_t mb = fsm_map_bytes(f);
+  if (c->map_bytes < mb) {
+    if (c->d_local) cudaFree(c->d_local);
+    if (c->d_all) cudaFree(c->d_all);
+    c->d_local = c->d_all = nullptr;
+    c->map_bytes = 0;
+    if (cudaMalloc(&c->d_local, mb) != cudaSuccess || cudaMalloc(&c->d_all, mb * c->nranks) != cudaSuccess)
+      return gspec_set_error(FSM_ENOMEM, "map buffers");
+    c->map_bytes = mb;
+  }
+  cudaStream_t st = opts ? reinterpret_cast<cudaStream_t>(opts->stream) : nullptr;
+  const int rc = fsm_shard_map(f, d_shard, shard_len, d_lookback, lookback_len, opts, c->d_local, d_chunk_ends_local);
+  if (rc && f->shard_mode != 4) return rc;
+  nvtxRangePushA("ncclAllGather (shard maps)");
+  ncclResult_t r = nccl().allGather(c->d_local, c->d_all, mb, ncclUint8, c->comm, st);
+  nvtxRangePop();
+  if (r != ncclSuccess)
+    return gspec_set_error(FSM_ENCCL, nccl().getErrorString ? nccl().getErrorString(r) : "ncclAllGather");
+  return fsm_shard_finish_async(f, c->d_all, (uint32_t)c->nranks, (uint32_t)c->rank, opts, d_chunk_ends_local,
+                                ticket);
+}
+
 }  // extern "C"

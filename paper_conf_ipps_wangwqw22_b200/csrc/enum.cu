@@ -1,11 +1,12 @@
 // enum.cu — B5: the enumerative scheme (Mytkowicz et al. [23]).
 //
 // Every sub-chunk j (E bytes, E | B) is run from EVERY transformed state
-// (n+1 <= 32 incl. poison): M_j[q] = end state, C_j[q] = accepts on that path.
+// (n+1 <= 64 incl. poison): M_j[q] = end state, C_j[q] = accepts on that path.
+// Maps are W = 32 or 64 entries wide (W = 64: lane l of a warp holds entries l and l+32).
 // The real path is obtained by "connecting the end state of each chunk to the
 // start state of its successor", i.e. a prefix composition of maps:
 //   (M2,C2) o (M1,C1) = (M2[M1[q]], C1[q] + C2[M1[q]]).
-// Composition is one __shfl_sync per map (lane q holds entry q), applied as a
+// Composition is one __shfl_sync per map (lane q holds entry q; two for W = 64), applied as a
 // hierarchical scan: warps scan groups of 64 maps, group totals form the next
 // level, the top level (<= 64 maps) is scanned by one warp, and incoming
 // states/counts are pushed back down level by level.
@@ -18,7 +19,7 @@ namespace {
 constexpr uint32_t kGroup = 64;
 
 // K1: thread per sub-chunk, NE independent chains (ILP = NE).
-template <int MODE, int NE>
+template <int MODE, int NE, int W>
 __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* __restrict__ in, uint64_t len,
                                                   uint32_t E, uint64_t nsub, uint8_t* __restrict__ M,
                                                   uint64_t* __restrict__ Cn, Ctl* ctl_init, uint32_t q0t, uint64_t N) {
@@ -63,11 +64,32 @@ __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* 
       for (int q = 0; q < NE; q++) { code[q] = S::byte(img, smem, code[q], bb); acc[q] += S::acc(code[q]); }
     }
 #pragma unroll
-    for (int q = 0; q < 32; q++) {
+    for (int q = 0; q < W; q++) {
       const bool real = q < NE && (uint32_t)q < nt;
-      M[j * 32 + q] = (uint8_t)(real ? S::tid(img, code[q < NE ? q : 0]) : q);
-      Cn[j * 32 + q] = real ? acc[q < NE ? q : 0] : 0;
+      M[j * W + q] = (uint8_t)(real ? S::tid(img, code[q < NE ? q : 0]) : q);
+      Cn[j * W + q] = real ? acc[q < NE ? q : 0] : 0;
     }
+  }
+}
+
+// One composition step P <- M o P for a W-entry map held by a warp: lane l owns entries l
+// (and l + 32 when W = 64); m_lo / m_hi are this lane's entries of M.
+template <int W>
+__device__ __forceinline__ void compose_step(uint32_t& P0, uint32_t& P1, uint64_t& C0, uint64_t& C1, uint32_t m_lo,
+                                             uint32_t m_hi, uint64_t c_lo, uint64_t c_hi) {
+  if (W == 32) {
+    const uint32_t nP = __shfl_sync(0xffffffffu, m_lo, P0);
+    C0 += __shfl_sync(0xffffffffu, c_lo, P0);
+    P0 = nP;
+  } else {
+    const uint32_t a0 = __shfl_sync(0xffffffffu, m_lo, P0 & 31), b0 = __shfl_sync(0xffffffffu, m_hi, P0 & 31);
+    const uint64_t ca0 = __shfl_sync(0xffffffffu, c_lo, P0 & 31), cb0 = __shfl_sync(0xffffffffu, c_hi, P0 & 31);
+    const uint32_t a1 = __shfl_sync(0xffffffffu, m_lo, P1 & 31), b1 = __shfl_sync(0xffffffffu, m_hi, P1 & 31);
+    const uint64_t ca1 = __shfl_sync(0xffffffffu, c_lo, P1 & 31), cb1 = __shfl_sync(0xffffffffu, c_hi, P1 & 31);
+    C0 += P0 < 32 ? ca0 : cb0;
+    C1 += P1 < 32 ? ca1 : cb1;
+    P0 = P0 < 32 ? a0 : b0;
+    P1 = P1 < 32 ? a1 : b1;
   }
 }
 
@@ -76,42 +98,52 @@ __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* 
 // batches of kBatch (independent loads in flight) before the dependent shuffle chain
 // consumes them, so a group costs kGroup / kBatch memory round trips, not kGroup.
 constexpr int kBatch = 8;
+template <int W>
 __global__ void __launch_bounds__(128) k_enum_group(uint8_t* __restrict__ M, uint64_t* __restrict__ Cn, uint64_t cnt,
                                                    uint8_t* __restrict__ Mup, uint64_t* __restrict__ Cup) {
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
   const uint64_t ngroups = (cnt + kGroup - 1) / kGroup;
   for (uint64_t g = warp; g < ngroups; g += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
-    uint32_t P = lane;
-    uint64_t PC = 0;
+    uint32_t P0 = lane, P1 = lane + 32;
+    uint64_t C0 = 0, C1 = 0;
     const uint64_t j0 = g * kGroup, j1 = min(cnt, j0 + kGroup);
     for (uint64_t jb = j0; jb < j1; jb += kBatch) {
-      uint32_t m[kBatch];
-      uint64_t c[kBatch];
+      uint32_t m0[kBatch], m1[kBatch];
+      uint64_t c0[kBatch], c1[kBatch];
 #pragma unroll
       for (int u = 0; u < kBatch; u++) {
         const uint64_t j = min(jb + u, j1 - 1);
-        m[u] = M[j * 32 + lane];
-        c[u] = Cn[j * 32 + lane];
+        m0[u] = M[j * W + lane];
+        c0[u] = Cn[j * W + lane];
+        m1[u] = W == 64 ? M[j * W + 32 + lane] : 0u;
+        c1[u] = W == 64 ? Cn[j * W + 32 + lane] : 0ull;
       }
 #pragma unroll
       for (int u = 0; u < kBatch; u++) {
         if (jb + u >= j1) break;
-        const uint32_t nP = __shfl_sync(0xffffffffu, m[u], P);
-        PC += __shfl_sync(0xffffffffu, c[u], P);
-        P = nP;
-        M[(jb + u) * 32 + lane] = (uint8_t)P;
-        Cn[(jb + u) * 32 + lane] = PC;
+        compose_step<W>(P0, P1, C0, C1, m0[u], m1[u], c0[u], c1[u]);
+        M[(jb + u) * W + lane] = (uint8_t)P0;
+        Cn[(jb + u) * W + lane] = C0;
+        if (W == 64) {
+          M[(jb + u) * W + 32 + lane] = (uint8_t)P1;
+          Cn[(jb + u) * W + 32 + lane] = C1;
+        }
       }
     }
     if (Mup) {
-      Mup[g * 32 + lane] = (uint8_t)P;
-      Cup[g * 32 + lane] = PC;
+      Mup[g * W + lane] = (uint8_t)P0;
+      Cup[g * W + lane] = C0;
+      if (W == 64) {
+        Mup[g * W + 32 + lane] = (uint8_t)P1;
+        Cup[g * W + 32 + lane] = C1;
+      }
     }
   }
 }
 
 // Descend: incoming state/count of every map at level l from its group's entry.
+template <int W>
 __global__ void k_enum_descend(const uint8_t* __restrict__ P, const uint64_t* __restrict__ PC, uint64_t cnt,
                                const uint32_t* __restrict__ up_state, const uint64_t* __restrict__ up_cnt,
                                uint32_t top_entry, uint32_t* __restrict__ st, uint64_t* __restrict__ sc) {
@@ -123,18 +155,19 @@ __global__ void k_enum_descend(const uint8_t* __restrict__ P, const uint64_t* __
       st[j] = e;
       sc[j] = ec;
     } else {
-      st[j] = P[(j - 1) * 32 + e];
-      sc[j] = ec + PC[(j - 1) * 32 + e];
+      st[j] = P[(j - 1) * W + e];
+      sc[j] = ec + PC[(j - 1) * W + e];
     }
   }
 }
 
 // Outputs: chunk ends (original ids), final state (transformed), total count.
+template <int W>
 __global__ void k_enum_out(DevImage img, const uint32_t* __restrict__ st0, const uint8_t* __restrict__ P0top,
                            const uint64_t* __restrict__ PC0top, uint64_t top_last, uint32_t q0t, uint64_t nsub,
                            uint32_t per_chunk, uint64_t N, uint32_t* __restrict__ chunk_ends, Ctl* ctl,
                            uint32_t* __restrict__ x_final, void* h_out) {
-  const uint32_t fin = P0top[top_last * 32 + q0t];
+  const uint32_t fin = P0top[top_last * W + q0t];
   for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < N; c += (uint64_t)gridDim.x * blockDim.x) {
     const uint64_t jn = (c + 1) * per_chunk;  // first sub-chunk after chunk c
     const uint32_t s = jn < nsub ? st0[jn] : fin;
@@ -143,7 +176,7 @@ __global__ void k_enum_out(DevImage img, const uint32_t* __restrict__ st0, const
   if (blockIdx.x == 0) {
     if (threadIdx.x == 0) {
       *x_final = fin;
-      ctl->accept_count = PC0top[top_last * 32 + q0t];
+      ctl->accept_count = PC0top[top_last * W + q0t];
       __threadfence();
     }
     __syncthreads();
@@ -155,10 +188,10 @@ __global__ void k_enum_out(DevImage img, const uint32_t* __restrict__ st0, const
   }
 }
 
-template <int MODE, int NE>
+template <int MODE, int NE, int W>
 cudaError_t walk_t(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, uint8_t* M, uint64_t* Cn,
                    cudaStream_t st, int sms) {
-  auto kern = k_enum_walk<MODE, NE>;
+  auto kern = k_enum_walk<MODE, NE, W>;
   const uint32_t smem = smem_bytes_for(img);
   cudaError_t e = kernel_setup((const void*)kern, smem, 128, nullptr);
   if (e != cudaSuccess) return e;
@@ -173,9 +206,10 @@ template <int MODE>
 cudaError_t walk_m(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, uint8_t* M, uint64_t* Cn,
                    cudaStream_t st, int sms) {
   const uint32_t nt = img.n + 1;
-  if (nt <= 8) return walk_t<MODE, 8>(img, rp, E, nsub, M, Cn, st, sms);
-  if (nt <= 16) return walk_t<MODE, 16>(img, rp, E, nsub, M, Cn, st, sms);
-  return walk_t<MODE, 32>(img, rp, E, nsub, M, Cn, st, sms);
+  if (nt <= 8) return walk_t<MODE, 8, 32>(img, rp, E, nsub, M, Cn, st, sms);
+  if (nt <= 16) return walk_t<MODE, 16, 32>(img, rp, E, nsub, M, Cn, st, sms);
+  if (nt <= 32) return walk_t<MODE, 32, 32>(img, rp, E, nsub, M, Cn, st, sms);
+  return walk_t<MODE, 64, 64>(img, rp, E, nsub, M, Cn, st, sms);
 }
 
 // ---- small streams: the whole enumeration in ONE launch -------------------------
@@ -330,7 +364,7 @@ cudaError_t small_t(const DevImage& img, const RunParams& rp, uint32_t E, uint64
 template <int MODE>
 cudaError_t small_m(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, void* scratch,
                     uint32_t* ticket, uint32_t* chunk_ends, Ctl* ctl, cudaStream_t st) {
-  const uint32_t nt = img.n + 1;
+  const uint32_t nt = img.n + 1;  // <= 32 (the caller takes the multi-launch path for wider maps)
   if (nt <= 8) return small_t<MODE, 8>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
   if (nt <= 16) return small_t<MODE, 16>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
   return small_t<MODE, 32>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
@@ -359,12 +393,13 @@ cudaError_t launch_enum_small(const DevImage& img, const RunParams& rp, uint32_t
   }
 }
 
-// Scratch layout for the enumeration (levels of maps + per-level states).
+// Scratch layout for the enumeration (levels of maps + per-level states); maps of up to 64
+// entries (the carve in launch_enum_full uses the DFA's width, 32 or 64).
 uint64_t enum_scratch_bytes(uint64_t nsub) {
   auto r = [](uint64_t b) { return (b + 255) & ~255ull; };  // same rounding as the carve in launch_enum_full
   uint64_t tot = 0, cnt = nsub;
   for (int L = 0;; L++) {
-    tot += r(cnt * 32) + r(cnt * 32 * 8) + r(cnt * 4) + r(cnt * 8);
+    tot += r(cnt * 64) + r(cnt * 64 * 8) + r(cnt * 4) + r(cnt * 8);
     if (cnt <= kGroup || L + 1 == 16) break;
     cnt = (cnt + kGroup - 1) / kGroup;
   }
@@ -378,6 +413,7 @@ cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t 
                              uint32_t* d_chunk_ends, Ctl* d_ctl, uint32_t* d_x_final, cudaStream_t st, int sms,
                              int phases, const uint8_t** top_M, const uint64_t** top_C) {
   const uint64_t nsub = (rp.len + E - 1) / E;
+  const uint32_t W = img.n + 1 <= 32 ? 32u : 64u;  // map width
   // carve levels
   struct Lvl { uint8_t* M; uint64_t* C; uint32_t* s; uint64_t* sc; uint64_t cnt; };
   Lvl lv[16];
@@ -387,8 +423,8 @@ cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t 
   uint64_t cnt = nsub;
   for (;;) {
     lv[L].cnt = cnt;
-    lv[L].M = take(cnt * 32);
-    lv[L].C = reinterpret_cast<uint64_t*>(take(cnt * 32 * 8));
+    lv[L].M = take(cnt * W);
+    lv[L].C = reinterpret_cast<uint64_t*>(take(cnt * W * 8));
     lv[L].s = reinterpret_cast<uint32_t*>(take(cnt * 4));
     lv[L].sc = reinterpret_cast<uint64_t*>(take(cnt * 8));
     L++;
@@ -396,8 +432,8 @@ cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t 
     cnt = (cnt + kGroup - 1) / kGroup;
   }
   const uint64_t top_last = lv[L - 1].cnt - 1;
-  if (top_M) *top_M = lv[L - 1].M + top_last * 32;
-  if (top_C) *top_C = lv[L - 1].C + top_last * 32;
+  if (top_M) *top_M = lv[L - 1].M + top_last * W;
+  if (top_C) *top_C = lv[L - 1].C + top_last * W;
   cudaError_t e = cudaSuccess;
   if (phases & 1) {
   switch (img.mode) {
@@ -412,8 +448,12 @@ cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t 
     const uint64_t ng = (lv[l].cnt + kGroup - 1) / kGroup;
     uint64_t grid = (ng * 32 + 127) / 128;
     if (grid > (uint64_t)sms * 16) grid = (uint64_t)sms * 16;
-    k_enum_group<<<(unsigned)grid, 128, 0, st>>>(lv[l].M, lv[l].C, lv[l].cnt, l + 1 < L ? lv[l + 1].M : nullptr,
-                                                 l + 1 < L ? lv[l + 1].C : nullptr);
+    if (W == 32)
+      k_enum_group<32><<<(unsigned)grid, 128, 0, st>>>(lv[l].M, lv[l].C, lv[l].cnt, l + 1 < L ? lv[l + 1].M : nullptr,
+                                                       l + 1 < L ? lv[l + 1].C : nullptr);
+    else
+      k_enum_group<64><<<(unsigned)grid, 128, 0, st>>>(lv[l].M, lv[l].C, lv[l].cnt, l + 1 < L ? lv[l + 1].M : nullptr,
+                                                       l + 1 < L ? lv[l + 1].C : nullptr);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
   }
@@ -421,15 +461,25 @@ cudaError_t launch_enum_full(const DevImage& img, const RunParams& rp, uint32_t 
   for (int l = L - 1; l >= 0; l--) {
     uint64_t grid = (lv[l].cnt + 255) / 256;
     if (grid > (uint64_t)sms * 16) grid = (uint64_t)sms * 16;
-    k_enum_descend<<<(unsigned)grid, 256, 0, st>>>(lv[l].M, lv[l].C, lv[l].cnt, l + 1 < L ? lv[l + 1].s : nullptr,
-                                                   l + 1 < L ? lv[l + 1].sc : nullptr, rp.q0t, lv[l].s, lv[l].sc);
+    if (W == 32)
+      k_enum_descend<32><<<(unsigned)grid, 256, 0, st>>>(lv[l].M, lv[l].C, lv[l].cnt,
+                                                         l + 1 < L ? lv[l + 1].s : nullptr,
+                                                         l + 1 < L ? lv[l + 1].sc : nullptr, rp.q0t, lv[l].s, lv[l].sc);
+    else
+      k_enum_descend<64><<<(unsigned)grid, 256, 0, st>>>(lv[l].M, lv[l].C, lv[l].cnt,
+                                                         l + 1 < L ? lv[l + 1].s : nullptr,
+                                                         l + 1 < L ? lv[l + 1].sc : nullptr, rp.q0t, lv[l].s, lv[l].sc);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;
   }
   uint64_t grid = (rp.N + 255) / 256;
   if (grid > (uint64_t)sms * 16) grid = (uint64_t)sms * 16;
   if (grid < 1) grid = 1;
-  k_enum_out<<<(unsigned)grid, 256, 0, st>>>(img, lv[0].s, lv[L - 1].M, lv[L - 1].C, top_last, rp.q0t, nsub,
-                                             rp.B / E, rp.N, d_chunk_ends, d_ctl, d_x_final, rp.h_out);
+  if (W == 32)
+    k_enum_out<32><<<(unsigned)grid, 256, 0, st>>>(img, lv[0].s, lv[L - 1].M, lv[L - 1].C, top_last, rp.q0t, nsub,
+                                                   rp.B / E, rp.N, d_chunk_ends, d_ctl, d_x_final, rp.h_out);
+  else
+    k_enum_out<64><<<(unsigned)grid, 256, 0, st>>>(img, lv[0].s, lv[L - 1].M, lv[L - 1].C, top_last, rp.q0t, nsub,
+                                                   rp.B / E, rp.N, d_chunk_ends, d_ctl, d_x_final, rp.h_out);
   return cudaGetLastError();
 }
 

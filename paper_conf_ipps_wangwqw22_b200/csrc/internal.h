@@ -34,7 +34,8 @@ constexpr uint32_t kImgFull = 64;   // lookback > 2: pair images kept with multi
 constexpr uint32_t kLookbackMax = 16;
 constexpr uint32_t kVrMax = 16;     // VR^end / VR^others slots
 constexpr uint32_t kSlots = 2 * kVrMax;
-constexpr uint32_t kEnumMax = 32;   // ENUM: transformed states incl. poison
+constexpr uint32_t kEnumMax = 64;   // ENUM: transformed states incl. poison (maps of 32 or 64 entries)
+constexpr uint32_t kEnumSmallMax = 32;  // ENUM in one launch (k_enum_small): 32-entry maps only
 
 // POD device view of a loaded DFA, passed by value to every kernel.
 struct DevImage {
@@ -165,6 +166,7 @@ struct RunParams {
   Ctl* v0_ctl;
   uint32_t* v0_bflag;      // [tiles] tile-boundary arrival counters (+2 per run, never reset)
   uint32_t* v0_chunk_ends; // nullable: the run's chunk ends (original ids)
+  uint32_t tma_evict_normal;  // 1: input TMA loads with L2 evict_normal (else evict_first)
 };
 
 // GSPEC_STAMPS=1: kernels record the run timeline in Ctl::tl (one extra atomic per warp).
@@ -194,6 +196,26 @@ inline bool v0_disabled() {
     v = (e && atoi(e) == 1) ? 0 : 1;
   }
   return v != 0;
+}
+
+// TMA input L2 promotion (GSPEC_TMA_PROMO: 0 = 256 B default, 1 = 64 B, 2 = none) and the
+// input's L2 eviction policy (GSPEC_TMA_EVICT: 0 = evict_first default, 1 = evict_normal)
+inline int tma_promotion() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("GSPEC_TMA_PROMO");
+    v = e ? atoi(e) : 0;
+  }
+  return v;
+}
+
+inline int tma_evict_mode() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("GSPEC_TMA_EVICT");
+    v = e ? atoi(e) : 0;
+  }
+  return v;
 }
 
 inline bool pdl_enabled() {
@@ -403,6 +425,19 @@ struct fsm_s {
   size_t shard_bytes = 0;
   int shard_mode = -1;          // 0 fused/single path, 1 enum, 2 multi-path, 3 fused with cand[0], 4 map failed
   uint64_t shard_ticket = 0;
+  // asynchronous sharded steps (fsm_shard_finish_async / fsm_shard_wait): a ring of
+  // pending finishes, their result words in pinned memory
+  struct ShardPend {
+    bool active = false;
+    uint64_t seq = 0, N = 0, pipe_ticket = 0;
+    fsm_scheme scheme = FSM_SCHEME_AUTO;
+    bool done = false;       // finished synchronously (host fix-up modes): res/rc hold the outcome
+    int rc = 0;
+    fsm_result res{};
+  } spend[kRing];
+  uint32_t* h_sh = nullptr;              // pinned [kRing][8] result words of async finishes
+  cudaEvent_t sh_ev[kRing] = {};
+  uint64_t sh_next = 1;
   uint32_t last_nstamp = 0;            // verify phase timestamps of the last collected run
   uint64_t last_stamp[24] = {};
   uint64_t last_tl[4] = {};             // run timeline of the last collected run (GSPEC_STAMPS=1)

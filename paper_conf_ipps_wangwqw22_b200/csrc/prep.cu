@@ -141,9 +141,10 @@ __global__ void __launch_bounds__(256) k_qs_long(DevImage img, const uint32_t* _
         for (uint32_t i = 2; i < L; i++) s[h] = __ldg(ttc + (uint64_t)s[h] * img.C + __ldg(img.cls + w[i]));
     }
     // merge equal end states: the first entry of a group leads and sums the multiplicities
+    // (n2 is warp-uniform: the loops run over the pair image's entries only)
     uint32_t tot[2] = {0, 0};
     bool lead[2] = {m[0] != 0, m[1] != 0};
-    for (uint32_t k = 0; k < 64; k++) {
+    for (uint32_t k = 0; k < n2; k++) {
       const uint32_t sk = __shfl_sync(0xffffffffu, s[k >> 5], k & 31);
       const uint32_t mk = __shfl_sync(0xffffffffu, m[k >> 5], k & 31);
 #pragma unroll
@@ -155,7 +156,7 @@ __global__ void __launch_bounds__(256) k_qs_long(DevImage img, const uint32_t* _
     }
     // rank the leaders by (-multiplicity, id)
     uint32_t rank[2] = {0, 0}, nlead = 0;
-    for (uint32_t k = 0; k < 64; k++) {
+    for (uint32_t k = 0; k < n2; k++) {
       const uint32_t sk = __shfl_sync(0xffffffffu, s[k >> 5], k & 31);
       const uint32_t tk = __shfl_sync(0xffffffffu, tot[k >> 5], k & 31);
       const bool lk = __shfl_sync(0xffffffffu, (uint32_t)lead[k >> 5], k & 31) != 0;

@@ -371,7 +371,7 @@ cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_
 
 cudaError_t launch_map_enum(const uint8_t* topM, const unsigned long long* topC, uint32_t nt, uint32_t* mend,
                             unsigned long long* mcnt, cudaStream_t st) {
-  k_map_enum<<<1, 32, 0, st>>>(topM, topC, nt, mend, mcnt);
+  k_map_enum<<<1, 64, 0, st>>>(topM, topC, nt, mend, mcnt);
   return cudaGetLastError();
 }
 

@@ -53,6 +53,12 @@ __device__ __forceinline__ uint64_t evict_first_policy() {
   return p;
 }
 
+__device__ __forceinline__ uint64_t evict_normal_policy() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+
 __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int32_t x, int32_t y,
                                             uint64_t policy) {
   asm volatile(
@@ -253,7 +259,10 @@ __global__ void __launch_bounds__(KP > 8 ? 512 : 896, 1) k_spec_tma(const __grid
   uint8_t* wst = stages + (size_t)warp * S * kStageBytes;
   uint64_t* wbar = bars + warp * S;
 
-  const uint64_t pol = evict_first_policy();
+  // evict-first keeps a large table's cold rows in L2; a table that lives wholly in shared
+  // memory (rp.tma_evict_normal) lets the input's 256 B lines stay until the warp's next
+  // stages consume them (GSPEC_TMA_EVICT, A/B)
+  const uint64_t pol = rp.tma_evict_normal ? evict_normal_policy() : evict_first_policy();
   // producer cursor (lane 0): the item S ahead of the consumer, tracked without divisions
   uint64_t p_tile = 0;
   uint32_t p_sg = 0, p_s = 0;
@@ -598,7 +607,9 @@ bool encode_map(const RunParams& rp, uint64_t n_full, CUtensorMap* tm, bool gath
   cuuint32_t box[2] = {kRowBytes, gather ? 1u : 32u};
   cuuint32_t es[2] = {1, 1};
   return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(rp.in), dims, strides, box, es,
-             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B,
+             tma_promotion() == 1 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+             : tma_promotion() == 2 ? CU_TENSOR_MAP_L2_PROMOTION_NONE : CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 

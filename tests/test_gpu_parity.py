@@ -89,7 +89,7 @@ def test_configs_small_with_diagnostics(gs, name, length, scheme):
 @pytest.mark.parametrize("scheme", SCHEMES + ["enum"])
 def test_random_dfas(gs, seed, scheme):
     rng = np.random.default_rng(seed)
-    n = int(rng.integers(1, 31 if scheme == "enum" else 300))
+    n = int(rng.integers(1, 64 if scheme == "enum" else 300))
     ns = int(rng.integers(1, 257))
     name = f"rand:{n}:{ns}:{seed}"
     length = int(rng.integers(0, 200000))
@@ -434,10 +434,10 @@ def _perm_dfa(n, nsyms, seed):
     return t, 0, a
 
 
-@pytest.mark.parametrize("n", [31, 32])
+@pytest.mark.parametrize("n", [31, 32, 63, 64])
 def test_selector_enum_bound(gs, n):
-    """R19's ENUM leaf: n <= 31.  The GPU selector and the oracle pick the same scheme
-    on permutation DFAs of 31 and 32 states, and the picked scheme is exact."""
+    """R19's ENUM leaf: n <= 63 (maps of 32 or 64 entries).  The GPU selector and the
+    oracle pick the same scheme on permutation DFAs of 31..64 states, and it is exact."""
     t, s, a = _perm_dfa(n, 3, n)
     rng = np.random.default_rng(n)
     data = rng.integers(0, 3, 1 << 18).astype(np.uint8)
@@ -449,7 +449,7 @@ def test_selector_enum_bound(gs, n):
     assert ft["acc1"] == pytest.approx(of["acc1"]) and ft["acck"] == pytest.approx(of["acck"])
     assert ft["input_sensitivity"] == pytest.approx(of["sens"])
     assert oracle.select(of, n) == gs.SCHEMES[pick]
-    assert pick == ("enum" if n == 31 else "sre")
+    assert pick == ("enum" if n <= 63 else "sre")
     ref = oracle.run(t, s, a, data, 4096)
     check_equal(fsm.run(x, scheme="auto"), ref, 4096, n)
 

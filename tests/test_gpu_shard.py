@@ -185,3 +185,27 @@ def test_many_nonmerging_paths(gs, n, G):
     for r in outs:
         assert r.final_state == ref["final"] and r.accept_count == ref["count"]
     assert (ce[:len(ref["chunk_end"])].cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
+
+
+def test_library_nccl_async_steps(gs):
+    """fsm_run_sharded_async: several steps queued back to back on one 1-rank NCCL
+    communicator, each collected by fsm_shard_wait, every one exact (C2: fused mode; div7:
+    the host fix-up ENUM mode, finished inside the async call)."""
+    for name, length in (("c2", 8 << 20), ("c1", 1 << 20), ("c3", 4 << 20)):
+        w = gen.workload(name, length=length)
+        data = w.host()
+        ref = oracle.run(w.table, w.start, w.accept, data, 4096)
+        fsm = gs.FSM.load(w.table, w.start, w.accept)
+        comm = gs.Comm(1, 0, gs.Comm.unique_id())
+        x = torch.from_numpy(data).cuda()
+        comm.run_sharded(fsm, x)  # warm (selector, speculative-map check)
+        ce = torch.empty(gs.fsm_num_chunks(length), dtype=torch.int32, device="cuda")
+        tickets = [comm.run_sharded_async(fsm, x, chunk_ends=ce) for _ in range(5)]
+        for t in tickets:
+            r = gs.Comm.wait(fsm, t)
+            assert r.final_state == ref["final"] and r.accept_count == ref["count"], name
+        assert (ce.cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
+        with pytest.raises(gs.GSpecError):
+            gs.Comm.wait(fsm, tickets[0])  # already collected
+        comm.close()
+        fsm.close()

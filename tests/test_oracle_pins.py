@@ -723,14 +723,16 @@ def test_features_sens_c3s_region_boundary():
     assert max(seg_acc[4:]) > min(seg_acc[:4]) and f["sens"] >= 0.2  # the regions really differ
 
 
-def test_select_enum_bound_31_32():
-    """R19: the ENUM leaf needs n <= 31 real states (n + poison in one warp)."""
+def test_select_enum_bound_63_64():
+    """R19: the ENUM leaf needs n <= 63 real states (n + poison = two map entries per lane)."""
     f = {"acc1": 0.0, "acck": 0.0, "sens": 0.0, "uniq10": 31.0}
     assert oracle.select(f, 31) == oracle.ENUM
-    assert oracle.select(dict(f, uniq10=15.5), 31) == oracle.ENUM
-    assert oracle.select(dict(f, uniq10=15.4), 31) != oracle.ENUM
-    assert oracle.select(dict(f, uniq10=32.0), 32) != oracle.ENUM
-    assert oracle.select(dict(f, uniq10=32.0), 32) == oracle.SRE  # acck - acc1 < 0.5 (R19b)
+    assert oracle.select(dict(f, uniq10=32.0), 32) == oracle.ENUM
+    assert oracle.select(dict(f, uniq10=63.0), 63) == oracle.ENUM
+    assert oracle.select(dict(f, uniq10=31.5), 63) == oracle.ENUM
+    assert oracle.select(dict(f, uniq10=31.4), 63) != oracle.ENUM
+    assert oracle.select(dict(f, uniq10=64.0), 64) != oracle.ENUM
+    assert oracle.select(dict(f, uniq10=64.0), 64) == oracle.SRE  # acck - acc1 < 0.5 (R19b)
 
 
 def test_run_stream_div7_closed_form():

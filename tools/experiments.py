@@ -52,7 +52,9 @@ def main():
     for cfg in ("c2", "c3", "c3s", "c4"):
         w = gen.workload(cfg, length=length)
         x = torch.empty(length, dtype=torch.uint8, device="cuda")
-        w.device(x)
+        # c3s: straddle a normal / vowel-free region boundary (64 MiB regions) so the stream
+        # really is input-sensitive (the first 64 MiB alone is one normal region)
+        w.device(x, offset=((1 << 26) - length // 2) if cfg == "c3s" else 0)
         fsm = gs.FSM.load(w.table, w.start, w.accept)
         pick, feats = fsm.select_scheme(x)  # 8 spread portions of the stream (R20)
         ref = None
