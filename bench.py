@@ -437,7 +437,15 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         scheme, feats = fsm.select_scheme(prof, chunk_bytes=B)
         del prof
 
+        p2p = None
+        if dist is not None and args.exchange == "p2p":
+            from paper_conf_ipps_wangwqw22_b200.dist import p2p_setup
+
+            p2p = p2p_setup(fsm)
+
         def step():
+            if p2p is not None:
+                return p2p.run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
             if comm is not None:
                 return comm.run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
             if dist is not None:
@@ -455,13 +463,15 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         with ClockSampler(dev) as clk:
             ev0.record(stream)
-            if comm is not None:  # steps queued back to back: no host wait between them
+            if comm is not None and p2p is None:  # steps queued back to back: no host wait between them
                 res = async_sharded_steps(gs, comm, fsm, x, lb, scheme, B, ce, args.steps)
             else:
                 for _ in range(args.steps):
                     res = step()
             ev1.record(stream)
             torch.cuda.synchronize()
+        if p2p is not None:
+            p2p.close()
         if clk_all is None:
             clk_all = clk
         else:
@@ -496,8 +506,9 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": "c5", "desc": CONFIG_DESC["c5"], "headline_dfa": dfas[0], "bytes_total": L,
                    "chunk_bytes": B, "l2": "input (16 GiB / N per GPU) larger than the 126 MB L2; no flush",
-                   "parallelism": f"{world} contiguous shards + one allgather of state maps"
-                   + (" (library NCCL communicator, fsm_run_sharded)" if comm is not None else
+                   "parallelism": f"{world} contiguous shards + one exchange of state maps"
+                   + (" (peer-memory stores, fsm_run_sharded_p2p)" if dist is not None and args.exchange == "p2p" else
+                      " (library NCCL allgather, fsm_run_sharded_async)" if comm is not None else
                       " (torch.distributed allgather)" if dist is not None else " (single GPU, fsm_run)"),
                    "nccl_ranks": comm.nranks if comm is not None else 0},
         "per_dfa": per,
@@ -524,6 +535,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-per-dfa", action="store_true", help="skip the per-DFA sub-results of the default line")
     ap.add_argument("--ref-sample-mib", type=int, default=256)
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p"],
+                    help="N > 1: state maps by the library's NCCL allgather, or by peer-memory stores (fsm_p2p_*)")
     ap.add_argument("--c5-dfa", default="all", choices=["all"] + list(C5_DFAS))
     ap.add_argument("--c5-bytes", type=int, default=C5_LEN)
     args = ap.parse_args()
@@ -601,7 +614,15 @@ def main():
         if rank:
             w.device(lb, offset=rank * length - 16)
 
+        p2p = None
+        if args.exchange == "p2p":
+            from paper_conf_ipps_wangwqw22_b200.dist import p2p_setup
+
+            p2p = p2p_setup(fsm)
+
         def step():
+            if p2p is not None:
+                return p2p.run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
             if comm is not None:
                 return comm.run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
             return run_sharded(fsm, x, lb, scheme=scheme, chunk_bytes=B)
@@ -616,7 +637,7 @@ def main():
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         with ClockSampler(dev) as clk:
             ev0.record(stream)
-            if comm is not None:  # steps queued back to back: no host wait between them
+            if comm is not None and p2p is None:  # steps queued back to back: no host wait between them
                 res = async_sharded_steps(gs, comm, fsm, x, lb, scheme, B, ce_sh, args.steps)
             else:
                 for _ in range(args.steps):
@@ -653,7 +674,9 @@ def main():
 
             def e2e_step():
                 xd.copy_(h, non_blocking=True)                     # H2D of this rank's shard
-                if comm is not None:
+                if p2p is not None:
+                    r = p2p.run_sharded(fsm, xd, lb, scheme=scheme, chunk_bytes=B)
+                elif comm is not None:
                     r = comm.run_sharded(fsm, xd, lb, scheme=scheme, chunk_bytes=B)
                 else:
                     r = run_sharded(fsm, xd, lb, scheme=scheme, chunk_bytes=B)
@@ -693,8 +716,9 @@ def main():
                    "chunk_bytes": B, "scheme": scheme, "nstates": int(w.nstates), "spec_k": args.spec_k or None,
                    "lookback": args.lookback,
                    "l2": "input (1 GiB/GPU) larger than the 126 MB L2; no explicit flush",
-                   "parallelism": (f"dp{world} contiguous shards + one allgather of state maps"
-                                   + (" (library NCCL, fsm_run_sharded)" if comm is not None else "")
+                   "parallelism": (f"dp{world} contiguous shards + one exchange of state maps"
+                                   + (" (peer-memory stores, fsm_run_sharded_p2p)" if args.exchange == "p2p" else
+                                      " (library NCCL allgather, fsm_run_sharded_async)" if comm is not None else "")
                                    if world > 1 else "single GPU"),
                    "nccl_ranks": comm.nranks if comm is not None else 0},
         "pct_hbm_roofline_8TBs": round(100 * value / world / 8000.0, 2),

@@ -295,6 +295,25 @@ int fsm_run_sharded_async(fsm_t fsm, fsm_comm_t comm, const uint8_t* d_shard, ui
                           uint32_t* d_chunk_ends_local, uint64_t* ticket);
 void fsm_comm_free(fsm_comm_t comm);
 
+/* ---- peer-memory exchange (no collective library) ---------------
+ * The fused alternative of SURVEY §8(e): each rank owns a mailbox in its HBM (two
+ * step-parity sets of nranks map slots + arrival flags) that every peer maps through
+ * CUDA IPC (peer memory over NVLink / NVSwitch).  fsm_p2p_create allocates it and
+ * returns its 64-byte IPC handle; the caller exchanges the handles out of band (e.g.
+ * torch.distributed all_gather_object) and passes all nranks of them, in rank order, to
+ * fsm_p2p_open.  fsm_run_sharded_p2p = fsm_shard_map into the own slot, one kernel that
+ * stores the map into every peer's mailbox and raises its flag there, one kernel that
+ * waits (bounded: FSM_ENCCL after ~10 s) for every peer's flag, then fsm_shard_finish
+ * over the own mailbox.  Same results and error protocol as fsm_run_sharded.  One
+ * fsm_p2p_t per (handle, rank); every rank must run the same sequence of steps. */
+typedef struct fsm_p2p_s* fsm_p2p_t;
+int fsm_p2p_create(fsm_t fsm, int nranks, int rank, void* ipc_handle_out, fsm_p2p_t* out);
+int fsm_p2p_open(fsm_p2p_t p2p, const void* ipc_handles);
+int fsm_run_sharded_p2p(fsm_t fsm, fsm_p2p_t p2p, const uint8_t* d_shard, uint64_t shard_len,
+                        const uint8_t* d_lookback, uint32_t lookback_len, const fsm_run_opts* opts,
+                        uint32_t* d_chunk_ends_local, fsm_result* out_global);
+void fsm_p2p_free(fsm_p2p_t p2p);
+
 /* ---- introspection (tests) ------------------------------------------------- */
 /* perm/inv: host uint32 [nstates+1] (poison = nstates last); freq: uint64
  * [nstates]; mode/H/C: table format, hot rows, classes. Any pointer nullable. */

@@ -95,6 +95,11 @@ _lib.fsm_run_sharded.argtypes = [P, P, P, U64, P, U32, ctypes.POINTER(fsm_run_op
 _lib.fsm_run_sharded_async.argtypes = [P, P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(U64)]
 _lib.fsm_shard_finish_async.argtypes = [P, P, U32, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(U64)]
 _lib.fsm_shard_wait.argtypes = [P, U64, ctypes.POINTER(fsm_result)]
+_lib.fsm_p2p_create.argtypes = [P, ctypes.c_int, ctypes.c_int, P, ctypes.POINTER(P)]
+_lib.fsm_p2p_open.argtypes = [P, P]
+_lib.fsm_run_sharded_p2p.argtypes = [P, P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
+_lib.fsm_p2p_free.argtypes = [P]
+_lib.fsm_p2p_free.restype = None
 _lib.fsm_comm_free.argtypes = [P]
 _lib.fsm_comm_free.restype = None
 _lib.fsm_free.argtypes = [P]
@@ -405,6 +410,53 @@ class Comm:
     def close(self):
         if self._h:
             _lib.fsm_comm_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class P2P:
+    """Peer-memory state-map exchange (fsm_p2p_*): a mailbox in this GPU's HBM that every
+    peer maps through CUDA IPC.  handle -> exchange out of band -> open(all handles)."""
+
+    def __init__(self, fsm: "FSM", nranks: int, rank: int):
+        h = P()
+        buf = ctypes.create_string_buffer(64)
+        _check(_lib.fsm_p2p_create(fsm.handle, nranks, rank, buf, ctypes.byref(h)), "fsm_p2p_create")
+        self._h = h.value
+        self.handle = buf.raw
+        self.nranks, self.rank = nranks, rank
+
+    def open(self, handles):
+        """handles: the nranks 64-byte IPC handles, in rank order."""
+        assert len(handles) == self.nranks
+        blob = ctypes.create_string_buffer(b"".join(bytes(x) for x in handles), 64 * self.nranks)
+        _check(_lib.fsm_p2p_open(self._h, blob), "fsm_p2p_open")
+
+    def run_sharded(self, fsm: "FSM", shard, lookback=None, scheme="auto", chunk_bytes=4096, spec_k=0,
+                    chunk_ends=True, stream=None) -> Result:
+        """fsm_run_sharded_p2p: shard map, publish into every peer's mailbox, wait, finish."""
+        import torch
+
+        o = _run_opts(scheme, chunk_bytes, spec_k, stream=stream)
+        n = fsm_num_chunks(shard.numel(), chunk_bytes)
+        ce = torch.empty(max(n, 1), dtype=torch.int32, device=shard.device) if chunk_ends else None
+        lb = lookback if lookback is not None and lookback.numel() else None
+        r = fsm_result()
+        _check(_lib.fsm_run_sharded_p2p(fsm.handle, self._h, shard.data_ptr() if shard.numel() else None,
+                                        shard.numel(), lb.data_ptr() if lb is not None else None,
+                                        lb.numel() if lb is not None else 0, ctypes.byref(o),
+                                        ce.data_ptr() if ce is not None else None, ctypes.byref(r)),
+               "fsm_run_sharded_p2p")
+        return Result.from_c(r, ce[:n] if ce is not None else None)
+
+    def close(self):
+        if self._h:
+            _lib.fsm_p2p_free(self._h)
             self._h = None
 
     def __del__(self):

@@ -350,6 +350,10 @@ cudaError_t launch_qs_long(const DevImage& img, const uint32_t* d_ttc, const uin
 uint64_t pm_tree_scratch_bytes(uint64_t N, uint32_t k, uint32_t* levels);
 cudaError_t launch_pm_tree(const DevImage& img, const RunParams& rp, const RecStore& rs, uint32_t k, void* scratch,
                            Ctl* ctl, uint32_t* d_chunk_ends, int sms, cudaStream_t st, uint32_t* launches);
+cudaError_t launch_publish(const uint8_t* own_map, uint64_t mapb, uint8_t* const* peers, uint32_t G, uint32_t rank,
+                           uint32_t set, unsigned long long seq, cudaStream_t st);
+cudaError_t launch_wait_flags(const uint8_t* own_box, uint64_t mapb, uint32_t G, uint32_t rank, uint32_t set,
+                              unsigned long long seq, uint32_t* status, cudaStream_t st);
 cudaError_t launch_map_error(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, uint32_t code, cudaStream_t st);
 cudaError_t launch_set_u32(uint32_t* p, uint32_t v, uint32_t* p2, uint32_t v2, cudaStream_t st);
 cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_t* grp,

@@ -128,3 +128,22 @@ def unpack_map(buf: np.ndarray, nt: int):
     off, total = map_layout(nt)
     b = np.ascontiguousarray(buf[:total])
     return b[:nt * 4].view(np.uint32), b[off:off + nt * 8].view(np.uint64)
+
+
+def p2p_setup(fsm: FSM, group=None):
+    """A peer-memory exchange for this handle (fsm_p2p_*): every rank creates its mailbox,
+    the 64-byte IPC handles are exchanged with all_gather_object (host plumbing), and every
+    rank maps its peers' mailboxes.  Then P2P.run_sharded(fsm, shard, lookback) runs steps
+    without a collective library."""
+    import torch.distributed as dist
+
+    from . import P2P
+
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    p = P2P(fsm, world, rank)
+    handles = [None] * world
+    dist.all_gather_object(handles, p.handle, group=group)
+    p.open(handles)
+    dist.barrier(group)
+    return p

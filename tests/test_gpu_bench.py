@@ -23,14 +23,14 @@ def _bench(*args, env=None):
     return json.loads(lines[0])
 
 
-@pytest.mark.parametrize("gpus", [1, 2])
-def test_bench_c5_line(gpus):
+@pytest.mark.parametrize("gpus,exchange", [(1, "nccl"), (2, "nccl"), (2, "p2p")])
+def test_bench_c5_line(gpus, exchange):
     import gen
     import oracle
 
     L = 64 << 20
     d = _bench("--config", "c5", "--gpus", str(gpus), "--steps", "2", "--warmup", "3", "--c5-bytes", str(L),
-               env={"GSPEC_DIST_BACKEND": "gloo"} if gpus > 1 else None)
+               "--exchange", exchange, env={"GSPEC_DIST_BACKEND": "gloo"} if gpus > 1 else None)
     assert d["n_gpus"] == gpus and d["scaling"] == "strong" and d["config"]["workload"] == "c5"
     assert set(d["per_dfa"]) == {"c1", "c2", "c3", "c4"}
     for name, r in d["per_dfa"].items():
