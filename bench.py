@@ -570,7 +570,7 @@ def main():
             # only broadcasts the 128-byte unique id and provides barriers
             uid = [gs.Comm.unique_id() if rank == 0 else None]
             dist.broadcast_object_list(uid, src=0)
-            comm = gs.Comm(world, rank, uid[0])
+            comm = gs.Comm(world, rank, uid[0], device=dev)
         else:
             dist.init_process_group(backend)
     peak, peak_kind = _peaks()

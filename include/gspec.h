@@ -284,7 +284,8 @@ int fsm_shard_wait(fsm_t fsm, uint64_t ticket, fsm_result* out);
  * loaded at run time (libnccl.so.2); FSM_ENCCL if it is missing or fails. */
 typedef struct fsm_comm_s* fsm_comm_t;
 int fsm_comm_unique_id(void* id_out);
-int fsm_comm_init(int nranks, int rank, const void* unique_id, fsm_comm_t* out);
+/* device: the CUDA device of this rank (cudaSetDevice), -1 = the current one. */
+int fsm_comm_init(int nranks, int rank, const void* unique_id, int device, fsm_comm_t* out);
 int fsm_run_sharded(fsm_t fsm, fsm_comm_t comm, const uint8_t* d_shard, uint64_t shard_len,
                     const uint8_t* d_lookback, uint32_t lookback_len, const fsm_run_opts* opts,
                     uint32_t* d_chunk_ends_local, fsm_result* out_global);
@@ -293,6 +294,13 @@ int fsm_run_sharded(fsm_t fsm, fsm_comm_t comm, const uint8_t* d_shard, uint64_t
 int fsm_run_sharded_async(fsm_t fsm, fsm_comm_t comm, const uint8_t* d_shard, uint64_t shard_len,
                           const uint8_t* d_lookback, uint32_t lookback_len, const fsm_run_opts* opts,
                           uint32_t* d_chunk_ends_local, uint64_t* ticket);
+/* The SURVEY §8(b) form: the shard's offset and the stream's length instead of lookback
+ * bytes — the library gathers every rank's last 16 bytes (one tiny ncclAllGather, a host
+ * wait) and takes the 16 bytes before this shard from the nearest preceding non-empty
+ * shards.  shard_offset must be a multiple of chunk_bytes.  Then as fsm_run_sharded. */
+int fsm_run_sharded_at(fsm_t fsm, fsm_comm_t comm, const uint8_t* d_shard, uint64_t shard_offset,
+                       uint64_t shard_len, uint64_t total_len, const fsm_run_opts* opts,
+                       uint32_t* d_chunk_ends_local, fsm_result* out_global);
 void fsm_comm_free(fsm_comm_t comm);
 
 /* ---- peer-memory exchange (no collective library) ---------------

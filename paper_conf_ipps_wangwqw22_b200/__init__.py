@@ -90,7 +90,8 @@ _lib.fsm_get_records.argtypes = [P, U64, P, P, P, P, P, P]
 _lib.fsm_get_phase_times.argtypes = [P, P, ctypes.POINTER(U32)]
 _lib.fsm_get_timeline.argtypes = [P, P]
 _lib.fsm_comm_unique_id.argtypes = [P]
-_lib.fsm_comm_init.argtypes = [ctypes.c_int, ctypes.c_int, P, ctypes.POINTER(P)]
+_lib.fsm_comm_init.argtypes = [ctypes.c_int, ctypes.c_int, P, ctypes.c_int, ctypes.POINTER(P)]
+_lib.fsm_run_sharded_at.argtypes = [P, P, P, U64, U64, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
 _lib.fsm_run_sharded.argtypes = [P, P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
 _lib.fsm_run_sharded_async.argtypes = [P, P, P, U64, P, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(U64)]
 _lib.fsm_shard_finish_async.argtypes = [P, P, U32, U32, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(U64)]
@@ -356,10 +357,10 @@ class FSM:
 class Comm:
     """Library-owned NCCL communicator (fsm_comm_init); one per rank / GPU."""
 
-    def __init__(self, nranks: int, rank: int, unique_id: bytes):
+    def __init__(self, nranks: int, rank: int, unique_id: bytes, device: int = -1):
         h = P()
         buf = ctypes.create_string_buffer(bytes(unique_id), 128)
-        _check(_lib.fsm_comm_init(nranks, rank, buf, ctypes.byref(h)), "fsm_comm_init")
+        _check(_lib.fsm_comm_init(nranks, rank, buf, device, ctypes.byref(h)), "fsm_comm_init")
         self._h = h.value
         self.nranks, self.rank = nranks, rank
 
@@ -383,6 +384,21 @@ class Comm:
                                     lb.data_ptr() if lb is not None else None, lb.numel() if lb is not None else 0,
                                     ctypes.byref(o), ce.data_ptr() if ce is not None else None, ctypes.byref(r)),
                "fsm_run_sharded")
+        return Result.from_c(r, ce[:n] if ce is not None else None)
+
+    def run_sharded_at(self, fsm: "FSM", shard, shard_offset: int, total_len: int, scheme="auto",
+                       chunk_bytes=4096, spec_k=0, chunk_ends=True, stream=None) -> Result:
+        """fsm_run_sharded_at: as run_sharded, the lookback bytes fetched by the library."""
+        import torch
+
+        o = _run_opts(scheme, chunk_bytes, spec_k, stream=stream)
+        n = fsm_num_chunks(shard.numel(), chunk_bytes)
+        ce = torch.empty(max(n, 1), dtype=torch.int32, device=shard.device) if chunk_ends else None
+        r = fsm_result()
+        _check(_lib.fsm_run_sharded_at(fsm.handle, self._h, shard.data_ptr() if shard.numel() else None, shard_offset,
+                                       shard.numel(), total_len, ctypes.byref(o),
+                                       ce.data_ptr() if ce is not None else None, ctypes.byref(r)),
+               "fsm_run_sharded_at")
         return Result.from_c(r, ce[:n] if ce is not None else None)
 
     def run_sharded_async(self, fsm: "FSM", shard, lookback=None, scheme="auto", chunk_bytes=4096, spec_k=0,

@@ -7,8 +7,10 @@
 #include <nccl.h>
 #include <nvtx3/nvToolsExt.h>
 
+#include <algorithm>
 #include <cstring>
 #include <mutex>
+#include <vector>
 #include <string>
 
 #include "gspec.h"
@@ -67,10 +69,11 @@ int fsm_comm_unique_id(void* id_out) {
   return FSM_OK;
 }
 
-int fsm_comm_init(int nranks, int rank, const void* unique_id, fsm_comm_t* out) {
+int fsm_comm_init(int nranks, int rank, const void* unique_id, int device, fsm_comm_t* out) {
   if (!unique_id || !out || nranks < 1 || rank < 0 || rank >= nranks) return gspec_set_error(FSM_EINVAL, "bad comm args");
   NcclApi& a = nccl();
   if (!a.ok) return gspec_set_error(FSM_ENCCL, "libnccl.so.2 not loadable");
+  if (device >= 0 && cudaSetDevice(device) != cudaSuccess) return gspec_set_error(FSM_EINVAL, "bad device");
   ncclUniqueId id;
   std::memcpy(&id, unique_id, sizeof(id));
   fsm_comm_s* c = new fsm_comm_s();
@@ -83,6 +86,54 @@ int fsm_comm_init(int nranks, int rank, const void* unique_id, fsm_comm_t* out) 
   c->rank = rank;
   *out = c;
   return FSM_OK;
+}
+
+// The SURVEY §8(b) signature: the caller passes its shard's place in the stream and the
+// library fetches the lookback bytes itself — every rank's last 16 bytes are gathered with
+// one tiny ncclAllGather (17 bytes per rank: bytes + count) and the 16 bytes before this
+// shard are taken from the nearest preceding non-empty shards (shard_offset 0: none).
+int fsm_run_sharded_at(fsm_t f, fsm_comm_t c, const uint8_t* d_shard, uint64_t shard_offset, uint64_t shard_len,
+                       uint64_t total_len, const fsm_run_opts* opts, uint32_t* d_chunk_ends_local,
+                       fsm_result* out_global) {
+  if (!f || !c || !out_global) return gspec_set_error(FSM_EINVAL, "NULL handle/comm/out");
+  const uint32_t B = (opts && opts->chunk_bytes) ? opts->chunk_bytes : 4096;
+  if (shard_offset % B != 0 || shard_offset + shard_len > total_len)
+    return gspec_set_error(FSM_EINVAL, "shard not chunk-aligned / outside the stream");
+  cudaStream_t st = opts ? reinterpret_cast<cudaStream_t>(opts->stream) : nullptr;
+  const int G = c->nranks;
+  uint8_t *d_tail = nullptr, *d_tails = nullptr;
+  if (cudaMalloc(&d_tail, 32) != cudaSuccess || cudaMalloc(&d_tails, 32 * (size_t)G) != cudaSuccess) {
+    if (d_tail) cudaFree(d_tail);
+    return gspec_set_error(FSM_ENOMEM, "tail buffers");
+  }
+  const uint32_t n = (uint32_t)(shard_len < 16 ? shard_len : 16);
+  cudaMemsetAsync(d_tail, 0, 32, st);
+  if (n) cudaMemcpyAsync(d_tail + 16 - n, d_shard + shard_len - n, n, cudaMemcpyDeviceToDevice, st);
+  const uint8_t nb = (uint8_t)n;
+  cudaMemcpyAsync(d_tail + 16, &nb, 1, cudaMemcpyHostToDevice, st);
+  ncclResult_t r = nccl().allGather(d_tail, d_tails, 32, ncclUint8, c->comm, st);
+  std::vector<uint8_t> tails(32 * (size_t)G);
+  if (r == ncclSuccess)
+    cudaMemcpyAsync(tails.data(), d_tails, tails.size(), cudaMemcpyDeviceToHost, st);
+  const cudaError_t ce = cudaStreamSynchronize(st);
+  cudaFree(d_tail);
+  cudaFree(d_tails);
+  if (r != ncclSuccess) return gspec_set_error(FSM_ENCCL, "ncclAllGather (tails)");
+  if (ce != cudaSuccess) return gspec_set_error(FSM_ECUDA, "tail exchange");
+  std::vector<uint8_t> before;  // the stream's bytes before this shard, nearest last
+  for (int g = 0; g < c->rank; g++) {
+    const uint8_t m = tails[32 * (size_t)g + 16];
+    before.insert(before.end(), tails.begin() + 32 * (size_t)g + 16 - m, tails.begin() + 32 * (size_t)g + 16);
+  }
+  const size_t L = shard_offset == 0 ? 0 : std::min<size_t>(16, before.size());
+  uint8_t* d_lb = nullptr;
+  if (L) {
+    if (cudaMalloc(&d_lb, 16) != cudaSuccess) return gspec_set_error(FSM_ENOMEM, "lookback buffer");
+    cudaMemcpy(d_lb, before.data() + before.size() - L, L, cudaMemcpyHostToDevice);
+  }
+  const int rc = fsm_run_sharded(f, c, d_shard, shard_len, d_lb, (uint32_t)L, opts, d_chunk_ends_local, out_global);
+  if (d_lb) cudaFree(d_lb);
+  return rc;
 }
 
 void fsm_comm_free(fsm_comm_t c) {

@@ -91,15 +91,19 @@ def test_single_rank_nccl_group(gs):
 
 
 def test_library_nccl_single_rank(gs):
-    """fsm_comm_init + fsm_run_sharded with a real (1-rank) NCCL communicator."""
+    """fsm_comm_init + fsm_run_sharded (and the offset form fsm_run_sharded_at) with a real
+    (1-rank) NCCL communicator."""
     w = gen.workload("c2", length=8 << 20)
     data = w.host()
     ref = oracle.run(w.table, w.start, w.accept, data, 4096)
     fsm = gs.FSM.load(w.table, w.start, w.accept)
-    comm = gs.Comm(1, 0, gs.Comm.unique_id())
-    r = comm.run_sharded(fsm, torch.from_numpy(data).cuda())
-    assert r.final_state == ref["final"] and r.accept_count == ref["count"]
-    assert (r.chunk_ends.cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
+    comm = gs.Comm(1, 0, gs.Comm.unique_id(), device=0)
+    x = torch.from_numpy(data).cuda()
+    for r in (comm.run_sharded(fsm, x), comm.run_sharded_at(fsm, x, 0, x.numel())):
+        assert r.final_state == ref["final"] and r.accept_count == ref["count"]
+        assert (r.chunk_ends.cpu().numpy().view(np.uint32) == ref["chunk_end"]).all()
+    with pytest.raises(gs.GSpecError):
+        comm.run_sharded_at(fsm, x[4096:], 100, x.numel())  # not chunk-aligned
     comm.close()
 
 
