@@ -115,6 +115,11 @@ typedef struct {
    * scheme rounds = merge rounds, tasks_mustdo = stage-2 recoveries, verify_checks =
    * stage-2 steps, verify_matches = stage-2 jumps. */
   uint64_t pm_merge_checks, pm_invalid_marks, pm_jumps;
+  /* RR / NF with memoized helpers (opt-in GSPEC_LAZY_HELPERS=1, R28): helper
+   * records actually walked (a helper's record then holds its start at once and is walked
+   * when a verification first matches it); 0 with eager helpers.  tasks_helper and
+   * reread_bytes count every assigned helper either way, as the round semantics define. */
+  uint64_t helper_walks;
 } fsm_result;
 
 typedef struct {

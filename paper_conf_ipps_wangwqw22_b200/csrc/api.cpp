@@ -248,6 +248,7 @@ void fill_result_stats(fsm_result* out, const Ctl& h) {
   out->pm_merge_checks = h.pm_merge_checks;
   out->pm_invalid_marks = h.pm_invalid_marks;
   out->pm_jumps = h.pm_jumps;
+  out->helper_walks = h.helper_walks;
 }
 
 int select_auto(fsm_t f, const uint8_t* d_in, uint64_t len, const fsm_run_opts* opts);
@@ -320,6 +321,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
   rp.vr_oth = o.vr_oth;
   rp.q0_dev = q0_dev;
   rp.stamps = stamps_enabled() ? 1u : 0u;
+  rp.lazy_helpers = lazy_helpers_enabled() ? 1u : 0u;
   cudaEvent_t* ev = f->ev[slot];
   Ctl& h = f->h_ctl[slot];
   std::memset(&h, 0, sizeof(Ctl));

@@ -27,6 +27,7 @@ enum Mode : uint32_t {
 constexpr uint32_t kDeltaExc = 2;        // exceptions per delta row
 constexpr uint32_t kInvalidMap = 0xFFFFFFFEu;  // map entry of a speculative shard map that must be redone
 constexpr uint32_t kErrorMap = 0xFFFFFFFDu;    // map of a rank whose fsm_shard_map failed (count[0] = -status)
+constexpr uint32_t kPendEnd = 0xFFFFFFFCu;     // end of a memoized helper record not walked yet (R28)
 constexpr uint32_t kDeltaBaseMax = 8192;  // MODE_U16D: max shared-window offset of the staged table
 
 constexpr uint32_t kQsMax = 16;     // QS cap ("top 16 states")
@@ -139,6 +140,7 @@ struct Ctl {
   uint32_t finished, dense_rounds, dense_denied, pad2;
   // FSM_SCHEME_PM_TREE (pm_tree.cu): stage-1 lookups, entries marked invalid, stage-2 jumps
   uint64_t pm_merge_checks, pm_invalid_marks, pm_jumps;
+  uint64_t helper_walks;  // RR / NF helper records actually walked (memoized helpers, R28)
 };
 
 struct RunParams {
@@ -167,6 +169,7 @@ struct RunParams {
   uint32_t* v0_bflag;      // [tiles] tile-boundary arrival counters (+2 per run, never reset)
   uint32_t* v0_chunk_ends; // nullable: the run's chunk ends (original ids)
   uint32_t tma_evict_normal;  // 1: input TMA loads with L2 evict_normal (else evict_first)
+  uint32_t lazy_helpers;      // 1: RR / NF helper records are memoized (walked when first matched, R28)
 };
 
 // GSPEC_STAMPS=1: kernels record the run timeline in Ctl::tl (one extra atomic per warp).
@@ -216,6 +219,19 @@ inline int tma_evict_mode() {
     v = e ? atoi(e) : 0;
   }
   return v;
+}
+
+// RR / NF helpers memoized (R28): opt-in, GSPEC_LAZY_HELPERS=1.  Measured slower on C3
+// (RR 3.14 vs 2.53 ms, NF 8.56 vs 2.45 ms): the helpers the verification does consult sit
+// on its critical path, and walking them there, one per owner thread and pass, costs more
+// than walking every helper up front on the TMA task kernel.
+inline bool lazy_helpers_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("GSPEC_LAZY_HELPERS");
+    v = (e && atoi(e) == 1) ? 1 : 0;
+  }
+  return v != 0;
 }
 
 inline bool pdl_enabled() {

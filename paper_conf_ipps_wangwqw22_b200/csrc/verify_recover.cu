@@ -206,14 +206,37 @@ __device__ uint32_t untried_scan(const DevImage& img, const RunParams& rp, const
   return m;
 }
 
+// Memoized helpers (R28): a VR^others record whose end is kPendEnd holds only its start;
+// the first verification that matches it walks it (FSM_Processing from that start, with
+// path fusion) and stores its end and count.  Called by the chunk's owner thread only.
+template <int MODE>
+__device__ __forceinline__ void resolve_pending(const DevImage& img, const uint8_t* smem, const RunParams& rp,
+                                             const RecStore& rs, uint64_t c, uint32_t x, uint32_t* end,
+                                             uint32_t* cnt, Ctl* ctl) {
+  const uint32_t no = min(ld_cg(rs.n_oth + c), rp.vr_oth);
+  for (uint32_t sl = 0; sl < no; sl++) {
+    const uint64_t o = (uint64_t)(kVrMax + sl) * rs.cap + c;
+    if (ld_cg(rs.start + o) != x || ld_cg(rs.end + o) != kPendEnd) continue;
+    uint32_t e, k;
+    task_walk<MODE>(img, smem, rp, rs, c, x, &e, &k);
+    st_cg(rs.cnt + o, k);
+    st_cg(rs.end + o, e);
+    *end = e;
+    if (cnt) *cnt = k;
+    atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->helper_walks), 1ull);
+    return;
+  }
+}
+
 // Chained (Gauss-Seidel) relaxation pass over chunks [c0, hi) by one warp (see the
 // pass loop): x_{c+1} = F_c(x_c), F_c(x) = VR_c(x).end if x in dom VR_c else cur_end[c].
 // Returns whether any x_{c+1} changed.  Lane l holds chunk (b0 + l)'s default end and up
 // to kChainRec END records in registers; chunks with more records (or VR^others records)
 // fall back to the full lookup for their own step.
 constexpr int kChainRec = 8;
-__device__ bool chain_pass(const RecStore& rs, const RunParams& rp, uint64_t c0, uint64_t hi, uint64_t f,
-                           uint32_t tf) {
+template <int MODE>
+__device__ bool chain_pass(const DevImage& img, const uint8_t* smem, const RecStore& rs, const RunParams& rp,
+                           uint64_t c0, uint64_t hi, uint64_t f, uint32_t tf, Ctl* ctl) {
   const uint32_t lane = threadIdx.x & 31;
   bool ch = false;
   if (c0 >= hi) return false;
@@ -242,7 +265,10 @@ __device__ bool chain_pass(const RecStore& rs, const RunParams& rp, uint64_t c0,
         if (s[j] == x) { y = e[j]; hit = true; }
       if (lane == i && !hit && spill) {
         uint32_t y2;
-        if (vr_lookup(rs, rp.vr_end, rp.vr_oth, cc, x, &y2, nullptr)) y = y2;
+        if (vr_lookup(rs, rp.vr_end, rp.vr_oth, cc, x, &y2, nullptr)) {
+          if (y2 == kPendEnd) resolve_pending<MODE>(img, smem, rp, rs, cc, x, &y2, nullptr, ctl);
+          y = y2;
+        }
       }
       x = __shfl_sync(0xffffffffu, y, i);
       if (lane == i) mine = x;
@@ -486,7 +512,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       // round is always a normal pass (it does the bookkeeping below).
       const bool chain = it >= 3 && (it & 1u);
       if (chain) {
-        if (threadIdx.x < 32) ch = chain_pass(rs, rp, max(lo, f), hi, f, tf);
+        if (threadIdx.x < 32) ch = chain_pass<MODE>(img, smem, rs, rp, max(lo, f), hi, f, tf, ctl);
       } else
       // batched: a thread's kU chunks issue all their loads (incoming state, current
       // outgoing state, default end, record slot 0) before any is resolved; reading
@@ -511,6 +537,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
           uint32_t e;
           const bool hit = use_cache ? vr_lookup_cached(vc, (uint32_t)(c - lo), rs, rp.vr_end, rp.vr_oth, c, xin_c, &e)
                                      : vr_resolve(pre[u], rs, rp.vr_end, rp.vr_oth, c, xin_c, &e, nullptr);
+          if (hit && e == kPendEnd) resolve_pending<MODE>(img, smem, rp, rs, c, xin_c, &e, nullptr, ctl);
           rs.found[c] = hit;
           if (!hit) e = ce[u];  // F_c default: the chunk's end as of the round start
           if (xo[u] != e) {
@@ -754,8 +781,32 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     // after its walks (VR^others counts, QS cursors) is committed here first; the task
     // kernel writes each helper record at its precomputed ring slot oth_base[c] + j.
     if (helpers && rp.dense && rp.dense_slots > 0) {
-      const uint64_t nslots = nA + I;
+      const uint64_t nslots = rp.lazy_helpers ? nA : nA + I;  // memoized helpers are not walked here
       if (nslots >= 2048 && nslots * 16 >= N - f2) {
+        if (rp.lazy_helpers) {  // the helpers' pending records (start only) + their counters
+          const uint64_t T = (uint64_t)G * kBS, gt = (uint64_t)b * kBS + threadIdx.x;
+          uint64_t hel = 0, reread = 0;
+          for (uint64_t s2 = nA + gt; s2 < nA + I; s2 += T) {
+            const uint32_t c = __ldcg(rs.task_chunk + s2);
+            if (c == kNone) continue;
+            const uint32_t j = __ldcg(rs.task_j + s2);
+            if (j + rp.vr_oth >= __ldcg(rs.hcnt + c)) {  // FIFO survivors only (R16b)
+              const uint64_t o = (uint64_t)(kVrMax + (ld_cg(rs.oth_base + c) + j) % rp.vr_oth) * rs.cap + c;
+              st_cg(rs.start + o, __ldcg(rs.task_start + s2));
+              st_cg(rs.end + o, kPendEnd);
+              st_cg(rs.cnt + o, 0u);
+            }
+            hel++;
+            reread += min((uint64_t)rp.B, rp.len - (uint64_t)c * rp.B);
+          }
+          hel = block_sum<uint64_t>(hel, red64);
+          reread = block_sum<uint64_t>(reread, red64);
+          if (threadIdx.x == 0 && hel) {
+            atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_helper), (unsigned long long)hel);
+            atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->active_sum), (unsigned long long)hel);
+            atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->reread_bytes), (unsigned long long)reread);
+          }
+        }
         for (uint64_t c = max(lo, f2 + 1) + threadIdx.x; c < hi; c += kBS) {
           const uint32_t h = __ldcg(rs.hcnt + c);
           if (h) st_cg(rs.n_oth + c, ld_cg(rs.n_oth + c) + h);
@@ -778,8 +829,8 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         const uint32_t c = __ldcg(rs.task_chunk + s);
         if (c == kNone) continue;
         const uint32_t st = __ldcg(rs.task_start + s);
-        uint32_t e, cnt;
-        task_walk<MODE>(img, smem, rp, rs, c, st, &e, &cnt);
+        uint32_t e = kPendEnd, cnt = 0;
+        if (s < nA || !rp.lazy_helpers) task_walk<MODE>(img, smem, rp, rs, c, st, &e, &cnt);  // R28
         reread += min((uint64_t)rp.B, rp.len - (uint64_t)c * rp.B);
         if (s < nA) {  // VR^end: the chunk's own (must-do or SRE) record
           const uint32_t ne = ld_cg(rs.n_end + c);
@@ -855,6 +906,7 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
         if (c >= hi) break;
         uint32_t e = 0, cnt = 0;
         vr_resolve(pre[u], rs, rp.vr_end, rp.vr_oth, c, xin[u], &e, &cnt);
+        if (e == kPendEnd) resolve_pending<MODE>(img, smem, rp, rs, c, xin[u], &e, &cnt, ctl);
         total += cnt;
         if (chunk_ends) chunk_ends[c] = __ldg(img.inv + xo[u]);
       }

@@ -605,3 +605,40 @@ def test_cse_spec16(gs, name, length, B, k):
     sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme="cse", spec_k=k)
     for key in ("rounds", "tasks_mustdo", "tasks_sre", "reread_bytes", "verify_checks", "verify_matches"):
         assert res.stats[key] == sim[key], (key, res.stats[key], sim[key])
+
+
+@pytest.mark.parametrize("name,length,B,scheme", [("c3", 32 << 20, 4096, "rr"), ("c3s", 64 << 20, 4096, "nf"),
+                                                  ("rand:40:7:3", 4 << 20, 256, "rr"), ("c1", 1 << 20, 1024, "nf")])
+def test_memoized_helpers_match_eager(gs, name, length, B, scheme):
+    """R28: memoized RR / NF helpers (opt-in GSPEC_LAZY_HELPERS=1: walked when a
+    verification first matches them) give the eager helpers' results and round counters
+    exactly; only helper_walks differs.  The memoized run is a child process (the switch is
+    read once per process); this process runs the default eager helpers."""
+    import json
+    import os
+    import subprocess
+    import sys
+
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme=scheme)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    x = torch.from_numpy(data).cuda()
+    for _ in range(2):  # the second run uses the dense-round slots the first one sized
+        res = fsm.run(x, scheme=scheme, chunk_bytes=B)
+        check_equal(res, ref, B, w.nstates)
+        for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks",
+                  "verify_matches"):
+            assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+    assert res.stats["helper_walks"] == 0  # eager by default
+    code = ("import sys, json, torch; sys.path.insert(0, '.'); import gen, paper_conf_ipps_wangwqw22_b200 as gs;"
+            f"w = gen.workload({name!r}, length={length}); x = torch.empty({length}, dtype=torch.uint8, device='cuda');"
+            "w.device(x); f = gs.FSM.load(w.table, w.start, w.accept);"
+            f"r = [f.run(x, scheme={scheme!r}, chunk_bytes={B}) for _ in range(2)][-1];"
+            "print(json.dumps([r.final_state, r.accept_count, r.stats['tasks_helper'], r.stats['helper_walks']]))")
+    env = dict(os.environ, GSPEC_LAZY_HELPERS="1")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env, cwd=root, timeout=600)
+    assert out.returncode == 0, out.stderr[-2000:]
+    fin, cnt, th, hw = json.loads(out.stdout.strip().splitlines()[-1])
+    assert (fin, cnt, th) == (res.final_state, res.accept_count, res.stats["tasks_helper"]) and hw <= th
