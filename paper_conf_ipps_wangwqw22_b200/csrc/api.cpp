@@ -1525,9 +1525,18 @@ int shard_map_body(fsm_t f, const uint8_t* d_shard, uint64_t len, const uint8_t*
       }
       if ((rc = run_enqueue(f, d_shard, len, o, scheme, f->img.q0t, d_chunk_ends_local, &f->shard_ticket, S.cand)))
         return rc;
-      CUDA_TRY(launch_map_fused(S.cand, d_ncand, dcnt, &f->d_ctl->xfin,
-                                reinterpret_cast<const unsigned long long*>(&f->d_ctl->accept_count), mend, mcnt,
-                                (lb_len != 0 && !exact) ? d_unmerged : nullptr, o.st));
+      if (f->p2p_pub) {  // peer-memory exchange: the map kernel also sends the map (p2p.cu)
+        const auto& pp = *f->p2p_pub;
+        CUDA_TRY(launch_map_fused_publish(S.cand, d_ncand, dcnt, &f->d_ctl->xfin,
+                                          reinterpret_cast<const unsigned long long*>(&f->d_ctl->accept_count), mend,
+                                          mcnt, (lb_len != 0 && !exact) ? d_unmerged : nullptr, pp.mapb, pp.peers,
+                                          pp.G, pp.rank, pp.set, pp.seq, o.st));
+        f->p2p_published = true;
+      } else {
+        CUDA_TRY(launch_map_fused(S.cand, d_ncand, dcnt, &f->d_ctl->xfin,
+                                  reinterpret_cast<const unsigned long long*>(&f->d_ctl->accept_count), mend, mcnt,
+                                  (lb_len != 0 && !exact) ? d_unmerged : nullptr, o.st));
+      }
       f->shard_mode = 3;
       return FSM_OK;
     }

@@ -366,6 +366,11 @@ cudaError_t launch_qs_long(const DevImage& img, const uint32_t* d_ttc, const uin
 uint64_t pm_tree_scratch_bytes(uint64_t N, uint32_t k, uint32_t* levels);
 cudaError_t launch_pm_tree(const DevImage& img, const RunParams& rp, const RecStore& rs, uint32_t k, void* scratch,
                            Ctl* ctl, uint32_t* d_chunk_ends, int sms, cudaStream_t st, uint32_t* launches);
+cudaError_t launch_map_fused_publish(const uint32_t* cand, const uint32_t* ncand_p, const long long* dcnt,
+                                     const uint32_t* fin_p, const unsigned long long* count_p, uint32_t* mend,
+                                     unsigned long long* mcnt, const uint32_t* unmerged, uint64_t mapb,
+                                     uint8_t* const* peers, uint32_t G, uint32_t rank, uint32_t set,
+                                     unsigned long long seq, cudaStream_t st);
 cudaError_t launch_publish(const uint8_t* own_map, uint64_t mapb, uint8_t* const* peers, uint32_t G, uint32_t rank,
                            uint32_t set, unsigned long long seq, cudaStream_t st);
 cudaError_t launch_wait_flags(const uint8_t* own_box, uint64_t mapb, uint32_t G, uint32_t rank, uint32_t set,
@@ -464,12 +469,22 @@ struct fsm_s {
   void* batch_base = nullptr;            // fsm_run_batch scratch (offsets, chunk bases, records, totals)
   size_t batch_bytes = 0;
   cudaEvent_t batch_ev[2] = {nullptr, nullptr};
-  uint8_t* prof_buf = nullptr;
+  uint8_t* prof_buf = nullptr;           // FSM_SCHEME_AUTO's spread 1 MiB profile sample
+  // set by fsm_run_sharded_p2p around its fsm_shard_map call: the fused-mode map kernel then
+  // also publishes the map to the peers (k_map_fused_publish) and sets p2p_published
+  struct P2PPub {
+    uint64_t mapb;
+    uint8_t* const* peers;
+    uint32_t G, rank, set;
+    unsigned long long seq;
+  };
+  const P2PPub* p2p_pub = nullptr;
+  bool p2p_published = false;
   void* img2_base = nullptr;             // lookback > 2: full pair images (built at first use)
   uint32_t *img2_s = nullptr, *img2_m = nullptr;
   uint8_t* img2_n = nullptr;
   void* qsc_base = nullptr;              // lookback > 2: per-run QS table [N][kQsMax] + lengths
-  uint64_t qsc_cap = 0;           // FSM_SCHEME_AUTO's spread 1 MiB profile sample
+  uint64_t qsc_cap = 0;
   void* pm_base = nullptr;               // FSM_SCHEME_PM_TREE scratch (level maps, jump list)
   size_t pm_bytes = 0;
   void* multi_base = nullptr;            // fsm_run_multi scratch when this handle is fsms[0] (its device)

@@ -2,9 +2,11 @@
 // (SURVEY §8(e) "fused alternative"): every rank owns a mailbox in its
 // own HBM — two sets (by step parity) of G map slots plus G arrival flags — mapped into
 // every peer through CUDA IPC (NVLink / NVSwitch peer memory between GPUs).  A step is
-//   map kernels (fsm_shard_map, into this rank's own slot)
-//   -> k_publish: one CTA stores the map into slot [rank] of every peer's mailbox, fences
-//      system-wide and raises the flag [rank] there (remote stores, no NCCL launch)
+//   map kernels (fsm_shard_map, into this rank's own slot); in the fused mode the last
+//      of them, k_map_fused_publish (shard.cu), writes the candidates' map entries AND
+//      stores the finished map into slot [rank] of every peer's mailbox, fences
+//      system-wide and raises the flag [rank] there — the compute step and the exchange in
+//      one kernel, no NCCL launch; the other modes publish with k_publish (the same stores)
 //   -> k_wait_flags: spins (with nanosleep, bounded) until every peer's flag for this
 //      step has arrived in the own mailbox
 //   -> fsm_shard_finish over the own mailbox (compose, fix-up), as after an allgather.
@@ -170,12 +172,19 @@ int fsm_run_sharded_p2p(fsm_t f, fsm_p2p_t p, const uint8_t* d_shard, uint64_t s
     const unsigned long long seq = ++p->seq;
     const uint32_t set = (uint32_t)(seq & 1);
     uint8_t* own_slot = p->box + ((uint64_t)set * G + rank) * p->mapb;
+    // the fused-mode map kernel sends the map itself (k_map_fused_publish); the other modes
+    // (exact fallbacks, ENUM shards, an error map) publish with k_publish afterwards
+    const fsm_s::P2PPub pub{p->mapb, p->d_peers, G, rank, set, seq};
+    f->p2p_pub = &pub;
+    f->p2p_published = false;
     rc = exact ? fsm_shard_map_exact(f, d_shard, shard_len, d_lookback, lookback_len, opts, own_slot,
                                      d_chunk_ends_local)
                : fsm_shard_map(f, d_shard, shard_len, d_lookback, lookback_len, opts, own_slot, d_chunk_ends_local);
+    f->p2p_pub = nullptr;
     if (rc && f->shard_mode != 4) return rc;  // (a failed map publishes its error map like any other)
     const int map_rc = rc;
-    if (gspec::launch_publish(own_slot, p->mapb, p->d_peers, G, rank, set, seq, st) != cudaSuccess ||
+    const bool sent = f->p2p_published && !rc;
+    if ((!sent && gspec::launch_publish(own_slot, p->mapb, p->d_peers, G, rank, set, seq, st) != cudaSuccess) ||
         gspec::launch_wait_flags(p->box, p->mapb, G, rank, set, seq, p->d_status, st) != cudaSuccess ||
         cudaMemcpyAsync(p->h_status, p->d_status, 4, cudaMemcpyDeviceToHost, st) != cudaSuccess)
       return gspec_set_error(FSM_ECUDA, "p2p publish / wait launch");

@@ -161,6 +161,39 @@ __global__ void k_map_fused(const uint32_t* __restrict__ cand, const uint32_t* _
   }
 }
 
+// P2P exchange (p2p.cu), fused mode: ONE kernel computes this rank's map entries (as
+// k_map_fused) and sends the finished map to every peer — one CTA writes the candidates'
+// entries, then stores the whole map (k_map_init wrote the rest earlier in the stream) into
+// slot [rank] of every peer's mailbox, fences system-wide and raises its flag there.
+__global__ void __launch_bounds__(1024) k_map_fused_publish(
+    const uint32_t* __restrict__ cand, const uint32_t* __restrict__ ncand_p, const long long* __restrict__ dcnt,
+    const uint32_t* __restrict__ fin_p, const unsigned long long* __restrict__ count_p, uint32_t* __restrict__ mend,
+    unsigned long long* __restrict__ mcnt, const uint32_t* __restrict__ unmerged, uint64_t mapb,
+    uint8_t* const* __restrict__ peers, uint32_t G, uint32_t rank, uint32_t set, unsigned long long seq) {
+  const uint32_t ncand = *ncand_p;
+  const uint32_t fin = (unmerged && *unmerged) ? kInvalidMap : *fin_p;
+  const unsigned long long c0 = *count_p;
+  for (uint32_t i = threadIdx.x; i < ncand; i += blockDim.x) {
+    mend[cand[i]] = fin;
+    mcnt[cand[i]] = (unsigned long long)((long long)c0 + dcnt[i]);
+  }
+  __syncthreads();  // the whole map is final (block-scope: this CTA wrote the candidates)
+  __threadfence();
+  const uint4* src = reinterpret_cast<const uint4*>(mend);
+  const uint64_t words = mapb / 16;
+  for (uint32_t g = 0; g < G; g++) {
+    if (g == rank) continue;
+    uint4* dst = reinterpret_cast<uint4*>(peers[g] + ((uint64_t)set * G + rank) * mapb);
+    for (uint64_t i = threadIdx.x; i < words; i += blockDim.x) dst[i] = __ldcg(src + i);
+  }
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x < G && threadIdx.x != rank) {
+    unsigned long long* flags = reinterpret_cast<unsigned long long*>(peers[threadIdx.x] + 2ull * G * mapb);
+    *reinterpret_cast<volatile unsigned long long*>(flags + (uint64_t)set * G + rank) = seq;
+  }
+}
+
 // finish (fused mode): locate this rank's start among the candidates and write
 // the chunk ends walked before it merged with the reference path
 __global__ void k_fix_prefix_fused(const uint32_t* __restrict__ states, const uint32_t* __restrict__ cand,
@@ -337,6 +370,16 @@ cudaError_t launch_map_fused(const uint32_t* cand, const uint32_t* ncand_p, cons
                              const unsigned long long* count_p, uint32_t* mend, unsigned long long* mcnt,
                              const uint32_t* unmerged, cudaStream_t st) {
   k_map_fused<<<8, 256, 0, st>>>(cand, ncand_p, dcnt, fin_p, count_p, mend, mcnt, unmerged);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_map_fused_publish(const uint32_t* cand, const uint32_t* ncand_p, const long long* dcnt,
+                                     const uint32_t* fin_p, const unsigned long long* count_p, uint32_t* mend,
+                                     unsigned long long* mcnt, const uint32_t* unmerged, uint64_t mapb,
+                                     uint8_t* const* peers, uint32_t G, uint32_t rank, uint32_t set,
+                                     unsigned long long seq, cudaStream_t st) {
+  k_map_fused_publish<<<1, 1024, 0, st>>>(cand, ncand_p, dcnt, fin_p, count_p, mend, mcnt, unmerged, mapb, peers, G,
+                                          rank, set, seq);
   return cudaGetLastError();
 }
 
