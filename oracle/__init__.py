@@ -71,6 +71,10 @@ def lib():
                                           ctypes.POINTER(SimResult), ctypes.POINTER(PmStats)]
         L.or_features_compute.argtypes = [P, U32, U32, U32, P, P, U64, U32, U32, U32, ctypes.POINTER(Features)]
         L.or_select.argtypes = [ctypes.POINTER(Features), U32]
+        L.or_conv_lengths.argtypes = [P, U32, U32, P, U64, U32, P]
+        L.or_conv_lengths.restype = U32
+        L.or_select_chunk.argtypes = [P, U32, U64, U64]
+        L.or_select_chunk.restype = U32
         _LIB = L
     return _LIB
 
@@ -294,3 +298,21 @@ def features(table, start, accept, data, B=4096, k=4, qs_cap=16, policy=0):
 def select(feat: dict, nstates: int) -> int:
     f = Features(feat["acc1"], feat["acck"], feat["sens"], feat["uniq10"])
     return int(lib().or_select(ctypes.byref(f), nstates))
+
+
+def conv_lengths(table, start, accept, data, wmax=16384, policy=0):
+    """Convergence lengths of the lookback-2 image over 4 KiB-spaced windows (reading
+    R29): uint32 per window, 0xFFFFFFFF = not converged within wmax."""
+    perm, inv, _, tt, acc = transform(table, accept, policy, data if policy == 1 else None, start)
+    n, ns = _c(table, np.uint32).shape
+    d = _c(data, np.uint8)
+    nwin = lib().or_conv_lengths(tt.ctypes.data, n, ns, d.ctypes.data, d.size, wmax, None)
+    out = np.zeros(max(nwin, 1), dtype=np.uint32)
+    lib().or_conv_lengths(tt.ctypes.data, n, ns, d.ctypes.data, d.size, wmax, out.ctypes.data)
+    return out[:nwin]
+
+
+def select_chunk(d, length, min_chunks):
+    """Chunk size (granularity) from convergence lengths (reading R29)."""
+    d = _c(d, np.uint32)
+    return int(lib().or_select_chunk(d.ctypes.data if d.size else None, d.size, length, min_chunks))

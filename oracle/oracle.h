@@ -149,6 +149,14 @@ int or_features_compute(const uint32_t* tt, uint32_t nt, uint32_t nsyms, uint32_
                         const uint8_t* in, uint64_t len, uint32_t B, uint32_t k, uint32_t qs_cap,
                         or_features* out);
 
+/* Convergence lengths of the lookback image over 4 KiB-spaced windows (reading
+ * R29).  Returns the number of windows; d_out nullable. */
+uint32_t or_conv_lengths(const uint32_t* tt, uint32_t nt, uint32_t nsyms, const uint8_t* in, uint64_t len,
+                         uint32_t wmax, uint32_t* d_out);
+
+/* Chunk size from the convergence lengths (reading R29). */
+uint32_t or_select_chunk(const uint32_t* d, uint32_t nwin, uint64_t len, uint64_t min_chunks);
+
 /* Decision tree (Fig. 6 reconstructed, reading c.4 #19). Returns a scheme id. */
 int or_select(const or_features* f, uint32_t nstates);
 

@@ -748,3 +748,86 @@ def test_run_stream_div7_closed_form():
     assert r["final"] == int("".join(map(str, bits)), 2) % 7
     assert r["accept"] == int(r["final"] == 0)
     assert r["count"] == int((res == 0).sum())
+
+
+# ------------------------------------------- convergence lengths (R29) -------
+def _conv_windows(length, wmax):
+    return [j * 4096 for j in range(1, length) if j * 4096 + wmax <= length and 1 <= j % 32 <= 28]
+
+
+def test_conv_lengths_reset_closed_form():
+    """R29 on C3 (AC x Z16, the counter reset by '#'): the lookback image holds states with
+    different counter values (vowels move every path's counter alike, so they cannot meet
+    before a reset) and the reset byte sends every AC state to the root and every counter
+    to 0 — so all paths meet exactly at the window's first '#': d = that offset + 1
+    rounded up to 64 bytes, or 'never' when the window holds no '#'.  Windows whose
+    2-byte lookback contains '#' (a counter already known) are left out of the pin."""
+    w = gen.workload("c3", length=600 << 10, seed=7)
+    data = w.host()
+    wmax = 4096  # one '#' per 8 KiB block: about half the windows reach one
+    assert all(gen.RESET_BYTE not in lit for lit in w.literals)
+    d = oracle.conv_lengths(w.table, w.start, w.accept, data, wmax=wmax)
+    wins = _conv_windows(len(data), wmax)
+    assert len(d) == len(wins) > 100
+    checked = reach = 0
+    for p, dw in zip(wins, d):
+        if gen.RESET_BYTE in bytes(data[p - 2:p]):
+            continue
+        seg = bytes(data[p:p + wmax])
+        r = seg.find(bytes([gen.RESET_BYTE]))
+        expect = 0xFFFFFFFF if r < 0 else -(-(r + 1) // 64) * 64
+        assert int(dw) == expect, (p, r, int(dw))
+        checked += 1
+        reach += r >= 0
+    assert checked > 100 and 0 < reach < checked
+
+
+def test_conv_lengths_permutation_and_constant():
+    """div7 (every symbol permutes the states: paths never meet) -> never; a DFA whose
+    next state depends on the symbol only (lookback image = one state) -> 0."""
+    t, s, a = gen.dfa_div7()
+    rng = np.random.default_rng(3)
+    bits = rng.integers(0, 2, 300 << 10).astype(np.uint8)
+    d = oracle.conv_lengths(t, s, a, bits, wmax=8192)
+    assert len(d) == len(_conv_windows(bits.size, 8192)) and (d == 0xFFFFFFFF).all()
+    n, ns = 5, 8
+    tc = np.tile((np.arange(ns) % n).astype(np.uint32), (n, 1))
+    data = rng.integers(0, ns, 200 << 10).astype(np.uint8)
+    d = oracle.conv_lengths(tc, 0, np.array([1, 0, 0, 0, 0], np.uint8), data, wmax=4096)
+    assert len(d) > 0 and (d == 0).all()
+
+
+def test_conv_lengths_two_state_merge_bruteforce():
+    """A 3-state DFA where symbol 0 sends every state to 0 and other symbols permute
+    states 1 <-> 2 (and fix 0): paths from distinct states meet at the first 0 symbol.
+    Brute force per window: the image (from the 2 lookback symbols) and the first 0."""
+    # row s: symbol 0 -> 0; symbol 1 -> swap 1/2 (0 stays 0); symbol 2 -> identity
+    t = np.array([[0, 0, 0], [0, 2, 1], [0, 1, 2]], np.uint32)
+    rng = np.random.default_rng(11)
+    data = rng.choice(3, size=160 << 10, p=[0.0005, 0.4995, 0.5]).astype(np.uint8)
+    d = oracle.conv_lengths(t, 0, np.array([1, 0, 0], np.uint8), data, wmax=8192)
+    for p, dw in zip(_conv_windows(data.size, 8192), d):
+        img = {int(t[int(t[q, data[p - 2]]), data[p - 1]]) for q in range(3)}
+        if len(img) <= 1:
+            assert dw == 0
+            continue
+        r = np.nonzero(data[p:p + 8192] == 0)[0]
+        expect = 0xFFFFFFFF if r.size == 0 else -(-(int(r[0]) + 1) // 64) * 64
+        assert int(dw) == expect
+
+
+def test_select_chunk_rule():
+    """R29's rule: the smallest W in {4, 8, 16} KiB with >= 3/4 of the windows converged
+    within W and >= min_chunks chunks of W (W = 4 KiB always allowed); else 4 KiB."""
+    never = 0xFFFFFFFF
+    G = 1 << 30
+    assert oracle.select_chunk([0] * 8, G, 113664) == 4096
+    assert oracle.select_chunk([], G, 113664) == 4096
+    assert oracle.select_chunk([never] * 8, G, 113664) == 4096
+    d8 = [64, 4096, 5000, 8192, 8000, 7000, 6000, never]  # 2/8 within 4K, 7/8 within 8K
+    assert oracle.select_chunk(d8, G, 113664) == 8192
+    assert oracle.select_chunk(d8, G, 131073) == 4096        # 1 GiB / 8 KiB = 131072 chunks < 131073
+    d16 = [64, 9000, 10000, 12000, 16384, 16000, 5000, never]  # 2/8 within 8K, 7/8 within 16K
+    assert oracle.select_chunk(d16, 16 * G, 113664) == 16384
+    assert oracle.select_chunk(d16, G, 113664) == 4096
+    assert oracle.select_chunk([64, 64, 64, never], G, 113664) == 4096  # exactly 3/4 within 4K
