@@ -167,7 +167,7 @@ class _Pinned:
             os.sched_setaffinity(0, self.old)
 
 
-def cpu_baseline(w, sample_cap=256 << 20, check=None, x=None):
+def cpu_baseline(w, sample_cap=256 << 20, check=None, x=None, B=4096):
     """The oracle (plain sequential C, oracle/) on one pinned host core, bounded sample
     (the first min(len, 256 MiB) bytes of the stream), median of 3 runs.  check
     (nullable): callable(sample_len) -> the GPU result on the same prefix, compared with
@@ -187,7 +187,7 @@ def cpu_baseline(w, sample_cap=256 << 20, check=None, x=None):
     with _Pinned() as pin:
         for _ in range(3):
             t0 = time.perf_counter()
-            r = oracle.run(w.table, w.start, w.accept, data, 4096)
+            r = oracle.run(w.table, w.start, w.accept, data, B)
             times.append(time.perf_counter() - t0)
             assert r["status"] == 0
     dt = sorted(times)[1]
@@ -260,13 +260,12 @@ def _roofline(name, length, spec_ms, peak, peak_kind):
             "achieved_def": "input bytes per launch / CUDA-event duration of the spec launch on its stream"}
 
 
-def measure_single(gs, w, x, args, fsm, scheme, with_clocks=True):
+def measure_single(gs, w, x, args, fsm, scheme, B, with_clocks=True):
     """K back-to-back runs of the whole stream on this GPU (fsm_run_async queue), timed by
     two CUDA events on the launching stream; spec / verify splits from the library's
     own per-run events."""
     import torch
 
-    B = args.chunk_bytes
     length = x.numel()
     stream = torch.cuda.current_stream()
     ce = torch.empty(gs.fsm_num_chunks(length, B), dtype=torch.int32, device="cuda")
@@ -347,10 +346,11 @@ def per_dfa_result(gs, name, args, peak, peak_kind, with_cpu=True):
     prof = torch.empty(1 << 20, dtype=torch.uint8, device="cuda")
     w.device(prof, offset=w.length)
     fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof.cpu().numpy())
-    scheme, feats = fsm.select_scheme(x, chunk_bytes=args.chunk_bytes)  # spread profile (R20)
-    m = measure_single(gs, w, x, args, fsm, scheme, with_clocks=False)
+    scheme, feats = fsm.select_scheme(x)  # spread profile (R20); chunk size (R29) for this stream
+    B = args.chunk_bytes or feats["chunk_bytes"]
+    m = measure_single(gs, w, x, args, fsm, scheme, B, with_clocks=False)
     out = {"value": round(m["value"], 3), "unit": "GB/s", "ms_per_step": round(m["ms"], 4),
-           "bytes": w.length, "scheme": scheme, "nstates": int(w.nstates),
+           "bytes": w.length, "scheme": scheme, "chunk_bytes": B, "nstates": int(w.nstates),
            "pct_hbm_roofline_8TBs": round(100 * m["value"] / 8000.0, 2),
            "breakdown_ms": {"spec_exec": round(m["spec_ms"], 4), "verify_recover": round(m["ver_ms"], 4)},
            "roofline": _roofline(name, w.length, m["spec_ms"], peak, peak_kind), "diagnostics": m["diag"],
@@ -358,7 +358,7 @@ def per_dfa_result(gs, name, args, peak, peak_kind, with_cpu=True):
            "features": {k: round(v, 4) if isinstance(v, float) else v for k, v in feats.items()}}
     if with_cpu:
         out["cpu_baseline"], out["parity"] = cpu_baseline(
-            w, sample_cap=64 << 20, x=x, check=lambda n: fsm.run(x[:n], scheme=scheme, chunk_bytes=args.chunk_bytes))
+            w, sample_cap=64 << 20, x=x, check=lambda n: fsm.run(x[:n], scheme=scheme, chunk_bytes=B), B=B)
     fsm.close()
     del x
     torch.cuda.empty_cache()
@@ -417,25 +417,26 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
     import gen
     from paper_conf_ipps_wangwqw22_b200.dist import run_sharded, shard_bounds
 
-    B = args.chunk_bytes
     L = args.c5_bytes
     per = {}
     dfas = C5_DFAS if args.c5_dfa == "all" else (args.c5_dfa,)
     clk_all = None
     for name in dfas:
         w = gen.workload(name, length=L)
+        fsm = gs.FSM.load(w.table, w.start, w.accept)
+        # selector per DFA (offline profiling, P:363): every rank profiles the same 8 spread
+        # portions of the global stream (R20), so every rank picks the same scheme and the
+        # same chunk size (R29, for L / world bytes per GPU) — the shard bounds follow it
+        prof = spread_profile(w, L)
+        scheme, feats = fsm.select_scheme(prof, stream_len=L // world)
+        B = args.chunk_bytes or feats["chunk_bytes"]
+        del prof
         lo, hi = shard_bounds(L, world, rank, B)
         x = torch.empty(hi - lo, dtype=torch.uint8, device="cuda")
         w.device(x, offset=lo)
         lb = torch.empty(min(16, lo), dtype=torch.uint8, device="cuda")
         if lo:  # the 16 bytes before the shard (pure function of the offset): its candidate set
             w.device(lb, offset=lo - lb.numel())
-        fsm = gs.FSM.load(w.table, w.start, w.accept)
-        # selector per DFA (offline profiling, P:363): every rank profiles the same 8 spread
-        # portions of the global stream (R20), so every rank picks the same scheme
-        prof = spread_profile(w, L)
-        scheme, feats = fsm.select_scheme(prof, chunk_bytes=B)
-        del prof
 
         p2p = None
         if dist is not None and args.exchange == "p2p":
@@ -491,7 +492,7 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
             dist.all_reduce(t2, op=dist.ReduceOp.MAX)
             agree = bool((t == t2).all().item())
         per[name] = {"value": round(value, 3), "unit": "GB/s", "ms_per_step": round(ms, 4), "bytes": L,
-                     "bytes_per_rank": hi - lo, "scheme": scheme, "nstates": int(w.nstates),
+                     "bytes_per_rank": hi - lo, "scheme": scheme, "chunk_bytes": B, "nstates": int(w.nstates),
                      "pct_hbm_roofline_8TBs_per_gpu": round(100 * value / world / 8000.0, 2),
                      "latency_ms_per_GB": round(ms * 1e9 / L, 4), "ranks_agree": agree,
                      "final_state": res.final_state, "accept_count": res.accept_count,
@@ -505,7 +506,9 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         "warmup": max(3, args.warmup), "ms_per_step": head["ms_per_step"], "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": "c5", "desc": CONFIG_DESC["c5"], "headline_dfa": dfas[0], "bytes_total": L,
-                   "chunk_bytes": B, "l2": "input (16 GiB / N per GPU) larger than the 126 MB L2; no flush",
+                   "chunk_bytes": "per DFA (per_dfa[*].chunk_bytes: the selector's R29 recommendation)"
+                   if not args.chunk_bytes else args.chunk_bytes,
+                   "l2": "input (16 GiB / N per GPU) larger than the 126 MB L2; no flush",
                    "parallelism": f"{world} contiguous shards + one exchange of state maps"
                    + (" (peer-memory stores, fsm_run_sharded_p2p)" if dist is not None and args.exchange == "p2p" else
                       " (library NCCL allgather, fsm_run_sharded_async)" if comm is not None else
@@ -528,7 +531,9 @@ def main():
     ap.add_argument("--impl", default="own", choices=["own", "reference"])
     ap.add_argument("--config", default="c2", choices=sorted(CONFIG_DESC))
     ap.add_argument("--scheme", default="auto")
-    ap.add_argument("--chunk-bytes", type=int, default=4096)
+    ap.add_argument("--chunk-bytes", type=int, default=0,
+                    help="chunk size B; 0 = the selector's recommendation (reading R29, 4096 unless the "
+                         "profile's lookback images converge only over longer chunks)")
     ap.add_argument("--spec-k", type=int, default=0, help="paths per chunk for pm / pm_tree / cse (0 = default)")
     ap.add_argument("--lookback", type=int, default=2, help="lookback symbols per chunk prediction (2..16, R25)")
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -599,10 +604,12 @@ def main():
     scheme = args.scheme
     feats = None
     del prof
-    if scheme == "auto":  # offline profiling, untimed: 8 spread portions of the stream (R20)
+    if scheme == "auto" or not B:  # offline profiling, untimed: 8 spread portions of the stream (R20)
         sp = spread_profile(w, length * world)
-        scheme, feats = fsm.select_scheme(sp, chunk_bytes=B)
+        sel, feats = fsm.select_scheme(sp, stream_len=length)
         del sp
+        scheme = sel if scheme == "auto" else scheme
+        B = B or feats["chunk_bytes"]  # chunk size (granularity) from the profile (R29)
 
     lb = None
     if world > 1:
@@ -652,7 +659,7 @@ def main():
                                                                   "tasks_helper", "reread_bytes", "verify_checks",
                                                                   "verify_matches")}}
     else:
-        m = measure_single(gs, w, x, args, fsm, scheme)
+        m = measure_single(gs, w, x, args, fsm, scheme, B)
         res = m["result"]
         ms = m["ms"]
     total_bytes = length * world
@@ -737,7 +744,7 @@ def main():
         line["config"]["features"] = {k: round(v, 4) if isinstance(v, float) else v for k, v in feats.items()}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"], parity = cpu_baseline(
-            w, x=x, check=lambda n: fsm.run(x[:n], scheme=scheme, chunk_bytes=B))
+            w, x=x, check=lambda n: fsm.run(x[:n], scheme=scheme, chunk_bytes=B), B=B)
         if parity is not None:
             line["parity"] = parity
     if world == 1 and args.config == "c2" and args.scheme == "auto" and not args.no_per_dfa:

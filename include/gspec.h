@@ -90,7 +90,7 @@ typedef struct {
   fsm_scheme scheme;    /* FSM_SCHEME_*                                                  */
   uint32_t chunk_bytes; /* B: chunk c = [cB, min(len,(c+1)B)); multiple of 16; 0 = 4096   */
   uint32_t spec_k;      /* paths per chunk: PM (4) / CSE (8); 1..16; 0 = default   */
-  uint32_t lookback;    /* lookback symbols (2); only 2 is supported; 0 = 2        */
+  uint32_t lookback;    /* lookback symbols L (2); 2..16 (reading R25); 0 = 2     */
   uint32_t qs_cap;      /* K: ranked candidates kept per chunk (16); 1..16; 0 = 16 */
   uint32_t vr_end;      /* VR^end slots per chunk (16); 1..16; 0 = 16              */
   uint32_t vr_others;   /* VR^others slots per chunk (16); 1..16; 0 = 16           */
@@ -128,6 +128,14 @@ typedef struct {
   double input_sensitivity; /* max-min of per-segment acc1 over 8 segments (R19)       */
   double uniq10;            /* mean #unique states after 10 transitions from all */
   uint32_t nstates;
+  /* Granularity (reading R29): windows every 4 KiB of the profile, each
+   * walking every state of its lookback-2 image until all paths are in one state
+   * (checked every 64 B, up to 16 KiB).  conv{4,8,16}k = fraction of windows converged
+   * within that many bytes; chunk_bytes = the smallest of 4/8/16 KiB with a fraction
+   * >= 3/4 that still leaves >= SMs x 768 chunks of the stream (len as passed), else
+   * 4096.  A recommendation: fsm_run uses opts->chunk_bytes as given. */
+  uint32_t chunk_bytes;
+  double conv4k, conv8k, conv16k;
 } fsm_features;
 
 /* Load a DFA.  table: host uint32 [nstates][nsyms], row-major, original ids;
@@ -232,6 +240,13 @@ int fsm_run_host(fsm_t fsm, const uint8_t* h_input, uint64_t len, const fsm_run_
  * cached choice profiles the run's own input this way.  feat nullable. */
 int fsm_select_scheme(fsm_t fsm, const uint8_t* d_sample, uint64_t len, const fsm_run_opts* opts,
                       fsm_scheme* out, fsm_features* feat);
+
+/* The chunk-size rule of reading R29 for a stream of stream_len bytes per GPU, from the
+ * convergence fractions of features filled by fsm_select_scheme (e.g. when the profile
+ * was a sample of a longer stream): the smallest W in {4096, 8192, 16384} with
+ * conv{W} >= 3/4 and stream_len / W >= SMs x 768 (W = 4096 exempt), else 4096.
+ * Host-only; the current device's SM count.  NULL -> 4096. */
+uint32_t fsm_chunk_for(const fsm_features* feat, uint64_t stream_len);
 
 /* ---- multi-GPU contiguous sharding --------------------
  * A shard is a contiguous, chunk-aligned byte range [offset, offset+len) of

@@ -62,10 +62,13 @@ class fsm_multi_result(ctypes.Structure):
 
 class fsm_features(ctypes.Structure):
     _fields_ = [("acc1", ctypes.c_double), ("acck", ctypes.c_double), ("input_sensitivity", ctypes.c_double),
-                ("uniq10", ctypes.c_double), ("nstates", U32)]
+                ("uniq10", ctypes.c_double), ("nstates", U32), ("chunk_bytes", U32), ("conv4k", ctypes.c_double),
+                ("conv8k", ctypes.c_double), ("conv16k", ctypes.c_double)]
 
 
 _lib.fsm_load.argtypes = [P, U32, U32, U32, P, ctypes.POINTER(fsm_load_opts), ctypes.POINTER(P)]
+_lib.fsm_chunk_for.argtypes = [ctypes.POINTER(fsm_features), U64]
+_lib.fsm_chunk_for.restype = U32
 _lib.fsm_num_chunks.argtypes = [U64, U32]
 _lib.fsm_num_chunks.restype = U64
 _lib.fsm_run.argtypes = [P, P, U64, ctypes.POINTER(fsm_run_opts), P, ctypes.POINTER(fsm_result)]
@@ -270,13 +273,17 @@ class FSM:
                                  ce.ctypes.data if ce is not None else None, ctypes.byref(r)), "fsm_run_host")
         return Result.from_c(r, ce[:n] if ce is not None else None)
 
-    def select_scheme(self, sample, chunk_bytes=4096, spec_k=4, stream=None):
-        """fsm_select_scheme on a uint8 CUDA tensor: (scheme name, features dict)."""
+    def select_scheme(self, sample, chunk_bytes=4096, spec_k=4, stream=None, stream_len=None):
+        """fsm_select_scheme on a uint8 CUDA tensor: (scheme name, features dict).  The
+        dict's chunk_bytes is the recommended chunk size (reading R29) for a stream of
+        stream_len bytes per GPU (default: the sample's own length; fsm_chunk_for)."""
         o = _run_opts("sre", chunk_bytes, spec_k, stream=stream)
         out = ctypes.c_int(0)
         ft = fsm_features()
         _check(_lib.fsm_select_scheme(self._h, sample.data_ptr() if sample.numel() else None, sample.numel(),
                                       ctypes.byref(o), ctypes.byref(out), ctypes.byref(ft)), "fsm_select_scheme")
+        if stream_len is not None:
+            ft.chunk_bytes = _lib.fsm_chunk_for(ctypes.byref(ft), stream_len)
         return SCHEME_NAMES[out.value], {k: getattr(ft, k) for k, _ in fsm_features._fields_}
 
     # ---- introspection --------------------------------------------------------

@@ -1227,6 +1227,7 @@ int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_
   // i (len - 128 KiB) / 7, 4 KiB-aligned), gathered into one 1 MiB sample, so the
   // input-sensitivity feature compares different portions of the stream.
   constexpr uint64_t kSlice = 128 << 10, kSample = 8 * kSlice;
+  const uint64_t stream_len = len;  // the chunk-size rule's occupancy bound (R29)
   if (len > kSample) {
     if (!f->prof_buf) CUDA_TRY(cudaMalloc(&f->prof_buf, kSample));
     for (uint64_t i = 0; i < 8; i++) {
@@ -1244,7 +1245,12 @@ int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_
   const uint64_t N = r.nchunks;
   // 2. features on the device
   const uint32_t words = (f->n + 1 + 31) / 32;
-  const size_t need = 32 * 8 + 64ull * words * 4 + 64;
+  // convergence windows (R29): p = 4096 j, j mod 32 in [1, 28], p + kConvMax <= len
+  constexpr uint32_t kConvMax = 16384;
+  uint32_t nwin = 0;
+  for (uint64_t j = 1; j * 4096 + kConvMax <= len; j++) nwin += (j % 32 >= 1 && j % 32 <= 28);
+  const size_t conv_off = 32 * 8 + 64ull * words * 4 + 64;
+  const size_t need = conv_off + 4ull * nwin + 16;
   if (f->feat_bytes < need) {
     if (f->feat_base) cudaFree(f->feat_base);
     f->feat_base = nullptr;
@@ -1277,6 +1283,23 @@ int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_
     }
     if (len >= 10) ft.uniq10 = (double)h[20] / 64.0;
   }
+  // R29: convergence lengths of the lookback image -> recommended chunk size
+  ft.chunk_bytes = 4096;
+  if (nwin > 0) {
+    uint32_t* d_conv = reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(f->feat_base) + conv_off);
+    CUDA_TRY(launch_feat_conv(f->img, f->d_ttc, d_sample, nwin, kConvMax, d_conv, o.st));
+    std::vector<uint32_t> dv(nwin);
+    CUDA_TRY(cudaMemcpyAsync(dv.data(), d_conv, 4ull * nwin, cudaMemcpyDeviceToHost, o.st));
+    CUDA_TRY(cudaStreamSynchronize(o.st));
+    double* conv[3] = {&ft.conv4k, &ft.conv8k, &ft.conv16k};
+    for (uint32_t W = 4096, i = 0; W <= kConvMax; W *= 2, i++) {
+      uint64_t k = 0;
+      for (uint32_t d : dv) k += d <= W;
+      *conv[i] = (double)k / nwin;  // exact at 3/4 (0.75 is representable)
+    }
+    ft.chunk_bytes = fsm_chunk_for(&ft, stream_len);
+  }
+  f->auto_chunk = ft.chunk_bytes;
   const fsm_scheme pick = tree_select(ft, f->n);
   if (N > 1) f->acc1_hint = ft.acc1;
   f->auto_scheme = pick;
@@ -1284,6 +1307,15 @@ int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_
   *outp = pick;
   if (feat) *feat = ft;
   return FSM_OK;
+}
+
+uint32_t fsm_chunk_for(const fsm_features* ft, uint64_t stream_len) {
+  if (!ft) return 4096;
+  const uint64_t min_chunks = (uint64_t)device_sms() * 768;  // 24 warps per SM of one-chunk lanes
+  const double conv[3] = {ft->conv4k, ft->conv8k, ft->conv16k};
+  for (uint32_t W = 4096, i = 0; i < 3; W *= 2, i++)
+    if (conv[i] >= 0.75 && (W == 4096 || stream_len / W >= min_chunks)) return W;
+  return 4096;
 }
 
 int fsm_get_transform(fsm_t f, uint32_t* perm, uint32_t* inv, uint64_t* freq, uint32_t* mode, uint32_t* hot_rows,

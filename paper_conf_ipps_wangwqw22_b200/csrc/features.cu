@@ -3,7 +3,8 @@
 //    starts of an exact run on the profile sample, per 8 segments (input
 //    sensitivity = max - min of per-segment spec-1 accuracy);
 //  * uniq10: #unique states after 10 transitions from all states, averaged
-//    over 64 evenly spaced positions (a lightweight convergence profile).
+//    over 64 evenly spaced positions (a lightweight convergence profile);
+//  * convergence lengths of the lookback image (reading R29) -> chunk size.
 #include "internal.h"
 #include "walk.cuh"
 
@@ -49,7 +50,41 @@ __global__ void k_feat_uniq(DevImage img, const uint32_t* __restrict__ ttc, cons
   if ((threadIdx.x & 31) == 0 && u) atomicAdd(uniq, (unsigned long long)u);
 }
 
+// Convergence length of the lookback image (reading R29): one warp per window w (start
+// p = 4096 j, j = 32 (w / 28) + 1 + w % 28, so a window stays inside one 128 KiB profile
+// portion); lane i walks the i-th ranked state of the window's lookback-2 image (lanes past
+// the image repeat state 0), and after every 64 bytes the warp votes whether every path is
+// in one state.  dout[w] = bytes to that point, 0 for a one-state image, ~0 past wmax.
+__global__ void k_feat_conv(DevImage img, const uint32_t* __restrict__ ttc, const uint8_t* __restrict__ in,
+                            uint32_t nwin, uint32_t wmax, uint32_t* __restrict__ dout) {
+  const uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (w >= nwin) return;
+  const uint64_t p = ((uint64_t)(w / 28) * 32 + 1 + w % 28) * 4096;
+  const uint32_t pair = (uint32_t)img.cls[in[p - 2]] * img.C + img.cls[in[p - 1]];
+  const uint32_t ql = min((uint32_t)img.qs2_len[pair], (uint32_t)kQsMax);
+  uint32_t d = 0;
+  if (ql > 1) {
+    uint32_t t = img.qs2[(uint64_t)pair * kQsMax + (lane < ql ? lane : 0)];
+    d = 0xFFFFFFFFu;
+    for (uint32_t i = 0; i < wmax; i += 64) {
+      for (uint32_t k = 0; k < 64; k++) t = ttc[(uint64_t)t * img.C + img.cls[in[p + i + k]]];
+      if (__all_sync(0xffffffffu, t == __shfl_sync(0xffffffffu, t, 0))) {
+        d = i + 64;
+        break;
+      }
+    }
+  }
+  if (lane == 0) dout[w] = d;
+}
+
 }  // namespace
+
+cudaError_t launch_feat_conv(const DevImage& img, const uint32_t* d_ttc, const uint8_t* in, uint32_t nwin,
+                             uint32_t wmax, uint32_t* d_out, cudaStream_t st) {
+  if (nwin == 0) return cudaSuccess;
+  k_feat_conv<<<(nwin + 3) / 4, 128, 0, st>>>(img, d_ttc, in, nwin, wmax, d_out);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_features_raw(const DevImage& img, const uint32_t* d_ttc, const uint8_t* in, uint64_t len,
                                 uint32_t B, uint64_t N, const uint32_t* d_x, uint32_t k, uint32_t qs_cap,

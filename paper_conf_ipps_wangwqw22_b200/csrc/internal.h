@@ -366,6 +366,8 @@ cudaError_t launch_qs_long(const DevImage& img, const uint32_t* d_ttc, const uin
 uint64_t pm_tree_scratch_bytes(uint64_t N, uint32_t k, uint32_t* levels);
 cudaError_t launch_pm_tree(const DevImage& img, const RunParams& rp, const RecStore& rs, uint32_t k, void* scratch,
                            Ctl* ctl, uint32_t* d_chunk_ends, int sms, cudaStream_t st, uint32_t* launches);
+cudaError_t launch_feat_conv(const DevImage& img, const uint32_t* d_ttc, const uint8_t* in, uint32_t nwin,
+                             uint32_t wmax, uint32_t* d_out, cudaStream_t st);
 cudaError_t launch_map_fused_publish(const uint32_t* cand, const uint32_t* ncand_p, const long long* dcnt,
                                      const uint32_t* fin_p, const unsigned long long* count_p, uint32_t* mend,
                                      unsigned long long* mcnt, const uint32_t* unmerged, uint64_t mapb,
@@ -479,6 +481,7 @@ struct fsm_s {
     unsigned long long seq;
   };
   const P2PPub* p2p_pub = nullptr;
+  uint32_t auto_chunk = 0;  // the selector's recommended chunk size (R29), 0 before a selection
   bool p2p_published = false;
   void* img2_base = nullptr;             // lookback > 2: full pair images (built at first use)
   uint32_t *img2_s = nullptr, *img2_m = nullptr;

@@ -780,9 +780,12 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
     // behind us, like SRE's dense rounds.  The per-chunk helper bookkeeping that E does
     // after its walks (VR^others counts, QS cursors) is committed here first; the task
     // kernel writes each helper record at its precomputed ring slot oth_base[c] + j.
-    if (helpers && rp.dense && rp.dense_slots > 0) {
+    if (helpers && rp.dense) {
       const uint64_t nslots = rp.lazy_helpers ? nA : nA + I;  // memoized helpers are not walked here
-      if (nslots >= 2048 && nslots * 16 >= N - f2) {
+      const bool dense_round = nslots >= 2048 && nslots * 16 >= N - f2;
+      // no task kernel left behind us: run it here (phase E) and tell the host to queue one next run
+      if (dense_round && rp.dense_slots == 0 && b == 0 && threadIdx.x == 0) vctl->dense_denied = 1;
+      if (dense_round && rp.dense_slots > 0) {
         if (rp.lazy_helpers) {  // the helpers' pending records (start only) + their counters
           const uint64_t T = (uint64_t)G * kBS, gt = (uint64_t)b * kBS + threadIdx.x;
           uint64_t hel = 0, reread = 0;

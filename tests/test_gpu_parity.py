@@ -276,7 +276,8 @@ def test_async_queue(gs):
     ("c3", 32 << 20, 4096, "sre", 16), ("c3", (24 << 20) + 1000, 4096, "sre", 16), ("c3s", 160 << 20, 8192, "sre", 16),
     ("c3", 32 << 20, 4096, "cse", 16), ("c3", 32 << 20, 4096, "rr", 16), ("c3", 32 << 20, 4096, "nf", 16),
     ("c3", (24 << 20) + 1000, 4096, "rr", 16), ("c3", (24 << 20) + 1000, 4096, "nf", 2),
-    ("c3s", 160 << 20, 8192, "nf", 16), ("c3", 16 << 20, 4096, "nf", 1)])
+    ("c3s", 160 << 20, 8192, "nf", 16), ("c3", 16 << 20, 4096, "nf", 1), ("c3", 48 << 20, 8192, "sre", 16),
+    ("c3", 48 << 20, 8192, "rr", 16), ("c3", (40 << 20) + 4100, 8192, "nf", 4)])
 def test_dense_recovery_rounds(gs, name, length, B, scheme, vr_oth):
     """SRE / RR / NF (and CSE's SRE rounds) on a low-accuracy DFA: rounds where many
     chunks re-execute go to the TMA-gather task kernel over the round's task list (RR /
@@ -295,8 +296,26 @@ def test_dense_recovery_rounds(gs, name, length, B, scheme, vr_oth):
                   "verify_matches"):
             assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
     assert res.stats["tasks_sre"] > 2048  # the dense path really ran
-    if scheme in ("rr", "nf"):
+    if scheme in ("rr", "nf") and B == 4096:
         assert res.stats["tasks_helper"] > 2048
+
+
+@pytest.mark.parametrize("scheme", ["sre", "rr", "nf"])
+def test_dense_slots_follow_previous_run(gs, scheme):
+    """Device-driven dense rounds: a run that needed a dense round but had no task-kernel
+    slot queued (the selector's 1 MiB profile run used none) runs it in-kernel and makes
+    the next run queue one — for RR / NF as for SRE."""
+    w, data = _wl("c3", 48 << 20)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    x = torch.from_numpy(data).cuda()
+    fsm.select_scheme(x[: 1 << 20])  # a small profile: no dense round there
+    r1 = fsm.run(x, scheme=scheme, chunk_bytes=8192)
+    r2 = fsm.run(x, scheme=scheme, chunk_bytes=8192)
+    assert r1.stats["kernel_launches"] == 2  # spec + verify (the dense round ran in-kernel)
+    assert r2.stats["kernel_launches"] >= 5  # + task kernel, finish, verify per queued slot
+    for k in ("rounds", "tasks_sre", "tasks_helper", "verify_matches"):
+        assert r1.stats[k] == r2.stats[k]
+    assert r1.final_state == r2.final_state and r1.accept_count == r2.accept_count
 
 
 @pytest.mark.parametrize("name,length,B", [("c1", 1 << 20, 4096), ("c2", 4 << 20, 16384), ("c3", 2 << 20, 8192),
@@ -550,8 +569,40 @@ def test_selector_spread_profile(gs, name):
         assert of["sens"] >= 0.2
     res = fsm.run(x[:64 << 20], scheme="auto")  # the cached choice
     assert res.scheme == pick
+    # R29: convergence fractions of the same spread sample equal the oracle's, and the
+    # chunk-size rule (1 GiB on this GPU's SMs) picks 8 KiB for C3 / C3s (one '#' per
+    # 8 KiB block: a wrong start re-converges within 8 KiB in >= 3/4 of the windows), 4 KiB for C2
+    d = oracle.conv_lengths(w.table, w.start, w.accept, sample, wmax=16384)
+    for W, key in ((4096, "conv4k"), (8192, "conv8k"), (16384, "conv16k")):
+        assert ft[key] == pytest.approx(float((d <= W).sum()) / d.size, abs=0)
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    assert ft["chunk_bytes"] == oracle.select_chunk(d, L, sms * 768)
+    assert ft["chunk_bytes"] == (4096 if name == "c2" else 8192)
     del x
     torch.cuda.empty_cache()
+
+
+@pytest.mark.parametrize("name,length", [("c1", 1 << 20), ("c2", 1 << 20), ("c3", 1 << 20), ("c4", 1 << 20),
+                                         ("rand:40:7:3", 600000), ("rand:300:4:1", 1 << 20), ("c3s", 900000)])
+def test_conv_fractions_match_oracle(gs, name, length):
+    """R29: the selector's convergence fractions (k_feat_conv, one warp per window) equal the
+    oracle's convergence lengths counted at 4 / 8 / 16 KiB on the same sample, and its chunk
+    recommendation equals the oracle's rule for the sample's own length and for a 1 GiB
+    and a 16 GiB stream (fsm_chunk_for)."""
+    w, data = _wl(name, length)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    _, ft = fsm.select_scheme(torch.from_numpy(data).cuda())
+    d = oracle.conv_lengths(w.table, w.start, w.accept, data, wmax=16384)
+    assert d.size > 0
+    for W, key in ((4096, "conv4k"), (8192, "conv8k"), (16384, "conv16k")):
+        assert ft[key] == pytest.approx(float((d <= W).sum()) / d.size, abs=0), key
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    assert ft["chunk_bytes"] == oracle.select_chunk(d, length, sms * 768) == 4096  # too short for larger chunks
+    for L in (1 << 30, 16 << 30):
+        _, f2 = fsm.select_scheme(torch.from_numpy(data).cuda(), stream_len=L)
+        assert f2["chunk_bytes"] == oracle.select_chunk(d, L, sms * 768)
+    if name == "c1":
+        assert ft["conv16k"] == 0.0  # div7 permutes its states: never converges
 
 
 @pytest.mark.parametrize("name,length,B", [("c2", 4 << 20, 4096), ("c3", 4 << 20, 4096), ("c4", 2 << 20, 4096),
