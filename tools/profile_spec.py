@@ -1,5 +1,5 @@
 """Run the bench workload's fsm_run a few times (for ncu captures).
-usage: python tools/profile_spec.py [config] [scheme] [reps]"""
+usage: python tools/profile_spec.py [config] [scheme] [reps] [chunk_bytes]"""
 import sys
 sys.path.insert(0, '.')
 import torch
@@ -14,9 +14,10 @@ w.device(x)
 prof = torch.empty(1 << 20, dtype=torch.uint8, device='cuda')
 w.device(prof, offset=w.length)  # disjoint training trace, as bench.py
 fsm = gs.FSM.load(w.table, w.start, w.accept, profile=prof.cpu().numpy())
-fsm.select_scheme(x)  # as bench.py (spread profile, R20): gates the dense-round slots and the fused round 0
+_, feats = fsm.select_scheme(x)  # as bench.py (spread profile, R20): dense-round slots, fused round 0
+B = int(sys.argv[4]) if len(sys.argv) > 4 else feats["chunk_bytes"]  # as bench.py: the R29 recommendation
 for i in range(reps):
-    r = fsm.run(x, scheme=scheme)
+    r = fsm.run(x, scheme=scheme, chunk_bytes=B)
 torch.cuda.synchronize()
 print(r.final_state, r.accept_count, r.stats['ms_spec'], r.stats['ms_verify'])
 print("verify phase times (us):", [round(v, 1) for v in fsm.phase_times()])
