@@ -1667,7 +1667,8 @@ int fsm_shard_finish(fsm_t f, const void* d_maps, uint32_t G, uint32_t rank, con
   const uint32_t nt = f->n + 1;
   if (!f->d_small) CUDA_TRY(cudaMalloc(&f->d_small, 64 * sizeof(uint32_t)));  // (a map that failed early)
   CUDA_TRY(launch_compose(reinterpret_cast<const uint8_t*>(d_maps), G, map_bytes_nt(nt), map_cnt_off(nt), f->img.q0t,
-                          rank, f->d_small, o.st));
+                          rank, f->d_small, o.st, f->p2p_wait ? f->p2p_wait->flags : nullptr,
+                          f->p2p_wait ? f->p2p_wait->seq : 0, f->p2p_wait ? f->p2p_wait->status : nullptr));
   if (f->shard_mode == 3) {
     // fused mode: this rank's chunk ends before the merge point are fixed on the device
     ShardScratch S3;

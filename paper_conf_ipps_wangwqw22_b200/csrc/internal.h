@@ -375,8 +375,6 @@ cudaError_t launch_map_fused_publish(const uint32_t* cand, const uint32_t* ncand
                                      unsigned long long seq, cudaStream_t st);
 cudaError_t launch_publish(const uint8_t* own_map, uint64_t mapb, uint8_t* const* peers, uint32_t G, uint32_t rank,
                            uint32_t set, unsigned long long seq, cudaStream_t st);
-cudaError_t launch_wait_flags(const uint8_t* own_box, uint64_t mapb, uint32_t G, uint32_t rank, uint32_t set,
-                              unsigned long long seq, uint32_t* status, cudaStream_t st);
 cudaError_t launch_map_error(uint32_t* mend, unsigned long long* mcnt, uint32_t nt, uint32_t code, cudaStream_t st);
 cudaError_t launch_set_u32(uint32_t* p, uint32_t v, uint32_t* p2, uint32_t v2, cudaStream_t st);
 cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_t* grp,
@@ -385,7 +383,9 @@ cudaError_t launch_map_write(const uint32_t* cand, uint32_t ncand, const uint32_
 cudaError_t launch_map_enum(const uint8_t* topM, const unsigned long long* topC, uint32_t nt, uint32_t* mend,
                             unsigned long long* mcnt, cudaStream_t st);
 cudaError_t launch_compose(const uint8_t* maps, uint32_t G, uint64_t map_bytes, uint64_t cnt_off, uint32_t q0t,
-                           uint32_t rank, uint32_t* out, cudaStream_t st);
+                           uint32_t rank, uint32_t* out, cudaStream_t st,
+                           const unsigned long long* wflags = nullptr, unsigned long long seq = 0,
+                           uint32_t* wstatus = nullptr);
 cudaError_t launch_fix_prefix(const uint32_t* states, uint32_t ncand, uint32_t ci, uint32_t nj, const uint32_t* inv,
                               uint32_t* chunk_ends, cudaStream_t st);
 
@@ -481,6 +481,14 @@ struct fsm_s {
     unsigned long long seq;
   };
   const P2PPub* p2p_pub = nullptr;
+  // set by fsm_run_sharded_p2p around its fsm_shard_finish call: the composition kernel first
+  // waits for the peers' arrival flags of this step (k_compose's wflags), no separate wait kernel
+  struct P2PWait {
+    const unsigned long long* flags;  // this step's G flags in the own mailbox
+    unsigned long long seq;
+    uint32_t* status;
+  };
+  const P2PWait* p2p_wait = nullptr;
   uint32_t auto_chunk = 0;  // the selector's recommended chunk size (R29), 0 before a selection
   bool p2p_published = false;
   void* img2_base = nullptr;             // lookback > 2: full pair images (built at first use)

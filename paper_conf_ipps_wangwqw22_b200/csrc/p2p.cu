@@ -7,9 +7,9 @@
 //      stores the finished map into slot [rank] of every peer's mailbox, fences
 //      system-wide and raises the flag [rank] there — the compute step and the exchange in
 //      one kernel, no NCCL launch; the other modes publish with k_publish (the same stores)
-//   -> k_wait_flags: spins (with nanosleep, bounded) until every peer's flag for this
-//      step has arrived in the own mailbox
-//   -> fsm_shard_finish over the own mailbox (compose, fix-up), as after an allgather.
+//   -> fsm_shard_finish over the own mailbox (compose, fix-up), as after an allgather; its
+//      composition kernel (k_compose, shard.cu) first spins (nanosleep, bounded) until every
+//      peer's flag for this step has arrived — the wait fused into the receiver's compose.
 // Steps alternate between the two sets, so a fast rank's next publish never overwrites
 // a map a slow peer is still composing.
 #include <cuda_runtime.h>
@@ -22,14 +22,6 @@
 
 namespace gspec {
 namespace {
-
-constexpr unsigned long long kSpinLimit = 20ull * 1000 * 1000 * 1000;  // ~10 s of %globaltimer ns
-
-__device__ __forceinline__ unsigned long long gtime() {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
 
 // one CTA: copy this rank's map (mapb bytes, 16-aligned) into slot [rank] of set `set` of
 // every peer's mailbox, then raise this rank's flag in each of them
@@ -51,28 +43,6 @@ __global__ void __launch_bounds__(1024) k_publish(const uint8_t* __restrict__ ow
   }
 }
 
-// one thread: wait until every peer's flag of this step (set, seq) has arrived here
-__global__ void k_wait_flags(const uint8_t* __restrict__ own_box, uint64_t mapb, uint32_t G, uint32_t rank,
-                             uint32_t set, unsigned long long seq, uint32_t* __restrict__ status) {
-  if (threadIdx.x || blockIdx.x) return;
-  const volatile unsigned long long* flags =
-      reinterpret_cast<const volatile unsigned long long*>(own_box + 2ull * G * mapb) + (uint64_t)set * G;
-  const unsigned long long t0 = gtime();
-  uint32_t st = 0;
-  for (uint32_t g = 0; g < G && !st; g++) {
-    if (g == rank) continue;
-    while (flags[g] != seq) {
-      __nanosleep(200);
-      if (gtime() - t0 > kSpinLimit) {
-        st = 1 + g;  // a peer never published this step
-        break;
-      }
-    }
-  }
-  __threadfence();
-  *status = st;
-}
-
 }  // namespace
 
 cudaError_t launch_publish(const uint8_t* own_map, uint64_t mapb, uint8_t* const* peers, uint32_t G, uint32_t rank,
@@ -81,11 +51,6 @@ cudaError_t launch_publish(const uint8_t* own_map, uint64_t mapb, uint8_t* const
   return cudaGetLastError();
 }
 
-cudaError_t launch_wait_flags(const uint8_t* own_box, uint64_t mapb, uint32_t G, uint32_t rank, uint32_t set,
-                              unsigned long long seq, uint32_t* status, cudaStream_t st) {
-  k_wait_flags<<<1, 32, 0, st>>>(own_box, mapb, G, rank, set, seq, status);
-  return cudaGetLastError();
-}
 
 }  // namespace gspec
 
@@ -184,11 +149,18 @@ int fsm_run_sharded_p2p(fsm_t f, fsm_p2p_t p, const uint8_t* d_shard, uint64_t s
     if (rc && f->shard_mode != 4) return rc;  // (a failed map publishes its error map like any other)
     const int map_rc = rc;
     const bool sent = f->p2p_published && !rc;
-    if ((!sent && gspec::launch_publish(own_slot, p->mapb, p->d_peers, G, rank, set, seq, st) != cudaSuccess) ||
-        gspec::launch_wait_flags(p->box, p->mapb, G, rank, set, seq, p->d_status, st) != cudaSuccess ||
-        cudaMemcpyAsync(p->h_status, p->d_status, 4, cudaMemcpyDeviceToHost, st) != cudaSuccess)
-      return gspec_set_error(FSM_ECUDA, "p2p publish / wait launch");
+    if (!sent && gspec::launch_publish(own_slot, p->mapb, p->d_peers, G, rank, set, seq, st) != cudaSuccess)
+      return gspec_set_error(FSM_ECUDA, "p2p publish launch");
+    // the receiver side: fsm_shard_finish's composition kernel waits for the peers' flags of
+    // this step before it reads a map (k_compose's wflags) — no separate wait kernel
+    const fsm_s::P2PWait wt{reinterpret_cast<const unsigned long long*>(p->box + 2ull * G * p->mapb) +
+                                (uint64_t)set * G,
+                            seq, p->d_status};
+    f->p2p_wait = &wt;
     rc = fsm_shard_finish(f, p->box + (uint64_t)set * G * p->mapb, G, rank, opts, d_chunk_ends_local, out_global);
+    f->p2p_wait = nullptr;
+    if (cudaMemcpyAsync(p->h_status, p->d_status, 4, cudaMemcpyDeviceToHost, st) != cudaSuccess)
+      return gspec_set_error(FSM_ECUDA, "p2p status readback");
     if (cudaStreamSynchronize(st) != cudaSuccess) return gspec_set_error(FSM_ECUDA, "p2p step");
     if (*p->h_status) return gspec_set_error(FSM_ENCCL, "p2p exchange: a peer never published its map");
     if (rc == FSM_EAGAIN) continue;  // every rank redoes the exact map

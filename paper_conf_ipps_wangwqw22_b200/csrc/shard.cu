@@ -268,10 +268,36 @@ __global__ void k_map_enum(const uint8_t* __restrict__ topM, const unsigned long
 // s_0 = q0; s_{h+1} = M_h[s_h]: out = {s_rank, final, err, count_lo, count_hi}.  With
 // `staged` the G maps are first copied into shared memory by the whole block (coalesced),
 // so the dependent chain of G lookups runs on shared memory instead of G L2 round trips.
+// wflags (P2P exchange, p2p.cu; nullptr otherwise): the receiver side of the peer-memory
+// exchange fused in — thread 0 first waits (nanosleep spin, bounded ~10 s) until every
+// peer's arrival flag of this step equals seq, reports 0 / 1 + the missing rank to
+// *wstatus, and only then is any map read (the maps arrive by the peers' remote stores).
 __global__ void k_compose(const uint8_t* __restrict__ maps_g, uint32_t G, uint64_t map_bytes, uint64_t cnt_off,
-                          uint32_t q0t, uint32_t rank, uint32_t* __restrict__ out, uint32_t staged) {
+                          uint32_t q0t, uint32_t rank, uint32_t* __restrict__ out, uint32_t staged,
+                          const unsigned long long* wflags, unsigned long long seq, uint32_t* wstatus) {
   extern __shared__ __align__(16) uint8_t sm_maps[];
   const uint8_t* maps = maps_g;
+  if (wflags) {
+    if (threadIdx.x == 0) {
+      uint64_t t0, t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+      uint32_t st = 0;
+      for (uint32_t g = 0; g < G && !st; g++) {
+        if (g == rank) continue;
+        while (*reinterpret_cast<const volatile unsigned long long*>(wflags + g) != seq) {
+          __nanosleep(200);
+          asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+          if (t - t0 > 20ull * 1000 * 1000 * 1000) {
+            st = 1 + g;  // a peer never published this step
+            break;
+          }
+        }
+      }
+      __threadfence();
+      *wstatus = st;
+    }
+    __syncthreads();
+  }
   if (staged) {
     const uint64_t words = G * map_bytes / 4;
     for (uint64_t i = threadIdx.x; i < words; i += blockDim.x)
@@ -286,18 +312,18 @@ __global__ void k_compose(const uint8_t* __restrict__ maps_g, uint32_t G, uint64
     if (h == rank) srank = s;
     const uint32_t* me = reinterpret_cast<const uint32_t*>(maps + h * map_bytes);
     const unsigned long long* mc = reinterpret_cast<const unsigned long long*>(maps + h * map_bytes + cnt_off);
-    const uint32_t e = me[s];
+    const uint32_t e = staged ? me[s] : __ldcg(me + s);
     if (e == kErrorMap) {  // rank h's fsm_shard_map failed: report its status and rank
       out[0] = q0t;
       out[1] = q0t;
       out[2] = 3;
-      out[3] = (uint32_t)mc[0];
+      out[3] = (uint32_t)(staged ? mc[0] : __ldcg(mc));
       out[4] = h;
       return;
     }
     if (e == kNoState) { err = 1; break; }
     if (e == kInvalidMap) { err = 2; break; }  // a rank's speculative map must be redone
-    c += mc[s];
+    c += staged ? mc[s] : __ldcg(mc + s);
     s = e;
   }
   out[0] = srank;
@@ -419,14 +445,15 @@ cudaError_t launch_map_enum(const uint8_t* topM, const unsigned long long* topC,
 }
 
 cudaError_t launch_compose(const uint8_t* maps, uint32_t G, uint64_t map_bytes, uint64_t cnt_off, uint32_t q0t,
-                           uint32_t rank, uint32_t* out, cudaStream_t st) {
+                           uint32_t rank, uint32_t* out, cudaStream_t st, const unsigned long long* wflags,
+                           unsigned long long seq, uint32_t* wstatus) {
   const uint64_t bytes = (uint64_t)G * map_bytes;
   uint32_t staged = bytes <= 96 * 1024 && map_bytes % 8 == 0;
   if (staged && kernel_setup((const void*)k_compose, (uint32_t)bytes, 256, nullptr) != cudaSuccess) staged = 0;
   if (staged)
-    k_compose<<<1, 256, (uint32_t)bytes, st>>>(maps, G, map_bytes, cnt_off, q0t, rank, out, 1u);
+    k_compose<<<1, 256, (uint32_t)bytes, st>>>(maps, G, map_bytes, cnt_off, q0t, rank, out, 1u, wflags, seq, wstatus);
   else
-    k_compose<<<1, 32, 0, st>>>(maps, G, map_bytes, cnt_off, q0t, rank, out, 0u);
+    k_compose<<<1, 32, 0, st>>>(maps, G, map_bytes, cnt_off, q0t, rank, out, 0u, wflags, seq, wstatus);
   return cudaGetLastError();
 }
 
