@@ -462,14 +462,22 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         torch.cuda.synchronize()
         stream = torch.cuda.current_stream()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        pend = []
         with ClockSampler(dev) as clk:
             ev0.record(stream)
             if comm is not None and p2p is None:  # steps queued back to back: no host wait between them
                 res = async_sharded_steps(gs, comm, fsm, x, lb, scheme, B, ce, args.steps)
+            elif dist is None:  # one GPU: fsm_run_async queue (no host wait between steps either)
+                for _ in range(args.steps):
+                    if len(pend) >= 16:
+                        res = fsm.wait(pend.pop(0))
+                    pend.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce))
             else:
                 for _ in range(args.steps):
                     res = step()
             ev1.record(stream)
+            for t in pend:
+                res = fsm.wait(t)
             torch.cuda.synchronize()
         if p2p is not None:
             p2p.close()
@@ -642,6 +650,7 @@ def main():
         torch.cuda.synchronize()
         stream = torch.cuda.current_stream()
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        pend = []
         with ClockSampler(dev) as clk:
             ev0.record(stream)
             if comm is not None and p2p is None:  # steps queued back to back: no host wait between them
