@@ -158,6 +158,43 @@ def test_invalid_symbol_is_loud(gs):
         assert e.value.status == gs.FSM_ESYMBOL
 
 
+@pytest.mark.parametrize("name,length,B", [("c1", (16 << 20) + 5, 4096), ("rand:40:3:2", (12 << 20) + 333, 4096),
+                                           ("rand:60:4:7", 10 << 20, 2048), ("rand:9:2:4", (6 << 20) + 17, 1024),
+                                           ("c1", 3 << 20, 4096)])
+def test_enum_four_symbol_table(gs, name, length, B):
+    """ENUM on small alphabets walks 16-byte vectors four symbols per lookup (T4, DESIGN.md
+    §5.3); the unaligned tail and vectors holding a byte >= 4 take the one-symbol step.
+    Bit-exact against the oracle, with T4 on and off (GSPEC_T4=0)."""
+    import os
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    x = torch.from_numpy(data).cuda()
+    for flag in ("1", "0"):
+        os.environ["GSPEC_T4"] = flag
+        try:
+            res = fsm.run(x, scheme="enum", chunk_bytes=B)
+        finally:
+            os.environ.pop("GSPEC_T4", None)
+        check_equal(res, ref, B, w.nstates)
+
+
+@pytest.mark.parametrize("bad", [3, 9, 255])
+def test_enum_four_symbol_table_invalid(gs, bad):
+    """A byte >= nsyms inside a T4 vector: a value < 4 goes to poison through T4 itself, a
+    larger one through the one-symbol fallback — FSM_ESYMBOL either way, and a stream whose
+    invalid byte sits in the unaligned tail too."""
+    t, s, a = gen.dfa_div7()
+    fsm = gs.FSM.load(t, s, a)
+    rng = np.random.default_rng(bad)
+    for pos in (5 << 20, (8 << 20) - 3):
+        data = rng.integers(0, 2, 8 << 20).astype(np.uint8)
+        data[pos] = bad
+        with pytest.raises(gs.GSpecError) as e:
+            fsm.run(torch.from_numpy(data).cuda(), scheme="enum", chunk_bytes=4096)
+        assert e.value.status == gs.FSM_ESYMBOL
+
+
 @pytest.mark.parametrize("policy", [0, 1])
 def test_policies_and_transform(gs, policy):
     w, data = _wl("c3", 1 << 20)
