@@ -832,25 +832,28 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
   const uint32_t* d_ttc = nullptr;
   if ((rc = upload(f, &d_ttc, ttc))) return bail(rc);
   f->d_ttc = d_ttc;
-  // 4-symbol step table for the enumerative walk on small alphabets: the
-  // transformation P:319-330 applied to strings of 4 symbols — entry (tid, combo) is the tid
-  // after the 4 symbols (a value >= nsyms -> poison) and how many of the 4 states accept
-  img.T4 = nullptr;
-  img.t4_bytes = 0;
+  // multi-symbol step table for the enumerative walk on small alphabets: the
+  // transformation P:319-330 applied to strings of K symbols — entry (tid, combo) is the tid
+  // after the K symbols (a value >= nsyms -> poison) and how many of the K states accept
+  img.TK = nullptr;
+  img.tk_bytes = 0;
+  img.tk_syms = 0;
   if (mode == MODE_U8 && nsyms <= 4 && nt <= 64) {
-    std::vector<uint32_t> t4((uint64_t)nt * 256);
+    const uint32_t K = nsyms <= 2 ? 8 : 4, bits = 8 / K, row = 257;  // words per row (kTkRow)
+    std::vector<uint32_t> tk(((uint64_t)nt * row + 3) & ~3ull, 0);  // staged in 16-byte pieces
     for (uint32_t t = 0; t < nt; t++)
       for (uint32_t cb = 0; cb < 256; cb++) {
         uint32_t x = t, k = 0;
-        for (uint32_t i = 0; i < 4; i++) {
-          const uint32_t sym = (cb >> (2 * i)) & 3u;
+        for (uint32_t i = 0; i < K; i++) {
+          const uint32_t sym = (cb >> (bits * i)) & ((1u << bits) - 1u);
           x = (x == P || sym >= nsyms) ? P : ttc[(uint64_t)x * C + f->cls[sym]];
           k += acc_t[x];
         }
-        t4[(uint64_t)t * 256 + cb] = x << 10 | k << 24;
+        tk[(uint64_t)t * row + cb] = x * row * 4 | k << 24;
       }
-    if ((rc = upload(f, &img.T4, t4))) return bail(rc);
-    img.t4_bytes = nt * 1024;
+    if ((rc = upload(f, &img.TK, tk))) return bail(rc);
+    img.tk_bytes = (uint32_t)tk.size() * 4;
+    img.tk_syms = K;
   }
 
   // ---- 4. lookback pair table on the device ----

@@ -18,26 +18,9 @@ namespace {
 
 constexpr uint32_t kGroup = 64;
 
-__host__ __device__ inline uint32_t t4_off(const DevImage& img) { return (smem_bytes_for(img) + 15u) & ~15u; }
-
-// One 4-symbol step of every chain through T4: w = 4 input bytes, each < 4;
-// combo = their 2-bit values packed by one multiply (b0 + 4 b1 + 16 b2 + 64 b3 lands in bits
-// 24-31 with no carries from the other partial products); a chain's code is its T4 row's byte
-// offset (tid << 10), the entry's top byte counts the accepting states among the 4.
-template <int NE>
-__device__ __forceinline__ void t4_step(uint32_t t4base, uint32_t w, uint32_t (&sc)[NE], uint32_t (&acc)[NE]) {
-  const uint32_t cb = t4base + (((w * 0x01041040u) >> 24) << 2);
-#pragma unroll
-  for (int q = 0; q < NE; q++) {
-    const uint32_t e = lds_u32(cb + sc[q]);
-    sc[q] = e & 0xFFFFFFu;
-    acc[q] += e >> 24;
-  }
-}
-
 // K1: thread per sub-chunk, NE independent chains (ILP = NE).  SUPER: the 16-byte vectors
-// whose bytes are all < 4 advance through T4 four symbols per lookup; any other byte (and
-// the unaligned head / the tail) takes the one-symbol step of the transformed table.
+// whose bytes are all symbols TK covers advance K symbols per lookup (walk.cuh); any other
+// byte (and the unaligned head / the tail) takes the one-symbol step of the transformed table.
 template <int MODE, int NE, int W, bool SUPER = false>
 __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* __restrict__ in, uint64_t len,
                                                   uint32_t E, uint64_t nsub, uint8_t* __restrict__ M,
@@ -46,25 +29,26 @@ __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* 
   if (ctl_init && blockIdx.x == 0) init_ctl(ctl_init, q0t, N);  // the run's control block (no H2D copy)
   stage_table(img, smem);
   if (SUPER) {
-    const uint4* src = reinterpret_cast<const uint4*>(img.T4);
-    uint4* dst = reinterpret_cast<uint4*>(smem + t4_off(img));
-    for (uint32_t i = threadIdx.x; i < img.t4_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
+    const uint4* src = reinterpret_cast<const uint4*>(img.TK);
+    uint4* dst = reinterpret_cast<uint4*>(smem + tk_off(img));
+    for (uint32_t i = threadIdx.x; i < img.tk_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
   }
   __syncthreads();
   using S = Step<MODE>;
   const uint32_t nt = img.n + 1;
-  const uint32_t t4base = static_cast<uint32_t>(__cvta_generic_to_shared(smem)) + t4_off(img);
+  const uint32_t tkbase = static_cast<uint32_t>(__cvta_generic_to_shared(smem)) + tk_off(img);
+  const uint32_t K = img.tk_syms;
   for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < nsub; j += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t code[NE], acc[NE];
 #pragma unroll
     for (int q = 0; q < NE; q++) {
-      code[q] = SUPER ? ((uint32_t)q < nt ? q : 0) << 10 : __ldg(img.tid2code + ((uint32_t)q < nt ? q : 0));
+      code[q] = SUPER ? ((uint32_t)q < nt ? q : 0) * kTkRow : __ldg(img.tid2code + ((uint32_t)q < nt ? q : 0));
       acc[q] = 0;
     }
     const uint64_t lo = j * E, n = min((uint64_t)E, len - lo);
     const uint8_t* p = in + lo;
     uint64_t i = 0;
-    if (SUPER) {  // codes are T4 row offsets here; back to table codes for the byte steps below
+    if (SUPER) {  // codes are TK row offsets here; back to table codes for the byte steps below
       if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
         const uint4* v = reinterpret_cast<const uint4*>(p);
         const uint64_t nv = n / 16;
@@ -85,14 +69,11 @@ __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* 
           const uint64_t t16 = g0 + k;
           if (t16 >= nv) break;
           const uint4 qv = cur[k];
-          if (((qv.x | qv.y | qv.z | qv.w) & 0xFCFCFCFCu) == 0) {
-            t4_step<NE>(t4base, qv.x, code, acc);
-            t4_step<NE>(t4base, qv.y, code, acc);
-            t4_step<NE>(t4base, qv.z, code, acc);
-            t4_step<NE>(t4base, qv.w, code, acc);
-          } else {  // a byte >= 4 (an invalid symbol): these 16 bytes one by one
+          if (tk_vector_ok(qv, K)) {
+            tk_vector<NE>(tkbase, K, qv, code, acc);
+          } else {  // a byte TK does not cover (an invalid symbol): these 16 bytes one by one
 #pragma unroll
-            for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + (code[q] >> 10));
+            for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + code[q] / kTkRow);
             const uint8_t* b16 = reinterpret_cast<const uint8_t*>(v + t16);
             for (int k = 0; k < 16; k++) {
               const uint32_t bb = __ldg(b16 + k);
@@ -100,14 +81,14 @@ __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* 
               for (int q = 0; q < NE; q++) { code[q] = S::byte(img, smem, code[q], bb); acc[q] += S::acc(code[q]); }
             }
 #pragma unroll
-            for (int q = 0; q < NE; q++) code[q] = S::tid(img, code[q]) << 10;
+            for (int q = 0; q < NE; q++) code[q] = S::tid(img, code[q]) * kTkRow;
           }
           }
         }
         i = (n / 16) * 16;
       }
 #pragma unroll
-      for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + (code[q] >> 10));
+      for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + code[q] / kTkRow);
     } else if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
       const uint4* v = reinterpret_cast<const uint4*>(p);
       for (uint64_t t16 = 0; t16 < n / 16; t16++) {
@@ -261,7 +242,7 @@ template <int MODE, int NE, int W, bool SUPER = false>
 cudaError_t walk_t(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, uint8_t* M, uint64_t* Cn,
                    cudaStream_t st, int sms) {
   auto kern = k_enum_walk<MODE, NE, W, SUPER>;
-  const uint32_t smem = SUPER ? t4_off(img) + img.t4_bytes : smem_bytes_for(img);
+  const uint32_t smem = SUPER ? tk_off(img) + img.tk_bytes : smem_bytes_for(img);
   cudaError_t e = kernel_setup((const void*)kern, smem, 128, nullptr);
   if (e != cudaSuccess) return e;
   uint64_t grid = (nsub + 127) / 128;
@@ -275,7 +256,7 @@ template <int MODE>
 cudaError_t walk_m(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, uint8_t* M, uint64_t* Cn,
                    cudaStream_t st, int sms) {
   const uint32_t nt = img.n + 1;
-  if (MODE == MODE_U8 && img.T4 && !t4_disabled()) {  // small alphabet: 4 symbols per lookup
+  if (MODE == MODE_U8 && img.TK && !tk_disabled()) {  // small alphabet: K symbols per lookup
     if (nt <= 8) return walk_t<MODE, 8, 32, true>(img, rp, E, nsub, M, Cn, st, sms);
     if (nt <= 16) return walk_t<MODE, 16, 32, true>(img, rp, E, nsub, M, Cn, st, sms);
     if (nt <= 32) return walk_t<MODE, 32, 32, true>(img, rp, E, nsub, M, Cn, st, sms);

@@ -47,12 +47,12 @@ struct DevImage {
   uint32_t H;       // hot rows in smem (MODE_U16/U32); all rows for MODE_U8
   uint32_t q0t;     // transformed start state
   uint32_t smem_table_bytes;  // bytes of the smem copy of the table
-  // ENUM on small alphabets (nsyms <= 4, nt <= 64, MODE_U8): 4-symbol step table
-  // T4[tid][combo] (combo = the 4 symbols' 2-bit values, first symbol in bits 0-1) =
-  // (tid after the 4 symbols) << 10 | (accepting states among the 4) << 24; staged after
-  // the table; nullptr when not built.  DESIGN.md §5.3.
-  const uint32_t* T4;
-  uint32_t t4_bytes;
+  // ENUM on small alphabets (nsyms <= 4, nt <= 64, MODE_U8): multi-symbol step table
+  // TK[tid][combo] (walk.cuh; K = 8 symbols for nsyms <= 2, else 4) staged after the
+  // table; nullptr when not built.  DESIGN.md §5.3.
+  const uint32_t* TK;
+  uint32_t tk_bytes;
+  uint32_t tk_syms;  // K
   const uint8_t* T8;          // MODE_U8: [256 codes][256 bytes] next code
   const uint16_t* T16;        // MODE_U16: [nt][C]
   const uint32_t* T32;        // MODE_U32: [nt][C]
@@ -294,9 +294,9 @@ inline cudaError_t kernel_setup(const void* kern, uint32_t smem, int block, int*
   return cudaSuccess;
 }
 
-// GSPEC_T4=0: the enumerative walk ignores the 4-symbol table (A/B; tests compare both)
-inline bool t4_disabled() {
-  const char* e = getenv("GSPEC_T4");
+// GSPEC_TK=0: the enumerative walk ignores the multi-symbol table (A/B; tests compare both)
+inline bool tk_disabled() {
+  const char* e = getenv("GSPEC_TK");
   return e && e[0] == '0';
 }
 

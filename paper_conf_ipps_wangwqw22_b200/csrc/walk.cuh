@@ -207,6 +207,57 @@ struct Step<MODE_U16H> : StepPM {};
 template <>
 struct Step<MODE_U32> : StepClassed<uint32_t, 31, false> {};
 
+// Multi-symbol step table for the enumerative walk on small alphabets:
+// TK[tid][combo] advances K symbols per lookup — K = 8 one-bit symbols (nsyms <= 2) or K = 4
+// two-bit symbols (nsyms <= 4); combo packs the K symbols, the first in the lowest bits.
+// Rows are 257 words (kTkRow bytes) so row r starts at bank r: lanes in different states that
+// read the same combo hit different banks.  A chain's code is its row's byte offset
+// (tid * kTkRow); an entry = next code | (accepting states among the K) << 24.
+constexpr uint32_t kTkRow = 257 * 4;
+__host__ __device__ inline uint32_t tk_off(const DevImage& img) { return (smem_bytes_for(img) + 15u) & ~15u; }
+
+// combo of 8 one-bit symbols (bytes 0/1) in w0, w1: one multiply per word gathers its 4
+// bytes' low bits into bits 24-27 (the other partial products occupy single bits below 24:
+// no carries), the second word's land in bits 28-31 and are shifted to 4-7
+__device__ __forceinline__ uint32_t tk_pack8(uint32_t w0, uint32_t w1) {
+  return ((w0 * 0x01020408u) >> 24) | ((w1 * 0x01020408u) >> 20);
+}
+// combo of 4 two-bit symbols (bytes < 4): b0 + 4 b1 + 16 b2 + 64 b3 in bits 24-31, same argument
+__device__ __forceinline__ uint32_t tk_pack4(uint32_t w) { return (w * 0x01041040u) >> 24; }
+
+// every byte of the vector is a symbol the table covers (< 2 for K = 8, < 4 for K = 4)
+__device__ __forceinline__ bool tk_vector_ok(const uint4& q, uint32_t K) {
+  return ((q.x | q.y | q.z | q.w) & (K == 8 ? 0xFEFEFEFEu : 0xFCFCFCFCu)) == 0;
+}
+
+template <int NE>
+__device__ __forceinline__ void tk_lookup(uint32_t tkbase, uint32_t combo, uint32_t (&sc)[NE], uint32_t (&acc)[NE],
+                                          int np) {
+  const uint32_t cb = tkbase + (combo << 2);
+#pragma unroll
+  for (int q = 0; q < NE; q++) {
+    if (q >= np) break;
+    const uint32_t e = lds_u32(cb + sc[q]);
+    sc[q] = e & 0xFFFFFFu;
+    acc[q] += e >> 24;
+  }
+}
+
+// the first np chains over one 16-byte vector (tk_vector_ok) through TK
+template <int NE>
+__device__ __forceinline__ void tk_vector(uint32_t tkbase, uint32_t K, const uint4& q, uint32_t (&sc)[NE],
+                                          uint32_t (&acc)[NE], int np = NE) {
+  if (K == 8) {
+    tk_lookup<NE>(tkbase, tk_pack8(q.x, q.y), sc, acc, np);
+    tk_lookup<NE>(tkbase, tk_pack8(q.z, q.w), sc, acc, np);
+  } else {
+    tk_lookup<NE>(tkbase, tk_pack4(q.x), sc, acc, np);
+    tk_lookup<NE>(tkbase, tk_pack4(q.y), sc, acc, np);
+    tk_lookup<NE>(tkbase, tk_pack4(q.z), sc, acc, np);
+    tk_lookup<NE>(tkbase, tk_pack4(q.w), sc, acc, np);
+  }
+}
+
 // Walk one path over [p, p+n) bytes from `code`; returns end code, adds accepts.
 template <int MODE>
 __device__ __forceinline__ uint32_t walk_bytes(const DevImage& img, const uint8_t* s, const uint8_t* p, uint64_t n,

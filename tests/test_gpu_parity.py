@@ -160,35 +160,40 @@ def test_invalid_symbol_is_loud(gs):
 
 @pytest.mark.parametrize("name,length,B", [("c1", (16 << 20) + 5, 4096), ("rand:40:3:2", (12 << 20) + 333, 4096),
                                            ("rand:60:4:7", 10 << 20, 2048), ("rand:9:2:4", (6 << 20) + 17, 1024),
-                                           ("c1", 3 << 20, 4096)])
+                                           ("c1", 3 << 20, 4096), ("rand:12:3:5", (9 << 20) + 64, 4096),
+                                           ("rand:14:30:2", (8 << 20) + 1000, 4096), ("rand:5:4:3", 5 << 20, 512)])
 def test_enum_four_symbol_table(gs, name, length, B):
-    """ENUM on small alphabets walks 16-byte vectors four symbols per lookup (T4, DESIGN.md
-    §5.3); the unaligned tail and vectors holding a byte >= 4 take the one-symbol step.
-    Bit-exact against the oracle, with T4 on and off (GSPEC_T4=0)."""
+    """ENUM on small alphabets walks 16-byte vectors K symbols per lookup (TK: K = 8 for
+    nsyms <= 2, 4 for nsyms <= 4); the unaligned tail and vectors holding a
+    byte TK does not cover take the one-symbol step.  Bit-exact against the oracle with TK on
+    and off (GSPEC_TK=0), for nt from 6 to 61 (rows padded to 257 words, staged in 16-byte
+    pieces) and a 30-symbol DFA that has no TK."""
     import os
     w, data = _wl(name, length)
     ref = oracle.run(w.table, w.start, w.accept, data, B)
     fsm = gs.FSM.load(w.table, w.start, w.accept)
     x = torch.from_numpy(data).cuda()
     for flag in ("1", "0"):
-        os.environ["GSPEC_T4"] = flag
+        os.environ["GSPEC_TK"] = flag
         try:
             res = fsm.run(x, scheme="enum", chunk_bytes=B)
         finally:
-            os.environ.pop("GSPEC_T4", None)
+            os.environ.pop("GSPEC_TK", None)
         check_equal(res, ref, B, w.nstates)
 
 
-@pytest.mark.parametrize("bad", [3, 9, 255])
-def test_enum_four_symbol_table_invalid(gs, bad):
-    """A byte >= nsyms inside a T4 vector: a value < 4 goes to poison through T4 itself, a
-    larger one through the one-symbol fallback — FSM_ESYMBOL either way, and a stream whose
-    invalid byte sits in the unaligned tail too."""
-    t, s, a = gen.dfa_div7()
-    fsm = gs.FSM.load(t, s, a)
+@pytest.mark.parametrize("name,nsyms,bad", [("c1", 2, 3), ("c1", 2, 9), ("c1", 2, 255), ("rand:20:3:6", 3, 3),
+                                            ("rand:20:3:6", 3, 200)])
+def test_enum_four_symbol_table_invalid(gs, name, nsyms, bad):
+    """An invalid byte (>= nsyms) inside a TK vector: div7 (K = 8, one-bit symbols) sends any
+    such byte through the one-symbol fallback; a 3-symbol DFA (K = 4, two-bit symbols) steps
+    the value 3 to the poison state through TK itself and larger values through the fallback
+    — FSM_ESYMBOL either way, also when the byte sits in the unaligned tail."""
+    w, _ = _wl(name, 1 << 16)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
     rng = np.random.default_rng(bad)
     for pos in (5 << 20, (8 << 20) - 3):
-        data = rng.integers(0, 2, 8 << 20).astype(np.uint8)
+        data = rng.integers(0, nsyms, 8 << 20).astype(np.uint8)
         data[pos] = bad
         with pytest.raises(gs.GSpecError) as e:
             fsm.run(torch.from_numpy(data).cuda(), scheme="enum", chunk_bytes=4096)
