@@ -272,12 +272,23 @@ def measure_single(gs, w, x, args, fsm, scheme, B, with_clocks=True):
     kw = {"spec_k": args.spec_k, "lookback": args.lookback}
     kr = [fsm.run(x, scheme=scheme, chunk_bytes=B, **kw) for _ in range(3)]
     verify_phases = [round(float(v), 1) for v in fsm.phase_times()]
+    # at most WINDOW runs in flight (the handle's ring holds 32): waiting for the oldest while
+    # the GPU works on the others never leaves it idle
+    WINDOW = 16
+    done = []
+
+    def enqueue(pend):
+        if len(pend) >= WINDOW:
+            done.append(fsm.wait(pend.pop(0)))
+        pend.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce, **kw))
+
     pending = []
     for _ in range(max(3, args.warmup)):
-        pending.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce, **kw))
+        enqueue(pending)
     for t in pending:
         fsm.wait(t)
     pending.clear()
+    done.clear()
     torch.cuda.synchronize()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     clk = ClockSampler(torch.cuda.current_device()) if with_clocks else None
@@ -285,14 +296,13 @@ def measure_single(gs, w, x, args, fsm, scheme, B, with_clocks=True):
         clk.__enter__()
     ev0.record(stream)
     for _ in range(args.steps):
-        pending.append(fsm.run_async(x, scheme=scheme, chunk_bytes=B, chunk_ends=ce, **kw))
+        enqueue(pending)
     ev1.record(stream)
     torch.cuda.synchronize()
     if clk:
         clk.__exit__()
     spec_ms, ver_ms, launches = [], [], 0
-    for t in pending:
-        res = fsm.wait(t)
+    for res in done + [fsm.wait(t) for t in pending]:
         spec_ms.append(res.stats["ms_spec"])
         ver_ms.append(res.stats["ms_verify"])
         launches += res.stats["kernel_launches"]  # counted by the library per run

@@ -18,6 +18,58 @@ namespace {
 
 constexpr uint32_t kGroup = 64;
 
+// The 16-byte-aligned vectors of [p, p+n) through TK, NE chains: codes are TK
+// row offsets (tid * kTkRow) on entry; a vector holding a byte TK does not cover goes one
+// symbol at a time through the transformed table.  On return the codes are table codes again
+// and the result is the number of bytes consumed (0 when p is not 16-byte aligned).
+template <int MODE, int NE>
+__device__ __forceinline__ uint64_t tk_walk(const DevImage& img, const uint8_t* smem, uint32_t tkbase, uint32_t K,
+                                            const uint8_t* p, uint64_t n, uint32_t (&code)[NE], uint32_t (&acc)[NE]) {
+  using S = Step<MODE>;
+  uint64_t i = 0;
+  if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
+    const uint4* v = reinterpret_cast<const uint4*>(p);
+    const uint64_t nv = n / 16;
+    // the lookups are cheap now: keep PF 16-byte loads in flight ahead of them
+    constexpr int PF = NE <= 16 ? 4 : 1;
+    uint4 buf[PF];
+#pragma unroll
+    for (int k = 0; k < PF; k++) buf[k] = (uint64_t)k < nv ? __ldg(v + k) : make_uint4(0, 0, 0, 0);
+    for (uint64_t g0 = 0; g0 < nv; g0 += PF) {
+      uint4 cur[PF];
+#pragma unroll
+      for (int k = 0; k < PF; k++) {
+        cur[k] = buf[k];
+        buf[k] = g0 + PF + k < nv ? __ldg(v + g0 + PF + k) : make_uint4(0, 0, 0, 0);
+      }
+#pragma unroll
+      for (int k = 0; k < PF; k++) {
+        const uint64_t t16 = g0 + k;
+        if (t16 >= nv) break;
+        const uint4 qv = cur[k];
+        if (tk_vector_ok(qv, K)) {
+          tk_vector<NE>(tkbase, K, qv, code, acc);
+        } else {  // a byte TK does not cover (an invalid symbol): these 16 bytes one by one
+#pragma unroll
+          for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + code[q] / kTkRow);
+          const uint8_t* b16 = reinterpret_cast<const uint8_t*>(v + t16);
+          for (int b = 0; b < 16; b++) {
+            const uint32_t bb = __ldg(b16 + b);
+#pragma unroll
+            for (int q = 0; q < NE; q++) { code[q] = S::byte(img, smem, code[q], bb); acc[q] += S::acc(code[q]); }
+          }
+#pragma unroll
+          for (int q = 0; q < NE; q++) code[q] = S::tid(img, code[q]) * kTkRow;
+        }
+      }
+    }
+    i = nv * 16;
+  }
+#pragma unroll
+  for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + code[q] / kTkRow);
+  return i;
+}
+
 // K1: thread per sub-chunk, NE independent chains (ILP = NE).  SUPER: the 16-byte vectors
 // whose bytes are all symbols TK covers advance K symbols per lookup (walk.cuh); any other
 // byte (and the unaligned head / the tail) takes the one-symbol step of the transformed table.
@@ -48,47 +100,8 @@ __global__ void __launch_bounds__(128) k_enum_walk(DevImage img, const uint8_t* 
     const uint64_t lo = j * E, n = min((uint64_t)E, len - lo);
     const uint8_t* p = in + lo;
     uint64_t i = 0;
-    if (SUPER) {  // codes are TK row offsets here; back to table codes for the byte steps below
-      if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
-        const uint4* v = reinterpret_cast<const uint4*>(p);
-        const uint64_t nv = n / 16;
-        // the lookups are cheap now: keep PF 16-byte loads in flight ahead of them
-        constexpr int PF = NE <= 16 ? 4 : 1;
-        uint4 buf[PF];
-#pragma unroll
-        for (int k = 0; k < PF; k++) buf[k] = (uint64_t)k < nv ? __ldg(v + k) : make_uint4(0, 0, 0, 0);
-        for (uint64_t g0 = 0; g0 < nv; g0 += PF) {
-          uint4 cur[PF];
-#pragma unroll
-          for (int k = 0; k < PF; k++) {
-            cur[k] = buf[k];
-            buf[k] = g0 + PF + k < nv ? __ldg(v + g0 + PF + k) : make_uint4(0, 0, 0, 0);
-          }
-#pragma unroll
-          for (int k = 0; k < PF; k++) {
-          const uint64_t t16 = g0 + k;
-          if (t16 >= nv) break;
-          const uint4 qv = cur[k];
-          if (tk_vector_ok(qv, K)) {
-            tk_vector<NE>(tkbase, K, qv, code, acc);
-          } else {  // a byte TK does not cover (an invalid symbol): these 16 bytes one by one
-#pragma unroll
-            for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + code[q] / kTkRow);
-            const uint8_t* b16 = reinterpret_cast<const uint8_t*>(v + t16);
-            for (int k = 0; k < 16; k++) {
-              const uint32_t bb = __ldg(b16 + k);
-#pragma unroll
-              for (int q = 0; q < NE; q++) { code[q] = S::byte(img, smem, code[q], bb); acc[q] += S::acc(code[q]); }
-            }
-#pragma unroll
-            for (int q = 0; q < NE; q++) code[q] = S::tid(img, code[q]) * kTkRow;
-          }
-          }
-        }
-        i = (n / 16) * 16;
-      }
-#pragma unroll
-      for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + code[q] / kTkRow);
+    if (SUPER) {  // codes are TK row offsets until tk_walk returns
+      i = tk_walk<MODE, NE>(img, smem, tkbase, K, p, n, code, acc);
     } else if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
       const uint4* v = reinterpret_cast<const uint4*>(p);
       for (uint64_t t16 = 0; t16 < n / 16; t16++) {
@@ -277,7 +290,7 @@ cudaError_t walk_m(const DevImage& img, const RunParams& rp, uint32_t E, uint64_
 constexpr int kSmallT = 128;
 constexpr int kSmallCTAs = 64;
 
-template <int MODE, int NE>
+template <int MODE, int NE, bool SUPER = false>
 __global__ void __launch_bounds__(kSmallT) k_enum_small(DevImage img, RunParams rp, uint32_t E, uint64_t nsub,
                                                        uint8_t* __restrict__ P, uint64_t* __restrict__ PC,
                                                        uint8_t* __restrict__ AM, uint64_t* __restrict__ AC,
@@ -290,6 +303,11 @@ __global__ void __launch_bounds__(kSmallT) k_enum_small(DevImage img, RunParams 
   __shared__ uint32_t last;
   if (rp.ctl_init && blockIdx.x == 0) init_ctl(rp.ctl_init, rp.q0t, rp.N);
   stage_table(img, smem);
+  if (SUPER) {
+    const uint4* src = reinterpret_cast<const uint4*>(img.TK);
+    uint4* dst = reinterpret_cast<uint4*>(smem + tk_off(img));
+    for (uint32_t i = threadIdx.x; i < img.tk_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
+  }
   __syncthreads();
   using S = Step<MODE>;
   const uint32_t nt = img.n + 1, t = threadIdx.x;
@@ -298,15 +316,22 @@ __global__ void __launch_bounds__(kSmallT) k_enum_small(DevImage img, RunParams 
     uint32_t code[NE], acc[NE];
 #pragma unroll
     for (int q = 0; q < NE; q++) {
-      code[q] = __ldg(img.tid2code + ((uint32_t)q < nt ? q : 0));
+      code[q] = SUPER ? ((uint32_t)q < nt ? q : 0) * kTkRow : __ldg(img.tid2code + ((uint32_t)q < nt ? q : 0));
       acc[q] = 0;
+    }
+    if (SUPER && j >= nsub) {
+#pragma unroll
+      for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + code[q] / kTkRow);
     }
     if (j < nsub) {
       const uint64_t lo = j * E, n = min((uint64_t)E, rp.len - lo);
       const uint8_t* p = rp.in + lo;
       const uint4* v = reinterpret_cast<const uint4*>(p);
       uint64_t i = 0;
-      if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
+      if (SUPER) {
+        i = tk_walk<MODE, NE>(img, smem, static_cast<uint32_t>(__cvta_generic_to_shared(smem)) + tk_off(img),
+                              img.tk_syms, p, n, code, acc);
+      } else if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
         for (uint64_t t16 = 0; t16 < n / 16; t16++) {
           const uint4 qv = __ldg(v + t16);
           const uint32_t w[4] = {qv.x, qv.y, qv.z, qv.w};
@@ -399,11 +424,11 @@ __global__ void __launch_bounds__(kSmallT) k_enum_small(DevImage img, RunParams 
   }
 }
 
-template <int MODE, int NE>
+template <int MODE, int NE, bool SUPER = false>
 cudaError_t small_t(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, void* scratch,
                     uint32_t* ticket, uint32_t* chunk_ends, Ctl* ctl, cudaStream_t st) {
-  auto kern = k_enum_small<MODE, NE>;
-  const uint32_t smem = smem_bytes_for(img);
+  auto kern = k_enum_small<MODE, NE, SUPER>;
+  const uint32_t smem = SUPER ? tk_off(img) + img.tk_bytes : smem_bytes_for(img);
   cudaError_t e = kernel_setup((const void*)kern, smem, kSmallT, nullptr);
   if (e != cudaSuccess) return e;
   uint8_t* p = reinterpret_cast<uint8_t*>(scratch);
@@ -421,6 +446,11 @@ template <int MODE>
 cudaError_t small_m(const DevImage& img, const RunParams& rp, uint32_t E, uint64_t nsub, void* scratch,
                     uint32_t* ticket, uint32_t* chunk_ends, Ctl* ctl, cudaStream_t st) {
   const uint32_t nt = img.n + 1;  // <= 32 (the caller takes the multi-launch path for wider maps)
+  if (MODE == MODE_U8 && img.TK && !tk_disabled()) {  // small alphabet: K symbols per lookup
+    if (nt <= 8) return small_t<MODE, 8, true>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
+    if (nt <= 16) return small_t<MODE, 16, true>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
+    return small_t<MODE, 32, true>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
+  }
   if (nt <= 8) return small_t<MODE, 8>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
   if (nt <= 16) return small_t<MODE, 16>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);
   return small_t<MODE, 32>(img, rp, E, nsub, scratch, ticket, chunk_ends, ctl, st);

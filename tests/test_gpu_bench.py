@@ -51,3 +51,12 @@ def test_fused_round0_verification_path():
                          capture_output=True, text=True, timeout=900, env=e, cwd=ROOT)
     assert out.returncode == 0, out.stdout[-3000:] + out.stderr[-2000:]
     assert " passed" in out.stdout
+
+
+@pytest.mark.parametrize("config,steps", [("c1", 40), ("c2", 35)])
+def test_bench_more_steps_than_the_run_ring(config, steps):
+    """The driver picks K: more timed steps than a handle keeps runs in flight (32) must still
+    produce one line (bench.py keeps at most 16 runs queued, waiting for the oldest)."""
+    line = _bench("--config", config, "--steps", str(steps), "--warmup", "3", "--e2e-steps", "0",
+                  "--no-cpu-baseline", "--no-per-dfa")
+    assert line["steps"] == steps and line["value"] > 0 and line["gpu_launches"] >= steps

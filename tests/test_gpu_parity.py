@@ -161,13 +161,16 @@ def test_invalid_symbol_is_loud(gs):
 @pytest.mark.parametrize("name,length,B", [("c1", (16 << 20) + 5, 4096), ("rand:40:3:2", (12 << 20) + 333, 4096),
                                            ("rand:60:4:7", 10 << 20, 2048), ("rand:9:2:4", (6 << 20) + 17, 1024),
                                            ("c1", 3 << 20, 4096), ("rand:12:3:5", (9 << 20) + 64, 4096),
-                                           ("rand:14:30:2", (8 << 20) + 1000, 4096), ("rand:5:4:3", 5 << 20, 512)])
+                                           ("rand:14:30:2", (8 << 20) + 1000, 4096), ("rand:5:4:3", 5 << 20, 512),
+                                           ("c1", 1 << 20, 4096), ("rand:9:2:4", 300001, 1024),
+                                           ("rand:30:3:8", (1 << 20) + 9, 4096)])
 def test_enum_four_symbol_table(gs, name, length, B):
     """ENUM on small alphabets walks 16-byte vectors K symbols per lookup (TK: K = 8 for
     nsyms <= 2, 4 for nsyms <= 4); the unaligned tail and vectors holding a
-    byte TK does not cover take the one-symbol step.  Bit-exact against the oracle with TK on
-    and off (GSPEC_TK=0), for nt from 6 to 61 (rows padded to 257 words, staged in 16-byte
-    pieces) and a 30-symbol DFA that has no TK."""
+    byte TK does not cover take the one-symbol step — in the multi-launch walk and in the
+    single-launch kernel of streams up to 2 MiB.  Bit-exact against the oracle with TK on and
+    off (GSPEC_TK=0), for nt from 6 to 61 (rows padded to 257 words, staged in 16-byte pieces)
+    and a 30-symbol DFA that has no TK."""
     import os
     w, data = _wl(name, length)
     ref = oracle.run(w.table, w.start, w.accept, data, B)
