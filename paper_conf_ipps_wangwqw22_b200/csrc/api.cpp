@@ -1322,7 +1322,6 @@ int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_
     }
     ft.chunk_bytes = fsm_chunk_for(&ft, stream_len);
   }
-  f->auto_chunk = ft.chunk_bytes;
   const fsm_scheme pick = tree_select(ft, f->n);
   if (N > 1) f->acc1_hint = ft.acc1;
   f->auto_scheme = pick;

@@ -501,7 +501,6 @@ struct fsm_s {
     uint32_t* status;
   };
   const P2PWait* p2p_wait = nullptr;
-  uint32_t auto_chunk = 0;  // the selector's recommended chunk size (R29), 0 before a selection
   bool p2p_published = false;
   void* img2_base = nullptr;             // lookback > 2: full pair images (built at first use)
   uint32_t *img2_s = nullptr, *img2_m = nullptr;

@@ -86,18 +86,6 @@ __device__ __forceinline__ T block_sum(T v, T* red) {
   return s;  // valid in thread 0
 }
 
-__device__ __forceinline__ uint64_t block_min(uint64_t v, uint64_t* red) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v = min(v, (uint64_t)__shfl_down_sync(0xffffffffu, (unsigned long long)v, o));
-  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
-  __syncthreads();
-  uint64_t s = ~0ull;
-  if (threadIdx.x == 0)
-    for (int w = 0; w < kBS / 32; w++) s = min(s, red[w]);
-  __syncthreads();
-  return s;
-}
-
 // One block reduction for a relaxation pass: OR(changed), MIN(frontier), SUM(checks), SUM(matches).
 __device__ __forceinline__ void block_reduce_pass(bool ch, uint64_t& fm, uint64_t& checks, uint64_t& matches,
                                                   uint64_t (*red)[kBS / 32], bool* any) {
