@@ -70,6 +70,21 @@ def test_fake_collective(gs, name, length, G, L):
     assert (ce == ref["chunk_end"]).all()
 
 
+@pytest.mark.parametrize("name,length,G,B,scheme", [("c3", (48 << 20) + 8192 * 3, 8, 8192, "sre"),
+                                                  ("c3s", 40 << 20, 3, 8192, "nf"), ("c2", 24 << 20, 4, 16384, "sre"),
+                                                  ("c1", (6 << 20) + 100, 3, 8192, "enum")])
+def test_fake_collective_recommended_chunks(gs, name, length, G, B, scheme):
+    """The sharded pipeline at the chunk sizes the selector recommends (R29: 8 / 16 KiB), as
+    bench.py --config c5 runs it: shard bounds on B, dense SRE / NF rounds inside the shards."""
+    w = gen.workload(name, length=length)
+    data = w.host()
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    outs, ce = sharded_fake(gs, w, data, G, B=B, scheme=scheme, L=16)
+    for r in outs:
+        assert r.final_state == ref["final"] and r.accept_count == ref["count"]
+    assert (ce == ref["chunk_end"]).all()
+
+
 def test_single_rank_nccl_group(gs):
     import os
     import torch.distributed as dist
