@@ -396,43 +396,53 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       git++;
       const uint64_t f2 = vctl->it_fm[slot];
       const uint64_t nt = vctl->it_ntask[slot];
+      const uint32_t chg = vctl->changed[slot];  // (set before the barrier, final here)
       if (b == 0 && threadIdx.x == 0) {
+        // commit the round on the control block: every field is loaded in one batch of
+        // independent loads, then written — not a chain of read-modify-write L2 round trips
+        // on the critical path of the run's last CTA (it cost ~6 us per run on C2)
+        const uint64_t ic = vctl->it_checks[slot], im = vctl->it_matches[slot], ir = vctl->it_reread[slot];
+        const uint64_t vc = vctl->verify_checks, vm = vctl->verify_matches, ji = vctl->jacobi_iters;
+        const uint64_t tm = vctl->tasks_mustdo, ts = vctl->tasks_sre, rb = vctl->reread_bytes;
+        const uint64_t as = vctl->active_sum, rd = vctl->rounds;
+        const uint32_t tf2h = f2 < N ? ld_cg(rs.x + f2) : 0u;
         if (rp.dense && nt >= 2048 && nt * 16 >= N) vctl->dense_denied = 1;  // a dense round ran here
-        vctl->verify_checks = vctl->verify_checks + vctl->it_checks[slot];
-        vctl->verify_matches = vctl->verify_matches + vctl->it_matches[slot];
-        vctl->jacobi_iters = vctl->jacobi_iters + 1;
-        vctl->fmin = f2;
+        uint64_t nvc = vc + ic, nvm = vm + im, fmin = f2;
+        if (f2 < N) {  // the must-do is chunk f2
+          vctl->tasks_mustdo = tm + 1;
+          vctl->tasks_sre = ts + (nt - 1);
+          vctl->reread_bytes = rb + ir;
+          vctl->active_sum = as + nt;
+          vctl->rounds = rd + 1;
+          vctl->f = f2;
+          vctl->tf = tf2h;
+          if (chg == 0) {  // round 1 settled without its pass (below)
+            nvc += N - f2;
+            nvm += N - f2;
+            fmin = N;
+          }
+        }
+        vctl->verify_checks = nvc;
+        vctl->verify_matches = nvm;
+        vctl->jacobi_iters = ji + 1;
+        vctl->fmin = fmin;
       }
       if (f2 >= N) {
         z_early = true;
         break;
       }
       const uint32_t tf2 = ld_cg(rs.x + f2);  // = end_{f2-1}: not rewritten by the tasks
-      if (b == 0 && threadIdx.x == 0) {      // commit the round (the must-do is chunk f2)
-        vctl->tasks_mustdo = vctl->tasks_mustdo + 1;
-        vctl->tasks_sre = vctl->tasks_sre + (nt - 1);
-        vctl->reread_bytes = vctl->reread_bytes + vctl->it_reread[slot];
-        vctl->active_sum = vctl->active_sum + nt;
-        vctl->rounds = vctl->rounds + 1;
-        vctl->f = f2;
-        vctl->tf = tf2;
-      }
       f = f2;
       tf = tf2;
       rnd++;
       last_tasks = nt;
-      if (vctl->changed[slot] == 0) {
+      if (chg == 0) {
         // No task changed its chunk's end (every recovery merged with the round-0 path —
         // the usual case for convergent DFAs): the incoming states x are those of round 0,
         // and every chunk now holds a record for its incoming state (its round-0 record, or
         // the task's from x_c).  Round 1's verification therefore matches every chunk from
-        // f2 on: count its N - f2 checks (all matches, per the round semantics) and finish
-        // without the pass.
-        if (b == 0 && threadIdx.x == 0) {
-          vctl->verify_checks = vctl->verify_checks + (N - f2);
-          vctl->verify_matches = vctl->verify_matches + (N - f2);
-          vctl->fmin = N;
-        }
+        // f2 on: its N - f2 checks (all matches, per the round semantics) were counted
+        // above, and the run finishes without the pass.
         z_early = true;
         break;
       }
@@ -903,15 +913,21 @@ __global__ void __launch_bounds__(kBS) k_verify_recover(DevImage img, RunParams 
       }
     }
     if (z_early) {  // counts summed by the round-0 pass (complete: every CTA added before its barrier)
-      if (b == 0 && threadIdx.x == 0) ctl->accept_count = ld_cg64(&ctl->ntask[1]);
+      if (b == 0 && threadIdx.x == 0) {
+        const uint64_t acc_sum = ld_cg64(&ctl->ntask[1]);  // (both loads in flight together)
+        const uint32_t xf = ld_cg(rs.x + N);
+        ctl->accept_count = acc_sum;
+        ctl->xfin = xf;
+        ctl->finished = 1;  // before this CTA's fence + ticket: the publishing CTA sees it
+      }
     } else {
       total = block_sum<uint64_t>(total, red64);
       if (threadIdx.x == 0)
         atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->accept_count), (unsigned long long)total);
-    }
-    if (b == 0 && threadIdx.x == 0) {
-      ctl->xfin = ld_cg(rs.x + N);
-      ctl->finished = 1;  // before this CTA's fence + ticket: the publishing CTA sees it
+      if (b == 0 && threadIdx.x == 0) {
+        ctl->xfin = ld_cg(rs.x + N);
+        ctl->finished = 1;  // before this CTA's fence + ticket: the publishing CTA sees it
+      }
     }
     stamp();
     if (rp.h_out) {
