@@ -71,6 +71,7 @@ def lib():
                                           ctypes.POINTER(SimResult), ctypes.POINTER(PmStats)]
         L.or_features_compute.argtypes = [P, U32, U32, U32, P, P, U64, U32, U32, U32, ctypes.POINTER(Features)]
         L.or_select.argtypes = [ctypes.POINTER(Features), U32]
+        L.or_select_variant.argtypes = [ctypes.POINTER(Features), U32, ctypes.c_int]
         L.or_conv_lengths.argtypes = [P, U32, U32, P, U64, U32, P]
         L.or_conv_lengths.restype = U32
         L.or_select_chunk.argtypes = [P, U32, U64, U64]
@@ -295,8 +296,11 @@ def features(table, start, accept, data, B=4096, k=4, qs_cap=16, policy=0):
     return {"acc1": f.acc1, "acck": f.acck, "sens": f.sens, "uniq10": f.uniq10}
 
 
-def select(feat: dict, nstates: int) -> int:
+def select(feat: dict, nstates: int, paper_tree: bool = False) -> int:
+    """The selector's decision tree (R19); paper_tree: without the B200 gate R19b."""
     f = Features(feat["acc1"], feat["acck"], feat["sens"], feat["uniq10"])
+    if paper_tree:
+        return int(lib().or_select_variant(ctypes.byref(f), nstates, 1))
     return int(lib().or_select(ctypes.byref(f), nstates))
 
 

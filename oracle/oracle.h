@@ -159,6 +159,8 @@ uint32_t or_select_chunk(const uint32_t* d, uint32_t nwin, uint64_t len, uint64_
 
 /* Decision tree (Fig. 6 reconstructed, reading c.4 #19). Returns a scheme id. */
 int or_select(const or_features* f, uint32_t nstates);
+/* variant 0 = or_select; 1 = the reconstructed tree without the B200 gate R19b. */
+int or_select_variant(const or_features* f, uint32_t nstates, int variant);
 
 #ifdef __cplusplus
 }

@@ -831,3 +831,28 @@ def test_select_chunk_rule():
     assert oracle.select_chunk(d16, 16 * G, 113664) == 16384
     assert oracle.select_chunk(d16, G, 113664) == 4096
     assert oracle.select_chunk([64, 64, 64, never], G, 113664) == 4096  # exactly 3/4 within 4K
+
+
+def test_select_paper_tree_variant():
+    """R19 without the B200 gate R19b (the paper's Fig. 6 as reconstructed): once ENUM, SRE
+    (uniq10 <= 4) and PM are excluded, input sensitivity >= 0.2 -> NF, else RR; the default
+    tree sends the same features to SRE while the spec-k gain stays below 0.5."""
+    f = {"acc1": 0.2, "acck": 0.6, "sens": 0.3, "uniq10": 16.0}
+    assert oracle.select(f, 816, paper_tree=True) == oracle.NF
+    assert oracle.select(dict(f, sens=0.1), 816, paper_tree=True) == oracle.RR
+    assert oracle.select(f, 816) == oracle.SRE
+    assert oracle.select(dict(f, acck=0.75), 816) == oracle.NF  # gain >= 0.5: both trees agree
+    assert oracle.select(dict(f, acck=0.95, acc1=0.7), 816, paper_tree=True) == oracle.PM
+    assert oracle.select(dict(f, uniq10=3.0), 816, paper_tree=True) == oracle.SRE
+    assert oracle.select(dict(f, uniq10=40.0), 63, paper_tree=True) == oracle.ENUM
+
+
+def test_select_paper_tree_on_c3s_boundary():
+    """The input-sensitive stream across a normal / vowel-free region boundary (features
+    pinned by brute force above): the paper's tree picks NF."""
+    w = gen.workload("c3s")
+    B, N = 4096, 65
+    data = w.host((1 << 26) - 33 * B, N * B)
+    f = oracle.features(w.table, w.start, w.accept, data, B=B)
+    assert f["sens"] >= 0.2
+    assert oracle.select(f, w.nstates, paper_tree=True) == oracle.NF
