@@ -614,8 +614,11 @@ fsm_scheme tree_select(const fsm_features& ft, uint32_t n) {
   if (ft.uniq10 <= 4.0) return FSM_SCHEME_SRE;
   if (ft.acck >= 0.9 && ft.acck - ft.acc1 >= 0.2) return FSM_SCHEME_PM;
   // R19b: helpers cost a full chunk walk on a saturated GPU; RR/NF only when the
-  // extra lookback candidates catch most mispredictions
-  if (ft.acck - ft.acc1 < 0.5) return FSM_SCHEME_SRE;
+  // extra lookback candidates catch most mispredictions (GSPEC_SELECTOR=paper: the
+  // reconstructed tree without this gate)
+  const char* sel = getenv("GSPEC_SELECTOR");
+  const bool paper = sel && std::strcmp(sel, "paper") == 0;
+  if (!paper && ft.acck - ft.acc1 < 0.5) return FSM_SCHEME_SRE;
   if (ft.input_sensitivity >= 0.2) return FSM_SCHEME_NF;
   return FSM_SCHEME_RR;
 }

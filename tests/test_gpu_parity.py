@@ -627,6 +627,33 @@ def test_selector_spread_profile(gs, name):
     torch.cuda.empty_cache()
 
 
+def test_selector_paper_tree_picks_nf_on_c3s(gs):
+    """GSPEC_SELECTOR=paper: the reconstructed Fig. 6 tree without the B200 gate (R19b) —
+    on the input-sensitive 1 GiB stream the selector picks NF, as the oracle's
+    variant does on the same spread profile; then the NF run is bit-exact on a prefix."""
+    import os
+    L = 1 << 30
+    w = gen.workload("c3s", length=L)
+    x = torch.empty(L, dtype=torch.uint8, device="cuda")
+    w.device(x)
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    os.environ["GSPEC_SELECTOR"] = "paper"
+    try:
+        pick, ft = fsm.select_scheme(x)
+    finally:
+        os.environ.pop("GSPEC_SELECTOR", None)
+    of = oracle.features(w.table, w.start, w.accept, _spread_host(w, L), B=4096)
+    assert gs.SCHEMES[pick] == oracle.select(of, w.nstates, paper_tree=True) == oracle.NF
+    assert oracle.select(of, w.nstates) == oracle.SRE  # the default tree (R19b)
+    n = 96 << 20
+    ref = oracle.run(w.table, w.start, w.accept, x[:n].cpu().numpy(), 8192)
+    res = fsm.run(x[:n], scheme="auto", chunk_bytes=8192)
+    assert res.scheme == "nf"
+    check_equal(res, ref, 8192, w.nstates)
+    del x
+    torch.cuda.empty_cache()
+
+
 @pytest.mark.parametrize("name,length", [("c1", 1 << 20), ("c2", 1 << 20), ("c3", 1 << 20), ("c4", 1 << 20),
                                          ("rand:40:7:3", 600000), ("rand:300:4:1", 1 << 20), ("c3s", 900000)])
 def test_conv_fractions_match_oracle(gs, name, length):
