@@ -156,6 +156,8 @@ int fsm_run_sharded_p2p(fsm_t f, fsm_p2p_t p, const uint8_t* d_shard, uint64_t s
     const fsm_s::P2PWait wt{reinterpret_cast<const unsigned long long*>(p->box + 2ull * G * p->mapb) +
                                 (uint64_t)set * G,
                             seq, p->d_status};
+    if (cudaMemsetAsync(p->d_status, 0, 4, st) != cudaSuccess)  // (a finish that fails early leaves it 0)
+      return gspec_set_error(FSM_ECUDA, "p2p status reset");
     f->p2p_wait = &wt;
     rc = fsm_shard_finish(f, p->box + (uint64_t)set * G * p->mapb, G, rank, opts, d_chunk_ends_local, out_global);
     f->p2p_wait = nullptr;
