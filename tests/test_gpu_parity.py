@@ -627,6 +627,24 @@ def test_selector_spread_profile(gs, name):
     torch.cuda.empty_cache()
 
 
+@pytest.mark.parametrize("length", [0, 1, 100, 20000, 21 << 10, 200 << 10])
+def test_selector_short_samples(gs, length):
+    """Profiles too short for a convergence window (or empty) still select, and recommend the
+    default chunk size; the fractions match the oracle's windows (none below 20 KiB)."""
+    w, data = _wl("c3", max(length, 1))
+    data = data[:length]
+    fsm = gs.FSM.load(w.table, w.start, w.accept)
+    pick, ft = fsm.select_scheme(torch.from_numpy(data.copy()).cuda())
+    assert pick in gs.SCHEMES and ft["chunk_bytes"] == 4096
+    d = oracle.conv_lengths(w.table, w.start, w.accept, data, wmax=16384) if length else np.zeros(0, np.uint32)
+    assert (d.size == 0) == (length < 4096 + 16384 + 1)  # the first window needs 4 KiB + 16 KiB
+    if d.size == 0:
+        assert ft["conv4k"] == ft["conv8k"] == ft["conv16k"] == 0.0
+    else:
+        for W, key in ((4096, "conv4k"), (8192, "conv8k"), (16384, "conv16k")):
+            assert ft[key] == pytest.approx(float((d <= W).sum()) / d.size, abs=0)
+
+
 def test_selector_paper_tree_picks_nf_on_c3s(gs):
     """GSPEC_SELECTOR=paper: the reconstructed Fig. 6 tree without the B200 gate (R19b) —
     on the input-sensitive 1 GiB stream the selector picks NF, as the oracle's
