@@ -60,3 +60,14 @@ def test_bench_more_steps_than_the_run_ring(config, steps):
     line = _bench("--config", config, "--steps", str(steps), "--warmup", "3", "--e2e-steps", "0",
                   "--no-cpu-baseline", "--no-per-dfa")
     assert line["steps"] == steps and line["value"] > 0 and line["gpu_launches"] >= steps
+
+
+def test_bench_default_line_two_ranks():
+    """The default line under bench.py's own relaunch at N = 2 (ranks sharing cuda:0 over gloo;
+    the driver's multi-GPU run takes the same path with NCCL): weak scaling, 1 GiB per rank
+    shard of one global stream, the end-to-end leg, one JSON line from rank 0."""
+    d = _bench("--gpus", "2", "--steps", "3", "--warmup", "3", "--e2e-steps", "1", "--no-cpu-baseline",
+               env={"GSPEC_DIST_BACKEND": "gloo"})
+    assert d["n_gpus"] == 2 and d["scaling"] == "weak" and d["config"]["workload"] == "c2"
+    assert d["value"] > 0 and d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 1 << 30
+    assert d["roofline"]["frac"] > 0 and d["gpu_launches"] > 0
