@@ -67,6 +67,7 @@ class ClockSampler:
         self._stop = threading.Event()
         self._t = None
         self._nvml = None
+        self._max_mhz = None
         try:
             import pynvml
             import torch
@@ -79,13 +80,16 @@ class ClockSampler:
             except Exception:
                 h = pynvml.nvmlDeviceGetHandleByIndex(index)
             self._nvml = (pynvml, h)
+            self._max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)  # before the timed region
         except Exception:
             self._nvml = None
 
     def _sample_nvml(self):
         nv, h = self._nvml
         sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
-        mx = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+        if self._max_mhz is None:  # constant, and ~6 ms per call (the other two take microseconds)
+            self._max_mhz = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+        mx = self._max_mhz
         try:
             rs = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
         except Exception:
@@ -110,6 +114,10 @@ class ClockSampler:
             self._stop.wait(0.0005 if self._nvml else 0.1)
 
     def __enter__(self):
+        # a short GIL switch interval so the sampler thread gets its turns while the main
+        # thread queues the timed steps (the GPU is ahead of the host: no effect on the timing)
+        self._swi = sys.getswitchinterval()
+        sys.setswitchinterval(2e-4)
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
         return self
@@ -118,6 +126,7 @@ class ClockSampler:
         self._stop.set()
         if self._t:
             self._t.join(timeout=10)
+        sys.setswitchinterval(self._swi)
 
     def summary(self):
         if not self.samples:
@@ -240,6 +249,15 @@ def run_reference(args):
     return 0
 
 
+def _head_start():
+    """A ~1 ms GPU spin queued right before the first timing event: while it runs the host
+    queues the first steps, so the event pair times the K steps' device work rather than the
+    host's latency to enqueue the first one (the spin itself is outside the timed region)."""
+    import torch
+
+    torch.cuda._sleep(2_000_000)
+
+
 def _median(v):
     v = sorted(v)
     return v[len(v) // 2] if v else None
@@ -294,6 +312,7 @@ def measure_single(gs, w, x, args, fsm, scheme, B, with_clocks=True):
     clk = ClockSampler(torch.cuda.current_device()) if with_clocks else None
     if clk:
         clk.__enter__()
+    _head_start()
     ev0.record(stream)
     for _ in range(args.steps):
         enqueue(pending)
@@ -474,6 +493,7 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         pend = []
         with ClockSampler(dev) as clk:
+            _head_start()
             ev0.record(stream)
             if comm is not None and p2p is None:  # steps queued back to back: no host wait between them
                 res = async_sharded_steps(gs, comm, fsm, x, lb, scheme, B, ce, args.steps)
@@ -527,6 +547,7 @@ def run_c5(args, gs, dist, world, rank, dev, comm, peak, peak_kind):
                    "chunk_bytes": "per DFA (per_dfa[*].chunk_bytes: the selector's R29 recommendation)"
                    if not args.chunk_bytes else args.chunk_bytes,
                    "l2": "input (16 GiB / N per GPU) larger than the 126 MB L2; no flush",
+                   "timing": "CUDA events around the K steps after a ~1 ms GPU spin (host head start), max over ranks",
                    "parallelism": f"{world} contiguous shards + one exchange of state maps"
                    + (" (peer-memory stores, fsm_run_sharded_p2p)" if dist is not None and args.exchange == "p2p" else
                       " (library NCCL allgather, fsm_run_sharded_async)" if comm is not None else
@@ -662,6 +683,7 @@ def main():
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         pend = []
         with ClockSampler(dev) as clk:
+            _head_start()
             ev0.record(stream)
             if comm is not None and p2p is None:  # steps queued back to back: no host wait between them
                 res = async_sharded_steps(gs, comm, fsm, x, lb, scheme, B, ce_sh, args.steps)
@@ -742,6 +764,8 @@ def main():
                    "chunk_bytes": B, "scheme": scheme, "nstates": int(w.nstates), "spec_k": args.spec_k or None,
                    "lookback": args.lookback,
                    "l2": "input (1 GiB/GPU) larger than the 126 MB L2; no explicit flush",
+                   "timing": "CUDA events on the launching stream around the K steps (a ~1 ms GPU spin queued "
+                             "before the first event lets the host queue ahead; it is outside the region)",
                    "parallelism": (f"dp{world} contiguous shards + one exchange of state maps"
                                    + (" (peer-memory stores, fsm_run_sharded_p2p)" if args.exchange == "p2p" else
                                       " (library NCCL allgather, fsm_run_sharded_async)" if comm is not None else "")
