@@ -120,6 +120,10 @@ typedef struct {
    * when a verification first matches it); 0 with eager helpers.  tasks_helper and
    * reread_bytes count every assigned helper either way, as the round semantics define. */
   uint64_t helper_walks;
+  /* Bytes the dense-round task kernels actually walked (R30: a task stops where
+   * its path meets the chunk's round-0 path at a checkpoint, so this is at most
+   * reread_bytes' share of those rounds); diagnostic, 0 when no dense round ran. */
+  uint64_t task_walked_bytes;
 } fsm_result;
 
 typedef struct {

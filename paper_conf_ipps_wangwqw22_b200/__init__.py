@@ -48,7 +48,8 @@ class fsm_result(ctypes.Structure):
                 ("tasks_sre", U64), ("tasks_helper", U64), ("reread_bytes", U64), ("verify_checks", U64),
                 ("verify_matches", U64), ("avg_active_workers", ctypes.c_double), ("ms_spec", ctypes.c_double),
                 ("ms_verify", ctypes.c_double), ("kernel_launches", U32), ("pm_merge_checks", U64),
-                ("pm_invalid_marks", U64), ("pm_jumps", U64), ("helper_walks", U64)]
+                ("pm_invalid_marks", U64), ("pm_jumps", U64), ("helper_walks", U64),
+                ("task_walked_bytes", U64)]
 
 
 class fsm_batch_result(ctypes.Structure):

@@ -249,6 +249,7 @@ void fill_result_stats(fsm_result* out, const Ctl& h) {
   out->pm_invalid_marks = h.pm_invalid_marks;
   out->pm_jumps = h.pm_jumps;
   out->helper_walks = h.helper_walks;
+  out->task_walked_bytes = h.walked_bytes;
 }
 
 int select_auto(fsm_t f, const uint8_t* d_in, uint64_t len, const fsm_run_opts* opts);
@@ -420,6 +421,27 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     rp.dense = ((scheme == FSM_SCHEME_SRE || scheme == FSM_SCHEME_CSE || scheme == FSM_SCHEME_RR ||
                  scheme == FSM_SCHEME_NF) && len / o.B > 0 && o.B % 64 == 0 &&
                 (reinterpret_cast<uintptr_t>(d_in) & 15u) == 0 && f->acc1_hint < 0.5) ? 1u : 0u;
+    // R30: the round-0 TMA walk checkpoints its path so dense tasks stop where they meet it
+    {
+      const uint32_t sh = ck_shift_default();
+      if (rp.dense && rp.k == 1 && sh && !spec_path_generic_only() && o.B % (1u << sh) == 0 &&
+          o.B >= (2u << sh)) {
+        const size_t nck = (size_t)(o.B / (1u << sh) - 1) * N * sizeof(uint2);
+        const size_t need = ((nck + 255) & ~(size_t)255) + 2 * f->rs.cap * 16;  // + the passes' chain lists
+        if (f->ck_bytes < need) {
+          CUDA_TRY(cudaStreamSynchronize(o.st));  // queued runs may still read the old array
+          if (f->ck_base) cudaFree(f->ck_base);
+          f->ck_base = nullptr;
+          f->ck_bytes = 0;
+          CUDA_TRY(cudaMalloc(&f->ck_base, need));
+          f->ck_bytes = need;
+        }
+        rp.ck = reinterpret_cast<uint2*>(f->ck_base);
+        rp.ck_shift = sh;
+        rp.ck_seg = ck_seg_for(o.B, sh);
+        rp.ck_list = reinterpret_cast<uint8_t*>(f->ck_base) + ((nck + 255) & ~(size_t)255);
+      }
+    }
     {
       // accurate SRE (no dense rounds expected): round 0's verification and its inline
       // recoveries run inside the TMA spec kernel as its tiles finish (RunParams::v0); the
@@ -432,7 +454,9 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       rp.v0_chunk_ends = d_chunk_ends;
       rp.tma_evict_normal = tma_evict_mode() == 1 ? 1u : 0u;
       NvtxRange nv_("speculative execution (round 0)");
-      CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st));
+      uint64_t tma_done = 0;
+      CUDA_TRY(launch_spec_exec(f->img, rp, f->rs, o.st, &tma_done));
+      if (tma_done < len / o.B) rp.ck_shift = 0;  // the full chunks were not walked by the TMA kernel: no checkpoints
     }
     {  // TMA kernel over the full chunks + the generic kernel for a tail chunk (or everything)
       const bool tma = !spec_path_generic_only() && len / o.B > 0 && o.B % 64 == 0 &&
@@ -454,7 +478,8 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       CUDA_TRY(launch_task_dense(f->img, rp, f->rs, f->d_ctl, f->sm_count, o.st));
       rp.dense_slots = slots - 1 - r;
       CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
-      pd.launches += 3;  // task kernel + finish + verify (no-ops once the run is complete)
+      // task kernel (R30: one launch per segment pass) + finish + verify (no-ops once the run is complete)
+      pd.launches += 2 + (rp.ck_shift && rp.ck_seg ? (o.B + rp.ck_seg - 1) / rp.ck_seg : 1u);
     }
     pd.dense_slots = slots;
     pd.dense = rp.dense != 0;
@@ -902,6 +927,7 @@ void fsm_free(fsm_t f) {
     if (e) cudaEventDestroy(e);
   if (f->multi_base) cudaFree(f->multi_base);
   if (f->pm_base) cudaFree(f->pm_base);
+  if (f->ck_base) cudaFree(f->ck_base);
   if (f->prof_buf) cudaFree(f->prof_buf);
   if (f->img2_base) cudaFree(f->img2_base);
   if (f->qsc_base) cudaFree(f->qsc_base);

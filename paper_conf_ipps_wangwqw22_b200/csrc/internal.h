@@ -147,6 +147,9 @@ struct Ctl {
   // FSM_SCHEME_PM_TREE (pm_tree.cu): stage-1 lookups, entries marked invalid, stage-2 jumps
   uint64_t pm_merge_checks, pm_invalid_marks, pm_jumps;
   uint64_t helper_walks;  // RR / NF helper records actually walked (memoized helpers, R28)
+  uint64_t walked_bytes;  // bytes the dense-round task kernels actually walked (R30 early exit)
+  uint32_t segn[3];       // checkpointed dense round: chains appended by pass p in segn[p % 3] (R30)
+  uint32_t pad3;
 };
 
 struct RunParams {
@@ -176,6 +179,13 @@ struct RunParams {
   uint32_t* v0_chunk_ends; // nullable: the run's chunk ends (original ids)
   uint32_t tma_evict_normal;  // 1: input TMA loads with L2 evict_normal (else evict_first)
   uint32_t lazy_helpers;      // 1: RR / NF helper records are memoized (walked when first matched, R28)
+  // checkpointed dense rounds (R30): the round-0 TMA walk stores {code, count so far}
+  // of its path every 2^ck_shift bytes at ck[j * N + c] (j = bytes / 2^ck_shift - 1); a dense
+  // task stops at the first checkpoint where it meets that path.  ck_shift 0 = off.
+  uint2* ck;
+  uint32_t ck_shift;
+  uint32_t ck_seg;  // bytes per segment pass of a checkpointed dense round (0: plain task kernel)
+  void* ck_list;    // the passes' two lists of running chains, [2][rs.cap] x 16 B
 };
 
 // GSPEC_STAMPS=1: kernels record the run timeline in Ctl::tl (one extra atomic per warp).
@@ -216,6 +226,34 @@ inline int tma_promotion() {
     v = e ? atoi(e) : 0;
   }
   return v;
+}
+
+// R30 checkpoint interval of dense rounds (GSPEC_CK: bytes, a power of two >= 64; 0 = off,
+// the plain TMA task kernel).  Returns log2 of the interval, 0 when off.
+inline uint32_t ck_shift_default() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("GSPEC_CK");
+    const long b = e ? atol(e) : 512;
+    v = 0;
+    if (b >= 64 && (b & (b - 1)) == 0)
+      while ((1l << v) < b) v++;
+  }
+  return (uint32_t)v;
+}
+
+// R30 segment of a checkpointed dense-round pass (GSPEC_CK_SEG: bytes, a multiple of the
+// checkpoint interval; default a quarter of the chunk rounded up to the interval).
+inline uint32_t ck_seg_for(uint32_t B, uint32_t ck_shift) {
+  static long v = -2;
+  if (v == -2) {
+    const char* e = getenv("GSPEC_CK_SEG");
+    v = e ? atol(e) : -1;
+  }
+  const uint32_t cp = 1u << ck_shift;
+  uint32_t seg = v > 0 ? (uint32_t)v : (B / 4 + cp - 1) / cp * cp;
+  seg = (seg + cp - 1) / cp * cp;
+  return seg < cp ? cp : seg;
 }
 
 inline int tma_evict_mode() {
@@ -313,7 +351,9 @@ inline int device_sms() {
 // ---- launchers (each returns the cudaError_t of the launch) ------------------
 cudaError_t launch_build_qs2_raw(const uint32_t* d_ttc, uint32_t n, uint32_t C, uint32_t* scratch, uint32_t grid,
                                  uint32_t* qs2, uint8_t* qs2_len, uint32_t* qs2_img, cudaStream_t st);
-cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st);
+// *tma_done (nullable): chunks the TMA spec kernel walked (the rest went to the generic kernel)
+cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st,
+                             uint64_t* tma_done = nullptr);
 cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, int sms, cudaStream_t st,
                             uint64_t* n_done);
 // Dense recovery round, device-driven: if the preceding verify launch left a dense round
@@ -509,6 +549,8 @@ struct fsm_s {
   uint64_t qsc_cap = 0;
   void* pm_base = nullptr;               // FSM_SCHEME_PM_TREE scratch (level maps, jump list)
   size_t pm_bytes = 0;
+  void* ck_base = nullptr;               // R30: round-0 path checkpoints [B / 2^ck_shift - 1][N]
+  size_t ck_bytes = 0;
   void* multi_base = nullptr;            // fsm_run_multi scratch when this handle is fsms[0] (its device)
   size_t multi_cap = 0;
   cudaEvent_t multi_ev[2] = {nullptr, nullptr};

@@ -179,12 +179,15 @@ cudaError_t launch_spec_generic(const DevImage& img, const RunParams& rp, const 
   }
 }
 
-cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st) {
+cudaError_t launch_spec_exec(const DevImage& img, const RunParams& rp, const RecStore& rs, cudaStream_t st,
+                             uint64_t* tma_done) {
+  if (tma_done) *tma_done = 0;
   if (rp.N == 0) return cudaSuccess;
   const int sms = device_sms();
   uint64_t done = 0;
   cudaError_t e = spec_path_generic_only() ? cudaErrorNotSupported : launch_spec_tma(img, rp, rs, sms, st, &done);
   if (e != cudaSuccess && e != cudaErrorNotSupported) return e;
+  if (tma_done && e == cudaSuccess) *tma_done = done;
   RunParams rp2 = rp;
   if (e == cudaErrorNotSupported) {
     cudaGetLastError();  // clear

@@ -20,6 +20,7 @@ namespace {
 
 constexpr uint32_t kRowBytes = 64;              // box inner extent (bytes per chunk per stage)
 constexpr uint32_t kStageBytes = 32 * kRowBytes;  // 32 rows (chunks) per box
+constexpr uint32_t kNoTask = 0xFFFFFFFFu;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -342,30 +343,27 @@ __global__ void __launch_bounds__(KP > 8 ? 512 : 896, 1) k_spec_tma(const __grid
 #pragma unroll
       for (int u = 0; u < (int)(kRowBytes / 16); u++) {
         const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ ((lane >> 1) & 3)) << 4));  // SWIZZLE_64B
-        const uint32_t w[4] = {q.x, q.y, q.z, q.w};
-#pragma unroll
-        for (int t = 0; t < 4; t++) {
-          code[0] = Sx::template word<0>(img, table, code[0], w[t]); acc[0] += Sx::acc(code[0]);
-          code[0] = Sx::template word<1>(img, table, code[0], w[t]); acc[0] += Sx::acc(code[0]);
-          code[0] = Sx::template word<2>(img, table, code[0], w[t]); acc[0] += Sx::acc(code[0]);
-          code[0] = Sx::template word<3>(img, table, code[0], w[t]); acc[0] += Sx::acc(code[0]);
-        }
+        walk16<MODE>(img, table, q, code[0], acc[0]);
       }
     } else {
 #pragma unroll
       for (int u = 0; u < (int)(kRowBytes / 16); u++) {
         const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ ((lane >> 1) & 3)) << 4));  // SWIZZLE_64B
-        const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+        if (KP == 1) {
+          walk16<MODE>(img, table, q, code[0], acc[0]);
+        } else {  // the paths share each symbol's class lookup
+          const uint32_t w[4] = {q.x, q.y, q.z, q.w};
 #pragma unroll
-        for (int t = 0; t < 4; t++) {
+          for (int t = 0; t < 4; t++) {
+            const uint32_t u1[1] = {w[t]};
+            uint32_t k4[4];
+            cls_words<MODE, 1>(img, table, u1, k4);
 #pragma unroll
-          for (int p = 0; p < KP; p++) { code[p] = Sx::template word<0>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+            for (int i = 0; i < 4; i++) {
 #pragma unroll
-          for (int p = 0; p < KP; p++) { code[p] = Sx::template word<1>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
-#pragma unroll
-          for (int p = 0; p < KP; p++) { code[p] = Sx::template word<2>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
-#pragma unroll
-          for (int p = 0; p < KP; p++) { code[p] = Sx::template word<3>(img, table, code[p], w[t]); acc[p] += Sx::acc(code[p]); }
+              for (int p = 0; p < KP; p++) { code[p] = Sx::next(img, table, code[p], k4[i]); acc[p] += Sx::acc(code[p]); }
+            }
+          }
         }
       }
       if (KP > 1) {  // DFA determinism: paths that meet stay together; once all have met, walk one
@@ -378,6 +376,11 @@ __global__ void __launch_bounds__(KP > 8 ? 512 : 896, 1) k_spec_tma(const __grid
           for (int p = 0; p < KP; p++) dacc[p] = acc[p] - acc[0];
         }
       }
+    }
+    if (!TASKS && KP == 1 && rp.ck_shift && c < n_full) {  // R30: checkpoint of the round-0 path
+      const uint32_t pe = (sg + 1) * kRowBytes;
+      if ((pe & ((1u << rp.ck_shift) - 1u)) == 0 && pe < rp.B)
+        rp.ck[(uint64_t)((pe >> rp.ck_shift) - 1) * rp.N + c] = make_uint2(code[0], acc[0]);
     }
     __syncwarp();
     if (it + S < items) issue_next();  // refill this stage
@@ -508,7 +511,208 @@ __global__ void __launch_bounds__(KP > 8 ? 512 : 896, 1) k_spec_tma(const __grid
                 (unsigned long long)(n_mustdo + n_sre + n_hel));
       atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->reread_bytes),
                 (unsigned long long)((n_mustdo + n_sre + n_hel) * rp.B));
+      atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->walked_bytes),
+                (unsigned long long)((n_mustdo + n_sre + n_hel) * rp.B));
     }
+  }
+}
+
+// Checkpointed dense recovery round (R30), one segment pass.  The same task list
+// and records as k_spec_tma<TASKS>, but a task stops as soon as its path meets the chunk's
+// round-0 path at a checkpoint (rp.ck, written by the round-0 walk every 2^ck_shift bytes):
+// by determinism the rest of the path is the round-0 path, so end = ref_end and count =
+// (the task's count so far) + (ref_cnt - the round-0 count at the checkpoint).  A warp's
+// lanes step together, so a lane that stops early only idles; the round is therefore cut
+// into passes over byte segments [pass * seg, (pass + 1) * seg) of the chunks: pass 0 walks
+// every task of the list over the first segment, and the tasks still running at its end
+// are appended (task, code, count) to a compact list that pass 1 walks over the next
+// segment, and so on — every pass starts with full warps.  Every chain of a pass is at the
+// same byte offset, so a stage is still 8 TMA gather4 loads of one 64 B column of 32 chunks.
+// Counters: segn[p % 3] = entries appended by pass p (pass p clears segn[(p + 1) % 3], the
+// finish kernel all three).
+struct SegEntry {
+  uint32_t t, code, acc, pad;
+};
+
+template <int MODE, int S>
+__global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUtensorMap tmap, DevImage img,
+                                                     RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off,
+                                                     Ctl* ctl, uint32_t pass, uint32_t seg, SegEntry* seg_list) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  const uint32_t nwarps = blockDim.x / 32;
+  const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint8_t* table = smem_raw;
+  uint8_t* stages = smem_raw + table_off;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(stages + (size_t)nwarps * S * kStageBytes);
+  uint32_t* prow = reinterpret_cast<uint32_t*>(bars + ((nwarps * S + 1) & ~1u)) + warp * 32;
+  stage_table(img, table);
+  pdl_wait();
+  if (!__ldcg(&ctl->dense_pending)) return;  // spare slot: the run needs no dense round
+  const uint32_t B = rp.B;
+  const uint32_t x0 = pass * seg, x1 = min(B, x0 + seg);
+  if (x0 >= B) return;
+  const uint64_t ntask = __ldcg(reinterpret_cast<const unsigned long long*>(&ctl->ntask[0]));
+  const uint64_t f2 = __ldcg(reinterpret_cast<const unsigned long long*>(&ctl->fmin));
+  const uint64_t nA = __ldcg(reinterpret_cast<const unsigned long long*>(&ctl->nA));
+  const uint64_t cap = rs.cap;
+  const SegEntry* in_list = seg_list + (uint64_t)((pass + 1) & 1) * cap;  // written by pass - 1
+  SegEntry* out_list = seg_list + (uint64_t)(pass & 1) * cap;
+  const uint64_t n_in = pass == 0 ? ntask : (uint64_t)__ldcg(&ctl->segn[(pass + 2) % 3]);
+  if (blockIdx.x == 0 && threadIdx.x == 0) ctl->segn[(pass + 1) % 3] = 0;  // pass + 1's output
+  pdl_launch_dependents();
+  const uint64_t ngroups = (n_in + 31) / 32;
+  const uint64_t gw = (uint64_t)warp * gridDim.x + blockIdx.x, tw = (uint64_t)gridDim.x * nwarps;
+  if (gw >= ngroups) return;  // (no block barrier below: warps are independent)
+  if (lane == 0)
+    for (int s = 0; s < S; s++) mbar_init(bars + warp * S + s, 1);
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  __syncwarp();
+  using Sx = Step<MODE>;
+  uint8_t* wst = stages + (size_t)warp * S * kStageBytes;
+  uint64_t* wbar = bars + warp * S;
+  const uint64_t pol = evict_first_policy();
+  const uint32_t ckm = (1u << rp.ck_shift) - 1u;
+  const uint32_t segs = (x1 - x0) / kRowBytes;
+  const uint64_t my_groups = (ngroups - gw + tw - 1) / tw;
+  const uint64_t items = my_groups * segs;
+  unsigned long long n_mustdo = 0, n_sre = 0, n_hel = 0, walked = 0;
+
+  uint64_t p_group = 0;
+  uint32_t p_sg = 0, p_s = 0;
+  auto issue_next = [&]() {  // every lane of the warp (lane 0 issues)
+    if (p_sg == 0) {  // new group: its 32 chunks
+      const uint64_t idx = (gw + p_group * tw) * 32 + lane;
+      uint32_t pc = 0;
+      if (idx < n_in) {
+        const uint32_t t = pass == 0 ? (uint32_t)idx : __ldcg(&in_list[idx].t);
+        pc = __ldcg(rs.task_chunk + t);
+      }
+      __syncwarp();
+      prow[lane] = (uint32_t)min((uint64_t)pc, n_full - 1);
+      __syncwarp();
+    }
+    if (lane == 0) {
+      mbar_expect_tx(wbar + p_s, kStageBytes);
+#pragma unroll
+      for (int g = 0; g < 8; g++)
+        tma_gather4(wst + (size_t)p_s * kStageBytes + g * 4 * kRowBytes, &tmap, wbar + p_s,
+                    (int32_t)(x0 + p_sg * kRowBytes), reinterpret_cast<const uint4*>(prow)[g], pol);
+    }
+    if (++p_sg == segs) { p_sg = 0; p_group++; }
+    if (++p_s == (uint32_t)S) p_s = 0;
+  };
+  for (uint64_t it = 0; it < items && it < (uint64_t)S; it++) issue_next();
+
+  uint32_t t = 0, c = 0, st0 = 0, code = 0, acc = 0;
+  bool live = false;  // this lane's chain still walks
+  uint64_t group_i = 0;
+  uint32_t sg = 0, s = 0, phase = 0;
+  for (uint64_t it = 0; it < items; it++) {
+    if (sg == 0) {  // new group: this lane's chain
+      const uint64_t idx = (gw + group_i * tw) * 32 + lane;
+      live = false;
+      code = __ldg(img.tid2code + q0_of(rp));  // any valid code for an idle lane
+      acc = 0;
+      if (idx < n_in) {
+        if (pass == 0) {
+          t = (uint32_t)idx;
+          c = __ldcg(rs.task_chunk + t);
+          st0 = (c < n_full && c >= f2) ? __ldcg(rs.task_start + t) : kNoTask;
+          if (st0 != kNoTask) {
+            live = true;
+            code = __ldg(img.tid2code + st0);
+          }
+        } else {
+          const SegEntry e = in_list[idx];
+          t = e.t;
+          c = __ldcg(rs.task_chunk + t);
+          st0 = __ldcg(rs.task_start + t);
+          code = e.code;
+          acc = e.acc;
+          live = true;
+        }
+      }
+    }
+    mbar_wait(wbar + s, phase);
+    uint32_t k = code, a = acc;
+    const uint8_t* row = wst + (size_t)s * kStageBytes + lane * kRowBytes;
+#pragma unroll
+    for (int u = 0; u < (int)(kRowBytes / 16); u++) {
+      const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ ((lane >> 1) & 3)) << 4));  // SWIZZLE_64B
+      walk16<MODE>(img, table, q, k, a);
+    }
+    __syncwarp();
+    if (it + S < items) issue_next();  // refill this stage
+    if (live) {
+      code = k;
+      acc = a;
+      walked += kRowBytes;
+      const uint32_t pe = x0 + (sg + 1) * kRowBytes;
+      bool fin = false;
+      uint32_t e = 0, cnt = 0;
+      if (pe >= B) {
+        fin = true;
+        e = Sx::tid(img, code);
+        cnt = acc;
+      } else if ((pe & ckm) == 0) {
+        const uint2 ck = __ldcg(rp.ck + (uint64_t)((pe >> rp.ck_shift) - 1) * rp.N + c);
+        if (ck.x == code) {  // met the round-0 path: the rest of the chunk is its path
+          fin = true;
+          e = __ldcg(rs.ref_end + c);
+          cnt = acc + (__ldcg(rs.ref_cnt + c) - ck.y);
+        }
+      }
+      if (fin) {
+        live = false;
+        if (t >= nA) {  // RR / NF helper: VR^others at its precomputed ring slot
+          const uint32_t j = __ldcg(rs.task_j + t);
+          if (j + rp.vr_oth >= __ldcg(rs.hcnt + c)) {  // not evicted within its own round (R16)
+            const uint64_t o = (uint64_t)(kVrMax + (__ldcg(rs.oth_base + c) + j) % rp.vr_oth) * rs.cap + c;
+            __stcg(rs.start + o, st0);
+            __stcg(rs.end + o, e);
+            __stcg(rs.cnt + o, cnt);
+          }
+          n_hel++;
+        } else {  // A-task: VR^end, the chunk's end moves (Alg. 3 L17)
+          const uint32_t ne = __ldcg(rs.n_end + c);
+          const uint64_t o = (uint64_t)(ne % rp.vr_end) * rs.cap + c;
+          __stcg(rs.start + o, st0);
+          __stcg(rs.end + o, e);
+          __stcg(rs.cnt + o, cnt);
+          __stcg(rs.n_end + c, ne + 1);
+          __stcg(rs.x + c + 1, e);
+          __stcg(rs.cur_end + c, e);
+          if (c == f2) n_mustdo++; else n_sre++;
+        }
+      }
+    }
+    if (sg == segs - 1) {  // segment done: the chains still walking go to the next pass's list
+      const uint32_t m = __ballot_sync(0xffffffffu, live);
+      if (m) {
+        uint32_t base = 0;
+        if (lane == 0) base = atomicAdd(&ctl->segn[pass % 3], (uint32_t)__popc(m));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (live) out_list[base + __popc(m & ((1u << lane) - 1u))] = SegEntry{t, code, acc, 0u};
+      }
+    }
+    if (++sg == segs) { sg = 0; group_i++; }
+    if (++s == (uint32_t)S) { s = 0; phase ^= 1u; }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    n_mustdo += __shfl_down_sync(0xffffffffu, n_mustdo, o);
+    n_sre += __shfl_down_sync(0xffffffffu, n_sre, o);
+    n_hel += __shfl_down_sync(0xffffffffu, n_hel, o);
+    walked += __shfl_down_sync(0xffffffffu, walked, o);
+  }
+  if (lane == 0 && n_mustdo + n_sre + n_hel + walked) {
+    atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_mustdo), n_mustdo);
+    atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_sre), n_sre);
+    if (n_hel) atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->tasks_helper), n_hel);
+    atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->active_sum), n_mustdo + n_sre + n_hel);
+    atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->reread_bytes), (n_mustdo + n_sre + n_hel) * B);
+    atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->walked_bytes), walked);
   }
 }
 
@@ -597,6 +801,50 @@ cudaError_t launch_tma_m(const CUtensorMap& tm, const DevImage& img, const RunPa
   return launch_tma_s<MODE, 16, false>(tm, img, rp, rs, n_full, sms, st, 0, 0, nullptr);
 }
 
+// R30: the segment passes of a checkpointed dense round (one CTA per SM, warps chosen as
+// for the task kernel; each pass reads its list length on the device)
+template <int MODE, int S>
+cudaError_t launch_seg_t(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
+                         uint64_t n_full, int sms, cudaStream_t st, Ctl* ctl, uint32_t seg, void* seg_list) {
+  auto kern = k_task_seg<MODE, S>;
+  const uint32_t tbytes = smem_bytes_for(img);
+  const uint32_t per_warp = S * kStageBytes + S * 8 + 128;
+  const uint32_t avail = 227 * 1024 - ((tbytes + 1023) & ~1023u) - 64;
+  uint32_t w = std::min<uint32_t>(28, avail / per_warp);
+  if (const char* ev = getenv("GSPEC_CK_WARPS")) w = std::min<uint32_t>(w, (uint32_t)std::max(4, atoi(ev)));
+  if (w < 4) return cudaErrorInvalidConfiguration;
+  const uint32_t table_off = (tbytes + 1023) & ~1023u;
+  const uint32_t smem = table_off + w * S * kStageBytes + ((w * S + 1) & ~1u) * 8 + w * 128;
+  cudaError_t e = kernel_setup((const void*)kern, smem, (int)(w * 32), nullptr);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)sms);
+  cfg.blockDim = dim3(w * 32);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  const uint32_t passes = (rp.B + seg - 1) / seg;
+  for (uint32_t p = 0; p < passes; p++) {
+    e = cudaLaunchKernelEx(&cfg, kern, tm, img, rp, rs, n_full, table_off, ctl, p, seg,
+                           reinterpret_cast<SegEntry*>(seg_list));
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+
+template <int MODE>
+cudaError_t launch_seg_s(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
+                         uint64_t n_full, int sms, cudaStream_t st, Ctl* ctl, uint32_t seg, void* seg_list) {
+  const uint32_t tbytes = smem_bytes_for(img);
+  if (tbytes + 24 * (3 * kStageBytes) + 2048 + 24 * 128 <= 227 * 1024)
+    return launch_seg_t<MODE, 3>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list);
+  return launch_seg_t<MODE, 2>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list);
+}
+
 // gather = false: box {64 B, 32 chunks} (tiles of consecutive chunks);
 // gather = true: box {64 B, 1 chunk} for tile::gather4 (4 arbitrary chunks per load)
 bool encode_map(const RunParams& rp, uint64_t n_full, CUtensorMap* tm, bool gather = false) {
@@ -648,6 +896,19 @@ cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecS
   *n_done = 0;
   const uint64_t n_full = rp.len / rp.B;
   CUtensorMap tm;
+  if (rp.ck_shift && rp.ck_seg && tma_applies(rp, n_full) && encode_map(rp, n_full, &tm, true)) {  // R30
+    cudaError_t e;
+    const uint32_t sg = rp.ck_seg;
+    switch (img.mode) {
+      case MODE_U8: e = launch_seg_s<MODE_U8>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
+      case MODE_U16: e = launch_seg_s<MODE_U16>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
+      case MODE_U16H: e = launch_seg_s<MODE_U16H>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
+      case MODE_U16D: e = launch_seg_s<MODE_U16D>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
+      default: e = launch_seg_s<MODE_U32>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
+    }
+    if (e == cudaSuccess) *n_done = n_full;
+    return e;
+  }
   if (!tma_applies(rp, n_full) || !encode_map(rp, n_full, &tm, true)) return cudaErrorNotSupported;
   const uint64_t tile0 = 0, f2 = 0, ntask = n_full;  // launch-shape hints; the kernel reads the real values
   cudaError_t e;

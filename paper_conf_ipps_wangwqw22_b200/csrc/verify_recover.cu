@@ -1009,6 +1009,7 @@ __global__ void __launch_bounds__(256) k_dense_finish(DevImage img, RunParams rp
   __shared__ uint32_t nh;
   __shared__ uint32_t hslot[64];
   if (!ctl->dense_pending) return;  // no dense round was handed over (spare slot)
+  if (threadIdx.x == 0) ctl->segn[0] = ctl->segn[1] = ctl->segn[2] = 0;  // R30 pass lists, for the next round
   const uint64_t f2 = ctl->fmin;
   const uint64_t ntask = ctl->ntask[0], nA = ctl->nA;
   if (threadIdx.x == 0) {

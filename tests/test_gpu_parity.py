@@ -783,3 +783,59 @@ def test_memoized_helpers_match_eager(gs, name, length, B, scheme):
     assert out.returncode == 0, out.stderr[-2000:]
     fin, cnt, th, hw = json.loads(out.stdout.strip().splitlines()[-1])
     assert (fin, cnt, th) == (res.final_state, res.accept_count, res.stats["tasks_helper"]) and hw <= th
+
+
+@pytest.mark.parametrize("name,length,B,scheme,ck", [
+    ("c3", 32 << 20, 8192, "sre", None), ("c3", (24 << 20) + 1000, 4096, "sre", "64"),
+    ("c3s", 96 << 20, 8192, "nf", None), ("c3", 32 << 20, 8192, "rr", "2048"), ("c3", 16 << 20, 4096, "nf", "4096"),
+    ("c3", 48 << 20, 16384, "sre", "0")])
+def test_checkpointed_dense_rounds(gs, name, length, B, scheme, ck):
+    """R30: dense-round tasks stop where their path meets the chunk's round-0 path at a
+    checkpoint (every GSPEC_CK bytes of the round-0 walk, default 512; 0 = off).  Results,
+    records and round counters equal the oracle's for every interval (the interval is read
+    once per process: non-default ones run in a child process); with checkpoints the task
+    kernel walks far fewer bytes than the tasks' nominal chunk bytes (C3: the counter part
+    of the state converges at the chunk's reset byte)."""
+    import json
+    import os
+    import subprocess
+    import sys
+
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme=scheme)
+    keys = ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes", "verify_checks", "verify_matches")
+    if ck is None:  # the default interval, in this process
+        fsm = gs.FSM.load(w.table, w.start, w.accept)
+        x = torch.from_numpy(data).cuda()
+        for _ in range(2):  # the second run has the dense-round slots the first one sized
+            res = fsm.run(x, scheme=scheme, chunk_bytes=B)
+            check_equal(res, ref, B, w.nstates)
+            for k in keys:
+                assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+        assert res.stats["tasks_sre"] > 1024
+        walked = res.stats["task_walked_bytes"]
+        assert 0 < walked < 0.75 * res.stats["reread_bytes"], (walked, res.stats["reread_bytes"])
+        return
+    code = ("import sys, json, torch, numpy as np; sys.path.insert(0, '.'); import gen, paper_conf_ipps_wangwqw22_b200 as gs;"
+            f"w = gen.workload({name!r}, length={length}); x = torch.empty({length}, dtype=torch.uint8, device='cuda');"
+            "w.device(x); f = gs.FSM.load(w.table, w.start, w.accept);"
+            f"r = [f.run(x, scheme={scheme!r}, chunk_bytes={B}) for _ in range(2)][-1];"
+            "ce = r.chunk_ends.cpu().numpy().view(np.uint32);"
+            "print(json.dumps([r.final_state, r.accept_count, int(ce.astype(np.uint64).sum()), int(ce[::97].astype(np.uint64).sum()),"
+            f" r.stats, {length}]))")
+    env = dict(os.environ, GSPEC_CK=ck)
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, env=env, cwd=root, timeout=600)
+    assert out.returncode == 0, out.stderr[-2000:]
+    fin, cnt, s_all, s_97, stats, _ = json.loads(out.stdout.strip().splitlines()[-1])
+    rce = ref["chunk_end"].astype(np.uint64)
+    assert (fin, cnt) == (ref["final"], ref["count"])
+    assert (s_all, s_97) == (int(rce.sum()), int(rce[::97].sum()))
+    for k in keys:
+        assert stats[k] == sim[k], (k, stats[k], sim[k])
+    if int(ck) == 0 or B < 2 * int(ck):  # off (or no checkpoint inside a chunk): whole chunks
+        assert 0 < stats["task_walked_bytes"] <= stats["reread_bytes"]
+        assert stats["task_walked_bytes"] % B == 0
+    else:
+        assert 0 < stats["task_walked_bytes"] < stats["reread_bytes"]
