@@ -425,7 +425,7 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
     {
       const uint32_t sh = ck_shift_default();
       if (rp.dense && rp.k == 1 && sh && !spec_path_generic_only() && o.B % (1u << sh) == 0 &&
-          o.B >= (2u << sh)) {
+          o.B >= (2u << sh) && f->conv_hint > 0.0) {
         const size_t nck = (size_t)(o.B / (1u << sh) - 1) * N * sizeof(uint2);
         const size_t need = ((nck + 255) & ~(size_t)255) + 2 * f->rs.cap * 16;  // + the passes' chain lists
         if (f->ck_bytes < need) {
@@ -1353,6 +1353,7 @@ int fsm_select_scheme(fsm_t f, const uint8_t* d_sample, uint64_t len, const fsm_
   }
   const fsm_scheme pick = tree_select(ft, f->n);
   if (N > 1) f->acc1_hint = ft.acc1;
+  if (nwin > 0) f->conv_hint = ft.conv16k;  // R30: no window converged within 16 KiB -> no checkpoints
   f->auto_scheme = pick;
   f->auto_selected = true;
   *outp = pick;

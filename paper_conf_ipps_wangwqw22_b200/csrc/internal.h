@@ -489,6 +489,7 @@ struct fsm_s {
   int device = 0;
   fsm_scheme auto_scheme = FSM_SCHEME_SRE;
   double acc1_hint = 0.0;            // spec-1 accuracy from the selector's profile (dense-round gate)
+  double conv_hint = 1.0;            // profile's fraction of windows converged within 16 KiB (R30 gate; 1 = unknown)
   uint32_t dense_hint = 4;           // task-kernel slots queued per dense run (dense rounds last seen)
   bool shard_prefer_exact = false;   // a speculative shard map was invalid once: use the exact map
   uint32_t* enum_ticket = nullptr;   // single-launch ENUM: finished-CTA counter (zeroed once)
