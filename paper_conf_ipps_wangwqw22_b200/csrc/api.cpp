@@ -585,30 +585,71 @@ bool plan_delta_rows(fsm_t f, const std::vector<uint32_t>& ttc, uint32_t nt, uin
     const uint64_t want = strtoull(e, nullptr, 10);
     if (want > H) H = std::min<uint64_t>(want, hmax);
   }
-  // codes: hot t -> t*C, poison -> H*C (stored as hot row H), cold t -> HC1 + (t - H)
-  const uint64_t HC1 = (H + 1) * C;
-  std::vector<uint32_t> code(nt);
+  // One-exception plan (the step drops a compare and a select): the smallest H1 >= H such that
+  // the rows needing two exceptions against [0, H1) — X — can be hot too (slots H1+1..), within
+  // the budget and the code limits.  GSPEC_DELTA_EXC=2 keeps the two-exception plan (A/B).
+  std::vector<uint32_t> X;
+  uint32_t exc = kDeltaExc;
+  {
+    const char* e = getenv("GSPEC_DELTA_EXC");
+    if (!(e && atoi(e) == 2)) {
+      for (uint64_t h1 = H; h1 <= hmax; h1++) {
+        std::vector<uint32_t> x;
+        bool ok = true;
+        for (uint64_t t = h1; t < nr && ok; t++) {
+          const uint32_t* ft = &first[t * (kDeltaExc + 1)];
+          if (!(ft[0] < h1 || ft[1] < h1)) x.push_back((uint32_t)t);
+          ok = h1 + x.size() <= hmax;
+        }
+        const uint64_t hot = h1 + 1 + x.size(), ncold = nr - h1 - x.size();
+        if (!ok || hot * C + ncold > 0x7FFFu || 2 * hot * C + kDeltaBaseMax > 0xFFFFu) continue;
+        const uint64_t bytes1 = ((hot * C * 2 + 255) & ~255ull) + 256 + ncold * 8;
+        if (bytes1 > budget) continue;
+        H = h1;
+        X = std::move(x);
+        exc = 1;
+        break;
+      }
+    }
+  }
+  // codes: hot t -> slot*C (top-H tids: slot t; poison: slot H, stored as hot row H; the X tids:
+  // slots H+1..), cold t -> HC1 + its rank among the cold tids
+  const uint64_t HC1 = (H + 1 + X.size()) * C;
+  std::vector<uint32_t> slot(nt, 0xFFFFFFFFu);
+  for (uint32_t t = 0; t < H; t++) slot[t] = t;
+  slot[nr] = (uint32_t)H;
+  for (size_t i = 0; i < X.size(); i++) slot[X[i]] = (uint32_t)(H + 1 + i);
+  std::vector<uint32_t> code(nt), cold;
   for (uint32_t t = 0; t < nt; t++) {
     const uint32_t a = tid2code[t] >> 15;  // accept flag of the plain u16 code
-    const uint64_t c = t < H ? (uint64_t)t * C : t == nr ? H * C : HC1 + (t - H);
+    uint64_t c;
+    if (slot[t] != 0xFFFFFFFFu) {
+      c = (uint64_t)slot[t] * C;
+    } else {
+      c = HC1 + cold.size();
+      cold.push_back(t);
+    }
     code[t] = (uint32_t)c | (a << 15);
   }
   const uint64_t hot_b = HC1 * 2;
   const uint64_t cls_off = (hot_b + 255) & ~255ull;
   const uint64_t delta_off = cls_off + 256;
-  const uint64_t bytes = (delta_off + (uint64_t)(nr - H) * 8 + 15) & ~15ull;
+  const uint64_t bytes = (delta_off + (uint64_t)cold.size() * 8 + 15) & ~15ull;
   if (bytes > budget) return false;
   std::vector<uint16_t> im(bytes / 2, 0);
   for (uint64_t t = 0; t < H; t++)
     for (uint32_t c = 0; c < C; c++) im[t * C + c] = (uint16_t)code[ttc[t * C + c]];
   for (uint32_t c = 0; c < C; c++) im[H * C + c] = (uint16_t)code[nr];
+  for (size_t i = 0; i < X.size(); i++)
+    for (uint32_t c = 0; c < C; c++) im[(H + 1 + i) * C + c] = (uint16_t)code[ttc[(uint64_t)X[i] * C + c]];
   uint8_t* cm = reinterpret_cast<uint8_t*>(im.data()) + cls_off;
   for (uint32_t b = 0; b < 256; b++) cm[b] = (uint8_t)(2 * f->cls[b]);
   uint2* dl = reinterpret_cast<uint2*>(reinterpret_cast<uint8_t*>(im.data()) + delta_off);
-  for (uint32_t t = (uint32_t)H; t < nr; t++) {
+  for (size_t ci = 0; ci < cold.size(); ci++) {
+    const uint32_t t = cold[ci];
     const uint32_t* ft = &first[(uint64_t)t * (kDeltaExc + 1)];
     uint32_t j = kNo;
-    for (uint32_t e = 0; e <= kDeltaExc && j == kNo; e++)
+    for (uint32_t e = 0; e <= exc && j == kNo; e++)
       if (ft[e] < H) j = ft[e];
     if (j == kNo) return false;  // unreachable (checked above)
     uint32_t ex[kDeltaExc] = {0xFF, 0xFF}, ec[kDeltaExc] = {0, 0}, k = 0;
@@ -618,14 +659,15 @@ bool plan_delta_rows(fsm_t f, const std::vector<uint32_t>& ttc, uint32_t nt, uin
         ec[k] = code[ttc[(uint64_t)t * C + c]];
         k++;
       }
-    dl[t - H] = make_uint2((uint32_t)(2 * C * j) << 16 | ex[1] << 8 | ex[0], (ec[0] & 0xFFFFu) | (ec[1] << 16));
+    dl[ci] = make_uint2((uint32_t)(2 * C * j) << 16 | ex[1] << 8 | ex[0], (ec[0] & 0xFFFFu) | (ec[1] << 16));
   }
   out->assign(reinterpret_cast<const uint2*>(im.data()), reinterpret_cast<const uint2*>(im.data()) + bytes / 8);
   tid2code = code;
   code2tid.assign(0x8000, nr);
   for (uint32_t t = 0; t < nt; t++) code2tid[code[t] & 0x7FFFu] = t;
   img->H = (uint32_t)H;
-  img->D = nr - (uint32_t)H;
+  img->D = (uint32_t)cold.size();
+  img->delta_exc = exc;
   img->HC1 = (uint32_t)HC1;
   img->cls_off = (uint32_t)cls_off;
   img->delta_off = (uint32_t)delta_off;
@@ -1377,7 +1419,7 @@ int fsm_get_transform(fsm_t f, uint32_t* perm, uint32_t* inv, uint64_t* freq, ui
   if (inv) std::copy(f->inv.begin(), f->inv.end(), inv);
   if (freq) std::copy(f->freq.begin(), f->freq.end(), freq);
   if (mode) *mode = f->img.mode == MODE_U16H ? (uint32_t)MODE_U16 : f->img.mode == MODE_U16D ? 4u : f->img.mode;
-  if (hot_rows) *hot_rows = f->img.H;
+  if (hot_rows) *hot_rows = f->img.mode == MODE_U16D ? f->img.HC1 / f->img.C - 1 : f->img.H;  // full real rows
   if (nclasses) *nclasses = f->img.C;
   return FSM_OK;
 }

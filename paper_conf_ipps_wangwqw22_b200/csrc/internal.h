@@ -25,6 +25,7 @@ enum Mode : uint32_t {
 };
 
 constexpr uint32_t kDeltaExc = 2;        // exceptions per delta row
+constexpr int MODE_U16D1 = 6;  // template-only: MODE_U16D image with delta_exc == 1 (the walk kernels' step)
 constexpr uint32_t kInvalidMap = 0xFFFFFFFEu;  // map entry of a speculative shard map that must be redone
 constexpr uint32_t kErrorMap = 0xFFFFFFFDu;    // map of a rank whose fsm_shard_map failed (count[0] = -status)
 constexpr uint32_t kPendEnd = 0xFFFFFFFCu;     // end of a memoized helper record not walked yet (R28)
@@ -75,7 +76,11 @@ struct DevImage {
   uint32_t delta_off;         // byte offset of the delta rows (16-aligned)
   uint32_t D;                 // delta rows (cold real tids)
   uint32_t cls_off;           // byte offset of the doubled class map (256-aligned)
-  uint32_t HC1;               // (H + 1) * C: the first cold code
+  uint32_t HC1;               // (H + 1) * C (+ X * C): the first cold code
+  // 1 when every delta row has at most one exception (e1 = 0xFF, y = code0): the hot set is then
+  // the top-H tids plus the X tids that need two (hot slots H+1.., after the poison row), and the
+  // walk kernels use the one-exception step; 2 otherwise
+  uint32_t delta_exc;
 };
 
 // Global record store (hierarchical store, level 3).

@@ -76,15 +76,19 @@ __device__ __forceinline__ uint32_t lit_excl_scan(uint32_t v, uint32_t* wsum, ui
 //   QS_c = lookback-2 ranking (qs_cap), dequeues start at entry 1 (round 0 ran the front,
 //   R9).  Records are pushed to VR_cid in tid order (helpers, then the chunk's own thread);
 //   a thread tid >= fr with found == false takes its new end (L28-29).
+__host__ __device__ inline uint32_t lit_arrays_off(const DevImage& img) { return (smem_bytes_for(img) + 15u) & ~15u; }
+
 template <int MODE>
 __global__ void __launch_bounds__(kLitMax) k_literal(DevImage img, RunParams rp, RecStore rs, Ctl* ctl,
                                                     uint32_t* __restrict__ chunk_ends) {
   extern __shared__ __align__(1024) uint8_t smem[];
-  __shared__ uint32_t endc_sh[kLitMax];
-  __shared__ uint32_t pair_sh[kLitMax];    // QS_c = qs2[pair_sh[c]] (chunk 0: [q0])
-  __shared__ uint32_t cur_sh[kLitMax];     // QS_c dequeue cursor
-  __shared__ uint32_t pre_sh[kLitMax];     // NF: exclusive prefix of the remaining entries
-  __shared__ uint32_t take_sh[kLitMax];    // entries of QS_c dequeued by helpers this iteration
+  // the per-chunk arrays live in dynamic shared memory behind the table: the table must start
+  // near the shared window's base (a delta-row image holds absolute 16-bit row offsets)
+  uint32_t* endc_sh = reinterpret_cast<uint32_t*>(smem + lit_arrays_off(img));
+  uint32_t* pair_sh = endc_sh + kLitMax;   // QS_c = qs2[pair_sh[c]] (chunk 0: [q0])
+  uint32_t* cur_sh = pair_sh + kLitMax;    // QS_c dequeue cursor
+  uint32_t* pre_sh = cur_sh + kLitMax;     // NF: exclusive prefix of the remaining entries
+  uint32_t* take_sh = pre_sh + kLitMax;    // entries of QS_c dequeued by helpers this iteration
   __shared__ uint32_t wsum[32];
   __shared__ int mark;
   __shared__ unsigned long long red[kLitMax / 32][6];
@@ -250,7 +254,7 @@ template <int MODE>
 cudaError_t launch_lit(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, uint32_t* ce,
                        cudaStream_t st) {
   auto kern = k_literal<MODE>;
-  const uint32_t smem = smem_bytes_for(img);
+  const uint32_t smem = lit_arrays_off(img) + 5 * kLitMax * 4;
   cudaError_t e = kernel_setup((const void*)kern, smem, kLitMax, nullptr);
   if (e != cudaSuccess) return e;
   const uint32_t threads = (uint32_t)((rp.N + 31) / 32 * 32);

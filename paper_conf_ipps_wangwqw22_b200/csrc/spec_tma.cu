@@ -881,7 +881,10 @@ cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecS
     case MODE_U8: e = launch_tma_m<MODE_U8>(tm, img, rp, rs, n_full, sms, st); break;
     case MODE_U16: e = launch_tma_m<MODE_U16>(tm, img, rp, rs, n_full, sms, st); break;
     case MODE_U16H: e = launch_tma_m<MODE_U16H>(tm, img, rp, rs, n_full, sms, st); break;
-    case MODE_U16D: e = launch_tma_m<MODE_U16D>(tm, img, rp, rs, n_full, sms, st); break;
+    case MODE_U16D:
+      e = img.delta_exc == 1 ? launch_tma_m<MODE_U16D1>(tm, img, rp, rs, n_full, sms, st)
+                             : launch_tma_m<MODE_U16D>(tm, img, rp, rs, n_full, sms, st);
+      break;
     default: e = launch_tma_m<MODE_U32>(tm, img, rp, rs, n_full, sms, st); break;
   }
   if (e == cudaSuccess) *n_done = n_full;
@@ -903,7 +906,10 @@ cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecS
       case MODE_U8: e = launch_seg_s<MODE_U8>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
       case MODE_U16: e = launch_seg_s<MODE_U16>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
       case MODE_U16H: e = launch_seg_s<MODE_U16H>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
-      case MODE_U16D: e = launch_seg_s<MODE_U16D>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
+      case MODE_U16D:
+        e = img.delta_exc == 1 ? launch_seg_s<MODE_U16D1>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list)
+                               : launch_seg_s<MODE_U16D>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list);
+        break;
       default: e = launch_seg_s<MODE_U32>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
     }
     if (e == cudaSuccess) *n_done = n_full;
@@ -916,7 +922,10 @@ cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecS
     case MODE_U8: e = launch_tma_s<MODE_U8, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
     case MODE_U16: e = launch_tma_s<MODE_U16, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
     case MODE_U16H: e = launch_tma_s<MODE_U16H, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
-    case MODE_U16D: e = launch_tma_s<MODE_U16D, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
+    case MODE_U16D:
+      e = img.delta_exc == 1 ? launch_tma_s<MODE_U16D1, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask)
+                             : launch_tma_s<MODE_U16D, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask);
+      break;
     default: e = launch_tma_s<MODE_U32, 1, true>(tm, img, rp, rs, n_full, sms, st, tile0, f2, ctl, ntask); break;
   }
   if (e == cudaSuccess) *n_done = n_full;

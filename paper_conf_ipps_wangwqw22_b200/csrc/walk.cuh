@@ -158,7 +158,12 @@ __device__ __forceinline__ uint2 lds_u64(uint32_t saddr) {
 // trip, no divergence, and no multiply by C on the path (the class map holds 2*class).
 // The step is ALU-pipe-bound on C4 (math_pipe_throttle): this form needs ~10 ALU-pipe
 // and ~3 FMA-pipe instructions per symbol.
-struct StepDelta {
+// EXC = 1 (img.delta_exc == 1, template mode MODE_U16D1): every delta row has one exception
+// (y = its code), so the step drops the second compare and select: ~8 instead of ~10
+// ALU-pipe instructions per symbol.  The EXC = 2 reader also reads EXC = 1 images (e1 = 0xFF
+// never matches an even 2*class), so kernels off the hot path keep Step<MODE_U16D>.
+template <int EXC>
+struct StepDeltaT {
   static constexpr uint32_t kShift = 15;
   static __device__ __forceinline__ uint32_t row(const DevImage& img, uint32_t base, uint32_t code, uint32_t cl2) {
     const uint32_t c = code & 0x7FFFu;
@@ -170,9 +175,13 @@ struct StepDelta {
         : "+r"(dx), "+r"(dy)
         : "r"(c), "r"(img.HC1), "r"(da));
     uint32_t v = lds_u16((dx >> 16) + cl2);
-    const uint32_t x = dx ^ (cl2 * 0x101u);
-    v = (x & 0xFFu) == 0 ? (dy & 0xFFFFu) : v;
-    v = (x & 0xFF00u) == 0 ? (dy >> 16) : v;
+    if constexpr (EXC == 1) {
+      v = ((dx ^ cl2) & 0xFFu) == 0 ? dy : v;
+    } else {
+      const uint32_t x = dx ^ (cl2 * 0x101u);
+      v = (x & 0xFFu) == 0 ? (dy & 0xFFFFu) : v;
+      v = (x & 0xFF00u) == 0 ? (dy >> 16) : v;
+    }
     return v;
   }
   static __device__ __forceinline__ uint32_t byte(const DevImage& img, const uint8_t* s, uint32_t code, uint32_t b) {
@@ -200,7 +209,9 @@ struct StepDelta {
 template <>
 struct Step<MODE_U16> : StepClassed<uint16_t, 15, false> {};
 template <>
-struct Step<MODE_U16D> : StepDelta {};
+struct Step<MODE_U16D> : StepDeltaT<2> {};
+template <>
+struct Step<MODE_U16D1> : StepDeltaT<1> {};
 // MODE_U16H: every row in shared memory, pre-multiplied codes (code = 2*t*C | accept: the
 // row's byte offset with the accept flag in bit 0) and a doubled class map, so the entry
 // address is code - (code & 1) + (base + 256 + 2*class): LOP3 + IADD3 on the dependent chain.
@@ -259,12 +270,16 @@ __device__ __forceinline__ void walk16(const DevImage& img, const uint8_t* s, co
                                        uint32_t& acc) {
   using S = Step<MODE>;
   const uint32_t w[4] = {q.x, q.y, q.z, q.w};
-  uint32_t cl[16];
-  cls_words<MODE, 4>(img, s, w, cl);
 #pragma unroll
-  for (int i = 0; i < 16; i++) {
-    code = S::next(img, s, code, cl[i]);
-    acc += S::acc(code);
+  for (int t = 0; t < 4; t++) {  // a word's 4 class lookups at a time (register pressure at 72)
+    const uint32_t u[1] = {w[t]};
+    uint32_t cl[4];
+    cls_words<MODE, 1>(img, s, u, cl);
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+      code = S::next(img, s, code, cl[i]);
+      acc += S::acc(code);
+    }
   }
 }
 
