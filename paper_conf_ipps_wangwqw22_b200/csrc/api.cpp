@@ -479,7 +479,8 @@ int run_enqueue(fsm_t f, const uint8_t* d_in, uint64_t len, const Opts& o, fsm_s
       rp.dense_slots = slots - 1 - r;
       CUDA_TRY(launch_verify_recover(f->img, rp, f->rs, f->d_ctl, f->d_block_tmp, d_chunk_ends, o.st, f->sm_count));
       // task kernel (R30: one launch per segment pass) + finish + verify (no-ops once the run is complete)
-      pd.launches += 2 + (rp.ck_shift && rp.ck_seg ? (o.B + rp.ck_seg - 1) / rp.ck_seg : 1u);
+      const bool seg = rp.ck_shift && rp.ck_seg;  // (no tail chunk: the last pass commits, no finish kernel)
+      pd.launches += (seg && len % o.B == 0 ? 1u : 2u) + (seg ? (o.B + rp.ck_seg - 1) / rp.ck_seg : 1u);
     }
     pd.dense_slots = slots;
     pd.dense = rp.dense != 0;

@@ -67,9 +67,10 @@ struct DevImage {
   const uint32_t* inv;        // [nt] tid -> original id (poison -> n)
   const uint8_t* acc;         // [nt] accept by tid
   // MODE_U16D: the whole shared-memory table image
-  //   [hot rows 0..H-1][poison row (= row H)][pad to 256][class map: 2*class, 256 B][delta rows]
-  // Codes are pre-multiplied: hot tid t -> t*C, poison -> H*C, cold tid t -> HC1 + (t - H),
-  // accept flag in bit 15.  Delta row of a cold tid: x = (2*C*base tid) << 16 | e1 << 8 | e0
+  //   [hot rows 0..H-1][poison row (= row H)][rows of the X tids][pad to 256][class map: 2*class,
+  //   256 B][delta rows]
+  // Codes are pre-multiplied: hot tid t < H -> t*C, poison -> H*C, X tid -> its slot*C (H+1..),
+  // cold tid -> HC1 + its rank among the cold tids, accept flag in bit 15.  Delta row of a cold tid: x = (2*C*base tid) << 16 | e1 << 8 | e0
   // (e = 2*exception class, 0xFF = none; the row offset is made absolute at staging),
   // y = code0 | code1 << 16.
   const uint2* Dl;
@@ -154,7 +155,7 @@ struct Ctl {
   uint64_t helper_walks;  // RR / NF helper records actually walked (memoized helpers, R28)
   uint64_t walked_bytes;  // bytes the dense-round task kernels actually walked (R30 early exit)
   uint32_t segn[3];       // checkpointed dense round: chains appended by pass p in segn[p % 3] (R30)
-  uint32_t pad3;
+  uint32_t seg_done;      // R30 last pass: warps done (the last one commits the round; reset by it)
 };
 
 struct RunParams {

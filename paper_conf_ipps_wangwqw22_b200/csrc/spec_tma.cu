@@ -537,7 +537,8 @@ struct SegEntry {
 template <int MODE, int S>
 __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUtensorMap tmap, DevImage img,
                                                      RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off,
-                                                     Ctl* ctl, uint32_t pass, uint32_t seg, SegEntry* seg_list) {
+                                                     Ctl* ctl, uint32_t pass, uint32_t seg, SegEntry* seg_list,
+                                                     uint32_t commit) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   const uint32_t nwarps = blockDim.x / 32;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -562,7 +563,8 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
   pdl_launch_dependents();
   const uint64_t ngroups = (n_in + 31) / 32;
   const uint64_t gw = (uint64_t)warp * gridDim.x + blockIdx.x, tw = (uint64_t)gridDim.x * nwarps;
-  if (gw >= ngroups) return;  // (no block barrier below: warps are independent)
+  // (no block barrier below: warps are independent; a warp without a group walks nothing but
+  // still takes its commit ticket)
   if (lane == 0)
     for (int s = 0; s < S; s++) mbar_init(bars + warp * S + s, 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -574,7 +576,7 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
   const uint64_t pol = evict_first_policy();
   const uint32_t ckm = (1u << rp.ck_shift) - 1u;
   const uint32_t segs = (x1 - x0) / kRowBytes;
-  const uint64_t my_groups = (ngroups - gw + tw - 1) / tw;
+  const uint64_t my_groups = gw < ngroups ? (ngroups - gw + tw - 1) / tw : 0;
   const uint64_t items = my_groups * segs;
   unsigned long long n_mustdo = 0, n_sre = 0, n_hel = 0, walked = 0;
 
@@ -714,6 +716,27 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
     atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->reread_bytes), (n_mustdo + n_sre + n_hel) * B);
     atomicAdd(reinterpret_cast<unsigned long long*>(&ctl->walked_bytes), walked);
   }
+  if (commit) {  // last pass, no tail chunk: the last warp commits the round (the finish kernel's job)
+    uint32_t last = 0;
+    if (lane == 0) {
+      __threadfence();
+      last = atomicAdd(&ctl->seg_done, 1u) == gridDim.x * nwarps - 1;
+    }
+    if (__shfl_sync(0xffffffffu, last, 0) && lane == 0) {
+      __threadfence();
+      ctl->segn[0] = ctl->segn[1] = ctl->segn[2] = 0;
+      ctl->rounds++;
+      ctl->dense_rounds++;
+      ctl->f = f2;
+      ctl->tf = __ldcg(rs.x + f2);
+      ctl->changed[0] = 0;  // the verify launch behind us starts its passes at slot 0
+      ctl->it_fm[0] = rp.N;
+      ctl->it_checks[0] = ctl->it_matches[0] = ctl->it_ntask[0] = ctl->it_reread[0] = 0;
+      ctl->seg_done = 0;
+      __threadfence();
+      ctl->dense_pending = 0;
+    }
+  }
 }
 
 using EncodeFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
@@ -805,7 +828,8 @@ cudaError_t launch_tma_m(const CUtensorMap& tm, const DevImage& img, const RunPa
 // for the task kernel; each pass reads its list length on the device)
 template <int MODE, int S>
 cudaError_t launch_seg_t(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
-                         uint64_t n_full, int sms, cudaStream_t st, Ctl* ctl, uint32_t seg, void* seg_list) {
+                         uint64_t n_full, int sms, cudaStream_t st, Ctl* ctl, uint32_t seg, void* seg_list,
+                         bool commit_last) {
   auto kern = k_task_seg<MODE, S>;
   const uint32_t tbytes = smem_bytes_for(img);
   const uint32_t per_warp = S * kStageBytes + S * 8 + 128;
@@ -830,7 +854,7 @@ cudaError_t launch_seg_t(const CUtensorMap& tm, const DevImage& img, const RunPa
   const uint32_t passes = (rp.B + seg - 1) / seg;
   for (uint32_t p = 0; p < passes; p++) {
     e = cudaLaunchKernelEx(&cfg, kern, tm, img, rp, rs, n_full, table_off, ctl, p, seg,
-                           reinterpret_cast<SegEntry*>(seg_list));
+                           reinterpret_cast<SegEntry*>(seg_list), (uint32_t)(commit_last && p + 1 == passes));
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;
@@ -838,11 +862,12 @@ cudaError_t launch_seg_t(const CUtensorMap& tm, const DevImage& img, const RunPa
 
 template <int MODE>
 cudaError_t launch_seg_s(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
-                         uint64_t n_full, int sms, cudaStream_t st, Ctl* ctl, uint32_t seg, void* seg_list) {
+                         uint64_t n_full, int sms, cudaStream_t st, Ctl* ctl, uint32_t seg, void* seg_list,
+                         bool commit_last) {
   const uint32_t tbytes = smem_bytes_for(img);
   if (tbytes + 24 * (3 * kStageBytes) + 2048 + 24 * 128 <= 227 * 1024)
-    return launch_seg_t<MODE, 3>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list);
-  return launch_seg_t<MODE, 2>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list);
+    return launch_seg_t<MODE, 3>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list, commit_last);
+  return launch_seg_t<MODE, 2>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list, commit_last);
 }
 
 // gather = false: box {64 B, 32 chunks} (tiles of consecutive chunks);
@@ -895,22 +920,25 @@ cudaError_t launch_spec_tma(const DevImage& img, const RunParams& rp, const RecS
 // chunks < n_full are walked here; the tail chunk (if its task is listed) is left to the
 // finish kernel.  Launched with the grid of a full list (one CTA per SM, persistent).
 cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, int sms,
-                            cudaStream_t st, uint64_t* n_done) {
+                            cudaStream_t st, uint64_t* n_done, bool* committed) {
   *n_done = 0;
+  if (committed) *committed = false;
   const uint64_t n_full = rp.len / rp.B;
   CUtensorMap tm;
   if (rp.ck_shift && rp.ck_seg && tma_applies(rp, n_full) && encode_map(rp, n_full, &tm, true)) {  // R30
     cudaError_t e;
     const uint32_t sg = rp.ck_seg;
+    const bool cm = n_full == rp.N;  // no tail chunk: the last pass commits, no finish kernel
+    if (committed) *committed = cm;
     switch (img.mode) {
-      case MODE_U8: e = launch_seg_s<MODE_U8>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
-      case MODE_U16: e = launch_seg_s<MODE_U16>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
-      case MODE_U16H: e = launch_seg_s<MODE_U16H>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
+      case MODE_U8: e = launch_seg_s<MODE_U8>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
+      case MODE_U16: e = launch_seg_s<MODE_U16>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
+      case MODE_U16H: e = launch_seg_s<MODE_U16H>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
       case MODE_U16D:
-        e = img.delta_exc == 1 ? launch_seg_s<MODE_U16D1>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list)
-                               : launch_seg_s<MODE_U16D>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list);
+        e = img.delta_exc == 1 ? launch_seg_s<MODE_U16D1>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm)
+                               : launch_seg_s<MODE_U16D>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm);
         break;
-      default: e = launch_seg_s<MODE_U32>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list); break;
+      default: e = launch_seg_s<MODE_U32>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
     }
     if (e == cudaSuccess) *n_done = n_full;
     return e;

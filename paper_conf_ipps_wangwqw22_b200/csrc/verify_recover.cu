@@ -1094,20 +1094,22 @@ cudaError_t launch_dense_finish(const DevImage& img, const RunParams& rp, const 
 }  // namespace
 
 cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecStore& rs, Ctl* ctl, int sms,
-                            cudaStream_t st, uint64_t* n_done);
+                            cudaStream_t st, uint64_t* n_done, bool* committed);
 
 cudaError_t launch_task_dense(const DevImage& img, const RunParams& rp_in, const RecStore& rs, Ctl* ctl, int sms,
                               cudaStream_t st) {
   RunParams rp = rp_in;
   rp.ctl_init = nullptr;  // the control block is live: never re-initialise it mid-run
   uint64_t done = 0;
-  cudaError_t e = launch_task_tma(img, rp, rs, ctl, sms, st, &done);
+  bool committed = false;
+  cudaError_t e = launch_task_tma(img, rp, rs, ctl, sms, st, &done, &committed);
   if (e == cudaErrorNotSupported) {
     cudaGetLastError();
     done = 0;  // the finish kernel walks everything (slow, but exact)
   } else if (e != cudaSuccess) {
     return e;
   }
+  if (committed) return cudaSuccess;  // R30: the last segment pass committed the round
   switch (img.mode) {
     case MODE_U8: return launch_dense_finish<MODE_U8>(img, rp, rs, ctl, done, st);
     case MODE_U16: return launch_dense_finish<MODE_U16>(img, rp, rs, ctl, done, st);
