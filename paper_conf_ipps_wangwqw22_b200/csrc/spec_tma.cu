@@ -559,6 +559,7 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
   const SegEntry* in_list = seg_list + (uint64_t)((pass + 1) & 1) * cap;  // written by pass - 1
   SegEntry* out_list = seg_list + (uint64_t)(pass & 1) * cap;
   const uint64_t n_in = pass == 0 ? ntask : (uint64_t)__ldcg(&ctl->segn[(pass + 2) % 3]);
+  if (n_in > cap) __trap();
   if (blockIdx.x == 0 && threadIdx.x == 0) ctl->segn[(pass + 1) % 3] = 0;  // pass + 1's output
   pdl_launch_dependents();
   const uint64_t ngroups = (n_in + 31) / 32;
@@ -630,6 +631,8 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
           t = e.t;
           c = __ldcg(rs.task_chunk + t);
           st0 = __ldcg(rs.task_start + t);
+          // guards (compute-sanitizer is unavailable on the GPU pool; a violated bound traps)
+          if (idx >= cap || t >= ntask || c < f2 || c >= n_full) __trap();
           code = e.code;
           acc = e.acc;
           live = true;
@@ -695,7 +698,11 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
         uint32_t base = 0;
         if (lane == 0) base = atomicAdd(&ctl->segn[pass % 3], (uint32_t)__popc(m));
         base = __shfl_sync(0xffffffffu, base, 0);
-        if (live) out_list[base + __popc(m & ((1u << lane) - 1u))] = SegEntry{t, code, acc, 0u};
+        if (live) {
+          const uint32_t o = base + __popc(m & ((1u << lane) - 1u));
+          if (o >= n_in || o >= cap) __trap();  // a pass never appends more chains than it read
+          out_list[o] = SegEntry{t, code, acc, 0u};
+        }
       }
     }
     if (++sg == segs) { sg = 0; group_i++; }
