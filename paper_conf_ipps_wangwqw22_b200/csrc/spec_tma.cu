@@ -534,17 +534,20 @@ struct SegEntry {
   uint32_t t, code, acc, pad;
 };
 
-template <int MODE, int S>
+// RB: bytes of a chunk per stage (64: SWIZZLE_64B boxes; 128: SWIZZLE_128B, half the TMA
+// issue work per byte — 8 gather4 loads per stage either way)
+template <int MODE, int S, int RB>
 __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUtensorMap tmap, DevImage img,
                                                      RunParams rp, RecStore rs, uint64_t n_full, uint32_t table_off,
                                                      Ctl* ctl, uint32_t pass, uint32_t seg, SegEntry* seg_list,
                                                      uint32_t commit) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
+  constexpr uint32_t kRowB = RB, kStB = 32 * RB;
   const uint32_t nwarps = blockDim.x / 32;
   const uint32_t warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   uint8_t* table = smem_raw;
   uint8_t* stages = smem_raw + table_off;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(stages + (size_t)nwarps * S * kStageBytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(stages + (size_t)nwarps * S * kStB);
   uint32_t* prow = reinterpret_cast<uint32_t*>(bars + ((nwarps * S + 1) & ~1u)) + warp * 32;
   stage_table(img, table);
   pdl_wait();
@@ -572,11 +575,11 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncwarp();
   using Sx = Step<MODE>;
-  uint8_t* wst = stages + (size_t)warp * S * kStageBytes;
+  uint8_t* wst = stages + (size_t)warp * S * kStB;
   uint64_t* wbar = bars + warp * S;
   const uint64_t pol = evict_first_policy();
   const uint32_t ckm = (1u << rp.ck_shift) - 1u;
-  const uint32_t segs = (x1 - x0) / kRowBytes;
+  const uint32_t segs = (x1 - x0) / kRowB;
   const uint64_t my_groups = gw < ngroups ? (ngroups - gw + tw - 1) / tw : 0;
   const uint64_t items = my_groups * segs;
   unsigned long long n_mustdo = 0, n_sre = 0, n_hel = 0, walked = 0;
@@ -596,11 +599,11 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
       __syncwarp();
     }
     if (lane == 0) {
-      mbar_expect_tx(wbar + p_s, kStageBytes);
+      mbar_expect_tx(wbar + p_s, kStB);
 #pragma unroll
       for (int g = 0; g < 8; g++)
-        tma_gather4(wst + (size_t)p_s * kStageBytes + g * 4 * kRowBytes, &tmap, wbar + p_s,
-                    (int32_t)(x0 + p_sg * kRowBytes), reinterpret_cast<const uint4*>(prow)[g], pol);
+        tma_gather4(wst + (size_t)p_s * kStB + g * 4 * kRowB, &tmap, wbar + p_s, (int32_t)(x0 + p_sg * kRowB),
+                    reinterpret_cast<const uint4*>(prow)[g], pol);
     }
     if (++p_sg == segs) { p_sg = 0; p_group++; }
     if (++p_s == (uint32_t)S) p_s = 0;
@@ -641,10 +644,11 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
     }
     mbar_wait(wbar + s, phase);
     uint32_t k = code, a = acc;
-    const uint8_t* row = wst + (size_t)s * kStageBytes + lane * kRowBytes;
+    const uint8_t* row = wst + (size_t)s * kStB + lane * kRowB;
 #pragma unroll
-    for (int u = 0; u < (int)(kRowBytes / 16); u++) {
-      const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ ((lane >> 1) & 3)) << 4));  // SWIZZLE_64B
+    for (int u = 0; u < (int)(kRowB / 16); u++) {  // SWIZZLE_64B / SWIZZLE_128B: chunk u ^ (row bits)
+      const uint32_t sw = RB == 64 ? ((lane >> 1) & 3) : (lane & 7);
+      const uint4 q = *reinterpret_cast<const uint4*>(row + ((u ^ sw) << 4));
       walk16<MODE>(img, table, q, k, a);
     }
     __syncwarp();
@@ -652,8 +656,8 @@ __global__ void __launch_bounds__(896, 1) k_task_seg(const __grid_constant__ CUt
     if (live) {
       code = k;
       acc = a;
-      walked += kRowBytes;
-      const uint32_t pe = x0 + (sg + 1) * kRowBytes;
+      walked += kRowB;
+      const uint32_t pe = x0 + (sg + 1) * kRowB;
       bool fin = false;
       uint32_t e = 0, cnt = 0;
       if (pe >= B) {
@@ -833,19 +837,20 @@ cudaError_t launch_tma_m(const CUtensorMap& tm, const DevImage& img, const RunPa
 
 // R30: the segment passes of a checkpointed dense round (one CTA per SM, warps chosen as
 // for the task kernel; each pass reads its list length on the device)
-template <int MODE, int S>
+template <int MODE, int S, int RB>
 cudaError_t launch_seg_t(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
                          uint64_t n_full, int sms, cudaStream_t st, Ctl* ctl, uint32_t seg, void* seg_list,
-                         bool commit_last) {
-  auto kern = k_task_seg<MODE, S>;
+                         bool commit_last, uint32_t pass) {
+  auto kern = k_task_seg<MODE, S, RB>;
+  constexpr uint32_t kStB = 32 * RB;
   const uint32_t tbytes = smem_bytes_for(img);
-  const uint32_t per_warp = S * kStageBytes + S * 8 + 128;
+  const uint32_t per_warp = S * kStB + S * 8 + 128;
   const uint32_t avail = 227 * 1024 - ((tbytes + 1023) & ~1023u) - 64;
   uint32_t w = std::min<uint32_t>(28, avail / per_warp);
   if (const char* ev = getenv("GSPEC_CK_WARPS")) w = std::min<uint32_t>(w, (uint32_t)std::max(4, atoi(ev)));
   if (w < 4) return cudaErrorInvalidConfiguration;
   const uint32_t table_off = (tbytes + 1023) & ~1023u;
-  const uint32_t smem = table_off + w * S * kStageBytes + ((w * S + 1) & ~1u) * 8 + w * 128;
+  const uint32_t smem = table_off + w * S * kStB + ((w * S + 1) & ~1u) * 8 + w * 128;
   cudaError_t e = kernel_setup((const void*)kern, smem, (int)(w * 32), nullptr);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
@@ -859,35 +864,44 @@ cudaError_t launch_seg_t(const CUtensorMap& tm, const DevImage& img, const RunPa
   cfg.attrs = at;
   cfg.numAttrs = pdl_enabled() ? 1 : 0;
   const uint32_t passes = (rp.B + seg - 1) / seg;
+  return cudaLaunchKernelEx(&cfg, kern, tm, img, rp, rs, n_full, table_off, ctl, pass, seg,
+                            reinterpret_cast<SegEntry*>(seg_list), (uint32_t)(commit_last && pass + 1 == passes));
+}
+
+template <int MODE>
+cudaError_t launch_seg_s(const CUtensorMap& tm, const CUtensorMap& tm128, bool r128, const DevImage& img,
+                         const RunParams& rp, const RecStore& rs, uint64_t n_full, int sms, cudaStream_t st, Ctl* ctl,
+                         uint32_t seg, void* seg_list, bool commit_last) {
+  const uint32_t tbytes = smem_bytes_for(img);
+  const bool s3 = tbytes + 24 * (3 * kStageBytes) + 2048 + 24 * 128 <= 227 * 1024;
+  const uint32_t passes = (rp.B + seg - 1) / seg;
   for (uint32_t p = 0; p < passes; p++) {
-    e = cudaLaunchKernelEx(&cfg, kern, tm, img, rp, rs, n_full, table_off, ctl, p, seg,
-                           reinterpret_cast<SegEntry*>(seg_list), (uint32_t)(commit_last && p + 1 == passes));
+    cudaError_t e;
+    // pass 0 (every task: bound by the shared pipe) keeps 64 B rows and the most warps; the later
+    // passes (fewer chains: bound by a warp's issue latency) take 128 B rows, half the TMA issue
+    // work per byte (R30)
+    if (p > 0 && r128)
+      e = launch_seg_t<MODE, 2, 128>(tm128, img, rp, rs, n_full, sms, st, ctl, seg, seg_list, commit_last, p);
+    else if (s3)
+      e = launch_seg_t<MODE, 3, 64>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list, commit_last, p);
+    else
+      e = launch_seg_t<MODE, 2, 64>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list, commit_last, p);
     if (e != cudaSuccess) return e;
   }
   return cudaSuccess;
 }
 
-template <int MODE>
-cudaError_t launch_seg_s(const CUtensorMap& tm, const DevImage& img, const RunParams& rp, const RecStore& rs,
-                         uint64_t n_full, int sms, cudaStream_t st, Ctl* ctl, uint32_t seg, void* seg_list,
-                         bool commit_last) {
-  const uint32_t tbytes = smem_bytes_for(img);
-  if (tbytes + 24 * (3 * kStageBytes) + 2048 + 24 * 128 <= 227 * 1024)
-    return launch_seg_t<MODE, 3>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list, commit_last);
-  return launch_seg_t<MODE, 2>(tm, img, rp, rs, n_full, sms, st, ctl, seg, seg_list, commit_last);
-}
-
 // gather = false: box {64 B, 32 chunks} (tiles of consecutive chunks);
 // gather = true: box {64 B, 1 chunk} for tile::gather4 (4 arbitrary chunks per load)
-bool encode_map(const RunParams& rp, uint64_t n_full, CUtensorMap* tm, bool gather = false) {
+bool encode_map(const RunParams& rp, uint64_t n_full, CUtensorMap* tm, bool gather = false, uint32_t rowb = kRowBytes) {
   EncodeFn enc = get_encode();
   if (!enc) return false;
   cuuint64_t dims[2] = {rp.B, n_full};
   cuuint64_t strides[1] = {rp.B};
-  cuuint32_t box[2] = {kRowBytes, gather ? 1u : 32u};
+  cuuint32_t box[2] = {rowb, gather ? 1u : 32u};
   cuuint32_t es[2] = {1, 1};
   return enc(tm, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t*>(rp.in), dims, strides, box, es,
-             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, rowb == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
              tma_promotion() == 1 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
              : tma_promotion() == 2 ? CU_TENSOR_MAP_L2_PROMOTION_NONE : CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
@@ -936,16 +950,27 @@ cudaError_t launch_task_tma(const DevImage& img, const RunParams& rp, const RecS
     cudaError_t e;
     const uint32_t sg = rp.ck_seg;
     const bool cm = n_full == rp.N;  // no tail chunk: the last pass commits, no finish kernel
+    // 128 B rows when the chunk, the segment and the checkpoint interval are multiples of 128 and
+    // two 4 KiB stages per warp leave room for >= 16 warps beside the table (GSPEC_CK_ROW=64: off)
+    CUtensorMap tm128;
+    static int row_env = -1;
+    if (row_env < 0) {
+      const char* e = getenv("GSPEC_CK_ROW");
+      row_env = e ? atoi(e) : 128;
+    }
+    const bool r128 = row_env == 128 && rp.B % 128 == 0 && sg % 128 == 0 && (1u << rp.ck_shift) % 128 == 0 &&
+                      smem_bytes_for(img) + 16 * (2 * 4096 + 16 + 128) + 2048 <= 227 * 1024 &&
+                      encode_map(rp, n_full, &tm128, true, 128);
     if (committed) *committed = cm;
     switch (img.mode) {
-      case MODE_U8: e = launch_seg_s<MODE_U8>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
-      case MODE_U16: e = launch_seg_s<MODE_U16>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
-      case MODE_U16H: e = launch_seg_s<MODE_U16H>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
+      case MODE_U8: e = launch_seg_s<MODE_U8>(tm, tm128, r128, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
+      case MODE_U16: e = launch_seg_s<MODE_U16>(tm, tm128, r128, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
+      case MODE_U16H: e = launch_seg_s<MODE_U16H>(tm, tm128, r128, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
       case MODE_U16D:
-        e = img.delta_exc == 1 ? launch_seg_s<MODE_U16D1>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm)
-                               : launch_seg_s<MODE_U16D>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm);
+        e = img.delta_exc == 1 ? launch_seg_s<MODE_U16D1>(tm, tm128, r128, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm)
+                               : launch_seg_s<MODE_U16D>(tm, tm128, r128, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm);
         break;
-      default: e = launch_seg_s<MODE_U32>(tm, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
+      default: e = launch_seg_s<MODE_U32>(tm, tm128, r128, img, rp, rs, n_full, sms, st, ctl, sg, rp.ck_list, cm); break;
     }
     if (e == cudaSuccess) *n_done = n_full;
     return e;
