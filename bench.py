@@ -328,7 +328,7 @@ def measure_single(gs, w, x, args, fsm, scheme, B, with_clocks=True):
     ms = ev0.elapsed_time(ev1) / args.steps
     st0 = kr[-1].stats
     diag = {k: st0[k] for k in ("rounds", "tasks_total", "tasks_mustdo", "tasks_sre", "tasks_helper", "reread_bytes",
-                                "verify_checks", "verify_matches")}
+                                "verify_checks", "verify_matches", "task_walked_bytes")}
     diag["runtime_speculation_accuracy"] = round(st0["verify_matches"] / max(1, st0["verify_checks"]), 6)
     diag["avg_active_workers"] = round(float(st0.get("avg_active_workers", 0.0)), 2)
     return {"ms": ms, "value": length / (ms * 1e-3) / 1e9, "spec_ms": _median(spec_ms), "ver_ms": _median(ver_ms),
