@@ -156,8 +156,9 @@ __device__ __forceinline__ uint2 lds_u64(uint32_t saddr) {
 // shared-memory traffic for it), then one row entry is read at (x >> 16) + 2*class
 // and the exceptions override by select — two dependent shared-memory loads, no L2
 // trip, no divergence, and no multiply by C on the path (the class map holds 2*class).
-// The step is ALU-pipe-bound on C4 (math_pipe_throttle): this form needs ~10 ALU-pipe
-// and ~3 FMA-pipe instructions per symbol.
+// With two exceptions this form needs ~10 ALU-pipe and ~3 FMA-pipe instructions per symbol
+// (ALU and shared pipes co-bound on C4); the one-exception step below needs ~8, which leaves
+// the kernel bound by the shared-memory pipe alone.
 // EXC = 1 (img.delta_exc == 1, template mode MODE_U16D1): every delta row has one exception
 // (y = its code), so the step drops the second compare and select: ~8 instead of ~10
 // ALU-pipe instructions per symbol.  The EXC = 2 reader also reads EXC = 1 images (e1 = 0xFF
@@ -168,7 +169,7 @@ struct StepDeltaT {
   static __device__ __forceinline__ uint32_t row(const DevImage& img, uint32_t base, uint32_t code, uint32_t cl2) {
     const uint32_t c = code & 0x7FFFu;
     uint32_t dx = c * 0x20000u + ((base << 16) | 0xFFFFu), dy = 0;
-    uint32_t da;  // c*8 + const on the FMA pipe (the ALU pipe is the bound)
+    uint32_t da;  // c*8 + const on the FMA pipe (keeps the ALU pipe free)
     asm("mad.lo.u32 %0, %1, 8, %2;" : "=r"(da) : "r"(c), "r"(base + img.delta_off - img.HC1 * 8u));
     asm volatile(
         "{\n .reg .pred p;\n setp.ge.u32 p, %2, %3;\n @p ld.shared.v2.u32 {%0, %1}, [%4];\n}\n"
