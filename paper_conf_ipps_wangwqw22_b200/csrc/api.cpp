@@ -909,9 +909,12 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
   img.TK = nullptr;
   img.tk_bytes = 0;
   img.tk_syms = 0;
+  img.pk_off = 0;
   if (mode == MODE_U8 && nsyms <= 4 && nt <= 64) {
     const uint32_t K = nsyms <= 2 ? 8 : 4, bits = 8 / K, row = 257;  // words per row (kTkRow)
-    std::vector<uint32_t> tk(((uint64_t)nt * row + 3) & ~3ull, 0);  // staged in 16-byte pieces
+    const bool pk = K == 8 && nt <= 8 && !tk_pk_disabled();
+    const uint64_t tk_words = ((uint64_t)nt * row + 3) & ~3ull;      // staged in 16-byte pieces
+    std::vector<uint32_t> tk(tk_words + (pk ? 512 : 0), 0);
     for (uint32_t t = 0; t < nt; t++)
       for (uint32_t cb = 0; cb < 256; cb++) {
         uint32_t x = t, k = 0;
@@ -921,7 +924,14 @@ int fsm_load(const uint32_t* table, uint32_t n, uint32_t nsyms, uint32_t start, 
           k += acc_t[x];
         }
         tk[(uint64_t)t * row + cb] = x * row * 4 | k << 24;
+        if (pk)  // packed map: byte t of PK[cb] = next tid | count << 4 (tids and counts < 16)
+          reinterpret_cast<uint8_t*>(tk.data() + tk_words)[cb * 8 + t] = (uint8_t)(x | k << 4);
       }
+    if (pk) {
+      for (uint32_t cb = 0; cb < 256; cb++)  // unused entries t >= nt: identity, no count
+        for (uint32_t t = nt; t < 8; t++) reinterpret_cast<uint8_t*>(tk.data() + tk_words)[cb * 8 + t] = (uint8_t)t;
+      img.pk_off = (uint32_t)(tk_words * 4);
+    }
     if ((rc = upload(f, &img.TK, tk))) return bail(rc);
     img.tk_bytes = (uint32_t)tk.size() * 4;
     img.tk_syms = K;

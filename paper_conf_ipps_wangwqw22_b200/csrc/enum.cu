@@ -27,6 +27,13 @@ __device__ __forceinline__ uint64_t tk_walk(const DevImage& img, const uint8_t* 
                                             const uint8_t* p, uint64_t n, uint32_t (&code)[NE], uint32_t (&acc)[NE]) {
   using S = Step<MODE>;
   uint64_t i = 0;
+  // packed maps (img.pk_off, K = 8, nt <= 8): code[] holds tids inside the vector loop
+  const bool pk = NE == 8 && img.pk_off != 0;
+  const uint32_t pkbase = tkbase + img.pk_off;
+  if (pk) {
+#pragma unroll
+    for (int q = 0; q < NE; q++) code[q] /= kTkRow;
+  }
   if ((reinterpret_cast<uintptr_t>(p) & 15u) == 0) {
     const uint4* v = reinterpret_cast<const uint4*>(p);
     const uint64_t nv = n / 16;
@@ -48,10 +55,13 @@ __device__ __forceinline__ uint64_t tk_walk(const DevImage& img, const uint8_t* 
         if (t16 >= nv) break;
         const uint4 qv = cur[k];
         if (tk_vector_ok(qv, K)) {
-          tk_vector<NE>(tkbase, K, qv, code, acc);
+          if (pk)
+            pk_vector<NE>(pkbase, qv, code, acc);
+          else
+            tk_vector<NE>(tkbase, K, qv, code, acc);
         } else {  // a byte TK does not cover (an invalid symbol): these 16 bytes one by one
 #pragma unroll
-          for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + code[q] / kTkRow);
+          for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + (pk ? code[q] : code[q] / kTkRow));
           const uint8_t* b16 = reinterpret_cast<const uint8_t*>(v + t16);
           for (int b = 0; b < 16; b++) {
             const uint32_t bb = __ldg(b16 + b);
@@ -59,14 +69,14 @@ __device__ __forceinline__ uint64_t tk_walk(const DevImage& img, const uint8_t* 
             for (int q = 0; q < NE; q++) { code[q] = S::byte(img, smem, code[q], bb); acc[q] += S::acc(code[q]); }
           }
 #pragma unroll
-          for (int q = 0; q < NE; q++) code[q] = S::tid(img, code[q]) * kTkRow;
+          for (int q = 0; q < NE; q++) code[q] = S::tid(img, code[q]) * (pk ? 1u : kTkRow);
         }
       }
     }
     i = nv * 16;
   }
 #pragma unroll
-  for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + code[q] / kTkRow);
+  for (int q = 0; q < NE; q++) code[q] = __ldg(img.tid2code + (pk ? code[q] : code[q] / kTkRow));
   return i;
 }
 

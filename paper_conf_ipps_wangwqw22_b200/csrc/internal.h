@@ -54,6 +54,10 @@ struct DevImage {
   const uint32_t* TK;
   uint32_t tk_bytes;
   uint32_t tk_syms;  // K
+  // K = 8 and nt <= 8: byte offset in the staged TK image of the packed-map
+  // table PK[combo] (8 bytes: byte t = the tid after the 8 symbols from tid t | accepting states
+  // among them << 4), so ONE lookup advances all 8 enumeration chains by 8 symbols; 0 = none
+  uint32_t pk_off;
   const uint8_t* T8;          // MODE_U8: [256 codes][256 bytes] next code
   const uint16_t* T16;        // MODE_U16: [nt][C]
   const uint32_t* T32;        // MODE_U32: [nt][C]
@@ -260,6 +264,16 @@ inline uint32_t ck_seg_for(uint32_t B, uint32_t ck_shift) {
   uint32_t seg = v > 0 ? (uint32_t)v : (B / 4 + cp - 1) / cp * cp;
   seg = (seg + cp - 1) / cp * cp;
   return seg < cp ? cp : seg;
+}
+
+// GSPEC_TK_PK=0: enumeration on small alphabets without the packed-map table (A/B)
+inline bool tk_pk_disabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("GSPEC_TK_PK");
+    v = (e && atoi(e) == 0) ? 1 : 0;
+  }
+  return v != 0;
 }
 
 inline int tma_evict_mode() {

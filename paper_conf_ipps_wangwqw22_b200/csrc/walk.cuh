@@ -320,6 +320,24 @@ __device__ __forceinline__ void tk_lookup(uint32_t tkbase, uint32_t combo, uint3
   }
 }
 
+// all (<= 8) chains over one 16-byte vector of one-bit symbols through the packed maps PK
+// (DevImage::pk_off): per 8 symbols ONE 8-byte lookup, then each chain takes byte t of it
+// with a PRMT (selector = its tid) — next tid in the low nibble, accepting states above
+template <int NE>
+__device__ __forceinline__ void pk_vector(uint32_t pkbase, const uint4& q, uint32_t (&t)[NE], uint32_t (&acc)[NE]) {
+  const uint2 e0 = lds_u64(pkbase + tk_pack8(q.x, q.y) * 8u);
+  const uint2 e1 = lds_u64(pkbase + tk_pack8(q.z, q.w) * 8u);
+#pragma unroll
+  for (int j = 0; j < NE; j++) {
+    uint32_t x;
+    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(x) : "r"(e0.x), "r"(e0.y), "r"(t[j]));
+    acc[j] += (x >> 4) & 0xFu;
+    asm("prmt.b32 %0, %1, %2, %3;" : "=r"(x) : "r"(e1.x), "r"(e1.y), "r"(x & 0xFu));
+    t[j] = x & 0xFu;
+    acc[j] += (x >> 4) & 0xFu;
+  }
+}
+
 // the first np chains over one 16-byte vector (tk_vector_ok) through TK
 template <int NE>
 __device__ __forceinline__ void tk_vector(uint32_t tkbase, uint32_t K, const uint4& q, uint32_t (&sc)[NE],
