@@ -266,14 +266,11 @@ inline uint32_t ck_seg_for(uint32_t B, uint32_t ck_shift) {
   return seg < cp ? cp : seg;
 }
 
-// GSPEC_TK_PK=0: enumeration on small alphabets without the packed-map table (A/B)
+// GSPEC_TK_PK=0: enumeration on small alphabets without the packed-map table (A/B; read at
+// every fsm_load)
 inline bool tk_pk_disabled() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("GSPEC_TK_PK");
-    v = (e && atoi(e) == 0) ? 1 : 0;
-  }
-  return v != 0;
+  const char* e = getenv("GSPEC_TK_PK");
+  return e && atoi(e) == 0;
 }
 
 inline int tma_evict_mode() {

@@ -839,3 +839,54 @@ def test_checkpointed_dense_rounds(gs, name, length, B, scheme, ck):
         assert stats["task_walked_bytes"] % B == 0
     else:
         assert 0 < stats["task_walked_bytes"] < stats["reread_bytes"]
+
+
+@pytest.mark.parametrize("name,length,B", [("c1", (16 << 20) + 5, 4096), ("rand:7:2:3", (6 << 20) + 17, 1024),
+                                           ("rand:5:2:9", 3 << 20, 4096), ("c1", 1 << 20, 4096)])
+def test_enum_packed_maps_on_off(gs, name, length, B):
+    """DESIGN.md §5.3 packed maps (K = 8, nt <= 8: one 8-byte lookup per 8 symbols for all
+    chains): bit-exact against the oracle with the packed maps (default) and without them
+    (GSPEC_TK_PK=0 at load: per-chain TK lookups), in the multi-launch walk and the
+    single-launch kernel (<= 2 MiB), with unaligned tails."""
+    import os
+    w, data = _wl(name, length)
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    x = torch.from_numpy(data).cuda()
+    for flag in ("1", "0"):
+        os.environ["GSPEC_TK_PK"] = flag
+        try:
+            fsm = gs.FSM.load(w.table, w.start, w.accept)
+        finally:
+            os.environ.pop("GSPEC_TK_PK", None)
+        res = fsm.run(x, scheme="enum", chunk_bytes=B)
+        check_equal(res, ref, B, w.nstates)
+        fsm.close()
+
+
+@pytest.mark.parametrize("exc", ["1", "2"])
+@pytest.mark.parametrize("scheme", ["sre", "rr", "cse"])
+def test_delta_rows_exception_plans(gs, exc, scheme):
+    """C4's delta rows with the one-exception plan (default: the rows needing
+    two exceptions are hot, the walk kernels use the one-exception step) and with the
+    two-exception plan (GSPEC_DELTA_EXC=2 at load) — both bit-exact against the oracle, round
+    counters equal to the oracle's simulation; every other kernel reads either image with the
+    two-exception step."""
+    import os
+    w, data = _wl("c4", 4 << 20)
+    B = 4096
+    ref = oracle.run(w.table, w.start, w.accept, data, B)
+    sim = oracle.simulate(w.table, w.start, w.accept, data, B, scheme=scheme)
+    os.environ["GSPEC_DELTA_EXC"] = exc
+    try:
+        fsm = gs.FSM.load(w.table, w.start, w.accept)
+    finally:
+        os.environ.pop("GSPEC_DELTA_EXC", None)
+    assert fsm.transform()["mode"] == "u16d"
+    res = fsm.run(torch.from_numpy(data).cuda(), scheme=scheme, chunk_bytes=B)
+    check_equal(res, ref, B, w.nstates)
+    for k in ("rounds", "tasks_mustdo", "tasks_sre", "tasks_helper", "verify_checks", "verify_matches"):
+        assert res.stats[k] == sim[k], (k, res.stats[k], sim[k])
+    lit = fsm.run_literal(torch.from_numpy(data[: 1 << 20]).cuda(), scheme="sre", chunk_bytes=B)
+    ref1 = oracle.run(w.table, w.start, w.accept, data[: 1 << 20], B)
+    assert lit.final_state == ref1["final"] and lit.accept_count == ref1["count"]
+    fsm.close()
